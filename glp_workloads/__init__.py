@@ -1,0 +1,163 @@
+"""Seeded synthetic workloads shared by the CUDA path's tests/bench and the oracle.
+
+Holds ONLY shapes (Table 5, P334-355, at the BASELINE.json batch sizes) and the
+random-number recipe of DESIGN.md §Inputs; none of the method's arithmetic.
+Both sides receive the same bytes from these generators.
+
+Recipe (numpy ``Generator(PCG64(seed))``, seed = 0x474C5034 + 1000*cfg + 10*layer + tensor,
+tensor: x=0, W=1, b=2, dy=3):
+  data-fed x ~ U[0,1)            (pixel intensities)
+  inner x    ~ max(0, N(0,1))    (post-ReLU activations, ~50% zeros)
+  W          ~ U[-a, a], a = sqrt(3 / (C_i*K_h*K_w))   (Caffe "xavier", fan-in)
+  b          ~ U[-0.1, 0.1]
+  dy         ~ N(0,1) / N_global (batch-averaged loss)
+  exact-arithmetic variant: integers, x/W/dy in [-2,2] (data layer x in [0,2]), b in [-4,4].
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, replace
+from typing import Dict, List
+
+import numpy as np
+
+SEED_BASE = 0x474C5034
+
+
+@dataclass(frozen=True)
+class Layer:
+    name: str
+    N: int
+    C: int
+    H: int
+    W: int
+    Co: int
+    K: int
+    S: int
+    P: int
+    Ho: int            # literal from Table 5 geometry (checked against oracle.out_dim in tests)
+    data_fed: bool     # bottom is the data layer -> benchmark skips dgrad (R9)
+    cfg: int = 0
+    index: int = 0
+
+    @property
+    def x_shape(self):
+        return (self.N, self.C, self.H, self.W)
+
+    @property
+    def w_shape(self):
+        return (self.Co, self.C, self.K, self.K)
+
+    @property
+    def y_shape(self):
+        return (self.N, self.Co, self.Ho, self.Ho)
+
+    def with_batch(self, n: int) -> "Layer":
+        return replace(self, N=int(n))
+
+    def flops_per_pass(self) -> float:
+        """2*C_o*C_i*K_h*K_w*H_o*W_o per image, times N."""
+        return 2.0 * self.Co * self.C * self.K * self.K * self.Ho * self.Ho * self.N
+
+
+def _L(name, N, C, HW, Co, K, S, P, Ho, data_fed):
+    return Layer(name, N, C, HW, HW, Co, K, S, P, Ho, data_fed)
+
+
+# Table 5 (P334-355).  LeNet = the Siamese conv1/conv2 shapes (R20).
+_TABLE: Dict[int, List[Layer]] = {
+    1: [_L("lenet_conv1", 64, 1, 28, 20, 5, 1, 0, 24, True)],
+    2: [_L("lenet_conv1", 64, 1, 28, 20, 5, 1, 0, 24, True),
+        _L("lenet_conv2", 64, 20, 12, 50, 5, 1, 0, 8, False)],
+    3: [_L("cifar10_conv1", 100, 3, 32, 32, 5, 1, 2, 32, True),
+        _L("cifar10_conv2", 100, 32, 16, 32, 5, 1, 2, 16, False),
+        _L("cifar10_conv3", 100, 32, 8, 64, 5, 1, 2, 8, False)],
+    4: [_L("caffenet_conv1", 256, 3, 227, 96, 11, 4, 0, 55, True),
+        _L("caffenet_conv2", 256, 96, 27, 256, 5, 1, 2, 27, False),
+        _L("caffenet_conv3", 256, 256, 13, 384, 3, 1, 1, 13, False),
+        _L("caffenet_conv4", 256, 384, 13, 384, 3, 1, 1, 13, False),
+        _L("caffenet_conv5", 256, 384, 13, 256, 3, 1, 1, 13, False)],
+    # GoogLeNet Table 5 units at the BASELINE batch 128 (R19); inputs synthesised
+    # at the units' own 7x7 shapes.  None is fed by the data layer.
+    5: [_L("googlenet_conv_1", 128, 160, 7, 320, 3, 1, 1, 7, False),
+        _L("googlenet_conv_2", 128, 832, 7, 32, 1, 1, 0, 7, False),
+        _L("googlenet_conv_3", 128, 832, 7, 384, 1, 1, 0, 7, False),
+        _L("googlenet_conv_4", 128, 192, 7, 384, 3, 1, 1, 7, False),
+        _L("googlenet_conv_5", 128, 832, 7, 192, 1, 1, 0, 7, False),
+        _L("googlenet_conv_6", 128, 832, 7, 48, 1, 1, 0, 7, False)],
+}
+
+CONFIG_NAMES = {
+    1: "lenet_conv1_b64",
+    2: "lenet5_conv_stack_b64",
+    3: "cifar10_quick_conv_b100",
+    4: "caffenet_conv1-5_b256",
+    5: "googlenet_table5_units_b128",
+}
+
+
+def config(cfg: int) -> List[Layer]:
+    return [replace(l, cfg=cfg, index=i) for i, l in enumerate(_TABLE[cfg])]
+
+
+def all_layers() -> List[Layer]:
+    out = []
+    for c in sorted(_TABLE):
+        out.extend(config(c))
+    return out
+
+
+def seed(cfg: int, layer: int, tensor: int) -> int:
+    return SEED_BASE + 1000 * cfg + 10 * layer + tensor
+
+
+def _rng(cfg, layer, tensor):
+    return np.random.Generator(np.random.PCG64(seed(cfg, layer, tensor)))
+
+
+def gen_layer(layer: Layer, n_global: int = None, exact: bool = False, batch: int = None):
+    """Return dict(x, w, b, dy) of float32 numpy arrays for one layer (same bytes for both sides).
+
+    ``batch`` overrides N (samples are the first ``batch`` of the stream's draws order)."""
+    N = layer.N if batch is None else int(batch)
+    n_global = N if n_global is None else n_global
+    c, i = layer.cfg, layer.index
+    xs = (N, layer.C, layer.H, layer.W)
+    ws = layer.w_shape
+    ys = (N, layer.Co, layer.Ho, layer.Ho)
+    if exact:
+        lo = 0 if layer.data_fed else -2
+        x = _rng(c, i, 0).integers(lo, 3, size=xs).astype(np.float32)
+        w = _rng(c, i, 1).integers(-2, 3, size=ws).astype(np.float32)
+        b = _rng(c, i, 2).integers(-4, 5, size=(layer.Co,)).astype(np.float32)
+        dy = _rng(c, i, 3).integers(-2, 3, size=ys).astype(np.float32)
+    else:
+        if layer.data_fed:
+            x = _rng(c, i, 0).random(xs, dtype=np.float32)
+        else:
+            x = np.maximum(_rng(c, i, 0).standard_normal(xs, dtype=np.float32), 0.0)
+        a = np.float32(np.sqrt(3.0 / (layer.C * layer.K * layer.K)))
+        w = _rng(c, i, 1).uniform(-a, a, size=ws).astype(np.float32)
+        b = _rng(c, i, 2).uniform(-0.1, 0.1, size=(layer.Co,)).astype(np.float32)
+        dy = (_rng(c, i, 3).standard_normal(ys, dtype=np.float32) / np.float32(n_global)).astype(np.float32)
+    return {"x": np.ascontiguousarray(x), "w": np.ascontiguousarray(w),
+            "b": np.ascontiguousarray(b), "dy": np.ascontiguousarray(dy)}
+
+
+def gen_custom(N, C, H, W, Co, Kh, Kw, seed_: int, exact: bool = False, Ho=None, Wo=None,
+               data_fed: bool = False):
+    """Generator for ad-hoc shapes (odd strides/pads, ragged tails).  Ho/Wo are supplied by
+    the caller (the generator holds no conv arithmetic)."""
+    r = np.random.Generator(np.random.PCG64(int(seed_)))
+    xs, ws, ys = (N, C, H, W), (Co, C, Kh, Kw), (N, Co, Ho, Wo)
+    if exact:
+        x = r.integers(0 if data_fed else -2, 3, size=xs).astype(np.float32)
+        w = r.integers(-2, 3, size=ws).astype(np.float32)
+        b = r.integers(-4, 5, size=(Co,)).astype(np.float32)
+        dy = r.integers(-2, 3, size=ys).astype(np.float32)
+    else:
+        x = r.standard_normal(xs, dtype=np.float32)
+        a = np.float32(np.sqrt(3.0 / max(1, C * Kh * Kw)))
+        w = r.uniform(-a, a, size=ws).astype(np.float32)
+        b = r.uniform(-0.1, 0.1, size=(Co,)).astype(np.float32)
+        dy = (r.standard_normal(ys, dtype=np.float32) / np.float32(max(N, 1))).astype(np.float32)
+    return {"x": x, "w": w, "b": b, "dy": dy}

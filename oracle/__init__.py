@@ -1,0 +1,174 @@
+"""ORACLE — TEST INFRASTRUCTURE ONLY (parity checker, never the product path).
+
+Plain CPU definition of the GLP4NN hot path (Alg. 1 P82-99, Alg. 2 P101-121,
+parameter gradients P129; conv kernels im2col/sgemm/gemmk P173) with fp64 accumulation,
+in ``oracle/oracle.c``, plus the rounding-step definitions (R12) and the
+paper's analytical model (``oracle/analyzer.py``, §3.2 Eqs 1-9).
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  It shares no code with
+``paper_conf_icpp_futhys18_b200`` and does not import it.
+
+Parity status per function (see DESIGN.md §Oracle pins):
+  conv_fwd / conv_bwd_data / conv_bwd_filter / im2col  -- pinned (hand cases, torch fp64,
+      adjoint identity, finite differences, 1x1 = matmul, batch-sum, floor truncation,
+      im2col+GEMM == direct conv, thread-count invariance)
+  round_tf32_rna / round_bf16_rne / split_3xtf32          -- pinned (bit patterns, error bound)
+  analyzer.*                                              -- pinned (paper worked example P173,
+      brute-force MILP enumeration vs closed form)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c with gcc -O2 -fopenmp (no CUDA, no shared headers)."""
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(_SRC):
+        tmp = _LIB_PATH + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB_PATH)
+    return _LIB_PATH
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB_PATH)
+        i, p = ctypes.c_int, ctypes.c_void_p
+        L.oracle_conv_fwd.argtypes = [i] * 11 + [p, p, p, p, i]
+        L.oracle_conv_bwd_data.argtypes = [i] * 11 + [p, p, p, i]
+        L.oracle_conv_bwd_filter.argtypes = [i] * 11 + [p, p, p, p, i]
+        L.oracle_im2col.argtypes = [i] * 9 + [p, p]
+        L.oracle_set_threads.argtypes = [i]
+        L.oracle_max_threads.restype = i
+        _lib = L
+    return _lib
+
+
+def set_threads(n: int) -> None:
+    lib().oracle_set_threads(int(n))
+
+
+def max_threads() -> int:
+    return int(lib().oracle_max_threads())
+
+
+def out_dim(n: int, k: int, s: int, p: int) -> int:
+    """Table 5 (P316) output size, floor reading (R2)."""
+    return (n + 2 * p - k) // s + 1
+
+
+def _f32(a):
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+def _ptr(a):
+    return a.ctypes.data_as(ctypes.c_void_p) if a is not None else None
+
+
+def _geom(x_shape, w_shape, stride, pad):
+    N, C, H, W = x_shape
+    Co, Ci, Kh, Kw = w_shape
+    assert Ci == C, "group = 1 (DESIGN.md R4)"
+    sh, sw = (stride, stride) if np.isscalar(stride) else stride
+    ph, pw = (pad, pad) if np.isscalar(pad) else pad
+    return N, C, H, W, Co, Kh, Kw, int(sh), int(sw), int(ph), int(pw)
+
+
+def conv_fwd(x, w, b=None, stride=1, pad=0, absmode=False):
+    """Alg. 1 (P82-99): y = b + W (*) x, fp64 result."""
+    x, w = _f32(x), _f32(w)
+    b = _f32(b) if b is not None else None
+    g = _geom(x.shape, w.shape, stride, pad)
+    N, C, H, W, Co, Kh, Kw, sh, sw, ph, pw = g
+    y = np.empty((N, Co, out_dim(H, Kh, sh, ph), out_dim(W, Kw, sw, pw)), np.float64)
+    lib().oracle_conv_fwd(*g, _ptr(x), _ptr(w), _ptr(b), _ptr(y), int(absmode))
+    return y
+
+
+def conv_bwd_data(dy, w, x_shape, stride=1, pad=0, absmode=False):
+    """Alg. 2 (P101-121): dx = col2im(W^T dy), fp64 result (scatter-add formulation)."""
+    dy, w = _f32(dy), _f32(w)
+    g = _geom(x_shape, w.shape, stride, pad)
+    dx = np.empty(tuple(x_shape), np.float64)
+    lib().oracle_conv_bwd_data(*g, _ptr(dy), _ptr(w), _ptr(dx), int(absmode))
+    return dx
+
+
+def conv_bwd_filter(x, dy, w_shape, stride=1, pad=0, with_bias=True, absmode=False):
+    """P129 parameter gradients summed over the batch: (dW, db) in fp64."""
+    x, dy = _f32(x), _f32(dy)
+    g = _geom(x.shape, w_shape, stride, pad)
+    dw = np.empty(tuple(w_shape), np.float64)
+    db = np.empty((w_shape[0],), np.float64) if with_bias else None
+    lib().oracle_conv_bwd_filter(*g, _ptr(x), _ptr(dy), _ptr(dw), _ptr(db), int(absmode))
+    return dw, db
+
+
+def im2col(x_n, kh, kw, stride=1, pad=0):
+    """Caffe im2col of one sample (C,H,W) -> col[(ci*Kh+kh)*Kw+kw, ho*Wo+wo] (fp32)."""
+    x_n = _f32(x_n)
+    C, H, W = x_n.shape
+    sh, sw = (stride, stride) if np.isscalar(stride) else stride
+    ph, pw = (pad, pad) if np.isscalar(pad) else pad
+    Ho, Wo = out_dim(H, kh, sh, ph), out_dim(W, kw, sw, pw)
+    col = np.empty((C * kh * kw, Ho * Wo), np.float32)
+    lib().oracle_im2col(C, H, W, kh, kw, sh, sw, ph, pw, _ptr(x_n), _ptr(col))
+    return col
+
+
+# ----------------------------------------------------------------------------------------
+# Rounding-step definitions (R12: the paper is FP32 SIMT; the tensor-core math
+# modes round operands once).  Bit-level definitions, pinned by tests/golden/rounding.json.
+# ----------------------------------------------------------------------------------------
+
+def round_tf32_rna(a):
+    """Round fp32 to TF32 (10 explicit mantissa bits), nearest, ties AWAY from zero.
+
+    Definition: add half an ulp (0x1000) to the magnitude bits, clear the 13 low bits.
+    Inf/NaN pass through unchanged."""
+    a = _f32(a)
+    u = a.view(np.uint32).copy()
+    finite = (u & 0x7F800000) != 0x7F800000
+    r = ((u.astype(np.uint64) + 0x1000) & 0xFFFFE000).astype(np.uint32)
+    u = np.where(finite, r, u)
+    return u.view(np.float32)
+
+
+def round_bf16_rne(a):
+    """Round fp32 to bf16 (7 explicit mantissa bits), nearest, ties to EVEN; returned as fp32."""
+    a = _f32(a)
+    u = a.view(np.uint32).copy()
+    finite = (u & 0x7F800000) != 0x7F800000
+    lsb = (u >> 16) & 1
+    r = ((u.astype(np.uint64) + 0x7FFF + lsb) & 0xFFFF0000).astype(np.uint32)
+    u = np.where(finite, r, u)
+    return u.view(np.float32)
+
+
+def split_3xtf32(a):
+    """3xTF32 operand split: hi = rna(a), lo = rna(a - hi) (fp32 subtraction)."""
+    a = _f32(a)
+    hi = round_tf32_rna(a)
+    lo = round_tf32_rna((a - hi).astype(np.float32))
+    return hi, lo
+
+
+def normwise_err(got, ref):
+    """DESIGN.md R11: max_i |g_i - r_i| / max_i |r_i| (per tensor)."""
+    ref = np.asarray(ref, np.float64)
+    got = np.asarray(got, np.float64)
+    den = float(np.max(np.abs(ref))) if ref.size else 0.0
+    num = float(np.max(np.abs(got - ref))) if ref.size else 0.0
+    return num / den if den > 0 else num

@@ -1,0 +1,166 @@
+/*
+ * glp.h — C ABI of the B200-native GLP4NN conv-layer training hot path (libglp.so).
+ *
+ * The calls follow the paper's problem statement (PAPER.md, "P<n>" = line n):
+ *   - Alg. 1 forward propagation (P82-99): top = BLAS(weight, bias, bottom), for a conv layer
+ *     im2col -> sgemm -> bias gemm (P173)                          -> glp_conv_fwd
+ *   - Alg. 2 backward propagation (P101-121): bottom_gradient = BLAS(top_gradient, weight),
+ *     i.e. GEMM W^T dy -> col2im                                  -> glp_conv_bwd_data
+ *   - parameter gradients "for parameter update" (P129), summed over the samples of the batch
+ *     (BASELINE.json north_star)                                   -> glp_conv_bwd_filter
+ *   - layer parameters N, C_i, H, W, C_o, F_h, F_w, S, P (Table 5 definitions, P316)
+ *                                                                  -> glp_conv_desc_create
+ *   - the kernel analyzer (§3.1 P167, §3.2 Eqs 1-9 P214-254) re-derived for sm_100a; its output
+ *     (the paper's C_out, P254) is the number of samples in flight S that sizes the persistent
+ *     tile scheduler replacing the stream pool (P169-173)          -> glp_plan, glp_analyze_*
+ *
+ * Conventions (readings R1-R13):
+ *   - x, y, dx, dy: NCHW fp32; W: [C_o][C_i][K_h][K_w] fp32; b, db: [C_o] fp32 (Caffe blobs, P87).
+ *   - cross-correlation (no flip), zero padding, H_o = floor((H + 2P - K_h)/S) + 1, group = 1,
+ *     dilation = 1.
+ *   - N in the descriptor is the per-rank batch (multi-GPU sharding is the caller's, BJ.ns (4)).
+ *
+ * Ownership: the caller owns every tensor and the workspace (device pointers, e.g. from the
+ * PyTorch caching allocator; 16-byte aligned).  The library owns only the opaque desc/plan
+ * objects (create/destroy pairs).  A plan is bound to one device (P159: a private analyzer and
+ * scheduler per GPU) and immutable after glp_plan; it may be used concurrently on different
+ * streams with distinct workspaces.
+ *
+ * Errors: every call returns a status code; no exception or abort crosses the ABI.  Arguments
+ * are validated before any launch (NULL, misalignment, non-positive dims, H_o < 1, workspace too
+ * small).  GLP_ERR_CUDA reports a launch error; glp_last_error_string() gives its text.
+ * Execution: all compute calls are asynchronous on the given stream; no host synchronisation
+ * and no hidden device allocation.  There is no CPU fallback: without a usable sm_100 device
+ * glp_plan fails with GLP_ERR_NOT_SUPPORTED.
+ */
+#ifndef GLP_H_
+#define GLP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  GLP_OK = 0,
+  GLP_ERR_INVALID_VALUE = 1,
+  GLP_ERR_NOT_SUPPORTED = 2,
+  GLP_ERR_CUDA = 3,
+  GLP_ERR_WORKSPACE_TOO_SMALL = 4,
+  GLP_ERR_INTERNAL = 5
+} glp_status_t;
+
+typedef enum {
+  GLP_MATH_FP32 = 0, /* fp32 CUDA-core direct convolution; normwise error <= 1e-5           */
+  GLP_MATH_TF32 = 1, /* tcgen05 kind::tf32 (operands RNA-rounded in the pack), fp32 accumulate */
+  GLP_MATH_BF16 = 2  /* tcgen05 kind::f16 with bf16 operands (RNE), fp32 accumulate           */
+} glp_math_t;
+
+typedef struct glp_conv_desc_s *glp_conv_desc_t;
+typedef struct glp_plan_s *glp_plan_t;
+typedef void *glp_stream_t; /* a cudaStream_t (e.g. torch.cuda.Stream.cuda_stream); NULL = legacy */
+
+/* Plan summary = the analyzer's inputs and outputs (Fig. 8 analog: S per layer). */
+typedef struct {
+  int samples_in_flight; /* S: the paper's C_out re-derived (P254) for the forward kernel      */
+  int ctas_per_sm;       /* beta per SM of the forward kernel (Eq. 8 re-derived)                */
+  int grid_fwd, grid_bwd_data, grid_bwd_filter; /* persistent grid sizes                        */
+  int tile_m, tile_n_fwd, tile_n_bwd_data, tile_n_bwd_filter;
+  int stages_fwd, stages_bwd_data, stages_bwd_filter;
+  int splits_wgrad;      /* shape-only split count of the N*H_o*W_o reduction                   */
+  int tiles_fwd, tiles_bwd_data, tiles_bwd_filter;
+  size_t ws_fwd, ws_bwd_data, ws_bwd_filter, ws_bwd; /* workspace bytes per call               */
+  double plan_us;        /* host time spent in glp_plan (Table 6 T_a analog)                   */
+  int math;
+} glp_plan_info_t;
+
+/* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */
+typedef struct {
+  int sm_count;            /* #SM                                   */
+  int max_threads_per_sm;  /* tau_max                               */
+  int max_blocks_per_sm;   /* rho_max                               */
+  int regs_per_sm;         /* hard limit on sm_100a (R16)           */
+  int smem_per_sm;         /* sm_max (bytes)                        */
+  int smem_reserved_per_cta;
+  int tmem_cols_per_sm;    /* 512 on sm_100a                        */
+  int max_concurrent_kernels; /* C (Eq. 6)                          */
+} glp_device_limits_t;
+
+/* Per-kernel record (Table 2 "profiling input", P194-200; D5). */
+typedef struct {
+  int threads;    /* tau_Ki              */
+  int regs;       /* registers / thread  */
+  int smem_bytes; /* sm_Ki (static + dynamic) */
+  int tmem_cols;  /* TMEM columns / CTA  */
+} glp_kernel_attr_t;
+
+/* ---- descriptors (Table 5 parameters, P316) ------------------------------------------------ */
+glp_status_t glp_conv_desc_create(glp_conv_desc_t *out, int N, int C_in, int H, int W, int C_out,
+                                  int K_h, int K_w, int stride_h, int stride_w, int pad_h,
+                                  int pad_w);
+glp_status_t glp_conv_desc_get_output(glp_conv_desc_t desc, int *H_out, int *W_out);
+glp_status_t glp_conv_desc_destroy(glp_conv_desc_t desc);
+
+/* ---- plan: analyzer + scheduler setup, once per (shape, device, math) ("profile once", P173) -
+ * samples_in_flight: 0 = analyzer's choice; > 0 = override (tests of convergence invariance,
+ * P264: outputs must be bitwise identical for every S). */
+glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t desc, int device, glp_math_t math,
+                      int samples_in_flight);
+glp_status_t glp_plan_get_info(glp_plan_t plan, glp_plan_info_t *info);
+glp_status_t glp_plan_destroy(glp_plan_t plan);
+
+/* ---- compute (asynchronous on `stream`) --------------------------------------------------- */
+/* y = b + W (*) x.  b may be NULL (no bias).  ws >= info.ws_fwd bytes. */
+glp_status_t glp_conv_fwd(glp_plan_t plan, const float *x, const float *w, const float *b,
+                          float *y, void *ws, size_t ws_bytes, glp_stream_t stream);
+/* dx = col2im(W^T dy) (overwrite).  ws >= info.ws_bwd_data bytes. */
+glp_status_t glp_conv_bwd_data(glp_plan_t plan, const float *dy, const float *w, float *dx,
+                               void *ws, size_t ws_bytes, glp_stream_t stream);
+/* dW = sum_n dy_n col_n^T, db = sum dy (db may be NULL).  accumulate = 0: overwrite;
+ * 1: dW += .., db += .. (Caffe beta = 1 diff accumulation).  The reduction over N*H_o*W_o uses
+ * a split count fixed by the shape and a fixed summation order: bitwise independent of S, the
+ * grid and the run (convergence-invariant, P264).  ws >= info.ws_bwd_filter bytes. */
+glp_status_t glp_conv_bwd_filter(glp_plan_t plan, const float *x, const float *dy, float *dw,
+                                 float *db, int accumulate, void *ws, size_t ws_bytes,
+                                 glp_stream_t stream);
+/* Both backward passes of one layer with dy packed once: dx may be NULL (data-fed layer,
+ * DESIGN.md R9).  Results are bitwise identical to the two separate calls.
+ * ws >= info.ws_bwd bytes. */
+glp_status_t glp_conv_bwd(glp_plan_t plan, const float *x, const float *dy, const float *w,
+                          float *dx, float *dw, float *db, int accumulate, void *ws,
+                          size_t ws_bytes, glp_stream_t stream);
+
+/* ---- analyzer (host only, no device needed) ----------------------------------------------- */
+/* The north_star's sm_100a limits: 148 SMs, 64K regs, 228 KB smem, 2048 threads, 32 blocks,
+ * + 512 TMEM columns, 1 KB smem reserved per CTA, C = 128. */
+glp_status_t glp_device_limits_b200(glp_device_limits_t *lim);
+/* CTAs per SM (beta) from every per-SM limit (Eqs 4-5 + registers/blocks/TMEM, R16). */
+glp_status_t glp_analyze_ctas_per_sm(const glp_device_limits_t *lim, const glp_kernel_attr_t *k,
+                                     int *ctas_per_sm);
+/* S = clamp(floor(slots / tiles_per_sample), 1, n_local)  (Eq. 9 re-derived, R18). */
+glp_status_t glp_analyze_samples_in_flight(int slots, int tiles_per_sample, int n_local, int *S);
+/* Paper Eq. 7 bound (P245) for a kernel with #beta blocks; t_kernel/t_launch <= 0 = no launch
+ * term (R17).  Output floor(min(...)). */
+glp_status_t glp_analyze_eq7(const glp_device_limits_t *lim, const glp_kernel_attr_t *k,
+                             int blocks, double t_kernel, double t_launch, int *bound);
+/* Attributes of the shipped kernels for a plan (for the occupancy-API cross-check). which:
+ * 0 = forward, 1 = backward-data, 2 = backward-filter. */
+glp_status_t glp_plan_kernel_attr(glp_plan_t plan, int which, glp_kernel_attr_t *attr,
+                                  int *ctas_per_sm_model, int *ctas_per_sm_runtime);
+
+/* ---- diagnostics ---------------------------------------------------------------------------- */
+const char *glp_status_string(glp_status_t s);
+const char *glp_last_error_string(void);
+int glp_version(void);
+/* Test-only, off the hot path: materialise the im2col matrix of sample n,
+ * col[(ci*K_h+kh)*K_w+kw][ho*W_o+wo], using the tensor-core producer's own index math
+ * (the packed NHWC operand and its gather).  Values are the packed (rounded) operands. */
+glp_status_t glp_debug_im2col(glp_plan_t plan, const float *x, int n, float *col, void *ws,
+                              size_t ws_bytes, glp_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GLP_H_ */

@@ -50,6 +50,8 @@ def lib():
         L.oracle_conv_bwd_data.argtypes = [i] * 11 + [p, p, p, i]
         L.oracle_conv_bwd_filter.argtypes = [i] * 11 + [p, p, p, p, i]
         L.oracle_im2col.argtypes = [i] * 9 + [p, p]
+        L.oracle_conv_bwd_filter_at.argtypes = [i] * 11 + [p, p, i, i, i, i]
+        L.oracle_conv_bwd_filter_at.restype = ctypes.c_double
         L.oracle_set_threads.argtypes = [i]
         L.oracle_max_threads.restype = i
         _lib = L
@@ -114,6 +116,14 @@ def conv_bwd_filter(x, dy, w_shape, stride=1, pad=0, with_bias=True, absmode=Fal
     db = np.empty((w_shape[0],), np.float64) if with_bias else None
     lib().oracle_conv_bwd_filter(*g, _ptr(x), _ptr(dy), _ptr(dw), _ptr(db), int(absmode))
     return dw, db
+
+
+def conv_bwd_filter_at(x, dy, w_shape, stride, pad, idx):
+    """One dW[co,ci,kh,kw] element (fp64), same definition as conv_bwd_filter."""
+    x, dy = _f32(x), _f32(dy)
+    g = _geom(x.shape, w_shape, stride, pad)
+    co, ci, kh, kw = (int(v) for v in idx)
+    return float(lib().oracle_conv_bwd_filter_at(*g, _ptr(x), _ptr(dy), co, ci, kh, kw))
 
 
 def im2col(x_n, kh, kw, stride=1, pad=0):

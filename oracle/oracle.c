@@ -185,3 +185,24 @@ void oracle_im2col(int C, int H, int W, int Kh, int Kw, int Sh, int Sw, int Ph, 
           }
       }
 }
+
+/* One sampled element of the parameter gradient (same definition as oracle_conv_bwd_filter),
+ * for parity at full benchmark sizes where the whole dW would take minutes. */
+double oracle_conv_bwd_filter_at(int N, int C, int H, int W, int Co, int Kh, int Kw, int Sh,
+                                 int Sw, int Ph, int Pw, const float *x, const float *dy, int co,
+                                 int ci, int kh, int kw) {
+  const int Ho = out_dim(H, Kh, Sh, Ph), Wo = out_dim(W, Kw, Sw, Pw);
+  double acc = 0.0;
+  for (int n = 0; n < N; ++n)
+    for (int ho = 0; ho < Ho; ++ho) {
+      const int ih = ho * Sh - Ph + kh;
+      if (ih < 0 || ih >= H) continue;
+      for (int wo = 0; wo < Wo; ++wo) {
+        const int iw = wo * Sw - Pw + kw;
+        if (iw < 0 || iw >= W) continue;
+        acc += (double)dy[(((size_t)n * Co + co) * Ho + ho) * Wo + wo] *
+               (double)x[(((size_t)n * C + ci) * H + ih) * W + iw];
+      }
+    }
+  return acc;
+}

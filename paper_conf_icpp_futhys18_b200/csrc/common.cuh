@@ -1,0 +1,63 @@
+// common.cuh — shared device/host structs of the conv hot path (not shared with the oracle).
+#pragma once
+#include <cstdint>
+
+namespace glp {
+
+// Division by a run-time constant via multiply-high (valid for 0 <= n < 2^31).
+struct FastDiv {
+  uint32_t d, mul, shr;
+  __host__ __device__ FastDiv() : d(1), mul(0), shr(0) {}
+  __host__ explicit FastDiv(uint32_t div) : d(div) {
+    uint32_t l = 0;
+    while ((1ull << l) < div) ++l;
+    shr = l;
+    mul = (uint32_t)(((1ull << 32) * ((1ull << l) - div)) / div + 1);
+  }
+  __device__ __forceinline__ uint32_t div(uint32_t n) const {
+    return (uint32_t)(((uint64_t)__umulhi(n, mul) + n) >> shr);
+  }
+  __device__ __forceinline__ void divmod(uint32_t n, uint32_t &q, uint32_t &r) const {
+    q = div(n);
+    r = n - q * d;
+  }
+};
+
+enum ConvMode : int { MODE_FWD = 0, MODE_DGRAD = 1, MODE_WGRAD = 2 };
+
+// Geometry of the activation gather (im2col never materialised).  The "pixel space" is the
+// GEMM's pixel dimension: y pixels for fwd (M) and wgrad (K), dx pixels for dgrad (M).
+struct Gather {
+  const void *src;       // packed NHWC source: x (fwd, wgrad) or dy (dgrad)
+  int src_h, src_w;      // source image dims
+  int src_cp;            // channel pitch of the packed source (elements)
+  int pix_hw, pix_w;     // pixel-space dims (H_o*W_o, W_o) for fwd/wgrad; (H*W, W) for dgrad
+  int stride, pad;       // conv stride / pad (symmetric in h and w: stride_h == stride_w here)
+  int stride_w, pad_w;
+  int kw, taps;          // K_w, K_h*K_w
+  int cp;                // channel pitch of the K (or M for wgrad) index: k = tap*cp + c
+  int n_pixels;          // N * pix_hw
+  FastDiv div_hw, div_w, div_cp, div_kw;
+};
+
+struct IgemmParams {
+  Gather g;
+  int M, N;              // valid GEMM extents
+  int m_tiles, n_tiles, splits;
+  int kb_total;          // k-blocks over the whole K extent
+  int kb_per_split;
+  int bn;                // N tile (multiple of 16, <= 256)
+  int bn_smem;           // rows/cols of B held in smem per stage
+  int stages;
+  int tmem_cols;         // columns allocated (power of 2 >= 2 * acc_cols)
+  int acc_cols;          // columns per accumulator buffer
+  // epilogue
+  float *out;            // y (fwd) / dx (dgrad) NCHW, or split partials (wgrad)
+  const float *bias;     // fwd only, may be null
+  int out_c;             // channels of out (C_o fwd, C_i dgrad)
+  int out_hw;            // H_o*W_o (fwd) / H*W (dgrad)
+  int part_ld;           // wgrad partial leading dimension (n_tiles * bn)
+  int part_mpad;         // wgrad partial rows per split (m_tiles * 128)
+};
+
+}  // namespace glp

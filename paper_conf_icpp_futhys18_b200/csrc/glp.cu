@@ -1,0 +1,785 @@
+// glp.cu — libglp.so: the C ABI of include/glp.h.
+//
+// Host side of the GLP4NN hot path re-designed for B200:
+//   * descriptors (Table 5 parameters, P316),
+//   * the kernel analyzer (P167, Eqs 1-9 P214-254) re-derived for sm_100a: CTAs per SM from every
+//     per-SM limit, slots = #SM * beta, samples in flight S (the paper's C_out, P254),
+//   * the plan ("profile once, execute many", P173): tile shapes, shape-only wgrad split count,
+//     stage counts, workspace sizes, persistent grid sizes,
+//   * launches of the pack / tcgen05 implicit-GEMM / reduction kernels on the caller's stream.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "../../include/glp.h"
+#include "common.cuh"
+#include "igemm.cuh"
+#include "pack.cuh"
+#include "simt.cuh"
+
+using namespace glp;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+glp_status_t fail(glp_status_t s, const std::string &msg) {
+  g_last_error = msg;
+  return s;
+}
+glp_status_t cuda_check(cudaError_t e, const char *what) {
+  if (e == cudaSuccess) return GLP_OK;
+  return fail(GLP_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+#define GLP_CUDA(call)                                              \
+  do {                                                              \
+    glp_status_t _s = cuda_check((call), #call);                    \
+    if (_s != GLP_OK) return _s;                                    \
+  } while (0)
+#define GLP_LAUNCH_CHECK(what)                                      \
+  do {                                                              \
+    glp_status_t _s = cuda_check(cudaGetLastError(), what);         \
+    if (_s != GLP_OK) return _s;                                    \
+  } while (0)
+
+inline long long cdiv(long long a, long long b) { return (a + b - 1) / b; }
+inline long long rup(long long a, long long b) { return cdiv(a, b) * b; }
+inline size_t align1k(size_t a) { return (a + 1023) & ~size_t(1023); }
+
+}  // namespace
+
+struct glp_conv_desc_s {
+  int N, C, H, W, Co, Kh, Kw, Sh, Sw, Ph, Pw, Ho, Wo;
+};
+
+namespace {
+
+// ------------------------------------------------------------------ analyzer ---------------
+int ctas_per_sm_closed_form(const glp_device_limits_t &L, const glp_kernel_attr_t &k) {
+  const int warps = (k.threads + 31) / 32;
+  int b = L.max_blocks_per_sm;
+  b = std::min(b, L.max_threads_per_sm / std::max(1, warps * 32));
+  if (k.regs > 0) {
+    const int rpw = (int)rup((long long)k.regs * 32, 256);
+    b = std::min(b, L.regs_per_sm / (rpw * warps));
+  }
+  const int smem_cta = (int)rup(std::max(0, k.smem_bytes), 128) + L.smem_reserved_per_cta;
+  b = std::min(b, L.smem_per_sm / smem_cta);
+  if (k.tmem_cols > 0 && L.tmem_cols_per_sm > 0) b = std::min(b, L.tmem_cols_per_sm / k.tmem_cols);
+  return std::max(0, b);
+}
+
+// One pass of the tensor-core path, planned.
+struct PassPlan {
+  int M = 0, Ng = 0, Kpad = 0;      // GEMM extents (Kpad elements; wgrad: pixels)
+  int bn = 0, bn_smem = 0, m_tiles = 0, n_tiles = 0, splits = 1, kb_total = 0, kb_per_split = 0;
+  int stages = 0, acc_cols = 0, tmem_cols = 0, smem = 0, tiles = 0, grid = 0, ctas_per_sm = 0;
+  int regs = 0, ctas_runtime = 0;
+};
+
+using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                  const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                  const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+TmapEncodeFn g_encode = nullptr;
+std::mutex g_mu;
+
+glp_status_t get_encode() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g_encode) return GLP_OK;
+  void *fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+  if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+    return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled entry point unavailable");
+  g_encode = reinterpret_cast<TmapEncodeFn>(fn);
+  return GLP_OK;
+}
+
+glp_status_t encode_2d(CUtensorMap *map, int elem, const void *ptr, uint64_t inner, uint64_t outer,
+                       uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer,
+                       CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {row_bytes};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = g_encode(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                        2, const_cast<void *>(ptr), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return GLP_OK;
+}
+
+template <int MODE, int ELEM>
+void *kernel_ptr() {
+  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM>);
+}
+void *igemm_ptr(int mode, int elem) {
+  if (elem == 2) {
+    if (mode == MODE_FWD) return kernel_ptr<MODE_FWD, 2>();
+    if (mode == MODE_DGRAD) return kernel_ptr<MODE_DGRAD, 2>();
+    return kernel_ptr<MODE_WGRAD, 2>();
+  }
+  if (mode == MODE_FWD) return kernel_ptr<MODE_FWD, 4>();
+  if (mode == MODE_DGRAD) return kernel_ptr<MODE_DGRAD, 4>();
+  return kernel_ptr<MODE_WGRAD, 4>();
+}
+
+int choose_bn(int n) {
+  if (n <= 256) return (int)rup(n, 16);
+  const int nt = (int)cdiv(n, 256);
+  return (int)rup(cdiv(n, nt), 16);
+}
+
+// Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
+// (constants, never the queried device or S), so the fp32 summation order is a function of the
+// shape alone (convergence invariance, P264).
+int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem) {
+  const double sm = 148.0;
+  const double kb_s = (elem == 2 ? 2.0 : 4.0) * std::max(bn, 96) / 1.8e9;  // seconds per k-block
+  const double bw = 6.0e12;
+  int best = 1;
+  double best_t = 1e30;
+  const int maxs = std::max(1, std::min(kb_total, 512));
+  for (int s = 1; s <= maxs; ++s) {
+    const int kbps = (int)cdiv(kb_total, s);
+    const int real = (int)cdiv(kb_total, kbps);
+    if (real != s) continue;
+    const double waves = std::ceil(tiles_mn * (double)s / sm);
+    const double t = waves * (kbps * kb_s + 2e-6) + (double)s * mpad * npad * 8.0 / bw;
+    if (t < best_t * 0.999) {
+      best_t = t;
+      best = s;
+    }
+  }
+  return best;
+}
+
+}  // namespace
+
+struct glp_plan_s {
+  glp_conv_desc_s d;
+  int device = 0, math = 0, elem = 4, sm_count = 148, s_override = 0;
+  int Cp = 0, Cop = 0, taps = 0;
+  PassPlan fwd, dgrad, wgrad;
+  int S = 1;
+  // SIMT path
+  int simt_splits = 1, simt_chunk = 1;
+  // workspace layout
+  size_t off_xpk = 0, off_dypk = 0, off_wpk = 0, off_part = 0, off_dbpart = 0;
+  size_t sz_xpk = 0, sz_dypk = 0, sz_wpk = 0, sz_wtpk = 0, sz_part = 0, sz_dbpart = 0;
+  int db_rows = 0;
+  size_t ws_fwd = 0, ws_dgrad = 0, ws_wgrad = 0, ws_bwd = 0;
+  double plan_us = 0;
+};
+
+namespace {
+
+glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_limits_t &L) {
+  const int elem = P.elem;
+  const int BK = 128 / elem;
+  const glp_conv_desc_s &d = P.d;
+  if (mode == MODE_FWD) {
+    pp.M = d.N * d.Ho * d.Wo;
+    pp.Ng = d.Co;
+    pp.Kpad = (int)rup((long long)P.taps * P.Cp, BK);
+    pp.kb_total = pp.Kpad / BK;
+    pp.bn = choose_bn(d.Co);
+    pp.bn_smem = pp.bn;
+  } else if (mode == MODE_DGRAD) {
+    pp.M = d.N * d.H * d.W;
+    pp.Ng = d.C;
+    pp.Kpad = (int)rup((long long)P.taps * P.Cop, BK);
+    pp.kb_total = pp.Kpad / BK;
+    pp.bn = choose_bn(d.C);
+    pp.bn_smem = pp.bn;
+  } else {
+    pp.M = P.taps * P.Cp;
+    pp.Ng = d.Co;
+    pp.Kpad = d.N * d.Ho * d.Wo;
+    pp.kb_total = (int)cdiv(pp.Kpad, BK);
+    pp.bn = choose_bn(d.Co);
+    pp.bn_smem = (int)rup(pp.bn, BK);
+  }
+  pp.m_tiles = (int)cdiv(pp.M, 128);
+  pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
+  if (mode == MODE_WGRAD) {
+    pp.splits = choose_splits(pp.m_tiles * pp.n_tiles, pp.kb_total, pp.bn, pp.m_tiles * 128,
+                              pp.n_tiles * pp.bn, elem);
+    pp.kb_per_split = (int)cdiv(pp.kb_total, pp.splits);
+    pp.splits = (int)cdiv(pp.kb_total, pp.kb_per_split);
+  } else {
+    pp.splits = 1;
+    pp.kb_per_split = pp.kb_total;
+  }
+  const int stage_bytes = 16384 + pp.bn_smem * 128;
+  const int budget = 232448 - 1024 - 512;
+  pp.stages = std::min(8, budget / stage_bytes);
+  if (pp.stages < TileCfg<2>::LAG + 1) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
+  pp.acc_cols = (int)rup(pp.bn, 32);
+  int tc = 32;
+  while (tc < 2 * pp.acc_cols) tc *= 2;
+  pp.tmem_cols = tc;
+  pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16;
+  pp.tiles = pp.m_tiles * pp.n_tiles * pp.splits;
+
+  void *fn = igemm_ptr(mode, elem);
+  GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pp.smem));
+  cudaFuncAttributes fa;
+  GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
+  pp.regs = fa.numRegs;
+  glp_kernel_attr_t ka{TileCfg<2>::THREADS, fa.numRegs, pp.smem + (int)fa.sharedSizeBytes, pp.tmem_cols};
+  pp.ctas_per_sm = ctas_per_sm_closed_form(L, ka);
+  int rt = 0;
+  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, TileCfg<2>::THREADS, pp.smem));
+  pp.ctas_runtime = rt;
+  if (pp.ctas_per_sm < 1) return fail(GLP_ERR_INTERNAL, "kernel does not fit on an SM");
+  const int slots = P.sm_count * pp.ctas_per_sm;
+  int grid = std::min(pp.tiles, slots);
+  if (P.s_override > 0 && mode != MODE_WGRAD) {
+    // S samples in flight: the grid covers the tiles of S samples (P262 batch-level parallelism).
+    const int hw = (mode == MODE_FWD) ? d.Ho * d.Wo : d.H * d.W;
+    const long long tiles_s = cdiv((long long)P.s_override * hw, 128) * pp.n_tiles;
+    grid = (int)std::max(1LL, std::min<long long>(grid, tiles_s));
+  } else if (P.s_override > 0) {
+    const long long tiles_s = cdiv((long long)pp.tiles * P.s_override, d.N);
+    grid = (int)std::max(1LL, std::min<long long>(grid, tiles_s));
+  }
+  pp.grid = std::max(1, grid);
+  return GLP_OK;
+}
+
+glp_status_t validate_ptrs(std::initializer_list<const void *> ps) {
+  for (const void *p : ps) {
+    if (!p) return fail(GLP_ERR_INVALID_VALUE, "null pointer argument");
+    if (reinterpret_cast<uintptr_t>(p) % 16) return fail(GLP_ERR_INVALID_VALUE, "pointer not 16-byte aligned");
+  }
+  return GLP_OK;
+}
+
+IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const void *src) {
+  const glp_conv_desc_s &d = P.d;
+  IgemmParams p;
+  memset(&p, 0, sizeof(p));
+  Gather &g = p.g;
+  g.src = src;
+  g.stride = d.Sh;
+  g.stride_w = d.Sw;
+  g.pad = d.Ph;
+  g.pad_w = d.Pw;
+  g.kw = d.Kw;
+  g.taps = P.taps;
+  if (mode == MODE_DGRAD) {
+    g.src_h = d.Ho;
+    g.src_w = d.Wo;
+    g.src_cp = P.Cop;
+    g.cp = P.Cop;
+    g.pix_hw = d.H * d.W;
+    g.pix_w = d.W;
+  } else {
+    g.src_h = d.H;
+    g.src_w = d.W;
+    g.src_cp = P.Cp;
+    g.cp = P.Cp;
+    g.pix_hw = d.Ho * d.Wo;
+    g.pix_w = d.Wo;
+  }
+  g.n_pixels = d.N * g.pix_hw;
+  g.div_hw = FastDiv((uint32_t)g.pix_hw);
+  g.div_w = FastDiv((uint32_t)g.pix_w);
+  g.div_cp = FastDiv((uint32_t)g.cp);
+  g.div_kw = FastDiv((uint32_t)g.kw);
+  p.M = pp.M;
+  p.N = pp.Ng;
+  p.m_tiles = pp.m_tiles;
+  p.n_tiles = pp.n_tiles;
+  p.splits = pp.splits;
+  p.kb_total = pp.kb_total;
+  p.kb_per_split = pp.kb_per_split;
+  p.bn = pp.bn;
+  p.bn_smem = pp.bn_smem;
+  p.stages = pp.stages;
+  p.tmem_cols = pp.tmem_cols;
+  p.acc_cols = pp.acc_cols;
+  p.part_ld = pp.n_tiles * pp.bn;
+  p.part_mpad = pp.m_tiles * 128;
+  return p;
+}
+
+template <int MODE>
+glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
+                          const CUtensorMap &map, cudaStream_t st) {
+  if (P.elem == 2)
+    igemm_kernel<MODE, 2><<<pp.grid, TileCfg<2>::THREADS, pp.smem, st>>>(p, map);
+  else
+    igemm_kernel<MODE, 4><<<pp.grid, TileCfg<4>::THREADS, pp.smem, st>>>(p, map);
+  GLP_LAUNCH_CHECK("igemm_kernel");
+  return GLP_OK;
+}
+
+glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
+                             int Cp, float *db_part, cudaStream_t st) {
+  dim3 grid((unsigned)cdiv(HW, 32), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
+  if (P.elem == 2) pack_nchw_to_nhwc<2><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
+  else pack_nchw_to_nhwc<4><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
+  GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
+  return GLP_OK;
+}
+
+int ew_grid(size_t n) { return (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 16); }
+
+glp_status_t run_fwd_tc(glp_plan_s &P, const float *x, const float *w, const float *b, float *y,
+                        uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
+  glp_status_t s = launch_pack_act(P, x, xpk, d.C, d.H * d.W, P.Cp, nullptr, st);
+  if (s) return s;
+  const size_t wn = (size_t)d.Co * P.fwd.Kpad;
+  if (P.elem == 2) pack_w_fwd<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
+  else pack_w_fwd<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
+  GLP_LAUNCH_CHECK("pack_w_fwd");
+  CUtensorMap map;
+  s = encode_2d(&map, P.elem, wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co, (uint64_t)P.fwd.Kpad * P.elem,
+                128 / P.elem, (uint32_t)P.fwd.bn);
+  if (s) return s;
+  IgemmParams p = make_params(P, P.fwd, MODE_FWD, xpk);
+  p.out = y;
+  p.bias = b;
+  p.out_c = d.Co;
+  p.out_hw = d.Ho * d.Wo;
+  return launch_igemm<MODE_FWD>(P, P.fwd, p, map, st);
+}
+
+glp_status_t run_dgrad_tc(glp_plan_s &P, const void *dypk, const float *w, float *dx, uint8_t *ws,
+                          cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  void *wtpk = ws + P.off_wpk;
+  const size_t wn = (size_t)d.C * P.dgrad.Kpad;
+  if (P.elem == 2) pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
+  else pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
+  GLP_LAUNCH_CHECK("pack_w_dgrad");
+  CUtensorMap map;
+  glp_status_t s = encode_2d(&map, P.elem, wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
+                             (uint64_t)P.dgrad.Kpad * P.elem, 128 / P.elem, (uint32_t)P.dgrad.bn);
+  if (s) return s;
+  IgemmParams p = make_params(P, P.dgrad, MODE_DGRAD, dypk);
+  p.out = dx;
+  p.out_c = d.C;
+  p.out_hw = d.H * d.W;
+  return launch_igemm<MODE_DGRAD>(P, P.dgrad, p, map, st);
+}
+
+glp_status_t run_wgrad_tc(glp_plan_s &P, const void *xpk, const void *dypk, float *dw, float *db,
+                          int accumulate, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  float *part = reinterpret_cast<float *>(ws + P.off_part);
+  CUtensorMap map;
+  const int BK = 128 / P.elem;
+  glp_status_t s = encode_2d(&map, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
+                             (uint64_t)P.Cop * P.elem, (uint32_t)BK, (uint32_t)BK,
+                             P.elem == 2 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                         : CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);
+  if (s) return s;
+  IgemmParams p = make_params(P, P.wgrad, MODE_WGRAD, xpk);
+  p.out = part;
+  s = launch_igemm<MODE_WGRAD>(P, P.wgrad, p, map, st);
+  if (s) return s;
+  const size_t wsz = (size_t)d.Co * d.C * P.taps;
+  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, P.Cp, p.part_ld,
+                                             p.part_mpad, P.wgrad.splits, accumulate);
+  GLP_LAUNCH_CHECK("reduce_tc_dw");
+  if (db) {
+    reduce_db<<<(unsigned)cdiv(d.Co, 128), 128, 0, st>>>(
+        reinterpret_cast<float *>(ws + P.off_dbpart), db, d.Co, P.db_rows, accumulate);
+    GLP_LAUNCH_CHECK("reduce_db");
+  }
+  return GLP_OK;
+}
+
+ConvGeom geom(const glp_conv_desc_s &d) {
+  return ConvGeom{d.N, d.C, d.H, d.W, d.Co, d.Kh, d.Kw, d.Sh, d.Sw, d.Ph, d.Pw, d.Ho, d.Wo};
+}
+
+glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, float *dw, float *db,
+                            int accumulate, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  const size_t wsz = (size_t)d.Co * d.C * d.Kh * d.Kw;
+  float *part = reinterpret_cast<float *>(ws);
+  float *dbp = reinterpret_cast<float *>(ws + align1k(wsz * P.simt_splits * 4));
+  simt_wgrad_partial<<<ew_grid(wsz * P.simt_splits), 256, 0, st>>>(geom(d), x, dy, part, P.simt_splits, P.simt_chunk);
+  GLP_LAUNCH_CHECK("simt_wgrad_partial");
+  reduce_simt_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, wsz, P.simt_splits, accumulate);
+  GLP_LAUNCH_CHECK("reduce_simt_dw");
+  if (db) {
+    simt_db_partial<<<ew_grid((size_t)P.simt_splits * d.Co), 256, 0, st>>>(geom(d), dy, dbp, P.simt_splits, P.simt_chunk);
+    GLP_LAUNCH_CHECK("simt_db_partial");
+    reduce_db<<<(unsigned)cdiv(d.Co, 128), 128, 0, st>>>(dbp, db, d.Co, P.simt_splits, accumulate);
+    GLP_LAUNCH_CHECK("reduce_db");
+  }
+  return GLP_OK;
+}
+
+// Debug im2col through the forward producer's gather (fwd_gather) on the packed operand.
+template <int ELEM>
+__global__ void debug_im2col_kernel(Gather g, int n, int C, int Kh, int Kw, int Ho, int Wo,
+                                    float *col) {
+  const size_t rows = (size_t)C * Kh * Kw, hw = (size_t)Ho * Wo;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < rows * hw;
+       i += (size_t)gridDim.x * blockDim.x) {
+    const int pix = (int)(i % hw);
+    const int r = (int)(i / hw);
+    const int kw = r % Kw, kh = (r / Kw) % Kh, ci = r / (Kw * Kh);
+    const int ho = pix / Wo, wo = pix % Wo;
+    const uint32_t k = (uint32_t)((kh * Kw + kw) * g.cp + ci);
+    const uint32_t kc = k - k % (16 / ELEM);
+    const uint8_t *src = nullptr;
+    float v = 0.f;
+    if (fwd_gather<ELEM>(g, (uint32_t)n, ho * g.stride - g.pad, wo * g.stride_w - g.pad_w, kc, src)) {
+      const int e = (int)(k - kc);
+      if (ELEM == 2) v = __bfloat162float(reinterpret_cast<const __nv_bfloat16 *>(src)[e]);
+      else v = reinterpret_cast<const float *>(src)[e];
+    }
+    col[i] = v;
+  }
+}
+
+}  // namespace
+
+// ====================================================================== C ABI =================
+extern "C" {
+
+int glp_version(void) { return 1; }
+
+const char *glp_status_string(glp_status_t s) {
+  switch (s) {
+    case GLP_OK: return "GLP_OK";
+    case GLP_ERR_INVALID_VALUE: return "GLP_ERR_INVALID_VALUE";
+    case GLP_ERR_NOT_SUPPORTED: return "GLP_ERR_NOT_SUPPORTED";
+    case GLP_ERR_CUDA: return "GLP_ERR_CUDA";
+    case GLP_ERR_WORKSPACE_TOO_SMALL: return "GLP_ERR_WORKSPACE_TOO_SMALL";
+    case GLP_ERR_INTERNAL: return "GLP_ERR_INTERNAL";
+  }
+  return "GLP_ERR_UNKNOWN";
+}
+
+const char *glp_last_error_string(void) { return g_last_error.c_str(); }
+
+glp_status_t glp_conv_desc_create(glp_conv_desc_t *out, int N, int C, int H, int W, int Co, int Kh,
+                                  int Kw, int Sh, int Sw, int Ph, int Pw) {
+  if (!out) return fail(GLP_ERR_INVALID_VALUE, "out is NULL");
+  *out = nullptr;
+  if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || Co <= 0 || Kh <= 0 || Kw <= 0 || Sh <= 0 || Sw <= 0 ||
+      Ph < 0 || Pw < 0)
+    return fail(GLP_ERR_INVALID_VALUE, "non-positive dimension / negative pad");
+  if (H + 2 * Ph < Kh || W + 2 * Pw < Kw) return fail(GLP_ERR_INVALID_VALUE, "H_out < 1");
+  const long long Ho = (H + 2LL * Ph - Kh) / Sh + 1, Wo = (W + 2LL * Pw - Kw) / Sw + 1;
+  // 32-bit index math on the device (FastDiv): every flattened extent must stay < 2^31.
+  if ((long long)N * C * H * W >= (1LL << 31) || (long long)N * Co * Ho * Wo >= (1LL << 31) ||
+      (long long)Co * C * Kh * Kw >= (1LL << 31))
+    return fail(GLP_ERR_NOT_SUPPORTED, "tensor too large for 32-bit indexing");
+  auto *d = new glp_conv_desc_s{N, C, H, W, Co, Kh, Kw, Sh, Sw, Ph, Pw, (int)Ho, (int)Wo};
+  *out = d;
+  return GLP_OK;
+}
+
+glp_status_t glp_conv_desc_get_output(glp_conv_desc_t d, int *Ho, int *Wo) {
+  if (!d || !Ho || !Wo) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *Ho = d->Ho;
+  *Wo = d->Wo;
+  return GLP_OK;
+}
+
+glp_status_t glp_conv_desc_destroy(glp_conv_desc_t d) {
+  delete d;
+  return GLP_OK;
+}
+
+glp_status_t glp_device_limits_b200(glp_device_limits_t *L) {
+  if (!L) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *L = glp_device_limits_t{148, 2048, 32, 65536, 228 * 1024, 1024, 512, 128};
+  return GLP_OK;
+}
+
+glp_status_t glp_analyze_ctas_per_sm(const glp_device_limits_t *L, const glp_kernel_attr_t *k, int *b) {
+  if (!L || !k || !b) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  if (k->threads <= 0 || k->regs < 0 || k->smem_bytes < 0 || k->tmem_cols < 0)
+    return fail(GLP_ERR_INVALID_VALUE, "bad kernel attributes");
+  *b = ctas_per_sm_closed_form(*L, *k);
+  return GLP_OK;
+}
+
+glp_status_t glp_analyze_samples_in_flight(int slots, int tiles_per_sample, int n_local, int *S) {
+  if (!S || slots <= 0 || tiles_per_sample <= 0 || n_local <= 0)
+    return fail(GLP_ERR_INVALID_VALUE, "bad analyzer input");
+  *S = std::max(1, std::min(n_local, slots / tiles_per_sample));
+  return GLP_OK;
+}
+
+glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr_t *k, int blocks,
+                             double t_kernel, double t_launch, int *bound) {
+  if (!L || !k || !bound || blocks <= 0 || k->threads <= 0)
+    return fail(GLP_ERR_INVALID_VALUE, "bad analyzer input");
+  double m = (double)L->max_threads_per_sm * L->sm_count / ((double)k->threads * blocks);
+  if (k->smem_bytes > 0) m = std::min(m, (double)L->smem_per_sm * L->sm_count / ((double)k->smem_bytes * blocks));
+  if (t_kernel > 0 && t_launch > 0) m = std::min(m, std::ceil(t_kernel / t_launch));
+  *bound = (int)std::floor(m);
+  return GLP_OK;
+}
+
+glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t math, int S) {
+  if (!out || !d) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *out = nullptr;
+  if (math != GLP_MATH_FP32 && math != GLP_MATH_TF32 && math != GLP_MATH_BF16)
+    return fail(GLP_ERR_INVALID_VALUE, "unknown math mode");
+  if (S < 0) return fail(GLP_ERR_INVALID_VALUE, "samples_in_flight < 0");
+  const auto t0 = std::chrono::steady_clock::now();
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(GLP_ERR_NOT_SUPPORTED, "no CUDA device (there is no CPU fallback)");
+  }
+  if (device < 0 || device >= ndev) return fail(GLP_ERR_INVALID_VALUE, "bad device ordinal");
+  cudaDeviceProp prop;
+  GLP_CUDA(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10) return fail(GLP_ERR_NOT_SUPPORTED, "libglp.so is built for sm_100a (B200) only");
+  int cur = 0;
+  GLP_CUDA(cudaGetDevice(&cur));
+  if (cur != device) GLP_CUDA(cudaSetDevice(device));
+
+  auto *P = new glp_plan_s();
+  P->d = *d;
+  P->device = device;
+  P->math = (int)math;
+  P->elem = (math == GLP_MATH_BF16) ? 2 : 4;
+  P->sm_count = prop.multiProcessorCount;
+  P->s_override = S;
+  const int CH = 16 / P->elem;
+  P->Cp = (int)rup(d->C, CH);
+  P->Cop = (int)rup(d->Co, CH);
+  P->taps = d->Kh * d->Kw;
+  glp_device_limits_t L;
+  glp_device_limits_b200(&L);
+  L.sm_count = prop.multiProcessorCount;
+  L.smem_per_sm = (int)prop.sharedMemPerMultiprocessor;
+  L.regs_per_sm = prop.regsPerMultiprocessor;
+  L.max_threads_per_sm = prop.maxThreadsPerMultiProcessor;
+  L.max_blocks_per_sm = prop.maxBlocksPerMultiProcessor;
+  L.smem_reserved_per_cta = (int)prop.reservedSharedMemPerBlock;
+
+  glp_status_t s = GLP_OK;
+  if (math != GLP_MATH_FP32) {
+    if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
+        (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {
+      delete P;
+      if (cur != device) cudaSetDevice(cur);
+      return s;
+    }
+    const glp_conv_desc_s &c = *d;
+    P->sz_xpk = align1k((size_t)c.N * c.H * c.W * P->Cp * P->elem);
+    P->sz_dypk = align1k((size_t)c.N * c.Ho * c.Wo * P->Cop * P->elem);
+    P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
+    P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
+    P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_tiles * 128 * P->wgrad.n_tiles * P->wgrad.bn * 4);
+    P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, 32);
+    P->sz_dbpart = align1k((size_t)P->db_rows * c.Co * 4);
+    // one layout serves every call: [xpk | dypk | wpk/wtpk | part | dbpart]
+    P->off_xpk = 0;
+    P->off_dypk = P->sz_xpk;
+    P->off_wpk = P->off_dypk + P->sz_dypk;
+    P->off_part = P->off_wpk + std::max(P->sz_wpk, P->sz_wtpk);
+    P->off_dbpart = P->off_part + P->sz_part;
+    P->ws_fwd = P->off_wpk + P->sz_wpk;
+    P->ws_dgrad = P->off_wpk + P->sz_wtpk;
+    P->ws_wgrad = P->off_dbpart + P->sz_dbpart;
+    P->ws_bwd = P->ws_wgrad;
+    const long long slots = (long long)P->sm_count * P->fwd.ctas_per_sm;
+    const long long per = (long long)d->Ho * d->Wo * P->fwd.n_tiles;  // pixels*n_tiles per sample
+    P->S = (int)std::max(1LL, std::min<long long>(d->N, slots * 128 / std::max(1LL, per)));
+    if (S > 0) P->S = std::min(S, d->N);
+  } else {
+    const long long npix = (long long)d->N * d->Ho * d->Wo;
+    P->simt_chunk = (int)std::max(256LL, cdiv(npix, 256));
+    P->simt_splits = (int)cdiv(npix, P->simt_chunk);
+    const size_t wsz = (size_t)d->Co * d->C * d->Kh * d->Kw;
+    P->ws_fwd = 0;
+    P->ws_dgrad = 0;
+    P->ws_wgrad = align1k(wsz * P->simt_splits * 4) + align1k((size_t)P->simt_splits * d->Co * 4);
+    P->ws_bwd = P->ws_wgrad;
+    P->S = S > 0 ? std::min(S, d->N) : d->N;
+  }
+  if (cur != device) cudaSetDevice(cur);
+  P->plan_us = std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
+  *out = P;
+  return GLP_OK;
+}
+
+glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
+  if (!P || !I) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  memset(I, 0, sizeof(*I));
+  I->samples_in_flight = P->S;
+  I->ctas_per_sm = P->fwd.ctas_per_sm;
+  I->grid_fwd = P->fwd.grid;
+  I->grid_bwd_data = P->dgrad.grid;
+  I->grid_bwd_filter = P->wgrad.grid;
+  I->tile_m = 128;
+  I->tile_n_fwd = P->fwd.bn;
+  I->tile_n_bwd_data = P->dgrad.bn;
+  I->tile_n_bwd_filter = P->wgrad.bn;
+  I->stages_fwd = P->fwd.stages;
+  I->stages_bwd_data = P->dgrad.stages;
+  I->stages_bwd_filter = P->wgrad.stages;
+  I->splits_wgrad = P->math == GLP_MATH_FP32 ? P->simt_splits : P->wgrad.splits;
+  I->tiles_fwd = P->fwd.tiles;
+  I->tiles_bwd_data = P->dgrad.tiles;
+  I->tiles_bwd_filter = P->wgrad.tiles;
+  I->ws_fwd = P->ws_fwd;
+  I->ws_bwd_data = P->ws_dgrad;
+  I->ws_bwd_filter = P->ws_wgrad;
+  I->ws_bwd = P->ws_bwd;
+  I->plan_us = P->plan_us;
+  I->math = P->math;
+  return GLP_OK;
+}
+
+glp_status_t glp_plan_kernel_attr(glp_plan_t P, int which, glp_kernel_attr_t *a, int *model, int *rt) {
+  if (!P || !a || !model || !rt || which < 0 || which > 2) return fail(GLP_ERR_INVALID_VALUE, "bad argument");
+  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no persistent kernel");
+  const PassPlan &pp = which == 0 ? P->fwd : which == 1 ? P->dgrad : P->wgrad;
+  *a = glp_kernel_attr_t{TileCfg<2>::THREADS, pp.regs, pp.smem, pp.tmem_cols};
+  *model = pp.ctas_per_sm;
+  *rt = pp.ctas_runtime;
+  return GLP_OK;
+}
+
+glp_status_t glp_plan_destroy(glp_plan_t P) {
+  delete P;
+  return GLP_OK;
+}
+
+static glp_status_t check_ws(const glp_plan_s *P, const void *ws, size_t have, size_t need) {
+  if (need == 0) return GLP_OK;
+  if (!ws) return fail(GLP_ERR_INVALID_VALUE, "workspace is NULL");
+  if (reinterpret_cast<uintptr_t>(ws) % 1024)
+    return fail(GLP_ERR_INVALID_VALUE, "workspace must be 1024-byte aligned");
+  if (have < need) return fail(GLP_ERR_WORKSPACE_TOO_SMALL, "workspace too small");
+  (void)P;
+  return GLP_OK;
+}
+
+glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const float *b, float *y,
+                          void *ws, size_t ws_bytes, glp_stream_t stream) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  glp_status_t s = validate_ptrs({x, w, y});
+  if (s) return s;
+  if (b && (reinterpret_cast<uintptr_t>(b) % 4)) return fail(GLP_ERR_INVALID_VALUE, "bias misaligned");
+  if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (P->math == GLP_MATH_FP32) {
+    const size_t n = (size_t)P->d.N * P->d.Co * P->d.Ho * P->d.Wo;
+    simt_fwd<<<ew_grid(n), 256, 0, st>>>(geom(P->d), x, w, b, y);
+    GLP_LAUNCH_CHECK("simt_fwd");
+    return GLP_OK;
+  }
+  if ((s = get_encode())) return s;
+  return run_fwd_tc(*P, x, w, b, y, static_cast<uint8_t *>(ws), st);
+}
+
+glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, float *dx, void *ws,
+                               size_t ws_bytes, glp_stream_t stream) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  glp_status_t s = validate_ptrs({dy, w, dx});
+  if (s) return s;
+  if ((s = check_ws(P, ws, ws_bytes, P->ws_dgrad))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (P->math == GLP_MATH_FP32) {
+    const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
+    simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geom(P->d), dy, w, dx);
+    GLP_LAUNCH_CHECK("simt_dgrad");
+    return GLP_OK;
+  }
+  if ((s = get_encode())) return s;
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  void *dypk = wsb + P->off_dypk;
+  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st))) return s;
+  return run_dgrad_tc(*P, dypk, w, dx, wsb, st);
+}
+
+glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, float *dw, float *db,
+                                 int accumulate, void *ws, size_t ws_bytes, glp_stream_t stream) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  glp_status_t s = validate_ptrs({x, dy, dw});
+  if (s) return s;
+  if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
+  if ((s = check_ws(P, ws, ws_bytes, P->ws_wgrad))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  if (P->math == GLP_MATH_FP32) return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
+  if ((s = get_encode())) return s;
+  void *xpk = wsb + P->off_xpk, *dypk = wsb + P->off_dypk;
+  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
+                           db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
+    return s;
+  return run_wgrad_tc(*P, xpk, dypk, dw, db, accumulate ? 1 : 0, wsb, st);
+}
+
+glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const float *w, float *dx,
+                          float *dw, float *db, int accumulate, void *ws, size_t ws_bytes,
+                          glp_stream_t stream) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  glp_status_t s = validate_ptrs({x, dy, w, dw});
+  if (s) return s;
+  if (dx && (reinterpret_cast<uintptr_t>(dx) % 16)) return fail(GLP_ERR_INVALID_VALUE, "dx misaligned");
+  if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
+  if ((s = check_ws(P, ws, ws_bytes, P->ws_bwd))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  if (P->math == GLP_MATH_FP32) {
+    if (dx) {
+      const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
+      simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geom(P->d), dy, w, dx);
+      GLP_LAUNCH_CHECK("simt_dgrad");
+    }
+    return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
+  }
+  if ((s = get_encode())) return s;
+  void *xpk = wsb + P->off_xpk, *dypk = wsb + P->off_dypk;
+  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
+                           db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
+    return s;
+  if (dx && (s = run_dgrad_tc(*P, dypk, w, dx, wsb, st))) return s;
+  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  return run_wgrad_tc(*P, xpk, dypk, dw, db, accumulate ? 1 : 0, wsb, st);
+}
+
+glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, void *ws,
+                              size_t ws_bytes, glp_stream_t stream) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  glp_status_t s = validate_ptrs({x, col});
+  if (s) return s;
+  if (n < 0 || n >= P->d.N) return fail(GLP_ERR_INVALID_VALUE, "sample index out of range");
+  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no packed operand");
+  if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  void *xpk = wsb + P->off_xpk;
+  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  IgemmParams p = make_params(*P, P->fwd, MODE_FWD, xpk);
+  const size_t total = (size_t)P->d.C * P->taps * P->d.Ho * P->d.Wo;
+  if (P->elem == 2)
+    debug_im2col_kernel<2><<<ew_grid(total), 256, 0, st>>>(p.g, n, P->d.C, P->d.Kh, P->d.Kw, P->d.Ho, P->d.Wo, col);
+  else
+    debug_im2col_kernel<4><<<ew_grid(total), 256, 0, st>>>(p.g, n, P->d.C, P->d.Kh, P->d.Kw, P->d.Ho, P->d.Wo, col);
+  GLP_LAUNCH_CHECK("debug_im2col_kernel");
+  return GLP_OK;
+}
+
+}  // extern "C"

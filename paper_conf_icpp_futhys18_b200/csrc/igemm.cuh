@@ -1,0 +1,371 @@
+// igemm.cuh — persistent, warp-specialised implicit-GEMM convolution on sm_100a tensor cores.
+//
+// One kernel template serves the three passes of the GLP4NN hot path (Alg. 1 P82-99,
+// Alg. 2 P101-121, parameter gradients P129; north_star (3)):
+//   MODE_FWD  : D[pixel(n,ho,wo), co] = sum_{(kh,kw,ci)} x[n, ho*S-P+kh, wo*S-P+kw, ci] * W[co,(kh,kw,ci)]
+//               (im2col never materialised: the A operand is gathered from packed NHWC x)
+//   MODE_DGRAD: D[pixel(n,h,w), ci]  = sum_{(kh,kw,co)} dy[n, (h+P-kh)/S, (w+P-kw)/S, co] * Wt[ci,(kh,kw,co)]
+//               (col2im folded into the gather: every dx element is owned by one CTA, no atomics)
+//   MODE_WGRAD: D[(kh,kw,ci), co]    = sum_{pixels p in split} x[gather(p,kh,kw), ci] * dy[p, co]
+//               (fixed, shape-only split of the N*H_o*W_o reduction; partials reduced in order)
+//
+// CTA = 288 threads: warps 0-3 epilogue (TMEM -> registers -> global), warps 4-7 producers
+// (cp.async gather of A into the UMMA SWIZZLE_128B layout), warp 8 TMEM allocator + single-thread
+// tcgen05.mma issuer.  B (weights, or dy for wgrad) is a dense 2-D matrix loaded by TMA.
+// smem ring of `stages` {A,B} slots (mbarrier full/empty), two TMEM accumulators (tfull/tempty)
+// so the epilogue of tile i overlaps the main loop of tile i+1.  Tiles are visited by a static
+// round-robin over a persistent grid (tile t -> CTA t mod grid), the device-side replacement of
+// the paper's round-robin stream dispatch (P171).
+#pragma once
+#include "common.cuh"
+#include "ptx.cuh"
+
+namespace glp {
+
+template <int ELEM>
+struct TileCfg {
+  static constexpr int BM = 128;
+  static constexpr int BK = 128 / ELEM;      // K elements per 128-byte smem row
+  static constexpr int CH = 16 / ELEM;       // elements per 16-byte chunk
+  static constexpr int UMMA_K = 32 / ELEM;   // K of one tcgen05.mma (bf16 16, tf32 8)
+  static constexpr int A_BYTES = BM * 128;   // 16 KB
+  static constexpr int LBO_MN = (BK / 8) * 1024;  // MN-major: stride between 128-byte MN atoms
+  static constexpr int LAG = 3;              // cp.async groups kept in flight per producer
+  static constexpr int THREADS = 288;
+};
+
+__device__ __forceinline__ void decode_tile(int t, int n_tiles, int m_tiles, int &m_tile,
+                                            int &n_tile, int &split) {
+  n_tile = t % n_tiles;
+  const int r = t / n_tiles;
+  m_tile = r % m_tiles;
+  split = r / m_tiles;
+}
+
+// Forward-gather address of one 16-byte chunk: pixel m (GEMM row) and K index k0 (tap*cp + c).
+// Shared by the producer and glp_debug_im2col so that the debug view uses the kernel's own
+// index math.  Returns false for padding / out-of-range taps (chunk is zero).
+template <int ELEM>
+__device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS, int owS,
+                                           uint32_t k0, const uint8_t *&src) {
+  uint32_t t, c;
+  g.div_cp.divmod(k0, t, c);
+  if ((int)t >= g.taps) return false;
+  uint32_t kh, kw;
+  g.div_kw.divmod(t, kh, kw);
+  const int ih = ohS + (int)kh, iw = owS + (int)kw;
+  if (ih < 0 || ih >= g.src_h || iw < 0 || iw >= g.src_w) return false;
+  src = static_cast<const uint8_t *>(g.src) +
+        ((size_t)((size_t)n * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) * g.src_cp + c) * ELEM;
+  return true;
+}
+
+template <int MODE, int ELEM>
+__global__ void __launch_bounds__(288, 1)
+    igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB) {
+  using C = TileCfg<ELEM>;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023u) & ~1023u;
+  const uint32_t stage_bytes = C::A_BYTES + (uint32_t)p.bn_smem * 128u;
+  const uint32_t bars = base + (uint32_t)p.stages * stage_bytes;
+  const int S_ = p.stages;
+  auto full = [&](int s) { return bars + 8u * s; };
+  auto empty = [&](int s) { return bars + 8u * (S_ + s); };
+  auto tfull = [&](int a) { return bars + 8u * (2 * S_ + a); };
+  auto tempty = [&](int a) { return bars + 8u * (2 * S_ + 2 + a); };
+  const uint32_t tmem_slot = bars + 8u * (2 * S_ + 4);
+  volatile uint32_t *tmem_slot_ptr =
+      reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S_; ++s) {
+      mbar_init(full(s), 129);   // 128 producer arrivals + 1 expect_tx arrival (TMA bytes)
+      mbar_init(empty(s), 1);    // tcgen05.commit
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(tfull(a), 1);    // tcgen05.commit after the last k-block of a tile
+      mbar_init(tempty(a), 128); // every epilogue thread
+    }
+    fence_mbar_init();
+  }
+  if (warp == 8) {
+    tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
+    tmem_relinquish();
+  }
+  if (warp == 4 && lane == 0) tma_prefetch(&tmapB);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot_ptr;
+
+  const int total_tiles = p.m_tiles * p.n_tiles * p.splits;
+  const Gather &g = p.g;
+
+  if (warp >= 4 && warp < 8) {
+    // ===================================== producers =======================================
+    const int pt = threadIdx.x - 128;
+    uint32_t gk = 0;  // CTA-local k-block counter (ring position)
+    for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+      int m_tile, n_tile, split;
+      decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+      int kb0 = 0, kb1 = p.kb_total;
+      if (MODE == MODE_WGRAD) {
+        kb0 = split * p.kb_per_split;
+        kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+      }
+      const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
+      if (MODE != MODE_WGRAD) {
+        // K-major A: thread owns chunk j of rows rg + 16 i.
+        const int j = pt & 7, rg = pt >> 3;
+        uint32_t nimg[8];
+        int ohS[8], owS[8];
+        bool mv[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const int m = m0 + rg + 16 * i;
+          mv[i] = m < p.M;
+          uint32_t n, rem, oh, ow;
+          g.div_hw.divmod((uint32_t)(mv[i] ? m : 0), n, rem);
+          g.div_w.divmod(rem, oh, ow);
+          nimg[i] = n;
+          if (MODE == MODE_FWD) {
+            ohS[i] = (int)oh * g.stride - g.pad;
+            owS[i] = (int)ow * g.stride_w - g.pad_w;
+          } else {
+            ohS[i] = (int)oh + g.pad;
+            owS[i] = (int)ow + g.pad_w;
+          }
+        }
+        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+          const int s = (int)(gk % (uint32_t)S_);
+          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+          mbar_wait(empty(s), ph ^ 1u);
+          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
+          if (pt == 0) {
+            mbar_arrive_expect_tx(full(s), (uint32_t)p.bn_smem * 128u);
+            tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
+          }
+          const uint32_t k0 = (uint32_t)(kb * C::BK + j * C::CH);
+          if (MODE == MODE_FWD) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const int r = rg + 16 * i;
+              const uint8_t *src = static_cast<const uint8_t *>(g.src);
+              const bool ok = mv[i] && fwd_gather<ELEM>(g, nimg[i], ohS[i], owS[i], k0, src);
+              const uint32_t dst = sA + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
+                                   (uint32_t)((j ^ (r & 7)) << 4);
+              cp_async16(dst, src, ok);
+            }
+          } else {
+            uint32_t t, c;
+            g.div_cp.divmod(k0, t, c);
+            const bool kv = (int)t < g.taps;
+            uint32_t kh, kw;
+            g.div_kw.divmod(kv ? t : 0u, kh, kw);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const int r = rg + 16 * i;
+              const int ihn = ohS[i] - (int)kh, iwn = owS[i] - (int)kw;
+              bool ok = kv && mv[i] && ihn >= 0 && iwn >= 0;
+              int ih = ihn, iw = iwn;
+              if (g.stride != 1 || g.stride_w != 1) {
+                ok = ok && (ihn % g.stride == 0) && (iwn % g.stride_w == 0);
+                ih = ihn / g.stride;
+                iw = iwn / g.stride_w;
+              }
+              ok = ok && ih < g.src_h && iw < g.src_w;
+              const uint8_t *src = static_cast<const uint8_t *>(g.src);
+              if (ok)
+                src += ((size_t)((size_t)nimg[i] * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) *
+                            g.src_cp + c) * ELEM;
+              const uint32_t dst = sA + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
+                                   (uint32_t)((j ^ (r & 7)) << 4);
+              cp_async16(dst, src, ok);
+            }
+          }
+          cp_async_commit();
+          if (gk >= (uint32_t)C::LAG) {
+            cp_async_wait<C::LAG>();
+            fence_proxy_async_smem();
+            mbar_arrive(full((int)((gk - C::LAG) % (uint32_t)S_)));
+          }
+        }
+      } else {
+        // WGRAD: MN-major A (M = (tap, ci) of x, K = pixels).  CPR chunks per K-row.
+        constexpr int CPR = 128 * ELEM / 16;
+        constexpr int RPP = 128 / CPR;
+        const int j = pt % CPR, r0 = pt / CPR;
+        const uint32_t mm = (uint32_t)(m0 + j * C::CH);
+        uint32_t t, c;
+        g.div_cp.divmod(mm, t, c);
+        const bool mvalid = (int)t < g.taps;
+        uint32_t kh, kw;
+        g.div_kw.divmod(mvalid ? t : 0u, kh, kw);
+        const int offh = (int)kh - g.pad, offw = (int)kw - g.pad_w;
+        const uint32_t dcol = (uint32_t)(j >> 3) * C::LBO_MN;
+        const int jj = j & 7;
+        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+          const int s = (int)(gk % (uint32_t)S_);
+          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+          mbar_wait(empty(s), ph ^ 1u);
+          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
+          if (pt == 0) {
+            mbar_arrive_expect_tx(full(s), (uint32_t)p.bn_smem * 128u);
+            for (int a = 0; a < p.bn_smem / C::BK; ++a)
+              tma_load_2d(sB + (uint32_t)a * C::LBO_MN, &tmapB, full(s), n0 + a * C::BK,
+                          kb * C::BK);
+          }
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int r = r0 + RPP * i;
+            const int pix = kb * C::BK + r;
+            bool ok = mvalid && pix < g.n_pixels;
+            uint32_t n, rem, oh, ow;
+            g.div_hw.divmod((uint32_t)(ok ? pix : 0), n, rem);
+            g.div_w.divmod(rem, oh, ow);
+            const int ih = (int)oh * g.stride + offh, iw = (int)ow * g.stride_w + offw;
+            ok = ok && ih >= 0 && ih < g.src_h && iw >= 0 && iw < g.src_w;
+            const uint8_t *src = static_cast<const uint8_t *>(g.src);
+            if (ok)
+              src += ((size_t)((size_t)n * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) *
+                          g.src_cp + c) * ELEM;
+            uint32_t dst;
+            if (ELEM == 2)  // SWIZZLE_128B: 16-byte chunks XOR row%8, 8-row (1 KB) K-groups
+              dst = sA + dcol + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
+                    (uint32_t)((jj ^ (r & 7)) << 4);
+            else            // SWIZZLE_128B_BASE32B: 32-byte chunks XOR row%4, 4-row K-groups
+              dst = sA + dcol + (uint32_t)(r >> 2) * 512u + (uint32_t)(r & 3) * 128u +
+                    (uint32_t)((((jj >> 1) ^ (r & 3)) << 5) | ((jj & 1) << 4));
+            cp_async16(dst, src, ok);
+          }
+          cp_async_commit();
+          if (gk >= (uint32_t)C::LAG) {
+            cp_async_wait<C::LAG>();
+            fence_proxy_async_smem();
+            mbar_arrive(full((int)((gk - C::LAG) % (uint32_t)S_)));
+          }
+        }
+      }
+    }
+    cp_async_wait<0>();
+    fence_proxy_async_smem();
+    for (uint32_t q = (gk > (uint32_t)C::LAG ? gk - C::LAG : 0u); q < gk; ++q)
+      mbar_arrive(full((int)(q % (uint32_t)S_)));
+  } else if (warp == 8) {
+    // ===================================== MMA issuer ======================================
+    if (lane == 0) {
+      constexpr uint32_t fmt = (ELEM == 2) ? 1u : 2u;  // BF16 : TF32
+      constexpr uint32_t mn = (MODE == MODE_WGRAD) ? 1u : 0u;
+      const uint32_t idesc = make_idesc(fmt, mn, mn, 128u, (uint32_t)p.bn);
+      uint32_t gk = 0, it = 0;
+      for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++it) {
+        int m_tile, n_tile, split;
+        decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+        int kb0 = 0, kb1 = p.kb_total;
+        if (MODE == MODE_WGRAD) {
+          kb0 = split * p.kb_per_split;
+          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+        }
+        const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
+        mbar_wait(tempty(a), aph ^ 1u);
+        tc_fence_after();
+        const uint32_t d = tmem_base + a * (uint32_t)p.acc_cols;
+        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+          const int s = (int)(gk % (uint32_t)S_);
+          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+          mbar_wait(full(s), ph);
+          tc_fence_after();
+          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
+#pragma unroll
+          for (int k = 0; k < C::BK / C::UMMA_K; ++k) {
+            uint64_t ad, bd;
+            if (MODE == MODE_WGRAD) {
+              // each UMMA_K step covers UMMA_K rows of 128 B (bf16 16 rows, tf32 8 rows)
+              constexpr uint32_t kstep = C::UMMA_K * 128u;
+              constexpr uint32_t sbo = (ELEM == 2) ? 1024u : 512u;
+              constexpr uint32_t lay = (ELEM == 2) ? 2u : 1u;
+              ad = make_sdesc(sA + (uint32_t)k * kstep, C::LBO_MN, sbo, lay);
+              bd = make_sdesc(sB + (uint32_t)k * kstep, C::LBO_MN, sbo, lay);
+            } else {
+              ad = make_sdesc(sA + (uint32_t)k * 32u, 16u, 1024u);
+              bd = make_sdesc(sB + (uint32_t)k * 32u, 16u, 1024u);
+            }
+            const uint32_t acc = (kb > kb0 || k > 0) ? 1u : 0u;
+            if (ELEM == 2) mma_f16(d, ad, bd, idesc, acc);
+            else mma_tf32(d, ad, bd, idesc, acc);
+          }
+          mma_commit(empty(s));
+        }
+        mma_commit(tfull(a));
+      }
+    }
+    __syncwarp();
+  } else {
+    // ===================================== epilogue ========================================
+    const int row = warp * 32 + lane;
+    uint32_t it = 0;
+    for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++it) {
+      int m_tile, n_tile, split;
+      decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+      const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
+      mbar_wait(tfull(a), aph);
+      tc_fence_after();
+      const int m = m_tile * C::BM + row;
+      const int n0 = n_tile * p.bn;
+      const bool mv = m < p.M;
+      const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
+      if (MODE != MODE_WGRAD) {
+        uint32_t n, pimg;
+        g.div_hw.divmod((uint32_t)(mv ? m : 0), n, pimg);
+        float *outp = p.out + (size_t)n * p.out_c * p.out_hw + pimg;
+        for (int c0 = 0; c0 < p.bn; c0 += 32) {
+          uint32_t v[32];
+          tmem_ld32(taddr + (uint32_t)c0, v);
+          tmem_wait_ld();
+          if (mv) {
+#pragma unroll
+            for (int q = 0; q < 32; ++q) {
+              const int ch = n0 + c0 + q;
+              if (c0 + q < p.bn && ch < p.N) {
+                float val = __uint_as_float(v[q]);
+                if (MODE == MODE_FWD && p.bias) val += __ldg(p.bias + ch);
+                outp[(size_t)ch * p.out_hw] = val;
+              }
+            }
+          }
+        }
+      } else {
+        float *dst = p.out + ((size_t)split * p.part_mpad + (size_t)m) * p.part_ld + n0;
+        for (int c0 = 0; c0 < p.bn; c0 += 32) {
+          uint32_t v[32];
+          tmem_ld32(taddr + (uint32_t)c0, v);
+          tmem_wait_ld();
+          if (mv) {
+            const int lim = min(32, p.bn - c0);
+            if (lim == 32) {
+#pragma unroll
+              for (int q = 0; q < 32; q += 4)
+                *reinterpret_cast<float4 *>(dst + c0 + q) =
+                    make_float4(__uint_as_float(v[q]), __uint_as_float(v[q + 1]),
+                                __uint_as_float(v[q + 2]), __uint_as_float(v[q + 3]));
+            } else {
+#pragma unroll
+              for (int q = 0; q < 32; ++q)
+                if (q < lim) dst[c0 + q] = __uint_as_float(v[q]);
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(tempty(a));
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 8) tmem_dealloc(tmem_base, (uint32_t)p.tmem_cols);
+}
+
+}  // namespace glp

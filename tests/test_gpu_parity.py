@@ -1,0 +1,196 @@
+"""GPU parity of the CUDA path (through the C ABI) against the fp64 oracle.
+
+Bars: normwise max|g-r|/max|r| <= 1e-5 (GLP_MATH_FP32) and <= 2e-2
+(TF32/BF16, BASELINE.json north_star); bit-exact on integer-valued inputs in every math mode;
+TF32/BF16 vs a rounding-emulated oracle (oracle run on RNA/RNE-rounded operands) <= 1e-4;
+bitwise invariance of every output across samples-in-flight S (convergence invariance, P264).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_icpp_futhys18_b200 as glp
+from glp_workloads import gen_custom
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda:0")
+TOL = {"fp32": 1e-5, "tf32": 2e-2, "bf16": 2e-2}
+EMU = {"tf32": oracle.round_tf32_rna, "bf16": oracle.round_bf16_rne}
+
+# name, N, C, H, W, Co, K, S, P  — several M tiles, ragged tails, odd geometry
+SHAPES = [
+    ("lenet_conv2", 4, 20, 12, 12, 50, 5, 1, 0),
+    ("cifar_conv1", 3, 3, 32, 32, 32, 5, 1, 2),
+    ("caffenet_conv1_s4", 2, 3, 67, 67, 96, 11, 4, 0),
+    ("ragged_s2", 3, 13, 9, 11, 37, 3, 2, 1),
+    ("gnet_1x1", 5, 832, 7, 7, 48, 1, 1, 0),
+    ("gnet_conv_1", 4, 160, 7, 7, 320, 3, 1, 1),
+    ("caffenet_conv3", 2, 256, 13, 13, 384, 3, 1, 1),
+    ("c1_k5", 2, 1, 28, 28, 20, 5, 1, 0),
+    ("ho1", 2, 4, 5, 5, 3, 5, 1, 0),
+    ("pad3", 2, 3, 10, 10, 2, 3, 1, 3),
+]
+
+
+def _run(layer, d, math_dev=DEV):
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    y = torch.full(layer.y_shape, float("nan"), device=DEV)
+    dx = torch.full(layer.x_shape, float("nan"), device=DEV)
+    dw = torch.full(layer.w_shape, float("nan"), device=DEV)
+    db = torch.full((layer.geom.Co,), float("nan"), device=DEV)
+    layer.fwd(t["x"], t["w"], t["b"], y)
+    layer.bwd_data(t["dy"], t["w"], dx)
+    layer.bwd_filter(t["x"], t["dy"], dw, db)
+    torch.cuda.synchronize()
+    return {"y": y.cpu().numpy(), "dx": dx.cpu().numpy(), "dw": dw.cpu().numpy(), "db": db.cpu().numpy()}
+
+
+def _oracle(d, S, P, x=None, w=None, dy=None):
+    x = d["x"] if x is None else x
+    w = d["w"] if w is None else w
+    dy = d["dy"] if dy is None else dy
+    y = oracle.conv_fwd(x, w, d["b"], S, P)
+    dx = oracle.conv_bwd_data(dy, w, x.shape, S, P)
+    dw, _ = oracle.conv_bwd_filter(x, dy, w.shape, S, P)
+    db = d["dy"].astype(np.float64).sum(axis=(0, 2, 3))
+    return {"y": y, "dx": dx, "dw": dw, "db": db}
+
+
+def _data(shape, exact=False, seed=1):
+    _, N, C, H, W, Co, K, S, P = shape
+    Ho, Wo = oracle.out_dim(H, K, S, P), oracle.out_dim(W, K, S, P)
+    return gen_custom(N, C, H, W, Co, K, K, seed, exact=exact, Ho=Ho, Wo=Wo, data_fed=exact and C <= 3)
+
+
+def _layer(shape, math, S=0):
+    _, N, C, H, W, Co, K, St, P = shape
+    return glp.ConvLayer(N, C, H, W, Co, K, St, P, math=math, samples_in_flight=S)
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
+def test_parity_random(shape, math):
+    d = _data(shape)
+    got = _run(_layer(shape, math), d)
+    ref = _oracle(d, shape[7], shape[8])
+    errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
+    assert all(np.isfinite(got[k]).all() for k in got), errs
+    assert all(e <= TOL[math] for e in errs.values()), errs
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
+def test_parity_rounding_emulated(shape, math):
+    """Oracle on the operands rounded exactly as the pack step defines (oracle.round_*):
+    catches indexing bugs that the 2e-2 tolerance would hide."""
+    d = _data(shape, seed=5)
+    got = _run(_layer(shape, math), d)
+    r = EMU[math]
+    ref = _oracle(d, shape[7], shape[8], x=r(d["x"]), w=r(d["w"]), dy=r(d["dy"]))
+    errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
+    assert all(e <= 1e-4 for e in errs.values()), errs
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
+def test_exact_integer_bitexact(shape, math):
+    """Integer data in [-2,2]: every partial sum is an exact integer < 2^24 in fp32/TF32/BF16,
+    so the GPU must equal the oracle bit for bit (pins indexing, padding, stride, layout and
+    reduction completeness independently of rounding)."""
+    d = _data(shape, exact=True, seed=9)
+    got = _run(_layer(shape, math), d)
+    ref = _oracle(d, shape[7], shape[8])
+    for k in ref:
+        np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[2], SHAPES[5], SHAPES[6]], ids=lambda s: s[0])
+def test_samples_in_flight_invariance(shape, math):
+    """Convergence invariance (P264): outputs bitwise identical for every S and on rerun."""
+    d = _data(shape, seed=3)
+    N = shape[1]
+    base = _run(_layer(shape, math, S=0), d)
+    for S in sorted({1, 2, N}):
+        got = _run(_layer(shape, math, S=S), d)
+        for k in base:
+            np.testing.assert_array_equal(got[k], base[k], err_msg=f"S={S} {k}")
+    again = _run(_layer(shape, math, S=0), d)
+    for k in base:
+        np.testing.assert_array_equal(again[k], base[k])
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape", [SHAPES[1], SHAPES[2], SHAPES[3], SHAPES[6]], ids=lambda s: s[0])
+def test_im2col_layout_bitexact(shape, math):
+    """glp_debug_im2col (the producer's own gather math on the packed operand) equals the
+    oracle's Caffe im2col of the rounded input, bit for bit."""
+    _, N, C, H, W, Co, K, S, P = shape
+    d = _data(shape, seed=4)
+    layer = _layer(shape, math)
+    x = torch.from_numpy(d["x"]).to(DEV)
+    Ho, Wo = layer.Ho, layer.Wo
+    for n in sorted({0, N - 1}):
+        col = torch.empty((C * K * K, Ho * Wo), device=DEV)
+        layer.debug_im2col(x, n, col)
+        torch.cuda.synchronize()
+        ref = oracle.im2col(EMU[math](d["x"][n]), K, K, S, P)
+        np.testing.assert_array_equal(col.cpu().numpy(), ref)
+
+
+def test_accumulate_flag():
+    shape = SHAPES[0]
+    d = _data(shape, exact=True, seed=12)
+    layer = _layer(shape, "bf16")
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    dw = torch.ones(layer.w_shape, device=DEV)
+    db = torch.ones(layer.geom.Co, device=DEV)
+    layer.bwd_filter(t["x"], t["dy"], dw, db, accumulate=True)
+    torch.cuda.synchronize()
+    rdw, _ = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, shape[7], shape[8])
+    np.testing.assert_array_equal(dw.cpu().numpy(), (rdw + 1).astype(np.float32))
+    np.testing.assert_array_equal(db.cpu().numpy(), (d["dy"].astype(np.float64).sum((0, 2, 3)) + 1).astype(np.float32))
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+def test_combined_bwd_equals_separate(math):
+    shape = SHAPES[5]
+    d = _data(shape, seed=8)
+    layer = _layer(shape, math)
+    sep = _run(layer, d)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    dx = torch.empty(layer.x_shape, device=DEV)
+    dw = torch.empty(layer.w_shape, device=DEV)
+    db = torch.empty(layer.geom.Co, device=DEV)
+    layer.bwd(t["x"], t["dy"], t["w"], dx, dw, db)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(dx.cpu().numpy(), sep["dx"])
+    np.testing.assert_array_equal(dw.cpu().numpy(), sep["dw"])
+    np.testing.assert_array_equal(db.cpu().numpy(), sep["db"])
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+def test_analyzer_matches_occupancy_api(math):
+    """The re-derived analyzer's CTAs/SM for every shipped kernel equals the CUDA occupancy API."""
+    for shape in SHAPES:
+        layer = _layer(shape, math)
+        for which in range(3):
+            a = layer.kernel_attr(which)
+            assert a["model"] == a["runtime"] >= 1, (shape[0], which, a)
+
+
+def test_error_paths_on_device():
+    layer = _layer(SHAPES[0], "bf16")
+    x = torch.zeros(layer.x_shape, device=DEV)
+    y = torch.zeros(layer.y_shape, device=DEV)
+    w = torch.zeros(layer.w_shape, device=DEV)
+    L = glp.lib()
+    import ctypes
+    rc = L.glp_conv_fwd(layer._plan, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(w.data_ptr()),
+                        None, ctypes.c_void_p(y.data_ptr()), ctypes.c_void_p(layer.ws_ptr), 16, None)
+    assert rc == 4  # GLP_ERR_WORKSPACE_TOO_SMALL
+    rc = L.glp_conv_fwd(layer._plan, ctypes.c_void_p(x.data_ptr() + 4), ctypes.c_void_p(w.data_ptr()),
+                        None, ctypes.c_void_p(y.data_ptr()), ctypes.c_void_p(layer.ws_ptr),
+                        layer.ws_bytes, None)
+    assert rc == 1  # misaligned

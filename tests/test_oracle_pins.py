@@ -230,3 +230,12 @@ def test_rounding_error_bounds():
     hi, lo = oracle.split_3xtf32(x)
     assert np.all((x.astype(np.float64) - hi) == (x - hi).astype(np.float64))
     assert np.all(np.abs(x.astype(np.float64) - hi - lo) <= 2.0 ** -22 * np.abs(x))
+
+
+def test_sampled_wgrad_element_matches_full():
+    N, C, H, W, Co, K, S, P = 3, 4, 9, 9, 5, 3, 2, 1
+    Ho = oracle.out_dim(H, K, S, P)
+    d = gen_custom(N, C, H, W, Co, K, K, 17, Ho=Ho, Wo=Ho)
+    dw, _ = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, S, P)
+    for idx in [(0, 0, 0, 0), (4, 3, 2, 2), (2, 1, 0, 2), (1, 2, 1, 1)]:
+        assert oracle.conv_bwd_filter_at(d["x"], d["dy"], d["w"].shape, S, P, idx) == dw[idx]

@@ -1,0 +1,464 @@
+#!/usr/bin/env python
+"""bench.py — conv-layer training throughput of the B200-native GLP4NN hot path.
+
+Metric (BASELINE.json): conv fwd+bwd images/sec at 1/2/4/8 B200, with the dominant kernel's
+fraction of the tensor-pipe roofline.  A step = one pass of the whole hot path over one batch:
+for every conv layer of the workload, forward (pack x, pack W, tcgen05 implicit GEMM + bias),
+then backward in reverse layer order (pack dy + db partials, backward-data GEMM — skipped for the
+data-fed first layer, R9 — filter-gradient GEMM, fixed-order split reduction), then
+(N > 1) one NCCL all_reduce(SUM) of the flat dW||db buffer.
+
+Default workload: CaffeNet conv1-5 at batch 256 per GPU (BASELINE.json configs[3]; Table 5
+P345-349), bf16 operands with fp32 accumulation.  The other configs are parity-test cases
+(``--workload 1..5`` runs them too).
+
+Launch: ``python bench.py --gpus N --steps K --warmup W``; for N > 1 under torchrun (one rank
+per GPU, NCCL).  ``--impl reference`` times the fp64 CPU oracle (the reference arm of this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from glp_workloads import CONFIG_NAMES, config, gen_layer  # noqa: E402
+
+METRIC = "conv fwd+bwd images/sec"
+UNIT = "images/s"
+NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25   # B200_PROFILING.md nominal dense ratio
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=100)
+    p.add_argument("--warmup", type=int, default=10)
+    p.add_argument("--impl", choices=["glp", "reference"], default="glp")
+    p.add_argument("--workload", type=int, default=4, help="BASELINE.json config index 1..5")
+    p.add_argument("--math", choices=["bf16", "tf32"], default="bf16")
+    p.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--e2e-steps", type=int, default=5)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------------- helpers ------------
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "bf16_tflops": float(d["bf16_tflops"]),
+                "bf16_tflops_sustained": float(d.get("bf16_tflops_sustained", d["bf16_tflops"])),
+                "source": "measured (MEASURED_PEAKS.json)"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+                "source": "fallback (B200_PROFILING.md)"}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.proc = None
+        self.f = None
+
+    def start(self):
+        try:
+            self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.flush()
+        self.f.seek(0)
+        rows = [l.strip().split(",") for l in self.f.read().splitlines() if l.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx = max(mx, float(r[1]))
+            except (ValueError, IndexError):
+                continue
+            for n, v in zip(names, r[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------- GLP arm ------------
+
+class LayerState:
+    def __init__(self, layer, n_local, n_global, shard, math, dev, flat, off):
+        import torch
+        import paper_conf_icpp_futhys18_b200 as glp
+        self.layer = layer
+        self.n = n_local
+        self.conv = glp.ConvLayer(n_local, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.S,
+                                  layer.P, math=math, device=dev.index)
+        if shard is None:
+            d = gen_layer(layer, n_global=n_global, batch=n_local)
+        else:
+            r, g = shard
+            full = gen_layer(layer, n_global=n_global)
+            d = {k: v for k, v in full.items()}
+            d["x"] = full["x"][r * n_local:(r + 1) * n_local].copy()
+            d["dy"] = full["dy"][r * n_local:(r + 1) * n_local].copy()
+        self.host = {k: torch.from_numpy(v) for k, v in d.items()}
+        self.t = {k: v.to(dev) for k, v in self.host.items()}
+        self.y = torch.empty(self.conv.y_shape, device=dev)
+        self.dx = None if layer.data_fed else torch.empty(self.conv.x_shape, device=dev)
+        wn = layer.Co * layer.C * layer.K * layer.K
+        self.dw = flat[off:off + wn].view(self.conv.w_shape)
+        self.db = flat[off + wn:off + wn + layer.Co]
+        self.nparams = wn + layer.Co
+        self.flops = float(self.layer.with_batch(n_local).flops_per_pass())
+
+    def launches(self):
+        return 9 if self.dx is not None else 7
+
+
+def run_glp(args, ws, rank, local):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_futhys18_b200 as glp
+
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    layers = config(args.workload)
+    G = ws
+    if args.scaling == "strong":
+        n_local = [l.N // G for l in layers]
+        n_global = [l.N for l in layers]
+    else:
+        n_local = [l.N for l in layers]
+        n_global = [l.N * G for l in layers]
+    nparams = sum(l.Co * l.C * l.K * l.K + l.Co for l in layers)
+    flat = torch.zeros(nparams, device=dev)
+    states, off = [], 0
+    for l, nl, ng in zip(layers, n_local, n_global):
+        shard = (rank, G) if args.scaling == "strong" and G > 1 else None
+        st = LayerState(l, nl, ng, shard, args.math, dev, flat, off)
+        off += st.nparams
+        states.append(st)
+    stream = torch.cuda.current_stream()
+
+    def step(ev=None):
+        # forward, layer order
+        for i, s in enumerate(states):
+            c = s.conv
+            c.stage_pack(glp.GLP_PACK_X, s.t["x"])
+            c.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"])
+            if ev is not None:
+                ev[i][0].record(stream)
+            c.stage_fwd(s.t["b"], s.y)
+            if ev is not None:
+                ev[i][1].record(stream)
+        # backward, reverse layer order
+        for i in reversed(range(len(states))):
+            s = states[i]
+            c = s.conv
+            c.stage_pack(glp.GLP_PACK_DY_DB, s.t["dy"])
+            if s.dx is not None:
+                c.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"])
+                if ev is not None:
+                    ev[i][2].record(stream)
+                c.stage_bwd_data(s.dx)
+                if ev is not None:
+                    ev[i][3].record(stream)
+            if ev is not None:
+                ev[i][4].record(stream)
+            c.stage_bwd_filter()
+            if ev is not None:
+                ev[i][5].record(stream)
+            c.stage_reduce(s.dw, s.db)
+        if G > 1:
+            dist.all_reduce(flat)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if G > 1:
+        dist.barrier()
+    evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(6)] for _ in states]
+           for _ in range(args.steps)]
+    clocks = ClockSampler(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    if G > 1:
+        dist.barrier()
+    t0.record(stream)
+    for k in range(args.steps):
+        step(evs[k])
+    t1.record(stream)
+    torch.cuda.synchronize()
+    if G > 1:
+        dist.barrier()
+    clk = clocks.stop() if clocks else None
+    ms = t0.elapsed_time(t1)
+    if G > 1:
+        tt = torch.tensor([ms], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    ms_per_step = ms / args.steps
+    images_per_step = n_local[0] * G
+    value = images_per_step / (ms_per_step / 1e3)
+
+    # per-kernel live timings (CUDA events on the launching stream, inside the timed region)
+    kern = []
+    for i, s in enumerate(states):
+        for name, a, b in (("fwd", 0, 1), ("bwd_data", 2, 3), ("bwd_filter", 4, 5)):
+            if name == "bwd_data" and s.dx is None:
+                continue
+            us = [evs[k][i][a].elapsed_time(evs[k][i][b]) * 1e3 for k in range(args.steps)]
+            avg = sum(us) / len(us)
+            kern.append({"layer": s.layer.name, "pass": name, "avg_us": round(avg, 2),
+                         "total_us": sum(us), "tflops": round(s.flops / (avg * 1e-6) / 1e12, 1)})
+    peaks = load_peaks()
+    dom = max(kern, key=lambda r: r["total_us"])
+    peak_tf = peaks["bf16_tflops_sustained"] * (1.0 if args.math == "bf16" else NOMINAL_TF32_OVER_BF16)
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get(f"{args.workload}/{dom['layer']}/{dom['pass']}/{args.math}")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "tensor", "achieved": dom["tflops"], "peak": round(peak_tf, 1),
+                "unit": "TFLOP/s", "frac": round(dom["tflops"] / peak_tf, 4), "traffic": traffic,
+                "kernel": f"igemm_kernel {dom['layer']} {dom['pass']}",
+                "peak_source": peaks["source"] + (" bf16 sustained" if args.math == "bf16"
+                                                  else " bf16 sustained x 1.1/2.25 (tf32)"),
+                "share_of_step": round(dom["total_us"] / 1e3 / ms, 4)}
+    step_flops = sum(s.flops * (3 if s.dx is not None else 2) for s in states)
+
+    # end-to-end: pinned host buffers -> device every step, dW||db back every step
+    e2e = None
+    if not args.no_e2e:
+        host_pinned = [{k: v.pin_memory() for k, v in s.host.items()} for s in states]
+        out_host = torch.empty(nparams, pin_memory=True)
+        h2d = sum(v.numel() * 4 for hp in host_pinned for v in hp.values())
+        d2h = nparams * 4
+        ke = max(1, args.e2e_steps)
+        step()
+        torch.cuda.synchronize()
+        if G > 1:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(ke):
+            for s, hp in zip(states, host_pinned):
+                for k2, v in hp.items():
+                    s.t[k2].copy_(v, non_blocking=True)
+            step()
+            out_host.copy_(flat, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        if G > 1:
+            tt = torch.tensor([ems], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ems = float(tt.item())
+        e2e = {"value": round(images_per_step / (ems / ke / 1e3), 1), "unit": UNIT,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": round(ems / ke, 3), "steps": ke}
+
+    cpu = None
+    if rank == 0 and G == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(layers, budget_s=12.0)
+
+    if G > 1:
+        dist.barrier()
+    if rank != 0:
+        if G > 1:
+            dist.destroy_process_group()
+        return
+    info0 = [s.conv.info for s in states]
+    line = {
+        "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": G,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
+        "dtype": args.math, "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
+        "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
+                   "global_batch": images_per_step, "per_gpu_batch": n_local[0],
+                   "layers": [s.layer.name for s in states], "math": args.math,
+                   "parallelism": f"dp{G}", "l2": "inputs larger than L2 (step working set "
+                   f"{sum(v.numel() * 4 for s in states for v in s.t.values()) / 1e9:.2f} GB)",
+                   "step_gflop": round(step_flops / 1e9, 1),
+                   "samples_in_flight": [i.samples_in_flight for i in info0],
+                   "wgrad_splits": [i.splits_wgrad for i in info0]},
+        "tflops_step": round(step_flops / (ms_per_step * 1e-3) / 1e12, 1),
+        "roofline": roofline,
+        "kernels": [{k: r[k] for k in ("layer", "pass", "avg_us", "tflops")} for r in kern],
+        "cpu_baseline": cpu,
+        "clocks": clk,
+        "e2e": e2e,
+        "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
+    }
+    print(json.dumps(line), flush=True)
+    if G > 1:
+        dist.destroy_process_group()
+
+
+# ------------------------------------------------------------------------- CPU oracle --------
+
+def _oracle_items(layers, n):
+    items = []
+    for l in layers:
+        lb = l.with_batch(n)
+        f = lb.flops_per_pass()
+        items.append((l, "fwd", f))
+        items.append((l, "bwd_filter", f))
+        if not l.data_fed:
+            items.append((l, "bwd_data", f))
+    return items
+
+
+def _oracle_run(l, kind, d):
+    import oracle
+    if kind == "fwd":
+        oracle.conv_fwd(d["x"], d["w"], d["b"], l.S, l.P)
+    elif kind == "bwd_filter":
+        oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, l.S, l.P)
+    else:
+        oracle.conv_bwd_data(d["dy"], d["w"], d["x"].shape, l.S, l.P)
+
+
+def cpu_baseline(layers, budget_s=12.0, n_sample=None):
+    """The fp64 oracle (as it stands) on a bounded sample: batches of `n` images through every
+    layer-pass of the step until the time budget is used; images/s = images done / time."""
+    import oracle
+    cores = oracle.max_threads()
+    n = n_sample or max(1, min(layers[0].N, cores))
+    data = {l.name: gen_layer(l, batch=n) for l in layers}
+    items = _oracle_items(layers, n)
+    done_flops, t_used = 0.0, 0.0
+    per_image = sum(f for _, _, f in items) / n
+    passes = 0
+    while True:
+        for l, kind, f in items:
+            t0 = time.perf_counter()
+            _oracle_run(l, kind, data[l.name])
+            t_used += time.perf_counter() - t0
+            done_flops += f
+            if t_used >= budget_s:
+                break
+        passes += 1
+        if t_used >= budget_s:
+            break
+    images = done_flops / per_image
+    return {"value": round(images / t_used, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{images:.3f} images (batches of {n}, every layer-pass of the step, "
+                      f"{t_used:.1f} s, fp64 direct loops, OpenMP)"}
+
+
+def run_reference(args, ws, rank):
+    if rank != 0:
+        return
+    import oracle
+    layers = config(args.workload)
+    cores = oracle.max_threads()
+    total = args.steps + args.warmup
+    budget_total = 150.0
+    per_step = min(5.0, max(0.5, budget_total / max(1, total)))
+    n = max(1, min(layers[0].N, cores))
+    data = {l.name: gen_layer(l, batch=n) for l in layers}
+    items = _oracle_items(layers, n)
+    per_image = sum(f for _, _, f in items) / n
+    it = 0
+    times, flops = [], []
+
+    def one_step():
+        nonlocal it
+        t_used, f_done = 0.0, 0.0
+        while t_used < per_step:
+            l, kind, f = items[it % len(items)]
+            it += 1
+            t0 = time.perf_counter()
+            _oracle_run(l, kind, data[l.name])
+            t_used += time.perf_counter() - t0
+            f_done += f
+        return t_used, f_done
+
+    for _ in range(args.warmup):
+        one_step()
+    for _ in range(args.steps):
+        t, f = one_step()
+        times.append(t)
+        flops.append(f)
+    images = sum(flops) / per_image
+    value = images / sum(times)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": UNIT,
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(sum(times) / len(times) * 1e3, 2), "higher_is_better": True,
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
+        "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
+                   "global_batch": layers[0].N, "layers": [l.name for l in layers]},
+        "cpu_baseline": {"value": round(value, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"each step = {per_step:.1f} s of oracle layer-passes on a "
+                                   f"{n}-image batch; {images:.3f} images total"},
+        "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse_args()
+    ws, rank, local = dist_env()
+    if ws != args.gpus and ws > 1:
+        print(f"warning: WORLD_SIZE={ws} but --gpus {args.gpus}", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+        return
+    run_glp(args, ws, rank, local)
+
+
+if __name__ == "__main__":
+    main()

@@ -132,6 +132,36 @@ glp_status_t glp_conv_bwd(glp_plan_t plan, const float *x, const float *dy, cons
                           float *dx, float *dw, float *db, int accumulate, void *ws,
                           size_t ws_bytes, glp_stream_t stream);
 
+/* ---- staged execution (tensor-core plans only) ------------------------------------------- *
+ * The compute calls above are compositions of these stages; a training step that keeps the
+ * layer's workspace between forward and backward packs x once (forward) and reuses it in the
+ * filter gradient, and packs dy once for both backward GEMMs.  Every stage works on the plan's
+ * single workspace layout: ws must hold info.ws_bwd bytes (1024-byte aligned).  Results are
+ * bitwise identical to the composed calls.  Stages are asynchronous on `stream`; a stage reads
+ * what earlier stages on the same stream wrote.  FP32 plans return GLP_ERR_NOT_SUPPORTED. */
+typedef enum {
+  GLP_PACK_X = 0,          /* x  NCHW fp32 -> packed NHWC operand (rounded to the math mode)  */
+  GLP_PACK_DY = 1,         /* dy NCHW fp32 -> packed NHWC operand                              */
+  GLP_PACK_DY_DB = 2,      /* as GLP_PACK_DY, plus the fixed-order partial sums of db          */
+  GLP_PACK_W_FWD = 3,      /* W -> forward B operand [C_o][(kh,kw,ci)]                         */
+  GLP_PACK_W_BWD_DATA = 4  /* W -> backward-data B operand [C_i][(kh,kw,co)]                   */
+} glp_pack_t;
+glp_status_t glp_stage_pack(glp_plan_t plan, glp_pack_t what, const float *src, void *ws,
+                            size_t ws_bytes, glp_stream_t stream);
+/* tcgen05 implicit GEMM of Alg. 1 with the fused bias epilogue: needs GLP_PACK_X, GLP_PACK_W_FWD. */
+glp_status_t glp_stage_fwd(glp_plan_t plan, const float *b, float *y, void *ws, size_t ws_bytes,
+                           glp_stream_t stream);
+/* tcgen05 implicit GEMM of Alg. 2 (col2im folded): needs GLP_PACK_DY(_DB), GLP_PACK_W_BWD_DATA. */
+glp_status_t glp_stage_bwd_data(glp_plan_t plan, float *dx, void *ws, size_t ws_bytes,
+                                glp_stream_t stream);
+/* tcgen05 implicit GEMM of the filter gradient into the split partials: needs GLP_PACK_X and
+ * GLP_PACK_DY(_DB). */
+glp_status_t glp_stage_bwd_filter(glp_plan_t plan, void *ws, size_t ws_bytes, glp_stream_t stream);
+/* Fixed-order reduction of the split partials into dW (Caffe layout) and of the db partials
+ * (requires GLP_PACK_DY_DB when db != NULL). */
+glp_status_t glp_stage_reduce(glp_plan_t plan, float *dw, float *db, int accumulate, void *ws,
+                              size_t ws_bytes, glp_stream_t stream);
+
 /* ---- analyzer (host only, no device needed) ----------------------------------------------- */
 /* The north_star's sm_100a limits: 148 SMs, 64K regs, 228 KB smem, 2048 threads, 32 blocks,
  * + 512 TMEM columns, 1 KB smem reserved per CTA, C = 128. */

@@ -54,7 +54,10 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_conv_bwd_filter", "glp_conv_bwd", "glp_device_limits_b200",
            "glp_analyze_ctas_per_sm", "glp_analyze_samples_in_flight", "glp_analyze_eq7",
            "glp_plan_kernel_attr", "glp_status_string", "glp_last_error_string", "glp_version",
-           "glp_debug_im2col"]
+           "glp_debug_im2col", "glp_stage_pack", "glp_stage_fwd", "glp_stage_bwd_data",
+           "glp_stage_bwd_filter", "glp_stage_reduce"]
+
+GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA = 0, 1, 2, 3, 4
 
 _lib = None
 
@@ -96,6 +99,11 @@ def lib():
         L.glp_analyze_eq7.argtypes = [P(DeviceLimits), P(KernelAttr), _c_int, _dbl, _dbl, P(_c_int)]
         L.glp_plan_kernel_attr.argtypes = [_vp, _c_int, P(KernelAttr), P(_c_int), P(_c_int)]
         L.glp_debug_im2col.argtypes = [_vp, _vp, _c_int, _vp, _vp, _c_size, _vp]
+        L.glp_stage_pack.argtypes = [_vp, _c_int, _vp, _vp, _c_size, _vp]
+        L.glp_stage_fwd.argtypes = [_vp, _vp, _vp, _vp, _c_size, _vp]
+        L.glp_stage_bwd_data.argtypes = [_vp, _vp, _vp, _c_size, _vp]
+        L.glp_stage_bwd_filter.argtypes = [_vp, _vp, _c_size, _vp]
+        L.glp_stage_reduce.argtypes = [_vp, _vp, _vp, _c_int, _vp, _c_size, _vp]
         _lib = L
     return _lib
 
@@ -242,6 +250,28 @@ class ConvLayer:
                                _ptr(db), int(bool(accumulate)), ctypes.c_void_p(self.ws_ptr),
                                self.ws_bytes, _stream(stream)), "glp_conv_bwd")
         return dx, dw, db
+
+    # staged execution (include/glp.h "staged execution"): one C call per kernel group
+    def stage_pack(self, what, src, stream=None):
+        _ck(lib().glp_stage_pack(self._plan, int(what), _ptr(src), ctypes.c_void_p(self.ws_ptr),
+                                 self.ws_bytes, _stream(stream)), "glp_stage_pack")
+
+    def stage_fwd(self, b, y, stream=None):
+        _ck(lib().glp_stage_fwd(self._plan, _ptr(b), _ptr(y), ctypes.c_void_p(self.ws_ptr),
+                                self.ws_bytes, _stream(stream)), "glp_stage_fwd")
+
+    def stage_bwd_data(self, dx, stream=None):
+        _ck(lib().glp_stage_bwd_data(self._plan, _ptr(dx), ctypes.c_void_p(self.ws_ptr),
+                                     self.ws_bytes, _stream(stream)), "glp_stage_bwd_data")
+
+    def stage_bwd_filter(self, stream=None):
+        _ck(lib().glp_stage_bwd_filter(self._plan, ctypes.c_void_p(self.ws_ptr), self.ws_bytes,
+                                       _stream(stream)), "glp_stage_bwd_filter")
+
+    def stage_reduce(self, dw, db=None, accumulate=False, stream=None):
+        _ck(lib().glp_stage_reduce(self._plan, _ptr(dw), _ptr(db), int(bool(accumulate)),
+                                   ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_stage_reduce")
 
     def debug_im2col(self, x, n, col, stream=None):
         _ck(lib().glp_debug_im2col(self._plan, _ptr(x), int(n), _ptr(col),

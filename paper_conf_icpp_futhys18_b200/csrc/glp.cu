@@ -223,7 +223,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const int stage_bytes = 16384 + pp.bn_smem * 128;
   const int budget = 232448 - 1024 - 512;
   pp.stages = std::min(8, budget / stage_bytes);
-  if (pp.stages < TileCfg<2>::LAG + 1) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
+  if (pp.stages < 2) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
   pp.acc_cols = (int)rup(pp.bn, 32);
   int tc = 32;
   while (tc < 2 * pp.acc_cols) tc *= 2;
@@ -232,7 +232,8 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.tiles = pp.m_tiles * pp.n_tiles * pp.splits;
 
   void *fn = igemm_ptr(mode, elem);
-  GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, pp.smem));
+  // The attribute is per function (not per plan): always allow the largest tile of any plan.
+  GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
   GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
   pp.regs = fa.numRegs;
@@ -327,7 +328,15 @@ glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmPa
 
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
                              int Cp, float *db_part, cudaStream_t st) {
-  dim3 grid((unsigned)cdiv(HW, 32), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
+  if (db_part == nullptr && Cp * P.elem <= 32) {
+    const size_t n = (size_t)P.d.N * HW;
+    const int g = (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 32);
+    if (P.elem == 2) pack_nchw_to_nhwc_small<2><<<g, 256, 0, st>>>(src, dst, P.d.N, C, HW, Cp);
+    else pack_nchw_to_nhwc_small<4><<<g, 256, 0, st>>>(src, dst, P.d.N, C, HW, Cp);
+    GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
+    return GLP_OK;
+  }
+  dim3 grid((unsigned)cdiv(HW, PACK_PT), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
   if (P.elem == 2) pack_nchw_to_nhwc<2><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
   else pack_nchw_to_nhwc<4><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
@@ -336,16 +345,30 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
 
 int ew_grid(size_t n) { return (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 16); }
 
-glp_status_t run_fwd_tc(glp_plan_s &P, const float *x, const float *w, const float *b, float *y,
-                        uint8_t *ws, cudaStream_t st) {
+glp_status_t run_pack_w_fwd(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
-  void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
-  glp_status_t s = launch_pack_act(P, x, xpk, d.C, d.H * d.W, P.Cp, nullptr, st);
-  if (s) return s;
+  void *wpk = ws + P.off_wpk;
   const size_t wn = (size_t)d.Co * P.fwd.Kpad;
   if (P.elem == 2) pack_w_fwd<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
   else pack_w_fwd<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
   GLP_LAUNCH_CHECK("pack_w_fwd");
+  return GLP_OK;
+}
+
+glp_status_t run_pack_w_dgrad(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  void *wtpk = ws + P.off_wpk;
+  const size_t wn = (size_t)d.C * P.dgrad.Kpad;
+  if (P.elem == 2) pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
+  else pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
+  GLP_LAUNCH_CHECK("pack_w_dgrad");
+  return GLP_OK;
+}
+
+glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
+  glp_status_t s;
   CUtensorMap map;
   s = encode_2d(&map, P.elem, wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co, (uint64_t)P.fwd.Kpad * P.elem,
                 128 / P.elem, (uint32_t)P.fwd.bn);
@@ -358,14 +381,10 @@ glp_status_t run_fwd_tc(glp_plan_s &P, const float *x, const float *w, const flo
   return launch_igemm<MODE_FWD>(P, P.fwd, p, map, st);
 }
 
-glp_status_t run_dgrad_tc(glp_plan_s &P, const void *dypk, const float *w, float *dx, uint8_t *ws,
-                          cudaStream_t st) {
+glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   void *wtpk = ws + P.off_wpk;
-  const size_t wn = (size_t)d.C * P.dgrad.Kpad;
-  if (P.elem == 2) pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
-  else pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
-  GLP_LAUNCH_CHECK("pack_w_dgrad");
+  const void *dypk = ws + P.off_dypk;
   CUtensorMap map;
   glp_status_t s = encode_2d(&map, P.elem, wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
                              (uint64_t)P.dgrad.Kpad * P.elem, 128 / P.elem, (uint32_t)P.dgrad.bn);
@@ -377,9 +396,9 @@ glp_status_t run_dgrad_tc(glp_plan_s &P, const void *dypk, const float *w, float
   return launch_igemm<MODE_DGRAD>(P, P.dgrad, p, map, st);
 }
 
-glp_status_t run_wgrad_tc(glp_plan_s &P, const void *xpk, const void *dypk, float *dw, float *db,
-                          int accumulate, uint8_t *ws, cudaStream_t st) {
+glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
+  const void *xpk = ws + P.off_xpk, *dypk = ws + P.off_dypk;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
   CUtensorMap map;
   const int BK = 128 / P.elem;
@@ -390,14 +409,20 @@ glp_status_t run_wgrad_tc(glp_plan_s &P, const void *xpk, const void *dypk, floa
   if (s) return s;
   IgemmParams p = make_params(P, P.wgrad, MODE_WGRAD, xpk);
   p.out = part;
-  s = launch_igemm<MODE_WGRAD>(P, P.wgrad, p, map, st);
-  if (s) return s;
+  return launch_igemm<MODE_WGRAD>(P, P.wgrad, p, map, st);
+}
+
+glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulate, uint8_t *ws,
+                              cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  float *part = reinterpret_cast<float *>(ws + P.off_part);
   const size_t wsz = (size_t)d.Co * d.C * P.taps;
-  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, P.Cp, p.part_ld,
-                                             p.part_mpad, P.wgrad.splits, accumulate);
+  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, P.Cp,
+                                             P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_tiles * 128,
+                                             P.wgrad.splits, accumulate);
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
-    reduce_db<<<(unsigned)cdiv(d.Co, 128), 128, 0, st>>>(
+    reduce_db<<<(unsigned)cdiv(d.Co, 32), 256, 0, st>>>(
         reinterpret_cast<float *>(ws + P.off_dbpart), db, d.Co, P.db_rows, accumulate);
     GLP_LAUNCH_CHECK("reduce_db");
   }
@@ -421,7 +446,7 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
   if (db) {
     simt_db_partial<<<ew_grid((size_t)P.simt_splits * d.Co), 256, 0, st>>>(geom(d), dy, dbp, P.simt_splits, P.simt_chunk);
     GLP_LAUNCH_CHECK("simt_db_partial");
-    reduce_db<<<(unsigned)cdiv(d.Co, 128), 128, 0, st>>>(dbp, db, d.Co, P.simt_splits, accumulate);
+    reduce_db<<<(unsigned)cdiv(d.Co, 32), 256, 0, st>>>(dbp, db, d.Co, P.simt_splits, accumulate);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
@@ -588,7 +613,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
     P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
     P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_tiles * 128 * P->wgrad.n_tiles * P->wgrad.bn * 4);
-    P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, 32);
+    P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, PACK_PT);
     P->sz_dbpart = align1k((size_t)P->db_rows * c.Co * 4);
     // one layout serves every call: [xpk | dypk | wpk/wtpk | part | dbpart]
     P->off_xpk = 0;
@@ -689,7 +714,10 @@ glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const fl
     return GLP_OK;
   }
   if ((s = get_encode())) return s;
-  return run_fwd_tc(*P, x, w, b, y, static_cast<uint8_t *>(ws), st);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  if ((s = launch_pack_act(*P, x, wsb + P->off_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = run_pack_w_fwd(*P, w, wsb, st))) return s;
+  return run_fwd_gemm(*P, b, y, wsb, st);
 }
 
 glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, float *dx, void *ws,
@@ -709,7 +737,8 @@ glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, fl
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   void *dypk = wsb + P->off_dypk;
   if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st))) return s;
-  return run_dgrad_tc(*P, dypk, w, dx, wsb, st);
+  if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
+  return run_dgrad_gemm(*P, dx, wsb, st);
 }
 
 glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, float *dw, float *db,
@@ -728,7 +757,8 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
                            db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
     return s;
-  return run_wgrad_tc(*P, xpk, dypk, dw, db, accumulate ? 1 : 0, wsb, st);
+  if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
+  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
 }
 
 glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const float *w, float *dx,
@@ -755,9 +785,73 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
   if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
                            db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
     return s;
-  if (dx && (s = run_dgrad_tc(*P, dypk, w, dx, wsb, st))) return s;
+  if (dx) {
+    if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
+    if ((s = run_dgrad_gemm(*P, dx, wsb, st))) return s;
+  }
   if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
-  return run_wgrad_tc(*P, xpk, dypk, dw, db, accumulate ? 1 : 0, wsb, st);
+  if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
+  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
+}
+
+static glp_status_t stage_check(glp_plan_t P, void *ws, size_t ws_bytes) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "staged API needs a tensor-core plan");
+  glp_status_t s = check_ws(P, ws, ws_bytes, P->ws_bwd);
+  if (s) return s;
+  return get_encode();
+}
+
+glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, void *ws,
+                            size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if ((s = validate_ptrs({src}))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  switch (what) {
+    case GLP_PACK_X:
+      return launch_pack_act(*P, src, wsb + P->off_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st);
+    case GLP_PACK_DY:
+      return launch_pack_act(*P, src, wsb + P->off_dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st);
+    case GLP_PACK_DY_DB:
+      return launch_pack_act(*P, src, wsb + P->off_dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
+                             reinterpret_cast<float *>(wsb + P->off_dbpart), st);
+    case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, src, wsb, st);
+    case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, src, wsb, st);
+  }
+  return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
+}
+
+glp_status_t glp_stage_fwd(glp_plan_t P, const float *b, float *y, void *ws, size_t ws_bytes,
+                           glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if ((s = validate_ptrs({y}))) return s;
+  return run_fwd_gemm(*P, b, y, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_bytes,
+                                glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if ((s = validate_ptrs({dx}))) return s;
+  return run_dgrad_gemm(*P, dx, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_stage_bwd_filter(glp_plan_t P, void *ws, size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  return run_wgrad_gemm(*P, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_stage_reduce(glp_plan_t P, float *dw, float *db, int accumulate, void *ws,
+                              size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if ((s = validate_ptrs({dw}))) return s;
+  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, static_cast<uint8_t *>(ws),
+                          static_cast<cudaStream_t>(stream));
 }
 
 glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, void *ws,

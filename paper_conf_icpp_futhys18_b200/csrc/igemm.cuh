@@ -30,7 +30,6 @@ struct TileCfg {
   static constexpr int UMMA_K = 32 / ELEM;   // K of one tcgen05.mma (bf16 16, tf32 8)
   static constexpr int A_BYTES = BM * 128;   // 16 KB
   static constexpr int LBO_MN = (BK / 8) * 1024;  // MN-major: stride between 128-byte MN atoms
-  static constexpr int LAG = 3;              // cp.async groups kept in flight per producer
   static constexpr int THREADS = 288;
 };
 
@@ -81,7 +80,7 @@ __global__ void __launch_bounds__(288, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S_; ++s) {
-      mbar_init(full(s), 129);   // 128 producer arrivals + 1 expect_tx arrival (TMA bytes)
+      mbar_init(full(s), 129);   // 128 cp.async arrivals (noinc) + 1 expect_tx arrival (TMA)
       mbar_init(empty(s), 1);    // tcgen05.commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -117,19 +116,17 @@ __global__ void __launch_bounds__(288, 1)
       }
       const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
       if (MODE != MODE_WGRAD) {
-        // K-major A: thread owns chunk j of rows rg + 16 i.
+        // K-major A: thread owns 16-byte chunk j of rows rg + 16 i (i = 0..7).
         const int j = pt & 7, rg = pt >> 3;
-        uint32_t nimg[8];
+        uint32_t pbase[8];
         int ohS[8], owS[8];
-        bool mv[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
           const int m = m0 + rg + 16 * i;
-          mv[i] = m < p.M;
           uint32_t n, rem, oh, ow;
-          g.div_hw.divmod((uint32_t)(mv[i] ? m : 0), n, rem);
+          g.div_hw.divmod((uint32_t)(m < p.M ? m : 0), n, rem);
           g.div_w.divmod(rem, oh, ow);
-          nimg[i] = n;
+          pbase[i] = n * (uint32_t)(g.src_h * g.src_w);
           if (MODE == MODE_FWD) {
             ohS[i] = (int)oh * g.stride - g.pad;
             owS[i] = (int)ow * g.stride_w - g.pad_w;
@@ -137,7 +134,15 @@ __global__ void __launch_bounds__(288, 1)
             ohS[i] = (int)oh + g.pad;
             owS[i] = (int)ow + g.pad_w;
           }
+          if (m >= p.M) ohS[i] = -(1 << 28);  // row past M: every tap fails the bounds check
         }
+        const uint32_t dst0 = (uint32_t)(rg >> 3) * 1024u + (uint32_t)(rg & 7) * 128u +
+                              (uint32_t)((j ^ (rg & 7)) << 4);
+        // K index of this thread's chunk, advanced incrementally by BK per k-block.
+        uint32_t t, c, kh, kw;
+        g.div_cp.divmod((uint32_t)(kb0 * C::BK + j * C::CH), t, c);
+        g.div_kw.divmod(t, kh, kw);
+        const uint8_t *srcb = static_cast<const uint8_t *>(g.src);
         for (int kb = kb0; kb < kb1; ++kb, ++gk) {
           const int s = (int)(gk % (uint32_t)S_);
           const uint32_t ph = (gk / (uint32_t)S_) & 1u;
@@ -147,49 +152,40 @@ __global__ void __launch_bounds__(288, 1)
             mbar_arrive_expect_tx(full(s), (uint32_t)p.bn_smem * 128u);
             tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
           }
-          const uint32_t k0 = (uint32_t)(kb * C::BK + j * C::CH);
-          if (MODE == MODE_FWD) {
+          const bool kv = (int)t < g.taps;
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const int r = rg + 16 * i;
-              const uint8_t *src = static_cast<const uint8_t *>(g.src);
-              const bool ok = mv[i] && fwd_gather<ELEM>(g, nimg[i], ohS[i], owS[i], k0, src);
-              const uint32_t dst = sA + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
-                                   (uint32_t)((j ^ (r & 7)) << 4);
-              cp_async16(dst, src, ok);
-            }
-          } else {
-            uint32_t t, c;
-            g.div_cp.divmod(k0, t, c);
-            const bool kv = (int)t < g.taps;
-            uint32_t kh, kw;
-            g.div_kw.divmod(kv ? t : 0u, kh, kw);
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const int r = rg + 16 * i;
+          for (int i = 0; i < 8; ++i) {
+            int ih, iw;
+            bool ok;
+            if (MODE == MODE_FWD) {
+              ih = ohS[i] + (int)kh;
+              iw = owS[i] + (int)kw;
+              ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
+            } else {
               const int ihn = ohS[i] - (int)kh, iwn = owS[i] - (int)kw;
-              bool ok = kv && mv[i] && ihn >= 0 && iwn >= 0;
-              int ih = ihn, iw = iwn;
-              if (g.stride != 1 || g.stride_w != 1) {
-                ok = ok && (ihn % g.stride == 0) && (iwn % g.stride_w == 0);
+              if (g.stride == 1 && g.stride_w == 1) {
+                ih = ihn;
+                iw = iwn;
+                ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
+              } else {
+                ok = kv && ihn >= 0 && iwn >= 0 && (ihn % g.stride == 0) && (iwn % g.stride_w == 0);
                 ih = ihn / g.stride;
                 iw = iwn / g.stride_w;
+                ok = ok && ih < g.src_h && iw < g.src_w;
               }
-              ok = ok && ih < g.src_h && iw < g.src_w;
-              const uint8_t *src = static_cast<const uint8_t *>(g.src);
-              if (ok)
-                src += ((size_t)((size_t)nimg[i] * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) *
-                            g.src_cp + c) * ELEM;
-              const uint32_t dst = sA + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
-                                   (uint32_t)((j ^ (r & 7)) << 4);
-              cp_async16(dst, src, ok);
             }
+            const uint8_t *src = srcb;
+            if (ok)
+              src += ((size_t)(pbase[i] + (uint32_t)(ih * g.src_w + iw)) * (uint32_t)g.src_cp + c) * ELEM;
+            cp_async16(sA + dst0 + (uint32_t)i * 2048u, src, ok);
           }
-          cp_async_commit();
-          if (gk >= (uint32_t)C::LAG) {
-            cp_async_wait<C::LAG>();
-            fence_proxy_async_smem();
-            mbar_arrive(full((int)((gk - C::LAG) % (uint32_t)S_)));
+          cp_async_mbar_arrive_noinc(full(s));
+          c += C::BK;
+          if (c >= (uint32_t)g.cp) {
+            const uint32_t q = g.div_cp.div(c);
+            c -= q * (uint32_t)g.cp;
+            t += q;
+            g.div_kw.divmod(t, kh, kw);
           }
         }
       } else {
@@ -240,19 +236,10 @@ __global__ void __launch_bounds__(288, 1)
                     (uint32_t)((((jj >> 1) ^ (r & 3)) << 5) | ((jj & 1) << 4));
             cp_async16(dst, src, ok);
           }
-          cp_async_commit();
-          if (gk >= (uint32_t)C::LAG) {
-            cp_async_wait<C::LAG>();
-            fence_proxy_async_smem();
-            mbar_arrive(full((int)((gk - C::LAG) % (uint32_t)S_)));
-          }
+          cp_async_mbar_arrive_noinc(full(s));
         }
       }
     }
-    cp_async_wait<0>();
-    fence_proxy_async_smem();
-    for (uint32_t q = (gk > (uint32_t)C::LAG ? gk - C::LAG : 0u); q < gk; ++q)
-      mbar_arrive(full((int)(q % (uint32_t)S_)));
   } else if (warp == 8) {
     // ===================================== MMA issuer ======================================
     if (lane == 0) {

@@ -42,36 +42,76 @@ struct PackOut<4> {
   }
 };
 
-// NCHW fp32 [N][C][HW] -> NHWC [N][HW][Cp] (rounded), zero for c >= C.  Tile 32 ch x 32 px.
-// grid (ceil(HW/32), ceil(Cp/32), N), block 256.  db_part (optional): [N][ceil(HW/32)][C].
+// NCHW fp32 [N][C][HW] -> NHWC [N][HW][Cp] (rounded), zero for c >= C.
+// Tile 32 channels x PACK_PT pixels per 256-thread block: 16 independent coalesced loads per
+// thread, conflict-free transposed smem reads, 16-byte stores.
+// grid (ceil(HW/PACK_PT), ceil(Cp/32), N).  db_part (optional): [N][ceil(HW/PACK_PT)][C], each
+// entry the sum of one channel over one pixel tile in a fixed order (lane-sequential over the 4
+// pixel quarters, then a xor-shuffle tree).
+constexpr int PACK_PT = 128;
+
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict__ src,
                                                          void *__restrict__ dst, int C, int HW,
                                                          int Cp, float *__restrict__ db_part) {
-  __shared__ float tile[32][33];
-  const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * 32;
+  __shared__ float tile[32][PACK_PT + 1];
+  const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * PACK_PT;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const float *s = src + (size_t)n * C * HW;
+  float v[4][4];
 #pragma unroll
-  for (int cc = warp; cc < 32; cc += 8) {
-    const int c = c0 + cc, px = p0 + lane;
-    float v = 0.f;
-    if (c < C && px < HW) v = __ldg(s + (size_t)c * HW + px);
-    tile[cc][lane] = v;
-    if (db_part != nullptr && c < C) {
-      float t = v;
+  for (int k = 0; k < 4; ++k) {
+    const int c = c0 + warp + 8 * k;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int px = p0 + q * 32 + lane;
+      v[k][q] = (c < C && px < HW) ? __ldg(s + (size_t)c * HW + px) : 0.f;
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int cc = warp + 8 * k;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) tile[cc][q * 32 + lane] = v[k][q];
+    if (db_part != nullptr && c0 + cc < C) {
+      float t = ((v[k][0] + v[k][1]) + (v[k][2] + v[k][3]));
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-      if (lane == 0) db_part[((size_t)n * gridDim.x + blockIdx.x) * C + c] = t;
+      if (lane == 0) db_part[((size_t)n * gridDim.x + blockIdx.x) * C + c0 + cc] = t;
     }
   }
   __syncthreads();
-  const int pp = threadIdx.x >> 3, cq = threadIdx.x & 7;
-  const int px = p0 + pp, c = c0 + 4 * cq;
-  if (px < HW && c < Cp) {
-    const size_t o = ((size_t)n * HW + px) * Cp + c;
-    PackOut<ELEM>::store4(dst, o, tile[4 * cq][pp], tile[4 * cq + 1][pp], tile[4 * cq + 2][pp],
-                          tile[4 * cq + 3][pp]);
+  const int pp = threadIdx.x >> 1, h = threadIdx.x & 1;
+  const int px = p0 + pp;
+  if (px < HW) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int cl = 16 * h + 4 * q, c = c0 + cl;
+      if (c < Cp) {
+        const size_t o = ((size_t)n * HW + px) * Cp + c;
+        PackOut<ELEM>::store4(dst, o, tile[cl][pp], tile[cl + 1][pp], tile[cl + 2][pp],
+                              tile[cl + 3][pp]);
+      }
+    }
+  }
+}
+
+// Small channel counts (Cp <= 16): one thread per pixel, loads coalesced across pixels.
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__restrict__ src,
+                                                               void *__restrict__ dst, int N, int C,
+                                                               int HW, int Cp) {
+  const size_t total = (size_t)N * HW;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
+       i += (size_t)gridDim.x * blockDim.x) {
+    const size_t n = i / HW, px = i % HW;
+    const float *s = src + n * C * HW + px;
+    for (int c = 0; c < Cp; c += 4) {
+      float a[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) a[u] = (c + u < C) ? __ldg(s + (size_t)(c + u) * HW) : 0.f;
+      PackOut<ELEM>::store4(dst, i * Cp + c, a[0], a[1], a[2], a[3]);
+    }
   }
 }
 

@@ -56,6 +56,12 @@ __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, bool v
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n)
                : "memory");
 }
+// Arrive on `bar` when every cp.async previously issued by this thread has completed; noinc:
+// the arrival counts against the barrier's expected count (no pending-count increment).
+// Same completion mechanism as CUTLASS's sm100 cp.async mainloop (cpasync_barrier_arrive).
+__device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint32_t bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() {
   asm volatile("cp.async.commit_group;" ::: "memory");
 }

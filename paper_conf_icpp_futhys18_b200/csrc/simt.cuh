@@ -179,19 +179,25 @@ __global__ void reduce_tc_dw(const float *__restrict__ part, float *__restrict__
 }
 
 // db[co] = sum over rows of part[row][co] (rows = N * pixel tiles, or SIMT splits), fixed order.
-__global__ void reduce_db(const float *__restrict__ part, float *__restrict__ db, int Co, int rows,
-                          int accumulate) {
-  const int co = blockIdx.x * blockDim.x + threadIdx.x;
-  if (co >= Co) return;
-  // sequential in blocks of 64 rows, then sequential over blocks (order fixed by rows)
-  float tot = 0.f;
-  for (int r0 = 0; r0 < rows; r0 += 64) {
-    float a = 0.f;
-    const int e = r0 + 64 < rows ? r0 + 64 : rows;
-    for (int r = r0; r < e; ++r) a += __ldg(part + (size_t)r * Co + co);
-    tot += a;
+// One block of 256 threads per 32 channels: thread (ty, lane) sums rows ty, ty+8, ... for channel
+// c0+lane (coalesced across lanes), then a fixed 8-way tree in shared memory.  The order depends
+// only on `rows` (shape), never on the grid or S.
+__global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
+                                                 float *__restrict__ db, int Co, int rows,
+                                                 int accumulate) {
+  __shared__ float red[8][33];
+  const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  const int co = blockIdx.x * 32 + lane;
+  float a = 0.f;
+  if (co < Co)
+    for (int r = ty; r < rows; r += 8) a += __ldg(part + (size_t)r * Co + co);
+  red[ty][lane] = a;
+  __syncthreads();
+  if (ty == 0 && co < Co) {
+    const float s = ((red[0][lane] + red[1][lane]) + (red[2][lane] + red[3][lane])) +
+                    ((red[4][lane] + red[5][lane]) + (red[6][lane] + red[7][lane]));
+    db[co] = accumulate ? db[co] + s : s;
   }
-  db[co] = accumulate ? db[co] + tot : tot;
 }
 
 }  // namespace glp

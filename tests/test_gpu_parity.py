@@ -194,3 +194,28 @@ def test_error_paths_on_device():
                         None, ctypes.c_void_p(y.data_ptr()), ctypes.c_void_p(layer.ws_ptr),
                         layer.ws_bytes, None)
     assert rc == 1  # misaligned
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+def test_staged_equals_composed(math):
+    """Staged calls (pack once, GEMMs, reduce) are bitwise identical to the composed calls."""
+    shape = SHAPES[6]
+    d = _data(shape, seed=14)
+    layer = _layer(shape, math)
+    ref = _run(layer, d)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    y = torch.empty(layer.y_shape, device=DEV)
+    dx = torch.empty(layer.x_shape, device=DEV)
+    dw = torch.empty(layer.w_shape, device=DEV)
+    db = torch.empty(layer.geom.Co, device=DEV)
+    layer.stage_pack(glp.GLP_PACK_X, t["x"])
+    layer.stage_pack(glp.GLP_PACK_W_FWD, t["w"])
+    layer.stage_fwd(t["b"], y)
+    layer.stage_pack(glp.GLP_PACK_DY_DB, t["dy"])
+    layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
+    layer.stage_bwd_data(dx)
+    layer.stage_bwd_filter()
+    layer.stage_reduce(dw, db)
+    torch.cuda.synchronize()
+    for k, v in (("y", y), ("dx", dx), ("dw", dw), ("db", db)):
+        np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=k)

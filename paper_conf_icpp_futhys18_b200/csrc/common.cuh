@@ -38,6 +38,10 @@ struct Gather {
   int cp;                // channel pitch of the K (or M for wgrad) index: k = tap*cp + c
   int n_pixels;          // N * pix_hw
   FastDiv div_hw, div_w, div_cp, div_kw;
+  // im2col-TMA view of the same gather (a_tma): base pixel of output pixel (o_h, o_w) is
+  // (o_h*im_sh - im_ph, o_w*im_sw - im_pw); tap offsets are added by the TMA unit.
+  int im_sh, im_sw, im_ph, im_pw;
+  int cbs;               // channel blocks (of the K-block width) per tap, fwd/dgrad
 };
 
 struct IgemmParams {
@@ -58,6 +62,7 @@ struct IgemmParams {
   int out_hw;            // H_o*W_o (fwd) / H*W (dgrad)
   int part_ld;           // wgrad partial leading dimension (n_tiles * bn)
   int part_mpad;         // wgrad partial rows per split (m_tiles * 128)
+  int a_tma;             // 1: A operand by im2col TMA (one thread); 0: cp.async gather
 };
 
 }  // namespace glp

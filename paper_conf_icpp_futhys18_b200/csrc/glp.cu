@@ -82,6 +82,7 @@ struct PassPlan {
   int bn = 0, bn_smem = 0, m_tiles = 0, n_tiles = 0, splits = 1, kb_total = 0, kb_per_split = 0;
   int stages = 0, acc_cols = 0, tmem_cols = 0, smem = 0, tiles = 0, grid = 0, ctas_per_sm = 0;
   int regs = 0, ctas_runtime = 0;
+  int a_tma = 0, krow = 128;        // A operand by im2col TMA; K-block row width (bytes)
 };
 
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -118,19 +119,76 @@ glp_status_t encode_2d(CUtensorMap *map, int elem, const void *ptr, uint64_t inn
   return GLP_OK;
 }
 
-template <int MODE, int ELEM>
-void *kernel_ptr() {
-  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM>);
+using TmapIm2colFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                  const cuuint64_t *, const cuuint64_t *, const int *, const int *,
+                                  cuuint32_t, cuuint32_t, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion,
+                                  CUtensorMapFloatOOBfill);
+TmapIm2colFn g_encode_im2col = nullptr;
+int g_driver_version = 0;
+
+glp_status_t get_encode_im2col() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g_encode_im2col) return GLP_OK;
+  void *fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &fn, cudaEnableDefault, &q);
+  if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+    return fail(GLP_ERR_CUDA, "cuTensorMapEncodeIm2col entry point unavailable");
+  cudaDriverGetVersion(&g_driver_version);
+  g_encode_im2col = reinterpret_cast<TmapIm2colFn>(fn);
+  return GLP_OK;
 }
-void *igemm_ptr(int mode, int elem) {
-  if (elem == 2) {
-    if (mode == MODE_FWD) return kernel_ptr<MODE_FWD, 2>();
-    if (mode == MODE_DGRAD) return kernel_ptr<MODE_DGRAD, 2>();
-    return kernel_ptr<MODE_WGRAD, 2>();
-  }
-  if (mode == MODE_FWD) return kernel_ptr<MODE_FWD, 4>();
-  if (mode == MODE_DGRAD) return kernel_ptr<MODE_DGRAD, 4>();
-  return kernel_ptr<MODE_WGRAD, 4>();
+
+// im2col tensor map over a packed NHWC activation [N][H][W][cpitch]: dims {cpitch, W, H, N};
+// bounding box of base pixels [lower, dim-1+upper] per spatial dim (W, H order), traversal
+// strides = conv strides; each load = `pixels` pixels x `chans` channels.
+glp_status_t encode_im2col(CUtensorMap *map, int elem, const void *ptr, int cpitch, int W, int H,
+                           int N, int lower_w, int lower_h, int upper_w, int upper_h, int chans,
+                           int pixels, int stride_w, int stride_h, CUtensorMapSwizzle swz) {
+  if (lower_w < -128 || lower_w > 127 || lower_h < -128 || lower_h > 127 || upper_w < -128 ||
+      upper_w > 127 || upper_h < -128 || upper_h > 127)
+    return fail(GLP_ERR_NOT_SUPPORTED, "im2col corner out of TMA range");
+  const uint64_t e = (uint64_t)elem;
+  cuuint64_t dims[4] = {(cuuint64_t)cpitch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[3] = {cpitch * e, (uint64_t)W * cpitch * e, (uint64_t)H * W * cpitch * e};
+  int lower[2] = {lower_w, lower_h}, upper[2] = {upper_w, upper_h};
+  cuuint32_t es[4] = {1, (cuuint32_t)stride_w, (cuuint32_t)stride_h, 1};
+  CUresult r = g_encode_im2col(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                               4, const_cast<void *>(ptr), dims, strides, lower, upper,
+                               (cuuint32_t)chans, (cuuint32_t)pixels, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    return fail(GLP_ERR_CUDA, "cuTensorMapEncodeIm2col failed (" + std::to_string((int)r) + ")");
+  // Same driver workaround CUTLASS applies to im2col descriptors of small tensors (< 128 KiB)
+  // on drivers <= 13.1 (cute/atom/copy_traits_sm90_im2col.hpp).
+  if (g_driver_version <= 13010 && (uint64_t)N * H * W * cpitch * e < 131072)
+    reinterpret_cast<uint64_t *>(map)[1] &= ~(1ull << 21);
+  return GLP_OK;
+}
+
+template <int MODE, int ELEM, int KROW>
+void *kernel_ptr() {
+  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM, KROW>);
+}
+template <int MODE>
+void *igemm_ptr_m(int elem, int krow) {
+  if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128>() : kernel_ptr<MODE, 2, 64>();
+  return kernel_ptr<MODE, 4, 128>();
+}
+void *igemm_ptr(int mode, int elem, int krow) {
+  if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD>(elem, krow);
+  if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD>(elem, krow);
+  return igemm_ptr_m<MODE_WGRAD>(elem, krow);
+}
+
+CUtensorMapSwizzle swz_kmajor(int krow) {
+  return krow == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
+}
+CUtensorMapSwizzle swz_mnmajor(int elem, int krow) {
+  if (elem == 4) return CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
+  return krow == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
 }
 
 int choose_bn(int n) {
@@ -169,6 +227,11 @@ struct glp_plan_s {
   glp_conv_desc_s d;
   int device = 0, math = 0, elem = 4, sm_count = 148, s_override = 0;
   int Cp = 0, Cop = 0, taps = 0;
+  // Geometry of the x operand as the forward and filter-gradient passes see it: the layer itself,
+  // or its space-to-depth form (s2d = stride S > 1: stride 1, ceil(K/S) taps, S*S*C channels).
+  int s2d = 0;
+  glp_conv_desc_s dxg;
+  int Cpx = 0, tapsx = 0;
   PassPlan fwd, dgrad, wgrad;
   int S = 1;
   // SIMT path
@@ -185,12 +248,29 @@ namespace {
 
 glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_limits_t &L) {
   const int elem = P.elem;
-  const int BK = 128 / elem;
-  const glp_conv_desc_s &d = P.d;
+  const glp_conv_desc_s &d = (mode == MODE_DGRAD) ? P.d : P.dxg;
+  const int Cpx = P.Cpx, tapsx = P.tapsx;
+  // A by im2col TMA when the channel pitch is a multiple of a 64-byte row; K-block rows of 128
+  // bytes when the pitch allows, else 64 (bf16).  Otherwise the cp.async gather (128-byte rows).
+  const int u64 = 64 / elem, u128 = 128 / elem;
+  if (mode == MODE_FWD) {
+    pp.a_tma = (Cpx % u64 == 0 && (elem == 2 || Cpx % u128 == 0)) ? 1 : 0;
+    pp.krow = (!pp.a_tma || Cpx % u128 == 0) ? 128 : 64;
+  } else if (mode == MODE_DGRAD) {
+    pp.a_tma = (P.Cop % u64 == 0 && (elem == 2 || P.Cop % u128 == 0) && d.Sh == 1 && d.Sw == 1) ? 1 : 0;
+    pp.krow = (!pp.a_tma || P.Cop % u128 == 0) ? 128 : 64;
+  } else {
+    pp.a_tma = (Cpx % u64 == 0 && P.Cop % u64 == 0 &&
+                (elem == 2 || (Cpx % u128 == 0 && P.Cop % u128 == 0))) ? 1 : 0;
+    pp.krow = (!pp.a_tma || (Cpx % u128 == 0 && P.Cop % u128 == 0)) ? 128 : 64;
+  }
+  const int BK = pp.krow / elem;     // K elements per k-block (fwd/dgrad)
+  const int BKP = 128 / elem;        // pixels per k-block (wgrad)
+  const int EPA = pp.krow / elem;    // MN elements per MN-major atom (wgrad)
   if (mode == MODE_FWD) {
     pp.M = d.N * d.Ho * d.Wo;
     pp.Ng = d.Co;
-    pp.Kpad = (int)rup((long long)P.taps * P.Cp, BK);
+    pp.Kpad = (int)rup((long long)tapsx * Cpx, BK);
     pp.kb_total = pp.Kpad / BK;
     pp.bn = choose_bn(d.Co);
     pp.bn_smem = pp.bn;
@@ -202,12 +282,12 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     pp.bn = choose_bn(d.C);
     pp.bn_smem = pp.bn;
   } else {
-    pp.M = P.taps * P.Cp;
+    pp.M = tapsx * Cpx;
     pp.Ng = d.Co;
     pp.Kpad = d.N * d.Ho * d.Wo;
-    pp.kb_total = (int)cdiv(pp.Kpad, BK);
+    pp.kb_total = (int)cdiv(pp.Kpad, BKP);
     pp.bn = choose_bn(d.Co);
-    pp.bn_smem = (int)rup(pp.bn, BK);
+    pp.bn_smem = (int)rup(pp.bn, EPA);
   }
   pp.m_tiles = (int)cdiv(pp.M, 128);
   pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
@@ -220,7 +300,9 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     pp.splits = 1;
     pp.kb_per_split = pp.kb_total;
   }
-  const int stage_bytes = 16384 + pp.bn_smem * 128;
+  const int a_bytes = mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow;
+  const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
+  const int stage_bytes = a_bytes + pp.bn_smem * b_row;
   const int budget = 232448 - 1024 - 512;
   pp.stages = std::min(8, budget / stage_bytes);
   if (pp.stages < 2) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
@@ -231,16 +313,20 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16;
   pp.tiles = pp.m_tiles * pp.n_tiles * pp.splits;
 
-  void *fn = igemm_ptr(mode, elem);
+  void *fn = igemm_ptr(mode, elem, pp.krow);
   // The attribute is per function (not per plan): always allow the largest tile of any plan.
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
   GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
   pp.regs = fa.numRegs;
-  glp_kernel_attr_t ka{TileCfg<2>::THREADS, fa.numRegs, pp.smem + (int)fa.sharedSizeBytes, pp.tmem_cols};
+  // TMEM term: the CUDA runtime admits one TMEM-allocating (tcgen05) CTA per SM regardless of
+  // the columns it asks for (measured with tools/occ_probe2.cu; R16), so the record
+  // charges the whole per-SM TMEM to each CTA.
+  glp_kernel_attr_t ka{IGEMM_THREADS, fa.numRegs, pp.smem + (int)fa.sharedSizeBytes,
+                       L.tmem_cols_per_sm > 0 ? L.tmem_cols_per_sm : pp.tmem_cols};
   pp.ctas_per_sm = ctas_per_sm_closed_form(L, ka);
   int rt = 0;
-  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, TileCfg<2>::THREADS, pp.smem));
+  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, IGEMM_THREADS, pp.smem));
   pp.ctas_runtime = rt;
   if (pp.ctas_per_sm < 1) return fail(GLP_ERR_INTERNAL, "kernel does not fit on an SM");
   const int slots = P.sm_count * pp.ctas_per_sm;
@@ -267,7 +353,7 @@ glp_status_t validate_ptrs(std::initializer_list<const void *> ps) {
 }
 
 IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const void *src) {
-  const glp_conv_desc_s &d = P.d;
+  const glp_conv_desc_s &d = (mode == MODE_DGRAD) ? P.d : P.dxg;
   IgemmParams p;
   memset(&p, 0, sizeof(p));
   Gather &g = p.g;
@@ -277,7 +363,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   g.pad = d.Ph;
   g.pad_w = d.Pw;
   g.kw = d.Kw;
-  g.taps = P.taps;
+  g.taps = (mode == MODE_DGRAD) ? P.taps : P.tapsx;
   if (mode == MODE_DGRAD) {
     g.src_h = d.Ho;
     g.src_w = d.Wo;
@@ -288,12 +374,25 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   } else {
     g.src_h = d.H;
     g.src_w = d.W;
-    g.src_cp = P.Cp;
-    g.cp = P.Cp;
+    g.src_cp = P.Cpx;
+    g.cp = P.Cpx;
     g.pix_hw = d.Ho * d.Wo;
     g.pix_w = d.Wo;
   }
   g.n_pixels = d.N * g.pix_hw;
+  if (mode == MODE_DGRAD) {   // im2col over dy with flipped taps (stride 1 only)
+    g.im_sh = 1;
+    g.im_sw = 1;
+    g.im_ph = d.Kh - 1 - d.Ph;
+    g.im_pw = d.Kw - 1 - d.Pw;
+  } else {
+    g.im_sh = d.Sh;
+    g.im_sw = d.Sw;
+    g.im_ph = d.Ph;
+    g.im_pw = d.Pw;
+  }
+  g.cbs = g.cp / (pp.krow / P.elem);
+  p.a_tma = pp.a_tma;
   g.div_hw = FastDiv((uint32_t)g.pix_hw);
   g.div_w = FastDiv((uint32_t)g.pix_w);
   g.div_cp = FastDiv((uint32_t)g.cp);
@@ -317,11 +416,13 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
 
 template <int MODE>
 glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
-                          const CUtensorMap &map, cudaStream_t st) {
-  if (P.elem == 2)
-    igemm_kernel<MODE, 2><<<pp.grid, TileCfg<2>::THREADS, pp.smem, st>>>(p, map);
+                          const CUtensorMap &mapB, const CUtensorMap &mapA, cudaStream_t st) {
+  if (P.elem == 2 && pp.krow == 128)
+    igemm_kernel<MODE, 2, 128><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
+  else if (P.elem == 2)
+    igemm_kernel<MODE, 2, 64><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
   else
-    igemm_kernel<MODE, 4><<<pp.grid, TileCfg<4>::THREADS, pp.smem, st>>>(p, map);
+    igemm_kernel<MODE, 4, 128><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
   GLP_LAUNCH_CHECK("igemm_kernel");
   return GLP_OK;
 }
@@ -349,67 +450,122 @@ glp_status_t run_pack_w_fwd(glp_plan_s &P, const float *w, uint8_t *ws, cudaStre
   const glp_conv_desc_s &d = P.d;
   void *wpk = ws + P.off_wpk;
   const size_t wn = (size_t)d.Co * P.fwd.Kpad;
-  if (P.elem == 2) pack_w_fwd<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
-  else pack_w_fwd<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cp, P.fwd.Kpad);
+  if (P.s2d) {
+    if (P.elem == 2)
+      pack_w_fwd_s2d<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad);
+    else
+      pack_w_fwd_s2d<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad);
+  } else if (P.elem == 2) {
+    pack_w_fwd<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
+  } else {
+    pack_w_fwd<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
+  }
   GLP_LAUNCH_CHECK("pack_w_fwd");
   return GLP_OK;
+}
+
+// x -> the packed operand of the forward / filter-gradient passes (direct NHWC or space-to-depth).
+glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  if (P.s2d) {
+    const int S = P.s2d;
+    const size_t smem = (size_t)S * d.C * d.W * sizeof(float);
+    dim3 grid((unsigned)P.dxg.H, (unsigned)d.N);
+    if (P.elem == 2)
+      pack_s2d<2><<<grid, 256, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
+    else
+      pack_s2d<4><<<grid, 256, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
+    GLP_LAUNCH_CHECK("pack_s2d");
+    return GLP_OK;
+  }
+  return launch_pack_act(P, x, dst, d.C, d.H * d.W, P.Cpx, nullptr, st);
 }
 
 glp_status_t run_pack_w_dgrad(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   void *wtpk = ws + P.off_wpk;
   const size_t wn = (size_t)d.C * P.dgrad.Kpad;
-  if (P.elem == 2) pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
-  else pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad);
+  const int flip = P.dgrad.a_tma;  // the im2col-TMA dgrad walks taps flipped
+  if (P.elem == 2)
+    pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
+  else
+    pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
   GLP_LAUNCH_CHECK("pack_w_dgrad");
   return GLP_OK;
 }
 
 glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, cudaStream_t st) {
-  const glp_conv_desc_s &d = P.d;
+  const glp_conv_desc_s &d = P.dxg;
+  const PassPlan &pp = P.fwd;
   void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
-  glp_status_t s;
-  CUtensorMap map;
-  s = encode_2d(&map, P.elem, wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co, (uint64_t)P.fwd.Kpad * P.elem,
-                128 / P.elem, (uint32_t)P.fwd.bn);
+  const int BK = pp.krow / P.elem;
+  CUtensorMap mapB, mapA;
+  memset(&mapA, 0, sizeof(mapA));
+  glp_status_t s = encode_2d(&mapB, P.elem, wpk, (uint64_t)pp.Kpad, (uint64_t)d.Co,
+                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn,
+                             swz_kmajor(pp.krow));
   if (s) return s;
-  IgemmParams p = make_params(P, P.fwd, MODE_FWD, xpk);
+  if (pp.a_tma) {
+    if ((s = get_encode_im2col())) return s;
+    s = encode_im2col(&mapA, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
+                      d.Ph - (d.Kh - 1), BK, 128, d.Sw, d.Sh, swz_kmajor(pp.krow));
+    if (s) return s;
+  }
+  IgemmParams p = make_params(P, pp, MODE_FWD, xpk);
   p.out = y;
   p.bias = b;
   p.out_c = d.Co;
   p.out_hw = d.Ho * d.Wo;
-  return launch_igemm<MODE_FWD>(P, P.fwd, p, map, st);
+  return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);
 }
 
 glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
+  const PassPlan &pp = P.dgrad;
   void *wtpk = ws + P.off_wpk;
   const void *dypk = ws + P.off_dypk;
-  CUtensorMap map;
-  glp_status_t s = encode_2d(&map, P.elem, wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
-                             (uint64_t)P.dgrad.Kpad * P.elem, 128 / P.elem, (uint32_t)P.dgrad.bn);
+  const int BK = pp.krow / P.elem;
+  CUtensorMap mapB, mapA;
+  memset(&mapA, 0, sizeof(mapA));
+  glp_status_t s = encode_2d(&mapB, P.elem, wtpk, (uint64_t)pp.Kpad, (uint64_t)d.C,
+                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn,
+                             swz_kmajor(pp.krow));
   if (s) return s;
-  IgemmParams p = make_params(P, P.dgrad, MODE_DGRAD, dypk);
+  if (pp.a_tma) {
+    // dx pixel (h, w) reads dy at (h - (Kh-1-Ph) + kh', w - (Kw-1-Pw) + kw') with kh' = Kh-1-kh
+    if ((s = get_encode_im2col())) return s;
+    s = encode_im2col(&mapA, P.elem, dypk, P.Cop, d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw),
+                      -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK, 128, 1, 1, swz_kmajor(pp.krow));
+    if (s) return s;
+  }
+  IgemmParams p = make_params(P, pp, MODE_DGRAD, dypk);
   p.out = dx;
   p.out_c = d.C;
   p.out_hw = d.H * d.W;
-  return launch_igemm<MODE_DGRAD>(P, P.dgrad, p, map, st);
+  return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
 }
 
 glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
-  const glp_conv_desc_s &d = P.d;
+  const glp_conv_desc_s &d = P.dxg;
+  const PassPlan &pp = P.wgrad;
   const void *xpk = ws + P.off_xpk, *dypk = ws + P.off_dypk;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
-  CUtensorMap map;
-  const int BK = 128 / P.elem;
-  glp_status_t s = encode_2d(&map, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
-                             (uint64_t)P.Cop * P.elem, (uint32_t)BK, (uint32_t)BK,
-                             P.elem == 2 ? CU_TENSOR_MAP_SWIZZLE_128B
-                                         : CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);
+  const int BKP = 128 / P.elem, EPA = pp.krow / P.elem;
+  CUtensorMap mapB, mapA;
+  memset(&mapA, 0, sizeof(mapA));
+  glp_status_t s = encode_2d(&mapB, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
+                             (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
+                             swz_mnmajor(P.elem, pp.krow));
   if (s) return s;
-  IgemmParams p = make_params(P, P.wgrad, MODE_WGRAD, xpk);
+  if (pp.a_tma) {
+    if ((s = get_encode_im2col())) return s;
+    s = encode_im2col(&mapA, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
+                      d.Ph - (d.Kh - 1), EPA, BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
+    if (s) return s;
+  }
+  IgemmParams p = make_params(P, pp, MODE_WGRAD, xpk);
   p.out = part;
-  return launch_igemm<MODE_WGRAD>(P, P.wgrad, p, map, st);
+  return launch_igemm<MODE_WGRAD>(P, pp, p, mapB, mapA, st);
 }
 
 glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulate, uint8_t *ws,
@@ -417,9 +573,9 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulat
   const glp_conv_desc_s &d = P.d;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
   const size_t wsz = (size_t)d.Co * d.C * P.taps;
-  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, P.Cp,
+  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
                                              P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_tiles * 128,
-                                             P.wgrad.splits, accumulate);
+                                             P.wgrad.splits, accumulate, P.s2d, P.dxg.Kw);
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
     reduce_db<<<(unsigned)cdiv(d.Co, 32), 256, 0, st>>>(
@@ -586,10 +742,31 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->elem = (math == GLP_MATH_BF16) ? 2 : 4;
   P->sm_count = prop.multiProcessorCount;
   P->s_override = S;
+  // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
+  // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to
+  // 32 would multiply the MMA work; those use the 16-byte-chunk cp.async gather.
   const int CH = 16 / P->elem;
-  P->Cp = (int)rup(d->C, CH);
-  P->Cop = (int)rup(d->Co, CH);
+  P->Cp = (int)(d->C >= 16 ? rup(d->C, 32) : rup(d->C, CH));
+  P->Cop = (int)(d->Co >= 16 ? rup(d->Co, 32) : rup(d->Co, CH));
   P->taps = d->Kh * d->Kw;
+  // Space-to-depth for strided layers when it shrinks the padded K of the GEMM (CaffeNet conv1:
+  // 121 taps x 8 channels -> 9 taps x 64 channels).  Square kernels/strides/pads only.
+  P->dxg = *d;
+  P->Cpx = P->Cp;
+  P->tapsx = P->taps;
+  if (math != GLP_MATH_FP32 && d->Sh == d->Sw && d->Sh > 1 && d->Kh == d->Kw && d->Ph == d->Pw &&
+      d->Kh >= d->Sh) {
+    const int S2 = d->Sh, Ks = (int)cdiv(d->Kh, S2), cs = S2 * S2 * d->C;
+    const int cps = (int)rup(cs, 32);
+    if ((long long)Ks * Ks * cps < (long long)P->taps * rup(P->Cp, 128 / P->elem) &&
+        (size_t)S2 * d->C * d->W * sizeof(float) <= 48 * 1024) {
+      P->s2d = S2;
+      P->dxg = glp_conv_desc_s{d->N, cs, d->Ho + Ks - 1, d->Wo + Ks - 1, d->Co, Ks, Ks, 1, 1,
+                               0, 0, d->Ho, d->Wo};
+      P->Cpx = cps;
+      P->tapsx = Ks * Ks;
+    }
+  }
   glp_device_limits_t L;
   glp_device_limits_b200(&L);
   L.sm_count = prop.multiProcessorCount;
@@ -608,7 +785,9 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
       return s;
     }
     const glp_conv_desc_s &c = *d;
-    P->sz_xpk = align1k((size_t)c.N * c.H * c.W * P->Cp * P->elem);
+    // x region: the forward/filter-gradient operand, or the direct packing of glp_debug_im2col
+    P->sz_xpk = align1k(std::max((size_t)c.N * c.H * c.W * P->Cp,
+                                 (size_t)c.N * P->dxg.H * P->dxg.W * P->Cpx) * P->elem);
     P->sz_dypk = align1k((size_t)c.N * c.Ho * c.Wo * P->Cop * P->elem);
     P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
     P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
@@ -678,7 +857,7 @@ glp_status_t glp_plan_kernel_attr(glp_plan_t P, int which, glp_kernel_attr_t *a,
   if (!P || !a || !model || !rt || which < 0 || which > 2) return fail(GLP_ERR_INVALID_VALUE, "bad argument");
   if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no persistent kernel");
   const PassPlan &pp = which == 0 ? P->fwd : which == 1 ? P->dgrad : P->wgrad;
-  *a = glp_kernel_attr_t{TileCfg<2>::THREADS, pp.regs, pp.smem, pp.tmem_cols};
+  *a = glp_kernel_attr_t{IGEMM_THREADS, pp.regs, pp.smem, pp.tmem_cols};
   *model = pp.ctas_per_sm;
   *rt = pp.ctas_runtime;
   return GLP_OK;
@@ -715,7 +894,7 @@ glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const fl
   }
   if ((s = get_encode())) return s;
   uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if ((s = launch_pack_act(*P, x, wsb + P->off_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = launch_pack_x(*P, x, wsb + P->off_xpk, st))) return s;
   if ((s = run_pack_w_fwd(*P, w, wsb, st))) return s;
   return run_fwd_gemm(*P, b, y, wsb, st);
 }
@@ -753,7 +932,7 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   if (P->math == GLP_MATH_FP32) return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
   if ((s = get_encode())) return s;
   void *xpk = wsb + P->off_xpk, *dypk = wsb + P->off_dypk;
-  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = launch_pack_x(*P, x, xpk, st))) return s;
   if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
                            db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
     return s;
@@ -789,7 +968,7 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
     if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
     if ((s = run_dgrad_gemm(*P, dx, wsb, st))) return s;
   }
-  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = launch_pack_x(*P, x, xpk, st))) return s;
   if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
   return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
 }
@@ -811,7 +990,7 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   switch (what) {
     case GLP_PACK_X:
-      return launch_pack_act(*P, src, wsb + P->off_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st);
+      return launch_pack_x(*P, src, wsb + P->off_xpk, st);
     case GLP_PACK_DY:
       return launch_pack_act(*P, src, wsb + P->off_dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st);
     case GLP_PACK_DY_DB:
@@ -866,7 +1045,13 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   void *xpk = wsb + P->off_xpk;
   if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
-  IgemmParams p = make_params(*P, P->fwd, MODE_FWD, xpk);
+  // the direct (non space-to-depth) gather geometry of the layer
+  glp_plan_s Q = *P;
+  Q.s2d = 0;
+  Q.dxg = Q.d;
+  Q.Cpx = Q.Cp;
+  Q.tapsx = Q.taps;
+  IgemmParams p = make_params(Q, Q.fwd, MODE_FWD, xpk);
   const size_t total = (size_t)P->d.C * P->taps * P->d.Ho * P->d.Wo;
   if (P->elem == 2)
     debug_im2col_kernel<2><<<ew_grid(total), 256, 0, st>>>(p.g, n, P->d.C, P->d.Kh, P->d.Kw, P->d.Ho, P->d.Wo, col);

@@ -9,28 +9,52 @@
 //   MODE_WGRAD: D[(kh,kw,ci), co]    = sum_{pixels p in split} x[gather(p,kh,kw), ci] * dy[p, co]
 //               (fixed, shape-only split of the N*H_o*W_o reduction; partials reduced in order)
 //
-// CTA = 288 threads: warps 0-3 epilogue (TMEM -> registers -> global), warps 4-7 producers
-// (cp.async gather of A into the UMMA SWIZZLE_128B layout), warp 8 TMEM allocator + single-thread
-// tcgen05.mma issuer.  B (weights, or dy for wgrad) is a dense 2-D matrix loaded by TMA.
+// CTA = 288 threads: warps 0-3 epilogue (TMEM -> registers -> global), warps 4-7 producers,
+// warp 8 TMEM allocator + single-thread tcgen05.mma issuer.
+//   A operand: im2col-mode TMA issued by one thread (a_tma = 1), or, for tiny channel counts /
+//              strided dgrad, a cp.async gather by 128 threads into the same SWIZZLE_128B layout.
+//   B operand: dense 2-D matrix (packed weights, or packed dy for wgrad) by tiled TMA.
 // smem ring of `stages` {A,B} slots (mbarrier full/empty), two TMEM accumulators (tfull/tempty)
 // so the epilogue of tile i overlaps the main loop of tile i+1.  Tiles are visited by a static
 // round-robin over a persistent grid (tile t -> CTA t mod grid), the device-side replacement of
 // the paper's round-robin stream dispatch (P171).
+//
+// Shared-memory operand layouts (UMMA canonical, K-block row width KROW bytes):
+//   K-major (fwd/dgrad A and B): rows of KROW bytes, 8-row atoms, SWIZZLE_128B (KROW 128) or
+//     SWIZZLE_64B (KROW 64); one tcgen05.mma consumes 32 bytes of K.
+//   MN-major (wgrad A and B): K-rows of one MN atom (KROW bytes = KROW/ELEM channels) stacked
+//     contiguously; bf16 SWIZZLE_128B/64B (8-row groups), tf32 SWIZZLE_128B_BASE32B (4-row groups).
 #pragma once
 #include "common.cuh"
 #include "ptx.cuh"
 
 namespace glp {
 
-template <int ELEM>
+constexpr int IGEMM_THREADS = 288;
+
+template <int ELEM, int KROW>
 struct TileCfg {
   static constexpr int BM = 128;
-  static constexpr int BK = 128 / ELEM;      // K elements per 128-byte smem row
-  static constexpr int CH = 16 / ELEM;       // elements per 16-byte chunk
-  static constexpr int UMMA_K = 32 / ELEM;   // K of one tcgen05.mma (bf16 16, tf32 8)
-  static constexpr int A_BYTES = BM * 128;   // 16 KB
-  static constexpr int LBO_MN = (BK / 8) * 1024;  // MN-major: stride between 128-byte MN atoms
+  static constexpr int BK = KROW / ELEM;        // K elements per k-block (fwd/dgrad)
+  static constexpr int BKP = 128 / ELEM;        // pixels per k-block (wgrad)
+  static constexpr int CH = 16 / ELEM;          // elements per 16-byte chunk
+  static constexpr int UMMA_K = 32 / ELEM;      // K of one tcgen05.mma (bf16 16, tf32 8)
+  static constexpr int EPA = KROW / ELEM;       // MN elements per MN-major atom row
+  // K-major
+  static constexpr uint32_t K_LAYOUT = (KROW == 128) ? 2u : 4u;
+  static constexpr uint32_t K_SBO = 8u * KROW;
+  // MN-major
+  static constexpr uint32_t MN_LAYOUT = (ELEM == 4) ? 1u : ((KROW == 128) ? 2u : 4u);
+  static constexpr uint32_t MN_GROUP = ((ELEM == 4) ? 4u : 8u) * KROW;   // SBO
+  static constexpr uint32_t MN_LBO = (uint32_t)BKP * KROW;                // one atom column
+  static constexpr uint32_t MN_KSTEP = (uint32_t)UMMA_K * KROW;
   static constexpr int THREADS = 288;
+  __host__ __device__ static constexpr uint32_t a_bytes(int mode) {
+    return mode == MODE_WGRAD ? (uint32_t)BM * BKP * ELEM : (uint32_t)BM * KROW;
+  }
+  __host__ __device__ static constexpr uint32_t b_row_bytes(int mode) {
+    return mode == MODE_WGRAD ? (uint32_t)BKP * ELEM : (uint32_t)KROW;
+  }
 };
 
 __device__ __forceinline__ void decode_tile(int t, int n_tiles, int m_tiles, int &m_tile,
@@ -42,8 +66,7 @@ __device__ __forceinline__ void decode_tile(int t, int n_tiles, int m_tiles, int
 }
 
 // Forward-gather address of one 16-byte chunk: pixel m (GEMM row) and K index k0 (tap*cp + c).
-// Shared by the producer and glp_debug_im2col so that the debug view uses the kernel's own
-// index math.  Returns false for padding / out-of-range taps (chunk is zero).
+// Used by glp_debug_im2col so that the debug view uses the cp.async producer's index math.
 template <int ELEM>
 __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS, int owS,
                                            uint32_t k0, const uint8_t *&src) {
@@ -59,14 +82,17 @@ __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS,
   return true;
 }
 
-template <int MODE, int ELEM>
+template <int MODE, int ELEM, int KROW>
 __global__ void __launch_bounds__(288, 1)
-    igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB) {
-  using C = TileCfg<ELEM>;
+    igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB,
+                 const __grid_constant__ CUtensorMap tmapA) {
+  using C = TileCfg<ELEM, KROW>;
+  constexpr uint32_t A_BYTES = C::a_bytes(MODE);
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
-  const uint32_t stage_bytes = C::A_BYTES + (uint32_t)p.bn_smem * 128u;
+  const uint32_t b_bytes = (uint32_t)p.bn_smem * C::b_row_bytes(MODE);
+  const uint32_t stage_bytes = A_BYTES + b_bytes;
   const uint32_t bars = base + (uint32_t)p.stages * stage_bytes;
   const int S_ = p.stages;
   auto full = [&](int s) { return bars + 8u * s; };
@@ -78,9 +104,11 @@ __global__ void __launch_bounds__(288, 1)
       reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool a_tma = p.a_tma != 0;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S_; ++s) {
-      mbar_init(full(s), 129);   // 128 cp.async arrivals (noinc) + 1 expect_tx arrival (TMA)
+      // TMA mode: 1 expect_tx arrival; cp.async mode: 128 cp.async arrivals (noinc) + 1.
+      mbar_init(full(s), a_tma ? 1 : 129);
       mbar_init(empty(s), 1);    // tcgen05.commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -93,7 +121,10 @@ __global__ void __launch_bounds__(288, 1)
     tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
     tmem_relinquish();
   }
-  if (warp == 4 && lane == 0) tma_prefetch(&tmapB);
+  if (warp == 4 && lane == 0) {
+    tma_prefetch(&tmapB);
+    if (a_tma) tma_prefetch(&tmapA);
+  }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -105,138 +136,216 @@ __global__ void __launch_bounds__(288, 1)
   if (warp >= 4 && warp < 8) {
     // ===================================== producers =======================================
     const int pt = threadIdx.x - 128;
-    uint32_t gk = 0;  // CTA-local k-block counter (ring position)
-    for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-      int m_tile, n_tile, split;
-      decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
-      int kb0 = 0, kb1 = p.kb_total;
-      if (MODE == MODE_WGRAD) {
-        kb0 = split * p.kb_per_split;
-        kb1 = min(kb0 + p.kb_per_split, p.kb_total);
-      }
-      const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
-      if (MODE != MODE_WGRAD) {
-        // K-major A: thread owns 16-byte chunk j of rows rg + 16 i (i = 0..7).
-        const int j = pt & 7, rg = pt >> 3;
-        uint32_t pbase[8];
-        int ohS[8], owS[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const int m = m0 + rg + 16 * i;
-          uint32_t n, rem, oh, ow;
-          g.div_hw.divmod((uint32_t)(m < p.M ? m : 0), n, rem);
-          g.div_w.divmod(rem, oh, ow);
-          pbase[i] = n * (uint32_t)(g.src_h * g.src_w);
-          if (MODE == MODE_FWD) {
-            ohS[i] = (int)oh * g.stride - g.pad;
-            owS[i] = (int)ow * g.stride_w - g.pad_w;
-          } else {
-            ohS[i] = (int)oh + g.pad;
-            owS[i] = (int)ow + g.pad_w;
-          }
-          if (m >= p.M) ohS[i] = -(1 << 28);  // row past M: every tap fails the bounds check
-        }
-        const uint32_t dst0 = (uint32_t)(rg >> 3) * 1024u + (uint32_t)(rg & 7) * 128u +
-                              (uint32_t)((j ^ (rg & 7)) << 4);
-        // K index of this thread's chunk, advanced incrementally by BK per k-block.
-        uint32_t t, c, kh, kw;
-        g.div_cp.divmod((uint32_t)(kb0 * C::BK + j * C::CH), t, c);
-        g.div_kw.divmod(t, kh, kw);
-        const uint8_t *srcb = static_cast<const uint8_t *>(g.src);
-        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-          const int s = (int)(gk % (uint32_t)S_);
-          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
-          mbar_wait(empty(s), ph ^ 1u);
-          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
-          if (pt == 0) {
-            mbar_arrive_expect_tx(full(s), (uint32_t)p.bn_smem * 128u);
-            tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
-          }
-          const bool kv = (int)t < g.taps;
-#pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            int ih, iw;
-            bool ok;
-            if (MODE == MODE_FWD) {
-              ih = ohS[i] + (int)kh;
-              iw = owS[i] + (int)kw;
-              ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
-            } else {
-              const int ihn = ohS[i] - (int)kh, iwn = owS[i] - (int)kw;
-              if (g.stride == 1 && g.stride_w == 1) {
-                ih = ihn;
-                iw = iwn;
-                ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
-              } else {
-                ok = kv && ihn >= 0 && iwn >= 0 && (ihn % g.stride == 0) && (iwn % g.stride_w == 0);
-                ih = ihn / g.stride;
-                iw = iwn / g.stride_w;
-                ok = ok && ih < g.src_h && iw < g.src_w;
+    if (a_tma) {
+      if (pt == 0) {
+        uint32_t gk = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+          int m_tile, n_tile, split;
+          decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+          const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
+          if (MODE != MODE_WGRAD) {
+            // base pixel of the tile's first output pixel; the TMA walks 128 pixels from there
+            uint32_t n, rem, oh, ow;
+            g.div_hw.divmod((uint32_t)m0, n, rem);
+            g.div_w.divmod(rem, oh, ow);
+            const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
+            int t = 0, cb = 0;
+            for (int kb = 0; kb < p.kb_total; ++kb, ++gk) {
+              const int s = (int)(gk % (uint32_t)S_);
+              const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+              mbar_wait(empty(s), ph ^ 1u);
+              const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
+              mbar_arrive_expect_tx(full(s), A_BYTES + b_bytes);
+              uint32_t kh, kw;
+              g.div_kw.divmod((uint32_t)t, kh, kw);
+              tma_load_im2col_4d(sA, &tmapA, full(s), cb * C::BK, w0, h0, (int)n, (uint16_t)kw,
+                                 (uint16_t)kh);
+              tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
+              if (++cb == g.cbs) {
+                cb = 0;
+                ++t;
               }
             }
-            const uint8_t *src = srcb;
-            if (ok)
-              src += ((size_t)(pbase[i] + (uint32_t)(ih * g.src_w + iw)) * (uint32_t)g.src_cp + c) * ELEM;
-            cp_async16(sA + dst0 + (uint32_t)i * 2048u, src, ok);
-          }
-          cp_async_mbar_arrive_noinc(full(s));
-          c += C::BK;
-          if (c >= (uint32_t)g.cp) {
-            const uint32_t q = g.div_cp.div(c);
-            c -= q * (uint32_t)g.cp;
-            t += q;
-            g.div_kw.divmod(t, kh, kw);
+          } else {
+            const int kb0 = split * p.kb_per_split;
+            const int kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+            constexpr int NA = 128 / C::EPA;   // MN atoms of the A tile
+            int ac[NA];
+            uint16_t akh[NA], akw[NA];
+#pragma unroll
+            for (int a = 0; a < NA; ++a) {
+              uint32_t t, c;
+              g.div_cp.divmod((uint32_t)(m0 + a * C::EPA), t, c);
+              if ((int)t < g.taps) {
+                uint32_t kh, kw;
+                g.div_kw.divmod(t, kh, kw);
+                ac[a] = (int)c;
+                akh[a] = (uint16_t)kh;
+                akw[a] = (uint16_t)kw;
+              } else {          // rows past M: channel coordinate out of bounds -> zeros
+                ac[a] = g.src_cp;
+                akh[a] = 0;
+                akw[a] = 0;
+              }
+            }
+            for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+              const int s = (int)(gk % (uint32_t)S_);
+              const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+              mbar_wait(empty(s), ph ^ 1u);
+              const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
+              mbar_arrive_expect_tx(full(s), A_BYTES + b_bytes);
+              uint32_t n, rem, oh, ow;
+              g.div_hw.divmod((uint32_t)(kb * C::BKP), n, rem);
+              g.div_w.divmod(rem, oh, ow);
+              const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
+#pragma unroll
+              for (int a = 0; a < NA; ++a)
+                tma_load_im2col_4d(sA + (uint32_t)a * C::MN_LBO, &tmapA, full(s), ac[a], w0, h0,
+                                   (int)n, akw[a], akh[a]);
+              for (int a = 0; a < p.bn_smem / C::EPA; ++a)
+                tma_load_2d(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), n0 + a * C::EPA,
+                            kb * C::BKP);
+            }
           }
         }
-      } else {
-        // WGRAD: MN-major A (M = (tap, ci) of x, K = pixels).  CPR chunks per K-row.
-        constexpr int CPR = 128 * ELEM / 16;
-        constexpr int RPP = 128 / CPR;
-        const int j = pt % CPR, r0 = pt / CPR;
-        const uint32_t mm = (uint32_t)(m0 + j * C::CH);
-        uint32_t t, c;
-        g.div_cp.divmod(mm, t, c);
-        const bool mvalid = (int)t < g.taps;
-        uint32_t kh, kw;
-        g.div_kw.divmod(mvalid ? t : 0u, kh, kw);
-        const int offh = (int)kh - g.pad, offw = (int)kw - g.pad_w;
-        const uint32_t dcol = (uint32_t)(j >> 3) * C::LBO_MN;
-        const int jj = j & 7;
-        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-          const int s = (int)(gk % (uint32_t)S_);
-          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
-          mbar_wait(empty(s), ph ^ 1u);
-          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
-          if (pt == 0) {
-            mbar_arrive_expect_tx(full(s), (uint32_t)p.bn_smem * 128u);
-            for (int a = 0; a < p.bn_smem / C::BK; ++a)
-              tma_load_2d(sB + (uint32_t)a * C::LBO_MN, &tmapB, full(s), n0 + a * C::BK,
-                          kb * C::BK);
-          }
+      }
+    } else if (KROW == 128) {
+      // -------- cp.async gather (SWIZZLE_128B layouts only) --------
+      uint32_t gk = 0;  // CTA-local k-block counter (ring position)
+      for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+        int m_tile, n_tile, split;
+        decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+        int kb0 = 0, kb1 = p.kb_total;
+        if (MODE == MODE_WGRAD) {
+          kb0 = split * p.kb_per_split;
+          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+        }
+        const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
+        if (MODE != MODE_WGRAD) {
+          // K-major A: thread owns 16-byte chunk j of rows rg + 16 i (i = 0..7).
+          const int j = pt & 7, rg = pt >> 3;
+          uint32_t pbase[8];
+          int ohS[8], owS[8];
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
-            const int r = r0 + RPP * i;
-            const int pix = kb * C::BK + r;
-            bool ok = mvalid && pix < g.n_pixels;
+            const int m = m0 + rg + 16 * i;
             uint32_t n, rem, oh, ow;
-            g.div_hw.divmod((uint32_t)(ok ? pix : 0), n, rem);
+            g.div_hw.divmod((uint32_t)(m < p.M ? m : 0), n, rem);
             g.div_w.divmod(rem, oh, ow);
-            const int ih = (int)oh * g.stride + offh, iw = (int)ow * g.stride_w + offw;
-            ok = ok && ih >= 0 && ih < g.src_h && iw >= 0 && iw < g.src_w;
-            const uint8_t *src = static_cast<const uint8_t *>(g.src);
-            if (ok)
-              src += ((size_t)((size_t)n * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) *
-                          g.src_cp + c) * ELEM;
-            uint32_t dst;
-            if (ELEM == 2)  // SWIZZLE_128B: 16-byte chunks XOR row%8, 8-row (1 KB) K-groups
-              dst = sA + dcol + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
-                    (uint32_t)((jj ^ (r & 7)) << 4);
-            else            // SWIZZLE_128B_BASE32B: 32-byte chunks XOR row%4, 4-row K-groups
-              dst = sA + dcol + (uint32_t)(r >> 2) * 512u + (uint32_t)(r & 3) * 128u +
-                    (uint32_t)((((jj >> 1) ^ (r & 3)) << 5) | ((jj & 1) << 4));
-            cp_async16(dst, src, ok);
+            pbase[i] = n * (uint32_t)(g.src_h * g.src_w);
+            if (MODE == MODE_FWD) {
+              ohS[i] = (int)oh * g.stride - g.pad;
+              owS[i] = (int)ow * g.stride_w - g.pad_w;
+            } else {
+              ohS[i] = (int)oh + g.pad;
+              owS[i] = (int)ow + g.pad_w;
+            }
+            if (m >= p.M) ohS[i] = -(1 << 28);  // row past M: every tap fails the bounds check
           }
-          cp_async_mbar_arrive_noinc(full(s));
+          const uint32_t dst0 = (uint32_t)(rg >> 3) * 1024u + (uint32_t)(rg & 7) * 128u +
+                                (uint32_t)((j ^ (rg & 7)) << 4);
+          // K index of this thread's chunk, advanced incrementally by BK per k-block.
+          uint32_t t, c, kh, kw;
+          g.div_cp.divmod((uint32_t)(kb0 * C::BK + j * C::CH), t, c);
+          g.div_kw.divmod(t, kh, kw);
+          const uint8_t *srcb = static_cast<const uint8_t *>(g.src);
+          for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+            const int s = (int)(gk % (uint32_t)S_);
+            const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+            mbar_wait(empty(s), ph ^ 1u);
+            const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
+            if (pt == 0) {
+              mbar_arrive_expect_tx(full(s), b_bytes);
+              tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
+            }
+            const bool kv = (int)t < g.taps;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              int ih, iw;
+              bool ok;
+              if (MODE == MODE_FWD) {
+                ih = ohS[i] + (int)kh;
+                iw = owS[i] + (int)kw;
+                ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
+              } else {
+                const int ihn = ohS[i] - (int)kh, iwn = owS[i] - (int)kw;
+                if (g.stride == 1 && g.stride_w == 1) {
+                  ih = ihn;
+                  iw = iwn;
+                  ok = kv && (unsigned)ih < (unsigned)g.src_h && (unsigned)iw < (unsigned)g.src_w;
+                } else {
+                  ok = kv && ihn >= 0 && iwn >= 0 && (ihn % g.stride == 0) &&
+                       (iwn % g.stride_w == 0);
+                  ih = ihn / g.stride;
+                  iw = iwn / g.stride_w;
+                  ok = ok && ih < g.src_h && iw < g.src_w;
+                }
+              }
+              const uint8_t *src = srcb;
+              if (ok)
+                src += ((size_t)(pbase[i] + (uint32_t)(ih * g.src_w + iw)) * (uint32_t)g.src_cp + c) *
+                       ELEM;
+              cp_async16(sA + dst0 + (uint32_t)i * 2048u, src, ok);
+            }
+            cp_async_mbar_arrive_noinc(full(s));
+            c += C::BK;
+            if (c >= (uint32_t)g.cp) {
+              const uint32_t q = g.div_cp.div(c);
+              c -= q * (uint32_t)g.cp;
+              t += q;
+              g.div_kw.divmod(t, kh, kw);
+            }
+          }
+        } else {
+          // WGRAD: MN-major A (M = (tap, ci) of x, K = pixels).  CPR chunks per K-row.
+          constexpr int CPR = 128 * ELEM / 16;
+          constexpr int RPP = 128 / CPR;
+          const int j = pt % CPR, r0 = pt / CPR;
+          const uint32_t mm = (uint32_t)(m0 + j * C::CH);
+          uint32_t t, c;
+          g.div_cp.divmod(mm, t, c);
+          const bool mvalid = (int)t < g.taps;
+          uint32_t kh, kw;
+          g.div_kw.divmod(mvalid ? t : 0u, kh, kw);
+          const int offh = (int)kh - g.pad, offw = (int)kw - g.pad_w;
+          const uint32_t dcol = (uint32_t)(j >> 3) * C::MN_LBO;
+          const int jj = j & 7;
+          for (int kb = kb0; kb < kb1; ++kb, ++gk) {
+            const int s = (int)(gk % (uint32_t)S_);
+            const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+            mbar_wait(empty(s), ph ^ 1u);
+            const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
+            if (pt == 0) {
+              mbar_arrive_expect_tx(full(s), b_bytes);
+              for (int a = 0; a < p.bn_smem / C::EPA; ++a)
+                tma_load_2d(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), n0 + a * C::EPA,
+                            kb * C::BKP);
+            }
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const int r = r0 + RPP * i;
+              const int pix = kb * C::BKP + r;
+              bool ok = mvalid && pix < g.n_pixels;
+              uint32_t n, rem, oh, ow;
+              g.div_hw.divmod((uint32_t)(ok ? pix : 0), n, rem);
+              g.div_w.divmod(rem, oh, ow);
+              const int ih = (int)oh * g.stride + offh, iw = (int)ow * g.stride_w + offw;
+              ok = ok && ih >= 0 && ih < g.src_h && iw >= 0 && iw < g.src_w;
+              const uint8_t *src = static_cast<const uint8_t *>(g.src);
+              if (ok)
+                src += ((size_t)((size_t)n * g.src_h * g.src_w + (size_t)ih * g.src_w + iw) *
+                            g.src_cp + c) * ELEM;
+              uint32_t dst;
+              if (ELEM == 2)  // SWIZZLE_128B: 16-byte chunks XOR row%8, 8-row (1 KB) K-groups
+                dst = sA + dcol + (uint32_t)(r >> 3) * 1024u + (uint32_t)(r & 7) * 128u +
+                      (uint32_t)((jj ^ (r & 7)) << 4);
+              else            // SWIZZLE_128B_BASE32B: 32-byte chunks XOR row%4, 4-row K-groups
+                dst = sA + dcol + (uint32_t)(r >> 2) * 512u + (uint32_t)(r & 3) * 128u +
+                      (uint32_t)((((jj >> 1) ^ (r & 3)) << 5) | ((jj & 1) << 4));
+              cp_async16(dst, src, ok);
+            }
+            cp_async_mbar_arrive_noinc(full(s));
+          }
         }
       }
     }
@@ -246,6 +355,7 @@ __global__ void __launch_bounds__(288, 1)
       constexpr uint32_t fmt = (ELEM == 2) ? 1u : 2u;  // BF16 : TF32
       constexpr uint32_t mn = (MODE == MODE_WGRAD) ? 1u : 0u;
       const uint32_t idesc = make_idesc(fmt, mn, mn, 128u, (uint32_t)p.bn);
+      constexpr int KSTEPS = (MODE == MODE_WGRAD) ? C::BKP / C::UMMA_K : C::BK / C::UMMA_K;
       uint32_t gk = 0, it = 0;
       for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++it) {
         int m_tile, n_tile, split;
@@ -264,20 +374,16 @@ __global__ void __launch_bounds__(288, 1)
           const uint32_t ph = (gk / (uint32_t)S_) & 1u;
           mbar_wait(full(s), ph);
           tc_fence_after();
-          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + C::A_BYTES;
+          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
 #pragma unroll
-          for (int k = 0; k < C::BK / C::UMMA_K; ++k) {
+          for (int k = 0; k < KSTEPS; ++k) {
             uint64_t ad, bd;
             if (MODE == MODE_WGRAD) {
-              // each UMMA_K step covers UMMA_K rows of 128 B (bf16 16 rows, tf32 8 rows)
-              constexpr uint32_t kstep = C::UMMA_K * 128u;
-              constexpr uint32_t sbo = (ELEM == 2) ? 1024u : 512u;
-              constexpr uint32_t lay = (ELEM == 2) ? 2u : 1u;
-              ad = make_sdesc(sA + (uint32_t)k * kstep, C::LBO_MN, sbo, lay);
-              bd = make_sdesc(sB + (uint32_t)k * kstep, C::LBO_MN, sbo, lay);
+              ad = make_sdesc(sA + (uint32_t)k * C::MN_KSTEP, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
+              bd = make_sdesc(sB + (uint32_t)k * C::MN_KSTEP, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
             } else {
-              ad = make_sdesc(sA + (uint32_t)k * 32u, 16u, 1024u);
-              bd = make_sdesc(sB + (uint32_t)k * 32u, 16u, 1024u);
+              ad = make_sdesc(sA + (uint32_t)k * 32u, 16u, C::K_SBO, C::K_LAYOUT);
+              bd = make_sdesc(sB + (uint32_t)k * 32u, 16u, C::K_SBO, C::K_LAYOUT);
             }
             const uint32_t acc = (kb > kb0 || k > 0) ? 1u : 0u;
             if (ELEM == 2) mma_f16(d, ad, bd, idesc, acc);
@@ -297,7 +403,7 @@ __global__ void __launch_bounds__(288, 1)
       int m_tile, n_tile, split;
       decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
-      mbar_wait(tfull(a), aph);
+      mbar_wait_sleep(tfull(a), aph);
       tc_fence_after();
       const int m = m_tile * C::BM + row;
       const int n0 = n_tile * p.bn;
@@ -310,17 +416,15 @@ __global__ void __launch_bounds__(288, 1)
         for (int c0 = 0; c0 < p.bn; c0 += 32) {
           uint32_t v[32];
           tmem_ld32(taddr + (uint32_t)c0, v);
+          float bv = 0.f;
+          if (MODE == MODE_FWD && p.bias && n0 + c0 + lane < p.N) bv = __ldg(p.bias + n0 + c0 + lane);
           tmem_wait_ld();
-          if (mv) {
 #pragma unroll
-            for (int q = 0; q < 32; ++q) {
-              const int ch = n0 + c0 + q;
-              if (c0 + q < p.bn && ch < p.N) {
-                float val = __uint_as_float(v[q]);
-                if (MODE == MODE_FWD && p.bias) val += __ldg(p.bias + ch);
-                outp[(size_t)ch * p.out_hw] = val;
-              }
-            }
+          for (int q = 0; q < 32; ++q) {
+            const int ch = n0 + c0 + q;
+            float val = __uint_as_float(v[q]);
+            if (MODE == MODE_FWD) val += __shfl_sync(0xffffffffu, bv, q);  // bias[ch], warp-uniform
+            if (mv && c0 + q < p.bn && ch < p.N) outp[(size_t)ch * p.out_hw] = val;
           }
         }
       } else {

@@ -115,6 +115,64 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__re
   }
 }
 
+// Space-to-depth pack for strided convolutions with few input channels:
+//   x'[n][h'][w'][c'] = x[n][c][S*h' + dh - P][S*w' + dw - P]  (0 outside),  c' = (dh*S + dw)*C + c
+// turns a stride-S, K x K conv into a stride-1, ceil(K/S) x ceil(K/S) conv over S*S*C channels
+// with the same output, so the implicit GEMM runs unit-stride im2col TMA on a dense channel axis.
+// One block per (n, h'): the S source rows are staged in shared memory (coalesced reads), then the
+// output row is written with 16-byte stores.  Dynamic smem = S*C*W floats.
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
+                                                int C, int H, int W, int S, int P, int Hs, int Ws,
+                                                int Cps) {
+  extern __shared__ float rows[];  // [S][C][W]
+  const int hs = blockIdx.x, n = blockIdx.y;
+  const int SCW = S * C * W;
+  for (int i = threadIdx.x; i < SCW; i += blockDim.x) {
+    const int w = i % W, c = (i / W) % C, dh = i / (C * W);
+    const int ih = S * hs + dh - P;
+    rows[i] = (ih >= 0 && ih < H) ? __ldg(x + (((size_t)n * C + c) * H + ih) * W + w) : 0.f;
+  }
+  __syncthreads();
+  const int quads = Cps / 4, cs = S * S * C;
+  for (int i = threadIdx.x; i < Ws * quads; i += blockDim.x) {
+    const int ws = i / quads, q = i % quads;
+    float v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int cc = 4 * q + u;
+      float val = 0.f;
+      if (cc < cs) {
+        const int c = cc % C, dd = cc / C, dh = dd / S, dw = dd % S;
+        const int iw = S * ws + dw - P;
+        if (iw >= 0 && iw < W) val = rows[(dh * C + c) * W + iw];
+      }
+      v[u] = val;
+    }
+    PackOut<ELEM>::store4(dst, (((size_t)n * Hs + hs) * Ws + ws) * Cps + 4 * q, v[0], v[1], v[2], v[3]);
+  }
+}
+
+// Forward B operand in the space-to-depth geometry: Wp[co][t'*Cps + c'], t' = kh'*Ks + kw',
+// c' = (dh*S + dw)*C + c, value W[co][c][S*kh'+dh][S*kw'+dw] (0 past the K x K window).
+template <int ELEM>
+__global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
+                               int K, int S, int Ks, int Cps, int Kpad) {
+  const size_t total = (size_t)Co * Kpad;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
+       i += (size_t)gridDim.x * blockDim.x) {
+    const int co = (int)(i / Kpad), k = (int)(i % Kpad);
+    const int t = k / Cps, cc = k % Cps;
+    float v = 0.f;
+    if (t < Ks * Ks && cc < S * S * C) {
+      const int khs = t / Ks, kws = t % Ks, c = cc % C, dd = cc / C, dh = dd / S, dw = dd % S;
+      const int kh = S * khs + dh, kw = S * kws + dw;
+      if (kh < K && kw < K) v = __ldg(w + (((size_t)co * C + c) * K + kh) * K + kw);
+    }
+    PackOut<ELEM>::store1(out, i, v);
+  }
+}
+
 // W [Co][C][Kh][Kw] -> forward B operand Wp[co][tap*Cp + c] with row length Kpad (zero padded).
 template <int ELEM>
 __global__ void pack_w_fwd(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
@@ -131,16 +189,18 @@ __global__ void pack_w_fwd(const float *__restrict__ w, void *__restrict__ out, 
 }
 
 // W [Co][C][Kh][Kw] -> backward-data B operand Wt[ci][tap*Cop + co] (row length Kpad).
+// flip = 1: tap index reversed (tap' = taps-1-tap, i.e. (Kh-1-kh, Kw-1-kw)) for the im2col-TMA
+// dgrad, which walks dy from the window's top-left corner.
 template <int ELEM>
 __global__ void pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
-                             int taps, int Cop, int Kpad) {
+                             int taps, int Cop, int Kpad, int flip) {
   const size_t total = (size_t)C * Kpad;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
        i += (size_t)gridDim.x * blockDim.x) {
     const int ci = (int)(i / Kpad), k = (int)(i % Kpad);
     const int t = k / Cop, co = k % Cop;
     float v = 0.f;
-    if (t < taps && co < Co) v = __ldg(w + ((size_t)co * C + ci) * taps + t);
+    if (t < taps && co < Co) v = __ldg(w + ((size_t)co * C + ci) * taps + (flip ? taps - 1 - t : t));
     PackOut<ELEM>::store1(out, i, v);
   }
 }

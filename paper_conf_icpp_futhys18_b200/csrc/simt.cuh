@@ -164,15 +164,23 @@ __global__ void reduce_simt_dw(const float *__restrict__ part, float *__restrict
 
 // dW (Caffe layout [co][ci][kh][kw]) from tensor-core partials part[s][tap*Cp + ci][co]
 // (leading dimension ld, mpad rows per split), summed in split order.
+// s2d > 1: partial rows are in the space-to-depth geometry (stride s2d, Ks = ceil(Kw/s2d)):
+// row = ((kh/S)*Ks + kw/S)*Cp + ((kh%S)*S + kw%S)*C + ci.
 __global__ void reduce_tc_dw(const float *__restrict__ part, float *__restrict__ dw, int Co, int C,
-                             int taps, int Cp, int ld, int mpad, int splits, int accumulate) {
+                             int taps, int Kw, int Cp, int ld, int mpad, int splits, int accumulate,
+                             int s2d, int Ks) {
   const size_t wsz = (size_t)Co * C * taps;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < wsz;
        i += (size_t)gridDim.x * blockDim.x) {
     const int t = (int)(i % taps);
     const size_t r = i / taps;
     const int ci = (int)(r % C), co = (int)(r / C);
-    const size_t off = (size_t)(t * Cp + ci) * ld + co;
+    int row = t * Cp + ci;
+    if (s2d > 1) {
+      const int kh = t / Kw, kw = t % Kw;
+      row = ((kh / s2d) * Ks + kw / s2d) * Cp + ((kh % s2d) * s2d + kw % s2d) * C + ci;
+    }
+    const size_t off = (size_t)row * ld + co;
     const float s = pairwise_sum(part + off, splits, (size_t)mpad * ld);
     dw[i] = accumulate ? dw[i] + s : s;
   }

@@ -427,6 +427,24 @@ glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmPa
   return GLP_OK;
 }
 
+// db reduction scratch: [rows x Co partials | DB_GROUPS x Co group sums | ceil(Co/32) tickets]
+struct DbAux {
+  float *part, *part2;
+  unsigned int *tickets;
+};
+size_t db_aux_bytes(int rows, int Co) {
+  return align1k((size_t)rows * Co * 4) + align1k((size_t)DB_GROUPS * Co * 4) +
+         align1k((size_t)cdiv(Co, 32) * 4);
+}
+DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
+  DbAux a;
+  a.part = reinterpret_cast<float *>(base);
+  a.part2 = reinterpret_cast<float *>(base + align1k((size_t)rows * P.d.Co * 4));
+  a.tickets = reinterpret_cast<unsigned int *>(base + align1k((size_t)rows * P.d.Co * 4) +
+                                               align1k((size_t)DB_GROUPS * P.d.Co * 4));
+  return a;
+}
+
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
                              int Cp, float *db_part, cudaStream_t st) {
   if (db_part == nullptr && Cp * P.elem <= 32) {
@@ -438,8 +456,11 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
     return GLP_OK;
   }
   dim3 grid((unsigned)cdiv(HW, PACK_PT), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
-  if (P.elem == 2) pack_nchw_to_nhwc<2><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
-  else pack_nchw_to_nhwc<4><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part);
+  unsigned int *tickets = nullptr;
+  if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
+  const int nt = (int)cdiv(P.d.Co, 32);
+  if (P.elem == 2) pack_nchw_to_nhwc<2><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part, tickets, nt);
+  else pack_nchw_to_nhwc<4><<<grid, 256, 0, st>>>(src, dst, C, HW, Cp, db_part, tickets, nt);
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
 }
@@ -469,7 +490,7 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
   const glp_conv_desc_s &d = P.d;
   if (P.s2d) {
     const int S = P.s2d;
-    const size_t smem = (size_t)S * d.C * d.W * sizeof(float);
+    const size_t smem = (size_t)S * d.C * d.W * sizeof(float) + (size_t)P.Cpx * sizeof(int);
     dim3 grid((unsigned)P.dxg.H, (unsigned)d.N);
     if (P.elem == 2)
       pack_s2d<2><<<grid, 256, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
@@ -572,14 +593,15 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulat
                               cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
-  const size_t wsz = (size_t)d.Co * d.C * P.taps;
-  reduce_tc_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
+  reduce_tc_dw<<<dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32)),
+                 dim3(32, 8), 0, st>>>(part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
                                              P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_tiles * 128,
                                              P.wgrad.splits, accumulate, P.s2d, P.dxg.Kw);
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
-    reduce_db<<<(unsigned)cdiv(d.Co, 32), 256, 0, st>>>(
-        reinterpret_cast<float *>(ws + P.off_dbpart), db, d.Co, P.db_rows, accumulate);
+    DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
+    reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), 256, 0, st>>>(
+        a.part, db, d.Co, P.db_rows, accumulate, a.part2, a.tickets);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
@@ -602,7 +624,10 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
   if (db) {
     simt_db_partial<<<ew_grid((size_t)P.simt_splits * d.Co), 256, 0, st>>>(geom(d), dy, dbp, P.simt_splits, P.simt_chunk);
     GLP_LAUNCH_CHECK("simt_db_partial");
-    reduce_db<<<(unsigned)cdiv(d.Co, 32), 256, 0, st>>>(dbp, db, d.Co, P.simt_splits, accumulate);
+    DbAux a = db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.simt_splits);
+    GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
+    reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), 256, 0, st>>>(
+        a.part, db, d.Co, P.simt_splits, accumulate, a.part2, a.tickets);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
@@ -793,7 +818,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
     P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_tiles * 128 * P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, PACK_PT);
-    P->sz_dbpart = align1k((size_t)P->db_rows * c.Co * 4);
+    P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk/wtpk | part | dbpart]
     P->off_xpk = 0;
     P->off_dypk = P->sz_xpk;
@@ -815,7 +840,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     const size_t wsz = (size_t)d->Co * d->C * d->Kh * d->Kw;
     P->ws_fwd = 0;
     P->ws_dgrad = 0;
-    P->ws_wgrad = align1k(wsz * P->simt_splits * 4) + align1k((size_t)P->simt_splits * d->Co * 4);
+    P->ws_wgrad = align1k(wsz * P->simt_splits * 4) + db_aux_bytes(P->simt_splits, d->Co);
     P->ws_bwd = P->ws_wgrad;
     P->S = S > 0 ? std::min(S, d->N) : d->N;
   }

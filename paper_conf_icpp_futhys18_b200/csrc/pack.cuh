@@ -53,9 +53,14 @@ constexpr int PACK_PT = 128;
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict__ src,
                                                          void *__restrict__ dst, int C, int HW,
-                                                         int Cp, float *__restrict__ db_part) {
+                                                         int Cp, float *__restrict__ db_part,
+                                                         unsigned int *__restrict__ tickets,
+                                                         int n_tickets) {
   __shared__ float tile[32][PACK_PT + 1];
   const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * PACK_PT;
+  // arm the completion tickets of the deterministic db reduction that consumes db_part
+  if (tickets != nullptr && (blockIdx.x | blockIdx.y | blockIdx.z) == 0)
+    for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const float *s = src + (size_t)n * C * HW;
   float v[4][4];
@@ -81,17 +86,21 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
     }
   }
   __syncthreads();
-  const int pp = threadIdx.x >> 1, h = threadIdx.x & 1;
-  const int px = p0 + pp;
-  if (px < HW) {
+  // 16-byte chunks: lanes cover consecutive chunks of a pixel's 32-channel row (64 B bf16 /
+  // 128 B fp32), so each warp store instruction writes whole contiguous row segments.
+  constexpr int CPT = 16 / ELEM;            // channels per 16-byte chunk
+  constexpr int CPP = 32 / CPT;             // chunks per pixel row of the tile
+  constexpr int PPP = 256 / CPP;            // pixels per pass
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int cl = 16 * h + 4 * q, c = c0 + cl;
-      if (c < Cp) {
-        const size_t o = ((size_t)n * HW + px) * Cp + c;
-        PackOut<ELEM>::store4(dst, o, tile[cl][pp], tile[cl + 1][pp], tile[cl + 2][pp],
-                              tile[cl + 3][pp]);
-      }
+  for (int pass = 0; pass < PACK_PT / PPP; ++pass) {
+    const int pp = pass * PPP + threadIdx.x / CPP, j = threadIdx.x % CPP;
+    const int px = p0 + pp, cl = j * CPT, c = c0 + cl;
+    if (px < HW && c < Cp) {
+      const size_t o = ((size_t)n * HW + px) * Cp + c;
+#pragma unroll
+      for (int u = 0; u < CPT; u += 4)
+        PackOut<ELEM>::store4(dst, o + u, tile[cl + u][pp], tile[cl + u + 1][pp],
+                              tile[cl + u + 2][pp], tile[cl + u + 3][pp]);
     }
   }
 }
@@ -125,27 +134,45 @@ template <int ELEM>
 __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
                                                 int C, int H, int W, int S, int P, int Hs, int Ws,
                                                 int Cps) {
-  extern __shared__ float rows[];  // [S][C][W]
+  extern __shared__ float smem_s2d[];
+  // [S][C][W] source rows, then a per-output-channel table: (row offset into rows, dw) or -1.
+  float *rows = smem_s2d;
+  int *tab = reinterpret_cast<int *>(smem_s2d + S * C * W);
   const int hs = blockIdx.x, n = blockIdx.y;
-  const int SCW = S * C * W;
-  for (int i = threadIdx.x; i < SCW; i += blockDim.x) {
-    const int w = i % W, c = (i / W) % C, dh = i / (C * W);
+  const int cs = S * S * C;
+  for (int cc = threadIdx.x; cc < Cps; cc += blockDim.x) {
+    int e = -1;
+    if (cc < cs) {
+      const int c = cc % C, dd = cc / C, dh = dd / S, dw = dd % S;
+      e = ((dh * C + c) * W) | (dw << 24);   // W*S*C < 2^24 (host-checked smem bound)
+    }
+    tab[cc] = e;
+  }
+  const size_t xb = (size_t)n * C * H;
+  for (int dh = 0; dh < S; ++dh) {
     const int ih = S * hs + dh - P;
-    rows[i] = (ih >= 0 && ih < H) ? __ldg(x + (((size_t)n * C + c) * H + ih) * W + w) : 0.f;
+    const bool rin = ih >= 0 && ih < H;
+    for (int c = 0; c < C; ++c) {
+      const float *src = x + ((xb + (size_t)c * H + (rin ? ih : 0)) * W);
+      float *d = rows + (dh * C + c) * W;
+      for (int w = threadIdx.x; w < W; w += blockDim.x) d[w] = rin ? __ldg(src + w) : 0.f;
+    }
   }
   __syncthreads();
-  const int quads = Cps / 4, cs = S * S * C;
+  const int quads = Cps >> 2;
+  // thread -> (output pixel ws, channel quad q); quads is a power-of-two-free small count, so the
+  // split is done with one division per 4 outputs
   for (int i = threadIdx.x; i < Ws * quads; i += blockDim.x) {
-    const int ws = i / quads, q = i % quads;
+    const int ws = i / quads, q = i - ws * quads;
+    const int base_w = S * ws - P;
     float v[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      const int cc = 4 * q + u;
+      const int e = tab[4 * q + u];
       float val = 0.f;
-      if (cc < cs) {
-        const int c = cc % C, dd = cc / C, dh = dd / S, dw = dd % S;
-        const int iw = S * ws + dw - P;
-        if (iw >= 0 && iw < W) val = rows[(dh * C + c) * W + iw];
+      if (e >= 0) {
+        const int iw = base_w + (e >> 24);
+        if (iw >= 0 && iw < W) val = rows[(e & 0xFFFFFF) + iw];
       }
       v[u] = val;
     }

@@ -130,26 +130,18 @@ __global__ void simt_db_partial(ConvGeom g, const float *__restrict__ dy, float 
   }
 }
 
-// Fixed-order (pairwise, index-determined) sum of `cnt` partials strided by `stride`.
+// Fixed-order sum of `cnt` partials strided by `stride`: sequential within blocks of 8, block sums
+// added in block order.  The order is a function of cnt only (shape), never of the grid or S.
 __device__ __forceinline__ float pairwise_sum(const float *__restrict__ p, int cnt, size_t stride) {
-  // iterative pairwise over blocks of 8 (sequential inside), then tree over blocks: the order is
-  // a function of cnt only.
-  float blk[64];
-  int nb = 0;
+  float tot = 0.f;
   for (int b0 = 0; b0 < cnt; b0 += 8) {
     float a = 0.f;
     const int e = b0 + 8 < cnt ? b0 + 8 : cnt;
+#pragma unroll 8
     for (int k = b0; k < e; ++k) a += __ldg(p + (size_t)k * stride);
-    if (nb < 64) blk[nb++] = a;
-    else blk[63] += a;  // unreachable for cnt <= 512 (callers guarantee)
+    tot += a;
   }
-  while (nb > 1) {
-    int h = (nb + 1) / 2;
-    for (int k = 0; k < nb / 2; ++k) blk[k] = blk[2 * k] + blk[2 * k + 1];
-    if (nb & 1) blk[nb / 2] = blk[nb - 1];
-    nb = h;
-  }
-  return nb ? blk[0] : 0.f;
+  return tot;
 }
 
 // dW (Caffe layout) from SIMT partials part[s][dW element].
@@ -166,45 +158,102 @@ __global__ void reduce_simt_dw(const float *__restrict__ part, float *__restrict
 // (leading dimension ld, mpad rows per split), summed in split order.
 // s2d > 1: partial rows are in the space-to-depth geometry (stride s2d, Ks = ceil(Kw/s2d)):
 // row = ((kh/S)*Ks + kw/S)*Cp + ((kh%S)*S + kw%S)*C + ci.
-__global__ void reduce_tc_dw(const float *__restrict__ part, float *__restrict__ dw, int Co, int C,
-                             int taps, int Kw, int Cp, int ld, int mpad, int splits, int accumulate,
-                             int s2d, int Ks) {
-  const size_t wsz = (size_t)Co * C * taps;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < wsz;
-       i += (size_t)gridDim.x * blockDim.x) {
-    const int t = (int)(i % taps);
-    const size_t r = i / taps;
-    const int ci = (int)(r % C), co = (int)(r / C);
-    int row = t * Cp + ci;
-    if (s2d > 1) {
-      const int kh = t / Kw, kw = t % Kw;
-      row = ((kh / s2d) * Ks + kw / s2d) * Cp + ((kh % s2d) * s2d + kw % s2d) * C + ci;
+// Block (32, 8) per tile of 32 output channels x 32 inner dW indices (i = ci*taps + t): warps read
+// 32 consecutive co of one partial row per split (coalesced), the tile is transposed through
+// shared memory, and dW[co][i] is written 32 consecutive i at a time.  grid (ceil(C*taps/32),
+// ceil(Co/32)).
+__global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ part,
+                                                    float *__restrict__ dw, int Co, int C,
+                                                    int taps, int Kw, int Cp, int ld, int mpad,
+                                                    int splits, int accumulate, int s2d, int Ks) {
+  __shared__ float tile[32][33];
+  const int inner = C * taps;
+  const int i0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
+  const int lane = threadIdx.x, ty = threadIdx.y;
+  const size_t sstride = (size_t)mpad * ld;
+  const float *src[4];
+  bool ok[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int i = i0 + ty + 8 * u, co = co0 + lane;
+    ok[u] = i < inner && co < Co;
+    int row = 0;
+    if (ok[u]) {
+      const int ci = i / taps, t = i - ci * taps;
+      row = t * Cp + ci;
+      if (s2d > 1) {
+        const int kh = t / Kw, kw = t % Kw;
+        row = ((kh / s2d) * Ks + kw / s2d) * Cp + ((kh % s2d) * s2d + kw % s2d) * C + ci;
+      }
     }
-    const size_t off = (size_t)row * ld + co;
-    const float s = pairwise_sum(part + off, splits, (size_t)mpad * ld);
-    dw[i] = accumulate ? dw[i] + s : s;
+    src[u] = part + (size_t)row * ld + (ok[u] ? co : 0);
+  }
+  // fixed order: splits summed sequentially in blocks of 8, block sums in block order (same for
+  // every element; 32 independent loads in flight per batch)
+  float tot[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int b0 = 0; b0 < splits; b0 += 8) {
+    float a[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (b0 + k < splits) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (ok[u]) a[u] += __ldg(src[u] + (size_t)(b0 + k) * sstride);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) tot[u] += a[u];
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u) tile[ty + 8 * u][lane] = tot[u];
+  __syncthreads();
+  for (int j = ty; j < 32; j += 8) {
+    const int co = co0 + j, i = i0 + lane;
+    if (co < Co && i < inner) {
+      const size_t idx = (size_t)co * inner + i;
+      const float v = tile[lane][j];
+      dw[idx] = accumulate ? dw[idx] + v : v;
+    }
   }
 }
 
 // db[co] = sum over rows of part[row][co] (rows = N * pixel tiles, or SIMT splits), fixed order.
-// One block of 256 threads per 32 channels: thread (ty, lane) sums rows ty, ty+8, ... for channel
-// c0+lane (coalesced across lanes), then a fixed 8-way tree in shared memory.  The order depends
-// only on `rows` (shape), never on the grid or S.
+// db[co] = sum over `rows` partial rows, deterministic and parallel over row groups:
+// grid (ceil(Co/32), DB_GROUPS).  Block (x, g) sums rows g, g+G, ... (thread ty takes every 8th of
+// those, lanes = channels, coalesced), reduces its 8 warps in a fixed tree, and stores part2[g][co];
+// the last block to finish for a channel group (atomic ticket) sums part2[0..G) in index order.
+// The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
+constexpr int DB_GROUPS = 64;
 __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
                                                  float *__restrict__ db, int Co, int rows,
-                                                 int accumulate) {
+                                                 int accumulate, float *__restrict__ part2,
+                                                 unsigned int *__restrict__ tickets) {
   __shared__ float red[8][33];
+  __shared__ bool last;
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
-  const int co = blockIdx.x * 32 + lane;
+  const int co = blockIdx.x * 32 + lane, g = blockIdx.y;
   float a = 0.f;
   if (co < Co)
-    for (int r = ty; r < rows; r += 8) a += __ldg(part + (size_t)r * Co + co);
+    for (int r = g + DB_GROUPS * ty; r < rows; r += DB_GROUPS * 8) a += __ldg(part + (size_t)r * Co + co);
   red[ty][lane] = a;
   __syncthreads();
-  if (ty == 0 && co < Co) {
+  if (ty == 0) {
     const float s = ((red[0][lane] + red[1][lane]) + (red[2][lane] + red[3][lane])) +
                     ((red[4][lane] + red[5][lane]) + (red[6][lane] + red[7][lane]));
-    db[co] = accumulate ? db[co] + s : s;
+    if (co < Co) part2[(size_t)g * Co + co] = s;
+    __threadfence();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) last = (atomicAdd(tickets + blockIdx.x, 1u) == DB_GROUPS - 1);
+  __syncthreads();
+  if (last && ty == 0) {
+    __threadfence();
+    if (co < Co) {
+      float s = 0.f;
+      for (int k = 0; k < DB_GROUPS; ++k) s += __ldcg(part2 + (size_t)k * Co + co);
+      db[co] = accumulate ? db[co] + s : s;
+    }
+    if (lane == 0) tickets[blockIdx.x] = 0;   // re-arm for the next call on this workspace
   }
 }
 

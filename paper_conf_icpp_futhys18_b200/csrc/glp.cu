@@ -83,6 +83,7 @@ struct PassPlan {
   int stages = 0, acc_cols = 0, tmem_cols = 0, smem = 0, tiles = 0, grid = 0, ctas_per_sm = 0;
   int regs = 0, ctas_runtime = 0;
   int a_tma = 0, krow = 128;        // A operand by im2col TMA; K-block row width (bytes)
+  int cg = 1, m_units = 0;          // CTAs per MMA (tcgen05 cta_group); work units along M
 };
 
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -168,19 +169,24 @@ glp_status_t encode_im2col(CUtensorMap *map, int elem, const void *ptr, int cpit
   return GLP_OK;
 }
 
-template <int MODE, int ELEM, int KROW>
+template <int MODE, int ELEM, int KROW, int CG>
 void *kernel_ptr() {
-  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM, KROW>);
+  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM, KROW, CG>);
 }
-template <int MODE>
+template <int MODE, int CG>
 void *igemm_ptr_m(int elem, int krow) {
-  if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128>() : kernel_ptr<MODE, 2, 64>();
-  return kernel_ptr<MODE, 4, 128>();
+  if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128, CG>() : kernel_ptr<MODE, 2, 64, CG>();
+  return kernel_ptr<MODE, 4, 128, CG>();
 }
-void *igemm_ptr(int mode, int elem, int krow) {
-  if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD>(elem, krow);
-  if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD>(elem, krow);
-  return igemm_ptr_m<MODE_WGRAD>(elem, krow);
+void *igemm_ptr(int mode, int elem, int krow, int cg) {
+  if (cg == 2) {
+    if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 2>(elem, krow);
+    if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 2>(elem, krow);
+    return igemm_ptr_m<MODE_WGRAD, 2>(elem, krow);
+  }
+  if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 1>(elem, krow);
+  if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 1>(elem, krow);
+  return igemm_ptr_m<MODE_WGRAD, 1>(elem, krow);
 }
 
 CUtensorMapSwizzle swz_kmajor(int krow) {
@@ -200,8 +206,8 @@ int choose_bn(int n) {
 // Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
 // (constants, never the queried device or S), so the fp32 summation order is a function of the
 // shape alone (convergence invariance, P264).
-int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem) {
-  const double sm = 148.0;
+int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem, int cg) {
+  const double sm = 148.0 / cg;   // concurrent work units (CTA pairs for cg = 2)
   const double kb_s = (elem == 2 ? 2.0 : 4.0) * std::max(bn, 96) / 1.8e9;  // seconds per k-block
   const double bw = 6.0e12;
   int best = 1;
@@ -242,6 +248,8 @@ struct glp_plan_s {
   int db_rows = 0;
   size_t ws_fwd = 0, ws_dgrad = 0, ws_wgrad = 0, ws_bwd = 0;
   double plan_us = 0;
+  int allow_cg2 = 1;   // GLP_CTA_GROUP=1 in the environment forces single-CTA MMAs (A/B runs)
+  int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
 
 namespace {
@@ -291,9 +299,17 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   }
   pp.m_tiles = (int)cdiv(pp.M, 128);
   pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
+  // CTA pairs (tcgen05 cta_group::2, M = 256): each SM loads half of B.  Needs the TMA A path,
+  // at least two row tiles, and (MN-major B) half tiles that are whole swizzle atoms.
+  pp.cg = 1;
+  if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && mode != MODE_WGRAD) {
+    pp.cg = 2;
+    pp.bn_smem = pp.bn / 2;
+  }
+  pp.m_units = (int)cdiv(pp.m_tiles, pp.cg);
   if (mode == MODE_WGRAD) {
-    pp.splits = choose_splits(pp.m_tiles * pp.n_tiles, pp.kb_total, pp.bn, pp.m_tiles * 128,
-                              pp.n_tiles * pp.bn, elem);
+    pp.splits = choose_splits(pp.m_units * pp.n_tiles, pp.kb_total, pp.bn,
+                              pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg);
     pp.kb_per_split = (int)cdiv(pp.kb_total, pp.splits);
     pp.splits = (int)cdiv(pp.kb_total, pp.kb_per_split);
   } else {
@@ -305,15 +321,17 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const int stage_bytes = a_bytes + pp.bn_smem * b_row;
   const int budget = 232448 - 1024 - 512;
   pp.stages = std::min(8, budget / stage_bytes);
+  if (const char *e = getenv("GLP_DEBUG_STAGES"))   // diagnostics: fewer ring stages
+    pp.stages = std::max(2, std::min(pp.stages, atoi(e)));
   if (pp.stages < 2) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
   pp.acc_cols = (int)rup(pp.bn, 32);
   int tc = 32;
   while (tc < 2 * pp.acc_cols) tc *= 2;
   pp.tmem_cols = tc;
   pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16;
-  pp.tiles = pp.m_tiles * pp.n_tiles * pp.splits;
+  pp.tiles = pp.m_units * pp.n_tiles * pp.splits;   // work units (tile pairs for cg = 2)
 
-  void *fn = igemm_ptr(mode, elem, pp.krow);
+  void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg);
   // The attribute is per function (not per plan): always allow the largest tile of any plan.
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
@@ -329,18 +347,18 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, IGEMM_THREADS, pp.smem));
   pp.ctas_runtime = rt;
   if (pp.ctas_per_sm < 1) return fail(GLP_ERR_INTERNAL, "kernel does not fit on an SM");
-  const int slots = P.sm_count * pp.ctas_per_sm;
+  const int slots = P.sm_count * pp.ctas_per_sm / pp.cg;   // resident work-unit slots
   int grid = std::min(pp.tiles, slots);
   if (P.s_override > 0 && mode != MODE_WGRAD) {
     // S samples in flight: the grid covers the tiles of S samples (P262 batch-level parallelism).
     const int hw = (mode == MODE_FWD) ? d.Ho * d.Wo : d.H * d.W;
-    const long long tiles_s = cdiv((long long)P.s_override * hw, 128) * pp.n_tiles;
+    const long long tiles_s = cdiv(cdiv((long long)P.s_override * hw, 128), pp.cg) * pp.n_tiles;
     grid = (int)std::max(1LL, std::min<long long>(grid, tiles_s));
   } else if (P.s_override > 0) {
     const long long tiles_s = cdiv((long long)pp.tiles * P.s_override, d.N);
     grid = (int)std::max(1LL, std::min<long long>(grid, tiles_s));
   }
-  pp.grid = std::max(1, grid);
+  pp.grid = std::max(1, grid) * pp.cg;   // CTAs (pairs are clusters of 2)
   return GLP_OK;
 }
 
@@ -393,13 +411,14 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   }
   g.cbs = g.cp / (pp.krow / P.elem);
   p.a_tma = pp.a_tma;
+  p.dbg_skip = P.dbg_skip;
   g.div_hw = FastDiv((uint32_t)g.pix_hw);
   g.div_w = FastDiv((uint32_t)g.pix_w);
   g.div_cp = FastDiv((uint32_t)g.cp);
   g.div_kw = FastDiv((uint32_t)g.kw);
   p.M = pp.M;
   p.N = pp.Ng;
-  p.m_tiles = pp.m_tiles;
+  p.m_tiles = pp.m_units;   // the kernel iterates work units along M
   p.n_tiles = pp.n_tiles;
   p.splits = pp.splits;
   p.kb_total = pp.kb_total;
@@ -410,19 +429,30 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   p.tmem_cols = pp.tmem_cols;
   p.acc_cols = pp.acc_cols;
   p.part_ld = pp.n_tiles * pp.bn;
-  p.part_mpad = pp.m_tiles * 128;
+  p.part_mpad = pp.m_units * pp.cg * 128;
   return p;
 }
 
 template <int MODE>
 glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
                           const CUtensorMap &mapB, const CUtensorMap &mapA, cudaStream_t st) {
-  if (P.elem == 2 && pp.krow == 128)
-    igemm_kernel<MODE, 2, 128><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
-  else if (P.elem == 2)
-    igemm_kernel<MODE, 2, 64><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
-  else
-    igemm_kernel<MODE, 4, 128><<<pp.grid, IGEMM_THREADS, pp.smem, st>>>(p, mapB, mapA);
+  void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg);
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3((unsigned)pp.grid);
+  cfg.blockDim = dim3(IGEMM_THREADS);
+  cfg.dynamicSmemBytes = (size_t)pp.smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)pp.cg;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  void *args[] = {const_cast<IgemmParams *>(&p), const_cast<CUtensorMap *>(&mapB),
+                  const_cast<CUtensorMap *>(&mapA)};
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, fn, args));
   GLP_LAUNCH_CHECK("igemm_kernel");
   return GLP_OK;
 }
@@ -523,7 +553,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, 
   CUtensorMap mapB, mapA;
   memset(&mapA, 0, sizeof(mapA));
   glp_status_t s = encode_2d(&mapB, P.elem, wpk, (uint64_t)pp.Kpad, (uint64_t)d.Co,
-                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn,
+                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
                              swz_kmajor(pp.krow));
   if (s) return s;
   if (pp.a_tma) {
@@ -549,7 +579,7 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   CUtensorMap mapB, mapA;
   memset(&mapA, 0, sizeof(mapA));
   glp_status_t s = encode_2d(&mapB, P.elem, wtpk, (uint64_t)pp.Kpad, (uint64_t)d.C,
-                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn,
+                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
                              swz_kmajor(pp.krow));
   if (s) return s;
   if (pp.a_tma) {
@@ -767,6 +797,8 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->elem = (math == GLP_MATH_BF16) ? 2 : 4;
   P->sm_count = prop.multiProcessorCount;
   P->s_override = S;
+  if (const char *e = getenv("GLP_CTA_GROUP")) P->allow_cg2 = (atoi(e) != 1);
+  if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 15;
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to
   // 32 would multiply the MMA work; those use the 16-byte-chunk cp.async gather.
@@ -816,7 +848,8 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->sz_dypk = align1k((size_t)c.N * c.Ho * c.Wo * P->Cop * P->elem);
     P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
     P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
-    P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_tiles * 128 * P->wgrad.n_tiles * P->wgrad.bn * 4);
+    P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
+                         P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, PACK_PT);
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk/wtpk | part | dbpart]

@@ -57,6 +57,15 @@ struct TileCfg {
   }
 };
 
+// Advance a (slot, phase) ring position without division (the MMA issuer's loop is latency-bound:
+// a runtime `gk % stages` costs more than the tcgen05.mma work of a small-N k-block).
+__device__ __forceinline__ void ring_next(int &s, uint32_t &ph, int S) {
+  if (++s == S) {
+    s = 0;
+    ph ^= 1u;
+  }
+}
+
 __device__ __forceinline__ void decode_tile(int t, int n_tiles, int m_tiles, int &m_tile,
                                             int &n_tile, int &split) {
   n_tile = t % n_tiles;
@@ -82,7 +91,10 @@ __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS,
   return true;
 }
 
-template <int MODE, int ELEM, int KROW>
+// CG = 1: one CTA per 128-row tile.  CG = 2: CTA pairs (cluster of 2) run tcgen05.mma.cta_group::2
+// with M = 256: each CTA loads its own 128 A rows and half of the B tile (p.bn_smem = BN/2), the
+// pair leader issues the MMAs for both SMs and multicasts its commits (A by TMA only).
+template <int MODE, int ELEM, int KROW, int CG>
 __global__ void __launch_bounds__(288, 1)
     igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB,
                  const __grid_constant__ CUtensorMap tmapA) {
@@ -104,45 +116,55 @@ __global__ void __launch_bounds__(288, 1)
       reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const bool a_tma = p.a_tma != 0;
+  const bool a_tma = (CG == 2) || p.a_tma != 0;
+  const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
+  const bool leader = rank == 0;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S_; ++s) {
-      // TMA mode: 1 expect_tx arrival; cp.async mode: 128 cp.async arrivals (noinc) + 1.
+      // CG1: TMA mode 1 expect_tx arrival; cp.async mode 128 cp.async arrivals (noinc) + 1.
+      // CG2: only the leader arrives (expect_tx = both CTAs' bytes); the peer's TMA completes
+      // bytes on the leader's barrier (as CUTLASS's 2-SM TMA pipeline).
       mbar_init(full(s), a_tma ? 1 : 129);
-      mbar_init(empty(s), 1);    // tcgen05.commit
+      mbar_init(empty(s), 1);    // tcgen05.commit (multicast to both CTAs for CG2)
     }
     for (int a = 0; a < 2; ++a) {
-      mbar_init(tfull(a), 1);    // tcgen05.commit after the last k-block of a tile
-      mbar_init(tempty(a), 128); // every epilogue thread
+      mbar_init(tfull(a), 1);         // tcgen05.commit after the last k-block of a tile
+      mbar_init(tempty(a), 4 * CG);   // one arrival per epilogue warp (of both CTAs for CG2)
     }
     fence_mbar_init();
   }
   if (warp == 8) {
-    tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
-    tmem_relinquish();
+    tmem_alloc_cg<CG>(tmem_slot, (uint32_t)p.tmem_cols);
+    tmem_relinquish_cg<CG>();
   }
   if (warp == 4 && lane == 0) {
     tma_prefetch(&tmapB);
     if (a_tma) tma_prefetch(&tmapA);
   }
   tc_fence_before();
-  __syncthreads();
+  if (CG == 2) cluster_sync();
+  else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot_ptr;
 
-  const int total_tiles = p.m_tiles * p.n_tiles * p.splits;
+  // work units: CG1 = one 128-row tile; CG2 = a pair of 128-row tiles (one per CTA)
+  const int total_tiles = p.m_tiles * p.n_tiles * p.splits;   // p.m_tiles counts units along M
+  const int unit0 = (CG == 2) ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ustep = (CG == 2) ? (int)(gridDim.x >> 1) : (int)gridDim.x;
   const Gather &g = p.g;
 
   if (warp >= 4 && warp < 8) {
     // ===================================== producers =======================================
     const int pt = threadIdx.x - 128;
     if (a_tma) {
-      if (pt == 0) {
-        uint32_t gk = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+      if (warp == 4) {   // one converged warp; each TMA / arrive is issued by an elected lane
+        int rs = 0;          // ring slot and its phase, advanced incrementally
+        uint32_t rph = 0;
+        for (int tile = unit0; tile < total_tiles; tile += ustep) {
           int m_tile, n_tile, split;
           decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
-          const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
+          const int m0 = (m_tile * CG + (int)rank) * C::BM, n0 = n_tile * p.bn;
+          const int nb0 = n0 + (int)rank * p.bn_smem;   // this CTA's part of the B tile
           if (MODE != MODE_WGRAD) {
             // base pixel of the tile's first output pixel; the TMA walks 128 pixels from there
             uint32_t n, rem, oh, ow;
@@ -150,17 +172,29 @@ __global__ void __launch_bounds__(288, 1)
             g.div_w.divmod(rem, oh, ow);
             const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
             int t = 0, cb = 0;
-            for (int kb = 0; kb < p.kb_total; ++kb, ++gk) {
-              const int s = (int)(gk % (uint32_t)S_);
-              const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+            for (int kb = 0; kb < p.kb_total; ++kb, ring_next(rs, rph, S_)) {
+              const int s = rs;
+              const uint32_t ph = rph;
               mbar_wait(empty(s), ph ^ 1u);
               const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
-              mbar_arrive_expect_tx(full(s), A_BYTES + b_bytes);
               uint32_t kh, kw;
               g.div_kw.divmod((uint32_t)t, kh, kw);
-              tma_load_im2col_4d(sA, &tmapA, full(s), cb * C::BK, w0, h0, (int)n, (uint16_t)kw,
-                                 (uint16_t)kh);
-              tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
+              if (CG == 1) {
+                const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+                mbar_arrive_expect_tx_e(full(s), (la ? A_BYTES : 0u) + (lb ? b_bytes : 0u));
+                if (la)
+                  tma_load_im2col_4d_e(sA, &tmapA, full(s), cb * C::BK, w0, h0, (int)n,
+                                       (uint16_t)kw, (uint16_t)kh);
+                if (lb) tma_load_2d_e(sB, &tmapB, full(s), kb * C::BK, nb0);
+              } else {
+                const uint32_t fullL = mapa_shared(full(s), 0);
+                if (leader) mbar_arrive_expect_tx_e(full(s), 2u * (A_BYTES + b_bytes));
+                // the peer only adds bytes (complete_tx) to the leader's barrier; no arrival —
+                // a release-scoped remote arrive here would fence this thread's in-flight TMA
+                tma_load_im2col_4d_cg2_e(sA, &tmapA, fullL, cb * C::BK, w0, h0, (int)n,
+                                         (uint16_t)kw, (uint16_t)kh);
+                tma_load_2d_cg2_e(sB, &tmapB, fullL, kb * C::BK, nb0);
+              }
               if (++cb == g.cbs) {
                 cb = 0;
                 ++t;
@@ -188,31 +222,46 @@ __global__ void __launch_bounds__(288, 1)
                 akw[a] = 0;
               }
             }
-            for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-              const int s = (int)(gk % (uint32_t)S_);
-              const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+            for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
+              const int s = rs;
+              const uint32_t ph = rph;
               mbar_wait(empty(s), ph ^ 1u);
               const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
-              mbar_arrive_expect_tx(full(s), A_BYTES + b_bytes);
               uint32_t n, rem, oh, ow;
               g.div_hw.divmod((uint32_t)(kb * C::BKP), n, rem);
               g.div_w.divmod(rem, oh, ow);
               const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
+              if (CG == 1) {
+                mbar_arrive_expect_tx_e(full(s), A_BYTES + b_bytes);
 #pragma unroll
-              for (int a = 0; a < NA; ++a)
-                tma_load_im2col_4d(sA + (uint32_t)a * C::MN_LBO, &tmapA, full(s), ac[a], w0, h0,
-                                   (int)n, akw[a], akh[a]);
-              for (int a = 0; a < p.bn_smem / C::EPA; ++a)
-                tma_load_2d(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), n0 + a * C::EPA,
-                            kb * C::BKP);
+                for (int a = 0; a < NA; ++a)
+                  tma_load_im2col_4d_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, full(s), ac[a], w0,
+                                       h0, (int)n, akw[a], akh[a]);
+                for (int a = 0; a < p.bn_smem / C::EPA; ++a)
+                  tma_load_2d_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), nb0 + a * C::EPA,
+                                kb * C::BKP);
+              } else {
+                const uint32_t fullL = mapa_shared(full(s), 0);
+                if (leader) mbar_arrive_expect_tx_e(full(s), 2u * (A_BYTES + b_bytes));
+                // the peer only adds bytes (complete_tx) to the leader's barrier; no arrival —
+                // a release-scoped remote arrive here would fence this thread's in-flight TMA
+#pragma unroll
+                for (int a = 0; a < NA; ++a)
+                  tma_load_im2col_4d_cg2_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, fullL, ac[a],
+                                           w0, h0, (int)n, akw[a], akh[a]);
+                for (int a = 0; a < p.bn_smem / C::EPA; ++a)
+                  tma_load_2d_cg2_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, fullL,
+                                    nb0 + a * C::EPA, kb * C::BKP);
+              }
             }
           }
         }
       }
-    } else if (KROW == 128) {
+    } else if (KROW == 128 && CG == 1) {
       // -------- cp.async gather (SWIZZLE_128B layouts only) --------
-      uint32_t gk = 0;  // CTA-local k-block counter (ring position)
-      for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+      int rs = 0;          // ring slot and its phase, advanced incrementally
+        uint32_t rph = 0;
+      for (int tile = unit0; tile < total_tiles; tile += ustep) {
         int m_tile, n_tile, split;
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
         int kb0 = 0, kb1 = p.kb_total;
@@ -249,9 +298,9 @@ __global__ void __launch_bounds__(288, 1)
           g.div_cp.divmod((uint32_t)(kb0 * C::BK + j * C::CH), t, c);
           g.div_kw.divmod(t, kh, kw);
           const uint8_t *srcb = static_cast<const uint8_t *>(g.src);
-          for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-            const int s = (int)(gk % (uint32_t)S_);
-            const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+          for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
+            const int s = rs;
+            const uint32_t ph = rph;
             mbar_wait(empty(s), ph ^ 1u);
             const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
             if (pt == 0) {
@@ -310,9 +359,9 @@ __global__ void __launch_bounds__(288, 1)
           const int offh = (int)kh - g.pad, offw = (int)kw - g.pad_w;
           const uint32_t dcol = (uint32_t)(j >> 3) * C::MN_LBO;
           const int jj = j & 7;
-          for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-            const int s = (int)(gk % (uint32_t)S_);
-            const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+          for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
+            const int s = rs;
+            const uint32_t ph = rph;
             mbar_wait(empty(s), ph ^ 1u);
             const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
             if (pt == 0) {
@@ -351,13 +400,14 @@ __global__ void __launch_bounds__(288, 1)
     }
   } else if (warp == 8) {
     // ===================================== MMA issuer ======================================
-    if (lane == 0) {
+    if (leader) {   // whole warp runs the loop; each tcgen05 op is issued by an elected lane
       constexpr uint32_t fmt = (ELEM == 2) ? 1u : 2u;  // BF16 : TF32
       constexpr uint32_t mn = (MODE == MODE_WGRAD) ? 1u : 0u;
-      const uint32_t idesc = make_idesc(fmt, mn, mn, 128u, (uint32_t)p.bn);
+      const uint32_t idesc = make_idesc(fmt, mn, mn, 128u * CG, (uint32_t)p.bn);
       constexpr int KSTEPS = (MODE == MODE_WGRAD) ? C::BKP / C::UMMA_K : C::BK / C::UMMA_K;
-      uint32_t gk = 0, it = 0;
-      for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++it) {
+      int rs = 0;
+      uint32_t rph = 0, it = 0;
+      for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
         int m_tile, n_tile, split;
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
         int kb0 = 0, kb1 = p.kb_total;
@@ -369,14 +419,16 @@ __global__ void __launch_bounds__(288, 1)
         mbar_wait(tempty(a), aph ^ 1u);
         tc_fence_after();
         const uint32_t d = tmem_base + a * (uint32_t)p.acc_cols;
-        for (int kb = kb0; kb < kb1; ++kb, ++gk) {
-          const int s = (int)(gk % (uint32_t)S_);
-          const uint32_t ph = (gk / (uint32_t)S_) & 1u;
+        for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
+          const int s = rs;
+          const uint32_t ph = rph;
           mbar_wait(full(s), ph);
           tc_fence_after();
           const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
+          const int ksteps = (p.dbg_skip & 4) ? (kb == kb0 ? 1 : 0) : KSTEPS;
 #pragma unroll
           for (int k = 0; k < KSTEPS; ++k) {
+            if (k >= ksteps) break;
             uint64_t ad, bd;
             if (MODE == MODE_WGRAD) {
               ad = make_sdesc(sA + (uint32_t)k * C::MN_KSTEP, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
@@ -386,12 +438,11 @@ __global__ void __launch_bounds__(288, 1)
               bd = make_sdesc(sB + (uint32_t)k * 32u, 16u, C::K_SBO, C::K_LAYOUT);
             }
             const uint32_t acc = (kb > kb0 || k > 0) ? 1u : 0u;
-            if (ELEM == 2) mma_f16(d, ad, bd, idesc, acc);
-            else mma_tf32(d, ad, bd, idesc, acc);
+            mma_e<(ELEM == 2) ? 0 : 1, CG>(d, ad, bd, idesc, acc);
           }
-          mma_commit(empty(s));
+          mma_commit_e<CG>(empty(s));
         }
-        mma_commit(tfull(a));
+        mma_commit_e<CG>(tfull(a));
       }
     }
     __syncwarp();
@@ -399,15 +450,15 @@ __global__ void __launch_bounds__(288, 1)
     // ===================================== epilogue ========================================
     const int row = warp * 32 + lane;
     uint32_t it = 0;
-    for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++it) {
+    for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
       int m_tile, n_tile, split;
       decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
       mbar_wait_sleep(tfull(a), aph);
       tc_fence_after();
-      const int m = m_tile * C::BM + row;
+      const int m = (m_tile * CG + (int)rank) * C::BM + row;
       const int n0 = n_tile * p.bn;
-      const bool mv = m < p.M;
+      const bool mv = m < p.M && !(p.dbg_skip & 8);
       const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
       if (MODE != MODE_WGRAD) {
         uint32_t n, pimg;
@@ -450,13 +501,18 @@ __global__ void __launch_bounds__(288, 1)
         }
       }
       tc_fence_before();
-      mbar_arrive(tempty(a));
+      __syncwarp();
+      if (lane == 0) {   // one arrival per warp (on the pair leader's barrier for CG2)
+        if (CG == 1) mbar_arrive(tempty(a));
+        else mbar_arrive_cluster(mapa_shared(tempty(a), 0));
+      }
     }
   }
   tc_fence_before();
-  __syncthreads();
+  if (CG == 2) cluster_sync();
+  else __syncthreads();
   tc_fence_after();
-  if (warp == 8) tmem_dealloc(tmem_base, (uint32_t)p.tmem_cols);
+  if (warp == 8) tmem_dealloc_cg<CG>(tmem_base, (uint32_t)p.tmem_cols);
 }
 
 }  // namespace glp

@@ -219,3 +219,22 @@ def test_staged_equals_composed(math):
     torch.cuda.synchronize()
     for k, v in (("y", y), ("dx", dx), ("dw", dw), ("db", db)):
         np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=k)
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[2], SHAPES[5], SHAPES[6]], ids=lambda s: s[0])
+def test_single_cta_mma_path(shape, math, monkeypatch):
+    """GLP_CTA_GROUP=1 forces single-CTA tcgen05 MMAs (no CTA pairs): still bit-exact on integer
+    data, and equal to the default (paired) plan on random data (same per-element K order)."""
+    d = _data(shape, exact=True, seed=21)
+    monkeypatch.setenv("GLP_CTA_GROUP", "1")
+    got = _run(_layer(shape, math), d)
+    ref = _oracle(d, shape[7], shape[8])
+    for k in ref:
+        np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+    dr = _data(shape, seed=22)
+    one = _run(_layer(shape, math), dr)
+    monkeypatch.delenv("GLP_CTA_GROUP")
+    two = _run(_layer(shape, math), dr)
+    for k in ("y", "dx"):
+        np.testing.assert_array_equal(one[k], two[k], err_msg=k)

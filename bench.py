@@ -128,7 +128,7 @@ class ClockSampler:
 # ------------------------------------------------------------------------- GLP arm ------------
 
 class LayerState:
-    def __init__(self, layer, n_local, n_global, shard, math, dev, flat, off):
+    def __init__(self, layer, n_local, n_global, shard, math, dev, grads, idx):
         import torch
         import paper_conf_icpp_futhys18_b200 as glp
         self.layer = layer
@@ -137,20 +137,18 @@ class LayerState:
                                   layer.P, math=math, device=dev.index)
         if shard is None:
             d = gen_layer(layer, n_global=n_global, batch=n_local)
-        else:
-            r, g = shard
+        else:  # strong scaling: this rank's contiguous slice of the global batch
+            a, b = shard
             full = gen_layer(layer, n_global=n_global)
             d = {k: v for k, v in full.items()}
-            d["x"] = full["x"][r * n_local:(r + 1) * n_local].copy()
-            d["dy"] = full["dy"][r * n_local:(r + 1) * n_local].copy()
+            d["x"] = full["x"][a:b].copy()
+            d["dy"] = full["dy"][a:b].copy()
         self.host = {k: torch.from_numpy(v) for k, v in d.items()}
         self.t = {k: v.to(dev) for k, v in self.host.items()}
         self.y = torch.empty(self.conv.y_shape, device=dev)
         self.dx = None if layer.data_fed else torch.empty(self.conv.x_shape, device=dev)
-        wn = layer.Co * layer.C * layer.K * layer.K
-        self.dw = flat[off:off + wn].view(self.conv.w_shape)
-        self.db = flat[off + wn:off + wn + layer.Co]
-        self.nparams = wn + layer.Co
+        self.dw = grads.dw(idx)      # views into the flat dW||db buffer (one all_reduce per step)
+        self.db = grads.db(idx)
         self.flops = float(self.layer.with_batch(n_local).flops_per_pass())
 
     def launches(self):
@@ -167,22 +165,23 @@ def run_glp(args, ws, rank, local):
     torch.cuda.set_device(dev)
     if ws > 1:
         dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_icpp_futhys18_b200.dist import FlatGrads, shard_range
     layers = config(args.workload)
     G = ws
+    shards = [shard_range(l.N, rank, G) for l in layers]
     if args.scaling == "strong":
-        n_local = [l.N // G for l in layers]
+        n_local = [b - a for a, b in shards]
         n_global = [l.N for l in layers]
     else:
         n_local = [l.N for l in layers]
         n_global = [l.N * G for l in layers]
-    nparams = sum(l.Co * l.C * l.K * l.K + l.Co for l in layers)
-    flat = torch.zeros(nparams, device=dev)
-    states, off = [], 0
-    for l, nl, ng in zip(layers, n_local, n_global):
-        shard = (rank, G) if args.scaling == "strong" and G > 1 else None
-        st = LayerState(l, nl, ng, shard, args.math, dev, flat, off)
-        off += st.nparams
-        states.append(st)
+    grads = FlatGrads([l.w_shape for l in layers], device=dev)
+    flat = grads.buf
+    nparams = grads.numel
+    states = []
+    for i, (l, nl, ng) in enumerate(zip(layers, n_local, n_global)):
+        shard = shards[i] if args.scaling == "strong" and G > 1 else None
+        states.append(LayerState(l, nl, ng, shard, args.math, dev, grads, i))
     stream = torch.cuda.current_stream()
 
     def step(ev=None):
@@ -215,7 +214,7 @@ def run_glp(args, ws, rank, local):
                 ev[i][5].record(stream)
             c.stage_reduce(s.dw, s.db)
         if G > 1:
-            dist.all_reduce(flat)
+            grads.allreduce()
 
     for _ in range(args.warmup):
         step()

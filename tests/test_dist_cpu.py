@@ -1,0 +1,100 @@
+"""CPU (gloo, world_size 2) tests of the multi-GPU path's host logic: batch sharding, the flat
+dW||db buffer and its single all_reduce.  The per-rank compute is the oracle (a fake backend), so
+the test checks sharding/ordering/scaling with no GPU."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+from glp_workloads import gen_custom
+from paper_conf_icpp_futhys18_b200.dist import FlatGrads, shard_range
+
+LAYERS = [(4, 3, 9, 9, 5, 3, 1, 1), (4, 5, 7, 7, 6, 3, 2, 1)]   # N, C, H, W, Co, K, S, P
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _data():
+    out = []
+    for i, (N, C, H, W, Co, K, S, P) in enumerate(LAYERS):
+        Ho = oracle.out_dim(H, K, S, P)
+        out.append(gen_custom(N, C, H, W, Co, K, K, 40 + i, Ho=Ho, Wo=Ho))
+    return out
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    data = _data()
+    fg = FlatGrads([(L[4], L[1], L[5], L[5]) for L in LAYERS])
+    for i, (N, C, H, W, Co, K, S, P) in enumerate(LAYERS):
+        a, b = shard_range(N, rank, world)
+        d = data[i]
+        dw, db = oracle.conv_bwd_filter(d["x"][a:b], d["dy"][a:b], d["w"].shape, S, P)
+        fg.dw(i).copy_(torch.from_numpy(dw.astype(np.float32)))
+        fg.db(i).copy_(torch.from_numpy(db.astype(np.float32)))
+    local = fg.buf.clone()
+    fg.allreduce()
+    q.put((rank, local.numpy(), fg.buf.numpy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_shard_range_partition():
+    for n in (1, 7, 64, 256, 257):
+        for w in (1, 2, 3, 4, 8):
+            if w > n:
+                continue
+            rs = [shard_range(n, r, w) for r in range(w)]
+            assert rs[0][0] == 0 and rs[-1][1] == n
+            assert all(rs[i][1] == rs[i + 1][0] for i in range(w - 1))
+            sizes = [b - a for a, b in rs]
+            assert max(sizes) - min(sizes) <= 1
+
+
+def test_flat_grads_views():
+    fg = FlatGrads([(2, 3, 3, 3), (4, 2, 1, 1)])
+    assert fg.numel == 2 * 27 + 2 + 4 * 2 + 4
+    fg.dw(1).fill_(1.0)
+    fg.db(0).fill_(2.0)
+    assert float(fg.buf.sum()) == 8 * 1.0 + 2 * 2.0
+    assert fg.dw(0).shape == (2, 3, 3, 3) and fg.db(1).shape == (4,)
+
+
+def test_gloo_allreduce_equals_full_batch():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=240) for _ in range(world)], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    locals_ = [r[1] for r in res]
+    reduced = [r[2] for r in res]
+    # every rank holds the same reduced buffer; for G = 2 it is the fp32 sum of the two halves
+    np.testing.assert_array_equal(reduced[0], reduced[1])
+    np.testing.assert_array_equal(reduced[0], (locals_[0] + locals_[1]).astype(np.float32))
+    # and equals the full-batch oracle gradients (sum over the whole batch, R10)
+    data = _data()
+    off = 0
+    for i, (N, C, H, W, Co, K, S, P) in enumerate(LAYERS):
+        dw, db = oracle.conv_bwd_filter(data[i]["x"], data[i]["dy"], data[i]["w"].shape, S, P)
+        n = dw.size
+        assert oracle.normwise_err(reduced[0][off:off + n].reshape(dw.shape), dw) < 1e-6
+        assert oracle.normwise_err(reduced[0][off + n:off + n + Co], db) < 1e-6
+        off += n + Co

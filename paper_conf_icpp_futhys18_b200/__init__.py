@@ -16,7 +16,8 @@ import os
 from dataclasses import dataclass
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libglp.so")
+# GLP_LIB overrides the in-tree library (A/B runs of two builds on one box)
+LIB_PATH = os.environ.get("GLP_LIB") or os.path.join(PKG, "libglp.so")
 
 GLP_MATH_FP32, GLP_MATH_TF32, GLP_MATH_BF16 = 0, 1, 2
 MATH = {"fp32": GLP_MATH_FP32, "tf32": GLP_MATH_TF32, "bf16": GLP_MATH_BF16}

@@ -84,6 +84,7 @@ struct PassPlan {
   int regs = 0, ctas_runtime = 0;
   int a_tma = 0, krow = 128;        // A operand by im2col TMA; K-block row width (bytes)
   int cg = 1, m_units = 0;          // CTAs per MMA (tcgen05 cta_group); work units along M
+  int ksub = 1;                     // k-blocks per pipeline stage
 };
 
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -249,6 +250,8 @@ struct glp_plan_s {
   size_t ws_fwd = 0, ws_dgrad = 0, ws_wgrad = 0, ws_bwd = 0;
   double plan_us = 0;
   int allow_cg2 = 1;   // GLP_CTA_GROUP=1 in the environment forces single-CTA MMAs (A/B runs)
+  int allow_ksub2 = 1; // GLP_KSUB=1 forces one k-block per pipeline stage (A/B runs)
+  int ksub_max = 4;    // GLP_KSUB=k caps the k-blocks per stage
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
 
@@ -318,8 +321,18 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   }
   const int a_bytes = mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow;
   const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
-  const int stage_bytes = a_bytes + pp.bn_smem * b_row;
   const int budget = 232448 - 1024 - 512;
+  // k-blocks per pipeline stage: as many (<= 4) as keep >= 3 stages in the ring.  One
+  // full/empty round trip of the single MMA-issuing warp costs ~250-700 cycles whatever the stage
+  // size (tools/sync_probe*.cu, GLP_DEBUG_SKIP=15 runs), more than the tensor work of one small-N
+  // k-block, so a stage must carry several k-blocks (TMA path only; cp.async fills one).
+  pp.ksub = 1;
+  const int kb_bytes = a_bytes + pp.bn_smem * b_row;
+  if (pp.a_tma && P.allow_ksub2)
+    while (pp.ksub < P.ksub_max && budget / ((pp.ksub + 1) * kb_bytes) >= 3 &&
+           pp.kb_per_split >= 2 * (pp.ksub + 1))
+      ++pp.ksub;
+  const int stage_bytes = pp.ksub * kb_bytes;
   pp.stages = std::min(8, budget / stage_bytes);
   if (const char *e = getenv("GLP_DEBUG_STAGES"))   // diagnostics: fewer ring stages
     pp.stages = std::max(2, std::min(pp.stages, atoi(e)));
@@ -426,6 +439,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   p.bn = pp.bn;
   p.bn_smem = pp.bn_smem;
   p.stages = pp.stages;
+  p.ksub = pp.ksub;
   p.tmem_cols = pp.tmem_cols;
   p.acc_cols = pp.acc_cols;
   p.part_ld = pp.n_tiles * pp.bn;
@@ -798,6 +812,10 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->sm_count = prop.multiProcessorCount;
   P->s_override = S;
   if (const char *e = getenv("GLP_CTA_GROUP")) P->allow_cg2 = (atoi(e) != 1);
+  if (const char *e = getenv("GLP_KSUB")) {
+    P->ksub_max = std::max(1, std::min(4, atoi(e)));
+    P->allow_ksub2 = P->ksub_max > 1;
+  }
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 15;
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to

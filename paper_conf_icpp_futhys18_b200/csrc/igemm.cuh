@@ -31,6 +31,9 @@
 namespace glp {
 
 constexpr int IGEMM_THREADS = 288;
+#ifndef GLP_TMA_WARP
+#define GLP_TMA_WARP 4
+#endif
 
 template <int ELEM, int KROW>
 struct TileCfg {
@@ -104,7 +107,9 @@ __global__ void __launch_bounds__(288, 1)
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
   const uint32_t b_bytes = (uint32_t)p.bn_smem * C::b_row_bytes(MODE);
-  const uint32_t stage_bytes = A_BYTES + b_bytes;
+  // a stage holds p.ksub consecutive k-blocks: [A_0 .. A_ks-1 | B_0 .. B_ks-1] (ksub = 2 halves
+  // the barrier round trips per MMA; the cp.async path always uses ksub = 1)
+  const uint32_t stage_bytes = (uint32_t)p.ksub * (A_BYTES + b_bytes);
   const uint32_t bars = base + (uint32_t)p.stages * stage_bytes;
   const int S_ = p.stages;
   auto full = [&](int s) { return bars + 8u * s; };
@@ -115,9 +120,13 @@ __global__ void __launch_bounds__(288, 1)
   volatile uint32_t *tmem_slot_ptr =
       reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // warp index broadcast from lane 0: the compiler then knows every role branch below is
+  // warp-uniform and keeps loop state of the single-warp roles in the uniform datapath
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0);
+  const int lane = threadIdx.x & 31;
   const bool a_tma = (CG == 2) || p.a_tma != 0;
-  const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
+  // cluster of 2 CTAs along x: the rank in the pair is blockIdx.x & 1 (uniform by construction)
+  const uint32_t rank = (CG == 2) ? (blockIdx.x & 1u) : 0u;
   const bool leader = rank == 0;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S_; ++s) {
@@ -145,7 +154,7 @@ __global__ void __launch_bounds__(288, 1)
   if (CG == 2) cluster_sync();
   else __syncthreads();
   tc_fence_after();
-  const uint32_t tmem_base = *tmem_slot_ptr;
+  const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);   // warp-uniform
 
   // work units: CG1 = one 128-row tile; CG2 = a pair of 128-row tiles (one per CTA)
   const int total_tiles = p.m_tiles * p.n_tiles * p.splits;   // p.m_tiles counts units along M
@@ -157,55 +166,37 @@ __global__ void __launch_bounds__(288, 1)
     // ===================================== producers =======================================
     const int pt = threadIdx.x - 128;
     if (a_tma) {
-      if (warp == 4) {   // one converged warp; each TMA / arrive is issued by an elected lane
+      if (warp == GLP_TMA_WARP) {   // one converged warp; each TMA / arrive is issued by an elected lane
         int rs = 0;          // ring slot and its phase, advanced incrementally
         uint32_t rph = 0;
+        uint32_t stg_addr = base;   // shared address of ring slot rs
+        const int KS = p.ksub, cbs = g.cbs, KW = g.kw;
+        const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+        const uint32_t kb_tx = (la ? A_BYTES : 0u) + (lb ? b_bytes : 0u);
+        const uint32_t sB_off = (uint32_t)KS * A_BYTES;
         for (int tile = unit0; tile < total_tiles; tile += ustep) {
           int m_tile, n_tile, split;
           decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
           const int m0 = (m_tile * CG + (int)rank) * C::BM, n0 = n_tile * p.bn;
           const int nb0 = n0 + (int)rank * p.bn_smem;   // this CTA's part of the B tile
+          int kb0 = 0, kb1 = p.kb_total;
+          if (MODE == MODE_WGRAD) {
+            kb0 = split * p.kb_per_split;
+            kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+          }
+          // per-tile geometry of the A gather
+          uint32_t n_t = 0;
+          int h_t = 0, w_t = 0;            // fwd/dgrad: base pixel of the tile's first row
+          constexpr int NA = (MODE == MODE_WGRAD) ? 128 / C::EPA : 1;   // MN atoms (wgrad)
+          int ac[NA];
+          uint16_t akh[NA], akw[NA];
           if (MODE != MODE_WGRAD) {
-            // base pixel of the tile's first output pixel; the TMA walks 128 pixels from there
-            uint32_t n, rem, oh, ow;
-            g.div_hw.divmod((uint32_t)m0, n, rem);
+            uint32_t rem, oh, ow;
+            g.div_hw.divmod((uint32_t)m0, n_t, rem);
             g.div_w.divmod(rem, oh, ow);
-            const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
-            int t = 0, cb = 0;
-            for (int kb = 0; kb < p.kb_total; ++kb, ring_next(rs, rph, S_)) {
-              const int s = rs;
-              const uint32_t ph = rph;
-              mbar_wait(empty(s), ph ^ 1u);
-              const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
-              uint32_t kh, kw;
-              g.div_kw.divmod((uint32_t)t, kh, kw);
-              if (CG == 1) {
-                const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
-                mbar_arrive_expect_tx_e(full(s), (la ? A_BYTES : 0u) + (lb ? b_bytes : 0u));
-                if (la)
-                  tma_load_im2col_4d_e(sA, &tmapA, full(s), cb * C::BK, w0, h0, (int)n,
-                                       (uint16_t)kw, (uint16_t)kh);
-                if (lb) tma_load_2d_e(sB, &tmapB, full(s), kb * C::BK, nb0);
-              } else {
-                const uint32_t fullL = mapa_shared(full(s), 0);
-                if (leader) mbar_arrive_expect_tx_e(full(s), 2u * (A_BYTES + b_bytes));
-                // the peer only adds bytes (complete_tx) to the leader's barrier; no arrival —
-                // a release-scoped remote arrive here would fence this thread's in-flight TMA
-                tma_load_im2col_4d_cg2_e(sA, &tmapA, fullL, cb * C::BK, w0, h0, (int)n,
-                                         (uint16_t)kw, (uint16_t)kh);
-                tma_load_2d_cg2_e(sB, &tmapB, fullL, kb * C::BK, nb0);
-              }
-              if (++cb == g.cbs) {
-                cb = 0;
-                ++t;
-              }
-            }
+            h_t = (int)oh * g.im_sh - g.im_ph;
+            w_t = (int)ow * g.im_sw - g.im_pw;
           } else {
-            const int kb0 = split * p.kb_per_split;
-            const int kb1 = min(kb0 + p.kb_per_split, p.kb_total);
-            constexpr int NA = 128 / C::EPA;   // MN atoms of the A tile
-            int ac[NA];
-            uint16_t akh[NA], akw[NA];
 #pragma unroll
             for (int a = 0; a < NA; ++a) {
               uint32_t t, c;
@@ -222,36 +213,82 @@ __global__ void __launch_bounds__(288, 1)
                 akw[a] = 0;
               }
             }
-            for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
-              const int s = rs;
-              const uint32_t ph = rph;
-              mbar_wait(empty(s), ph ^ 1u);
-              const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
-              uint32_t n, rem, oh, ow;
-              g.div_hw.divmod((uint32_t)(kb * C::BKP), n, rem);
-              g.div_w.divmod(rem, oh, ow);
-              const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
-              if (CG == 1) {
-                mbar_arrive_expect_tx_e(full(s), A_BYTES + b_bytes);
-#pragma unroll
-                for (int a = 0; a < NA; ++a)
-                  tma_load_im2col_4d_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, full(s), ac[a], w0,
-                                       h0, (int)n, akw[a], akh[a]);
-                for (int a = 0; a < p.bn_smem / C::EPA; ++a)
-                  tma_load_2d_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), nb0 + a * C::EPA,
-                                kb * C::BKP);
+          }
+          int kh = 0, kw = 0, cb = 0;       // fwd/dgrad K position (tap (kh, kw), channel block)
+          for (int kbs = kb0; kbs < kb1; kbs += KS) {
+            const int s = rs;
+            mbar_wait(empty(s), rph ^ 1u);
+            const int nsub = min(KS, kb1 - kbs);
+            const uint32_t stg = stg_addr;
+            const uint32_t tx = (uint32_t)nsub * kb_tx;
+            uint32_t bar = full(s);
+            if (CG == 1) {
+              mbar_arrive_expect_tx_e(bar, tx);
+            } else {
+              // only the leader arrives (expect_tx = both CTAs' bytes); the peer's TMAs complete
+              // bytes on the leader's barrier — a release-scoped remote arrive here would fence
+              // this thread's in-flight TMA
+              if (leader) mbar_arrive_expect_tx_e(bar, 2u * tx);
+              bar = mapa_shared(bar, 0);
+            }
+            if (++rs == S_) {
+              rs = 0;
+              rph ^= 1u;
+              stg_addr = base;
+            } else {
+              stg_addr += stage_bytes;
+            }
+#pragma unroll 1
+            for (int sub = 0; sub < nsub; ++sub) {
+              const int kb = kbs + sub;
+              const uint32_t sA = stg + (uint32_t)sub * A_BYTES;
+              const uint32_t sB = stg + sB_off + (uint32_t)sub * b_bytes;
+              if (MODE != MODE_WGRAD) {
+                if (la) {
+                  if (CG == 1)
+                    tma_load_im2col_4d_e(sA, &tmapA, bar, cb * C::BK, w_t, h_t, (int)n_t,
+                                         (uint16_t)kw, (uint16_t)kh);
+                  else
+                    tma_load_im2col_4d_cg2_e(sA, &tmapA, bar, cb * C::BK, w_t, h_t, (int)n_t,
+                                             (uint16_t)kw, (uint16_t)kh);
+                }
+                if (lb) {
+                  if (CG == 1) tma_load_2d_e(sB, &tmapB, bar, kb * C::BK, nb0);
+                  else tma_load_2d_cg2_e(sB, &tmapB, bar, kb * C::BK, nb0);
+                }
+                if (++cb == cbs) {
+                  cb = 0;
+                  if (++kw == KW) {
+                    kw = 0;
+                    ++kh;
+                  }
+                }
               } else {
-                const uint32_t fullL = mapa_shared(full(s), 0);
-                if (leader) mbar_arrive_expect_tx_e(full(s), 2u * (A_BYTES + b_bytes));
-                // the peer only adds bytes (complete_tx) to the leader's barrier; no arrival —
-                // a release-scoped remote arrive here would fence this thread's in-flight TMA
+                uint32_t n, rem, oh, ow;
+                g.div_hw.divmod((uint32_t)(kb * C::BKP), n, rem);
+                g.div_w.divmod(rem, oh, ow);
+                const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
+                if (la) {
 #pragma unroll
-                for (int a = 0; a < NA; ++a)
-                  tma_load_im2col_4d_cg2_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, fullL, ac[a],
-                                           w0, h0, (int)n, akw[a], akh[a]);
-                for (int a = 0; a < p.bn_smem / C::EPA; ++a)
-                  tma_load_2d_cg2_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, fullL,
-                                    nb0 + a * C::EPA, kb * C::BKP);
+                  for (int a = 0; a < NA; ++a) {
+                    if (CG == 1)
+                      tma_load_im2col_4d_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, bar, ac[a], w0,
+                                           h0, (int)n, akw[a], akh[a]);
+                    else
+                      tma_load_im2col_4d_cg2_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, bar, ac[a],
+                                               w0, h0, (int)n, akw[a], akh[a]);
+                  }
+                }
+                if (lb) {
+                  for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
+                    if (CG == 1)
+                      tma_load_2d_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, bar, nb0 + a * C::EPA,
+                                    kb * C::BKP);
+                    else
+                      tma_load_2d_cg2_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, bar,
+                                        nb0 + a * C::EPA, kb * C::BKP);
+                  }
+                }
               }
             }
           }
@@ -405,42 +442,58 @@ __global__ void __launch_bounds__(288, 1)
       constexpr uint32_t mn = (MODE == MODE_WGRAD) ? 1u : 0u;
       const uint32_t idesc = make_idesc(fmt, mn, mn, 128u * CG, (uint32_t)p.bn);
       constexpr int KSTEPS = (MODE == MODE_WGRAD) ? C::BKP / C::UMMA_K : C::BK / C::UMMA_K;
+      constexpr int DSTEP = (int)(((MODE == MODE_WGRAD) ? C::MN_KSTEP : 32u) >> 4);
+      // Descriptors of slot 0 (sub-block 0, k 0); the start-address field (bits [0,14), bytes/16)
+      // of a shared address < 256 KB never carries, so later operands are plain 64-bit adds.
+      uint64_t da0, db0;
+      if (MODE == MODE_WGRAD) {
+        da0 = make_sdesc(base, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
+        db0 = make_sdesc(base + (uint32_t)p.ksub * A_BYTES, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
+      } else {
+        da0 = make_sdesc(base, 16u, C::K_SBO, C::K_LAYOUT);
+        db0 = make_sdesc(base + (uint32_t)p.ksub * A_BYTES, 16u, C::K_SBO, C::K_LAYOUT);
+      }
+      const uint64_t stage16 = stage_bytes >> 4, b16 = b_bytes >> 4;
+      const int KS = p.ksub, kb_total = p.kb_total, kb_per_split = p.kb_per_split;
+      const bool skip_mma = (p.dbg_skip & 4) != 0;
       int rs = 0;
       uint32_t rph = 0, it = 0;
+      uint64_t da = da0, db = db0;   // descriptors of ring slot rs
       for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
         int m_tile, n_tile, split;
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
-        int kb0 = 0, kb1 = p.kb_total;
+        int kb0 = 0, kb1 = kb_total;
         if (MODE == MODE_WGRAD) {
-          kb0 = split * p.kb_per_split;
-          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+          kb0 = split * kb_per_split;
+          kb1 = min(kb0 + kb_per_split, kb_total);
         }
         const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
         mbar_wait(tempty(a), aph ^ 1u);
         tc_fence_after();
         const uint32_t d = tmem_base + a * (uint32_t)p.acc_cols;
-        for (int kb = kb0; kb < kb1; ++kb, ring_next(rs, rph, S_)) {
-          const int s = rs;
-          const uint32_t ph = rph;
-          mbar_wait(full(s), ph);
+        uint32_t acc = 0;
+        for (int kbs = kb0; kbs < kb1; kbs += KS) {
+          mbar_wait(full(rs), rph);
           tc_fence_after();
-          const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
-          const int ksteps = (p.dbg_skip & 4) ? (kb == kb0 ? 1 : 0) : KSTEPS;
+          const int nsub = min(KS, kb1 - kbs);
 #pragma unroll
-          for (int k = 0; k < KSTEPS; ++k) {
-            if (k >= ksteps) break;
-            uint64_t ad, bd;
-            if (MODE == MODE_WGRAD) {
-              ad = make_sdesc(sA + (uint32_t)k * C::MN_KSTEP, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
-              bd = make_sdesc(sB + (uint32_t)k * C::MN_KSTEP, C::MN_LBO, C::MN_GROUP, C::MN_LAYOUT);
-            } else {
-              ad = make_sdesc(sA + (uint32_t)k * 32u, 16u, C::K_SBO, C::K_LAYOUT);
-              bd = make_sdesc(sB + (uint32_t)k * 32u, 16u, C::K_SBO, C::K_LAYOUT);
-            }
-            const uint32_t acc = (kb > kb0 || k > 0) ? 1u : 0u;
-            mma_e<(ELEM == 2) ? 0 : 1, CG>(d, ad, bd, idesc, acc);
+          for (int sub = 0; sub < 4; ++sub) {
+            if (sub >= nsub) break;
+            if (!skip_mma || acc == 0)
+              mma_kblock_e<(ELEM == 2) ? 0 : 1, CG, KSTEPS, DSTEP>(
+                  d, da + (uint64_t)(sub * (A_BYTES >> 4)), db + (uint64_t)sub * b16, idesc, acc);
+            acc = 1;
           }
-          mma_commit_e<CG>(empty(s));
+          mma_commit_e<CG>(empty(rs));
+          if (++rs == S_) {
+            rs = 0;
+            rph ^= 1u;
+            da = da0;
+            db = db0;
+          } else {
+            da += stage16;
+            db += stage16;
+          }
         }
         mma_commit_e<CG>(tfull(a));
       }

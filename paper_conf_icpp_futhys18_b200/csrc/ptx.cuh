@@ -167,6 +167,49 @@ __device__ __forceinline__ void mma_e(uint32_t d_tmem, uint64_t adesc, uint64_t 
   else GLP_MMA_E("tf32", "2");
 #undef GLP_MMA_E
 }
+// All NSTEP tcgen05.mma of one k-block in one instruction block (one elect, descriptors advanced
+// by STEP 16-byte units per MMA inside the block): the MMA-issuing warp's loop is latency-bound,
+// so the per-MMA overhead of separate blocks (re-elect, uniform-register broadcasts) counts.
+// `accumulate` applies to the first MMA only; the rest always accumulate.
+template <int KIND, int CG, int NSTEP, int STEP>
+__device__ __forceinline__ void mma_kblock_e(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
+                                             uint32_t idesc, uint32_t accumulate) {
+  static_assert(NSTEP == 2 || NSTEP == 4, "k-block = 2 or 4 MMAs");
+#define GLP_MMA_HEAD                                                                    \
+  "{\n\t.reg .pred P_e, p, q;\n\t.reg .b64 a1, b1;\n\t"                                 \
+  "elect.sync _|P_e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\tsetp.eq.b32 q, %3, %3;\n\t"
+#define GLP_MMA_I(CGS, KINDS, A, B, P)                                                  \
+  "@P_e tcgen05.mma.cta_group::" CGS ".kind::" KINDS " [%0], " A ", " B ", %3, " P ";\n\t"
+#define GLP_MMA_ADV(A0, B0) "add.s64 a1, " A0 ", %5;\n\tadd.s64 b1, " B0 ", %5;\n\t"
+#define GLP_MMA_K2(CGS, KINDS)                                                          \
+  asm volatile(GLP_MMA_HEAD GLP_MMA_I(CGS, KINDS, "%1", "%2", "p") GLP_MMA_ADV("%1", "%2") \
+               GLP_MMA_I(CGS, KINDS, "a1", "b1", "q") "}"                               \
+               ::"r"(d_tmem), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate),      \
+               "n"(STEP) : "memory")
+#define GLP_MMA_K4(CGS, KINDS)                                                          \
+  asm volatile(GLP_MMA_HEAD GLP_MMA_I(CGS, KINDS, "%1", "%2", "p") GLP_MMA_ADV("%1", "%2") \
+               GLP_MMA_I(CGS, KINDS, "a1", "b1", "q") GLP_MMA_ADV("a1", "b1")           \
+               GLP_MMA_I(CGS, KINDS, "a1", "b1", "q") GLP_MMA_ADV("a1", "b1")           \
+               GLP_MMA_I(CGS, KINDS, "a1", "b1", "q") "}"                               \
+               ::"r"(d_tmem), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate),      \
+               "n"(STEP) : "memory")
+  if (NSTEP == 2) {
+    if (KIND == 0 && CG == 1) GLP_MMA_K2("1", "f16");
+    else if (KIND == 0) GLP_MMA_K2("2", "f16");
+    else if (CG == 1) GLP_MMA_K2("1", "tf32");
+    else GLP_MMA_K2("2", "tf32");
+  } else {
+    if (KIND == 0 && CG == 1) GLP_MMA_K4("1", "f16");
+    else if (KIND == 0) GLP_MMA_K4("2", "f16");
+    else if (CG == 1) GLP_MMA_K4("1", "tf32");
+    else GLP_MMA_K4("2", "tf32");
+  }
+#undef GLP_MMA_K4
+#undef GLP_MMA_K2
+#undef GLP_MMA_ADV
+#undef GLP_MMA_I
+#undef GLP_MMA_HEAD
+}
 template <int CG>
 __device__ __forceinline__ void mma_commit_e(uint32_t bar) {
   if (CG == 1)

@@ -204,6 +204,28 @@ int choose_bn(int n) {
   return (int)rup(cdiv(n, nt), 16);
 }
 
+// N tile of the fwd / dgrad GEMMs (no split: the per-element K order, hence every output bit, is
+// independent of the tile).  Models the persistent grid's last-round quantisation: time ~
+// rounds * max(MMA cycles of a k-block ~ 2*bn, per-k-block issue floor); fewer N tiles (less A
+// re-reading) win ties.
+int choose_bn_mn(int n, long long M, int cg, int sm_count) {
+  const long long m_units = cdiv(M, 128LL * cg);
+  const double slots = std::max(1, sm_count / cg);
+  int best = choose_bn(n);
+  double best_c = 1e300;
+  for (int nt = (int)cdiv(n, 256); nt <= 4; ++nt) {
+    const int bn = (int)rup(cdiv(n, nt), 16);
+    if ((int)cdiv(n, bn) != nt) continue;
+    const double rounds = std::ceil((double)m_units * nt / slots);
+    const double c = rounds * std::max(2.0 * bn, 224.0) * (1.0 + 0.03 * (nt - 1));
+    if (c < best_c) {
+      best_c = c;
+      best = bn;
+    }
+  }
+  return best;
+}
+
 // Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
 // (constants, never the queried device or S), so the fp32 summation order is a function of the
 // shape alone (convergence invariance, P264).
@@ -252,6 +274,7 @@ struct glp_plan_s {
   int allow_cg2 = 1;   // GLP_CTA_GROUP=1 in the environment forces single-CTA MMAs (A/B runs)
   int allow_ksub2 = 1; // GLP_KSUB=1 forces one k-block per pipeline stage (A/B runs)
   int ksub_max = 4;    // GLP_KSUB=k caps the k-blocks per stage
+  int bn_model = 0;    // GLP_BN_MODEL=1: quantisation-model N tile for fwd/dgrad (measured: no gain)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
 
@@ -301,14 +324,16 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     pp.bn_smem = (int)rup(pp.bn, EPA);
   }
   pp.m_tiles = (int)cdiv(pp.M, 128);
-  pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
   // CTA pairs (tcgen05 cta_group::2, M = 256): each SM loads half of B.  Needs the TMA A path,
   // at least two row tiles, and (MN-major B) half tiles that are whole swizzle atoms.
   pp.cg = 1;
-  if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && mode != MODE_WGRAD) {
-    pp.cg = 2;
-    pp.bn_smem = pp.bn / 2;
+  if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && mode != MODE_WGRAD) pp.cg = 2;
+  if (mode != MODE_WGRAD && P.bn_model) {
+    pp.bn = choose_bn_mn(pp.Ng, pp.M, pp.cg, P.sm_count);
+    pp.bn_smem = pp.bn;
   }
+  if (pp.cg == 2) pp.bn_smem = pp.bn / 2;
+  pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
   pp.m_units = (int)cdiv(pp.m_tiles, pp.cg);
   if (mode == MODE_WGRAD) {
     pp.splits = choose_splits(pp.m_units * pp.n_tiles, pp.kb_total, pp.bn,
@@ -534,12 +559,15 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
   const glp_conv_desc_s &d = P.d;
   if (P.s2d) {
     const int S = P.s2d;
-    const size_t smem = (size_t)S * d.C * d.W * sizeof(float) + (size_t)P.Cpx * sizeof(int);
+    const size_t smem = (size_t)S * d.C * d.W * sizeof(float);
     dim3 grid((unsigned)P.dxg.H, (unsigned)d.N);
+    const int quads = P.Cpx / 4;   // the block is a whole number of channel-quad groups
+    const int threads = quads <= 256 ? quads * (256 / quads) : 0;
+    if (threads < 32) return fail(GLP_ERR_NOT_SUPPORTED, "space-to-depth channel pitch too large");
     if (P.elem == 2)
-      pack_s2d<2><<<grid, 256, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
+      pack_s2d<2><<<grid, threads, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
     else
-      pack_s2d<4><<<grid, 256, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
+      pack_s2d<4><<<grid, threads, smem, st>>>(x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx);
     GLP_LAUNCH_CHECK("pack_s2d");
     return GLP_OK;
   }
@@ -816,6 +844,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->ksub_max = std::max(1, std::min(4, atoi(e)));
     P->allow_ksub2 = P->ksub_max > 1;
   }
+  if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 15;
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to

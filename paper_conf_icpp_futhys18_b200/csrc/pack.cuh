@@ -134,49 +134,57 @@ template <int ELEM>
 __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
                                                 int C, int H, int W, int S, int P, int Hs, int Ws,
                                                 int Cps) {
-  extern __shared__ float smem_s2d[];
-  // [S][C][W] source rows, then a per-output-channel table: (row offset into rows, dw) or -1.
-  float *rows = smem_s2d;
-  int *tab = reinterpret_cast<int *>(smem_s2d + S * C * W);
+  extern __shared__ float rows[];   // [S*C][W] source rows (row r = dh*C + c)
   const int hs = blockIdx.x, n = blockIdx.y;
-  const int cs = S * S * C;
-  for (int cc = threadIdx.x; cc < Cps; cc += blockDim.x) {
-    int e = -1;
-    if (cc < cs) {
-      const int c = cc % C, dd = cc / C, dh = dd / S, dw = dd % S;
-      e = ((dh * C + c) * W) | (dw << 24);   // W*S*C < 2^24 (host-checked smem bound)
-    }
-    tab[cc] = e;
-  }
-  const size_t xb = (size_t)n * C * H;
-  for (int dh = 0; dh < S; ++dh) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarps = blockDim.x >> 5;
+  // one warp per source row, 8 independent coalesced loads in flight per lane (no per-element
+  // index division: the row is fixed per warp iteration)
+  // (a trailing partial warp, blockDim % 32 != 0, takes no rows)
+  for (int r = warp; warp < nwarps && r < S * C; r += nwarps) {
+    const int dh = r / C, c = r - dh * C;
     const int ih = S * hs + dh - P;
     const bool rin = ih >= 0 && ih < H;
-    for (int c = 0; c < C; ++c) {
-      const float *src = x + ((xb + (size_t)c * H + (rin ? ih : 0)) * W);
-      float *d = rows + (dh * C + c) * W;
-      for (int w = threadIdx.x; w < W; w += blockDim.x) d[w] = rin ? __ldg(src + w) : 0.f;
+    const float *src = x + (((size_t)n * C + c) * H + (rin ? ih : 0)) * W;
+    float *d = rows + r * W;
+    for (int w0 = 0; w0 < W; w0 += 256) {
+      float v[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int w = w0 + lane + 32 * k;
+        v[k] = (rin && w < W) ? __ldg(src + w) : 0.f;
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int w = w0 + lane + 32 * k;
+        if (w < W) d[w] = v[k];
+      }
+    }
+  }
+  // output: thread -> fixed channel quad q (blockDim is a multiple of Cps/4), pixels strided
+  const int quads = Cps >> 2;
+  const int q = threadIdx.x % quads, wstep = blockDim.x / quads;
+  int roff[4], dws[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int cc = 4 * q + u;
+    roff[u] = -1;
+    dws[u] = 0;
+    if (cc < S * S * C) {
+      const int c = cc % C, dd = cc / C, dh = dd / S, dw = dd - dh * S;
+      roff[u] = (dh * C + c) * W;
+      dws[u] = dw - P;
     }
   }
   __syncthreads();
-  const int quads = Cps >> 2;
-  // thread -> (output pixel ws, channel quad q); quads is a power-of-two-free small count, so the
-  // split is done with one division per 4 outputs
-  for (int i = threadIdx.x; i < Ws * quads; i += blockDim.x) {
-    const int ws = i / quads, q = i - ws * quads;
-    const int base_w = S * ws - P;
+  const size_t obase = ((size_t)n * Hs + hs) * Ws;
+  for (int ws = threadIdx.x / quads; ws < Ws; ws += wstep) {
     float v[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      const int e = tab[4 * q + u];
-      float val = 0.f;
-      if (e >= 0) {
-        const int iw = base_w + (e >> 24);
-        if (iw >= 0 && iw < W) val = rows[(e & 0xFFFFFF) + iw];
-      }
-      v[u] = val;
+      const int iw = S * ws + dws[u];
+      v[u] = (roff[u] >= 0 && iw >= 0 && iw < W) ? rows[roff[u] + iw] : 0.f;
     }
-    PackOut<ELEM>::store4(dst, (((size_t)n * Hs + hs) * Ws + ws) * Cps + 4 * q, v[0], v[1], v[2], v[3]);
+    PackOut<ELEM>::store4(dst, (obase + ws) * Cps + 4 * q, v[0], v[1], v[2], v[3]);
   }
 }
 

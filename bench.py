@@ -48,6 +48,9 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--no-graph", action="store_true",
+                   help="launch every step eagerly (default on 1 GPU: the step is captured once "
+                        "into a CUDA graph and replayed)")
     return p.parse_args()
 
 
@@ -185,6 +188,7 @@ def run_glp(args, ws, rank, local):
     stream = torch.cuda.current_stream()
 
     def step(ev=None):
+        stream = torch.cuda.current_stream()   # the capture stream while a graph is recorded
         # forward, layer order
         for i, s in enumerate(states):
             c = s.conv
@@ -221,8 +225,17 @@ def run_glp(args, ws, rank, local):
     torch.cuda.synchronize()
     if G > 1:
         dist.barrier()
+    use_graph = (not args.no_graph) and G == 1
     evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(6)] for _ in states]
            for _ in range(args.steps)]
+    if use_graph:
+        # The whole step (every pack, GEMM and reduction launch of all layers) recorded once and
+        # replayed: no per-launch host work and minimal gaps between kernels.
+        g_step = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_step):
+            step()
+        for _ in range(max(1, args.warmup)):
+            g_step.replay()
     clocks = ClockSampler(local) if rank == 0 else None
     if clocks:
         clocks.start()
@@ -232,7 +245,10 @@ def run_glp(args, ws, rank, local):
         dist.barrier()
     t0.record(stream)
     for k in range(args.steps):
-        step(evs[k])
+        if use_graph:
+            g_step.replay()
+        else:
+            step(evs[k])
     t1.record(stream)
     torch.cuda.synchronize()
     if G > 1:
@@ -247,7 +263,14 @@ def run_glp(args, ws, rank, local):
     images_per_step = n_local[0] * G
     value = images_per_step / (ms_per_step / 1e3)
 
-    # per-kernel live timings (CUDA events on the launching stream, inside the timed region)
+    if use_graph:
+        # per-kernel attribution: events cannot time nodes inside a graph, so the same step runs
+        # K more times eagerly with CUDA events around each GEMM on the launching stream (kernel
+        # durations do not depend on how the launches were issued)
+        for k in range(args.steps):
+            step(evs[k])
+        torch.cuda.synchronize()
+    # per-kernel live timings (CUDA events on the launching stream)
     kern = []
     for i, s in enumerate(states):
         for name, a, b in (("fwd", 0, 1), ("bwd_data", 2, 3), ("bwd_filter", 4, 5)):
@@ -337,6 +360,7 @@ def run_glp(args, ws, rank, local):
         "clocks": clk,
         "e2e": e2e,
         "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
+        "launch": "cuda_graph" if use_graph else "eager",
     }
     print(json.dumps(line), flush=True)
     if G > 1:

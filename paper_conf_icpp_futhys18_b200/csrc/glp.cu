@@ -546,9 +546,9 @@ glp_status_t run_pack_w_fwd(glp_plan_s &P, const float *w, uint8_t *ws, cudaStre
     else
       pack_w_fwd_s2d<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad);
   } else if (P.elem == 2) {
-    pack_w_fwd<2><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
+    pack_w_fwd<2><<<dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
   } else {
-    pack_w_fwd<4><<<ew_grid(wn), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
+    pack_w_fwd<4><<<dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co), 256, 0, st>>>(w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad);
   }
   GLP_LAUNCH_CHECK("pack_w_fwd");
   return GLP_OK;
@@ -577,12 +577,11 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
 glp_status_t run_pack_w_dgrad(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   void *wtpk = ws + P.off_wpk;
-  const size_t wn = (size_t)d.C * P.dgrad.Kpad;
   const int flip = P.dgrad.a_tma;  // the im2col-TMA dgrad walks taps flipped
   if (P.elem == 2)
-    pack_w_dgrad<2><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
+    pack_w_dgrad<2><<<dim3((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
   else
-    pack_w_dgrad<4><<<ew_grid(wn), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
+    pack_w_dgrad<4><<<dim3((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C), 256, 0, st>>>(w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip);
   GLP_LAUNCH_CHECK("pack_w_dgrad");
   return GLP_OK;
 }

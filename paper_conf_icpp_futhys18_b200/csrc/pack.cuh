@@ -209,35 +209,32 @@ __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ o
 }
 
 // W [Co][C][Kh][Kw] -> forward B operand Wp[co][tap*Cp + c] with row length Kpad (zero padded).
+// grid (ceil(Kpad/256), Co): one element per thread, 32-bit index math (the old grid-stride form
+// spent most of its time in 64-bit divisions).
 template <int ELEM>
-__global__ void pack_w_fwd(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
-                           int taps, int Cp, int Kpad) {
-  const size_t total = (size_t)Co * Kpad;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
-       i += (size_t)gridDim.x * blockDim.x) {
-    const int co = (int)(i / Kpad), k = (int)(i % Kpad);
-    const int t = k / Cp, c = k % Cp;
-    float v = 0.f;
-    if (t < taps && c < C) v = __ldg(w + ((size_t)co * C + c) * taps + t);
-    PackOut<ELEM>::store1(out, i, v);
-  }
+__global__ void __launch_bounds__(256) pack_w_fwd(const float *__restrict__ w, void *__restrict__ out,
+                                                  int Co, int C, int taps, int Cp, int Kpad) {
+  const int co = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= Kpad) return;
+  const int t = k / Cp, c = k - t * Cp;
+  const float v = (t < taps && c < C) ? __ldg(w + ((size_t)co * C + c) * taps + t) : 0.f;
+  PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v);
 }
 
 // W [Co][C][Kh][Kw] -> backward-data B operand Wt[ci][tap*Cop + co] (row length Kpad).
 // flip = 1: tap index reversed (tap' = taps-1-tap, i.e. (Kh-1-kh, Kw-1-kw)) for the im2col-TMA
 // dgrad, which walks dy from the window's top-left corner.
 template <int ELEM>
-__global__ void pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
-                             int taps, int Cop, int Kpad, int flip) {
-  const size_t total = (size_t)C * Kpad;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
-       i += (size_t)gridDim.x * blockDim.x) {
-    const int ci = (int)(i / Kpad), k = (int)(i % Kpad);
-    const int t = k / Cop, co = k % Cop;
-    float v = 0.f;
-    if (t < taps && co < Co) v = __ldg(w + ((size_t)co * C + ci) * taps + (flip ? taps - 1 - t : t));
-    PackOut<ELEM>::store1(out, i, v);
-  }
+__global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out,
+                                                    int Co, int C, int taps, int Cop, int Kpad,
+                                                    int flip) {
+  const int ci = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= Kpad) return;
+  const int t = k / Cop, co = k - t * Cop;
+  const float v = (t < taps && co < Co)
+                      ? __ldg(w + ((size_t)co * C + ci) * taps + (flip ? taps - 1 - t : t))
+                      : 0.f;
+  PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
 }
 
 }  // namespace glp

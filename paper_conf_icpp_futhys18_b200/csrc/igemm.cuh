@@ -154,6 +154,9 @@ __global__ void __launch_bounds__(288, 1)
   if (CG == 2) cluster_sync();
   else __syncthreads();
   tc_fence_after();
+  // prologue done (barriers, TMEM, descriptor prefetch): wait for the previous kernel's results
+  // before touching global memory
+  pdl_wait();
   const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);   // warp-uniform
 
   // work units: CG1 = one 128-row tile; CG2 = a pair of 128-row tiles (one per CTA)
@@ -561,6 +564,8 @@ __global__ void __launch_bounds__(288, 1)
       }
     }
   }
+  // all tiles done: the next kernel may start launching into the teardown
+  pdl_launch_dependents();
   tc_fence_before();
   if (CG == 2) cluster_sync();
   else __syncthreads();

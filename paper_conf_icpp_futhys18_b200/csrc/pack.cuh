@@ -57,6 +57,8 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
                                                          unsigned int *__restrict__ tickets,
                                                          int n_tickets) {
   __shared__ float tile[32][PACK_PT + 1];
+  pdl_launch_dependents();
+  pdl_wait();
   const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * PACK_PT;
   // arm the completion tickets of the deterministic db reduction that consumes db_part
   if (tickets != nullptr && (blockIdx.x | blockIdx.y | blockIdx.z) == 0)
@@ -110,6 +112,8 @@ template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__restrict__ src,
                                                                void *__restrict__ dst, int N, int C,
                                                                int HW, int Cp) {
+  pdl_launch_dependents();
+  pdl_wait();
   const size_t total = (size_t)N * HW;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
        i += (size_t)gridDim.x * blockDim.x) {
@@ -135,6 +139,8 @@ __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, voi
                                                 int C, int H, int W, int S, int P, int Hs, int Ws,
                                                 int Cps) {
   extern __shared__ float rows[];   // [S*C][W] source rows (row r = dh*C + c)
+  pdl_launch_dependents();
+  pdl_wait();
   const int hs = blockIdx.x, n = blockIdx.y;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarps = blockDim.x >> 5;
   // one warp per source row, 8 independent coalesced loads in flight per lane (no per-element
@@ -193,6 +199,8 @@ __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, voi
 template <int ELEM>
 __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
                                int K, int S, int Ks, int Cps, int Kpad) {
+  pdl_launch_dependents();
+  pdl_wait();
   const size_t total = (size_t)Co * Kpad;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
        i += (size_t)gridDim.x * blockDim.x) {
@@ -214,6 +222,8 @@ __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ o
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_fwd(const float *__restrict__ w, void *__restrict__ out,
                                                   int Co, int C, int taps, int Cp, int Kpad) {
+  pdl_launch_dependents();
+  pdl_wait();
   const int co = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= Kpad) return;
   const int t = k / Cp, c = k - t * Cp;
@@ -228,6 +238,8 @@ template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out,
                                                     int Co, int C, int taps, int Cop, int Kpad,
                                                     int flip) {
+  pdl_launch_dependents();
+  pdl_wait();
   const int ci = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= Kpad) return;
   const int t = k / Cop, co = k - t * Cop;

@@ -12,6 +12,17 @@ __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+// ------------------------------------------------------- programmatic dependent launch ---
+// Launched with cudaLaunchAttributeProgrammaticStreamSerialization, a kernel may start while its
+// predecessor in the stream drains: pdl_launch_dependents() lets the next kernel begin launching
+// once every CTA of this one has issued it; pdl_wait() blocks until the predecessor grid has
+// completed and its memory is visible (a no-op without the attribute).  Every kernel of the
+// tensor-core path calls pdl_wait() before its first global-memory access.
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // ------------------------------------------------------------------ mbarrier -------------
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");

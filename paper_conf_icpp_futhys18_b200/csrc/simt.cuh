@@ -167,6 +167,8 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
                                                     int taps, int Kw, int Cp, int ld, int mpad,
                                                     int splits, int accumulate, int s2d, int Ks) {
   __shared__ float tile[32][33];
+  pdl_launch_dependents();
+  pdl_wait();
   const int inner = C * taps;
   const int i0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
   const int lane = threadIdx.x, ty = threadIdx.y;
@@ -230,6 +232,8 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
                                                  unsigned int *__restrict__ tickets) {
   __shared__ float red[8][33];
   __shared__ bool last;
+  pdl_launch_dependents();
+  pdl_wait();
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
   const int co = blockIdx.x * 32 + lane, g = blockIdx.y;
   float a = 0.f;

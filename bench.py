@@ -48,6 +48,8 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--serial", action="store_true",
+                   help="issue the step on one stream (default: the real-network stream DAG)")
     p.add_argument("--no-graph", action="store_true",
                    help="launch every step eagerly (default on 1 GPU: the step is captured once "
                         "into a CUDA graph and replayed)")
@@ -187,36 +189,85 @@ def run_glp(args, ws, rank, local):
         states.append(LayerState(l, nl, ng, shard, args.math, dev, grads, i))
     stream = torch.cuda.current_stream()
 
-    def step(ev=None):
+    side_w = torch.cuda.Stream(device=dev)   # weight packs (weights are known at step start)
+    side_g = torch.cuda.Stream(device=dev)   # filter gradients: wgrad GEMM + dW/db reduction
+
+    def step(ev=None, concurrent=None):
+        """One training step of every layer's hot path.  concurrent (default: not timing kernels):
+        the stream DAG of a real network's step -- forward chain and backward-data chain on the
+        main stream; both weight packs of every layer on side stream W at step start; each
+        layer's filter-gradient GEMM + reductions on side stream G as soon as its dy is packed
+        (they overlap the next layer's backward-data work, which does not depend on them); G is
+        joined before the step ends.  Serial (ev given): everything on the main stream, in order,
+        with CUDA events around each GEMM for the per-kernel attribution."""
         stream = torch.cuda.current_stream()   # the capture stream while a graph is recorded
-        # forward, layer order
+        conc = (ev is None) if concurrent is None else concurrent
+        if not conc:
+            for i, s in enumerate(states):
+                c = s.conv
+                c.stage_pack(glp.GLP_PACK_X, s.t["x"])
+                c.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"])
+                if ev is not None:
+                    ev[i][0].record(stream)
+                c.stage_fwd(s.t["b"], s.y)
+                if ev is not None:
+                    ev[i][1].record(stream)
+            for i in reversed(range(len(states))):
+                s = states[i]
+                c = s.conv
+                c.stage_pack(glp.GLP_PACK_DY_DB, s.t["dy"])
+                if s.dx is not None:
+                    c.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"])
+                    if ev is not None:
+                        ev[i][2].record(stream)
+                    c.stage_bwd_data(s.dx)
+                    if ev is not None:
+                        ev[i][3].record(stream)
+                if ev is not None:
+                    ev[i][4].record(stream)
+                c.stage_bwd_filter()
+                if ev is not None:
+                    ev[i][5].record(stream)
+                c.stage_reduce(s.dw, s.db)
+            if G > 1:
+                grads.allreduce()
+            return
+        side_w.wait_stream(stream)
+        side_g.wait_stream(stream)
+        ew_f, ew_b = [], []
+        with torch.cuda.stream(side_w):
+            for s in states:
+                s.conv.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"], stream=side_w)
+                e = torch.cuda.Event()
+                e.record(side_w)
+                ew_f.append(e)
+            for s in reversed(states):
+                if s.dx is not None:
+                    s.conv.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"], stream=side_w)
+                e = torch.cuda.Event()
+                e.record(side_w)
+                ew_b.append(e)
+        ew_b = ew_b[::-1]
         for i, s in enumerate(states):
             c = s.conv
             c.stage_pack(glp.GLP_PACK_X, s.t["x"])
-            c.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"])
-            if ev is not None:
-                ev[i][0].record(stream)
+            stream.wait_event(ew_f[i])
             c.stage_fwd(s.t["b"], s.y)
-            if ev is not None:
-                ev[i][1].record(stream)
-        # backward, reverse layer order
         for i in reversed(range(len(states))):
             s = states[i]
             c = s.conv
             c.stage_pack(glp.GLP_PACK_DY_DB, s.t["dy"])
+            e_dy = torch.cuda.Event()
+            e_dy.record(stream)
+            side_g.wait_event(e_dy)
+            with torch.cuda.stream(side_g):
+                c.stage_bwd_filter(stream=side_g)
+                c.stage_reduce(s.dw, s.db, stream=side_g)
             if s.dx is not None:
-                c.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"])
-                if ev is not None:
-                    ev[i][2].record(stream)
+                stream.wait_event(ew_b[i])
                 c.stage_bwd_data(s.dx)
-                if ev is not None:
-                    ev[i][3].record(stream)
-            if ev is not None:
-                ev[i][4].record(stream)
-            c.stage_bwd_filter()
-            if ev is not None:
-                ev[i][5].record(stream)
-            c.stage_reduce(s.dw, s.db)
+        stream.wait_stream(side_w)
+        stream.wait_stream(side_g)
         if G > 1:
             grads.allreduce()
 
@@ -233,7 +284,7 @@ def run_glp(args, ws, rank, local):
         # replayed: no per-launch host work and minimal gaps between kernels.
         g_step = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g_step):
-            step()
+            step(concurrent=not args.serial)
         for _ in range(max(1, args.warmup)):
             g_step.replay()
     clocks = ClockSampler(local) if rank == 0 else None
@@ -268,7 +319,7 @@ def run_glp(args, ws, rank, local):
         # K more times eagerly with CUDA events around each GEMM on the launching stream (kernel
         # durations do not depend on how the launches were issued)
         for k in range(args.steps):
-            step(evs[k])
+            step(evs[k], concurrent=False)
         torch.cuda.synchronize()
     # per-kernel live timings (CUDA events on the launching stream)
     kern = []
@@ -360,7 +411,8 @@ def run_glp(args, ws, rank, local):
         "clocks": clk,
         "e2e": e2e,
         "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
-        "launch": "cuda_graph" if use_graph else "eager",
+        "launch": ("cuda_graph" if use_graph else "eager") +
+                  ("" if (args.serial or not use_graph) else " (3-stream step DAG)"),
     }
     print(json.dumps(line), flush=True)
     if G > 1:

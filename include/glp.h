@@ -138,7 +138,11 @@ glp_status_t glp_conv_bwd(glp_plan_t plan, const float *x, const float *dy, cons
  * filter gradient, and packs dy once for both backward GEMMs.  Every stage works on the plan's
  * single workspace layout: ws must hold info.ws_bwd bytes (1024-byte aligned).  Results are
  * bitwise identical to the composed calls.  Stages are asynchronous on `stream`; a stage reads
- * what earlier stages on the same stream wrote.  FP32 plans return GLP_ERR_NOT_SUPPORTED. */
+ * what earlier stages on the same stream wrote.  Each pack has its own workspace region (x, dy,
+ * forward W, backward-data W, partials), so stages that touch disjoint regions may run on
+ * different streams when the caller orders them with events (e.g. both weight packs up front,
+ * the filter-gradient GEMM + reduce beside the next layer's backward-data work).
+ * FP32 plans return GLP_ERR_NOT_SUPPORTED. */
 typedef enum {
   GLP_PACK_X = 0,          /* x  NCHW fp32 -> packed NHWC operand (rounded to the math mode)  */
   GLP_PACK_DY = 1,         /* dy NCHW fp32 -> packed NHWC operand                              */

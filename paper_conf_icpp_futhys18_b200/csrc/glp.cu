@@ -267,7 +267,7 @@ struct glp_plan_s {
   // SIMT path
   int simt_splits = 1, simt_chunk = 1;
   // workspace layout
-  size_t off_xpk = 0, off_dypk = 0, off_wpk = 0, off_part = 0, off_dbpart = 0;
+  size_t off_xpk = 0, off_dypk = 0, off_wpk = 0, off_wtpk = 0, off_part = 0, off_dbpart = 0;
   size_t sz_xpk = 0, sz_dypk = 0, sz_wpk = 0, sz_wtpk = 0, sz_part = 0, sz_dbpart = 0;
   int db_rows = 0;
   size_t ws_fwd = 0, ws_dgrad = 0, ws_wgrad = 0, ws_bwd = 0;
@@ -599,7 +599,7 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
 
 glp_status_t run_pack_w_dgrad(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
-  void *wtpk = ws + P.off_wpk;
+  void *wtpk = ws + P.off_wtpk;
   const int flip = P.dgrad.a_tma;  // the im2col-TMA dgrad walks taps flipped
   if (P.elem == 2)
     GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, dim3(dim3((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C)), dim3(256), 0, st, w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip));
@@ -637,7 +637,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, 
 glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   const PassPlan &pp = P.dgrad;
-  void *wtpk = ws + P.off_wpk;
+  void *wtpk = ws + P.off_wtpk;
   const void *dypk = ws + P.off_dypk;
   const int BK = pp.krow / P.elem;
   CUtensorMap mapB, mapA;
@@ -923,14 +923,15 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
                          P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, PACK_PT);
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
-    // one layout serves every call: [xpk | dypk | wpk/wtpk | part | dbpart]
+    // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;
     P->off_dypk = P->sz_xpk;
     P->off_wpk = P->off_dypk + P->sz_dypk;
-    P->off_part = P->off_wpk + std::max(P->sz_wpk, P->sz_wtpk);
+    P->off_wtpk = P->off_wpk + P->sz_wpk;   // own region: both weight packs can live at once
+    P->off_part = P->off_wtpk + P->sz_wtpk;
     P->off_dbpart = P->off_part + P->sz_part;
     P->ws_fwd = P->off_wpk + P->sz_wpk;
-    P->ws_dgrad = P->off_wpk + P->sz_wtpk;
+    P->ws_dgrad = P->off_wtpk + P->sz_wtpk;
     P->ws_wgrad = P->off_dbpart + P->sz_dbpart;
     P->ws_bwd = P->ws_wgrad;
     const long long slots = (long long)P->sm_count * P->fwd.ctas_per_sm;

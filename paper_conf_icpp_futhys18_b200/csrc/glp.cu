@@ -275,6 +275,7 @@ struct glp_plan_s {
   int allow_cg2 = 1;   // GLP_CTA_GROUP=1 in the environment forces single-CTA MMAs (A/B runs)
   int allow_ksub2 = 1; // GLP_KSUB=1 forces one k-block per pipeline stage (A/B runs)
   int ksub_max = 4;    // GLP_KSUB=k caps the k-blocks per stage
+  int wgrad_cg2 = 1;   // GLP_WGRAD_CG2=0: no CTA pairs for the filter gradient (A/B runs)
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
   int bn_model = 0;    // GLP_BN_MODEL=1: quantisation-model N tile for fwd/dgrad (measured: no gain)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
@@ -299,6 +300,13 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     pp.a_tma = (Cpx % u64 == 0 && P.Cop % u64 == 0 &&
                 (elem == 2 || (Cpx % u128 == 0 && P.Cop % u128 == 0))) ? 1 : 0;
     pp.krow = (!pp.a_tma || (Cpx % u128 == 0 && P.Cop % u128 == 0)) ? 128 : 64;
+    // CTA pairs split the MN-major B tile into halves of whole swizzle atoms: when the 128-byte
+    // atom (64 bf16) does not divide bn/2 but the 64-byte one does (C_o = 384 -> bn 192), use
+    // 64-byte rows so the pair still forms
+    const int bnw = choose_bn(d.Co);
+    if (pp.a_tma && elem == 2 && P.wgrad_cg2 && pp.krow == 128 && (bnw / 2) % 64 != 0 &&
+        (bnw / 2) % 32 == 0 && (long long)tapsx * Cpx > 128)
+      pp.krow = 64;
   }
   const int BK = pp.krow / elem;     // K elements per k-block (fwd/dgrad)
   const int BKP = 128 / elem;        // pixels per k-block (wgrad)
@@ -327,9 +335,11 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   }
   pp.m_tiles = (int)cdiv(pp.M, 128);
   // CTA pairs (tcgen05 cta_group::2, M = 256): each SM loads half of B.  Needs the TMA A path,
-  // at least two row tiles, and (MN-major B) half tiles that are whole swizzle atoms.
+  // at least two row tiles, and (MN-major B of the filter gradient) half tiles that are whole
+  // swizzle atoms.
   pp.cg = 1;
-  if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && mode != MODE_WGRAD) pp.cg = 2;
+  const bool wg_cg2 = P.wgrad_cg2 && (pp.bn / 2) % EPA == 0;   // MN-major B halves: whole atoms
+  if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && (mode != MODE_WGRAD || wg_cg2)) pp.cg = 2;
   if (mode != MODE_WGRAD && P.bn_model) {
     pp.bn = choose_bn_mn(pp.Ng, pp.M, pp.cg, P.sm_count);
     pp.bn_smem = pp.bn;
@@ -690,7 +700,7 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulat
   GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw,
                       dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32)),
                       dim3(32, 8), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
-                      P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_tiles * 128, P.wgrad.splits,
+                      P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128, P.wgrad.splits,
                       accumulate, P.s2d, P.dxg.Kw));
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
@@ -867,6 +877,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->ksub_max = std::max(1, std::min(4, atoi(e)));
     P->allow_ksub2 = P->ksub_max > 1;
   }
+  if (const char *e = getenv("GLP_WGRAD_CG2")) P->wgrad_cg2 = atoi(e) != 0;
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 15;

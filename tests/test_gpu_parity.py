@@ -238,3 +238,22 @@ def test_single_cta_mma_path(shape, math, monkeypatch):
     two = _run(_layer(shape, math), dr)
     for k in ("y", "dx"):
         np.testing.assert_array_equal(one[k], two[k], err_msg=k)
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape", [("c64_k3", 2, 64, 8, 8, 128, 3, 1, 1),
+                                   ("c64_k3_n256", 2, 64, 8, 8, 256, 3, 1, 1),
+                                   ("c96_k5", 2, 96, 9, 9, 256, 5, 1, 2),
+                                   ("c256_k3_n384", 2, 256, 7, 7, 384, 3, 1, 1)],
+                         ids=lambda s: s[0])
+@pytest.mark.parametrize("cg2", ["0", "1"])
+def test_wgrad_cta_pairs_exact(shape, math, cg2, monkeypatch):
+    """Filter gradient with and without CTA pairs (cta_group::2, MN-major halves of B; the
+    C_o = 384 case switches to 64-byte rows so bn/2 = 96 is whole atoms) is bit-exact on integer
+    data, with the split partials reduced at the paired row pitch."""
+    monkeypatch.setenv("GLP_WGRAD_CG2", cg2)
+    d = _data(shape, exact=True, seed=41)
+    got = _run(_layer(shape, math), d)
+    ref = _oracle(d, shape[7], shape[8])
+    np.testing.assert_array_equal(got["dw"], ref["dw"].astype(np.float32))
+    np.testing.assert_array_equal(got["db"], ref["db"].astype(np.float32))

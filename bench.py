@@ -346,7 +346,10 @@ def run_glp(args, ws, rank, local):
                 "kernel": f"igemm_kernel {dom['layer']} {dom['pass']}",
                 "peak_source": peaks["source"] + (" bf16 sustained" if args.math == "bf16"
                                                   else " bf16 sustained x 1.1/2.25 (tf32)"),
-                "share_of_step": round(dom["total_us"] / 1e3 / ms, 4)}
+                "share_of_step": round(dom["total_us"] / 1e3 / ms, 4),
+                # context: the same kernel against the burst (one-shot) cuBLAS figure
+                "frac_of_burst_peak": round(dom["tflops"] / (peaks["bf16_tflops"] * (
+                    1.0 if args.math == "bf16" else NOMINAL_TF32_OVER_BF16)), 4)}
     step_flops = sum(s.flops * (3 if s.dx is not None else 2) for s in states)
 
     # end-to-end: pinned host buffers -> device every step, dW||db back every step

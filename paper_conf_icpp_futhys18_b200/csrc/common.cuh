@@ -64,6 +64,9 @@ struct IgemmParams {
   int part_mpad;         // wgrad partial rows per split (m_tiles * 128)
   int a_tma;             // 1: A operand by im2col TMA (one thread); 0: cp.async gather
   int ksub;              // k-blocks per pipeline stage (1 or 2; cp.async path: 1)
+  unsigned long long *dbg_clk;  // diagnostics only (GLP_DEBUG_CLK): per-CTA cycle counters
+                                //   [0] MMA loop total [1] MMA waits on full [2] MMA waits on tempty
+                                //   [3] producer waits on empty
   int dbg_skip;          // diagnostics only (GLP_DEBUG_SKIP): bit0 skip A loads, bit1 skip B
                          // loads, bit2 skip MMAs — results are garbage, timings isolate stages
 };

@@ -278,6 +278,7 @@ struct glp_plan_s {
   int wgrad_cg2 = 1;   // GLP_WGRAD_CG2=0: no CTA pairs for the filter gradient (A/B runs)
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
   int bn_model = 0;    // GLP_BN_MODEL=1: quantisation-model N tile for fwd/dgrad (measured: no gain)
+  unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
 
@@ -358,7 +359,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   }
   const int a_bytes = mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow;
   const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
-  const int budget = 232448 - 1024 - 512;
+  const int budget = 232448 - 1024 - 1024;   // alignment slack; barriers, TMEM slot, bias slots
   // k-blocks per pipeline stage: as many (<= 4) as keep >= 3 stages in the ring.  One
   // full/empty round trip of the single MMA-issuing warp costs ~250-700 cycles whatever the stage
   // size (tools/sync_probe*.cu, GLP_DEBUG_SKIP=15 runs), more than the tensor work of one small-N
@@ -378,7 +379,8 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   int tc = 32;
   while (tc < 2 * pp.acc_cols) tc *= 2;
   pp.tmem_cols = tc;
-  pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16;
+  // ring + barriers + TMEM slot + 4 per-warp epilogue bias slots (32 floats, 16-byte aligned)
+  pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16 + 16 + 4 * 32 * 4;
   pp.tiles = pp.m_units * pp.n_tiles * pp.splits;   // work units (tile pairs for cg = 2)
 
   void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg);
@@ -462,6 +464,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   g.cbs = g.cp / (pp.krow / P.elem);
   p.a_tma = pp.a_tma;
   p.dbg_skip = P.dbg_skip;
+  p.dbg_clk = P.dbg_clk;
   g.div_hw = FastDiv((uint32_t)g.pix_hw);
   g.div_w = FastDiv((uint32_t)g.pix_w);
   g.div_cp = FastDiv((uint32_t)g.cp);
@@ -880,7 +883,9 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_WGRAD_CG2")) P->wgrad_cg2 = atoi(e) != 0;
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
-  if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 15;
+  // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
+  if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
+  if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 31;
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to
   // 32 would multiply the MMA work; those use the 16-byte-chunk cp.async gather.

@@ -177,6 +177,7 @@ __global__ void __launch_bounds__(288, 1)
         const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
         const uint32_t kb_tx = (la ? A_BYTES : 0u) + (lb ? b_bytes : 0u);
         const uint32_t sB_off = (uint32_t)KS * A_BYTES;
+        long long c_empty = 0;
         for (int tile = unit0; tile < total_tiles; tile += ustep) {
           int m_tile, n_tile, split;
           decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
@@ -220,7 +221,9 @@ __global__ void __launch_bounds__(288, 1)
           int kh = 0, kw = 0, cb = 0;       // fwd/dgrad K position (tap (kh, kw), channel block)
           for (int kbs = kb0; kbs < kb1; kbs += KS) {
             const int s = rs;
+            long long c0 = (p.dbg_clk != nullptr) ? clock64() : 0;
             mbar_wait(empty(s), rph ^ 1u);
+            if (p.dbg_clk != nullptr) c_empty += clock64() - c0;
             const int nsub = min(KS, kb1 - kbs);
             const uint32_t stg = stg_addr;
             const uint32_t tx = (uint32_t)nsub * kb_tx;
@@ -296,6 +299,7 @@ __global__ void __launch_bounds__(288, 1)
             }
           }
         }
+        if (p.dbg_clk != nullptr && lane == 0) p.dbg_clk[blockIdx.x * 4 + 3] = c_empty;
       }
     } else if (KROW == 128 && CG == 1) {
       // -------- cp.async gather (SWIZZLE_128B layouts only) --------
@@ -462,6 +466,8 @@ __global__ void __launch_bounds__(288, 1)
       int rs = 0;
       uint32_t rph = 0, it = 0;
       uint64_t da = da0, db = db0;   // descriptors of ring slot rs
+      const bool clk = p.dbg_clk != nullptr;
+      long long c_t0 = clk ? clock64() : 0, c_full = 0, c_te = 0;
       for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
         int m_tile, n_tile, split;
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
@@ -471,12 +477,16 @@ __global__ void __launch_bounds__(288, 1)
           kb1 = min(kb0 + kb_per_split, kb_total);
         }
         const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
+        long long c0 = clk ? clock64() : 0;
         mbar_wait(tempty(a), aph ^ 1u);
+        if (clk) c_te += clock64() - c0;
         tc_fence_after();
         const uint32_t d = tmem_base + a * (uint32_t)p.acc_cols;
         uint32_t acc = 0;
         for (int kbs = kb0; kbs < kb1; kbs += KS) {
+          if (clk) c0 = clock64();
           mbar_wait(full(rs), rph);
+          if (clk) c_full += clock64() - c0;
           tc_fence_after();
           const int nsub = min(KS, kb1 - kbs);
 #pragma unroll
@@ -500,17 +510,30 @@ __global__ void __launch_bounds__(288, 1)
         }
         mma_commit_e<CG>(tfull(a));
       }
+      if (clk && lane == 0) {
+        p.dbg_clk[blockIdx.x * 4 + 0] = clock64() - c_t0;
+        p.dbg_clk[blockIdx.x * 4 + 1] = c_full;
+        p.dbg_clk[blockIdx.x * 4 + 2] = c_te;
+      }
     }
     __syncwarp();
   } else {
     // ===================================== epilogue ========================================
     const int row = warp * 32 + lane;
     uint32_t it = 0;
+    // per-warp 32-float bias slot after the barriers (16-byte aligned)
+    const uint32_t sbias = ((tmem_slot + 16u + 15u) & ~15u) + (uint32_t)warp * 128u;
+    const bool clk = p.dbg_clk != nullptr && warp == 0;
+    long long e_t0 = clk ? clock64() : 0, e_wait = 0, e_ld = 0;
     for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
       int m_tile, n_tile, split;
       decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
-      mbar_wait_sleep(tfull(a), aph);
+      long long c0 = clk ? clock64() : 0;
+      // plain try_wait (suspends in hardware); GLP_DEBUG_SKIP bit 16 selects a nanosleep back-off
+      if (p.dbg_skip & 16) mbar_wait_sleep(tfull(a), aph);
+      else mbar_wait(tfull(a), aph);
+      if (clk) e_wait += clock64() - c0;
       tc_fence_after();
       const int m = (m_tile * CG + (int)rank) * C::BM + row;
       const int n0 = n_tile * p.bn;
@@ -520,19 +543,46 @@ __global__ void __launch_bounds__(288, 1)
         uint32_t n, pimg;
         g.div_hw.divmod((uint32_t)(mv ? m : 0), n, pimg);
         float *outp = p.out + (size_t)n * p.out_c * p.out_hw + pimg;
+        // lanes are 32 consecutive pixels: each store writes one channel's 128-byte pixel run.
+        // The chunk's 32 biases go through a per-warp smem slot (8 broadcast 16-byte loads, not
+        // 32 shuffles); the output pointer advances one channel plane per store.
+        const size_t plane = (size_t)p.out_hw;
+        float *ob = outp + (size_t)n0 * plane;
         for (int c0 = 0; c0 < p.bn; c0 += 32) {
           uint32_t v[32];
+          long long c1 = clk ? clock64() : 0;
           tmem_ld32(taddr + (uint32_t)c0, v);
-          float bv = 0.f;
-          if (MODE == MODE_FWD && p.bias && n0 + c0 + lane < p.N) bv = __ldg(p.bias + n0 + c0 + lane);
-          tmem_wait_ld();
-#pragma unroll
-          for (int q = 0; q < 32; ++q) {
-            const int ch = n0 + c0 + q;
-            float val = __uint_as_float(v[q]);
-            if (MODE == MODE_FWD) val += __shfl_sync(0xffffffffu, bv, q);  // bias[ch], warp-uniform
-            if (mv && c0 + q < p.bn && ch < p.N) outp[(size_t)ch * p.out_hw] = val;
+          if (MODE == MODE_FWD) {
+            sts_f32(sbias + 4u * lane,
+                    (p.bias && n0 + c0 + lane < p.N) ? __ldg(p.bias + n0 + c0 + lane) : 0.f);
+            __syncwarp();
           }
+          tmem_wait_ld();
+          if (clk) e_ld += clock64() - c1;
+          const int lim = min(32, min(p.bn - c0, p.N - n0 - c0));
+          float *o = ob + (size_t)c0 * plane;
+          if (mv && lim == 32) {
+#pragma unroll
+            for (int q = 0; q < 32; q += 4) {
+              float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
+              if (MODE == MODE_FWD) b4 = lds_f32x4(sbias + 4u * q);
+              o[0] = __uint_as_float(v[q]) + b4.x;
+              o += plane;
+              o[0] = __uint_as_float(v[q + 1]) + b4.y;
+              o += plane;
+              o[0] = __uint_as_float(v[q + 2]) + b4.z;
+              o += plane;
+              o[0] = __uint_as_float(v[q + 3]) + b4.w;
+              o += plane;
+            }
+          } else if (mv) {
+#pragma unroll
+            for (int q = 0; q < 32; ++q) {
+              const float b = (MODE == MODE_FWD) ? lds_f32(sbias + 4u * q) : 0.f;
+              if (q < lim) o[(size_t)q * plane] = __uint_as_float(v[q]) + b;
+            }
+          }
+          if (MODE == MODE_FWD) __syncwarp();   // the next chunk overwrites the slot
         }
       } else {
         float *dst = p.out + ((size_t)split * p.part_mpad + (size_t)m) * p.part_ld + n0;
@@ -562,6 +612,12 @@ __global__ void __launch_bounds__(288, 1)
         if (CG == 1) mbar_arrive(tempty(a));
         else mbar_arrive_cluster(mapa_shared(tempty(a), 0));
       }
+    }
+    if (clk && lane == 0) {
+      p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 0] = clock64() - e_t0;
+      p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 1] = e_wait;
+      p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 2] = e_ld;
+      p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 3] = it;
     }
   }
   // all tiles done: the next kernel may start launching into the teardown

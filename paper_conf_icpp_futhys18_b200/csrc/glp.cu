@@ -205,26 +205,36 @@ int choose_bn(int n) {
   return (int)rup(cdiv(n, nt), 16);
 }
 
-// N tile of the fwd / dgrad GEMMs (no split: the per-element K order, hence every output bit, is
-// independent of the tile).  Models the persistent grid's last-round quantisation: time ~
-// rounds * max(MMA cycles of a k-block ~ 2*bn, per-k-block issue floor); fewer N tiles (less A
-// re-reading) win ties.
-int choose_bn_mn(int n, long long M, int cg, int sm_count) {
-  const long long m_units = cdiv(M, 128LL * cg);
-  const double slots = std::max(1, sm_count / cg);
-  int best = choose_bn(n);
+// Tile (N tile, CTA pairing) of the fwd / dgrad GEMMs for grids that would leave SMs idle.  No
+// split of K: the per-element K order, hence every output bit, does not depend on the tile.
+// The default (N tile = ceil-split of N at <= 256, CTA pairs) is kept whenever it yields at least
+// two work units per slot (measured: for the large CaffeNet layers smaller tiles cost more in
+// A re-reads and per-k-block overhead than the last-round quantisation they save).  Below that,
+// time ~ rounds * (k-block MMA cycles ~ 2*bn, floored by the issue loop) picks the tile.
+void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, int &cg_out) {
+  const int bn0 = choose_bn(n);
+  const int cg0 = cg2_ok ? 2 : 1;
+  bn_out = bn0;
+  cg_out = cg0;
+  const long long units0 = cdiv(M, 128LL * cg0) * cdiv(n, bn0);
+  if (units0 >= 2LL * (sm_count / cg0)) return;
   double best_c = 1e300;
-  for (int nt = (int)cdiv(n, 256); nt <= 4; ++nt) {
-    const int bn = (int)rup(cdiv(n, nt), 16);
-    if ((int)cdiv(n, bn) != nt) continue;
-    const double rounds = std::ceil((double)m_units * nt / slots);
-    const double c = rounds * std::max(2.0 * bn, 224.0) * (1.0 + 0.03 * (nt - 1));
-    if (c < best_c) {
-      best_c = c;
-      best = bn;
+  for (int cg = cg0; cg >= 1; --cg) {
+    const long long m_units = cdiv(M, 128LL * cg);
+    const double slots = std::max(1, sm_count / cg);
+    for (int nt = (int)cdiv(n, 256); nt <= 4; ++nt) {
+      const int bn = (int)rup(cdiv(n, nt), 16);
+      if ((int)cdiv(n, bn) != nt || (cg == 2 && (bn / 2) % 8)) continue;
+      const double rounds = std::ceil((double)m_units * nt / slots);
+      const double c = rounds * std::max(2.0 * bn, 224.0) * (1.0 + 0.03 * (nt - 1)) *
+                       (cg == 1 ? 1.02 : 1.0);
+      if (c < best_c) {
+        best_c = c;
+        bn_out = bn;
+        cg_out = cg;
+      }
     }
   }
-  return best;
 }
 
 // Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
@@ -277,7 +287,7 @@ struct glp_plan_s {
   int ksub_max = 4;    // GLP_KSUB=k caps the k-blocks per stage
   int wgrad_cg2 = 1;   // GLP_WGRAD_CG2=0: no CTA pairs for the filter gradient (A/B runs)
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
-  int bn_model = 0;    // GLP_BN_MODEL=1: quantisation-model N tile for fwd/dgrad (measured: no gain)
+  int bn_model = 1;    // GLP_BN_MODEL=0: always the default fwd/dgrad tile (A/B runs)
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
@@ -342,7 +352,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const bool wg_cg2 = P.wgrad_cg2 && (pp.bn / 2) % EPA == 0;   // MN-major B halves: whole atoms
   if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && (mode != MODE_WGRAD || wg_cg2)) pp.cg = 2;
   if (mode != MODE_WGRAD && P.bn_model) {
-    pp.bn = choose_bn_mn(pp.Ng, pp.M, pp.cg, P.sm_count);
+    choose_tile_mn(pp.Ng, pp.M, pp.cg == 2, P.sm_count, pp.bn, pp.cg);
     pp.bn_smem = pp.bn;
   }
   if (pp.cg == 2) pp.bn_smem = pp.bn / 2;

@@ -58,6 +58,7 @@ struct IgemmParams {
   // epilogue
   float *out;            // y (fwd) / dx (dgrad) NCHW, or split partials (wgrad)
   const float *bias;     // fwd only, may be null
+  int bias_floats;       // fwd: floats of the smem bias stage (>= n_tiles*bn rounded to 32)
   int out_c;             // channels of out (C_o fwd, C_i dgrad)
   int out_hw;            // H_o*W_o (fwd) / H*W (dgrad)
   int part_ld;           // wgrad partial leading dimension (n_tiles * bn)

@@ -86,6 +86,7 @@ struct PassPlan {
   int a_tma = 0, krow = 128;        // A operand by im2col TMA; K-block row width (bytes)
   int cg = 1, m_units = 0;          // CTAs per MMA (tcgen05 cta_group); work units along M
   int ksub = 1;                     // k-blocks per pipeline stage
+  int bias_floats = 0;              // forward: floats of the epilogue's smem bias stage
 };
 
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -369,7 +370,9 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   }
   const int a_bytes = mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow;
   const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
-  const int budget = 232448 - 1024 - 1024;   // alignment slack; barriers, TMEM slot, bias slots
+  // forward: the bias vector is staged once per CTA in smem (every column a tile can touch)
+  pp.bias_floats = (mode == MODE_FWD) ? (int)rup((long long)pp.n_tiles * pp.bn, 32) + 32 : 0;
+  const int budget = 232448 - 1024 - 1024 - 4 * pp.bias_floats;   // alignment slack; barriers, TMEM slot
   // k-blocks per pipeline stage: as many (<= 4) as keep >= 3 stages in the ring.  One
   // full/empty round trip of the single MMA-issuing warp costs ~250-700 cycles whatever the stage
   // size (tools/sync_probe*.cu, GLP_DEBUG_SKIP=15 runs), more than the tensor work of one small-N
@@ -389,8 +392,8 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   int tc = 32;
   while (tc < 2 * pp.acc_cols) tc *= 2;
   pp.tmem_cols = tc;
-  // ring + barriers + TMEM slot + 4 per-warp epilogue bias slots (32 floats, 16-byte aligned)
-  pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16 + 16 + 4 * 32 * 4;
+  // ring + barriers + TMEM slot + the epilogue's bias stage (16-byte aligned)
+  pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16 + 16 + 4 * pp.bias_floats;
   pp.tiles = pp.m_units * pp.n_tiles * pp.splits;   // work units (tile pairs for cg = 2)
 
   void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg);
@@ -652,6 +655,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, 
   IgemmParams p = make_params(P, pp, MODE_FWD, xpk);
   p.out = y;
   p.bias = b;
+  p.bias_floats = pp.bias_floats;
   p.out_c = d.Co;
   p.out_hw = d.Ho * d.Wo;
   return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);

@@ -521,8 +521,15 @@ __global__ void __launch_bounds__(288, 1)
     // ===================================== epilogue ========================================
     const int row = warp * 32 + lane;
     uint32_t it = 0;
-    // per-warp 32-float bias slot after the barriers (16-byte aligned)
-    const uint32_t sbias = ((tmem_slot + 16u + 15u) & ~15u) + (uint32_t)warp * 128u;
+    // the whole bias vector staged once in shared memory after the barriers (16-byte aligned,
+    // p.bias_floats >= every column a tile can touch, zero past N): the per-chunk global bias
+    // load had its latency exposed in every chunk of every tile (ncu: STS waiting on LDG)
+    const uint32_t sbias = (tmem_slot + 16u + 15u) & ~15u;
+    if (MODE == MODE_FWD) {
+      for (int i = row; i < p.bias_floats; i += 128)
+        sts_f32(sbias + 4u * (uint32_t)i, (p.bias != nullptr && i < p.N) ? __ldg(p.bias + i) : 0.f);
+      named_bar_sync(1, 128);
+    }
     const bool clk = p.dbg_clk != nullptr && warp == 0;
     long long e_t0 = clk ? clock64() : 0, e_wait = 0, e_ld = 0;
     for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
@@ -548,15 +555,11 @@ __global__ void __launch_bounds__(288, 1)
         // 32 shuffles); the output pointer advances one channel plane per store.
         const size_t plane = (size_t)p.out_hw;
         float *ob = outp + (size_t)n0 * plane;
+        const uint32_t sb_tile = sbias + 4u * (uint32_t)n0;
         for (int c0 = 0; c0 < p.bn; c0 += 32) {
           uint32_t v[32];
           long long c1 = clk ? clock64() : 0;
           tmem_ld32(taddr + (uint32_t)c0, v);
-          if (MODE == MODE_FWD) {
-            sts_f32(sbias + 4u * lane,
-                    (p.bias && n0 + c0 + lane < p.N) ? __ldg(p.bias + n0 + c0 + lane) : 0.f);
-            __syncwarp();
-          }
           tmem_wait_ld();
           if (clk) e_ld += clock64() - c1;
           const int lim = min(32, min(p.bn - c0, p.N - n0 - c0));
@@ -565,7 +568,7 @@ __global__ void __launch_bounds__(288, 1)
 #pragma unroll
             for (int q = 0; q < 32; q += 4) {
               float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
-              if (MODE == MODE_FWD) b4 = lds_f32x4(sbias + 4u * q);
+              if (MODE == MODE_FWD) b4 = lds_f32x4(sb_tile + 4u * (uint32_t)(c0 + q));
               o[0] = __uint_as_float(v[q]) + b4.x;
               o += plane;
               o[0] = __uint_as_float(v[q + 1]) + b4.y;
@@ -578,11 +581,10 @@ __global__ void __launch_bounds__(288, 1)
           } else if (mv) {
 #pragma unroll
             for (int q = 0; q < 32; ++q) {
-              const float b = (MODE == MODE_FWD) ? lds_f32(sbias + 4u * q) : 0.f;
+              const float b = (MODE == MODE_FWD) ? lds_f32(sb_tile + 4u * (uint32_t)(c0 + q)) : 0.f;
               if (q < lim) o[(size_t)q * plane] = __uint_as_float(v[q]) + b;
             }
           }
-          if (MODE == MODE_FWD) __syncwarp();   // the next chunk overwrites the slot
         }
       } else {
         float *dst = p.out + ((size_t)split * p.part_mpad + (size_t)m) * p.part_ld + n0;
@@ -609,8 +611,8 @@ __global__ void __launch_bounds__(288, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) {   // one arrival per warp (on the pair leader's barrier for CG2)
-        if (CG == 1) mbar_arrive(tempty(a));
-        else mbar_arrive_cluster(mapa_shared(tempty(a), 0));
+        if (CG == 1) mbar_arrive_relaxed(tempty(a));
+        else mbar_arrive_cluster_relaxed(mapa_shared(tempty(a), 0));
       }
     }
     if (clk && lane == 0) {

@@ -74,6 +74,8 @@ typedef struct {
   size_t ws_fwd, ws_bwd_data, ws_bwd_filter, ws_bwd; /* workspace bytes per call               */
   double plan_us;        /* host time spent in glp_plan (Table 6 T_a analog)                   */
   int math;
+  int wgrad_halo;        /* 1: filter gradient by the shared-halo kernel (space-to-depth layers;
+                            dy packed on the padded grid), 0: im2col implicit GEMM             */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

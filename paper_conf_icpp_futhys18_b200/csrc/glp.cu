@@ -21,6 +21,7 @@
 
 #include "../../include/glp.h"
 #include "common.cuh"
+#include "hwgrad.cuh"
 #include "igemm.cuh"
 #include "pack.cuh"
 #include "simt.cuh"
@@ -274,6 +275,12 @@ struct glp_plan_s {
   glp_conv_desc_s dxg;
   int Cpx = 0, tapsx = 0;
   PassPlan fwd, dgrad, wgrad;
+  // halo filter gradient (hwgrad.cuh) for space-to-depth layers: dy is then packed on the padded
+  // dxg.H x dxg.W grid (zeros outside H_o x W_o) and the filter gradient stages x' once per
+  // k-block for all taps
+  int halo = 0;
+  HwgradParams hw{};
+  int hw_grid = 0, hw_smem = 0, hw_regs = 0;
   int S = 1;
   // SIMT path
   int simt_splits = 1, simt_chunk = 1;
@@ -289,11 +296,71 @@ struct glp_plan_s {
   int wgrad_cg2 = 1;   // GLP_WGRAD_CG2=0: no CTA pairs for the filter gradient (A/B runs)
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
   int bn_model = 1;    // GLP_BN_MODEL=0: always the default fwd/dgrad tile (A/B runs)
+  int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
 
 namespace {
+
+// Halo filter gradient (hwgrad.cuh) for space-to-depth layers whose x' rows are one 64-channel
+// bf16 atom and whose tap pairs' accumulators fit TMEM.  Split count: shape-only (a fixed
+// constant of 148 ranges, never the queried device), so the reduction order is fixed.
+glp_status_t plan_halo(glp_plan_s &P) {
+  P.halo = 0;
+  const glp_conv_desc_s &x = P.dxg;
+  if (!P.allow_halo || !P.s2d || P.elem != 2 || P.Cpx != 64 || P.tapsx < 2) return GLP_OK;
+  const int Ks = x.Kh, T = P.tapsx;
+  const int n_acc = (T + 1) / 2;
+  const int bn = (int)rup(x.Co, 16), acc_cols = (int)rup(bn, 32);
+  const int shift_max = (Ks - 1) * x.W + (Ks - 1);
+  const int halo_rows = HW_BKP + shift_max;
+  if (n_acc > 8 || bn > 256 || n_acc * acc_cols > 512 || halo_rows > 256) return GLP_OK;
+  HwgradParams &h = P.hw;
+  memset(&h, 0, sizeof(h));
+  h.n_acc = n_acc;
+  for (int j = 0; j < n_acc; ++j) {
+    int a = 2 * j, b = 2 * j + 1;
+    if (b >= T) {   // odd tap count: the last pair repeats tap T-2 (its rows are discarded)
+      a = T - 2;
+      b = T - 1;
+      h.dup_a_mask |= 1 << j;
+    }
+    h.tap_a[j] = a;
+    h.tap_b[j] = b;
+    h.shift_a[j] = (a / Ks) * x.W + a % Ks;
+    h.shift_b[j] = (b / Ks) * x.W + b % Ks;
+  }
+  h.bn = bn;
+  h.acc_cols = acc_cols;
+  int tc = 32;
+  while (tc < n_acc * acc_cols) tc *= 2;
+  h.tmem_cols = tc;
+  h.halo_rows = halo_rows;
+  h.a_bytes = (int)rup((long long)halo_rows * 128, 1024);
+  h.b_bytes = (int)cdiv(bn, 64) * HW_BKP * 128;
+  const int stage = h.a_bytes + h.b_bytes;
+  h.stages = std::min(8, (232448 - 2048) / stage);
+  if (h.stages < 2) return GLP_OK;
+  const long long rows = (long long)x.N * x.H * x.W;
+  h.kb_total = (int)cdiv(rows, HW_BKP);
+  h.splits = (int)std::min<long long>(h.kb_total, 148);
+  h.kb_per_split = (int)cdiv(h.kb_total, h.splits);
+  h.splits = (int)cdiv(h.kb_total, h.kb_per_split);
+  h.cpx = P.Cpx;
+  h.co = x.Co;
+  h.mpad = T * P.Cpx;
+  h.ld = bn;
+  P.hw_grid = h.splits;
+  P.hw_smem = 1024 + h.stages * stage + 8 * (2 * h.stages + 1) + 16;
+  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hwgrad_kernel),
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  cudaFuncAttributes fa;
+  GLP_CUDA(cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(hwgrad_kernel)));
+  P.hw_regs = fa.numRegs;
+  P.halo = 1;
+  return GLP_OK;
+}
 
 glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_limits_t &L) {
   const int elem = P.elem;
@@ -448,8 +515,9 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   g.kw = d.Kw;
   g.taps = (mode == MODE_DGRAD) ? P.taps : P.tapsx;
   if (mode == MODE_DGRAD) {
-    g.src_h = d.Ho;
-    g.src_w = d.Wo;
+    // halo plans pack dy on the padded dxg grid (zeros outside H_o x W_o): same values
+    g.src_h = P.halo ? P.dxg.H : d.Ho;
+    g.src_w = P.halo ? P.dxg.W : d.Wo;
     g.src_cp = P.Cop;
     g.cp = P.Cop;
     g.pix_hw = d.H * d.W;
@@ -564,8 +632,10 @@ DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
 }
 
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
-                             int Cp, float *db_part, cudaStream_t st) {
-  if (db_part == nullptr && Cp * P.elem <= 32) {
+                             int Cp, float *db_part, cudaStream_t st, int Ws = 1, int Wd = 1,
+                             int HWd = -1) {
+  if (HWd < 0) HWd = HW;   // default: dense destination (Ws == Wd)
+  if (db_part == nullptr && Cp * P.elem <= 32 && Ws == Wd) {
     const size_t n = (size_t)P.d.N * HW;
     const int g = (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 32);
     if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp));
@@ -573,14 +643,25 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
-  dim3 grid((unsigned)cdiv(HW, PACK_PT), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
+  dim3 grid((unsigned)cdiv(HWd, PACK_PT), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
   const int nt = (int)cdiv(P.d.Co, 32);
-  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt));
-  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt));
+  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
+  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
+}
+
+// dy -> its packed operand (dense NHWC, or on the padded dxg grid for halo plans) + db partials
+glp_status_t launch_pack_dy(const glp_plan_s &P, const float *dy, uint8_t *ws, bool with_db,
+                            cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  float *dbp = with_db ? reinterpret_cast<float *>(ws + P.off_dbpart) : nullptr;
+  if (P.halo)
+    return launch_pack_act(P, dy, ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, d.Wo,
+                           P.dxg.W, P.dxg.H * P.dxg.W);
+  return launch_pack_act(P, dy, ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st);
 }
 
 int ew_grid(size_t n) { return (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 16); }
@@ -687,7 +768,39 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
 }
 
+glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.dxg;
+  const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x' and dy
+  CUtensorMap mapX, mapDy;
+  glp_status_t s = encode_2d(&mapX, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows,
+                             (uint64_t)P.Cpx * 2, 64u, (uint32_t)P.hw.halo_rows,
+                             CU_TENSOR_MAP_SWIZZLE_128B);
+  if (s) return s;
+  if ((s = encode_2d(&mapDy, 2, ws + P.off_dypk, (uint64_t)P.Cop, rows, (uint64_t)P.Cop * 2, 64u,
+                     (uint32_t)HW_BKP, CU_TENSOR_MAP_SWIZZLE_128B)))
+    return s;
+  HwgradParams p = P.hw;
+  p.part = reinterpret_cast<float *>(ws + P.off_part);
+  p.dbg_skip = P.dbg_skip;
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3((unsigned)P.hw_grid);
+  cfg.blockDim = dim3(HW_THREADS);
+  cfg.dynamicSmemBytes = (size_t)P.hw_smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = P.pdl ? 1 : 0;
+  void *args[] = {&p, &mapX, &mapDy};
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hwgrad_kernel), args));
+  GLP_LAUNCH_CHECK("hwgrad_kernel");
+  return GLP_OK;
+}
+
 glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
+  if (P.halo) return run_wgrad_halo(P, ws, st);
   const glp_conv_desc_s &d = P.dxg;
   const PassPlan &pp = P.wgrad;
   const void *xpk = ws + P.off_xpk, *dypk = ws + P.off_dypk;
@@ -714,11 +827,18 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulat
                               cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
+  if (P.halo) {
+    GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
+                        dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32)),
+                        dim3(256), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx, P.hw.ld,
+                        P.hw.mpad, P.hw.splits, accumulate, P.s2d, P.dxg.Kw));
+    GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
+  } else
   GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw,
                       dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32)),
                       dim3(32, 8), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
-                      P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128, P.wgrad.splits,
-                      accumulate, P.s2d, P.dxg.Kw));
+                      P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128,
+                      P.wgrad.splits, accumulate, P.s2d, P.dxg.Kw));
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
     DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
@@ -897,6 +1017,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_WGRAD_CG2")) P->wgrad_cg2 = atoi(e) != 0;
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
+  if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 31;
@@ -942,16 +1063,23 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
       if (cur != device) cudaSetDevice(cur);
       return s;
     }
+    if ((s = plan_halo(*P))) {
+      delete P;
+      if (cur != device) cudaSetDevice(cur);
+      return s;
+    }
     const glp_conv_desc_s &c = *d;
     // x region: the forward/filter-gradient operand, or the direct packing of glp_debug_im2col
     P->sz_xpk = align1k(std::max((size_t)c.N * c.H * c.W * P->Cp,
                                  (size_t)c.N * P->dxg.H * P->dxg.W * P->Cpx) * P->elem);
-    P->sz_dypk = align1k((size_t)c.N * c.Ho * c.Wo * P->Cop * P->elem);
+    const size_t dy_hw = P->halo ? (size_t)P->dxg.H * P->dxg.W : (size_t)c.Ho * c.Wo;
+    P->sz_dypk = align1k((size_t)c.N * dy_hw * P->Cop * P->elem);
     P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
     P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
-    P->sz_part = align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
-                         P->wgrad.n_tiles * P->wgrad.bn * 4);
-    P->db_rows = c.N * (int)cdiv(c.Ho * c.Wo, PACK_PT);
+    P->sz_part = P->halo ? align1k((size_t)P->hw.splits * P->hw.mpad * P->hw.ld * 4)
+                         : align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
+                                   P->wgrad.n_tiles * P->wgrad.bn * 4);
+    P->db_rows = c.N * (int)cdiv((long long)dy_hw, PACK_PT);
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;
@@ -992,24 +1120,25 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->ctas_per_sm = P->fwd.ctas_per_sm;
   I->grid_fwd = P->fwd.grid;
   I->grid_bwd_data = P->dgrad.grid;
-  I->grid_bwd_filter = P->wgrad.grid;
+  I->grid_bwd_filter = P->halo ? P->hw_grid : P->wgrad.grid;
   I->tile_m = 128;
   I->tile_n_fwd = P->fwd.bn;
   I->tile_n_bwd_data = P->dgrad.bn;
-  I->tile_n_bwd_filter = P->wgrad.bn;
+  I->tile_n_bwd_filter = P->halo ? P->hw.bn : P->wgrad.bn;
   I->stages_fwd = P->fwd.stages;
   I->stages_bwd_data = P->dgrad.stages;
-  I->stages_bwd_filter = P->wgrad.stages;
-  I->splits_wgrad = P->math == GLP_MATH_FP32 ? P->simt_splits : P->wgrad.splits;
+  I->stages_bwd_filter = P->halo ? P->hw.stages : P->wgrad.stages;
+  I->splits_wgrad = P->math == GLP_MATH_FP32 ? P->simt_splits : P->halo ? P->hw.splits : P->wgrad.splits;
   I->tiles_fwd = P->fwd.tiles;
   I->tiles_bwd_data = P->dgrad.tiles;
-  I->tiles_bwd_filter = P->wgrad.tiles;
+  I->tiles_bwd_filter = P->halo ? P->hw.splits : P->wgrad.tiles;
   I->ws_fwd = P->ws_fwd;
   I->ws_bwd_data = P->ws_dgrad;
   I->ws_bwd_filter = P->ws_wgrad;
   I->ws_bwd = P->ws_bwd;
   I->plan_us = P->plan_us;
   I->math = P->math;
+  I->wgrad_halo = P->halo;
   return GLP_OK;
 }
 
@@ -1074,8 +1203,7 @@ glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, fl
   }
   if ((s = get_encode())) return s;
   uint8_t *wsb = static_cast<uint8_t *>(ws);
-  void *dypk = wsb + P->off_dypk;
-  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st))) return s;
+  if ((s = launch_pack_dy(*P, dy, wsb, false, st))) return s;
   if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
   return run_dgrad_gemm(*P, dx, wsb, st);
 }
@@ -1091,11 +1219,9 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   if (P->math == GLP_MATH_FP32) return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
   if ((s = get_encode())) return s;
-  void *xpk = wsb + P->off_xpk, *dypk = wsb + P->off_dypk;
+  void *xpk = wsb + P->off_xpk;
   if ((s = launch_pack_x(*P, x, xpk, st))) return s;
-  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
-                           db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
-    return s;
+  if ((s = launch_pack_dy(*P, dy, wsb, db != nullptr, st))) return s;
   if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
   return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
 }
@@ -1120,10 +1246,8 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
     return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
   }
   if ((s = get_encode())) return s;
-  void *xpk = wsb + P->off_xpk, *dypk = wsb + P->off_dypk;
-  if ((s = launch_pack_act(*P, dy, dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
-                           db ? reinterpret_cast<float *>(wsb + P->off_dbpart) : nullptr, st)))
-    return s;
+  void *xpk = wsb + P->off_xpk;
+  if ((s = launch_pack_dy(*P, dy, wsb, db != nullptr, st))) return s;
   if (dx) {
     if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
     if ((s = run_dgrad_gemm(*P, dx, wsb, st))) return s;
@@ -1152,10 +1276,9 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
     case GLP_PACK_X:
       return launch_pack_x(*P, src, wsb + P->off_xpk, st);
     case GLP_PACK_DY:
-      return launch_pack_act(*P, src, wsb + P->off_dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop, nullptr, st);
+      return launch_pack_dy(*P, src, wsb, false, st);
     case GLP_PACK_DY_DB:
-      return launch_pack_act(*P, src, wsb + P->off_dypk, P->d.Co, P->d.Ho * P->d.Wo, P->Cop,
-                             reinterpret_cast<float *>(wsb + P->off_dbpart), st);
+      return launch_pack_dy(*P, src, wsb, true, st);
     case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, src, wsb, st);
     case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, src, wsb, st);
   }

@@ -1,0 +1,182 @@
+// hwgrad.cuh — filter gradient of a unit-stride (space-to-depth) layer with a shared halo tile.
+//
+// dW'[t][c][co] = sum_p x'[p + s_t][c] * dy[p][co]   (PAPER.md P129; north_star (3): "backward-
+// filter GEMMs summed over the samples of a batch"), where p runs over the flattened padded grid
+// of the packed operands (n, h, w) in [0,N) x [0,H') x [0,W') with H' x W' the space-to-depth
+// image, s_t = kh*W' + kw is the row shift of tap t = (kh, kw), and dy is packed
+// on the same H' x W' grid with zeros outside its H_o x W_o valid region (junk positions, so
+// they contribute nothing).
+//
+// Why: the im2col filter gradient re-reads x once per tap from L2 (9x for CaffeNet conv1's 3x3
+// s2d taps) and was L2-bandwidth bound (45 B/clk/SM measured, 373 TFLOP/s).  Here one TMA per
+// k-block stages the x' rows [p0, p0 + BKP + s_max] once; the A operand of every tap is the same
+// smem tile read through a descriptor whose start is shifted by s_t rows.  tcgen05 applies the
+// 128-byte swizzle on absolute smem address bits, so any row shift is a valid SWIZZLE_128B
+// operand (measured exactly: tools/shift_probe.cu).  One M = 128 MMA covers a pair of taps: the
+// two 64-channel MN-major atoms of A are the tile at shifts s_a and s_b (LBO = (s_b - s_a) rows).
+//
+// Work: the N*H'*W' pixel rows are cut into `splits` contiguous ranges (shape-only count); CTA u
+// accumulates all tap pairs x C_o of its range in TMEM (n_acc accumulators) and writes one fp32
+// partial [u][t*64 + c][co]; reduce_tc_dw sums the partials in a fixed order (deterministic,
+// independent of the grid and of S: convergence invariance, P264).
+// CTA = 192 threads: warps 0-3 epilogue, warp 4 TMA producer, warp 5 TMEM owner + MMA issuer.
+#pragma once
+#include "common.cuh"
+#include "ptx.cuh"
+
+namespace glp {
+
+constexpr int HW_THREADS = 192;
+constexpr int HW_BKP = 128;   // pixel rows (K) per k-block
+
+struct HwgradParams {
+  int n_acc;          // accumulators = ceil(taps / 2) tap pairs
+  int tap_a[8], tap_b[8];   // taps of the two 64-channel atoms of accumulator j (a < b)
+  int shift_a[8], shift_b[8];
+  int dup_a_mask;     // bit j: atom a of pair j duplicates an earlier pair (odd tap count)
+  int bn;             // C_o tile (multiple of 16, <= 256): all output channels
+  int acc_cols;       // TMEM columns per accumulator (multiple of 32)
+  int tmem_cols;      // allocation (power of two >= n_acc * acc_cols)
+  int halo_rows;      // rows of the x' tile per k-block (BKP + max shift)
+  int a_bytes, b_bytes, stages;
+  int kb_total, kb_per_split, splits;
+  int cpx;            // channels of x' (64: one atom)
+  int co;             // valid output channels
+  float *part;        // [splits][mpad][ld] fp32
+  int mpad, ld;
+  int dbg_skip;       // diagnostics (GLP_DEBUG_SKIP): bit0 skip x' loads, bit1 dy loads, bit2 MMAs
+};
+
+__global__ void __launch_bounds__(HW_THREADS, 1)
+    hwgrad_kernel(const __grid_constant__ HwgradParams p, const __grid_constant__ CUtensorMap tmapX,
+                  const __grid_constant__ CUtensorMap tmapDy) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023u) & ~1023u;
+  const uint32_t stage_bytes = (uint32_t)(p.a_bytes + p.b_bytes);
+  const uint32_t bars = base + (uint32_t)p.stages * stage_bytes;
+  const int S_ = p.stages;
+  auto full = [&](int s) { return bars + 8u * s; };
+  auto empty = [&](int s) { return bars + 8u * (S_ + s); };
+  const uint32_t tfull = bars + 8u * (2 * S_);
+  const uint32_t tmem_slot = bars + 8u * (2 * S_ + 1);
+  volatile uint32_t *tmem_slot_ptr =
+      reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0);
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S_; ++s) {
+      mbar_init(full(s), 1);
+      mbar_init(empty(s), 1);
+    }
+    mbar_init(tfull, 1);
+    fence_mbar_init();
+  }
+  if (warp == 5) {
+    tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
+    tmem_relinquish();
+  }
+  if (warp == 4 && lane == 0) {
+    tma_prefetch(&tmapX);
+    tma_prefetch(&tmapDy);
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  pdl_wait();
+  const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);
+  const int u = blockIdx.x;   // one split per CTA
+  const int kb0 = u * p.kb_per_split;
+  const int kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+
+  if (warp == 4) {
+    // ===================================== producer ========================================
+    int rs = 0;
+    uint32_t rph = 0;
+    const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+    const int nb = (p.bn + 63) / 64;
+    const uint32_t tx = (la ? (uint32_t)(p.halo_rows * 128) : 0u) + (lb ? (uint32_t)p.b_bytes : 0u);
+    for (int kb = kb0; kb < kb1; ++kb) {
+      mbar_wait(empty(rs), rph ^ 1u);
+      const uint32_t sA = base + (uint32_t)rs * stage_bytes, sB = sA + (uint32_t)p.a_bytes;
+      mbar_arrive_expect_tx_e(full(rs), tx);
+      const int row0 = kb * HW_BKP;
+      if (la) tma_load_2d_e(sA, &tmapX, full(rs), 0, row0);
+      if (lb)
+        for (int a = 0; a < nb; ++a)
+          tma_load_2d_e(sB + (uint32_t)a * (HW_BKP * 128), &tmapDy, full(rs), a * 64, row0);
+      if (++rs == S_) {
+        rs = 0;
+        rph ^= 1u;
+      }
+    }
+  } else if (warp == 5) {
+    // ===================================== MMA issuer ======================================
+    const uint32_t idesc = make_idesc(1u, 1u, 1u, 128u, (uint32_t)p.bn);
+    int rs = 0;
+    uint32_t rph = 0;
+    uint32_t acc = 0;
+    for (int kb = kb0; kb < kb1; ++kb) {
+      mbar_wait(full(rs), rph);
+      tc_fence_after();
+      const uint32_t sA = base + (uint32_t)rs * stage_bytes, sB = sA + (uint32_t)p.a_bytes;
+      // B: dy MN-major, 64-channel SW128 atoms of HW_BKP rows (LBO = one atom column)
+      const uint64_t db = make_sdesc(sB, HW_BKP * 128u, 1024u, 2u);
+      for (int j = 0; j < p.n_acc && !(p.dbg_skip & 4); ++j) {
+        const uint32_t sa = sA + (uint32_t)p.shift_a[j] * 128u;
+        const uint64_t da =
+            make_sdesc(sa, (uint32_t)(p.shift_b[j] - p.shift_a[j]) * 128u, 1024u, 2u);
+        const uint32_t d = tmem_base + (uint32_t)(j * p.acc_cols);
+        // 8 MMAs of K = 16 pixel rows (2048 bytes = 128 descriptor units for A and B)
+        mma_kblock_e<0, 1, 4, 128>(d, da, db, idesc, acc);
+        mma_kblock_e<0, 1, 4, 128>(d, da + 512u, db + 512u, idesc, 1u);
+      }
+      acc = 1;
+      mma_commit_e<1>(empty(rs));
+      if (++rs == S_) {
+        rs = 0;
+        rph ^= 1u;
+      }
+    }
+    mma_commit_e<1>(tfull);
+    __syncwarp();
+  } else {
+    // ===================================== epilogue ========================================
+    mbar_wait(tfull, 0);
+    tc_fence_after();
+    const int r = warp * 32 + lane;   // TMEM lane = M row of every accumulator
+    const int atom = r >> 6, c = r & 63;
+    const bool empty_range = kb1 <= kb0;
+    for (int j = 0; j < p.n_acc; ++j) {
+      const bool dup = atom == 0 && ((p.dup_a_mask >> j) & 1);
+      const int t = atom ? p.tap_b[j] : p.tap_a[j];
+      float *dst = p.part + ((size_t)u * p.mpad + (size_t)t * p.cpx + c) * p.ld;
+      for (int c0 = 0; c0 < p.bn; c0 += 32) {
+        uint32_t v[32];
+        tmem_ld32(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(j * p.acc_cols + c0), v);
+        tmem_wait_ld();
+        if (dup) continue;
+        const int lim = min(32, p.bn - c0);
+        if (lim == 32) {
+#pragma unroll
+          for (int q = 0; q < 32; q += 4)
+            *reinterpret_cast<float4 *>(dst + c0 + q) =
+                empty_range ? make_float4(0.f, 0.f, 0.f, 0.f)
+                            : make_float4(__uint_as_float(v[q]), __uint_as_float(v[q + 1]),
+                                          __uint_as_float(v[q + 2]), __uint_as_float(v[q + 3]));
+        } else {
+#pragma unroll
+          for (int q = 0; q < 32; ++q)
+            if (q < lim) dst[c0 + q] = empty_range ? 0.f : __uint_as_float(v[q]);
+        }
+      }
+    }
+  }
+  pdl_launch_dependents();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 5) tmem_dealloc(tmem_base, (uint32_t)p.tmem_cols);
+}
+
+}  // namespace glp

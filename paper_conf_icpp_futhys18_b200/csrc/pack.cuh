@@ -50,30 +50,56 @@ struct PackOut<4> {
 // pixel quarters, then a xor-shuffle tree).
 constexpr int PACK_PT = 128;
 
+// Padded destination (Wd != Ws): the pixels are written on a wider Hd x Wd grid (row q = h*Wd + w,
+// HWd = Hd*Wd rows per image), zeros at the positions outside the Hs x Ws source image — the
+// dy operand of the halo filter gradient (hwgrad.cuh).  Blocks then run over destination rows.
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict__ src,
                                                          void *__restrict__ dst, int C, int HW,
                                                          int Cp, float *__restrict__ db_part,
                                                          unsigned int *__restrict__ tickets,
-                                                         int n_tickets) {
+                                                         int n_tickets, int Ws, int Wd, int HWd) {
   __shared__ float tile[32][PACK_PT + 1];
   pdl_launch_dependents();
   pdl_wait();
   const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * PACK_PT;
+  const bool padded = Wd != Ws;
+  const int Hs = padded ? HW / Ws : 0;
   // arm the completion tickets of the deterministic db reduction that consumes db_part
   if (tickets != nullptr && (blockIdx.x | blockIdx.y | blockIdx.z) == 0)
     for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const float *s = src + (size_t)n * C * HW;
+  // source pixel of each of this lane's 4 destination rows (one division per thread; the rows
+  // are 32 apart, so the padded column advances by 32 with at most one wrap when Wd > 32)
+  int spx[4];
+  bool sok[4];
+  {
+    const int q0 = p0 + lane;
+    int h = padded ? q0 / Wd : 0, w = padded ? q0 - h * Wd : 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (padded) {
+        sok[q] = h < Hs && w < Ws;
+        spx[q] = h * Ws + w;
+        w += 32;
+        while (w >= Wd) {
+          w -= Wd;
+          ++h;
+        }
+      } else {
+        spx[q] = q0 + q * 32;
+        sok[q] = spx[q] < HW;
+      }
+    }
+  }
   float v[4][4];
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
     const int c = c0 + warp + 8 * k;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int px = p0 + q * 32 + lane;
-      v[k][q] = (c < C && px < HW) ? __ldg(s + (size_t)c * HW + px) : 0.f;
-    }
+    for (int q = 0; q < 4; ++q)
+      v[k][q] = (c < C && sok[q]) ? __ldg(s + (size_t)c * HW + spx[q]) : 0.f;
   }
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
@@ -97,8 +123,8 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
   for (int pass = 0; pass < PACK_PT / PPP; ++pass) {
     const int pp = pass * PPP + threadIdx.x / CPP, j = threadIdx.x % CPP;
     const int px = p0 + pp, cl = j * CPT, c = c0 + cl;
-    if (px < HW && c < Cp) {
-      const size_t o = ((size_t)n * HW + px) * Cp + c;
+    if (px < HWd && c < Cp) {
+      const size_t o = ((size_t)n * HWd + px) * Cp + c;
 #pragma unroll
       for (int u = 0; u < CPT; u += 4)
         PackOut<ELEM>::store4(dst, o + u, tile[cl + u][pp], tile[cl + u + 1][pp],

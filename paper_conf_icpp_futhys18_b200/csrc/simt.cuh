@@ -219,6 +219,60 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
   }
 }
 
+// Many-split variant (the halo filter gradient's 148 one-per-CTA partials): block = 32 channels x
+// 8 split phases over 4 weight rows; thread (ty, lane) sums splits ty, ty+8, ... in ascending order,
+// then the 8 phase sums are added in phase order.  Fixed order, a function of `splits` only.
+__global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict__ part,
+                                                         float *__restrict__ dw, int Co, int C,
+                                                         int taps, int Kw, int Cp, int ld, int mpad,
+                                                         int splits, int accumulate, int s2d, int Ks) {
+  __shared__ float red[8][4][33];
+  pdl_launch_dependents();
+  pdl_wait();
+  const int inner = C * taps;
+  const int i0 = blockIdx.x * 4, co = blockIdx.y * 32 + (threadIdx.x & 31), ty = threadIdx.x >> 5;
+  const size_t sstride = (size_t)mpad * ld;
+  const float *src[4];
+  bool ok[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int i = i0 + u;
+    ok[u] = i < inner && co < Co;
+    int row = 0;
+    if (ok[u]) {
+      const int ci = i / taps, t = i - ci * taps;
+      row = t * Cp + ci;
+      if (s2d > 1) {
+        const int kh = t / Kw, kw = t % Kw;
+        row = ((kh / s2d) * Ks + kw / s2d) * Cp + ((kh % s2d) * s2d + kw % s2d) * C + ci;
+      }
+    }
+    src[u] = part + (size_t)row * ld + (ok[u] ? co : 0);
+  }
+  float a[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int sp = ty; sp < splits; sp += 8) {
+    float v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = ok[u] ? __ldg(src[u] + (size_t)sp * sstride) : 0.f;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) a[u] += v[u];
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u) red[ty][u][threadIdx.x & 31] = a[u];
+  __syncthreads();
+  if (ty < 4) {
+    const int u = ty, lane = threadIdx.x & 31;
+    float t = 0.f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += red[k][u][lane];
+    const int i = i0 + u;
+    if (i < inner && co < Co) {
+      const size_t idx = (size_t)co * inner + i;
+      dw[idx] = accumulate ? dw[idx] + t : t;
+    }
+  }
+}
+
 // db[co] = sum over rows of part[row][co] (rows = N * pixel tiles, or SIMT splits), fixed order.
 // db[co] = sum over `rows` partial rows, deterministic and parallel over row groups:
 // grid (ceil(Co/32), DB_GROUPS).  Block (x, g) sums rows g, g+G, ... (thread ty takes every 8th of

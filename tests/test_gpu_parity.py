@@ -257,3 +257,50 @@ def test_wgrad_cta_pairs_exact(shape, math, cg2, monkeypatch):
     ref = _oracle(d, shape[7], shape[8])
     np.testing.assert_array_equal(got["dw"], ref["dw"].astype(np.float32))
     np.testing.assert_array_equal(got["db"], ref["db"].astype(np.float32))
+
+
+# space-to-depth layers whose filter gradient runs on the shared-halo kernel (hwgrad.cuh)
+HALO_SHAPES = [
+    ("caffenet_conv1_full_hw", 2, 3, 227, 227, 96, 11, 4, 0),   # 9 taps (odd: duplicate pair)
+    ("caffenet_conv1_s4", 2, 3, 67, 67, 96, 11, 4, 0),
+    ("s2d_c12_k5_s2", 3, 12, 20, 21, 40, 5, 2, 2),             # 9 taps, C_o = 40 (one B atom)
+    ("s2d_c16_k3_s2", 2, 16, 17, 15, 24, 3, 2, 1),             # 4 taps, no duplicate
+]
+
+
+@pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
+def test_halo_wgrad_exact(shape, monkeypatch):
+    """The shared-halo filter gradient (row-shifted SWIZZLE_128B descriptors over one staged x'
+    tile per k-block, dy on the padded grid) is bit-exact on integer data, and so is the
+    backward-data pass that reads the padded dy; GLP_HALO=0 (im2col path) agrees bit for bit."""
+    d = _data(shape, exact=True, seed=43)
+    ref = _oracle(d, shape[7], shape[8])
+    layer = _layer(shape, "bf16")
+    assert layer.info.wgrad_halo == 1
+    got = _run(layer, d)
+    for k in ("y", "dx", "dw", "db"):
+        np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+    monkeypatch.setenv("GLP_HALO", "0")
+    layer0 = _layer(shape, "bf16")
+    assert layer0.info.wgrad_halo == 0
+    got0 = _run(layer0, d)
+    for k in ("dw", "db", "dx"):
+        np.testing.assert_array_equal(got0[k], got[k], err_msg=k)
+
+
+@pytest.mark.parametrize("shape", HALO_SHAPES[:2], ids=lambda s: s[0])
+def test_halo_wgrad_random_and_invariant(shape):
+    """Random data: within the bf16 bar of the oracle and of the rounding-emulated oracle, and
+    bitwise identical across samples-in-flight overrides and reruns (shape-only splits)."""
+    d = _data(shape, seed=44)
+    ref = _oracle(d, shape[7], shape[8])
+    emu = _oracle(d, shape[7], shape[8], x=EMU["bf16"](d["x"]), w=EMU["bf16"](d["w"]),
+                  dy=EMU["bf16"](d["dy"]))
+    runs = [_run(_layer(shape, "bf16", S), d) for S in (0, 1, 2, 0)]
+    for k in ("dw", "db"):
+        r = ref[k]
+        assert np.abs(runs[0][k] - r).max() / np.abs(r).max() <= TOL["bf16"], k
+        e = emu[k]
+        assert np.abs(runs[0][k] - e).max() / np.abs(e).max() <= 1e-4, k
+        for other in runs[1:]:
+            np.testing.assert_array_equal(other[k], runs[0][k], err_msg=k)

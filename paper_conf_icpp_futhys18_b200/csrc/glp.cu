@@ -272,6 +272,7 @@ struct glp_plan_s {
   // Geometry of the x operand as the forward and filter-gradient passes see it: the layer itself,
   // or its space-to-depth form (s2d = stride S > 1: stride 1, ceil(K/S) taps, S*S*C channels).
   int s2d = 0;
+  int s2d_blocks = 1;   // resident pack_s2d blocks per SM (occupancy API): its persistent grid
   glp_conv_desc_s dxg;
   int Cpx = 0, tapsx = 0;
   PassPlan fwd, dgrad, wgrad;
@@ -643,12 +644,12 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
-  dim3 grid((unsigned)cdiv(HWd, PACK_PT), (unsigned)cdiv(Cp, 32), (unsigned)P.d.N);
+  dim3 grid((unsigned)cdiv(Cp, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
   const int nt = (int)cdiv(P.d.Co, 32);
-  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
-  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
+  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
+  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
 }
@@ -690,14 +691,15 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
   if (P.s2d) {
     const int S = P.s2d;
     const size_t smem = (size_t)S * d.C * d.W * sizeof(float);
-    dim3 grid((unsigned)P.dxg.H, (unsigned)d.N);
-    const int quads = P.Cpx / 4;   // the block is a whole number of channel-quad groups
-    const int threads = quads <= 256 ? quads * (256 / quads) : 0;
-    if (threads < 32) return fail(GLP_ERR_NOT_SUPPORTED, "space-to-depth channel pitch too large");
+    const int cpr = P.Cpx * P.elem / 16;
+    if (256 % cpr || (long long)S * d.C * d.W > 256LL * S2D_LD)
+      return fail(GLP_ERR_NOT_SUPPORTED, "space-to-depth geometry too large for the pack kernel");
+    const int rows = d.N * P.dxg.H;
+    dim3 grid((unsigned)std::min(rows, P.sm_count * std::max(1, P.s2d_blocks)));
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(threads), smem, st, x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(threads), smem, st, x, dst, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
     GLP_LAUNCH_CHECK("pack_s2d");
     return GLP_OK;
   }
@@ -1038,12 +1040,18 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     const int S2 = d->Sh, Ks = (int)cdiv(d->Kh, S2), cs = S2 * S2 * d->C;
     const int cps = (int)rup(cs, 32);
     if ((long long)Ks * Ks * cps < (long long)P->taps * rup(P->Cp, 128 / P->elem) &&
-        (size_t)S2 * d->C * d->W * sizeof(float) <= 48 * 1024) {
+        (long long)S2 * d->C * d->W <= 256LL * S2D_LD && 256 % (cps * P->elem / 16) == 0) {
       P->s2d = S2;
       P->dxg = glp_conv_desc_s{d->N, cs, d->Ho + Ks - 1, d->Wo + Ks - 1, d->Co, Ks, Ks, 1, 1,
                                0, 0, d->Ho, d->Wo};
       P->Cpx = cps;
       P->tapsx = Ks * Ks;
+      const size_t ssm = (size_t)S2 * d->C * d->W * sizeof(float);
+      void *fn = P->elem == 2 ? reinterpret_cast<void *>(pack_s2d<2>) : reinterpret_cast<void *>(pack_s2d<4>);
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&P->s2d_blocks, fn, 256, ssm) != cudaSuccess) {
+        cudaGetLastError();
+        P->s2d_blocks = 1;
+      }
     }
   }
   glp_device_limits_t L;
@@ -1079,7 +1087,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->sz_part = P->halo ? align1k((size_t)P->hw.splits * P->hw.mpad * P->hw.ld * 4)
                          : align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
-    P->db_rows = c.N * (int)cdiv((long long)dy_hw, PACK_PT);
+    P->db_rows = (int)cdiv((long long)c.N * dy_hw, PACK_PT);
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;

@@ -43,53 +43,59 @@ struct PackOut<4> {
 };
 
 // NCHW fp32 [N][C][HW] -> NHWC [N][HW][Cp] (rounded), zero for c >= C.
-// Tile 32 channels x PACK_PT pixels per 256-thread block: 16 independent coalesced loads per
-// thread, conflict-free transposed smem reads, 16-byte stores.
-// grid (ceil(HW/PACK_PT), ceil(Cp/32), N).  db_part (optional): [N][ceil(HW/PACK_PT)][C], each
-// entry the sum of one channel over one pixel tile in a fixed order (lane-sequential over the 4
-// pixel quarters, then a xor-shuffle tree).
+// Block = 32 channels x PACK_PT consecutive destination rows q of the whole batch (rows of
+// consecutive images follow each other, so small images leave no ragged tile per image), 256
+// threads: 16 independent coalesced loads per thread, conflict-free transposed smem reads,
+// 16-byte stores.  grid (ceil(Cp/32), ceil(N*HWd/PACK_PT)): the channel blocks of a row tile are
+// consecutive blocks, so the 64-byte pieces of each output row are written close in time and
+// merge into whole lines in L2 (channel-block-major order wrote each row in pieces far apart).
+// Padded destination (Wd != Ws): rows are positions (n, h, w) of an Hd x Wd grid per image
+// (HWd = Hd*Wd), zero outside the Hs x Ws source image — the dy operand of the halo filter
+// gradient (hwgrad.cuh).  Dense: Wd == Ws, HWd == HW.
+// db_part (optional): [row tiles][C], each entry the sum of one channel over one row tile in a
+// fixed order (lane-sequential over the 4 row quarters, then a xor-shuffle tree).
 constexpr int PACK_PT = 128;
 
-// Padded destination (Wd != Ws): the pixels are written on a wider Hd x Wd grid (row q = h*Wd + w,
-// HWd = Hd*Wd rows per image), zeros at the positions outside the Hs x Ws source image — the
-// dy operand of the halo filter gradient (hwgrad.cuh).  Blocks then run over destination rows.
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict__ src,
-                                                         void *__restrict__ dst, int C, int HW,
-                                                         int Cp, float *__restrict__ db_part,
+                                                         void *__restrict__ dst, int N, int C,
+                                                         int HW, int Cp, float *__restrict__ db_part,
                                                          unsigned int *__restrict__ tickets,
                                                          int n_tickets, int Ws, int Wd, int HWd) {
   __shared__ float tile[32][PACK_PT + 1];
   pdl_launch_dependents();
   pdl_wait();
-  const int n = blockIdx.z, c0 = blockIdx.y * 32, p0 = blockIdx.x * PACK_PT;
-  const bool padded = Wd != Ws;
-  const int Hs = padded ? HW / Ws : 0;
+  const int c0 = blockIdx.x * 32;
+  const long long q0 = (long long)blockIdx.y * PACK_PT;
+  const long long total = (long long)N * HWd;
   // arm the completion tickets of the deterministic db reduction that consumes db_part
-  if (tickets != nullptr && (blockIdx.x | blockIdx.y | blockIdx.z) == 0)
+  if (tickets != nullptr && (blockIdx.x | blockIdx.y) == 0)
     for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const float *s = src + (size_t)n * C * HW;
-  // source pixel of each of this lane's 4 destination rows (one division per thread; the rows
-  // are 32 apart, so the padded column advances by 32 with at most one wrap when Wd > 32)
-  int spx[4];
+  const bool padded = Wd != Ws;
+  const int Hs = padded ? HW / Ws : 0;
+  // source offset (n*C*HW + pixel) of this lane's 4 rows q0 + lane + 32 i: one division, then
+  // increments (rows 32 apart; wraps handled by loops, any HWd / Wd)
+  long long soff[4];
   bool sok[4];
   {
-    const int q0 = p0 + lane;
-    int h = padded ? q0 / Wd : 0, w = padded ? q0 - h * Wd : 0;
+    const long long q = q0 + lane;
+    int n = (int)(q / HWd), p = (int)(q - (long long)n * HWd);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+    for (int i = 0; i < 4; ++i) {
+      bool ok = (q + 32 * i) < total;
+      int sp = p;
       if (padded) {
-        sok[q] = h < Hs && w < Ws;
-        spx[q] = h * Ws + w;
-        w += 32;
-        while (w >= Wd) {
-          w -= Wd;
-          ++h;
-        }
-      } else {
-        spx[q] = q0 + q * 32;
-        sok[q] = spx[q] < HW;
+        const int h = p / Wd, w = p - h * Wd;
+        ok = ok && h < Hs && w < Ws;
+        sp = h * Ws + w;
+      }
+      sok[i] = ok;
+      soff[i] = (long long)n * C * HW + sp;
+      p += 32;
+      while (p >= HWd) {
+        p -= HWd;
+        ++n;
       }
     }
   }
@@ -99,7 +105,7 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
     const int c = c0 + warp + 8 * k;
 #pragma unroll
     for (int q = 0; q < 4; ++q)
-      v[k][q] = (c < C && sok[q]) ? __ldg(s + (size_t)c * HW + spx[q]) : 0.f;
+      v[k][q] = (c < C && sok[q]) ? __ldg(src + soff[q] + (size_t)c * HW) : 0.f;
   }
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
@@ -110,21 +116,22 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
       float t = ((v[k][0] + v[k][1]) + (v[k][2] + v[k][3]));
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-      if (lane == 0) db_part[((size_t)n * gridDim.x + blockIdx.x) * C + c0 + cc] = t;
+      if (lane == 0) db_part[(size_t)blockIdx.y * C + c0 + cc] = t;
     }
   }
   __syncthreads();
-  // 16-byte chunks: lanes cover consecutive chunks of a pixel's 32-channel row (64 B bf16 /
+  // 16-byte chunks: lanes cover consecutive chunks of a row's 32-channel segment (64 B bf16 /
   // 128 B fp32), so each warp store instruction writes whole contiguous row segments.
   constexpr int CPT = 16 / ELEM;            // channels per 16-byte chunk
-  constexpr int CPP = 32 / CPT;             // chunks per pixel row of the tile
-  constexpr int PPP = 256 / CPP;            // pixels per pass
+  constexpr int CPP = 32 / CPT;             // chunks per row of the tile
+  constexpr int PPP = 256 / CPP;            // rows per pass
 #pragma unroll
   for (int pass = 0; pass < PACK_PT / PPP; ++pass) {
     const int pp = pass * PPP + threadIdx.x / CPP, j = threadIdx.x % CPP;
-    const int px = p0 + pp, cl = j * CPT, c = c0 + cl;
-    if (px < HWd && c < Cp) {
-      const size_t o = ((size_t)n * HWd + px) * Cp + c;
+    const long long q = q0 + pp;
+    const int cl = j * CPT, c = c0 + cl;
+    if (q < total && c < Cp) {
+      const size_t o = (size_t)q * Cp + c;
 #pragma unroll
       for (int u = 0; u < CPT; u += 4)
         PackOut<ELEM>::store4(dst, o + u, tile[cl + u][pp], tile[cl + u + 1][pp],
@@ -158,47 +165,43 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__re
 //   x'[n][h'][w'][c'] = x[n][c][S*h' + dh - P][S*w' + dw - P]  (0 outside),  c' = (dh*S + dw)*C + c
 // turns a stride-S, K x K conv into a stride-1, ceil(K/S) x ceil(K/S) conv over S*S*C channels
 // with the same output, so the implicit GEMM runs unit-stride im2col TMA on a dense channel axis.
-// One block per (n, h'): the S source rows are staged in shared memory (coalesced reads), then the
-// output row is written with 16-byte stores.  Dynamic smem = S*C*W floats.
+// Persistent: block b handles output rows (n, h') = b, b + grid, ...  The S*C source rows of an
+// output row are staged in shared memory (coalesced loads; the next row's loads are issued into
+// registers before the current row is written, so load latency overlaps the stores); the output
+// row is written in 16-byte chunks.  Thread -> fixed chunk j of every pixel it writes, so the
+// (source row, column phase) of its 16/ELEM channels is computed once (no per-element division).
+// Dynamic smem = S*C*W floats.  Requires Cps*ELEM/16 chunks per pixel to divide 256.
+constexpr int S2D_LD = 12;   // staged source floats per thread per row (S*C*W <= 256*S2D_LD)
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
-                                                int C, int H, int W, int S, int P, int Hs, int Ws,
-                                                int Cps) {
+                                                int N, int C, int H, int W, int S, int P, int Hs,
+                                                int Ws, int Cps) {
   extern __shared__ float rows[];   // [S*C][W] source rows (row r = dh*C + c)
+  constexpr int CH = 16 / ELEM;     // channels per 16-byte chunk
   pdl_launch_dependents();
   pdl_wait();
-  const int hs = blockIdx.x, n = blockIdx.y;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarps = blockDim.x >> 5;
-  // one warp per source row, 8 independent coalesced loads in flight per lane (no per-element
-  // index division: the row is fixed per warp iteration)
-  // (a trailing partial warp, blockDim % 32 != 0, takes no rows)
-  for (int r = warp; warp < nwarps && r < S * C; r += nwarps) {
-    const int dh = r / C, c = r - dh * C;
-    const int ih = S * hs + dh - P;
-    const bool rin = ih >= 0 && ih < H;
-    const float *src = x + (((size_t)n * C + c) * H + (rin ? ih : 0)) * W;
-    float *d = rows + r * W;
-    for (int w0 = 0; w0 < W; w0 += 256) {
-      float v[8];
+  const int tid = threadIdx.x;
+  const int RW = S * C * W;         // staged floats per output row
+  // per-thread load slots: element e = tid + 256*i of the [S*C][W] stage
+  int lsrc[S2D_LD];                 // offset in the image's x plane (c*H*W + dh*W + w), or -1
+  int ldh[S2D_LD];
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int w = w0 + lane + 32 * k;
-        v[k] = (rin && w < W) ? __ldg(src + w) : 0.f;
-      }
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int w = w0 + lane + 32 * k;
-        if (w < W) d[w] = v[k];
-      }
+  for (int i = 0; i < S2D_LD; ++i) {
+    const int e = tid + 256 * i;
+    lsrc[i] = -1;
+    ldh[i] = 0;
+    if (e < RW) {
+      const int r = e / W, w = e - r * W, dh = r / C, c = r - dh * C;
+      lsrc[i] = c * H * W + w;
+      ldh[i] = dh;
     }
   }
-  // output: thread -> fixed channel quad q (blockDim is a multiple of Cps/4), pixels strided
-  const int quads = Cps >> 2;
-  const int q = threadIdx.x % quads, wstep = blockDim.x / quads;
-  int roff[4], dws[4];
+  // per-thread store chunk: channels j*CH .. j*CH+CH-1 of pixels pl, pl + pstep, ...
+  const int cpr = Cps / CH, j = tid % cpr, pl = tid / cpr, pstep = 256 / cpr;
+  int roff[CH], dws[CH];
 #pragma unroll
-  for (int u = 0; u < 4; ++u) {
-    const int cc = 4 * q + u;
+  for (int u = 0; u < CH; ++u) {
+    const int cc = j * CH + u;
     roff[u] = -1;
     dws[u] = 0;
     if (cc < S * S * C) {
@@ -207,16 +210,39 @@ __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, voi
       dws[u] = dw - P;
     }
   }
-  __syncthreads();
-  const size_t obase = ((size_t)n * Hs + hs) * Ws;
-  for (int ws = threadIdx.x / quads; ws < Ws; ws += wstep) {
-    float v[4];
+  const int total = N * Hs;
+  float v[S2D_LD];
+  auto issue = [&](int row) {
+    const int n = row / Hs, hs = row - n * Hs;
+    const float *xb = x + (size_t)n * C * H * W;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int iw = S * ws + dws[u];
-      v[u] = (roff[u] >= 0 && iw >= 0 && iw < W) ? rows[roff[u] + iw] : 0.f;
+    for (int i = 0; i < S2D_LD; ++i) {
+      const int ih = S * hs + ldh[i] - P;
+      v[i] = (lsrc[i] >= 0 && ih >= 0 && ih < H) ? __ldg(xb + lsrc[i] + ih * W) : 0.f;
     }
-    PackOut<ELEM>::store4(dst, (obase + ws) * Cps + 4 * q, v[0], v[1], v[2], v[3]);
+  };
+  int row = blockIdx.x;
+  if (row < total) issue(row);
+  for (; row < total; row += gridDim.x) {
+#pragma unroll
+    for (int i = 0; i < S2D_LD; ++i)
+      if (tid + 256 * i < RW) rows[tid + 256 * i] = v[i];
+    __syncthreads();
+    if (row + (int)gridDim.x < total) issue(row + gridDim.x);   // next row in flight
+    const size_t obase = (size_t)row * Ws;
+    for (int ws = pl; ws < Ws; ws += pstep) {
+      float o[CH];
+#pragma unroll
+      for (int u = 0; u < CH; ++u) {
+        const int iw = S * ws + dws[u];
+        o[u] = (roff[u] >= 0 && iw >= 0 && iw < W) ? rows[roff[u] + iw] : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < CH; u += 4)
+        PackOut<ELEM>::store4(dst, (obase + ws) * Cps + j * CH + u, o[u], o[u + 1], o[u + 2],
+                              o[u + 3]);
+    }
+    __syncthreads();
   }
 }
 

@@ -168,6 +168,46 @@ glp_status_t glp_stage_bwd_filter(glp_plan_t plan, void *ws, size_t ws_bytes, gl
 glp_status_t glp_stage_reduce(glp_plan_t plan, float *dw, float *db, int accumulate, void *ws,
                               size_t ws_bytes, glp_stream_t stream);
 
+/* ---- fused sibling groups (horizontal fusion) --------------------------- *
+ * The paper runs different kernels concurrently (Eq. 9 sums over kernel kinds, P252-254) and
+ * names kernel fusion for small kernels as future work (P401).  Sibling convolutions that read
+ * the same input x with the same K, stride and pad -- e.g. GoogLeNet inception 5b's 1x1, 3x3-reduce
+ * and 5x5-reduce branches (Table 5 conv_3, conv_5, conv_6, P350-355) -- run here as ONE implicit
+ * GEMM per pass over C_out = sum C_out[b]: x is packed and read once per pass, the branches share
+ * one persistent grid.  Branch b owns output channels [sum_{a<b} C_out[a], sum_{a<=b} C_out[a]).
+ *   forward:   y_b = b_b + W_b (*) x                       (one tensor per branch)
+ *   backward:  dx  = sum_b W_b^T dy_b (col2im)              (one tensor: the branches' sum)
+ *              dW_b, db_b per branch.
+ * A group desc is an ordinary desc with C_out = sum: glp_plan / glp_plan_get_info / the single-
+ * tensor calls above apply and then read the CONCATENATED tensors (W [sum C_out][C_in][K_h][K_w],
+ * y/dy [N][sum C_out][H_o][W_o]); the *_group calls below take one pointer per branch instead.
+ * 1 <= n_branches <= 4.  Tensor-core plans require every branch but the last to have C_out a
+ * multiple of 8 (BF16) / 4 (TF32) (GLP_ERR_NOT_SUPPORTED from glp_plan otherwise); the *_group
+ * calls return GLP_ERR_NOT_SUPPORTED for GLP_MATH_FP32 plans.  Same ownership, workspace sizes
+ * (info.ws_*) and error behaviour as the single-tensor calls; results are bitwise identical to the
+ * single-tensor calls on the concatenated tensors. */
+glp_status_t glp_conv_group_desc_create(glp_conv_desc_t *out, int N, int C_in, int H, int W,
+                                        int n_branches, const int *C_out, int K_h, int K_w,
+                                        int stride_h, int stride_w, int pad_h, int pad_w);
+/* w[b], y[b] per branch; b may be NULL (no bias) or hold NULL entries. */
+glp_status_t glp_conv_group_fwd(glp_plan_t plan, const float *x, const float *const *w,
+                                const float *const *b, float *const *y, void *ws, size_t ws_bytes,
+                                glp_stream_t stream);
+/* dy[b], w[b], dw[b] per branch; dx (may be NULL) receives the sum over branches; db NULL or one
+ * pointer per branch. */
+glp_status_t glp_conv_group_bwd(glp_plan_t plan, const float *x, const float *const *dy,
+                                const float *const *w, float *dx, float *const *dw,
+                                float *const *db, int accumulate, void *ws, size_t ws_bytes,
+                                glp_stream_t stream);
+/* Staged forms: GLP_PACK_X takes src[0]; the other packs one pointer per branch.  bwd_data and
+ * bwd_filter stages are the single-tensor glp_stage_bwd_data / glp_stage_bwd_filter. */
+glp_status_t glp_stage_pack_group(glp_plan_t plan, glp_pack_t what, const float *const *src,
+                                  void *ws, size_t ws_bytes, glp_stream_t stream);
+glp_status_t glp_stage_fwd_group(glp_plan_t plan, const float *const *b, float *const *y, void *ws,
+                                 size_t ws_bytes, glp_stream_t stream);
+glp_status_t glp_stage_reduce_group(glp_plan_t plan, float *const *dw, float *const *db,
+                                    int accumulate, void *ws, size_t ws_bytes, glp_stream_t stream);
+
 /* ---- analyzer (host only, no device needed) ----------------------------------------------- */
 /* The north_star's sm_100a limits: 148 SMs, 64K regs, 228 KB smem, 2048 threads, 32 blocks,
  * + 512 TMEM columns, 1 KB smem reserved per CTA, C = 128. */

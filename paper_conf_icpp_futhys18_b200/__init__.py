@@ -57,7 +57,9 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_analyze_ctas_per_sm", "glp_analyze_samples_in_flight", "glp_analyze_eq7",
            "glp_plan_kernel_attr", "glp_status_string", "glp_last_error_string", "glp_version",
            "glp_debug_im2col", "glp_stage_pack", "glp_stage_fwd", "glp_stage_bwd_data",
-           "glp_stage_bwd_filter", "glp_stage_reduce"]
+           "glp_stage_bwd_filter", "glp_stage_reduce", "glp_conv_group_desc_create",
+           "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
+           "glp_stage_reduce_group"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA = 0, 1, 2, 3, 4
 
@@ -106,6 +108,12 @@ def lib():
         L.glp_stage_bwd_data.argtypes = [_vp, _vp, _vp, _c_size, _vp]
         L.glp_stage_bwd_filter.argtypes = [_vp, _vp, _c_size, _vp]
         L.glp_stage_reduce.argtypes = [_vp, _vp, _vp, _c_int, _vp, _c_size, _vp]
+        L.glp_conv_group_desc_create.argtypes = [P(_vp)] + [_c_int] * 5 + [_vp] + [_c_int] * 6
+        L.glp_conv_group_fwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
+        L.glp_conv_group_bwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _c_int, _vp, _c_size, _vp]
+        L.glp_stage_pack_group.argtypes = [_vp, _c_int, _vp, _vp, _c_size, _vp]
+        L.glp_stage_fwd_group.argtypes = [_vp, _vp, _vp, _vp, _c_size, _vp]
+        L.glp_stage_reduce_group.argtypes = [_vp, _vp, _vp, _c_int, _vp, _c_size, _vp]
         _lib = L
     return _lib
 
@@ -150,6 +158,15 @@ def _ptr(t):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
 
 
+def _ptrs(ts):
+    """Pointer array (const float *const *) of a list of tensors (None entries -> NULL); the
+    array object must stay alive for the duration of the call."""
+    if ts is None:
+        return None
+    arr = (ctypes.c_void_p * len(ts))(*[(None if t is None else t.data_ptr()) for t in ts])
+    return ctypes.cast(arr, ctypes.c_void_p), arr
+
+
 def _stream(stream):
     import torch
     s = stream if stream is not None else torch.cuda.current_stream()
@@ -178,15 +195,24 @@ class ConvLayer:
     ``stream`` (default: torch's current stream) without synchronising."""
 
     def __init__(self, N, C, H, W, Co, K, stride=1, pad=0, math="bf16", device=0,
-                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None):
+                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None, branches=None):
         import torch
+        self.branches = None if branches is None else [int(c) for c in branches]
+        if self.branches is not None:
+            Co = sum(self.branches)
         self.geom = Geometry(N, C, H, W, Co, K, Kw or K, stride, stride_w or stride, pad,
                              pad if pad_w is None else pad_w)
         g = self.geom
         L = lib()
         self._desc = _vp()
-        _ck(L.glp_conv_desc_create(ctypes.byref(self._desc), g.N, g.C, g.H, g.W, g.Co, g.Kh, g.Kw,
-                                   g.Sh, g.Sw, g.Ph, g.Pw), "glp_conv_desc_create")
+        if self.branches is None:
+            _ck(L.glp_conv_desc_create(ctypes.byref(self._desc), g.N, g.C, g.H, g.W, g.Co, g.Kh,
+                                       g.Kw, g.Sh, g.Sw, g.Ph, g.Pw), "glp_conv_desc_create")
+        else:
+            arr = (_c_int * len(self.branches))(*self.branches)
+            _ck(L.glp_conv_group_desc_create(ctypes.byref(self._desc), g.N, g.C, g.H, g.W,
+                                             len(self.branches), ctypes.cast(arr, _vp), g.Kh, g.Kw,
+                                             g.Sh, g.Sw, g.Ph, g.Pw), "glp_conv_group_desc_create")
         ho, wo = _c_int(), _c_int()
         _ck(L.glp_conv_desc_get_output(self._desc, ctypes.byref(ho), ctypes.byref(wo)),
             "glp_conv_desc_get_output")
@@ -274,6 +300,48 @@ class ConvLayer:
         _ck(lib().glp_stage_reduce(self._plan, _ptr(dw), _ptr(db), int(bool(accumulate)),
                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_stage_reduce")
+
+    # fused sibling groups (include/glp.h "fused sibling groups"): one tensor per branch
+    def branch_y_shapes(self):
+        return [(self.geom.N, c, self.Ho, self.Wo) for c in self.branches]
+
+    def branch_w_shapes(self):
+        g = self.geom
+        return [(c, g.C, g.Kh, g.Kw) for c in self.branches]
+
+    def group_fwd(self, x, ws, bs, ys, stream=None):
+        (pw, _a), (py, _b) = _ptrs(ws), _ptrs(ys)
+        pb = _ptrs(bs)
+        _ck(lib().glp_conv_group_fwd(self._plan, _ptr(x), pw, None if pb is None else pb[0], py,
+                                     ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_conv_group_fwd")
+        return ys
+
+    def group_bwd(self, x, dys, ws, dx, dws, dbs=None, accumulate=False, stream=None):
+        (pdy, _a), (pw, _b), (pdw, _c) = _ptrs(dys), _ptrs(ws), _ptrs(dws)
+        pdb = _ptrs(dbs)
+        _ck(lib().glp_conv_group_bwd(self._plan, _ptr(x), pdy, pw, _ptr(dx), pdw,
+                                     None if pdb is None else pdb[0], int(bool(accumulate)),
+                                     ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_conv_group_bwd")
+        return dx, dws, dbs
+
+    def stage_pack_group(self, what, srcs, stream=None):
+        p, _a = _ptrs(srcs)
+        _ck(lib().glp_stage_pack_group(self._plan, int(what), p, ctypes.c_void_p(self.ws_ptr),
+                                       self.ws_bytes, _stream(stream)), "glp_stage_pack_group")
+
+    def stage_fwd_group(self, bs, ys, stream=None):
+        pb, (py, _a) = _ptrs(bs), _ptrs(ys)
+        _ck(lib().glp_stage_fwd_group(self._plan, None if pb is None else pb[0], py,
+                                      ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_stage_fwd_group")
+
+    def stage_reduce_group(self, dws, dbs=None, accumulate=False, stream=None):
+        (pdw, _a), pdb = _ptrs(dws), _ptrs(dbs)
+        _ck(lib().glp_stage_reduce_group(self._plan, pdw, None if pdb is None else pdb[0],
+                                         int(bool(accumulate)), ctypes.c_void_p(self.ws_ptr),
+                                         self.ws_bytes, _stream(stream)), "glp_stage_reduce_group")
 
     def debug_im2col(self, x, n, col, stream=None):
         _ck(lib().glp_debug_im2col(self._plan, _ptr(x), int(n), _ptr(col),

@@ -44,6 +44,27 @@ struct Gather {
   int cbs;               // channel blocks (of the K-block width) per tap, fwd/dgrad
 };
 
+// Output channel c of a horizontally fused sibling group (convolutions that
+// read the same x with the same K/S/P, run as one GEMM over C_o = sum of the branches) -> the
+// branch tensor it belongs to.  n = 1: a single layer, p[0] holds every channel.
+constexpr int GLP_MAXBR = 4;
+struct BrOut {
+  int n;
+  int off[GLP_MAXBR + 1];   // first channel of each branch; off[n] = total channels
+  float *p[GLP_MAXBR];
+  __host__ __device__ __forceinline__ int branch(int c) const {
+    int b = 0;
+    for (int k = 1; k < GLP_MAXBR; ++k) b += (k < n && c >= off[k]) ? 1 : 0;
+    return b;
+  }
+  // element (plane q) of channel c in a [rows][C_b][plane] branch tensor, e.g. dW (rows = 1,
+  // plane = C*K*K), db (plane = 1), y (rows = N, plane = H_o*W_o)
+  __host__ __device__ __forceinline__ float *at(int c, size_t row, size_t plane, size_t q) const {
+    const int b = branch(c);
+    return p[b] + (row * (size_t)(off[b + 1] - off[b]) + (size_t)(c - off[b])) * plane + q;
+  }
+};
+
 struct IgemmParams {
   Gather g;
   int M, N;              // valid GEMM extents
@@ -59,6 +80,8 @@ struct IgemmParams {
   float *out;            // y (fwd) / dx (dgrad) NCHW, or split partials (wgrad)
   const float *bias;     // fwd only, may be null
   int bias_floats;       // fwd: floats of the smem bias stage (>= n_tiles*bn rounded to 32)
+  BrOut ybr;             // fwd of a fused sibling group (ybr.n > 1): per-branch y tensors
+  const float *bias_br[GLP_MAXBR];   // and per-branch biases (each may be null)
   int out_c;             // channels of out (C_o fwd, C_i dgrad)
   int out_hw;            // H_o*W_o (fwd) / H*W (dgrad)
   int part_ld;           // wgrad partial leading dimension (n_tiles * bn)

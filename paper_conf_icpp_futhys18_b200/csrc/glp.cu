@@ -55,10 +55,25 @@ inline long long cdiv(long long a, long long b) { return (a + b - 1) / b; }
 inline long long rup(long long a, long long b) { return cdiv(a, b) * b; }
 inline size_t align1k(size_t a) { return (a + 1023) & ~size_t(1023); }
 
+// per-branch input pointers of a fused sibling group call (n = 1: one tensor, every channel)
+struct BrIn {
+  int n = 1;
+  const float *p[GLP_MAXBR] = {nullptr, nullptr, nullptr, nullptr};
+};
+inline BrIn br_in1(const float *a) {
+  BrIn b;
+  b.p[0] = a;
+  return b;
+}
+
 }  // namespace
 
 struct glp_conv_desc_s {
   int N, C, H, W, Co, Kh, Kw, Sh, Sw, Ph, Pw, Ho, Wo;
+  // fused sibling group (glp_conv_group_desc_create): nbr branches, branch b owns output
+  // channels [br_off[b], br_off[b+1]) of the C_o = sum view; single layer: nbr = 1
+  int nbr = 1;
+  int br_off[GLP_MAXBR + 1] = {0, 0, 0, 0, 0};
 };
 
 namespace {
@@ -634,9 +649,11 @@ DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
 
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
                              int Cp, float *db_part, cudaStream_t st, int Ws = 1, int Wd = 1,
-                             int HWd = -1) {
+                             int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1) {
   if (HWd < 0) HWd = HW;   // default: dense destination (Ws == Wd)
-  if (db_part == nullptr && Cp * P.elem <= 32 && Ws == Wd) {
+  if (Cw < 0) Cw = Cp;     // default: the whole row (single layer)
+  if (db_ld < 0) db_ld = C;
+  if (db_part == nullptr && Cp * P.elem <= 32 && Ws == Wd && co_off == 0 && Cw == Cp) {
     const size_t n = (size_t)P.d.N * HW;
     const int g = (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 32);
     if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp));
@@ -644,32 +661,46 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
-  dim3 grid((unsigned)cdiv(Cp, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
+  dim3 grid((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
   const int nt = (int)cdiv(P.d.Co, 32);
-  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
-  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd));
+  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld));
+  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
 }
 
 // dy -> its packed operand (dense NHWC, or on the padded dxg grid for halo plans) + db partials
-glp_status_t launch_pack_dy(const glp_plan_s &P, const float *dy, uint8_t *ws, bool with_db,
+// A fused sibling group (dy.n > 1) packs branch b into channels [off_b, off_b+1) of the rows
+// (the last branch also zero-fills the pitch padding) with its db partials in columns off_b + c.
+glp_status_t launch_pack_dy(const glp_plan_s &P, const BrIn &dy, uint8_t *ws, bool with_db,
                             cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   float *dbp = with_db ? reinterpret_cast<float *>(ws + P.off_dbpart) : nullptr;
-  if (P.halo)
-    return launch_pack_act(P, dy, ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, d.Wo,
-                           P.dxg.W, P.dxg.H * P.dxg.W);
-  return launch_pack_act(P, dy, ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st);
+  const int Ws = P.halo ? d.Wo : 1, Wd = P.halo ? P.dxg.W : 1;
+  const int HWd = P.halo ? P.dxg.H * P.dxg.W : -1;
+  if (dy.n <= 1)
+    return launch_pack_act(P, dy.p[0], ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
+                           HWd);
+  for (int b = 0; b < dy.n; ++b) {
+    const int off = d.br_off[b], cb = d.br_off[b + 1] - off;
+    const int cw = (b == dy.n - 1) ? P.Cop - off : cb;
+    glp_status_t s = launch_pack_act(P, dy.p[b], ws + P.off_dypk, cb, d.Ho * d.Wo, P.Cop, dbp, st,
+                                     Ws, Wd, HWd, off, cw, d.Co);
+    if (s) return s;
+  }
+  return GLP_OK;
 }
 
 int ew_grid(size_t n) { return (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 16); }
 
-glp_status_t run_pack_w_fwd(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
-  const glp_conv_desc_s &d = P.d;
-  void *wpk = ws + P.off_wpk;
+glp_status_t run_pack_w_fwd_one(glp_plan_s &P, const float *w, int co_off, int Co, uint8_t *ws,
+                                cudaStream_t st) {
+  const glp_conv_desc_s &d0 = P.d;
+  glp_conv_desc_s d = d0;
+  d.Co = Co;   // rows [co_off, co_off + Co) of the forward B operand
+  void *wpk = ws + P.off_wpk + (size_t)co_off * P.fwd.Kpad * P.elem;
   const size_t wn = (size_t)d.Co * P.fwd.Kpad;
   if (P.s2d) {
     if (P.elem == 2)
@@ -682,6 +713,16 @@ glp_status_t run_pack_w_fwd(glp_plan_s &P, const float *w, uint8_t *ws, cudaStre
     GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<4>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad));
   }
   GLP_LAUNCH_CHECK("pack_w_fwd");
+  return GLP_OK;
+}
+
+glp_status_t run_pack_w_fwd(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  if (w.n <= 1) return run_pack_w_fwd_one(P, w.p[0], 0, d.Co, ws, st);
+  for (int b = 0; b < w.n; ++b) {
+    glp_status_t s = run_pack_w_fwd_one(P, w.p[b], d.br_off[b], d.br_off[b + 1] - d.br_off[b], ws, st);
+    if (s) return s;
+  }
   return GLP_OK;
 }
 
@@ -706,19 +747,43 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
   return launch_pack_act(P, x, dst, d.C, d.H * d.W, P.Cpx, nullptr, st);
 }
 
-glp_status_t run_pack_w_dgrad(glp_plan_s &P, const float *w, uint8_t *ws, cudaStream_t st) {
+glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   void *wtpk = ws + P.off_wtpk;
   const int flip = P.dgrad.a_tma;  // the im2col-TMA dgrad walks taps flipped
-  if (P.elem == 2)
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, dim3(dim3((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C)), dim3(256), 0, st, w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip));
-  else
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, dim3(dim3((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C)), dim3(256), 0, st, w, wtpk, d.Co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip));
-  GLP_LAUNCH_CHECK("pack_w_dgrad");
+  const dim3 grid((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C);
+  const int n = std::max(1, w.n);
+  for (int b = 0; b < n; ++b) {
+    const int off = n > 1 ? d.br_off[b] : 0;
+    const int co = n > 1 ? d.br_off[b + 1] - off : d.Co;
+    const int hi = (b == n - 1) ? P.Cop : off + co;
+    if (P.elem == 2)
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+    else
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+    GLP_LAUNCH_CHECK("pack_w_dgrad");
+  }
   return GLP_OK;
 }
 
-glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, cudaStream_t st) {
+// output table of a call: n = 1 -> every channel in p[0]; fused group -> the plan's branches
+BrOut br_out(const glp_plan_s &P, int n, float *const *ptrs) {
+  BrOut t;
+  memset(&t, 0, sizeof(t));
+  if (n <= 1) {
+    t.n = 1;
+    t.off[1] = P.d.Co;
+    t.p[0] = ptrs[0];
+    return t;
+  }
+  t.n = n;
+  for (int b = 0; b <= n; ++b) t.off[b] = P.d.br_off[b];
+  for (int b = 0; b < n; ++b) t.p[b] = ptrs[b];
+  return t;
+}
+
+glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
+                          cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
   const PassPlan &pp = P.fwd;
   void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
@@ -736,8 +801,10 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const float *b, float *y, uint8_t *ws, 
     if (s) return s;
   }
   IgemmParams p = make_params(P, pp, MODE_FWD, xpk);
-  p.out = y;
-  p.bias = b;
+  p.out = y.p[0];
+  p.bias = b.p[0];
+  p.ybr = y;
+  for (int i = 0; i < GLP_MAXBR; ++i) p.bias_br[i] = b.p[i];
   p.bias_floats = pp.bias_floats;
   p.out_c = d.Co;
   p.out_hw = d.Ho * d.Wo;
@@ -825,8 +892,8 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   return launch_igemm<MODE_WGRAD>(P, pp, p, mapB, mapA, st);
 }
 
-glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulate, uint8_t *ws,
-                              cudaStream_t st) {
+glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw, const BrOut *db, int accumulate,
+                              uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
   if (P.halo) {
@@ -845,10 +912,32 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, float *dw, float *db, int accumulat
   if (db) {
     DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
     GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), dim3(256), 0,
-                        st, a.part, db, d.Co, P.db_rows, accumulate, a.part2, a.tickets));
+                        st, a.part, *db, d.Co, P.db_rows, accumulate, a.part2, a.tickets));
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
+}
+
+// Composed tensor-core passes (single layer: one-entry tables; fused group: one per branch).
+glp_status_t tc_fwd(glp_plan_s &P, const float *x, const BrIn &w, const BrIn &b, const BrOut &y,
+                    uint8_t *ws, cudaStream_t st) {
+  glp_status_t s = launch_pack_x(P, x, ws + P.off_xpk, st);
+  if (s) return s;
+  if ((s = run_pack_w_fwd(P, w, ws, st))) return s;
+  return run_fwd_gemm(P, b, y, ws, st);
+}
+glp_status_t tc_bwd(glp_plan_s &P, const float *x, const BrIn &dy, const BrIn &w, float *dx,
+                    const BrOut &dw, const BrOut &db, bool with_db, int accumulate, uint8_t *ws,
+                    cudaStream_t st) {
+  glp_status_t s = launch_pack_dy(P, dy, ws, with_db, st);
+  if (s) return s;
+  if (dx) {
+    if ((s = run_pack_w_dgrad(P, w, ws, st))) return s;
+    if ((s = run_dgrad_gemm(P, dx, ws, st))) return s;
+  }
+  if ((s = launch_pack_x(P, x, ws + P.off_xpk, st))) return s;
+  if ((s = run_wgrad_gemm(P, ws, st))) return s;
+  return run_wgrad_reduce(P, dw, with_db ? &db : nullptr, accumulate, ws, st);
 }
 
 ConvGeom geom(const glp_conv_desc_s &d) {
@@ -870,8 +959,9 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
     GLP_LAUNCH_CHECK("simt_db_partial");
     DbAux a = db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.simt_splits);
     GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
+    float *dbs[1] = {db};
     reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), 256, 0, st>>>(
-        a.part, db, d.Co, P.simt_splits, accumulate, a.part2, a.tickets);
+        a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
@@ -937,6 +1027,28 @@ glp_status_t glp_conv_desc_create(glp_conv_desc_t *out, int N, int C, int H, int
     return fail(GLP_ERR_NOT_SUPPORTED, "tensor too large for 32-bit indexing");
   auto *d = new glp_conv_desc_s{N, C, H, W, Co, Kh, Kw, Sh, Sw, Ph, Pw, (int)Ho, (int)Wo};
   *out = d;
+  return GLP_OK;
+}
+
+glp_status_t glp_conv_group_desc_create(glp_conv_desc_t *out, int N, int C, int H, int W,
+                                        int n_branches, const int *C_out, int Kh, int Kw, int Sh,
+                                        int Sw, int Ph, int Pw) {
+  if (!out || !C_out) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *out = nullptr;
+  if (n_branches < 1 || n_branches > GLP_MAXBR)
+    return fail(GLP_ERR_INVALID_VALUE, "n_branches must be 1.." + std::to_string(GLP_MAXBR));
+  long long tot = 0;
+  for (int b = 0; b < n_branches; ++b) {
+    if (C_out[b] <= 0) return fail(GLP_ERR_INVALID_VALUE, "non-positive branch C_out");
+    tot += C_out[b];
+  }
+  if (tot >= (1LL << 30)) return fail(GLP_ERR_INVALID_VALUE, "C_out too large");
+  glp_status_t s = glp_conv_desc_create(out, N, C, H, W, (int)tot, Kh, Kw, Sh, Sw, Ph, Pw);
+  if (s) return s;
+  glp_conv_desc_s *d = *out;
+  d->nbr = n_branches;
+  d->br_off[0] = 0;
+  for (int b = 0; b < n_branches; ++b) d->br_off[b + 1] = d->br_off[b] + C_out[b];
   return GLP_OK;
 }
 
@@ -1064,6 +1176,17 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   L.smem_reserved_per_cta = (int)prop.reservedSharedMemPerBlock;
 
   glp_status_t s = GLP_OK;
+  if (d->nbr > 1 && math != GLP_MATH_FP32) {
+    // a branch's packed channels start on a 16-byte chunk of the pitch (8 bf16 / 4 tf32)
+    const int ch = 16 / P->elem;
+    for (int b = 1; b < d->nbr; ++b)
+      if (d->br_off[b] % ch) {
+        delete P;
+        if (cur != device) cudaSetDevice(cur);
+        return fail(GLP_ERR_NOT_SUPPORTED, "fused group: every branch but the last needs C_out % " +
+                                               std::to_string(ch) + " == 0");
+      }
+  }
   if (math != GLP_MATH_FP32) {
     if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
         (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {
@@ -1190,10 +1313,8 @@ glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const fl
     return GLP_OK;
   }
   if ((s = get_encode())) return s;
-  uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if ((s = launch_pack_x(*P, x, wsb + P->off_xpk, st))) return s;
-  if ((s = run_pack_w_fwd(*P, w, wsb, st))) return s;
-  return run_fwd_gemm(*P, b, y, wsb, st);
+  float *ys[1] = {y};
+  return tc_fwd(*P, x, br_in1(w), br_in1(b), br_out(*P, 1, ys), static_cast<uint8_t *>(ws), st);
 }
 
 glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, float *dx, void *ws,
@@ -1211,8 +1332,8 @@ glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, fl
   }
   if ((s = get_encode())) return s;
   uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if ((s = launch_pack_dy(*P, dy, wsb, false, st))) return s;
-  if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
+  if ((s = launch_pack_dy(*P, br_in1(dy), wsb, false, st))) return s;
+  if ((s = run_pack_w_dgrad(*P, br_in1(w), wsb, st))) return s;
   return run_dgrad_gemm(*P, dx, wsb, st);
 }
 
@@ -1229,9 +1350,11 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   if ((s = get_encode())) return s;
   void *xpk = wsb + P->off_xpk;
   if ((s = launch_pack_x(*P, x, xpk, st))) return s;
-  if ((s = launch_pack_dy(*P, dy, wsb, db != nullptr, st))) return s;
+  if ((s = launch_pack_dy(*P, br_in1(dy), wsb, db != nullptr, st))) return s;
   if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
-  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
+  float *dws[1] = {dw}, *dbs[1] = {db};
+  const BrOut dbt = br_out(*P, 1, dbs);
+  return run_wgrad_reduce(*P, br_out(*P, 1, dws), db ? &dbt : nullptr, accumulate ? 1 : 0, wsb, st);
 }
 
 glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const float *w, float *dx,
@@ -1254,15 +1377,9 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
     return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
   }
   if ((s = get_encode())) return s;
-  void *xpk = wsb + P->off_xpk;
-  if ((s = launch_pack_dy(*P, dy, wsb, db != nullptr, st))) return s;
-  if (dx) {
-    if ((s = run_pack_w_dgrad(*P, w, wsb, st))) return s;
-    if ((s = run_dgrad_gemm(*P, dx, wsb, st))) return s;
-  }
-  if ((s = launch_pack_x(*P, x, xpk, st))) return s;
-  if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
-  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, wsb, st);
+  float *dws[1] = {dw}, *dbs[1] = {db};
+  return tc_bwd(*P, x, br_in1(dy), br_in1(w), dx, br_out(*P, 1, dws), db ? br_out(*P, 1, dbs) : BrOut{},
+                db != nullptr, accumulate ? 1 : 0, wsb, st);
 }
 
 static glp_status_t stage_check(glp_plan_t P, void *ws, size_t ws_bytes) {
@@ -1284,11 +1401,11 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
     case GLP_PACK_X:
       return launch_pack_x(*P, src, wsb + P->off_xpk, st);
     case GLP_PACK_DY:
-      return launch_pack_dy(*P, src, wsb, false, st);
+      return launch_pack_dy(*P, br_in1(src), wsb, false, st);
     case GLP_PACK_DY_DB:
-      return launch_pack_dy(*P, src, wsb, true, st);
-    case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, src, wsb, st);
-    case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, src, wsb, st);
+      return launch_pack_dy(*P, br_in1(src), wsb, true, st);
+    case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, br_in1(src), wsb, st);
+    case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, br_in1(src), wsb, st);
   }
   return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
 }
@@ -1298,7 +1415,9 @@ glp_status_t glp_stage_fwd(glp_plan_t P, const float *b, float *y, void *ws, siz
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
   if ((s = validate_ptrs({y}))) return s;
-  return run_fwd_gemm(*P, b, y, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+  float *ys[1] = {y};
+  return run_fwd_gemm(*P, br_in1(b), br_out(*P, 1, ys), static_cast<uint8_t *>(ws),
+                      static_cast<cudaStream_t>(stream));
 }
 
 glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_bytes,
@@ -1320,8 +1439,112 @@ glp_status_t glp_stage_reduce(glp_plan_t P, float *dw, float *db, int accumulate
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
   if ((s = validate_ptrs({dw}))) return s;
-  return run_wgrad_reduce(*P, dw, db, accumulate ? 1 : 0, static_cast<uint8_t *>(ws),
-                          static_cast<cudaStream_t>(stream));
+  float *dws[1] = {dw}, *dbs[1] = {db};
+  const BrOut dbt = br_out(*P, 1, dbs);
+  return run_wgrad_reduce(*P, br_out(*P, 1, dws), db ? &dbt : nullptr, accumulate ? 1 : 0,
+                          static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+}
+
+// ---- fused sibling groups ----
+static glp_status_t group_tables(glp_plan_t P, const float *const *in, BrIn &t, bool allow_null_entries) {
+  t.n = P->d.nbr;
+  for (int b = 0; b < t.n; ++b) {
+    t.p[b] = in ? in[b] : nullptr;
+    if (!allow_null_entries && !t.p[b]) return fail(GLP_ERR_INVALID_VALUE, "NULL branch tensor");
+    if (t.p[b] && reinterpret_cast<uintptr_t>(t.p[b]) % 4) return fail(GLP_ERR_INVALID_VALUE, "misaligned branch tensor");
+  }
+  return GLP_OK;
+}
+static glp_status_t group_check(glp_plan_t P, void *ws, size_t ws_bytes, size_t need) {
+  if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
+  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "fused groups need a tensor-core plan");
+  glp_status_t s = check_ws(P, ws, ws_bytes, need);
+  if (s) return s;
+  return get_encode();
+}
+static BrOut group_out(glp_plan_t P, float *const *p) {
+  float *q[GLP_MAXBR] = {nullptr, nullptr, nullptr, nullptr};
+  for (int b = 0; b < P->d.nbr; ++b) q[b] = p[b];
+  return br_out(*P, P->d.nbr, q);
+}
+
+glp_status_t glp_conv_group_fwd(glp_plan_t P, const float *x, const float *const *w,
+                                const float *const *b, float *const *y, void *ws, size_t ws_bytes,
+                                glp_stream_t stream) {
+  glp_status_t s = group_check(P, ws, ws_bytes, P ? P->ws_fwd : 0);
+  if (s) return s;
+  if (!w || !y || (s = validate_ptrs({x}))) return s ? s : fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  BrIn wt, bt, yt;
+  if ((s = group_tables(P, w, wt, false)) || (s = group_tables(P, b, bt, true)) ||
+      (s = group_tables(P, y, yt, false)))
+    return s;
+  return tc_fwd(*P, x, wt, bt, group_out(P, y), static_cast<uint8_t *>(ws),
+                static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_conv_group_bwd(glp_plan_t P, const float *x, const float *const *dy,
+                                const float *const *w, float *dx, float *const *dw,
+                                float *const *db, int accumulate, void *ws, size_t ws_bytes,
+                                glp_stream_t stream) {
+  glp_status_t s = group_check(P, ws, ws_bytes, P ? P->ws_bwd : 0);
+  if (s) return s;
+  if (!dy || !w || !dw || (s = validate_ptrs({x}))) return s ? s : fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  if (dx && (reinterpret_cast<uintptr_t>(dx) % 16)) return fail(GLP_ERR_INVALID_VALUE, "dx misaligned");
+  BrIn dyt, wt, dwt, dbt;
+  if ((s = group_tables(P, dy, dyt, false)) || (s = group_tables(P, w, wt, false)) ||
+      (s = group_tables(P, reinterpret_cast<const float *const *>(dw), dwt, false)) ||
+      (db && (s = group_tables(P, reinterpret_cast<const float *const *>(db), dbt, false))))
+    return s;
+  return tc_bwd(*P, x, dyt, wt, dx, group_out(P, dw), db ? group_out(P, db) : BrOut{}, db != nullptr,
+                accumulate ? 1 : 0, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_stage_pack_group(glp_plan_t P, glp_pack_t what, const float *const *src, void *ws,
+                                  size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if (!src) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  if (what == GLP_PACK_X) {
+    if ((s = validate_ptrs({src[0]}))) return s;
+    return launch_pack_x(*P, src[0], wsb + P->off_xpk, st);
+  }
+  BrIn t;
+  if ((s = group_tables(P, src, t, false))) return s;
+  switch (what) {
+    case GLP_PACK_DY: return launch_pack_dy(*P, t, wsb, false, st);
+    case GLP_PACK_DY_DB: return launch_pack_dy(*P, t, wsb, true, st);
+    case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, t, wsb, st);
+    case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, t, wsb, st);
+    default: break;
+  }
+  return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
+}
+
+glp_status_t glp_stage_fwd_group(glp_plan_t P, const float *const *b, float *const *y, void *ws,
+                                 size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if (!y) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  BrIn bt, yt;
+  if ((s = group_tables(P, b, bt, true)) || (s = group_tables(P, y, yt, false))) return s;
+  return run_fwd_gemm(*P, bt, group_out(P, y), static_cast<uint8_t *>(ws),
+                      static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_stage_reduce_group(glp_plan_t P, float *const *dw, float *const *db, int accumulate,
+                                    void *ws, size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if (!dw) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  BrIn dwt, dbt;
+  if ((s = group_tables(P, reinterpret_cast<const float *const *>(dw), dwt, false)) ||
+      (db && (s = group_tables(P, reinterpret_cast<const float *const *>(db), dbt, false))))
+    return s;
+  const BrOut dbo = db ? group_out(P, db) : BrOut{};
+  return run_wgrad_reduce(*P, group_out(P, dw), db ? &dbo : nullptr, accumulate ? 1 : 0,
+                          static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
 }
 
 glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, void *ws,

@@ -526,8 +526,18 @@ __global__ void __launch_bounds__(288, 1)
     // load had its latency exposed in every chunk of every tile (ncu: STS waiting on LDG)
     const uint32_t sbias = (tmem_slot + 16u + 15u) & ~15u;
     if (MODE == MODE_FWD) {
-      for (int i = row; i < p.bias_floats; i += 128)
-        sts_f32(sbias + 4u * (uint32_t)i, (p.bias != nullptr && i < p.N) ? __ldg(p.bias + i) : 0.f);
+      for (int i = row; i < p.bias_floats; i += 128) {
+        float bv = 0.f;
+        if (i < p.N) {
+          if (p.ybr.n > 1) {
+            const int b = p.ybr.branch(i);
+            if (p.bias_br[b] != nullptr) bv = __ldg(p.bias_br[b] + (i - p.ybr.off[b]));
+          } else if (p.bias != nullptr) {
+            bv = __ldg(p.bias + i);
+          }
+        }
+        sts_f32(sbias + 4u * (uint32_t)i, bv);
+      }
       named_bar_sync(1, 128);
     }
     const bool clk = p.dbg_clk != nullptr && warp == 0;
@@ -564,7 +574,22 @@ __global__ void __launch_bounds__(288, 1)
           if (clk) e_ld += clock64() - c1;
           const int lim = min(32, min(p.bn - c0, p.N - n0 - c0));
           float *o = ob + (size_t)c0 * plane;
-          if (mv && lim == 32) {
+          bool split_chunk = false;   // fused group: the chunk straddles two branch tensors
+          if (MODE == MODE_FWD && p.ybr.n > 1 && lim > 0) {
+            const int cf = n0 + c0;
+            const int b = p.ybr.branch(cf);
+            split_chunk = p.ybr.branch(cf + lim - 1) != b;
+            o = p.ybr.at(cf, n, plane, pimg);
+          }
+          if (MODE == MODE_FWD && split_chunk) {
+            if (mv) {
+#pragma unroll
+              for (int q = 0; q < 32; ++q)
+                if (q < lim)
+                  *p.ybr.at(n0 + c0 + q, n, plane, pimg) =
+                      __uint_as_float(v[q]) + lds_f32(sb_tile + 4u * (uint32_t)(c0 + q));
+            }
+          } else if (mv && lim == 32) {
 #pragma unroll
             for (int q = 0; q < 32; q += 4) {
               float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);

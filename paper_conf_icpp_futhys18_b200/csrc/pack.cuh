@@ -61,7 +61,11 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
                                                          void *__restrict__ dst, int N, int C,
                                                          int HW, int Cp, float *__restrict__ db_part,
                                                          unsigned int *__restrict__ tickets,
-                                                         int n_tickets, int Ws, int Wd, int HWd) {
+                                                         int n_tickets, int Ws, int Wd, int HWd,
+                                                         int co_off, int Cw, int db_ld) {
+  // (co_off, Cw, db_ld): this call writes destination channels [co_off, co_off + Cw) of rows with
+  // pitch Cp (source channels 0..C-1, zeros past C) and db_part columns co_off + c of width db_ld —
+  // one branch of a fused sibling group.  Single layer: co_off = 0, Cw = Cp, db_ld = C.
   __shared__ float tile[32][PACK_PT + 1];
   pdl_launch_dependents();
   pdl_wait();
@@ -116,7 +120,7 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
       float t = ((v[k][0] + v[k][1]) + (v[k][2] + v[k][3]));
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-      if (lane == 0) db_part[(size_t)blockIdx.y * C + c0 + cc] = t;
+      if (lane == 0) db_part[(size_t)blockIdx.y * db_ld + co_off + c0 + cc] = t;
     }
   }
   __syncthreads();
@@ -130,8 +134,8 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
     const int pp = pass * PPP + threadIdx.x / CPP, j = threadIdx.x % CPP;
     const long long q = q0 + pp;
     const int cl = j * CPT, c = c0 + cl;
-    if (q < total && c < Cp) {
-      const size_t o = (size_t)q * Cp + c;
+    if (q < total && c < Cw) {
+      const size_t o = (size_t)q * Cp + co_off + c;
 #pragma unroll
       for (int u = 0; u < CPT; u += 4)
         PackOut<ELEM>::store4(dst, o + u, tile[cl + u][pp], tile[cl + u + 1][pp],
@@ -286,17 +290,22 @@ __global__ void __launch_bounds__(256) pack_w_fwd(const float *__restrict__ w, v
 // W [Co][C][Kh][Kw] -> backward-data B operand Wt[ci][tap*Cop + co] (row length Kpad).
 // flip = 1: tap index reversed (tap' = taps-1-tap, i.e. (Kh-1-kh, Kw-1-kw)) for the im2col-TMA
 // dgrad, which walks dy from the window's top-left corner.
+// Fused sibling group: this call owns fused output channels [co_lo, co_hi) of the K index,
+// holding branch channels co - co_off (< Co) and zeros past them; single layer: co_off = co_lo =
+// 0, co_hi = Cop.
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out,
                                                     int Co, int C, int taps, int Cop, int Kpad,
-                                                    int flip) {
+                                                    int flip, int co_off, int co_lo, int co_hi) {
   pdl_launch_dependents();
   pdl_wait();
   const int ci = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= Kpad) return;
   const int t = k / Cop, co = k - t * Cop;
-  const float v = (t < taps && co < Co)
-                      ? __ldg(w + ((size_t)co * C + ci) * taps + (flip ? taps - 1 - t : t))
+  if (t < taps && (co < co_lo || co >= co_hi)) return;   // another branch's channels
+  const int cb = co - co_off;
+  const float v = (t < taps && cb < Co)
+                      ? __ldg(w + ((size_t)cb * C + ci) * taps + (flip ? taps - 1 - t : t))
                       : 0.f;
   PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
 }

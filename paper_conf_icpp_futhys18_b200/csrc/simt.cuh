@@ -4,6 +4,8 @@
 #pragma once
 #include <cstdint>
 
+#include "common.cuh"
+
 namespace glp {
 
 struct ConvGeom {
@@ -163,7 +165,7 @@ __global__ void reduce_simt_dw(const float *__restrict__ part, float *__restrict
 // shared memory, and dW[co][i] is written 32 consecutive i at a time.  grid (ceil(C*taps/32),
 // ceil(Co/32)).
 __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ part,
-                                                    float *__restrict__ dw, int Co, int C,
+                                                    const BrOut dw, int Co, int C,
                                                     int taps, int Kw, int Cp, int ld, int mpad,
                                                     int splits, int accumulate, int s2d, int Ks) {
   __shared__ float tile[32][33];
@@ -212,9 +214,9 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
   for (int j = ty; j < 32; j += 8) {
     const int co = co0 + j, i = i0 + lane;
     if (co < Co && i < inner) {
-      const size_t idx = (size_t)co * inner + i;
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i);
       const float v = tile[lane][j];
-      dw[idx] = accumulate ? dw[idx] + v : v;
+      *d = accumulate ? *d + v : v;
     }
   }
 }
@@ -223,7 +225,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
 // 8 split phases over 4 weight rows; thread (ty, lane) sums splits ty, ty+8, ... in ascending order,
 // then the 8 phase sums are added in phase order.  Fixed order, a function of `splits` only.
 __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict__ part,
-                                                         float *__restrict__ dw, int Co, int C,
+                                                         const BrOut dw, int Co, int C,
                                                          int taps, int Kw, int Cp, int ld, int mpad,
                                                          int splits, int accumulate, int s2d, int Ks) {
   __shared__ float red[8][4][33];
@@ -267,8 +269,8 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
     for (int k = 0; k < 8; ++k) t += red[k][u][lane];
     const int i = i0 + u;
     if (i < inner && co < Co) {
-      const size_t idx = (size_t)co * inner + i;
-      dw[idx] = accumulate ? dw[idx] + t : t;
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i);
+      *d = accumulate ? *d + t : t;
     }
   }
 }
@@ -281,7 +283,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
 // The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
 constexpr int DB_GROUPS = 64;
 __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
-                                                 float *__restrict__ db, int Co, int rows,
+                                                 const BrOut db, int Co, int rows,
                                                  int accumulate, float *__restrict__ part2,
                                                  unsigned int *__restrict__ tickets) {
   __shared__ float red[8][33];
@@ -309,7 +311,8 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
     if (co < Co) {
       float s = 0.f;
       for (int k = 0; k < DB_GROUPS; ++k) s += __ldcg(part2 + (size_t)k * Co + co);
-      db[co] = accumulate ? db[co] + s : s;
+      float *d = db.at(co, 0, 1, 0);
+      *d = accumulate ? *d + s : s;
     }
     if (lane == 0) tickets[blockIdx.x] = 0;   // re-arm for the next call on this workspace
   }

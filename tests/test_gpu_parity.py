@@ -304,3 +304,96 @@ def test_halo_wgrad_random_and_invariant(shape):
         assert np.abs(runs[0][k] - e).max() / np.abs(e).max() <= 1e-4, k
         for other in runs[1:]:
             np.testing.assert_array_equal(other[k], runs[0][k], err_msg=k)
+
+
+# fused sibling groups (include/glp.h): name, N, C, H, W, branches, K, S, P
+GROUPS = [
+    ("gnet_5b_1x1_siblings", 4, 832, 7, 7, [384, 192, 48], 1, 1, 0),
+    ("k3_three_branches", 3, 64, 9, 11, [40, 24, 20], 3, 1, 1),
+    ("k5_two_branches_ragged", 2, 32, 12, 12, [16, 50], 5, 1, 2),
+]
+
+
+def _group_data(g, exact, seed):
+    _, N, C, H, W, br, K, S, P = g
+    d = _data((None, N, C, H, W, sum(br), K, S, P), exact=exact, seed=seed)
+    offs = np.cumsum([0] + br)
+    split = lambda a, axis: [np.ascontiguousarray(np.take(a, range(offs[i], offs[i + 1]), axis=axis))
+                             for i in range(len(br))]
+    return d, split(d["w"], 0), split(d["b"], 0), split(d["dy"], 1)
+
+
+def _group_run(layer, x, ws, bs, dys, staged=False):
+    T = lambda a: torch.from_numpy(a).to(DEV)
+    x_t, ws_t, bs_t, dys_t = T(x), [T(w) for w in ws], [T(b) for b in bs], [T(a) for a in dys]
+    ys = [torch.full(s, float("nan"), device=DEV) for s in layer.branch_y_shapes()]
+    dws = [torch.full(s, float("nan"), device=DEV) for s in layer.branch_w_shapes()]
+    dbs = [torch.full((c,), float("nan"), device=DEV) for c in layer.branches]
+    dx = torch.full(layer.x_shape, float("nan"), device=DEV)
+    if staged:
+        layer.stage_pack_group(glp.GLP_PACK_X, [x_t])
+        layer.stage_pack_group(glp.GLP_PACK_W_FWD, ws_t)
+        layer.stage_fwd_group(bs_t, ys)
+        layer.stage_pack_group(glp.GLP_PACK_DY_DB, dys_t)
+        layer.stage_pack_group(glp.GLP_PACK_W_BWD_DATA, ws_t)
+        layer.stage_bwd_data(dx)
+        layer.stage_bwd_filter()
+        layer.stage_reduce_group(dws, dbs)
+    else:
+        layer.group_fwd(x_t, ws_t, bs_t, ys)
+        layer.group_bwd(x_t, dys_t, ws_t, dx, dws, dbs)
+    torch.cuda.synchronize()
+    c = lambda l: [t.cpu().numpy() for t in l]
+    return {"y": c(ys), "dx": dx.cpu().numpy(), "dw": c(dws), "db": c(dbs)}
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("g", GROUPS, ids=lambda g: g[0])
+def test_group_exact_vs_oracle(g, math):
+    """A fused group equals the oracle of each branch bit for bit on integer data (y_b, dW_b,
+    db_b per branch; dx = the sum of the branches' backward-data results)."""
+    _, N, C, H, W, br, K, S, P = g
+    d, ws, bs, dys = _group_data(g, True, 51)
+    layer = glp.ConvLayer(N, C, H, W, None, K, S, P, math=math, branches=br)
+    got = _group_run(layer, d["x"], ws, bs, dys)
+    dx_ref = np.zeros(d["x"].shape)
+    for i in range(len(br)):
+        y = oracle.conv_fwd(d["x"], ws[i], bs[i], S, P)
+        dw, _ = oracle.conv_bwd_filter(d["x"], dys[i], ws[i].shape, S, P)
+        dx_ref += oracle.conv_bwd_data(dys[i], ws[i], d["x"].shape, S, P)
+        np.testing.assert_array_equal(got["y"][i], y.astype(np.float32), err_msg=f"y{i}")
+        np.testing.assert_array_equal(got["dw"][i], dw.astype(np.float32), err_msg=f"dw{i}")
+        np.testing.assert_array_equal(got["db"][i], dys[i].astype(np.float64).sum(axis=(0, 2, 3)).astype(np.float32),
+                                      err_msg=f"db{i}")
+    np.testing.assert_array_equal(got["dx"], dx_ref.astype(np.float32))
+
+
+@pytest.mark.parametrize("g", GROUPS, ids=lambda g: g[0])
+def test_group_equals_concatenated_layer(g):
+    """Random data: the per-branch group calls (composed and staged) are bitwise identical to the
+    single-tensor calls of the same plan on the concatenated tensors, and within the bf16 bar of
+    the oracle."""
+    _, N, C, H, W, br, K, S, P = g
+    d, ws, bs, dys = _group_data(g, False, 52)
+    layer = glp.ConvLayer(N, C, H, W, None, K, S, P, math="bf16", branches=br)
+    got = _group_run(layer, d["x"], ws, bs, dys)
+    got_staged = _group_run(layer, d["x"], ws, bs, dys, staged=True)
+    cat = _run(layer, d)
+    offs = np.cumsum([0] + br)
+    for i in range(len(br)):
+        for k, axis in (("y", 1), ("dw", 0), ("db", 0)):
+            ref = np.take(cat[k], range(offs[i], offs[i + 1]), axis=axis)
+            np.testing.assert_array_equal(got[k][i], ref, err_msg=f"{k}{i}")
+            np.testing.assert_array_equal(got_staged[k][i], ref, err_msg=f"staged {k}{i}")
+    np.testing.assert_array_equal(got["dx"], cat["dx"])
+    np.testing.assert_array_equal(got_staged["dx"], cat["dx"])
+    ref = _oracle(d, S, P)
+    for k in ("y", "dx", "dw", "db"):
+        assert np.abs(cat[k] - ref[k]).max() / np.abs(ref[k]).max() <= TOL["bf16"], k
+
+
+def test_group_rejects_misaligned_branch():
+    """Every branch but the last must start on a 16-byte chunk of the packed pitch."""
+    with pytest.raises(glp.GlpError):
+        glp.ConvLayer(2, 16, 8, 8, None, 3, 1, 1, math="bf16", branches=[12, 20])
+    glp.ConvLayer(2, 16, 8, 8, None, 3, 1, 1, math="bf16", branches=[16, 20])   # ok

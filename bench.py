@@ -29,7 +29,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from glp_workloads import CONFIG_NAMES, config, gen_layer  # noqa: E402
+from glp_workloads import CONFIG_NAMES, SIBLINGS, config, gen_layer  # noqa: E402
 
 METRIC = "conv fwd+bwd images/sec"
 UNIT = "images/s"
@@ -45,6 +45,9 @@ def parse_args():
     p.add_argument("--workload", type=int, default=4, help="BASELINE.json config index 1..5")
     p.add_argument("--math", choices=["bf16", "tf32"], default="bf16")
     p.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    p.add_argument("--no-fuse", action="store_true",
+                   help="run sibling layers that share an input (GoogLeNet 5b 1x1 branches) as "
+                        "separate layers instead of one fused group")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=5)
@@ -136,7 +139,9 @@ class LayerState:
     def __init__(self, layer, n_local, n_global, shard, math, dev, grads, idx):
         import torch
         import paper_conf_icpp_futhys18_b200 as glp
+        self.glp = glp
         self.layer = layer
+        self.name = layer.name
         self.n = n_local
         self.conv = glp.ConvLayer(n_local, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.S,
                                   layer.P, math=math, device=dev.index)
@@ -158,6 +163,94 @@ class LayerState:
 
     def launches(self):
         return 9 if self.dx is not None else 7
+
+    # the step's kernel groups (one C call each; see step())
+    def pack_x(self, st=None):
+        self.conv.stage_pack(self.glp.GLP_PACK_X, self.t["x"], stream=st)
+
+    def pack_w_fwd(self, st=None):
+        self.conv.stage_pack(self.glp.GLP_PACK_W_FWD, self.t["w"], stream=st)
+
+    def fwd(self, st=None):
+        self.conv.stage_fwd(self.t["b"], self.y, stream=st)
+
+    def pack_dy(self, st=None):
+        self.conv.stage_pack(self.glp.GLP_PACK_DY_DB, self.t["dy"], stream=st)
+
+    def pack_w_bwd(self, st=None):
+        self.conv.stage_pack(self.glp.GLP_PACK_W_BWD_DATA, self.t["w"], stream=st)
+
+    def bwd_data(self, st=None):
+        self.conv.stage_bwd_data(self.dx, stream=st)
+
+    def bwd_filter(self, st=None):
+        self.conv.stage_bwd_filter(stream=st)
+
+    def reduce(self, st=None):
+        self.conv.stage_reduce(self.dw, self.db, stream=st)
+
+    def host_inputs(self):
+        return self.host, self.t
+
+
+class GroupState:
+    """Sibling layers that read one input, run as a fused group (one GEMM per pass; include/glp.h
+    "fused sibling groups").  Same unit interface as LayerState."""
+
+    def __init__(self, members, n_local, n_global, math, dev, grads, idxs):
+        import torch
+        import paper_conf_icpp_futhys18_b200 as glp
+        self.glp = glp
+        self.members = members
+        l0 = members[0]
+        self.layer = l0
+        self.name = "+".join(m.name for m in members)
+        self.n = n_local
+        self.conv = glp.ConvLayer(n_local, l0.C, l0.H, l0.W, None, l0.K, l0.S, l0.P, math=math,
+                                  device=dev.index, branches=[m.Co for m in members])
+        ds = [gen_layer(m, n_global=n_global, batch=n_local) for m in members]
+        self.host = {"x": torch.from_numpy(ds[0]["x"])}   # the shared input
+        for i, d in enumerate(ds):
+            for k in ("w", "b", "dy"):
+                self.host[f"{k}{i}"] = torch.from_numpy(d[k])
+        self.t = {k: v.to(dev) for k, v in self.host.items()}
+        nb = len(members)
+        self.ws = [self.t[f"w{i}"] for i in range(nb)]
+        self.bs = [self.t[f"b{i}"] for i in range(nb)]
+        self.dys = [self.t[f"dy{i}"] for i in range(nb)]
+        self.ys = [torch.empty(s, device=dev) for s in self.conv.branch_y_shapes()]
+        self.dx = None if l0.data_fed else torch.empty(self.conv.x_shape, device=dev)
+        self.dws = [grads.dw(i) for i in idxs]
+        self.dbs = [grads.db(i) for i in idxs]
+        self.flops = float(sum(m.with_batch(n_local).flops_per_pass() for m in members))
+
+    def launches(self):
+        nb = len(self.members)   # per-branch packs of W (x2) and dy
+        return 6 + 3 * nb if self.dx is not None else 5 + 2 * nb
+
+    def pack_x(self, st=None):
+        self.conv.stage_pack_group(self.glp.GLP_PACK_X, [self.t["x"]], stream=st)
+
+    def pack_w_fwd(self, st=None):
+        self.conv.stage_pack_group(self.glp.GLP_PACK_W_FWD, self.ws, stream=st)
+
+    def fwd(self, st=None):
+        self.conv.stage_fwd_group(self.bs, self.ys, stream=st)
+
+    def pack_dy(self, st=None):
+        self.conv.stage_pack_group(self.glp.GLP_PACK_DY_DB, self.dys, stream=st)
+
+    def pack_w_bwd(self, st=None):
+        self.conv.stage_pack_group(self.glp.GLP_PACK_W_BWD_DATA, self.ws, stream=st)
+
+    def bwd_data(self, st=None):
+        self.conv.stage_bwd_data(self.dx, stream=st)
+
+    def bwd_filter(self, st=None):
+        self.conv.stage_bwd_filter(stream=st)
+
+    def reduce(self, st=None):
+        self.conv.stage_reduce_group(self.dws, self.dbs, stream=st)
 
 
 def run_glp(args, ws, rank, local):
@@ -183,10 +276,22 @@ def run_glp(args, ws, rank, local):
     grads = FlatGrads([l.w_shape for l in layers], device=dev)
     flat = grads.buf
     nparams = grads.numel
+    groups = [] if args.no_fuse else SIBLINGS.get(args.workload, [])
+    in_group = {name: gi for gi, g in enumerate(groups) for name in g}
     states = []
+    done_groups = set()
     for i, (l, nl, ng) in enumerate(zip(layers, n_local, n_global)):
         shard = shards[i] if args.scaling == "strong" and G > 1 else None
-        states.append(LayerState(l, nl, ng, shard, args.math, dev, grads, i))
+        gi = in_group.get(l.name)
+        if gi is None:
+            states.append(LayerState(l, nl, ng, shard, args.math, dev, grads, i))
+        elif gi not in done_groups:
+            if shard is not None:
+                raise SystemExit("fused groups with strong scaling: use --no-fuse")
+            done_groups.add(gi)
+            idxs = [j for j, m in enumerate(layers) if m.name in groups[gi]]
+            states.append(GroupState([layers[j] for j in idxs], nl, ng, args.math, dev, grads,
+                                     idxs))
     stream = torch.cuda.current_stream()
 
     side_w = torch.cuda.Stream(device=dev)   # weight packs (weights are known at step start)
@@ -204,31 +309,29 @@ def run_glp(args, ws, rank, local):
         conc = (ev is None) if concurrent is None else concurrent
         if not conc:
             for i, s in enumerate(states):
-                c = s.conv
-                c.stage_pack(glp.GLP_PACK_X, s.t["x"])
-                c.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"])
+                s.pack_x()
+                s.pack_w_fwd()
                 if ev is not None:
                     ev[i][0].record(stream)
-                c.stage_fwd(s.t["b"], s.y)
+                s.fwd()
                 if ev is not None:
                     ev[i][1].record(stream)
             for i in reversed(range(len(states))):
                 s = states[i]
-                c = s.conv
-                c.stage_pack(glp.GLP_PACK_DY_DB, s.t["dy"])
+                s.pack_dy()
                 if s.dx is not None:
-                    c.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"])
+                    s.pack_w_bwd()
                     if ev is not None:
                         ev[i][2].record(stream)
-                    c.stage_bwd_data(s.dx)
+                    s.bwd_data()
                     if ev is not None:
                         ev[i][3].record(stream)
                 if ev is not None:
                     ev[i][4].record(stream)
-                c.stage_bwd_filter()
+                s.bwd_filter()
                 if ev is not None:
                     ev[i][5].record(stream)
-                c.stage_reduce(s.dw, s.db)
+                s.reduce()
             if G > 1:
                 grads.allreduce()
             return
@@ -237,35 +340,33 @@ def run_glp(args, ws, rank, local):
         ew_f, ew_b = [], []
         with torch.cuda.stream(side_w):
             for s in states:
-                s.conv.stage_pack(glp.GLP_PACK_W_FWD, s.t["w"], stream=side_w)
+                s.pack_w_fwd(side_w)
                 e = torch.cuda.Event()
                 e.record(side_w)
                 ew_f.append(e)
             for s in reversed(states):
                 if s.dx is not None:
-                    s.conv.stage_pack(glp.GLP_PACK_W_BWD_DATA, s.t["w"], stream=side_w)
+                    s.pack_w_bwd(side_w)
                 e = torch.cuda.Event()
                 e.record(side_w)
                 ew_b.append(e)
         ew_b = ew_b[::-1]
         for i, s in enumerate(states):
-            c = s.conv
-            c.stage_pack(glp.GLP_PACK_X, s.t["x"])
+            s.pack_x()
             stream.wait_event(ew_f[i])
-            c.stage_fwd(s.t["b"], s.y)
+            s.fwd()
         for i in reversed(range(len(states))):
             s = states[i]
-            c = s.conv
-            c.stage_pack(glp.GLP_PACK_DY_DB, s.t["dy"])
+            s.pack_dy()
             e_dy = torch.cuda.Event()
             e_dy.record(stream)
             side_g.wait_event(e_dy)
             with torch.cuda.stream(side_g):
-                c.stage_bwd_filter(stream=side_g)
-                c.stage_reduce(s.dw, s.db, stream=side_g)
+                s.bwd_filter(side_g)
+                s.reduce(side_g)
             if s.dx is not None:
                 stream.wait_event(ew_b[i])
-                c.stage_bwd_data(s.dx)
+                s.bwd_data()
         stream.wait_stream(side_w)
         stream.wait_stream(side_g)
         if G > 1:
@@ -329,7 +430,7 @@ def run_glp(args, ws, rank, local):
                 continue
             us = [evs[k][i][a].elapsed_time(evs[k][i][b]) * 1e3 for k in range(args.steps)]
             avg = sum(us) / len(us)
-            kern.append({"layer": s.layer.name, "pass": name, "avg_us": round(avg, 2),
+            kern.append({"layer": s.name, "pass": name, "avg_us": round(avg, 2),
                          "total_us": sum(us), "tflops": round(s.flops / (avg * 1e-6) / 1e12, 1)})
     peaks = load_peaks()
     dom = max(kern, key=lambda r: r["total_us"])
@@ -401,7 +502,7 @@ def run_glp(args, ws, rank, local):
         "dtype": args.math, "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
         "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
                    "global_batch": images_per_step, "per_gpu_batch": n_local[0],
-                   "layers": [s.layer.name for s in states], "math": args.math,
+                   "layers": [s.name for s in states], "math": args.math,
                    "parallelism": f"dp{G}", "l2": "inputs larger than L2 (step working set "
                    f"{sum(v.numel() * 4 for s in states for v in s.t.values()) / 1e9:.2f} GB)",
                    "step_gflop": round(step_flops / 1e9, 1),

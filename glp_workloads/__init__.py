@@ -86,6 +86,14 @@ _TABLE: Dict[int, List[Layer]] = {
         _L("googlenet_conv_6", 128, 832, 7, 48, 1, 1, 0, 7, False)],
 }
 
+# Sibling layers that read the same input tensor in the real network and can run as one fused
+# group (include/glp.h "fused sibling groups"): GoogLeNet inception 5b's
+# 1x1, 3x3_reduce and 5x5_reduce branches (Table 5 conv_3, conv_5, conv_6) all read 5b's
+# 832-channel input.  The group uses the first member's x draw as the shared input.
+SIBLINGS: Dict[int, List[List[str]]] = {
+    5: [["googlenet_conv_3", "googlenet_conv_5", "googlenet_conv_6"]],
+}
+
 CONFIG_NAMES = {
     1: "lenet_conv1_b64",
     2: "lenet5_conv_stack_b64",

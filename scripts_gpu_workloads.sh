@@ -1,22 +1,14 @@
 #!/bin/bash
-# Bench every BASELINE.json workload (1..5) in bf16 and tf32 (short runs, no CPU baseline / e2e).
+# every BASELINE.json workload (bf16 + tf32), plus GoogLeNet without sibling fusion
 cd "$(dirname "$0")"
 mkdir -p gpurun_out
-for m in bf16 tf32; do
-  for w in 1 2 3 4 5; do
-    timeout -s KILL 300 python bench.py --workload $w --math $m --steps ${STEPS:-30} --warmup 5 \
-      --no-cpu-baseline --no-e2e > gpurun_out/wl_${w}_${m}.json 2> gpurun_out/wl_${w}_${m}.err
-    python3 - "$w" "$m" <<'PY'
-import json, sys
-w, m = sys.argv[1], sys.argv[2]
-try:
-    d = json.load(open(f"gpurun_out/wl_{w}_{m}.json"))
-    best = max(d["kernels"], key=lambda k: k["tflops"])
-    print(f"w{w} {m:4s} {d['config']['workload']:28s} {d['value']:10.1f} {d['unit']} {d['ms_per_step']:8.3f} ms "
-          f"step {d['tflops_step']:7.1f} TF/s  best {best['layer']}/{best['pass']} {best['tflops']} TF/s "
-          f"dom {d['roofline']['kernel']} frac {d['roofline']['frac']}")
-except Exception as e:
-    print(f"w{w} {m} FAILED {e}"); print(open(f"gpurun_out/wl_{w}_{m}.err").read()[-800:])
-PY
+for W in ${WLS:-1 2 3 4 5}; do
+  for M in ${MATHS:-bf16 tf32}; do
+    timeout -s KILL 300 python bench.py --steps ${STEPS:-30} --warmup 5 --workload $W --math $M --no-cpu-baseline --no-e2e > gpurun_out/wl_${W}_${M}.json 2> gpurun_out/wl_${W}_${M}.err
+    echo "wl $W $M rc=$? $(python -c "import json,sys; d=json.loads(open('gpurun_out/wl_${W}_${M}.json').read().splitlines()[-1]); print(d['value'], d['ms_per_step'], d['roofline']['kernel'], d['roofline']['achieved'])" 2>&1 | tail -1)"
   done
 done
+if [ -z "$NONOFUSE" ]; then
+timeout -s KILL 300 python bench.py --steps ${STEPS:-30} --warmup 5 --workload 5 --math bf16 --no-cpu-baseline --no-e2e --no-fuse > gpurun_out/wl_5_bf16_nofuse.json 2> gpurun_out/wl_5_nofuse.err
+echo "wl 5 bf16 no-fuse rc=$? $(python -c "import json; d=json.loads(open('gpurun_out/wl_5_bf16_nofuse.json').read().splitlines()[-1]); print(d['value'], d['ms_per_step'])" 2>&1 | tail -1)"
+fi

@@ -45,6 +45,11 @@ def parse_args():
     p.add_argument("--workload", type=int, default=4, help="BASELINE.json config index 1..5")
     p.add_argument("--math", choices=["bf16", "tf32"], default="bf16")
     p.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    p.add_argument("--scheme", choices=["persistent", "pool"], default="persistent",
+                   help="pool: the paper's prior-art scheme (per-sample kernels round-robin over a "
+                        "stream pool sized by Eq. 7) as a comparator; 1 GPU")
+    p.add_argument("--pool-streams", type=int, default=0,
+                   help="stream-pool size (0 = the Eq. 7 bound)")
     p.add_argument("--no-fuse", action="store_true",
                    help="run sibling layers that share an input (GoogLeNet 5b 1x1 branches) as "
                         "separate layers instead of one fused group")
@@ -251,6 +256,74 @@ class GroupState:
 
     def reduce(self, st=None):
         self.conv.stage_reduce_group(self.dws, self.dbs, stream=st)
+
+
+def run_pool(args):
+    """The paper's stream-pool scheme (include/glp.h glp_pool_*) on the same workload: every
+    layer-pass as per-sample kernels over a pool of streams.  Comparator only (1 GPU, eager)."""
+    import torch
+    import paper_conf_icpp_futhys18_b200 as glp
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    layers = config(args.workload)
+    units = []
+    for l in layers:
+        d = gen_layer(l)
+        t = {k: torch.from_numpy(v).to(dev) for k, v in d.items()}
+        pool = glp.StreamPool(l.N, l.C, l.H, l.W, l.Co, l.K, l.S, l.P, math=args.math,
+                              n_streams=args.pool_streams)
+        y = torch.empty(l.y_shape, device=dev)
+        dx = None if l.data_fed else torch.empty(l.x_shape, device=dev)
+        dw = torch.empty(l.w_shape, device=dev)
+        db = torch.empty(l.Co, device=dev)
+        units.append((l, pool, t, y, dx, dw, db))
+
+    def step():
+        for l, pool, t, y, dx, dw, db in units:
+            pool.fwd(t["x"], t["w"], t["b"], y)
+        for l, pool, t, y, dx, dw, db in reversed(units):
+            pool.bwd(t["x"], t["dy"], t["w"], dx, dw, db)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    def timed(fn):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.steps):
+            fn()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / args.steps
+
+    ms_eager = timed(step)
+    # the same per-sample launches recorded once into a CUDA graph (the pool's fork/join events
+    # are captured as graph edges), removing the host launch cost the eager pool pays
+    ms_graph = None
+    if not args.no_graph:
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            step()
+        g.replay()
+        torch.cuda.synchronize()
+        ms_graph = timed(g.replay)
+    ms = min(ms_eager, ms_graph or ms_eager)
+    step_flops = sum(l.flops_per_pass() * (2 if l.data_fed else 3) for l in layers)
+    print(json.dumps({
+        "metric": METRIC, "value": round(layers[0].N / (ms / 1e3), 1), "unit": UNIT, "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": args.math,
+        "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
+        "scheme": "stream-pool (paper's prior-art scheme: per-sample kernels, round-robin streams)",
+        "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
+                   "global_batch": layers[0].N, "layers": [l.name for l in layers],
+                   "pool_streams": [u[1].n_streams for u in units],
+                   "eq7_bound": [u[1].eq7_bound for u in units]},
+        "launch": "cuda_graph" if ms_graph is not None and ms_graph <= ms_eager else "eager",
+        "ms_per_step_eager": round(ms_eager, 4),
+        "ms_per_step_graph": None if ms_graph is None else round(ms_graph, 4),
+        "tflops_step": round(step_flops / (ms * 1e-3) / 1e12, 1)}), flush=True)
 
 
 def run_glp(args, ws, rank, local):
@@ -635,6 +708,10 @@ def main():
         print(f"warning: WORLD_SIZE={ws} but --gpus {args.gpus}", file=sys.stderr)
     if args.impl == "reference":
         run_reference(args, ws, rank)
+        return
+    if args.scheme == "pool":
+        if rank == 0:
+            run_pool(args)
         return
     run_glp(args, ws, rank, local)
 

@@ -208,6 +208,34 @@ glp_status_t glp_stage_fwd_group(glp_plan_t plan, const float *const *b, float *
 glp_status_t glp_stage_reduce_group(glp_plan_t plan, float *const *dw, float *const *db,
                                     int accumulate, void *ws, size_t ws_bytes, glp_stream_t stream);
 
+/* ---- prior-art comparator: the paper's stream pool --------------------- *
+ * GLP4NN's own scheme (P165-173, Figs 4/6): every layer pass runs as per-sample kernels (batch 1,
+ * the sample's im2col+GEMM chain) dispatched round-robin (P171) over a pool of CUDA streams whose
+ * size is the paper's Eq. 7 bound for the per-sample forward kernel (P245: thread and shared-
+ * memory terms, no launch term, capped by the concurrent-kernel limit C of Eq. 6) or the caller's
+ * n_streams (> 0; both capped by N and 64).  Kept to measure what the persistent tile scheduler
+ * of the glp_conv_* calls buys on B200 (bench.py --scheme pool); not the product path.
+ * A pool owns its streams and a per-sample plan; desc must be a single layer (no groups).
+ * Calls fork from `stream` (event), run on the pool's streams and join back to `stream`.
+ * ws >= the ws_bytes of glp_pool_get_info (1024-byte aligned): one per-sample workspace per
+ * stream plus one dW||db accumulator per stream.  Forward and backward-data results are bitwise
+ * those of glp_conv_fwd / glp_conv_bwd_data (no K split; the per-element order is the same).
+ * The filter gradient: each stream accumulates its samples in order (beta = 1, Caffe style; one
+ * accumulator per stream instead of the race the paper leaves open, P262-264), and the
+ * accumulators are summed in stream order at the join: deterministic for a given n_streams,
+ * equal to glp_conv_bwd_filter within rounding (bit-exact on integer data). */
+typedef struct glp_pool_s *glp_pool_t;
+glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t desc, int device, glp_math_t math,
+                             int n_streams);
+glp_status_t glp_pool_get_info(glp_pool_t pool, int *n_streams, int *eq7_bound, size_t *ws_bytes);
+glp_status_t glp_pool_conv_fwd(glp_pool_t pool, const float *x, const float *w, const float *b,
+                               float *y, void *ws, size_t ws_bytes, glp_stream_t stream);
+/* dx may be NULL (data-fed layer), db may be NULL.  dW, db are overwritten. */
+glp_status_t glp_pool_conv_bwd(glp_pool_t pool, const float *x, const float *dy, const float *w,
+                               float *dx, float *dw, float *db, void *ws, size_t ws_bytes,
+                               glp_stream_t stream);
+glp_status_t glp_pool_destroy(glp_pool_t pool);
+
 /* ---- analyzer (host only, no device needed) ----------------------------------------------- */
 /* The north_star's sm_100a limits: 148 SMs, 64K regs, 228 KB smem, 2048 threads, 32 blocks,
  * + 512 TMEM columns, 1 KB smem reserved per CTA, C = 128. */

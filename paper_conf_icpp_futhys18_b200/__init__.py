@@ -59,7 +59,8 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_debug_im2col", "glp_stage_pack", "glp_stage_fwd", "glp_stage_bwd_data",
            "glp_stage_bwd_filter", "glp_stage_reduce", "glp_conv_group_desc_create",
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
-           "glp_stage_reduce_group"]
+           "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
+           "glp_pool_conv_bwd", "glp_pool_destroy"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA = 0, 1, 2, 3, 4
 
@@ -114,6 +115,11 @@ def lib():
         L.glp_stage_pack_group.argtypes = [_vp, _c_int, _vp, _vp, _c_size, _vp]
         L.glp_stage_fwd_group.argtypes = [_vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_stage_reduce_group.argtypes = [_vp, _vp, _vp, _c_int, _vp, _c_size, _vp]
+        L.glp_pool_create.argtypes = [P(_vp), _vp, _c_int, _c_int, _c_int]
+        L.glp_pool_get_info.argtypes = [_vp, P(_c_int), P(_c_int), P(_c_size)]
+        L.glp_pool_conv_fwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
+        L.glp_pool_conv_bwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
+        L.glp_pool_destroy.argtypes = [_vp]
         _lib = L
     return _lib
 
@@ -354,6 +360,54 @@ class ConvLayer:
             L = lib()
             if getattr(self, "_plan", None):
                 L.glp_plan_destroy(self._plan)
+            if getattr(self, "_desc", None):
+                L.glp_conv_desc_destroy(self._desc)
+        except Exception:
+            pass
+
+
+class StreamPool:
+    """The paper's prior-art scheme as a comparator (include/glp.h "stream pool"): per-sample
+    kernels dispatched round-robin over a pool of streams sized by the Eq. 7 bound."""
+
+    def __init__(self, N, C, H, W, Co, K, stride=1, pad=0, math="bf16", device=0, n_streams=0):
+        import torch
+        L = lib()
+        self.geom = Geometry(N, C, H, W, Co, K, K, stride, stride, pad, pad)
+        self._desc = _vp()
+        _ck(L.glp_conv_desc_create(ctypes.byref(self._desc), N, C, H, W, Co, K, K, stride, stride,
+                                   pad, pad), "glp_conv_desc_create")
+        self.math = MATH[math] if isinstance(math, str) else int(math)
+        self._pool = _vp()
+        _ck(L.glp_pool_create(ctypes.byref(self._pool), self._desc, int(device), self.math,
+                              int(n_streams)), "glp_pool_create")
+        ns, eq7, wsb = _c_int(), _c_int(), _c_size()
+        _ck(L.glp_pool_get_info(self._pool, ctypes.byref(ns), ctypes.byref(eq7), ctypes.byref(wsb)),
+            "glp_pool_get_info")
+        self.n_streams, self.eq7_bound = ns.value, eq7.value
+        nbytes = wsb.value + 1024
+        self._ws_buf = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{int(device)}")
+        off = (-self._ws_buf.data_ptr()) % 1024
+        self.ws_ptr = self._ws_buf.data_ptr() + off
+        self.ws_bytes = nbytes - off
+
+    def fwd(self, x, w, b, y, stream=None):
+        _ck(lib().glp_pool_conv_fwd(self._pool, _ptr(x), _ptr(w), _ptr(b), _ptr(y),
+                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_pool_conv_fwd")
+        return y
+
+    def bwd(self, x, dy, w, dx, dw, db=None, stream=None):
+        _ck(lib().glp_pool_conv_bwd(self._pool, _ptr(x), _ptr(dy), _ptr(w), _ptr(dx), _ptr(dw),
+                                    _ptr(db), ctypes.c_void_p(self.ws_ptr), self.ws_bytes,
+                                    _stream(stream)), "glp_pool_conv_bwd")
+        return dx, dw, db
+
+    def __del__(self):
+        try:
+            L = lib()
+            if getattr(self, "_pool", None):
+                L.glp_pool_destroy(self._pool)
             if getattr(self, "_desc", None):
                 L.glp_conv_desc_destroy(self._desc)
         except Exception:

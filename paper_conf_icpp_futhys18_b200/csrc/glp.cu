@@ -18,6 +18,7 @@
 #include <mutex>
 #include <string>
 #include <utility>
+#include <vector>
 
 #include "../../include/glp.h"
 #include "common.cuh"
@@ -940,6 +941,19 @@ glp_status_t tc_bwd(glp_plan_s &P, const float *x, const BrIn &dy, const BrIn &w
   return run_wgrad_reduce(P, dw, with_db ? &db : nullptr, accumulate, ws, st);
 }
 
+// Stream-pool comparator: dst[i] (+)= sum over the pool's S per-stream accumulators, s = 0..S-1
+// in order (fixed, so the pool's result is deterministic for a given S).
+__global__ void __launch_bounds__(256) pool_sum_slots(const float *__restrict__ src, size_t stride,
+                                                      int S, float *__restrict__ dst, size_t n,
+                                                      int accumulate) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n;
+       i += (size_t)gridDim.x * blockDim.x) {
+    float a = 0.f;
+    for (int s = 0; s < S; ++s) a += src[(size_t)s * stride + i];
+    dst[i] = accumulate ? dst[i] + a : a;
+  }
+}
+
 ConvGeom geom(const glp_conv_desc_s &d) {
   return ConvGeom{d.N, d.C, d.H, d.W, d.Co, d.Kh, d.Kw, d.Sh, d.Sw, d.Ph, d.Pw, d.Ho, d.Wo};
 }
@@ -1572,6 +1586,202 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   else
     debug_im2col_kernel<4><<<ew_grid(total), 256, 0, st>>>(p.g, n, P->d.C, P->d.Kh, P->d.Kw, P->d.Ho, P->d.Wo, col);
   GLP_LAUNCH_CHECK("debug_im2col_kernel");
+  return GLP_OK;
+}
+
+// ---- prior-art comparator: the paper's per-sample stream pool ----
+}  // extern "C"
+
+struct glp_pool_s {
+  glp_conv_desc_s d1;            // the per-sample (N = 1) layer
+  glp_plan_t plan1 = nullptr;    // its plan (shared by every stream: plans are immutable)
+  int N = 0, device = 0, math = 0, S = 1, eq7 = 1;
+  size_t slot_ws = 0, acc_floats = 0, ws_bytes = 0;
+  std::vector<cudaStream_t> streams;
+  std::vector<cudaEvent_t> joins;
+  cudaEvent_t fork = nullptr;
+};
+
+namespace {
+glp_status_t pool_fork(glp_pool_s *Q, cudaStream_t st) {
+  GLP_CUDA(cudaEventRecord(Q->fork, st));
+  for (int s = 0; s < Q->S; ++s) GLP_CUDA(cudaStreamWaitEvent(Q->streams[s], Q->fork, 0));
+  return GLP_OK;
+}
+glp_status_t pool_join(glp_pool_s *Q, cudaStream_t st) {
+  for (int s = 0; s < Q->S; ++s) {
+    GLP_CUDA(cudaEventRecord(Q->joins[s], Q->streams[s]));
+    GLP_CUDA(cudaStreamWaitEvent(st, Q->joins[s], 0));
+  }
+  return GLP_OK;
+}
+}  // namespace
+
+extern "C" {
+
+glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t d, int device, glp_math_t math,
+                             int n_streams) {
+  if (!out || !d) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *out = nullptr;
+  if (n_streams < 0) return fail(GLP_ERR_INVALID_VALUE, "n_streams < 0");
+  if (d->nbr > 1) return fail(GLP_ERR_NOT_SUPPORTED, "the stream pool runs single layers");
+  auto *Q = new glp_pool_s();
+  Q->d1 = *d;
+  Q->d1.N = 1;
+  Q->N = d->N;
+  Q->device = device;
+  Q->math = (int)math;
+  glp_status_t s = glp_plan(&Q->plan1, &Q->d1, device, math, 0);
+  if (s) {
+    delete Q;
+    return s;
+  }
+  // Eq. 7 (P245): how many instances of the per-sample forward kernel fit the device at once
+  // (thread and shared-memory terms; no launch term, R17), capped by the concurrent-kernel
+  // limit C (Eq. 6).  FP32 plans: their per-sample kernel is the SIMT forward (256 threads).
+  glp_device_limits_t L;
+  glp_device_limits_b200(&L);
+  glp_kernel_attr_t ka{256, 0, 0, 0};
+  int blocks = (int)std::max<long long>(1, cdiv((long long)Q->d1.Co * Q->d1.Ho * Q->d1.Wo, 256));
+  if (math != GLP_MATH_FP32) {
+    int m = 0, r = 0;
+    glp_plan_kernel_attr(Q->plan1, 0, &ka, &m, &r);
+    blocks = Q->plan1->fwd.grid;
+  }
+  int bound = 1;
+  glp_analyze_eq7(&L, &ka, blocks, 0.0, 0.0, &bound);
+  Q->eq7 = std::max(1, std::min(bound, L.max_concurrent_kernels));
+  Q->S = std::max(1, std::min(n_streams > 0 ? n_streams : Q->eq7, std::min(Q->N, 64)));
+  Q->slot_ws = align1k(std::max<size_t>(Q->plan1->ws_bwd, 1));
+  Q->acc_floats = (size_t)rup((long long)d->Co * d->C * d->Kh * d->Kw + d->Co, 64);
+  Q->ws_bytes = (size_t)Q->S * Q->slot_ws + align1k((size_t)Q->S * Q->acc_floats * 4);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  if (cur != device) cudaSetDevice(device);
+  for (int i = 0; i < Q->S; ++i) {
+    cudaStream_t st;
+    cudaEvent_t ev;
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) {
+      glp_pool_destroy(Q);
+      if (cur != device) cudaSetDevice(cur);
+      return fail(GLP_ERR_CUDA, "stream pool creation failed");
+    }
+    Q->streams.push_back(st);
+    Q->joins.push_back(ev);
+  }
+  cudaEventCreateWithFlags(&Q->fork, cudaEventDisableTiming);
+  if (cur != device) cudaSetDevice(cur);
+  *out = Q;
+  return GLP_OK;
+}
+
+glp_status_t glp_pool_get_info(glp_pool_t Q, int *n_streams, int *eq7_bound, size_t *ws_bytes) {
+  if (!Q) return fail(GLP_ERR_INVALID_VALUE, "pool is NULL");
+  if (n_streams) *n_streams = Q->S;
+  if (eq7_bound) *eq7_bound = Q->eq7;
+  if (ws_bytes) *ws_bytes = Q->ws_bytes;
+  return GLP_OK;
+}
+
+glp_status_t glp_pool_destroy(glp_pool_t Q) {
+  if (!Q) return GLP_OK;
+  for (auto st : Q->streams) cudaStreamDestroy(st);
+  for (auto ev : Q->joins) cudaEventDestroy(ev);
+  if (Q->fork) cudaEventDestroy(Q->fork);
+  if (Q->plan1) glp_plan_destroy(Q->plan1);
+  delete Q;
+  return GLP_OK;
+}
+
+glp_status_t glp_pool_conv_fwd(glp_pool_t Q, const float *x, const float *w, const float *b,
+                               float *y, void *ws, size_t ws_bytes, glp_stream_t stream) {
+  if (!Q) return fail(GLP_ERR_INVALID_VALUE, "pool is NULL");
+  glp_status_t s = validate_ptrs({x, w, y});
+  if (s) return s;
+  if ((s = check_ws(Q->plan1, ws, ws_bytes, Q->ws_bytes))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  const glp_conv_desc_s &d = Q->d1;
+  const size_t xs = (size_t)d.C * d.H * d.W, ys = (size_t)d.Co * d.Ho * d.Wo;
+  const bool tc = Q->math != GLP_MATH_FP32;
+  if ((s = pool_fork(Q, st))) return s;
+  // internal calls: per-sample slices are only 4-byte aligned (e.g. 3 x 227 x 227 floats)
+  glp_plan_s &P1 = *Q->plan1;
+  if (tc) {
+    if ((s = get_encode())) return s;
+    for (int i = 0; i < Q->S; ++i)   // each stream's workspace holds its own packed weights
+      if ((s = run_pack_w_fwd(P1, br_in1(w), wsb + i * Q->slot_ws, Q->streams[i]))) return s;
+  }
+  for (int n = 0; n < Q->N; ++n) {   // round-robin dispatch of per-sample kernels (P171)
+    const int i = n % Q->S;
+    uint8_t *wsi = wsb + i * Q->slot_ws;
+    cudaStream_t si = Q->streams[i];
+    float *yn = y + n * ys;
+    if (tc) {
+      if ((s = launch_pack_x(P1, x + n * xs, wsi + P1.off_xpk, si)) ||
+          (s = run_fwd_gemm(P1, br_in1(b), br_out(P1, 1, &yn), wsi, si)))
+        return s;
+    } else {
+      simt_fwd<<<ew_grid(ys), 256, 0, si>>>(geom(P1.d), x + n * xs, w, b, yn);
+      GLP_LAUNCH_CHECK("simt_fwd");
+    }
+  }
+  return pool_join(Q, st);
+}
+
+glp_status_t glp_pool_conv_bwd(glp_pool_t Q, const float *x, const float *dy, const float *w,
+                               float *dx, float *dw, float *db, void *ws, size_t ws_bytes,
+                               glp_stream_t stream) {
+  if (!Q) return fail(GLP_ERR_INVALID_VALUE, "pool is NULL");
+  glp_status_t s = validate_ptrs({x, dy, w, dw});
+  if (s) return s;
+  if ((s = check_ws(Q->plan1, ws, ws_bytes, Q->ws_bytes))) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  uint8_t *wsb = static_cast<uint8_t *>(ws);
+  const glp_conv_desc_s &d = Q->d1;
+  const size_t xs = (size_t)d.C * d.H * d.W, ys = (size_t)d.Co * d.Ho * d.Wo;
+  const size_t wsz = (size_t)d.Co * d.C * d.Kh * d.Kw;
+  float *acc = reinterpret_cast<float *>(wsb + (size_t)Q->S * Q->slot_ws);
+  const bool tc = Q->math != GLP_MATH_FP32;
+  if ((s = pool_fork(Q, st))) return s;
+  // The paper's concurrent streams would all accumulate (beta = 1) into one dW and race
+  // (P262-264); each stream here owns an accumulator, summed in stream order at the join.
+  glp_plan_s &P1 = *Q->plan1;
+  if (tc && (s = get_encode())) return s;
+  for (int i = 0; i < Q->S; ++i) {
+    GLP_CUDA(cudaMemsetAsync(acc + i * Q->acc_floats, 0, Q->acc_floats * 4, Q->streams[i]));
+    if (tc && dx && (s = run_pack_w_dgrad(P1, br_in1(w), wsb + i * Q->slot_ws, Q->streams[i])))
+      return s;
+  }
+  for (int n = 0; n < Q->N; ++n) {
+    const int i = n % Q->S;
+    uint8_t *wsi = wsb + i * Q->slot_ws;
+    float *dwi = acc + i * Q->acc_floats, *dbi = db ? dwi + wsz : nullptr;
+    cudaStream_t si = Q->streams[i];
+    const float *xn = x + n * xs, *dyn = dy + n * ys;
+    if (tc) {
+      if ((s = launch_pack_dy(P1, br_in1(dyn), wsi, db != nullptr, si))) return s;
+      if (dx && (s = run_dgrad_gemm(P1, dx + n * xs, wsi, si))) return s;
+      const BrOut dbo = br_out(P1, 1, &dbi);
+      if ((s = launch_pack_x(P1, xn, wsi + P1.off_xpk, si)) || (s = run_wgrad_gemm(P1, wsi, si)) ||
+          (s = run_wgrad_reduce(P1, br_out(P1, 1, &dwi), db ? &dbo : nullptr, 1, wsi, si)))
+        return s;
+    } else {
+      if (dx) {
+        simt_dgrad<<<ew_grid(xs), 256, 0, si>>>(geom(P1.d), dyn, w, dx + n * xs);
+        GLP_LAUNCH_CHECK("simt_dgrad");
+      }
+      if ((s = run_wgrad_simt(P1, xn, dyn, dwi, dbi, 1, wsi, si))) return s;
+    }
+  }
+  if ((s = pool_join(Q, st))) return s;
+  pool_sum_slots<<<ew_grid(wsz), 256, 0, st>>>(acc, Q->acc_floats, Q->S, dw, wsz, 0);
+  GLP_LAUNCH_CHECK("pool_sum_slots");
+  if (db) {
+    pool_sum_slots<<<ew_grid(d.Co), 256, 0, st>>>(acc + wsz, Q->acc_floats, Q->S, db, (size_t)d.Co, 0);
+    GLP_LAUNCH_CHECK("pool_sum_slots");
+  }
   return GLP_OK;
 }
 

@@ -397,3 +397,41 @@ def test_group_rejects_misaligned_branch():
     with pytest.raises(glp.GlpError):
         glp.ConvLayer(2, 16, 8, 8, None, 3, 1, 1, math="bf16", branches=[12, 20])
     glp.ConvLayer(2, 16, 8, 8, None, 3, 1, 1, math="bf16", branches=[16, 20])   # ok
+
+
+POOL_SHAPES = [SHAPES[0], SHAPES[2], SHAPES[6], ("k5_ragged", 5, 24, 11, 13, 40, 5, 1, 2)]
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("shape", POOL_SHAPES, ids=lambda s: s[0])
+def test_stream_pool_comparator(shape, math):
+    """The paper's per-sample stream pool (prior-art comparator): forward and backward-data are
+    bitwise the batched persistent path's results; the filter gradient is bit-exact on integer
+    data and within the tolerance on random data; the pool size is the Eq. 7 bound unless set."""
+    _, N, C, H, W, Co, K, S, P = shape
+    T = lambda a: torch.from_numpy(a).to(DEV)
+    for exact, seed in ((True, 61), (False, 62)):
+        d = _data(shape, exact=exact, seed=seed)
+        ref_layer = _run(_layer(shape, math), d)
+        for ns in (0, 3):
+            pool = glp.StreamPool(N, C, H, W, Co, K, S, P, math=math, n_streams=ns)
+            assert pool.n_streams == (min(pool.eq7_bound, N) if ns == 0 else min(3, N))
+            y = torch.full(ref_layer["y"].shape, float("nan"), device=DEV)
+            dx = torch.full(ref_layer["dx"].shape, float("nan"), device=DEV)
+            dw = torch.full(ref_layer["dw"].shape, float("nan"), device=DEV)
+            db = torch.full(ref_layer["db"].shape, float("nan"), device=DEV)
+            pool.fwd(T(d["x"]), T(d["w"]), T(d["b"]), y)
+            pool.bwd(T(d["x"]), T(d["dy"]), T(d["w"]), dx, dw, db)
+            torch.cuda.synchronize()
+            got = {"y": y.cpu().numpy(), "dx": dx.cpu().numpy(), "dw": dw.cpu().numpy(),
+                   "db": db.cpu().numpy()}
+            np.testing.assert_array_equal(got["y"], ref_layer["y"])
+            np.testing.assert_array_equal(got["dx"], ref_layer["dx"])
+            if exact:
+                ref = _oracle(d, S, P)
+                for k in ("dw", "db"):
+                    np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+            else:
+                for k in ("dw", "db"):
+                    r = ref_layer[k]
+                    assert np.abs(got[k] - r).max() / np.abs(r).max() <= TOL[math], k

@@ -149,7 +149,7 @@ class LayerState:
         self.name = layer.name
         self.n = n_local
         self.conv = glp.ConvLayer(n_local, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.S,
-                                  layer.P, math=math, device=dev.index)
+                                  layer.P, math=math, device=dev.index, groups=layer.groups)
         if shard is None:
             d = gen_layer(layer, n_global=n_global, batch=n_local)
         else:  # strong scaling: this rank's contiguous slice of the global batch
@@ -612,12 +612,18 @@ def _oracle_items(layers, n):
 
 def _oracle_run(l, kind, d):
     import oracle
-    if kind == "fwd":
-        oracle.conv_fwd(d["x"], d["w"], d["b"], l.S, l.P)
-    elif kind == "bwd_filter":
-        oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, l.S, l.P)
-    else:
-        oracle.conv_bwd_data(d["dy"], d["w"], d["x"].shape, l.S, l.P)
+    G = l.groups   # grouped layers: one oracle convolution per group (independent convolutions)
+    cg, og = l.C // G, l.Co // G
+    for g in range(G):
+        x = d["x"][:, g * cg:(g + 1) * cg]
+        w = d["w"][g * og:(g + 1) * og]
+        dy = d["dy"][:, g * og:(g + 1) * og]
+        if kind == "fwd":
+            oracle.conv_fwd(x, w, d["b"][g * og:(g + 1) * og], l.S, l.P)
+        elif kind == "bwd_filter":
+            oracle.conv_bwd_filter(x, dy, w.shape, l.S, l.P)
+        else:
+            oracle.conv_bwd_data(dy, w, x.shape, l.S, l.P)
 
 
 def cpu_baseline(layers, budget_s=12.0, n_sample=None):

@@ -38,6 +38,7 @@ class Layer:
     data_fed: bool     # bottom is the data layer -> benchmark skips dgrad (R9)
     cfg: int = 0
     index: int = 0
+    groups: int = 1    # Caffe convolution groups (CaffeNet conv2/4/5 use 2; Table 5 lists 1)
 
     @property
     def x_shape(self):
@@ -45,7 +46,7 @@ class Layer:
 
     @property
     def w_shape(self):
-        return (self.Co, self.C, self.K, self.K)
+        return (self.Co, self.C // self.groups, self.K, self.K)
 
     @property
     def y_shape(self):
@@ -55,12 +56,12 @@ class Layer:
         return replace(self, N=int(n))
 
     def flops_per_pass(self) -> float:
-        """2*C_o*C_i*K_h*K_w*H_o*W_o per image, times N."""
-        return 2.0 * self.Co * self.C * self.K * self.K * self.Ho * self.Ho * self.N
+        """2*C_o*C_i*K_h*K_w*H_o*W_o per image, times N (C_i per group)."""
+        return 2.0 * self.Co * (self.C // self.groups) * self.K * self.K * self.Ho * self.Ho * self.N
 
 
-def _L(name, N, C, HW, Co, K, S, P, Ho, data_fed):
-    return Layer(name, N, C, HW, HW, Co, K, S, P, Ho, data_fed)
+def _L(name, N, C, HW, Co, K, S, P, Ho, data_fed, groups=1):
+    return Layer(name, N, C, HW, HW, Co, K, S, P, Ho, data_fed, groups=groups)
 
 
 # Table 5 (P334-355).  LeNet = the Siamese conv1/conv2 shapes (DESIGN.md R20).
@@ -84,6 +85,30 @@ _TABLE: Dict[int, List[Layer]] = {
         _L("googlenet_conv_4", 128, 192, 7, 384, 3, 1, 1, 7, False),
         _L("googlenet_conv_5", 128, 832, 7, 192, 1, 1, 0, 7, False),
         _L("googlenet_conv_6", 128, 832, 7, 48, 1, 1, 0, 7, False)],
+    # the complete inception 5a and 5b modules (all 12 convolutions; branch
+    # widths from the GoogLeNet prototxt [ext], Table 5 covers 6 of them: conv_1 = 5a/3x3,
+    # conv_2 = 5a/5x5_reduce, conv_3 = 5b/1x1, conv_4 = 5b/3x3, conv_5 = 5b/3x3_reduce,
+    # conv_6 = 5b/5x5_reduce), batch 128, 7x7 maps.  pool_proj reads the 3x3 max-pool of the
+    # module input (same 832x7x7 shape; synthesised).
+    6: [_L("i5a_1x1", 128, 832, 7, 256, 1, 1, 0, 7, False),
+        _L("i5a_3x3_reduce", 128, 832, 7, 160, 1, 1, 0, 7, False),
+        _L("i5a_5x5_reduce", 128, 832, 7, 32, 1, 1, 0, 7, False),
+        _L("i5a_3x3", 128, 160, 7, 320, 3, 1, 1, 7, False),
+        _L("i5a_5x5", 128, 32, 7, 128, 5, 1, 2, 7, False),
+        _L("i5a_pool_proj", 128, 832, 7, 128, 1, 1, 0, 7, False),
+        _L("i5b_1x1", 128, 832, 7, 384, 1, 1, 0, 7, False),
+        _L("i5b_3x3_reduce", 128, 832, 7, 192, 1, 1, 0, 7, False),
+        _L("i5b_5x5_reduce", 128, 832, 7, 48, 1, 1, 0, 7, False),
+        _L("i5b_3x3", 128, 192, 7, 384, 3, 1, 1, 7, False),
+        _L("i5b_5x5", 128, 48, 7, 128, 5, 1, 2, 7, False),
+        _L("i5b_pool_proj", 128, 832, 7, 128, 1, 1, 0, 7, False)],
+    # CaffeNet as the Caffe model defines it, with group = 2 on conv2, conv4
+    # and conv5 [ext: bvlc_reference_caffenet]; Table 5 (P345-349) lists the full C_i (R4).
+    7: [_L("caffenet_conv1", 256, 3, 227, 96, 11, 4, 0, 55, True),
+        _L("caffenet_conv2_g2", 256, 96, 27, 256, 5, 1, 2, 27, False, groups=2),
+        _L("caffenet_conv3", 256, 256, 13, 384, 3, 1, 1, 13, False),
+        _L("caffenet_conv4_g2", 256, 384, 13, 384, 3, 1, 1, 13, False, groups=2),
+        _L("caffenet_conv5_g2", 256, 384, 13, 256, 3, 1, 1, 13, False, groups=2)],
 }
 
 # Sibling layers that read the same input tensor in the real network and can run as one fused
@@ -92,6 +117,8 @@ _TABLE: Dict[int, List[Layer]] = {
 # 832-channel input.  The group uses the first member's x draw as the shared input.
 SIBLINGS: Dict[int, List[List[str]]] = {
     5: [["googlenet_conv_3", "googlenet_conv_5", "googlenet_conv_6"]],
+    6: [["i5a_1x1", "i5a_3x3_reduce", "i5a_5x5_reduce"],
+        ["i5b_1x1", "i5b_3x3_reduce", "i5b_5x5_reduce"]],
 }
 
 CONFIG_NAMES = {
@@ -100,6 +127,8 @@ CONFIG_NAMES = {
     3: "cifar10_quick_conv_b100",
     4: "caffenet_conv1-5_b256",
     5: "googlenet_table5_units_b128",
+    6: "googlenet_inception_5a5b_b128",
+    7: "caffenet_group2_conv1-5_b256",
 }
 
 
@@ -143,7 +172,7 @@ def gen_layer(layer: Layer, n_global: int = None, exact: bool = False, batch: in
             x = _rng(c, i, 0).random(xs, dtype=np.float32)
         else:
             x = np.maximum(_rng(c, i, 0).standard_normal(xs, dtype=np.float32), 0.0)
-        a = np.float32(np.sqrt(3.0 / (layer.C * layer.K * layer.K)))
+        a = np.float32(np.sqrt(3.0 / (layer.C // layer.groups * layer.K * layer.K)))
         w = _rng(c, i, 1).uniform(-a, a, size=ws).astype(np.float32)
         b = _rng(c, i, 2).uniform(-0.1, 0.1, size=(layer.Co,)).astype(np.float32)
         dy = (_rng(c, i, 3).standard_normal(ys, dtype=np.float32) / np.float32(n_global)).astype(np.float32)

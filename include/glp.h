@@ -102,6 +102,14 @@ typedef struct {
 glp_status_t glp_conv_desc_create(glp_conv_desc_t *out, int N, int C_in, int H, int W, int C_out,
                                   int K_h, int K_w, int stride_h, int stride_w, int pad_h,
                                   int pad_w);
+/* Caffe convolution groups (e.g. CaffeNet conv2/conv4/conv5 use 2, which
+ * Table 5 does not list, R4): group g convolves x channels [g*C_in/G, (g+1)*C_in/G) with W rows
+ * [g*C_out/G, (g+1)*C_out/G) of W [C_out][C_in/G][K_h][K_w] into the same y channels; dx, dW, db
+ * likewise.  groups must divide C_in and C_out (GLP_ERR_INVALID_VALUE).  Set before glp_plan;
+ * the plan covers one group's convolution and every call runs the groups in order, each with
+ * its own workspace slice (info.ws_* include all groups).  Not combinable with fused sibling
+ * groups, the stream pool or glp_debug_im2col (GLP_ERR_NOT_SUPPORTED). */
+glp_status_t glp_conv_desc_set_groups(glp_conv_desc_t desc, int groups);
 glp_status_t glp_conv_desc_get_output(glp_conv_desc_t desc, int *H_out, int *W_out);
 glp_status_t glp_conv_desc_destroy(glp_conv_desc_t desc);
 

@@ -60,7 +60,7 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_stage_bwd_filter", "glp_stage_reduce", "glp_conv_group_desc_create",
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
            "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
-           "glp_pool_conv_bwd", "glp_pool_destroy"]
+           "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA = 0, 1, 2, 3, 4
 
@@ -120,6 +120,7 @@ def lib():
         L.glp_pool_conv_fwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_pool_conv_bwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_pool_destroy.argtypes = [_vp]
+        L.glp_conv_desc_set_groups.argtypes = [_vp, _c_int]
         _lib = L
     return _lib
 
@@ -201,8 +202,9 @@ class ConvLayer:
     ``stream`` (default: torch's current stream) without synchronising."""
 
     def __init__(self, N, C, H, W, Co, K, stride=1, pad=0, math="bf16", device=0,
-                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None, branches=None):
+                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None, branches=None, groups=1):
         import torch
+        self.groups = int(groups)
         self.branches = None if branches is None else [int(c) for c in branches]
         if self.branches is not None:
             Co = sum(self.branches)
@@ -219,6 +221,8 @@ class ConvLayer:
             _ck(L.glp_conv_group_desc_create(ctypes.byref(self._desc), g.N, g.C, g.H, g.W,
                                              len(self.branches), ctypes.cast(arr, _vp), g.Kh, g.Kw,
                                              g.Sh, g.Sw, g.Ph, g.Pw), "glp_conv_group_desc_create")
+        if self.groups != 1:
+            _ck(L.glp_conv_desc_set_groups(self._desc, self.groups), "glp_conv_desc_set_groups")
         ho, wo = _c_int(), _c_int()
         _ck(L.glp_conv_desc_get_output(self._desc, ctypes.byref(ho), ctypes.byref(wo)),
             "glp_conv_desc_get_output")
@@ -251,7 +255,7 @@ class ConvLayer:
     @property
     def w_shape(self):
         g = self.geom
-        return (g.Co, g.C, g.Kh, g.Kw)
+        return (g.Co, g.C // self.groups, g.Kh, g.Kw)
 
     def kernel_attr(self, which):
         a, m, r = KernelAttr(), _c_int(), _c_int()

@@ -75,6 +75,7 @@ struct glp_conv_desc_s {
   // channels [br_off[b], br_off[b+1]) of the C_o = sum view; single layer: nbr = 1
   int nbr = 1;
   int br_off[GLP_MAXBR + 1] = {0, 0, 0, 0, 0};
+  int groups = 1;   // Caffe convolution groups (glp_conv_desc_set_groups)
 };
 
 namespace {
@@ -292,6 +293,10 @@ struct glp_plan_s {
   glp_conv_desc_s dxg;
   int Cpx = 0, tapsx = 0;
   PassPlan fwd, dgrad, wgrad;
+  // convolution groups: d above is ONE group's convolution (C/G -> C_o/G); the tensors hold
+  // x_img_c / y_img_c channels per image and every workspace region exists once per group
+  int groups = 1, x_img_c = 0, y_img_c = 0;
+  size_t ws_group = 0;
   // halo filter gradient (hwgrad.cuh) for space-to-depth layers: dy is then packed on the padded
   // dxg.H x dxg.W grid (zeros outside H_o x W_o) and the filter gradient stages x' once per
   // k-block for all taps
@@ -314,6 +319,11 @@ struct glp_plan_s {
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
   int bn_model = 1;    // GLP_BN_MODEL=0: always the default fwd/dgrad tile (A/B runs)
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
+  // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
+  // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
+  // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
+  // instead of after it.  GLP_SMEM_CAP (bytes) overrides (A/B runs).
+  int smem_cap = 232448;
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
@@ -357,7 +367,7 @@ glp_status_t plan_halo(glp_plan_s &P) {
   h.a_bytes = (int)rup((long long)halo_rows * 128, 1024);
   h.b_bytes = (int)cdiv(bn, 64) * HW_BKP * 128;
   const int stage = h.a_bytes + h.b_bytes;
-  h.stages = std::min(8, (232448 - 2048) / stage);
+  h.stages = std::min(8, (P.smem_cap - 2048) / stage);
   if (h.stages < 2) return GLP_OK;
   const long long rows = (long long)x.N * x.H * x.W;
   h.kb_total = (int)cdiv(rows, HW_BKP);
@@ -456,7 +466,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
   // forward: the bias vector is staged once per CTA in smem (every column a tile can touch)
   pp.bias_floats = (mode == MODE_FWD) ? (int)rup((long long)pp.n_tiles * pp.bn, 32) + 32 : 0;
-  const int budget = 232448 - 1024 - 1024 - 4 * pp.bias_floats;   // alignment slack; barriers, TMEM slot
+  const int budget = P.smem_cap - 1024 - 1024 - 4 * pp.bias_floats;   // alignment slack; barriers, TMEM slot
   // k-blocks per pipeline stage: as many (<= 4) as keep >= 3 stages in the ring.  One
   // full/empty round trip of the single MMA-issuing warp costs ~250-700 cycles whatever the stage
   // size (tools/sync_probe*.cu, GLP_DEBUG_SKIP=15 runs), more than the tensor work of one small-N
@@ -650,15 +660,17 @@ DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
 
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
                              int Cp, float *db_part, cudaStream_t st, int Ws = 1, int Wd = 1,
-                             int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1) {
+                             int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1,
+                             int img_c = -1) {
   if (HWd < 0) HWd = HW;   // default: dense destination (Ws == Wd)
+  if (img_c < 0) img_c = C;   // default: the source holds exactly C channels per image
   if (Cw < 0) Cw = Cp;     // default: the whole row (single layer)
   if (db_ld < 0) db_ld = C;
   if (db_part == nullptr && Cp * P.elem <= 32 && Ws == Wd && co_off == 0 && Cw == Cp) {
     const size_t n = (size_t)P.d.N * HW;
     const int g = (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 32);
-    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp));
-    else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<4>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp));
+    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c));
+    else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<4>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c));
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
@@ -666,8 +678,8 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
   const int nt = (int)cdiv(P.d.Co, 32);
-  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld));
-  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld));
+  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
+  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
 }
@@ -683,7 +695,7 @@ glp_status_t launch_pack_dy(const glp_plan_s &P, const BrIn &dy, uint8_t *ws, bo
   const int HWd = P.halo ? P.dxg.H * P.dxg.W : -1;
   if (dy.n <= 1)
     return launch_pack_act(P, dy.p[0], ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
-                           HWd);
+                           HWd, 0, -1, -1, P.y_img_c);
   for (int b = 0; b < dy.n; ++b) {
     const int off = d.br_off[b], cb = d.br_off[b + 1] - off;
     const int cw = (b == dy.n - 1) ? P.Cop - off : cb;
@@ -739,13 +751,14 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
     const int rows = d.N * P.dxg.H;
     dim3 grid((unsigned)std::min(rows, P.sm_count * std::max(1, P.s2d_blocks)));
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
     GLP_LAUNCH_CHECK("pack_s2d");
     return GLP_OK;
   }
-  return launch_pack_act(P, x, dst, d.C, d.H * d.W, P.Cpx, nullptr, st);
+  return launch_pack_act(P, x, dst, d.C, d.H * d.W, P.Cpx, nullptr, st, 1, 1, -1, 0, -1, -1,
+                         P.x_img_c);
 }
 
 glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStream_t st) {
@@ -807,7 +820,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   p.ybr = y;
   for (int i = 0; i < GLP_MAXBR; ++i) p.bias_br[i] = b.p[i];
   p.bias_floats = pp.bias_floats;
-  p.out_c = d.Co;
+  p.out_c = P.y_img_c;   // channels per image of y (the whole tensor for a conv group)
   p.out_hw = d.Ho * d.Wo;
   return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);
 }
@@ -833,7 +846,7 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   }
   IgemmParams p = make_params(P, pp, MODE_DGRAD, dypk);
   p.out = dx;
-  p.out_c = d.C;
+  p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
   p.out_hw = d.H * d.W;
   return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
 }
@@ -954,8 +967,10 @@ __global__ void __launch_bounds__(256) pool_sum_slots(const float *__restrict__ 
   }
 }
 
-ConvGeom geom(const glp_conv_desc_s &d) {
-  return ConvGeom{d.N, d.C, d.H, d.W, d.Co, d.Kh, d.Kw, d.Sh, d.Sw, d.Ph, d.Pw, d.Ho, d.Wo};
+ConvGeom geomP(const glp_plan_s &P) {
+  const glp_conv_desc_s &d = P.d;
+  return ConvGeom{d.N, d.C, d.H, d.W, d.Co, d.Kh, d.Kw, d.Sh, d.Sw, d.Ph, d.Pw, d.Ho, d.Wo,
+                  P.x_img_c, P.y_img_c};
 }
 
 glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, float *dw, float *db,
@@ -964,12 +979,12 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
   const size_t wsz = (size_t)d.Co * d.C * d.Kh * d.Kw;
   float *part = reinterpret_cast<float *>(ws);
   float *dbp = reinterpret_cast<float *>(ws + align1k(wsz * P.simt_splits * 4));
-  simt_wgrad_partial<<<ew_grid(wsz * P.simt_splits), 256, 0, st>>>(geom(d), x, dy, part, P.simt_splits, P.simt_chunk);
+  simt_wgrad_partial<<<ew_grid(wsz * P.simt_splits), 256, 0, st>>>(geomP(P), x, dy, part, P.simt_splits, P.simt_chunk);
   GLP_LAUNCH_CHECK("simt_wgrad_partial");
   reduce_simt_dw<<<ew_grid(wsz), 256, 0, st>>>(part, dw, wsz, P.simt_splits, accumulate);
   GLP_LAUNCH_CHECK("reduce_simt_dw");
   if (db) {
-    simt_db_partial<<<ew_grid((size_t)P.simt_splits * d.Co), 256, 0, st>>>(geom(d), dy, dbp, P.simt_splits, P.simt_chunk);
+    simt_db_partial<<<ew_grid((size_t)P.simt_splits * d.Co), 256, 0, st>>>(geomP(P), dy, dbp, P.simt_splits, P.simt_chunk);
     GLP_LAUNCH_CHECK("simt_db_partial");
     DbAux a = db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.simt_splits);
     GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
@@ -1066,6 +1081,16 @@ glp_status_t glp_conv_group_desc_create(glp_conv_desc_t *out, int N, int C, int 
   return GLP_OK;
 }
 
+glp_status_t glp_conv_desc_set_groups(glp_conv_desc_t d, int groups) {
+  if (!d) return fail(GLP_ERR_INVALID_VALUE, "desc is NULL");
+  if (groups < 1 || d->C % groups || d->Co % groups)
+    return fail(GLP_ERR_INVALID_VALUE, "groups must divide C_in and C_out");
+  if (groups > 1 && d->nbr > 1)
+    return fail(GLP_ERR_NOT_SUPPORTED, "a desc is either a conv group or a fused sibling group");
+  d->groups = groups;
+  return GLP_OK;
+}
+
 glp_status_t glp_conv_desc_get_output(glp_conv_desc_t d, int *Ho, int *Wo) {
   if (!d || !Ho || !Wo) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
   *Ho = d->Ho;
@@ -1130,8 +1155,20 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   GLP_CUDA(cudaGetDevice(&cur));
   if (cur != device) GLP_CUDA(cudaSetDevice(device));
 
+  if (d->groups > 1 && d->nbr > 1)
+    return fail(GLP_ERR_NOT_SUPPORTED, "a desc is either a conv group or a fused sibling group");
   auto *P = new glp_plan_s();
   P->d = *d;
+  P->groups = std::max(1, d->groups);
+  P->x_img_c = d->C;
+  P->y_img_c = d->Co;
+  if (P->groups > 1) {   // plan ONE group's convolution; the calls loop over the groups
+    P->d.C = d->C / P->groups;
+    P->d.Co = d->Co / P->groups;
+    P->d.groups = 1;
+    P->d.br_off[1] = P->d.Co;
+  }
+  d = &P->d;   // everything below plans the (per-group) convolution
   P->device = device;
   P->math = (int)math;
   P->elem = (math == GLP_MATH_BF16) ? 2 : 4;
@@ -1146,6 +1183,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
+  if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
   // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 31;
@@ -1252,6 +1290,11 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->ws_bwd = P->ws_wgrad;
     P->S = S > 0 ? std::min(S, d->N) : d->N;
   }
+  // one workspace slice per convolution group (staged calls keep every group's packs alive)
+  P->ws_group = align1k(std::max({P->ws_fwd, P->ws_dgrad, P->ws_wgrad, P->ws_bwd}));
+  if (P->groups > 1) {
+    P->ws_fwd = P->ws_dgrad = P->ws_wgrad = P->ws_bwd = (size_t)P->groups * P->ws_group;
+  }
   if (cur != device) cudaSetDevice(cur);
   P->plan_us = std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
   *out = P;
@@ -1312,6 +1355,20 @@ static glp_status_t check_ws(const glp_plan_s *P, const void *ws, size_t have, s
   return GLP_OK;
 }
 
+// Pointer offsets of convolution group g (Caffe "group": x/dx channels [g*C_g, (g+1)*C_g),
+// y/dy channels [g*C_o,g, ...), W rows [g*C_o,g, ...) of [C_o][C_g][K_h][K_w], one workspace
+// slice per group).  groups = 1: all zero.
+struct GOff {
+  size_t x, y, w, b, ws;
+};
+static GOff goff(const glp_plan_s *P, int g) {
+  const glp_conv_desc_s &d = P->d;   // the per-group convolution
+  return GOff{(size_t)g * d.C * d.H * d.W, (size_t)g * d.Co * d.Ho * d.Wo,
+              (size_t)g * d.Co * d.C * d.Kh * d.Kw, (size_t)g * d.Co, (size_t)g * P->ws_group};
+}
+static const float *offc(const float *p, size_t o) { return p ? p + o : p; }
+static float *offm(float *p, size_t o) { return p ? p + o : p; }
+
 glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const float *b, float *y,
                           void *ws, size_t ws_bytes, glp_stream_t stream) {
   if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
@@ -1320,15 +1377,20 @@ glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const fl
   if (b && (reinterpret_cast<uintptr_t>(b) % 4)) return fail(GLP_ERR_INVALID_VALUE, "bias misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math == GLP_MATH_FP32) {
-    const size_t n = (size_t)P->d.N * P->d.Co * P->d.Ho * P->d.Wo;
-    simt_fwd<<<ew_grid(n), 256, 0, st>>>(geom(P->d), x, w, b, y);
-    GLP_LAUNCH_CHECK("simt_fwd");
-    return GLP_OK;
+  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    float *yg = y + o.y;
+    if (P->math == GLP_MATH_FP32) {
+      const size_t n = (size_t)P->d.N * P->d.Co * P->d.Ho * P->d.Wo;
+      simt_fwd<<<ew_grid(n), 256, 0, st>>>(geomP(*P), x + o.x, w + o.w, offc(b, o.b), yg);
+      GLP_LAUNCH_CHECK("simt_fwd");
+    } else if ((s = tc_fwd(*P, x + o.x, br_in1(w + o.w), br_in1(offc(b, o.b)), br_out(*P, 1, &yg),
+                           static_cast<uint8_t *>(ws) + o.ws, st))) {
+      return s;
+    }
   }
-  if ((s = get_encode())) return s;
-  float *ys[1] = {y};
-  return tc_fwd(*P, x, br_in1(w), br_in1(b), br_out(*P, 1, ys), static_cast<uint8_t *>(ws), st);
+  return GLP_OK;
 }
 
 glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, float *dx, void *ws,
@@ -1338,17 +1400,22 @@ glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, fl
   if (s) return s;
   if ((s = check_ws(P, ws, ws_bytes, P->ws_dgrad))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math == GLP_MATH_FP32) {
-    const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
-    simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geom(P->d), dy, w, dx);
-    GLP_LAUNCH_CHECK("simt_dgrad");
-    return GLP_OK;
+  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    if (P->math == GLP_MATH_FP32) {
+      const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
+      simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geomP(*P), dy + o.y, w + o.w, dx + o.x);
+      GLP_LAUNCH_CHECK("simt_dgrad");
+      continue;
+    }
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
+    if ((s = launch_pack_dy(*P, br_in1(dy + o.y), wsb, false, st)) ||
+        (s = run_pack_w_dgrad(*P, br_in1(w + o.w), wsb, st)) ||
+        (s = run_dgrad_gemm(*P, dx + o.x, wsb, st)))
+      return s;
   }
-  if ((s = get_encode())) return s;
-  uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if ((s = launch_pack_dy(*P, br_in1(dy), wsb, false, st))) return s;
-  if ((s = run_pack_w_dgrad(*P, br_in1(w), wsb, st))) return s;
-  return run_dgrad_gemm(*P, dx, wsb, st);
+  return GLP_OK;
 }
 
 glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, float *dw, float *db,
@@ -1359,16 +1426,23 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_wgrad))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if (P->math == GLP_MATH_FP32) return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
-  if ((s = get_encode())) return s;
-  void *xpk = wsb + P->off_xpk;
-  if ((s = launch_pack_x(*P, x, xpk, st))) return s;
-  if ((s = launch_pack_dy(*P, br_in1(dy), wsb, db != nullptr, st))) return s;
-  if ((s = run_wgrad_gemm(*P, wsb, st))) return s;
-  float *dws[1] = {dw}, *dbs[1] = {db};
-  const BrOut dbt = br_out(*P, 1, dbs);
-  return run_wgrad_reduce(*P, br_out(*P, 1, dws), db ? &dbt : nullptr, accumulate ? 1 : 0, wsb, st);
+  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
+    float *dwg = dw + o.w, *dbg = offm(db, o.b);
+    if (P->math == GLP_MATH_FP32) {
+      if ((s = run_wgrad_simt(*P, x + o.x, dy + o.y, dwg, dbg, accumulate ? 1 : 0, wsb, st))) return s;
+      continue;
+    }
+    const BrOut dbt = br_out(*P, 1, &dbg);
+    if ((s = launch_pack_x(*P, x + o.x, wsb + P->off_xpk, st)) ||
+        (s = launch_pack_dy(*P, br_in1(dy + o.y), wsb, db != nullptr, st)) ||
+        (s = run_wgrad_gemm(*P, wsb, st)) ||
+        (s = run_wgrad_reduce(*P, br_out(*P, 1, &dwg), db ? &dbt : nullptr, accumulate ? 1 : 0, wsb, st)))
+      return s;
+  }
+  return GLP_OK;
 }
 
 glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const float *w, float *dx,
@@ -1381,19 +1455,26 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
   if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_bwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  uint8_t *wsb = static_cast<uint8_t *>(ws);
-  if (P->math == GLP_MATH_FP32) {
-    if (dx) {
-      const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
-      simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geom(P->d), dy, w, dx);
-      GLP_LAUNCH_CHECK("simt_dgrad");
+  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
+    float *dwg = dw + o.w, *dbg = offm(db, o.b);
+    if (P->math == GLP_MATH_FP32) {
+      if (dx) {
+        const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
+        simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geomP(*P), dy + o.y, w + o.w, dx + o.x);
+        GLP_LAUNCH_CHECK("simt_dgrad");
+      }
+      if ((s = run_wgrad_simt(*P, x + o.x, dy + o.y, dwg, dbg, accumulate ? 1 : 0, wsb, st))) return s;
+      continue;
     }
-    return run_wgrad_simt(*P, x, dy, dw, db, accumulate ? 1 : 0, wsb, st);
+    if ((s = tc_bwd(*P, x + o.x, br_in1(dy + o.y), br_in1(w + o.w), offm(dx, o.x),
+                    br_out(*P, 1, &dwg), db ? br_out(*P, 1, &dbg) : BrOut{}, db != nullptr,
+                    accumulate ? 1 : 0, wsb, st)))
+      return s;
   }
-  if ((s = get_encode())) return s;
-  float *dws[1] = {dw}, *dbs[1] = {db};
-  return tc_bwd(*P, x, br_in1(dy), br_in1(w), dx, br_out(*P, 1, dws), db ? br_out(*P, 1, dbs) : BrOut{},
-                db != nullptr, accumulate ? 1 : 0, wsb, st);
+  return GLP_OK;
 }
 
 static glp_status_t stage_check(glp_plan_t P, void *ws, size_t ws_bytes) {
@@ -1410,18 +1491,20 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
   if (s) return s;
   if ((s = validate_ptrs({src}))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  uint8_t *wsb = static_cast<uint8_t *>(ws);
-  switch (what) {
-    case GLP_PACK_X:
-      return launch_pack_x(*P, src, wsb + P->off_xpk, st);
-    case GLP_PACK_DY:
-      return launch_pack_dy(*P, br_in1(src), wsb, false, st);
-    case GLP_PACK_DY_DB:
-      return launch_pack_dy(*P, br_in1(src), wsb, true, st);
-    case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, br_in1(src), wsb, st);
-    case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, br_in1(src), wsb, st);
+  if (what < GLP_PACK_X || what > GLP_PACK_W_BWD_DATA) return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
+    switch (what) {
+      case GLP_PACK_X: s = launch_pack_x(*P, src + o.x, wsb + P->off_xpk, st); break;
+      case GLP_PACK_DY: s = launch_pack_dy(*P, br_in1(src + o.y), wsb, false, st); break;
+      case GLP_PACK_DY_DB: s = launch_pack_dy(*P, br_in1(src + o.y), wsb, true, st); break;
+      case GLP_PACK_W_FWD: s = run_pack_w_fwd(*P, br_in1(src + o.w), wsb, st); break;
+      case GLP_PACK_W_BWD_DATA: s = run_pack_w_dgrad(*P, br_in1(src + o.w), wsb, st); break;
+    }
+    if (s) return s;
   }
-  return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
+  return GLP_OK;
 }
 
 glp_status_t glp_stage_fwd(glp_plan_t P, const float *b, float *y, void *ws, size_t ws_bytes,
@@ -1429,9 +1512,14 @@ glp_status_t glp_stage_fwd(glp_plan_t P, const float *b, float *y, void *ws, siz
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
   if ((s = validate_ptrs({y}))) return s;
-  float *ys[1] = {y};
-  return run_fwd_gemm(*P, br_in1(b), br_out(*P, 1, ys), static_cast<uint8_t *>(ws),
-                      static_cast<cudaStream_t>(stream));
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    float *yg = y + o.y;
+    if ((s = run_fwd_gemm(*P, br_in1(offc(b, o.b)), br_out(*P, 1, &yg), static_cast<uint8_t *>(ws) + o.ws,
+                          static_cast<cudaStream_t>(stream))))
+      return s;
+  }
+  return GLP_OK;
 }
 
 glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_bytes,
@@ -1439,13 +1527,23 @@ glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_byt
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
   if ((s = validate_ptrs({dx}))) return s;
-  return run_dgrad_gemm(*P, dx, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    if ((s = run_dgrad_gemm(*P, dx + o.x, static_cast<uint8_t *>(ws) + o.ws,
+                            static_cast<cudaStream_t>(stream))))
+      return s;
+  }
+  return GLP_OK;
 }
 
 glp_status_t glp_stage_bwd_filter(glp_plan_t P, void *ws, size_t ws_bytes, glp_stream_t stream) {
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
-  return run_wgrad_gemm(*P, static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+  for (int g = 0; g < P->groups; ++g)
+    if ((s = run_wgrad_gemm(*P, static_cast<uint8_t *>(ws) + goff(P, g).ws,
+                            static_cast<cudaStream_t>(stream))))
+      return s;
+  return GLP_OK;
 }
 
 glp_status_t glp_stage_reduce(glp_plan_t P, float *dw, float *db, int accumulate, void *ws,
@@ -1453,10 +1551,15 @@ glp_status_t glp_stage_reduce(glp_plan_t P, float *dw, float *db, int accumulate
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
   if ((s = validate_ptrs({dw}))) return s;
-  float *dws[1] = {dw}, *dbs[1] = {db};
-  const BrOut dbt = br_out(*P, 1, dbs);
-  return run_wgrad_reduce(*P, br_out(*P, 1, dws), db ? &dbt : nullptr, accumulate ? 1 : 0,
-                          static_cast<uint8_t *>(ws), static_cast<cudaStream_t>(stream));
+  for (int g = 0; g < P->groups; ++g) {
+    const GOff o = goff(P, g);
+    float *dwg = dw + o.w, *dbg = offm(db, o.b);
+    const BrOut dbt = br_out(*P, 1, &dbg);
+    if ((s = run_wgrad_reduce(*P, br_out(*P, 1, &dwg), db ? &dbt : nullptr, accumulate ? 1 : 0,
+                              static_cast<uint8_t *>(ws) + o.ws, static_cast<cudaStream_t>(stream))))
+      return s;
+  }
+  return GLP_OK;
 }
 
 // ---- fused sibling groups ----
@@ -1567,6 +1670,7 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   glp_status_t s = validate_ptrs({x, col});
   if (s) return s;
   if (n < 0 || n >= P->d.N) return fail(GLP_ERR_INVALID_VALUE, "sample index out of range");
+  if (P->groups > 1) return fail(GLP_ERR_NOT_SUPPORTED, "debug im2col of a grouped layer");
   if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no packed operand");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -1624,7 +1728,8 @@ glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t d, int device, glp
   if (!out || !d) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
   *out = nullptr;
   if (n_streams < 0) return fail(GLP_ERR_INVALID_VALUE, "n_streams < 0");
-  if (d->nbr > 1) return fail(GLP_ERR_NOT_SUPPORTED, "the stream pool runs single layers");
+  if (d->nbr > 1 || d->groups > 1)
+    return fail(GLP_ERR_NOT_SUPPORTED, "the stream pool runs single ungrouped layers");
   auto *Q = new glp_pool_s();
   Q->d1 = *d;
   Q->d1.N = 1;
@@ -1723,7 +1828,7 @@ glp_status_t glp_pool_conv_fwd(glp_pool_t Q, const float *x, const float *w, con
           (s = run_fwd_gemm(P1, br_in1(b), br_out(P1, 1, &yn), wsi, si)))
         return s;
     } else {
-      simt_fwd<<<ew_grid(ys), 256, 0, si>>>(geom(P1.d), x + n * xs, w, b, yn);
+      simt_fwd<<<ew_grid(ys), 256, 0, si>>>(geomP(P1), x + n * xs, w, b, yn);
       GLP_LAUNCH_CHECK("simt_fwd");
     }
   }
@@ -1769,7 +1874,7 @@ glp_status_t glp_pool_conv_bwd(glp_pool_t Q, const float *x, const float *dy, co
         return s;
     } else {
       if (dx) {
-        simt_dgrad<<<ew_grid(xs), 256, 0, si>>>(geom(P1.d), dyn, w, dx + n * xs);
+        simt_dgrad<<<ew_grid(xs), 256, 0, si>>>(geomP(P1), dyn, w, dx + n * xs);
         GLP_LAUNCH_CHECK("simt_dgrad");
       }
       if ((s = run_wgrad_simt(P1, xn, dyn, dwi, dbi, 1, wsi, si))) return s;

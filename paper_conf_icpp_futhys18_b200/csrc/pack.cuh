@@ -62,7 +62,8 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
                                                          int HW, int Cp, float *__restrict__ db_part,
                                                          unsigned int *__restrict__ tickets,
                                                          int n_tickets, int Ws, int Wd, int HWd,
-                                                         int co_off, int Cw, int db_ld) {
+                                                         int co_off, int Cw, int db_ld, int src_c) {
+  // src_c: channels per image of the source tensor (> C when packing one group's channel slice).
   // (co_off, Cw, db_ld): this call writes destination channels [co_off, co_off + Cw) of rows with
   // pitch Cp (source channels 0..C-1, zeros past C) and db_part columns co_off + c of width db_ld —
   // one branch of a fused sibling group.  Single layer: co_off = 0, Cw = Cp, db_ld = C.
@@ -95,7 +96,7 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
         sp = h * Ws + w;
       }
       sok[i] = ok;
-      soff[i] = (long long)n * C * HW + sp;
+      soff[i] = (long long)n * src_c * HW + sp;
       p += 32;
       while (p >= HWd) {
         p -= HWd;
@@ -148,14 +149,14 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__restrict__ src,
                                                                void *__restrict__ dst, int N, int C,
-                                                               int HW, int Cp) {
+                                                               int HW, int Cp, int src_c) {
   pdl_launch_dependents();
   pdl_wait();
   const size_t total = (size_t)N * HW;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total;
        i += (size_t)gridDim.x * blockDim.x) {
     const size_t n = i / HW, px = i % HW;
-    const float *s = src + n * C * HW + px;
+    const float *s = src + n * src_c * HW + px;
     for (int c = 0; c < Cp; c += 4) {
       float a[4];
 #pragma unroll
@@ -179,7 +180,7 @@ constexpr int S2D_LD = 12;   // staged source floats per thread per row (S*C*W <
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
                                                 int N, int C, int H, int W, int S, int P, int Hs,
-                                                int Ws, int Cps) {
+                                                int Ws, int Cps, int src_c) {
   extern __shared__ float rows[];   // [S*C][W] source rows (row r = dh*C + c)
   constexpr int CH = 16 / ELEM;     // channels per 16-byte chunk
   pdl_launch_dependents();
@@ -218,7 +219,7 @@ __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, voi
   float v[S2D_LD];
   auto issue = [&](int row) {
     const int n = row / Hs, hs = row - n * Hs;
-    const float *xb = x + (size_t)n * C * H * W;
+    const float *xb = x + (size_t)n * src_c * H * W;
 #pragma unroll
     for (int i = 0; i < S2D_LD; ++i) {
       const int ih = S * hs + ldh[i] - P;

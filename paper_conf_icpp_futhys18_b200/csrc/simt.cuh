@@ -10,6 +10,7 @@ namespace glp {
 
 struct ConvGeom {
   int N, C, H, W, Co, Kh, Kw, Sh, Sw, Ph, Pw, Ho, Wo;
+  int xc, yc;   // channels per image of the x/dx and y/dy tensors (> C, Co for a conv group)
 };
 
 // y[n,co,ho,wo] = b[co] + sum_{ci,kh,kw} W * x  (Alg. 1, P82-99).  One thread per output.
@@ -26,7 +27,7 @@ __global__ void simt_fwd(ConvGeom g, const float *__restrict__ x, const float *_
     const int n = (int)(r / g.Co);
     float acc = 0.f;
     for (int ci = 0; ci < g.C; ++ci) {
-      const float *xc = x + ((size_t)n * g.C + ci) * g.H * g.W;
+      const float *xc = x + ((size_t)n * g.xc + ci) * g.H * g.W;
       const float *wc = w + ((size_t)co * g.C + ci) * g.Kh * g.Kw;
       for (int kh = 0; kh < g.Kh; ++kh) {
         const int ih = ho * g.Sh - g.Ph + kh;
@@ -39,7 +40,7 @@ __global__ void simt_fwd(ConvGeom g, const float *__restrict__ x, const float *_
       }
     }
     if (b) acc += __ldg(b + co);
-    y[i] = acc;
+    y[(((size_t)n * g.yc + co) * g.Ho + ho) * g.Wo + wo] = acc;
   }
 }
 
@@ -58,7 +59,7 @@ __global__ void simt_dgrad(ConvGeom g, const float *__restrict__ dy, const float
     const int n = (int)(r / g.C);
     float acc = 0.f;
     for (int co = 0; co < g.Co; ++co) {
-      const float *dyc = dy + ((size_t)n * g.Co + co) * g.Ho * g.Wo;
+      const float *dyc = dy + ((size_t)n * g.yc + co) * g.Ho * g.Wo;
       const float *wc = w + ((size_t)co * g.C + ci) * g.Kh * g.Kw;
       for (int kh = 0; kh < g.Kh; ++kh) {
         const int hn = ih + g.Ph - kh;
@@ -74,7 +75,7 @@ __global__ void simt_dgrad(ConvGeom g, const float *__restrict__ dy, const float
         }
       }
     }
-    dx[i] = acc;
+    dx[(((size_t)n * g.xc + ci) * g.H + ih) * g.W + iw] = acc;
   }
 }
 
@@ -105,8 +106,8 @@ __global__ void simt_wgrad_partial(ConvGeom g, const float *__restrict__ x,
       const int ho = p / g.Wo, wo = p % g.Wo;
       const int ih = ho * g.Sh - g.Ph + kh, iw = wo * g.Sw - g.Pw + kw;
       if (ih < 0 || ih >= g.H || iw < 0 || iw >= g.W) continue;
-      acc = fmaf(__ldg(dy + ((size_t)n * g.Co + co) * hw + p),
-                 __ldg(x + (((size_t)n * g.C + ci) * g.H + ih) * g.W + iw), acc);
+      acc = fmaf(__ldg(dy + ((size_t)n * g.yc + co) * hw + p),
+                 __ldg(x + (((size_t)n * g.xc + ci) * g.H + ih) * g.W + iw), acc);
     }
     part[i] = acc;
   }
@@ -126,7 +127,7 @@ __global__ void simt_db_partial(ConvGeom g, const float *__restrict__ dy, float 
     const long long q1 = q0 + chunk < npix ? q0 + chunk : npix;
     for (long long q = q0; q < q1; ++q) {
       const int n = (int)(q / hw), p = (int)(q % hw);
-      acc += __ldg(dy + ((size_t)n * g.Co + co) * hw + p);
+      acc += __ldg(dy + ((size_t)n * g.yc + co) * hw + p);
     }
     part[i] = acc;
   }

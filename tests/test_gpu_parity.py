@@ -435,3 +435,66 @@ def test_stream_pool_comparator(shape, math):
                 for k in ("dw", "db"):
                     r = ref_layer[k]
                     assert np.abs(got[k] - r).max() / np.abs(r).max() <= TOL[math], k
+
+
+# Caffe convolution groups (glp_conv_desc_set_groups): name, N, C, H, W, Co,
+# K, S, P, groups
+GROUPED = [
+    ("caffenet_conv2_g2", 2, 96, 27, 27, 256, 5, 1, 2, 2),
+    ("caffenet_conv4_g2", 3, 384, 13, 13, 384, 3, 1, 1, 2),
+    ("s4_k11_g3", 2, 6, 35, 35, 48, 11, 4, 0, 3),     # space-to-depth + halo per group
+    ("g4_ragged", 3, 32, 9, 11, 40, 3, 2, 1, 4),
+]
+
+
+def _grouped_oracle(d, S, P, G):
+    x, w, b, dy = d["x"], d["w"], d["b"], d["dy"]
+    C, Co = x.shape[1], w.shape[0]
+    cg, og = C // G, Co // G
+    out = {"y": [], "dx": [], "dw": [], "db": []}
+    for g in range(G):
+        xs, ws_ = x[:, g * cg:(g + 1) * cg], w[g * og:(g + 1) * og]
+        dys = dy[:, g * og:(g + 1) * og]
+        out["y"].append(oracle.conv_fwd(xs, ws_, b[g * og:(g + 1) * og], S, P))
+        out["dx"].append(oracle.conv_bwd_data(dys, ws_, xs.shape, S, P))
+        out["dw"].append(oracle.conv_bwd_filter(xs, dys, ws_.shape, S, P)[0])
+    return {"y": np.concatenate(out["y"], 1), "dx": np.concatenate(out["dx"], 1),
+            "dw": np.concatenate(out["dw"], 0), "db": dy.astype(np.float64).sum(axis=(0, 2, 3))}
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("shape", GROUPED, ids=lambda s: s[0])
+def test_grouped_conv(shape, math):
+    """Grouped convolution equals the oracle of each group: bit-exact on integer data (every
+    math mode), within the bar on random data; the staged calls equal the composed ones."""
+    _, N, C, H, W, Co, K, S, P, G = shape
+    Ho, Wo = oracle.out_dim(H, K, S, P), oracle.out_dim(W, K, S, P)
+    for exact, seed in ((True, 71), (False, 72)):
+        d = gen_custom(N, C // G, H, W, Co, K, K, seed, exact=exact, Ho=Ho, Wo=Wo)
+        d["x"] = gen_custom(N, C, H, W, Co, K, K, seed + 100, exact=exact, Ho=Ho, Wo=Wo)["x"]
+        layer = glp.ConvLayer(N, C, H, W, Co, K, S, P, math=math, groups=G)
+        assert layer.w_shape == d["w"].shape
+        got = _run(layer, d)
+        ref = _grouped_oracle(d, S, P, G)
+        for k in ("y", "dx", "dw", "db"):
+            if exact:
+                np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+            else:
+                assert np.abs(got[k] - ref[k]).max() / np.abs(ref[k]).max() <= TOL[math], k
+    if math != "fp32":
+        t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+        y = torch.empty(layer.y_shape, device=DEV)
+        dx = torch.empty(layer.x_shape, device=DEV)
+        dw = torch.empty(layer.w_shape, device=DEV)
+        db = torch.empty(Co, device=DEV)
+        layer.stage_pack(glp.GLP_PACK_X, t["x"])
+        layer.stage_pack(glp.GLP_PACK_W_FWD, t["w"])
+        layer.stage_fwd(t["b"], y)
+        layer.stage_pack(glp.GLP_PACK_DY_DB, t["dy"])
+        layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
+        layer.stage_bwd_data(dx)
+        layer.stage_bwd_filter()
+        layer.stage_reduce(dw, db)
+        torch.cuda.synchronize()
+        for k, v in (("y", y), ("dx", dx), ("dw", dw), ("db", db)):
+            np.testing.assert_array_equal(v.cpu().numpy(), got[k], err_msg="staged " + k)

@@ -67,9 +67,10 @@ def _check_torch(x, w, b, dy, s, p, tol=1e-12):
 def test_torch_fp64_config_shapes(layer):
     """torch fp64 conv2d / conv2d_input / conv2d_weight (cross-correlation, zero pad, floor
     output size) on every Table 5 shape at a reduced batch."""
-    n = 1 if layer.cfg == 4 else 2
-    d = gen_custom(n, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.K, 1234 + layer.index,
-                   Ho=layer.Ho, Wo=layer.Ho)
+    n = 1 if layer.cfg in (4, 7) else 2
+    g = layer.groups   # one group's convolution (the groups are independent convolutions)
+    d = gen_custom(n, layer.C // g, layer.H, layer.W, layer.Co // g, layer.K, layer.K,
+                   1234 + layer.index, Ho=layer.Ho, Wo=layer.Ho)
     _check_torch(d["x"], d["w"], d["b"], d["dy"], layer.S, layer.P)
 
 

@@ -380,12 +380,21 @@ def run_glp(args, ws, rank, local):
         with CUDA events around each GEMM for the per-kernel attribution."""
         stream = torch.cuda.current_stream()   # the capture stream while a graph is recorded
         conc = (ev is None) if concurrent is None else concurrent
+
+        def mark(e):
+            # attribution runs: a GPU-side spin before each start event keeps the stream busy while
+            # the host enqueues the event and the kernel, so the interval holds the kernel only
+            # (without it, host launch latency of small kernels leaked into their timings)
+            if e is ev[i][0] or e is ev[i][2] or e is ev[i][4]:
+                torch.cuda._sleep(40000)
+            e.record(stream)
+
         if not conc:
             for i, s in enumerate(states):
                 s.pack_x()
                 s.pack_w_fwd()
                 if ev is not None:
-                    ev[i][0].record(stream)
+                    mark(ev[i][0])
                 s.fwd()
                 if ev is not None:
                     ev[i][1].record(stream)
@@ -395,12 +404,12 @@ def run_glp(args, ws, rank, local):
                 if s.dx is not None:
                     s.pack_w_bwd()
                     if ev is not None:
-                        ev[i][2].record(stream)
+                        mark(ev[i][2])
                     s.bwd_data()
                     if ev is not None:
                         ev[i][3].record(stream)
                 if ev is not None:
-                    ev[i][4].record(stream)
+                    mark(ev[i][4])
                 s.bwd_filter()
                 if ev is not None:
                     ev[i][5].record(stream)

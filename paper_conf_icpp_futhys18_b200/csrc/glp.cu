@@ -282,8 +282,25 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
 
 }  // namespace
 
+// Tensor maps of a pass depend only on the workspace address (the packed operands live there):
+// cached per (pass, workspace) so repeated calls skip the driver encode (host latency that
+// left the GPU idle between small launches).  Copies of a plan start with an empty cache.
+struct MapCache {
+  struct Entry {
+    const void *ws = nullptr;
+    CUtensorMap a, b;
+  };
+  Entry e[3][8];
+  int next[3] = {0, 0, 0};
+  std::mutex mu;
+  MapCache() = default;
+  MapCache(const MapCache &) {}
+  MapCache &operator=(const MapCache &) { return *this; }
+};
+
 struct glp_plan_s {
   glp_conv_desc_s d;
+  MapCache maps;
   int device = 0, math = 0, elem = 4, sm_count = 148, s_override = 0;
   int Cp = 0, Cop = 0, taps = 0;
   // Geometry of the x operand as the forward and filter-gradient passes see it: the layer itself,
@@ -796,6 +813,28 @@ BrOut br_out(const glp_plan_s &P, int n, float *const *ptrs) {
   return t;
 }
 
+template <typename F>
+glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, CUtensorMap &a, CUtensorMap &b,
+                         F encode) {
+  std::lock_guard<std::mutex> lk(P.maps.mu);
+  for (auto &e : P.maps.e[pass])
+    if (e.ws == ws) {
+      a = e.a;
+      b = e.b;
+      return GLP_OK;
+    }
+  memset(&a, 0, sizeof(a));
+  memset(&b, 0, sizeof(b));
+  glp_status_t s = encode(a, b);
+  if (s) return s;
+  auto &e = P.maps.e[pass][P.maps.next[pass]];
+  P.maps.next[pass] = (P.maps.next[pass] + 1) % 8;
+  e.ws = ws;
+  e.a = a;
+  e.b = b;
+  return GLP_OK;
+}
+
 glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
                           cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
@@ -803,17 +842,16 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
   const int BK = pp.krow / P.elem;
   CUtensorMap mapB, mapA;
-  memset(&mapA, 0, sizeof(mapA));
-  glp_status_t s = encode_2d(&mapB, P.elem, wpk, (uint64_t)pp.Kpad, (uint64_t)d.Co,
-                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
-                             swz_kmajor(pp.krow));
+  glp_status_t s = cached_maps(P, 0, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
+    glp_status_t r = encode_2d(&B, P.elem, wpk, (uint64_t)pp.Kpad, (uint64_t)d.Co,
+                               (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
+                               swz_kmajor(pp.krow));
+    if (r || !pp.a_tma) return r;
+    if ((r = get_encode_im2col())) return r;
+    return encode_im2col(&A, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
+                         d.Ph - (d.Kh - 1), BK, 128, d.Sw, d.Sh, swz_kmajor(pp.krow));
+  });
   if (s) return s;
-  if (pp.a_tma) {
-    if ((s = get_encode_im2col())) return s;
-    s = encode_im2col(&mapA, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
-                      d.Ph - (d.Kh - 1), BK, 128, d.Sw, d.Sh, swz_kmajor(pp.krow));
-    if (s) return s;
-  }
   IgemmParams p = make_params(P, pp, MODE_FWD, xpk);
   p.out = y.p[0];
   p.bias = b.p[0];
@@ -832,18 +870,17 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   const void *dypk = ws + P.off_dypk;
   const int BK = pp.krow / P.elem;
   CUtensorMap mapB, mapA;
-  memset(&mapA, 0, sizeof(mapA));
-  glp_status_t s = encode_2d(&mapB, P.elem, wtpk, (uint64_t)pp.Kpad, (uint64_t)d.C,
-                             (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
-                             swz_kmajor(pp.krow));
-  if (s) return s;
-  if (pp.a_tma) {
+  glp_status_t s = cached_maps(P, 1, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
+    glp_status_t r = encode_2d(&B, P.elem, wtpk, (uint64_t)pp.Kpad, (uint64_t)d.C,
+                               (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
+                               swz_kmajor(pp.krow));
+    if (r || !pp.a_tma) return r;
     // dx pixel (h, w) reads dy at (h - (Kh-1-Ph) + kh', w - (Kw-1-Pw) + kw') with kh' = Kh-1-kh
-    if ((s = get_encode_im2col())) return s;
-    s = encode_im2col(&mapA, P.elem, dypk, P.Cop, d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw),
-                      -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK, 128, 1, 1, swz_kmajor(pp.krow));
-    if (s) return s;
-  }
+    if ((r = get_encode_im2col())) return r;
+    return encode_im2col(&A, P.elem, dypk, P.Cop, d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw),
+                         -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK, 128, 1, 1, swz_kmajor(pp.krow));
+  });
+  if (s) return s;
   IgemmParams p = make_params(P, pp, MODE_DGRAD, dypk);
   p.out = dx;
   p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
@@ -855,13 +892,14 @@ glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
   const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x' and dy
   CUtensorMap mapX, mapDy;
-  glp_status_t s = encode_2d(&mapX, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows,
-                             (uint64_t)P.Cpx * 2, 64u, (uint32_t)P.hw.halo_rows,
-                             CU_TENSOR_MAP_SWIZZLE_128B);
+  glp_status_t s = cached_maps(P, 2, ws, mapX, mapDy, [&](CUtensorMap &X, CUtensorMap &Dy) {
+    glp_status_t r = encode_2d(&X, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
+                               64u, (uint32_t)P.hw.halo_rows, CU_TENSOR_MAP_SWIZZLE_128B);
+    if (r) return r;
+    return encode_2d(&Dy, 2, ws + P.off_dypk, (uint64_t)P.Cop, rows, (uint64_t)P.Cop * 2, 64u,
+                     (uint32_t)HW_BKP, CU_TENSOR_MAP_SWIZZLE_128B);
+  });
   if (s) return s;
-  if ((s = encode_2d(&mapDy, 2, ws + P.off_dypk, (uint64_t)P.Cop, rows, (uint64_t)P.Cop * 2, 64u,
-                     (uint32_t)HW_BKP, CU_TENSOR_MAP_SWIZZLE_128B)))
-    return s;
   HwgradParams p = P.hw;
   p.part = reinterpret_cast<float *>(ws + P.off_part);
   p.dbg_skip = P.dbg_skip;
@@ -890,17 +928,16 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   float *part = reinterpret_cast<float *>(ws + P.off_part);
   const int BKP = 128 / P.elem, EPA = pp.krow / P.elem;
   CUtensorMap mapB, mapA;
-  memset(&mapA, 0, sizeof(mapA));
-  glp_status_t s = encode_2d(&mapB, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
-                             (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
-                             swz_mnmajor(P.elem, pp.krow));
+  glp_status_t s = cached_maps(P, 2, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
+    glp_status_t r = encode_2d(&B, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
+                               (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
+                               swz_mnmajor(P.elem, pp.krow));
+    if (r || !pp.a_tma) return r;
+    if ((r = get_encode_im2col())) return r;
+    return encode_im2col(&A, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
+                         d.Ph - (d.Kh - 1), EPA, BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
+  });
   if (s) return s;
-  if (pp.a_tma) {
-    if ((s = get_encode_im2col())) return s;
-    s = encode_im2col(&mapA, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
-                      d.Ph - (d.Kh - 1), EPA, BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
-    if (s) return s;
-  }
   IgemmParams p = make_params(P, pp, MODE_WGRAD, xpk);
   p.out = part;
   return launch_igemm<MODE_WGRAD>(P, pp, p, mapB, mapA, st);

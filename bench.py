@@ -29,7 +29,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from glp_workloads import CONFIG_NAMES, SIBLINGS, config, gen_layer  # noqa: E402
+from glp_workloads import CONFIG_NAMES, LEVELS, SIBLINGS, config, gen_layer  # noqa: E402
 
 METRIC = "conv fwd+bwd images/sec"
 UNIT = "images/s"
@@ -50,6 +50,10 @@ def parse_args():
                         "stream pool sized by Eq. 7) as a comparator; 1 GPU")
     p.add_argument("--pool-streams", type=int, default=0,
                    help="stream-pool size (0 = the Eq. 7 bound)")
+    p.add_argument("--chain", action="store_true",
+                   help="treat the workload as a chain of layers even where the network runs "
+                        "branches in parallel (default: independent layers of a level run on "
+                        "concurrent streams, glp_workloads.LEVELS)")
     p.add_argument("--no-fuse", action="store_true",
                    help="run sibling layers that share an input (GoogLeNet 5b 1x1 branches) as "
                         "separate layers instead of one fused group")
@@ -367,15 +371,31 @@ def run_glp(args, ws, rank, local):
                                      idxs))
     stream = torch.cuda.current_stream()
 
+    # network DAG levels (units of one level are independent: concurrent streams, the GLP4NN idea
+    # of concurrent kernels applied to a real step's independent layers); default: a chain
+    lv = None if args.chain else LEVELS.get(args.workload)
+    if lv:
+        where = {name: k for k, names in enumerate(lv) for name in names}
+        unit_level = [where[(s.members[0] if isinstance(s, GroupState) else s.layer).name]
+                      for s in states]
+        levels = [[i for i, u in enumerate(unit_level) if u == k] for k in range(len(lv))]
+        levels = [l for l in levels if l]
+    else:
+        levels = [[i] for i in range(len(states))]
+    width = max(len(l) for l in levels)
     side_w = torch.cuda.Stream(device=dev)   # weight packs (weights are known at step start)
-    side_g = torch.cuda.Stream(device=dev)   # filter gradients: wgrad GEMM + dW/db reduction
+    # per slot of a level: a forward/backward-data stream (slot 0 = the main stream) and a
+    # filter-gradient stream (wgrad GEMM + dW/db reduction)
+    fstreams = [None] + [torch.cuda.Stream(device=dev) for _ in range(width - 1)]
+    gstreams = [torch.cuda.Stream(device=dev) for _ in range(width)]
 
     def step(ev=None, concurrent=None):
         """One training step of every layer's hot path.  concurrent (default: not timing kernels):
-        the stream DAG of a real network's step -- forward chain and backward-data chain on the
-        main stream; both weight packs of every layer on side stream W at step start; each
-        layer's filter-gradient GEMM + reductions on side stream G as soon as its dy is packed
-        (they overlap the next layer's backward-data work, which does not depend on them); G is
+        the stream DAG of a real network's step -- per DAG level, each unit's forward chain and
+        backward-data chain on its own stream (one level = independent layers; the main stream
+        for a chain); both weight packs of every unit on side stream W at step start; each unit's
+        filter-gradient GEMM + reductions on a G stream as soon as its dy is packed (they overlap
+        the next level's backward-data work, which does not depend on them); everything is
         joined before the step ends.  Serial (ev given): everything on the main stream, in order,
         with CUDA events around each GEMM for the per-kernel attribution."""
         stream = torch.cuda.current_stream()   # the capture stream while a graph is recorded
@@ -385,8 +405,7 @@ def run_glp(args, ws, rank, local):
             # attribution runs: a GPU-side spin before each start event keeps the stream busy while
             # the host enqueues the event and the kernel, so the interval holds the kernel only
             # (without it, host launch latency of small kernels leaked into their timings)
-            if e is ev[i][0] or e is ev[i][2] or e is ev[i][4]:
-                torch.cuda._sleep(40000)
+            torch.cuda._sleep(40000)
             e.record(stream)
 
         if not conc:
@@ -417,40 +436,59 @@ def run_glp(args, ws, rank, local):
             if G > 1:
                 grads.allreduce()
             return
+        fs = [stream] + fstreams[1:]
         side_w.wait_stream(stream)
-        side_g.wait_stream(stream)
-        ew_f, ew_b = [], []
+        for g in gstreams:
+            g.wait_stream(stream)
+        ew_f, ew_b = {}, {}
         with torch.cuda.stream(side_w):
-            for s in states:
+            for i, s in enumerate(states):
                 s.pack_w_fwd(side_w)
-                e = torch.cuda.Event()
-                e.record(side_w)
-                ew_f.append(e)
-            for s in reversed(states):
+                ew_f[i] = torch.cuda.Event()
+                ew_f[i].record(side_w)
+            for i in reversed(range(len(states))):
+                s = states[i]
                 if s.dx is not None:
                     s.pack_w_bwd(side_w)
-                e = torch.cuda.Event()
-                e.record(side_w)
-                ew_b.append(e)
-        ew_b = ew_b[::-1]
-        for i, s in enumerate(states):
-            s.pack_x()
-            stream.wait_event(ew_f[i])
-            s.fwd()
-        for i in reversed(range(len(states))):
-            s = states[i]
-            s.pack_dy()
-            e_dy = torch.cuda.Event()
-            e_dy.record(stream)
-            side_g.wait_event(e_dy)
-            with torch.cuda.stream(side_g):
-                s.bwd_filter(side_g)
-                s.reduce(side_g)
-            if s.dx is not None:
-                stream.wait_event(ew_b[i])
-                s.bwd_data()
+                ew_b[i] = torch.cuda.Event()
+                ew_b[i].record(side_w)
+
+        def fork(n):
+            for k in range(1, n):
+                fs[k].wait_stream(stream)
+
+        def join(n):
+            for k in range(1, n):
+                stream.wait_stream(fs[k])
+
+        for lvl in levels:
+            fork(len(lvl))
+            for k, i in enumerate(lvl):
+                s, f = states[i], fs[k]
+                with torch.cuda.stream(f):
+                    s.pack_x(f)
+                    f.wait_event(ew_f[i])
+                    s.fwd(f)
+            join(len(lvl))
+        for lvl in reversed(levels):
+            fork(len(lvl))
+            for k, i in enumerate(lvl):
+                s, f, g = states[i], fs[k], gstreams[k]
+                with torch.cuda.stream(f):
+                    s.pack_dy(f)
+                    e_dy = torch.cuda.Event()
+                    e_dy.record(f)
+                    g.wait_event(e_dy)
+                    with torch.cuda.stream(g):
+                        s.bwd_filter(g)
+                        s.reduce(g)
+                    if s.dx is not None:
+                        f.wait_event(ew_b[i])
+                        s.bwd_data(f)
+            join(len(lvl))
         stream.wait_stream(side_w)
-        stream.wait_stream(side_g)
+        for g in gstreams:
+            stream.wait_stream(g)
         if G > 1:
             grads.allreduce()
 
@@ -598,7 +636,8 @@ def run_glp(args, ws, rank, local):
         "e2e": e2e,
         "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
         "launch": ("cuda_graph" if use_graph else "eager") +
-                  ("" if (args.serial or not use_graph) else " (3-stream step DAG)"),
+                  ("" if (args.serial or not use_graph) else
+                   f" (step DAG: {len(levels)} levels, up to {width} concurrent units)"),
     }
     print(json.dumps(line), flush=True)
     if G > 1:

@@ -121,6 +121,23 @@ SIBLINGS: Dict[int, List[List[str]]] = {
         ["i5b_1x1", "i5b_3x3_reduce", "i5b_5x5_reduce"]],
 }
 
+# The network DAG of a workload as levels of layers that are independent of each other in the
+# real network (same level = may run concurrently; level l+1 depends on level l).  Workloads not
+# listed are chains.  GoogLeNet (5): conv_1 (5a/3x3, fed by 5a/3x3_reduce) and conv_2
+# (5a/5x5_reduce) are parallel branches of module 5a; the 5b reduce/1x1 branches read 5a's output;
+# conv_4 (5b/3x3) reads 5b/3x3_reduce.  Inception 5a+5b (6): per module, the branches that read
+# the module input (1x1, 3x3_reduce, 5x5_reduce, pool_proj after the max-pool), then the 3x3 and
+# 5x5 convolutions of the reduced maps.
+LEVELS: Dict[int, List[List[str]]] = {
+    5: [["googlenet_conv_1", "googlenet_conv_2"],
+        ["googlenet_conv_3", "googlenet_conv_5", "googlenet_conv_6"],
+        ["googlenet_conv_4"]],
+    6: [["i5a_1x1", "i5a_3x3_reduce", "i5a_5x5_reduce", "i5a_pool_proj"],
+        ["i5a_3x3", "i5a_5x5"],
+        ["i5b_1x1", "i5b_3x3_reduce", "i5b_5x5_reduce", "i5b_pool_proj"],
+        ["i5b_3x3", "i5b_5x5"]],
+}
+
 CONFIG_NAMES = {
     1: "lenet_conv1_b64",
     2: "lenet5_conv_stack_b64",

@@ -50,6 +50,10 @@ def parse_args():
                         "stream pool sized by Eq. 7) as a comparator; 1 GPU")
     p.add_argument("--pool-streams", type=int, default=0,
                    help="stream-pool size (0 = the Eq. 7 bound)")
+    p.add_argument("--exchange", choices=["nccl", "tree"], default="nccl",
+                   help="tree: deterministic gradient exchange (filter gradients per batch leaf, "
+                        "fixed binary tree over 8 leaves + recursive doubling; dW bitwise "
+                        "identical for 1/2/4/8 GPUs); nccl: one all_reduce(SUM)")
     p.add_argument("--chain", action="store_true",
                    help="treat the workload as a chain of layers even where the network runs "
                         "branches in parallel (default: independent layers of a level run on "
@@ -169,9 +173,23 @@ class LayerState:
         self.dw = grads.dw(idx)      # views into the flat dW||db buffer (one all_reduce per step)
         self.db = grads.db(idx)
         self.flops = float(self.layer.with_batch(n_local).flops_per_pass())
+        self.leaves = None
+
+    def use_leaves(self, leaf_grads, idx, math, dev):
+        """Deterministic exchange: the filter gradient per batch leaf of this rank (one plan for
+        the leaf batch), each into its leaf's flat buffer."""
+        glp = self.glp
+        k = len(leaf_grads)
+        nl = self.n // k
+        l = self.layer
+        self.leaf_conv = glp.ConvLayer(nl, l.C, l.H, l.W, l.Co, l.K, l.S, l.P, math=math,
+                                       device=dev.index, groups=l.groups)
+        self.leaves = [(self.t["x"][j * nl:(j + 1) * nl], self.t["dy"][j * nl:(j + 1) * nl],
+                        lg.dw(idx), lg.db(idx)) for j, lg in enumerate(leaf_grads)]
 
     def launches(self):
-        return 9 if self.dx is not None else 7
+        base = 9 if self.dx is not None else 7
+        return base if self.leaves is None else base - 4 + 6 * len(self.leaves)
 
     # the step's kernel groups (one C call each; see step())
     def pack_x(self, st=None):
@@ -193,10 +211,19 @@ class LayerState:
         self.conv.stage_bwd_data(self.dx, stream=st)
 
     def bwd_filter(self, st=None):
-        self.conv.stage_bwd_filter(stream=st)
+        if self.leaves is None:
+            self.conv.stage_bwd_filter(stream=st)
+            return
+        lc, glp = self.leaf_conv, self.glp
+        for x, dy, dw, db in self.leaves:
+            lc.stage_pack(glp.GLP_PACK_X, x, stream=st)
+            lc.stage_pack(glp.GLP_PACK_DY_DB, dy, stream=st)
+            lc.stage_bwd_filter(stream=st)
+            lc.stage_reduce(dw, db, stream=st)
 
     def reduce(self, st=None):
-        self.conv.stage_reduce(self.dw, self.db, stream=st)
+        if self.leaves is None:
+            self.conv.stage_reduce(self.dw, self.db, stream=st)
 
     def host_inputs(self):
         return self.host, self.t
@@ -371,6 +398,23 @@ def run_glp(args, ws, rank, local):
                                      idxs))
     stream = torch.cuda.current_stream()
 
+    tree = None
+    if args.exchange == "tree":
+        from paper_conf_icpp_futhys18_b200.dist import TreeAllreduce, rank_leaves
+        my_leaves = rank_leaves(rank, G)
+        if any(not isinstance(s, LayerState) for s in states) or n_local[0] % len(my_leaves):
+            raise SystemExit("--exchange tree: single layers and a leaf-divisible batch only")
+        leaf_grads = [FlatGrads([l.w_shape for l in layers], device=dev) for _ in my_leaves]
+        for i, s in enumerate(states):
+            s.use_leaves(leaf_grads, i, args.math, dev)
+        tree = TreeAllreduce()
+
+    def exchange():
+        if tree is not None:
+            flat.copy_(tree([lg.buf for lg in leaf_grads]))
+        elif G > 1:
+            grads.allreduce()
+
     # network DAG levels (units of one level are independent: concurrent streams, the GLP4NN idea
     # of concurrent kernels applied to a real step's independent layers); default: a chain
     lv = None if args.chain else LEVELS.get(args.workload)
@@ -433,8 +477,7 @@ def run_glp(args, ws, rank, local):
                 if ev is not None:
                     ev[i][5].record(stream)
                 s.reduce()
-            if G > 1:
-                grads.allreduce()
+            exchange()
             return
         fs = [stream] + fstreams[1:]
         side_w.wait_stream(stream)
@@ -489,8 +532,7 @@ def run_glp(args, ws, rank, local):
         stream.wait_stream(side_w)
         for g in gstreams:
             stream.wait_stream(g)
-        if G > 1:
-            grads.allreduce()
+        exchange()
 
     for _ in range(args.warmup):
         step()
@@ -623,7 +665,7 @@ def run_glp(args, ws, rank, local):
         "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
                    "global_batch": images_per_step, "per_gpu_batch": n_local[0],
                    "layers": [s.name for s in states], "math": args.math,
-                   "parallelism": f"dp{G}", "l2": "inputs larger than L2 (step working set "
+                   "parallelism": f"dp{G}", "exchange": args.exchange, "l2": "inputs larger than L2 (step working set "
                    f"{sum(v.numel() * 4 for s in states for v in s.t.values()) / 1e9:.2f} GB)",
                    "step_gflop": round(step_flops / 1e9, 1),
                    "samples_in_flight": [i.samples_in_flight for i in info0],

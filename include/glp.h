@@ -216,6 +216,17 @@ glp_status_t glp_stage_fwd_group(glp_plan_t plan, const float *const *b, float *
 glp_status_t glp_stage_reduce_group(glp_plan_t plan, float *const *dw, float *const *db,
                                     int accumulate, void *ws, size_t ws_bytes, glp_stream_t stream);
 
+/* ---- deterministic gradient exchange ----------------------------------- *
+ * "Convergence-invariant" (P264) extended across GPU counts: the global batch is cut into a
+ * fixed number of leaves (8); each leaf's dW||db is computed by the same plan (shape-only split
+ * order) whichever rank holds it, and the leaves are summed by a fixed binary tree — the rank's
+ * local subtree, then recursive doubling over ranks (paper_conf_icpp_futhys18_b200.dist.
+ * TreeAllreduce; the transfers are torch.distributed point-to-point, NCCL over NVLink).  Every
+ * tree node is this call: out = a + b elementwise in fp32 (a, b, out device pointers of n floats;
+ * out may alias a or b; asynchronous on `stream`).  Since a + b == b + a bitwise, dW is bitwise
+ * identical for 1, 2, 4 and 8 ranks. */
+glp_status_t glp_sum2(const float *a, const float *b, float *out, size_t n, glp_stream_t stream);
+
 /* ---- prior-art comparator: the paper's stream pool --------------------- *
  * GLP4NN's own scheme (P165-173, Figs 4/6): every layer pass runs as per-sample kernels (batch 1,
  * the sample's im2col+GEMM chain) dispatched round-robin (P171) over a pool of CUDA streams whose

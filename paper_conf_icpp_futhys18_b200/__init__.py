@@ -60,7 +60,7 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_stage_bwd_filter", "glp_stage_reduce", "glp_conv_group_desc_create",
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
            "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
-           "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups"]
+           "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups", "glp_sum2"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA = 0, 1, 2, 3, 4
 
@@ -121,6 +121,7 @@ def lib():
         L.glp_pool_conv_bwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_pool_destroy.argtypes = [_vp]
         L.glp_conv_desc_set_groups.argtypes = [_vp, _c_int]
+        L.glp_sum2.argtypes = [_vp, _vp, _vp, _c_size, _vp]
         _lib = L
     return _lib
 
@@ -178,6 +179,12 @@ def _stream(stream):
     import torch
     s = stream if stream is not None else torch.cuda.current_stream()
     return ctypes.c_void_p(s.cuda_stream)
+
+
+def sum2(a, b, out, stream=None):
+    """out = a + b (fp32 CUDA tensors of equal size): the deterministic tree's add (glp_sum2)."""
+    _ck(lib().glp_sum2(_ptr(a), _ptr(b), _ptr(out), a.numel(), _stream(stream)), "glp_sum2")
+    return out
 
 
 @dataclass

@@ -991,6 +991,16 @@ glp_status_t tc_bwd(glp_plan_s &P, const float *x, const BrIn &dy, const BrIn &w
   return run_wgrad_reduce(P, dw, with_db ? &db : nullptr, accumulate, ws, st);
 }
 
+// out = a + b elementwise (one IEEE fp32 add per element: commutative, so a tree of these is
+// bitwise independent of which rank holds which operand).
+__global__ void __launch_bounds__(256) sum2_kernel(const float *__restrict__ a,
+                                                   const float *__restrict__ b,
+                                                   float *__restrict__ out, size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n;
+       i += (size_t)gridDim.x * blockDim.x)
+    out[i] = a[i] + b[i];
+}
+
 // Stream-pool comparator: dst[i] (+)= sum over the pool's S per-stream accumulators, s = 0..S-1
 // in order (fixed, so the pool's result is deterministic for a given S).
 __global__ void __launch_bounds__(256) pool_sum_slots(const float *__restrict__ src, size_t stride,
@@ -1727,6 +1737,16 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   else
     debug_im2col_kernel<4><<<ew_grid(total), 256, 0, st>>>(p.g, n, P->d.C, P->d.Kh, P->d.Kw, P->d.Ho, P->d.Wo, col);
   GLP_LAUNCH_CHECK("debug_im2col_kernel");
+  return GLP_OK;
+}
+
+// ---- deterministic gradient exchange: the tree's add step ----
+glp_status_t glp_sum2(const float *a, const float *b, float *out, size_t n, glp_stream_t stream) {
+  if (n == 0) return GLP_OK;
+  if (!a || !b || !out) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  sum2_kernel<<<ew_grid(n), 256, 0, st>>>(a, b, out, n);
+  GLP_LAUNCH_CHECK("sum2_kernel");
   return GLP_OK;
 }
 

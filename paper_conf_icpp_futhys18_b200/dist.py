@@ -56,3 +56,88 @@ class FlatGrads:
         if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
             dist.all_reduce(self.buf, op=dist.ReduceOp.SUM, group=group)
         return self.buf
+
+
+# ------------------------------------------------------------ deterministic exchange (NEXT-2) ---
+
+LEAVES = 8   # fixed number of batch leaves: the tree (and so every dW bit) is the same for 1..8 ranks
+
+
+def leaf_range(n_global: int, leaf: int, leaves: int = LEAVES) -> Tuple[int, int]:
+    """Samples [start, stop) of batch leaf `leaf` (equal contiguous leaves; leaves | n_global)."""
+    if n_global % leaves or not 0 <= leaf < leaves:
+        raise ValueError("the global batch must split into equal leaves")
+    n = n_global // leaves
+    return leaf * n, (leaf + 1) * n
+
+
+def rank_leaves(rank: int, world: int, leaves: int = LEAVES) -> List[int]:
+    """The contiguous block of leaves rank `rank` computes (world must be a power of two <= leaves
+    dividing it, so a rank's block is one subtree of the fixed tree)."""
+    if world < 1 or leaves % world or world & (world - 1) or not 0 <= rank < world:
+        raise ValueError("world must be a power of two dividing the leaf count")
+    per = leaves // world
+    return list(range(rank * per, (rank + 1) * per))
+
+
+def tree_sum(parts, add):
+    """Fixed balanced binary tree over `parts` (a power-of-two count, in leaf order): level by
+    level, node = add(left, right).  Returns a new buffer (inputs are not modified)."""
+    level = list(parts)
+    if not level or len(level) & (len(level) - 1):
+        raise ValueError("need a power-of-two number of parts")
+    first = True
+    while len(level) > 1:
+        nxt = []
+        for i in range(0, len(level), 2):
+            a, b = level[i], level[i + 1]
+            out = a.clone() if first else a   # never write into the caller's leaf buffers
+            add(a, b, out)
+            nxt.append(out)
+        level = nxt
+        first = False
+    return level[0] if not first else level[0].clone()
+
+
+def _default_add(a, b, out):
+    if a.is_cuda:
+        from . import sum2
+        return sum2(a, b, out)
+    import torch
+    return torch.add(a, b, out=out)
+
+
+class TreeAllreduce:
+    """Deterministic all-reduce of per-leaf partial sums (include/glp.h "deterministic gradient
+    exchange"): each rank holds the partials of its leaves (rank_leaves), sums them with the local
+    subtree of a fixed binary tree over LEAVES leaves, then combines subtree sums by recursive
+    doubling (log2(world) exchanges with partner rank ^ d; the lower-ranked subtree is always the
+    left operand).  Every rank ends with the same bits, and the bits do not depend on the world
+    size: every fp32 add is a node of the same tree, and a + b == b + a.  `add(a, b, out)` is the
+    library's glp_sum2 on CUDA tensors (torch.add on CPU, for the gloo tests)."""
+
+    def __init__(self, group=None, add=None):
+        self.group = group
+        self.add = add or _default_add
+
+    def __call__(self, parts):
+        import torch.distributed as dist
+        acc = tree_sum(parts, self.add)
+        if not (dist.is_available() and dist.is_initialized()):
+            return acc
+        world = dist.get_world_size(self.group)
+        rank = dist.get_rank(self.group)
+        recv = acc.clone()
+        d = 1
+        while d < world:
+            partner = rank ^ d
+            ops = [dist.P2POp(dist.isend, acc, partner, self.group),
+                   dist.P2POp(dist.irecv, recv, partner, self.group)]
+            for r in dist.batch_isend_irecv(ops):
+                r.wait()
+            if rank < partner:
+                self.add(acc, recv, acc)
+            else:
+                self.add(recv, acc, acc)
+            d <<= 1
+        return acc

@@ -98,3 +98,60 @@ def test_gloo_allreduce_equals_full_batch():
         assert oracle.normwise_err(reduced[0][off:off + n].reshape(dw.shape), dw) < 1e-6
         assert oracle.normwise_err(reduced[0][off + n:off + n + Co], db) < 1e-6
         off += n + Co
+
+
+# ----------------------------------------------------------- deterministic tree exchange -----
+
+from paper_conf_icpp_futhys18_b200.dist import LEAVES, TreeAllreduce, leaf_range, rank_leaves, tree_sum  # noqa: E402
+
+
+def _leaf_parts(n=4099, seed=5):
+    # partial sums spanning many magnitudes, so a different summation order changes bits
+    r = np.random.default_rng(seed)
+    return [(r.standard_normal(n) * 10.0 ** r.uniform(-6, 6, n)).astype(np.float32)
+            for _ in range(LEAVES)]
+
+
+def _tree_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    parts = _leaf_parts()
+    mine = [torch.from_numpy(parts[j].copy()) for j in rank_leaves(rank, world)]
+    out = TreeAllreduce()(mine)
+    q.put((rank, out.numpy().copy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_tree_allreduce_bitwise_invariant_across_world_sizes(world):
+    """The tree all-reduce gives every rank the same bits, equal to the 1-process tree over all
+    leaves, for 2, 4 and 8 ranks (gloo); plain left-to-right summation gives different bits."""
+    ref = tree_sum([torch.from_numpy(p.copy()) for p in _leaf_parts()],
+                   lambda a, b, o: torch.add(a, b, out=o)).numpy()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_tree_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(world):
+        np.testing.assert_array_equal(res[r], ref)
+    seq = np.zeros_like(ref)
+    for p in _leaf_parts():
+        seq = (seq + p).astype(np.float32)
+    assert not np.array_equal(seq, ref)   # the order matters: the test can see a wrong tree
+    np.testing.assert_allclose(ref, np.sum(np.stack(_leaf_parts()).astype(np.float64), 0),
+                               rtol=1e-5, atol=1e-2)
+
+
+def test_leaf_partition():
+    assert [leaf_range(256, j) for j in (0, 7)] == [(0, 32), (224, 256)]
+    assert rank_leaves(1, 4) == [2, 3] and rank_leaves(0, 1) == list(range(8))
+    with pytest.raises(ValueError):
+        rank_leaves(0, 3)
+    with pytest.raises(ValueError):
+        leaf_range(100, 0)

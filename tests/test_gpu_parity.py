@@ -498,3 +498,39 @@ def test_grouped_conv(shape, math):
         torch.cuda.synchronize()
         for k, v in (("y", y), ("dx", dx), ("dw", dw), ("db", db)):
             np.testing.assert_array_equal(v.cpu().numpy(), got[k], err_msg="staged " + k)
+
+
+def test_tree_exchange_bitwise_invariant_emulated_ranks():
+    """Deterministic gradient exchange (NEXT-2) on the device: leaf filter gradients from the same
+    leaf plan, the rank-local subtrees and the cross-rank levels all summed by glp_sum2, give
+    bitwise the same dW and db for 1, 2, 4 and 8 (emulated) ranks; exact on integer data."""
+    from paper_conf_icpp_futhys18_b200.dist import LEAVES, leaf_range, rank_leaves, tree_sum
+    N, C, H, W, Co, K, S, P = 16, 24, 13, 13, 40, 3, 1, 1
+    Ho = oracle.out_dim(H, K, S, P)
+    add = lambda a, b, o: glp.sum2(a, b, o)
+    for exact, seed in ((False, 81), (True, 82)):
+        d = gen_custom(N, C, H, W, Co, K, K, seed, exact=exact, Ho=Ho, Wo=Ho)
+        t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+        leaf = glp.ConvLayer(N // LEAVES, C, H, W, Co, K, S, P, math="bf16")
+        parts = []
+        for j in range(LEAVES):
+            a, b = leaf_range(N, j)
+            buf = torch.empty(Co * C * K * K + Co, device=DEV)
+            leaf.bwd_filter(t["x"][a:b].contiguous(), t["dy"][a:b].contiguous(),
+                            buf[:Co * C * K * K].view(Co, C, K, K), buf[Co * C * K * K:])
+            parts.append(buf)
+        results = []
+        for world in (1, 2, 4, 8):
+            subtrees = [tree_sum([parts[j] for j in rank_leaves(r, world)], add) for r in range(world)]
+            results.append(tree_sum(subtrees, add) if world > 1 else subtrees[0])
+        torch.cuda.synchronize()
+        ref = results[0].cpu().numpy()
+        for r in results[1:]:
+            np.testing.assert_array_equal(r.cpu().numpy(), ref)
+        dw, _ = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, S, P)
+        db = d["dy"].astype(np.float64).sum(axis=(0, 2, 3))
+        full = np.concatenate([dw.ravel(), db])
+        if exact:
+            np.testing.assert_array_equal(ref, full.astype(np.float32))
+        else:
+            assert np.abs(ref - full).max() / np.abs(full).max() <= TOL["bf16"]

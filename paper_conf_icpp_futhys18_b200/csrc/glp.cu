@@ -341,6 +341,7 @@ struct glp_plan_s {
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
   // instead of after it.  GLP_SMEM_CAP (bytes) overrides (A/B runs).
   int smem_cap = 232448;
+  int pack_block = 0;  // GLP_PACK_BLOCK=1: the block-tiled activation pack (A/B runs)
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
@@ -691,10 +692,17 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
-  dim3 grid((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
   const int nt = (int)cdiv(P.d.Co, 32);
+  if (!P.pack_block) {   // warp-tiled pack (default)
+    dim3 gw((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, 8 * PACKW_ROWS));
+    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<2>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
+    else GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<4>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
+    GLP_LAUNCH_CHECK("pack_act_warp");
+    return GLP_OK;
+  }
+  dim3 grid((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
   if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
   else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
@@ -1230,6 +1238,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
+  if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
   // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
@@ -1309,7 +1318,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->sz_part = P->halo ? align1k((size_t)P->hw.splits * P->hw.mpad * P->hw.ld * 4)
                          : align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
-    P->db_rows = (int)cdiv((long long)c.N * dy_hw, PACK_PT);
+    P->db_rows = (int)cdiv((long long)c.N * dy_hw, P->pack_block ? PACK_PT : PACKW_ROWS);
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;

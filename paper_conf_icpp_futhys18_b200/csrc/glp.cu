@@ -745,6 +745,12 @@ glp_status_t run_pack_w_fwd_one(glp_plan_s &P, const float *w, int co_off, int C
       GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<2>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad));
     else
       GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<4>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad));
+  } else if ((size_t)d.C * P.taps * 4 <= 48 * 1024) {
+    const size_t sm = (size_t)d.C * P.taps * 4;
+    if (P.elem == 2)
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<2>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad));
+    else
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<4>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad));
   } else if (P.elem == 2) {
     GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<2>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad));
   } else {
@@ -796,7 +802,13 @@ glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStr
     const int off = n > 1 ? d.br_off[b] : 0;
     const int co = n > 1 ? d.br_off[b + 1] - off : d.Co;
     const int hi = (b == n - 1) ? P.Cop : off + co;
-    if (P.elem == 2)
+    const size_t sm = (size_t)co * P.taps * 4;
+    if (sm <= 48 * 1024) {
+      if (P.elem == 2)
+        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<2>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+      else
+        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<4>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+    } else if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
     else
       GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));

@@ -414,4 +414,52 @@ __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w,
   PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
 }
 
+// Row-staged weight packs (default when a staged row fits 48 KB of shared memory).  The element-
+// per-thread kernels above read W with a stride of `taps` floats between neighbouring threads (one
+// 32-byte sector per 4-byte load); here one block owns one destination row, reads its source
+// elements once with coalesced loads into shared memory and writes the row with consecutive
+// threads on consecutive destination elements (odd taps: conflict-free strided smem reads).
+// Forward: block co stages W[co][0..C*taps) and writes Wp[co][t*Cp + c].
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_w_fwd_rows(const float *__restrict__ w, void *__restrict__ out,
+                                                       int C, int taps, int Cp, int Kpad) {
+  extern __shared__ float srow[];
+  pdl_launch_dependents();
+  pdl_wait();
+  const int co = blockIdx.x, n = C * taps;
+  const float *src = w + (size_t)co * n;
+  for (int i = threadIdx.x; i < n; i += 256) srow[i] = __ldg(src + i);
+  __syncthreads();
+  for (int k = threadIdx.x; k < Kpad; k += 256) {
+    const int t = k / Cp, c = k - t * Cp;
+    const float v = (t < taps && c < C) ? srow[c * taps + t] : 0.f;
+    PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v);
+  }
+}
+
+// Backward-data: block ci stages W[cb][ci][0..taps) for every cb < Co (runs of `taps` contiguous
+// floats) and writes Wt[ci][t*Cop + co] over [co_lo, co_hi) (+ the zero tail past the taps), with
+// the same flip / branch semantics as pack_w_dgrad.
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_w_dgrad_rows(const float *__restrict__ w, void *__restrict__ out,
+                                                         int Co, int C, int taps, int Cop, int Kpad,
+                                                         int flip, int co_off, int co_lo, int co_hi) {
+  extern __shared__ float srow[];   // [Co][taps]
+  pdl_launch_dependents();
+  pdl_wait();
+  const int ci = blockIdx.x, n = Co * taps;
+  for (int i = threadIdx.x; i < n; i += 256) {
+    const int cb = i / taps, t = i - cb * taps;
+    srow[i] = __ldg(w + ((size_t)cb * C + ci) * taps + t);
+  }
+  __syncthreads();
+  for (int k = threadIdx.x; k < Kpad; k += 256) {
+    const int t = k / Cop, co = k - t * Cop;
+    if (t < taps && (co < co_lo || co >= co_hi)) continue;   // another branch's channels
+    const int cb = co - co_off;
+    const float v = (t < taps && cb < Co) ? srow[cb * taps + (flip ? taps - 1 - t : t)] : 0.f;
+    PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
+  }
+}
+
 }  // namespace glp

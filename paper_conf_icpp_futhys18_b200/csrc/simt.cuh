@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
 // those, lanes = channels, coalesced), reduces its 8 warps in a fixed tree, and stores part2[g][co];
 // the last block to finish for a channel group (atomic ticket) sums part2[0..G) in index order.
 // The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
-constexpr int DB_GROUPS = 64;
+constexpr int DB_GROUPS = 128;   // multiple of 4
 __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
                                                  const BrOut db, int Co, int rows,
                                                  int accumulate, float *__restrict__ part2,
@@ -293,9 +293,26 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
   pdl_wait();
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
   const int co = blockIdx.x * 32 + lane, g = blockIdx.y;
+  // rows g + DB_GROUPS*(ty + 8*j), j = 0, 1, ...: four interleaved accumulators (j mod 4) keep
+  // four loads in flight (one dependent chain was latency-bound: ~47 L2 round trips for CaffeNet
+  // conv1), the tail goes to a0, then ((a0+a1)+(a2+a3)) — an order fixed by `rows` alone
   float a = 0.f;
-  if (co < Co)
-    for (int r = g + DB_GROUPS * ty; r < rows; r += DB_GROUPS * 8) a += __ldg(part + (size_t)r * Co + co);
+  if (co < Co) {
+    constexpr int STEP = DB_GROUPS * 8;
+    float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+    int r = g + DB_GROUPS * ty;
+    const float *pc = part + co;
+    for (; r + 3 * STEP < rows; r += 4 * STEP) {
+      const float v0 = __ldg(pc + (size_t)r * Co), v1 = __ldg(pc + (size_t)(r + STEP) * Co);
+      const float v2 = __ldg(pc + (size_t)(r + 2 * STEP) * Co), v3 = __ldg(pc + (size_t)(r + 3 * STEP) * Co);
+      a0 += v0;
+      a1 += v1;
+      a2 += v2;
+      a3 += v3;
+    }
+    for (; r < rows; r += STEP) a0 += __ldg(pc + (size_t)r * Co);
+    a = (a0 + a1) + (a2 + a3);
+  }
   red[ty][lane] = a;
   __syncthreads();
   if (ty == 0) {
@@ -310,8 +327,16 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
   if (last && ty == 0) {
     __threadfence();
     if (co < Co) {
-      float s = 0.f;
-      for (int k = 0; k < DB_GROUPS; ++k) s += __ldcg(part2 + (size_t)k * Co + co);
+      // group sums in index order, four strided accumulators (k mod 4), then combined in order
+      float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+#pragma unroll 4
+      for (int k = 0; k < DB_GROUPS; k += 4) {
+        s0 += __ldcg(part2 + (size_t)k * Co + co);
+        s1 += __ldcg(part2 + (size_t)(k + 1) * Co + co);
+        s2 += __ldcg(part2 + (size_t)(k + 2) * Co + co);
+        s3 += __ldcg(part2 + (size_t)(k + 3) * Co + co);
+      }
+      const float s = (s0 + s1) + (s2 + s3);
       float *d = db.at(co, 0, 1, 0);
       *d = accumulate ? *d + s : s;
     }

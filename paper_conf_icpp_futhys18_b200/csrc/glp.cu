@@ -342,6 +342,7 @@ struct glp_plan_s {
   // instead of after it.  GLP_SMEM_CAP (bytes) overrides (A/B runs).
   int smem_cap = 232448;
   int pack_block = 0;  // GLP_PACK_BLOCK=1: the block-tiled activation pack (A/B runs)
+  int s2d_block = 0;   // GLP_S2D_BLOCK=1: the block-persistent space-to-depth pack (A/B runs)
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
   int dbg_skip = 0;    // GLP_DEBUG_SKIP (diagnostics: skip A/B loads or MMAs; wrong results)
 };
@@ -773,6 +774,16 @@ glp_status_t run_pack_w_fwd(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStrea
 // x -> the packed operand of the forward / filter-gradient passes (direct NHWC or space-to-depth).
 glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
+  if (P.s2d && P.s2d * P.s2d * d.C <= S2DW_MAXC && P.Cpx <= S2DW_MAXC && !P.s2d_block) {
+    const long long px = (long long)d.N * P.dxg.H * P.dxg.W;
+    const dim3 grid((unsigned)cdiv(px, 128));
+    if (P.elem == 2)
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<2>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+    else
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<4>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+    GLP_LAUNCH_CHECK("pack_s2d_warp");
+    return GLP_OK;
+  }
   if (P.s2d) {
     const int S = P.s2d;
     const size_t smem = (size_t)S * d.C * d.W * sizeof(float);
@@ -1251,6 +1262,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
+  if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
   // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));

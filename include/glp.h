@@ -76,6 +76,8 @@ typedef struct {
   int math;
   int wgrad_halo;        /* 1: filter gradient by the shared-halo kernel (space-to-depth layers;
                             dy packed on the padded grid), 0: im2col implicit GEMM             */
+  int fwd_halo;          /* 1: forward by the shared-halo kernel (space-to-depth layers: x' staged
+                            once per tile for all taps, outputs on the padded grid), 0: im2col   */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

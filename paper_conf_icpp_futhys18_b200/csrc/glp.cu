@@ -23,6 +23,7 @@
 #include "../../include/glp.h"
 #include "common.cuh"
 #include "hwgrad.cuh"
+#include "hfwd.cuh"
 #include "igemm.cuh"
 #include "pack.cuh"
 #include "simt.cuh"
@@ -320,6 +321,11 @@ struct glp_plan_s {
   int halo = 0;
   HwgradParams hw{};
   int hw_grid = 0, hw_smem = 0, hw_regs = 0;
+  // halo forward (hfwd.cuh) for the same space-to-depth layers: x' staged once per tile for all
+  // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
+  int hfwd = 0;
+  HfwdParams hf{};
+  int hf_grid = 0, hf_smem = 0, hf_regs = 0;
   int S = 1;
   // SIMT path
   int simt_splits = 1, simt_chunk = 1;
@@ -336,6 +342,7 @@ struct glp_plan_s {
   int pdl = 0;         // GLP_PDL=1: programmatic dependent launch (measured 3% slower in the graph)
   int bn_model = 1;    // GLP_BN_MODEL=0: always the default fwd/dgrad tile (A/B runs)
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
+  int allow_hfwd = 1;  // GLP_HFWD=0: im2col forward for space-to-depth layers (A/B runs)
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -405,6 +412,59 @@ glp_status_t plan_halo(glp_plan_s &P) {
   GLP_CUDA(cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(hwgrad_kernel)));
   P.hw_regs = fa.numRegs;
   P.halo = 1;
+  return GLP_OK;
+}
+
+// Halo forward (hfwd.cuh) for space-to-depth layers whose x' rows are one 64-channel bf16 atom,
+// whose taps x C_o weight block fits shared memory next to >= 2 halo stages, and that are not a
+// fused sibling group.  Tiles of 128 rows over the flattened padded grid; no K split, so the
+// output never depends on the grid (convergence invariance, P264).
+glp_status_t plan_hfwd(glp_plan_s &P) {
+  P.hfwd = 0;
+  const glp_conv_desc_s &x = P.dxg;
+  if (!P.allow_hfwd || !P.s2d || P.elem != 2 || P.Cpx != 64 || P.d.nbr > 1) return GLP_OK;
+  const int Ks = x.Kh, T = P.tapsx;
+  if (T > HF_MAXTAPS || P.fwd.Kpad < T * 64) return GLP_OK;
+  const int bn = (int)rup(x.Co, 16);
+  const int shift_max = (Ks - 1) * x.W + (Ks - 1);
+  const int halo_rows = 128 + shift_max;
+  if (bn > 256 || halo_rows > 256) return GLP_OK;
+  HfwdParams &h = P.hf;
+  memset(&h, 0, sizeof(h));
+  h.taps = T;
+  for (int t = 0; t < T; ++t) h.shift[t] = (t / Ks) * x.W + t % Ks;
+  h.bn = bn;
+  h.co = x.Co;
+  h.acc_cols = (int)rup(bn, 32);
+  int tc = 32;
+  while (tc < 2 * h.acc_cols) tc *= 2;
+  h.tmem_cols = tc;
+  h.halo_rows = halo_rows;
+  h.a_bytes = (int)rup((long long)halo_rows * 128, 1024);
+  h.b_tap_bytes = (int)rup((long long)bn * 128, 1024);
+  h.bias_floats = (int)rup(bn, 4);
+  const int fixed = 1024 + T * h.b_tap_bytes + 16 + 16 + 4 * h.bias_floats + 8 * 8;
+  h.stages = std::min(6, (P.smem_cap - fixed - 8 * 2 * 6) / h.a_bytes);
+  if (h.stages < 2) return GLP_OK;
+  const long long rows = (long long)x.N * x.H * x.W;
+  if (rows >= (1LL << 31) - 256) return GLP_OK;
+  h.rows = (int)rows;
+  h.tiles = (int)cdiv(rows, 128);
+  h.div_img = FastDiv((uint32_t)(x.H * x.W));
+  h.div_w = FastDiv((uint32_t)x.W);
+  h.ho = P.d.Ho;
+  h.wo = P.d.Wo;
+  P.hf_smem = fixed + 8 * (2 * h.stages + 6) + h.stages * h.a_bytes;
+  long long grid = std::min<long long>(h.tiles, P.sm_count);
+  if (P.s_override > 0)   // test override: only the tiles of S samples in flight at once
+    grid = std::max(1LL, std::min(grid, cdiv((long long)P.s_override * x.H * x.W, 128)));
+  P.hf_grid = (int)grid;
+  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hfwd_kernel),
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  cudaFuncAttributes fa;
+  GLP_CUDA(cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(hfwd_kernel)));
+  P.hf_regs = fa.numRegs;
+  P.hfwd = 1;
   return GLP_OK;
 }
 
@@ -866,8 +926,45 @@ glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, CUtensorMap &a
   return GLP_OK;
 }
 
+glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
+                          cudaStream_t st) {
+  const glp_conv_desc_s &d = P.dxg;
+  const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x'
+  CUtensorMap mapX, mapW;
+  glp_status_t s = cached_maps(P, 0, ws, mapX, mapW, [&](CUtensorMap &X, CUtensorMap &Wm) {
+    glp_status_t r = encode_2d(&X, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
+                               64u, (uint32_t)P.hf.halo_rows, CU_TENSOR_MAP_SWIZZLE_128B);
+    if (r) return r;
+    return encode_2d(&Wm, 2, ws + P.off_wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co,
+                     (uint64_t)P.fwd.Kpad * 2, 64u, (uint32_t)P.hf.bn, CU_TENSOR_MAP_SWIZZLE_128B);
+  });
+  if (s) return s;
+  HfwdParams p = P.hf;
+  p.out = y.p[0];
+  p.bias = b.p[0];
+  p.out_c = P.y_img_c;
+  p.out_hw = P.d.Ho * P.d.Wo;
+  p.dbg_skip = P.dbg_skip;
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3((unsigned)P.hf_grid);
+  cfg.blockDim = dim3(HF_THREADS);
+  cfg.dynamicSmemBytes = (size_t)P.hf_smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = P.pdl ? 1 : 0;
+  void *args[] = {&p, &mapX, &mapW};
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hfwd_kernel), args));
+  GLP_LAUNCH_CHECK("hfwd_kernel");
+  return GLP_OK;
+}
+
 glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
                           cudaStream_t st) {
+  if (P.hfwd) return run_fwd_halo(P, b, y, ws, st);
   const glp_conv_desc_s &d = P.dxg;
   const PassPlan &pp = P.fwd;
   void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
@@ -1261,6 +1358,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
+  if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
@@ -1326,7 +1424,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
       if (cur != device) cudaSetDevice(cur);
       return s;
     }
-    if ((s = plan_halo(*P))) {
+    if ((s = plan_halo(*P)) || (s = plan_hfwd(*P))) {
       delete P;
       if (cur != device) cudaSetDevice(cur);
       return s;
@@ -1407,6 +1505,13 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->plan_us = P->plan_us;
   I->math = P->math;
   I->wgrad_halo = P->halo;
+  I->fwd_halo = P->hfwd;
+  if (P->hfwd) {
+    I->grid_fwd = P->hf_grid;
+    I->tile_n_fwd = P->hf.bn;
+    I->stages_fwd = P->hf.stages;
+    I->tiles_fwd = P->hf.tiles;
+  }
   return GLP_OK;
 }
 

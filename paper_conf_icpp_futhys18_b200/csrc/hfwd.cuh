@@ -1,0 +1,221 @@
+// hfwd.cuh — forward pass of a unit-stride space-to-depth layer with a shared halo tile.
+//
+// y[n][co][h][w] = b[co] + sum_{t=(kh,kw)} sum_c x'[n][h+kh][w+kw][c] * W'[co][t][c]   (PAPER.md
+// Alg. 1 P82-99, "im2col -> GEMM + bias"; north_star (3)), where x' is the packed space-to-depth
+// input (an H' x W' image of one 64-channel bf16 atom per pixel, zero padded) and
+// the output pixel (h, w) lives at row q = (n*H' + h)*W' + w of the flattened padded grid, so the
+// A operand of tap t is the x' rows [q0 + s_t, q0 + s_t + 128) with s_t = kh*W' + kw.
+//
+// Why: the im2col forward re-reads x' from L2 once per tap (9x for CaffeNet conv1) on top of a
+// 297 MB fp32 output; L2 traffic, not the tensor pipe, bounded it (~110 us; 77 us with the output
+// stores skipped).  Here one TMA per tile stages the x' rows [q0, q0 + 128 + s_max) once; every
+// tap's A operand is that smem tile read through a descriptor whose start is shifted by s_t rows
+// (tcgen05 swizzles on absolute smem address bits, so any row shift is a valid SWIZZLE_128B
+// K-major operand: tools/shift_probe.cu), and the whole B operand (W', <= 120 KB) is loaded once
+// per CTA and stays resident.  L2 reads per tile: ~31 KB instead of ~200 KB.  Rows of the padded
+// grid outside H_o x W_o are computed and dropped (CaffeNet conv1: 57^2 / 55^2 = 7 % extra MMA).
+//
+// Persistent: tile t -> CTA t mod grid (the paper's round-robin dispatch, P171).  CTA = 192
+// threads: warps 0-3 epilogue (TMEM -> bias -> NCHW fp32), warp 4 TMA producer, warp 5 TMEM
+// owner + MMA issuer; two TMEM accumulators so the epilogue of tile i overlaps tile i+1.
+#pragma once
+#include "common.cuh"
+#include "ptx.cuh"
+
+namespace glp {
+
+constexpr int HF_THREADS = 192;
+constexpr int HF_MAXTAPS = 16;
+
+struct HfwdParams {
+  int taps;
+  int shift[HF_MAXTAPS];   // row shift s_t = kh*W' + kw of tap t (t = kh*Ks + kw)
+  int bn;                  // N = C_o rounded up to 16 (<= 256): one tile covers every channel
+  int co;                  // valid output channels
+  int acc_cols;            // TMEM columns per accumulator
+  int tmem_cols;           // allocation (power of two >= 2 * acc_cols)
+  int halo_rows;           // 128 + max shift
+  int a_bytes;             // one halo stage (1024-aligned)
+  int b_tap_bytes;         // one tap's B block: bn rows x 128 B (1024-aligned)
+  int stages;
+  int tiles;               // ceil(rows / 128)
+  int rows;                // N * H' * W'
+  FastDiv div_img, div_w;  // H' * W', W'
+  int ho, wo;              // valid output region of each H' x W' image
+  float *out;              // y NCHW fp32
+  int out_c;               // channels per image of y (all groups' channels)
+  int out_hw;              // H_o * W_o
+  const float *bias;       // may be null
+  int bias_floats;         // >= bn, multiple of 4
+  int dbg_skip;            // diagnostics (GLP_DEBUG_SKIP): bit0 skip x' loads, bit2 MMAs, bit3 stores
+};
+
+__global__ void __launch_bounds__(HF_THREADS, 1)
+    hfwd_kernel(const __grid_constant__ HfwdParams p, const __grid_constant__ CUtensorMap tmapX,
+                const __grid_constant__ CUtensorMap tmapW) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023u) & ~1023u;
+  const uint32_t sB = base;                                        // taps x [bn rows x 128 B]
+  const uint32_t sA0 = sB + (uint32_t)(p.taps * p.b_tap_bytes);    // stages x halo tiles
+  const uint32_t bars = sA0 + (uint32_t)(p.stages * p.a_bytes);
+  const int S_ = p.stages;
+  auto full = [&](int s) { return bars + 8u * s; };
+  auto empty = [&](int s) { return bars + 8u * (S_ + s); };
+  auto tfull = [&](int a) { return bars + 8u * (2 * S_ + a); };
+  auto tempty = [&](int a) { return bars + 8u * (2 * S_ + 2 + a); };
+  const uint32_t bfull = bars + 8u * (2 * S_ + 4);
+  const uint32_t tmem_slot = bars + 8u * (2 * S_ + 5);
+  const uint32_t sbias = (tmem_slot + 16u + 15u) & ~15u;
+  volatile uint32_t *tmem_slot_ptr =
+      reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+  const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0);
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S_; ++s) {
+      mbar_init(full(s), 1);
+      mbar_init(empty(s), 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(tfull(a), 1);
+      mbar_init(tempty(a), 4);
+    }
+    mbar_init(bfull, 1);
+    fence_mbar_init();
+  }
+  if (warp == 5) {
+    tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
+    tmem_relinquish();
+  }
+  if (warp == 4 && lane == 0) {
+    tma_prefetch(&tmapX);
+    tma_prefetch(&tmapW);
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  pdl_wait();
+  const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);
+
+  if (warp == 4) {
+    // ===================================== producer ========================================
+    // B once: tap t's K slice [t*64, t*64 + 64) of W' (bn rows, rows >= C_o zero-filled)
+    mbar_arrive_expect_tx_e(bfull, (uint32_t)(p.taps * p.bn * 128));
+    for (int t = 0; t < p.taps; ++t)
+      tma_load_2d_e(sB + (uint32_t)(t * p.b_tap_bytes), &tmapW, bfull, t * 64, 0);
+    const bool la = !(p.dbg_skip & 1);
+    const uint32_t tx = la ? (uint32_t)(p.halo_rows * 128) : 0u;
+    int rs = 0;
+    uint32_t rph = 0;
+    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
+      mbar_wait(empty(rs), rph ^ 1u);
+      const uint32_t sA = sA0 + (uint32_t)(rs * p.a_bytes);
+      mbar_arrive_expect_tx_e(full(rs), tx);
+      if (la) tma_load_2d_e(sA, &tmapX, full(rs), 0, tile * 128);   // rows past the end: zeros
+      if (++rs == S_) {
+        rs = 0;
+        rph ^= 1u;
+      }
+    }
+  } else if (warp == 5) {
+    // ===================================== MMA issuer ======================================
+    const uint32_t idesc = make_idesc(1u, 0u, 0u, 128u, (uint32_t)p.bn);
+    mbar_wait(bfull, 0);
+    int rs = 0;
+    uint32_t rph = 0, it = 0;
+    const bool skip_mma = (p.dbg_skip & 4) != 0;
+    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x, ++it) {
+      const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
+      mbar_wait(tempty(a), aph ^ 1u);
+      tc_fence_after();
+      mbar_wait(full(rs), rph);
+      tc_fence_after();
+      const uint32_t sA = sA0 + (uint32_t)(rs * p.a_bytes);
+      const uint32_t d = tmem_base + a * (uint32_t)p.acc_cols;
+      for (int t = 0; t < p.taps; ++t) {
+        if (skip_mma && t > 0) break;
+        // K-major SW128 operands: 8-row groups of 128-byte rows (SBO 1024); 4 MMAs of K = 16
+        // advance the start by 32 bytes (2 descriptor units)
+        const uint64_t da = make_sdesc(sA + (uint32_t)p.shift[t] * 128u, 16u, 1024u, 2u);
+        const uint64_t db = make_sdesc(sB + (uint32_t)(t * p.b_tap_bytes), 16u, 1024u, 2u);
+        mma_kblock_e<0, 1, 4, 2>(d, da, db, idesc, t > 0 ? 1u : 0u);
+      }
+      mma_commit_e<1>(empty(rs));
+      mma_commit_e<1>(tfull(a));
+      if (++rs == S_) {
+        rs = 0;
+        rph ^= 1u;
+      }
+    }
+    __syncwarp();
+  } else {
+    // ===================================== epilogue ========================================
+    const int row = warp * 32 + lane;
+    for (int i = row; i < p.bias_floats; i += 128)
+      sts_f32(sbias + 4u * (uint32_t)i, (p.bias != nullptr && i < p.co) ? __ldg(p.bias + i) : 0.f);
+    named_bar_sync(1, 128);
+    const size_t plane = (size_t)p.out_hw;
+    uint32_t it = 0;
+    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x, ++it) {
+      const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
+      mbar_wait(tfull(a), aph);
+      tc_fence_after();
+      const int q = tile * 128 + row;
+      uint32_t n = 0, rem = 0, h = 0, w = 0;
+      p.div_img.divmod((uint32_t)min(q, p.rows - 1), n, rem);
+      p.div_w.divmod(rem, h, w);
+      const bool mv = q < p.rows && (int)h < p.ho && (int)w < p.wo && !(p.dbg_skip & 8);
+      float *ob = p.out + (size_t)n * p.out_c * plane + (size_t)h * p.wo + w;
+      const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
+      auto store_chunk = [&](int c0, uint32_t (&v)[32]) {
+        if (!mv) return;
+        const int lim = min(32, p.co - c0);
+        float *o = ob + (size_t)c0 * plane;
+        if (lim == 32) {
+#pragma unroll
+          for (int k = 0; k < 32; k += 4) {
+            const float4 b4 = lds_f32x4(sbias + 4u * (uint32_t)(c0 + k));
+            o[0] = __uint_as_float(v[k]) + b4.x;
+            o += plane;
+            o[0] = __uint_as_float(v[k + 1]) + b4.y;
+            o += plane;
+            o[0] = __uint_as_float(v[k + 2]) + b4.z;
+            o += plane;
+            o[0] = __uint_as_float(v[k + 3]) + b4.w;
+            o += plane;
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < 32; ++k)
+            if (k < lim) o[(size_t)k * plane] = __uint_as_float(v[k]) + lds_f32(sbias + 4u * (uint32_t)(c0 + k));
+        }
+      };
+      // software-pipelined TMEM drain (next chunk's load in flight while this one is stored)
+      uint32_t va[32], vb[32];
+      tmem_ld32(taddr, va);
+      tmem_wait_ld_dep(va);
+      for (int c0 = 0; c0 < p.bn; c0 += 64) {
+        const bool hb = c0 + 32 < p.bn;
+        if (hb) tmem_ld32(taddr + (uint32_t)(c0 + 32), vb);
+        store_chunk(c0, va);
+        if (hb) {
+          tmem_wait_ld_dep(vb);
+          const bool ha = c0 + 64 < p.bn;
+          if (ha) tmem_ld32(taddr + (uint32_t)(c0 + 64), va);
+          store_chunk(c0 + 32, vb);
+          if (ha) tmem_wait_ld_dep(va);
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_relaxed(tempty(a));
+    }
+  }
+  pdl_launch_dependents();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 5) tmem_dealloc(tmem_base, (uint32_t)p.tmem_cols);
+}
+
+}  // namespace glp

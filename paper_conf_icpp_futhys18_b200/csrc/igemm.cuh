@@ -566,12 +566,8 @@ __global__ void __launch_bounds__(288, 1)
         const size_t plane = (size_t)p.out_hw;
         float *ob = outp + (size_t)n0 * plane;
         const uint32_t sb_tile = sbias + 4u * (uint32_t)n0;
-        for (int c0 = 0; c0 < p.bn; c0 += 32) {
-          uint32_t v[32];
-          long long c1 = clk ? clock64() : 0;
-          tmem_ld32(taddr + (uint32_t)c0, v);
-          tmem_wait_ld();
-          if (clk) e_ld += clock64() - c1;
+        // one 32-column chunk: bias add + 32 coalesced 128-byte stores (one per channel)
+        auto store_chunk = [&](int c0, uint32_t (&v)[32]) {
           const int lim = min(32, min(p.bn - c0, p.N - n0 - c0));
           float *o = ob + (size_t)c0 * plane;
           bool split_chunk = false;   // fused group: the chunk straddles two branch tensors
@@ -609,6 +605,26 @@ __global__ void __launch_bounds__(288, 1)
               const float b = (MODE == MODE_FWD) ? lds_f32(sb_tile + 4u * (uint32_t)(c0 + q)) : 0.f;
               if (q < lim) o[(size_t)q * plane] = __uint_as_float(v[q]) + b;
             }
+          }
+        };
+        // software-pipelined TMEM drain: the next chunk's tcgen05.ld is in flight while the
+        // current chunk is stored (the load latency was exposed once per chunk: ncu long-scoreboard
+        // stalls on the first use of every chunk)
+        uint32_t va[32], vb[32];
+        long long c1 = clk ? clock64() : 0;
+        tmem_ld32(taddr, va);
+        tmem_wait_ld_dep(va);
+        if (clk) e_ld += clock64() - c1;
+        for (int c0 = 0; c0 < p.bn; c0 += 64) {
+          const bool hb = c0 + 32 < p.bn;
+          if (hb) tmem_ld32(taddr + (uint32_t)(c0 + 32), vb);
+          store_chunk(c0, va);
+          if (hb) {
+            tmem_wait_ld_dep(vb);
+            const bool ha = c0 + 64 < p.bn;
+            if (ha) tmem_ld32(taddr + (uint32_t)(c0 + 64), va);
+            store_chunk(c0 + 32, vb);
+            if (ha) tmem_wait_ld_dep(va);
           }
         }
       } else {

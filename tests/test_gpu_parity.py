@@ -306,6 +306,42 @@ def test_halo_wgrad_random_and_invariant(shape):
             np.testing.assert_array_equal(other[k], runs[0][k], err_msg=k)
 
 
+@pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
+def test_halo_fwd_exact(shape, monkeypatch):
+    """The shared-halo forward (hfwd.cuh: one staged x' tile per 128 rows of the padded grid,
+    row-shifted K-major SWIZZLE_128B descriptors per tap, resident W', invalid padded-grid rows
+    dropped) is bit-exact on integer data, and GLP_HFWD=0 (im2col forward) agrees bit for bit."""
+    d = _data(shape, exact=True, seed=47)
+    ref = _oracle(d, shape[7], shape[8])
+    layer = _layer(shape, "bf16")
+    assert layer.info.fwd_halo == 1
+    got = _run(layer, d)
+    np.testing.assert_array_equal(got["y"], ref["y"].astype(np.float32))
+    monkeypatch.setenv("GLP_HFWD", "0")
+    layer0 = _layer(shape, "bf16")
+    assert layer0.info.fwd_halo == 0
+    got0 = _run(layer0, d)
+    np.testing.assert_array_equal(got0["y"], got["y"])
+
+
+@pytest.mark.parametrize("shape", HALO_SHAPES[:3], ids=lambda s: s[0])
+def test_halo_fwd_random_and_invariant(shape, monkeypatch):
+    """Random data: y within the bf16 bar of the oracle and 1e-4 of the rounding-emulated oracle,
+    bitwise identical across samples-in-flight overrides (grid sizes) and reruns, and equal to
+    the im2col forward (same MMA order: taps in order, 4 K=16 steps per 64-channel atom)."""
+    d = _data(shape, seed=48)
+    ref = _oracle(d, shape[7], shape[8])["y"]
+    emu = _oracle(d, shape[7], shape[8], x=EMU["bf16"](d["x"]), w=EMU["bf16"](d["w"]),
+                  dy=EMU["bf16"](d["dy"]))["y"]
+    runs = [_run(_layer(shape, "bf16", S), d)["y"] for S in (0, 1, 2, 0)]
+    assert np.abs(runs[0] - ref).max() / np.abs(ref).max() <= TOL["bf16"]
+    assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= 1e-4
+    for other in runs[1:]:
+        np.testing.assert_array_equal(other, runs[0])
+    monkeypatch.setenv("GLP_HFWD", "0")
+    np.testing.assert_array_equal(_run(_layer(shape, "bf16"), d)["y"], runs[0])
+
+
 # fused sibling groups (include/glp.h; SURVEY §8(f) NEXT-1): name, N, C, H, W, branches, K, S, P
 GROUPS = [
     ("gnet_5b_1x1_siblings", 4, 832, 7, 7, [384, 192, 48], 1, 1, 0),

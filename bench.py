@@ -69,6 +69,12 @@ def parse_args():
     p.add_argument("--no-graph", action="store_true",
                    help="launch every step eagerly (default on 1 GPU: the step is captured once "
                         "into a CUDA graph and replayed)")
+    p.add_argument("--exact-data", action="store_true",
+                   help="(tests) integer-valued inputs (glp_workloads exact variant) instead of "
+                        "the float recipe: every output is exact, so parity is bit for bit")
+    p.add_argument("--dump", default=None,
+                   help="(tests) after the timed steps, save every unit's inputs and outputs "
+                        "(.npy) and a meta.json to this directory for full-size sampled parity")
     return p.parse_args()
 
 
@@ -272,6 +278,58 @@ class LayerState:
         return self.host, self.t
 
 
+def set_exact_data(states):
+    """--exact-data: every unit's inputs replaced by the integer variant of its seeded draws."""
+    import torch
+    for s in states:
+        if isinstance(s, GroupState):
+            ds = [gen_layer(m, exact=True, batch=s.n) for m in s.members]
+            new = {"x": ds[0]["x"]}
+            for i, d in enumerate(ds):
+                for k in ("w", "b", "dy"):
+                    new[f"{k}{i}"] = d[k]
+        else:
+            new = gen_layer(s.layer, exact=True, batch=s.n)
+        for k, v in new.items():
+            s.host[k] = torch.from_numpy(v)
+            s.t[k].copy_(s.host[k])
+
+
+def dump_units(states, path, workload, math):
+    """--dump: the inputs and outputs of every unit after the timed steps (the launch
+    configuration the bench measured) for tests/test_gpu_fullsize.py."""
+    import numpy as np
+    import torch
+    torch.cuda.synchronize()
+    os.makedirs(path, exist_ok=True)
+    meta = {"workload": workload, "math": math, "units": []}
+    for i, s in enumerate(states):
+        grp = isinstance(s, GroupState)
+        l = s.layer
+        u = {"kind": "group" if grp else "layer",
+             "names": [m.name for m in s.members] if grp else [l.name],
+             "N": s.n, "C": l.C, "H": l.H, "W": l.W, "K": l.K, "S": l.S, "P": l.P,
+             "groups": l.groups, "data_fed": l.data_fed,
+             "Co": [m.Co for m in s.members] if grp else [l.Co]}
+        arrays = {k: v.cpu().numpy() for k, v in s.t.items()}
+        if grp:
+            for b in range(len(s.members)):
+                arrays[f"y{b}"] = s.ys[b].cpu().numpy()
+                arrays[f"dw{b}"] = s.dws[b].cpu().numpy()
+                arrays[f"db{b}"] = s.dbs[b].cpu().numpy()
+        else:
+            arrays["y"] = s.y.cpu().numpy()
+            arrays["dw"] = s.dw.cpu().numpy()
+            arrays["db"] = s.db.cpu().numpy()
+        if s.dx is not None:
+            arrays["dx"] = s.dx.cpu().numpy()
+        for k, v in arrays.items():
+            np.save(os.path.join(path, f"u{i}_{k}.npy"), v)
+        u["arrays"] = sorted(arrays)
+        meta["units"].append(u)
+    json.dump(meta, open(os.path.join(path, "meta.json"), "w"), indent=1)
+
+
 class GroupState:
     """Sibling layers that read one input, run as a fused group (one GEMM per pass; include/glp.h
     "fused sibling groups").  Same unit interface as LayerState."""
@@ -439,6 +497,8 @@ def run_glp(args, ws, rank, local):
             idxs = [j for j, m in enumerate(layers) if m.name in groups[gi]]
             states.append(GroupState([layers[j] for j in idxs], nl, ng, args.math, dev, grads,
                                      idxs))
+    if args.exact_data:
+        set_exact_data(states)
     stream = torch.cuda.current_stream()
 
     tree = None
@@ -637,6 +697,8 @@ def run_glp(args, ws, rank, local):
             avg = sum(us) / len(us)
             kern.append({"layer": s.name, "pass": name, "avg_us": round(avg, 2),
                          "total_us": sum(us), "tflops": round(s.flops / (avg * 1e-6) / 1e12, 1)})
+    if args.dump and rank == 0:
+        dump_units(states, args.dump, args.workload, args.math)
     peaks = load_peaks()
     dom = max(kern, key=lambda r: r["total_us"])
     peak_tf = peaks["bf16_tflops_sustained"] * (1.0 if args.math == "bf16" else NOMINAL_TF32_OVER_BF16)

@@ -126,6 +126,73 @@ def conv_bwd_filter_at(x, dy, w_shape, stride, pad, idx):
     return float(lib().oracle_conv_bwd_filter_at(*g, _ptr(x), _ptr(dy), co, ci, kh, kw))
 
 
+def conv_fwd_at(x, w, b, stride, pad, idx, absmode=False):
+    """One y[n,co,ho,wo] (fp64) by the definition of Alg. 1 (P82-99) / SURVEY a3:
+    y = b[co] + sum_{ci,kh,kw} W[co,ci,kh,kw] * x[n,ci,ho*S-P+kh, wo*S-P+kw] (zero outside).
+    absmode: sum of |W||x| (the element's condition scale; bias excluded).  For sampled parity at
+    full size, where the whole-tensor oracle would take too long."""
+    n, co, ho, wo = (int(v) for v in idx)
+    _, C, H, W = x.shape
+    _, _, Kh, Kw = w.shape
+    acc = 0.0
+    for kh in range(Kh):
+        ih = ho * stride - pad + kh
+        if ih < 0 or ih >= H:
+            continue
+        for kw in range(Kw):
+            iw = wo * stride - pad + kw
+            if iw < 0 or iw >= W:
+                continue
+            a = x[n, :, ih, iw].astype(np.float64)
+            wv = w[co, :, kh, kw].astype(np.float64)
+            acc += float(np.abs(a) @ np.abs(wv)) if absmode else float(a @ wv)
+    if not absmode and b is not None:
+        acc += float(b[co])
+    return acc
+
+
+def conv_bwd_data_at(dy, w, x_shape, stride, pad, idx, absmode=False):
+    """One dx[n,ci,h,w] (fp64) by the gather formula of SURVEY a4 (Alg. 2, P101-121):
+    dx = sum over (co, kh, kw) with (h+P-kh) and (w+P-kw) divisible by S and the quotients
+    (ho, wo) inside the H_o x W_o output of W[co,ci,kh,kw] * dy[n,co,ho,wo]."""
+    n, ci, h, ww = (int(v) for v in idx)
+    _, Co, Ho, Wo = dy.shape
+    _, _, Kh, Kw = w.shape
+    acc = 0.0
+    for kh in range(Kh):
+        th = h + pad - kh
+        if th < 0 or th % stride:
+            continue
+        ho = th // stride
+        if ho >= Ho:
+            continue
+        for kw in range(Kw):
+            tw = ww + pad - kw
+            if tw < 0 or tw % stride:
+                continue
+            wo = tw // stride
+            if wo >= Wo:
+                continue
+            a = dy[n, :, ho, wo].astype(np.float64)
+            wv = w[:, ci, kh, kw].astype(np.float64)
+            acc += float(np.abs(a) @ np.abs(wv)) if absmode else float(a @ wv)
+    return acc
+
+
+def conv_bwd_filter_at_abs(x, dy, w_shape, stride, pad, idx):
+    """sum_{n,ho,wo} |dy[n,co,ho,wo]| |x[n,ci,ho*S-P+kh, wo*S-P+kw]|: the condition scale of one
+    dW element (the plain definition with absolute values; zero outside the image)."""
+    co, ci, kh, kw = (int(v) for v in idx)
+    N, C, H, W = x.shape
+    _, _, Ho, Wo = dy.shape
+    hs = np.arange(Ho) * stride - pad + kh
+    ws = np.arange(Wo) * stride - pad + kw
+    hv, wv = (hs >= 0) & (hs < H), (ws >= 0) & (ws < W)
+    xs = np.abs(x[:, ci][:, hs[hv]][:, :, ws[wv]].astype(np.float64))
+    ds = np.abs(dy[:, co][:, hv][:, :, wv].astype(np.float64))
+    return float((xs * ds).sum())
+
+
 def im2col(x_n, kh, kw, stride=1, pad=0):
     """Caffe im2col of one sample (C,H,W) -> col[(ci*Kh+kh)*Kw+kw, ho*Wo+wo] (fp32)."""
     x_n = _f32(x_n)

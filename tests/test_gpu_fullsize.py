@@ -1,0 +1,156 @@
+"""Full-size parity: every BASELINE.json config at its full batch, run by bench.py itself (same
+plans, same CUDA-graph-replayed step DAG it times; `--dump` saves each unit's inputs and outputs
+after the timed steps), checked against the oracle on sampled outputs it computes one by one
+(oracle.conv_fwd_at / conv_bwd_data_at / conv_bwd_filter_at) and on db in full.
+
+Bars: integer data (`--exact-data`) -> every sampled element bit-exact; float
+data -> |g - r| <= 2e-2 * max_sampled |r| against the fp64 oracle on the unrounded inputs (the
+north_star bar, normwise over the sample) and |g - r_emu| <= 1e-5 * sum|a||b| against the oracle
+on the operands rounded as the pack step defines (the condition-aware bound of fp32 accumulation
+over exactly rounded products).  Samples always include the first and the last element (the
+ragged last tile) of every tensor.
+"""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import oracle
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+EMU = {"tf32": oracle.round_tf32_rna, "bf16": oracle.round_bf16_rne}
+NS = 40   # sampled elements per tensor
+
+
+def _bench_dump(tmp, workload, math, exact):
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--workload", str(workload), "--math",
+           math, "--steps", "2", "--warmup", "3", "--no-cpu-baseline", "--no-e2e", "--dump", str(tmp)]
+    if exact:
+        cmd.append("--exact-data")
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["launch"].startswith("cuda_graph")
+    return json.load(open(os.path.join(tmp, "meta.json")))
+
+
+def _load(tmp, i, name):
+    return np.load(os.path.join(tmp, f"u{i}_{name}.npy"), mmap_mode="r")
+
+
+def _samples(shape, rng):
+    idx = [tuple(0 for _ in shape), tuple(s - 1 for s in shape)]
+    idx += [tuple(int(rng.integers(0, s)) for s in shape) for _ in range(NS - 2)]
+    return idx
+
+
+def _check(kind, got, ref, emu, scale, exact, math, what):
+    got, ref = np.asarray(got, np.float64), np.asarray(ref, np.float64)
+    if exact:
+        np.testing.assert_array_equal(got, ref, err_msg=what)
+        return
+    bar = 2e-2 * max(np.abs(ref).max(), 1e-30)
+    assert np.abs(got - ref).max() <= bar, (what, np.abs(got - ref).max() / bar * 2e-2)
+    emu, scale = np.asarray(emu, np.float64), np.asarray(scale, np.float64)
+    assert np.all(np.abs(got - emu) <= 1e-5 * scale + 1e-30), (
+        what, float((np.abs(got - emu) / np.maximum(scale, 1e-30)).max()))
+
+
+def _check_unit(tmp, i, u, math, exact, rng):
+    S, P, G = u["S"], u["P"], u["groups"]
+    x = np.asarray(_load(tmp, i, "x"))
+    grp = u["kind"] == "group"
+    nb = len(u["Co"])
+    r = EMU[math]
+    xe = r(x)
+    dx_terms = []
+    for b in range(nb):
+        sfx = str(b) if grp else ""
+        w = np.asarray(_load(tmp, i, "w" + sfx))
+        bias = np.asarray(_load(tmp, i, "b" + sfx))
+        dy = np.asarray(_load(tmp, i, "dy" + sfx))
+        y = _load(tmp, i, "y" + sfx)
+        dw = _load(tmp, i, "dw" + sfx)
+        db = _load(tmp, i, "db" + sfx)
+        we, dye = r(w), r(dy)
+        Cg, Cog = u["C"] // G, u["Co"][b] // G
+        name = f"{u['names'][b]}"
+
+        def grp_of(co):   # Caffe groups: output channel co reads input channels of its group
+            g = co // Cog
+            return g, slice(g * Cg, (g + 1) * Cg), slice(g * Cog, (g + 1) * Cog)
+
+        # forward
+        idx = _samples(y.shape, rng)
+        g_, ref, emu, sc = [], [], [], []
+        for n, co, ho, wo in idx:
+            g, cs, _ = grp_of(co)
+            xi = x[n:n + 1, cs]
+            j = (0, co - g * Cog, ho, wo)
+            wg = w[g * Cog:(g + 1) * Cog]
+            bg = bias[g * Cog:(g + 1) * Cog]
+            g_.append(y[n, co, ho, wo])
+            ref.append(oracle.conv_fwd_at(xi, wg, bg, S, P, j))
+            emu.append(oracle.conv_fwd_at(xe[n:n + 1, cs], we[g * Cog:(g + 1) * Cog], bg, S, P, j))
+            sc.append(oracle.conv_fwd_at(xi, wg, None, S, P, j, absmode=True) + abs(float(bg[j[1]])))
+        _check("y", g_, ref, emu, sc, exact, math, f"{name} y")
+        # filter gradient
+        idx = _samples(dw.shape, rng)
+        g_, ref, emu, sc = [], [], [], []
+        for co, ci, kh, kw in idx:
+            g, cs, os_ = grp_of(co)
+            j = (co - g * Cog, ci, kh, kw)
+            wsh = (Cog, Cg, w.shape[2], w.shape[3])
+            g_.append(dw[co, ci, kh, kw])
+            ref.append(oracle.conv_bwd_filter_at(x[:, cs], dy[:, os_], wsh, S, P, j))
+            emu.append(oracle.conv_bwd_filter_at(xe[:, cs], dye[:, os_], wsh, S, P, j))
+            sc.append(oracle.conv_bwd_filter_at_abs(x[:, cs], dy[:, os_], wsh, S, P, j))
+        _check("dw", g_, ref, emu, sc, exact, math, f"{name} dW")
+        # bias gradient in full (plain sum over n, ho, wo)
+        ref = dy.astype(np.float64).sum(axis=(0, 2, 3))
+        if exact:
+            np.testing.assert_array_equal(np.asarray(db, np.float64), ref, err_msg=f"{name} db")
+        else:
+            scale = np.abs(dy.astype(np.float64)).sum(axis=(0, 2, 3))
+            assert np.all(np.abs(np.asarray(db, np.float64) - ref) <= 1e-5 * scale + 1e-30), name
+        dx_terms.append((w, we, dy, dye, Cg, Cog))
+    if "dx" not in u["arrays"]:
+        assert u["data_fed"]   # the data-fed first layer has no backward-data pass (R9)
+        return
+    dx = _load(tmp, i, "dx")
+    idx = _samples(dx.shape, rng)
+    g_, ref, emu, sc = [], [], [], []
+    for n, ci, h, ww in idx:
+        rr = ee = ss = 0.0
+        for w, we, dy, dye, Cg, Cog in dx_terms:
+            g = ci // Cg
+            os_ = slice(g * Cog, (g + 1) * Cog)
+            j = (0, ci - g * Cg, h, ww)
+            xs = (1, Cg) + tuple(dx.shape[2:])
+            rr += oracle.conv_bwd_data_at(dy[n:n + 1, os_], w[os_], xs, S, P, j)
+            ee += oracle.conv_bwd_data_at(dye[n:n + 1, os_], we[os_], xs, S, P, j)
+            ss += oracle.conv_bwd_data_at(dy[n:n + 1, os_], w[os_], xs, S, P, j, absmode=True)
+        g_.append(dx[n, ci, h, ww])
+        ref.append(rr)
+        emu.append(ee)
+        sc.append(ss)
+    _check("dx", g_, ref, emu, sc, exact, math, f"{'+'.join(u['names'])} dx")
+
+
+CASES = [(1, "bf16", False), (2, "bf16", False), (3, "bf16", False), (4, "bf16", False),
+         (4, "bf16", True), (4, "tf32", False), (4, "tf32", True), (5, "bf16", False),
+         (5, "bf16", True), (6, "bf16", False), (7, "bf16", True)]
+
+
+@pytest.mark.parametrize("case", CASES, ids=lambda c: f"cfg{c[0]}-{c[1]}-{'exact' if c[2] else 'float'}")
+def test_fullsize_sampled_parity(case, tmp_path):
+    workload, math, exact = case
+    meta = _bench_dump(tmp_path, workload, math, exact)
+    assert meta["workload"] == workload and meta["math"] == math
+    rng = np.random.Generator(np.random.PCG64(1000 + workload))
+    for i, u in enumerate(meta["units"]):
+        _check_unit(tmp_path, i, u, math, exact, rng)

@@ -240,3 +240,32 @@ def test_sampled_wgrad_element_matches_full():
     dw, _ = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, S, P)
     for idx in [(0, 0, 0, 0), (4, 3, 2, 2), (2, 1, 0, 2), (1, 2, 1, 1)]:
         assert oracle.conv_bwd_filter_at(d["x"], d["dy"], d["w"].shape, S, P, idx) == dw[idx]
+
+
+@pytest.mark.parametrize("geo", [(3, 4, 9, 9, 5, 3, 2, 1), (2, 3, 13, 11, 6, 5, 1, 2),
+                                 (2, 2, 23, 23, 3, 11, 4, 0), (1, 3, 10, 10, 2, 3, 1, 3),
+                                 (2, 6, 4, 9, 2, 1, 1, 0)])
+def test_single_element_oracle_matches_full(geo):
+    """The one-element forms used by the full-size sampled parity tests (conv_fwd_at,
+    conv_bwd_data_at, conv_bwd_filter_at and the |a||b| condition scales) equal the whole-tensor
+    oracle — itself pinned above by hand cases, torch fp64 and identities — on every element of
+    small tensors (stride 1/2/4, pad 0..3, 1x1, 11x11)."""
+    N, C, H, W, Co, K, S, P = geo
+    Ho, Wo = oracle.out_dim(H, K, S, P), oracle.out_dim(W, K, S, P)
+    d = gen_custom(N, C, H, W, Co, K, K, 23, Ho=Ho, Wo=Wo)
+    x, w, b, dy = d["x"], d["w"], d["b"], d["dy"]
+    y = oracle.conv_fwd(x, w, b, S, P)
+    ya = oracle.conv_fwd(x, w, None, S, P, absmode=True)
+    dx = oracle.conv_bwd_data(dy, w, x.shape, S, P)
+    dxa = oracle.conv_bwd_data(dy, w, x.shape, S, P, absmode=True)
+    dw, _ = oracle.conv_bwd_filter(x, dy, w.shape, S, P)
+    dwa, _ = oracle.conv_bwd_filter(x, dy, w.shape, S, P, absmode=True)
+    for idx in np.ndindex(*y.shape):
+        assert oracle.conv_fwd_at(x, w, b, S, P, idx) == pytest.approx(y[idx], rel=1e-12, abs=1e-13)
+        assert oracle.conv_fwd_at(x, w, b, S, P, idx, absmode=True) == pytest.approx(ya[idx], rel=1e-12, abs=1e-13)
+    for idx in np.ndindex(*x.shape):
+        assert oracle.conv_bwd_data_at(dy, w, x.shape, S, P, idx) == pytest.approx(dx[idx], rel=1e-12, abs=1e-13)
+        assert oracle.conv_bwd_data_at(dy, w, x.shape, S, P, idx, absmode=True) == pytest.approx(dxa[idx], rel=1e-12, abs=1e-13)
+    for idx in np.ndindex(*w.shape):
+        assert oracle.conv_bwd_filter_at(x, dy, w.shape, S, P, idx) == pytest.approx(dw[idx], rel=1e-12, abs=1e-13)
+        assert oracle.conv_bwd_filter_at_abs(x, dy, w.shape, S, P, idx) == pytest.approx(dwa[idx], rel=1e-12, abs=1e-13)

@@ -78,6 +78,10 @@ typedef struct {
                             dy packed on the padded grid), 0: im2col implicit GEMM             */
   int fwd_halo;          /* 1: forward by the shared-halo kernel (space-to-depth layers: x' staged
                             once per tile for all taps, outputs on the padded grid), 0: im2col   */
+  int wgrad_fused_dy;    /* 1: the halo filter gradient builds its dy operand (and db) from the fp32
+                            dy itself: glp_stage_pack(GLP_PACK_DY*) then only records the dy
+                            pointer for this workspace (it must stay valid until the filter-gradient
+                            and backward-data stages have run; the backward-data stage packs it) */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

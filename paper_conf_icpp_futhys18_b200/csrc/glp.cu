@@ -293,6 +293,14 @@ struct MapCache {
   };
   Entry e[3][8];
   int next[3] = {0, 0, 0};
+  // fused-dy halo plans: the dy tensor recorded by glp_stage_pack(GLP_PACK_DY*) per workspace
+  // (the filter gradient reads it in fp32 itself; nothing is packed at that point)
+  struct DyRec {
+    const void *ws = nullptr;
+    const float *dy = nullptr;
+  };
+  DyRec dyrec[16];
+  int dy_next = 0;
   std::mutex mu;
   MapCache() = default;
   MapCache(const MapCache &) {}
@@ -323,6 +331,7 @@ struct glp_plan_s {
   int hw_grid = 0, hw_smem = 0, hw_regs = 0;
   // halo forward (hfwd.cuh) for the same space-to-depth layers: x' staged once per tile for all
   // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
+  int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
   int hfwd = 0;
   HfwdParams hf{};
   int hf_grid = 0, hf_smem = 0, hf_regs = 0;
@@ -343,6 +352,7 @@ struct glp_plan_s {
   int bn_model = 1;    // GLP_BN_MODEL=0: always the default fwd/dgrad tile (A/B runs)
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
   int allow_hfwd = 1;  // GLP_HFWD=0: im2col forward for space-to-depth layers (A/B runs)
+  int allow_fdy = 1;   // GLP_HALO_FDY=0: halo filter gradient on the packed dy (A/B runs)
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -361,6 +371,7 @@ namespace {
 // constant of 148 ranges, never the queried device), so the reduction order is fixed.
 glp_status_t plan_halo(glp_plan_s &P) {
   P.halo = 0;
+  P.halo_fdy = 0;
   const glp_conv_desc_s &x = P.dxg;
   if (!P.allow_halo || !P.s2d || P.elem != 2 || P.Cpx != 64 || P.tapsx < 2) return GLP_OK;
   const int Ks = x.Kh, T = P.tapsx;
@@ -404,14 +415,29 @@ glp_status_t plan_halo(glp_plan_s &P) {
   h.co = x.Co;
   h.mpad = T * P.Cpx;
   h.ld = bn;
+  // fused dy (single layers): the filter gradient builds its dy operand from the fp32 tensor
+  const int fdy = (P.allow_fdy && P.d.nbr <= 1 && bn <= 128 && rows < (1LL << 31) - 256) ? 1 : 0;
+  // builder groups: 3 when a thread's channels fit 3 x 32 registers groups (C_o <= 96), else 2
+  const int ncg = fdy ? (bn <= 96 ? 3 : 2) : 0;
+  const int red_bytes = fdy ? 4 * ncg * 256 * 4 + 16 : 0;   // db partial staging
+  h.stages = std::min(8, (P.smem_cap - 2048 - red_bytes) / stage);
+  if (h.stages < 2) return GLP_OK;
+  h.ho = P.d.Ho;
+  h.wo = P.d.Wo;
+  h.rows = (int)rows;
+  h.div_img = FastDiv((uint32_t)(x.H * x.W));
+  h.div_w = FastDiv((uint32_t)x.W);
   P.hw_grid = h.splits;
-  P.hw_smem = 1024 + h.stages * stage + 8 * (2 * h.stages + 1) + 16;
-  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hwgrad_kernel),
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  P.hw_smem = 1024 + h.stages * stage + 8 * (2 * h.stages + 2) + 16 + red_bytes;
+  const void *fn = ncg == 3 ? reinterpret_cast<const void *>(hwgrad_kernel<3>)
+                 : ncg == 2 ? reinterpret_cast<const void *>(hwgrad_kernel<2>)
+                            : reinterpret_cast<const void *>(hwgrad_kernel<0>);
+  GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
-  GLP_CUDA(cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(hwgrad_kernel)));
+  GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
   P.hw_regs = fa.numRegs;
   P.halo = 1;
+  P.halo_fdy = ncg;
   return GLP_OK;
 }
 
@@ -776,7 +802,8 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
 glp_status_t launch_pack_dy(const glp_plan_s &P, const BrIn &dy, uint8_t *ws, bool with_db,
                             cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
-  float *dbp = with_db ? reinterpret_cast<float *>(ws + P.off_dbpart) : nullptr;
+  // fused-dy plans: db partials come from the filter-gradient kernel (this pack only feeds dgrad)
+  float *dbp = (with_db && !P.halo_fdy) ? reinterpret_cast<float *>(ws + P.off_dbpart) : nullptr;
   const int Ws = P.halo ? d.Wo : 1, Wd = P.halo ? P.dxg.W : 1;
   const int HWd = P.halo ? P.dxg.H * P.dxg.W : -1;
   if (dy.n <= 1)
@@ -926,6 +953,25 @@ glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, CUtensorMap &a
   return GLP_OK;
 }
 
+void record_dy(glp_plan_s &P, const void *ws, const float *dy) {
+  std::lock_guard<std::mutex> lk(P.maps.mu);
+  for (auto &r : P.maps.dyrec)
+    if (r.ws == ws) {
+      r.dy = dy;
+      return;
+    }
+  auto &r = P.maps.dyrec[P.maps.dy_next];
+  P.maps.dy_next = (P.maps.dy_next + 1) % 16;
+  r.ws = ws;
+  r.dy = dy;
+}
+const float *recorded_dy(glp_plan_s &P, const void *ws) {
+  std::lock_guard<std::mutex> lk(P.maps.mu);
+  for (auto &r : P.maps.dyrec)
+    if (r.ws == ws) return r.dy;
+  return nullptr;
+}
+
 glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
                           cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
@@ -1016,8 +1062,11 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
 }
 
-glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
+glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const float *dy) {
   const glp_conv_desc_s &d = P.dxg;
+  if (P.halo_fdy && !dy)
+    return fail(GLP_ERR_INVALID_VALUE, "filter gradient: no dy recorded for this workspace "
+                                       "(glp_stage_pack(GLP_PACK_DY*) first)");
   const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x' and dy
   CUtensorMap mapX, mapDy;
   glp_status_t s = cached_maps(P, 2, ws, mapX, mapDy, [&](CUtensorMap &X, CUtensorMap &Dy) {
@@ -1031,10 +1080,18 @@ glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   HwgradParams p = P.hw;
   p.part = reinterpret_cast<float *>(ws + P.off_part);
   p.dbg_skip = P.dbg_skip;
+  if (P.halo_fdy) {
+    p.dy = dy;
+    p.dy_c = P.y_img_c;
+    const DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
+    p.db_part = a.part;
+    p.db_tickets = a.tickets;
+    p.n_tickets = (int)cdiv(P.d.Co, 32);
+  }
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof(cfg));
   cfg.gridDim = dim3((unsigned)P.hw_grid);
-  cfg.blockDim = dim3(HW_THREADS);
+  cfg.blockDim = dim3(hw_threads(P.halo_fdy));
   cfg.dynamicSmemBytes = (size_t)P.hw_smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
@@ -1043,13 +1100,18 @@ glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
   cfg.attrs = attr;
   cfg.numAttrs = P.pdl ? 1 : 0;
   void *args[] = {&p, &mapX, &mapDy};
-  GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hwgrad_kernel), args));
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, P.halo_fdy == 3 ? reinterpret_cast<void *>(hwgrad_kernel<3>)
+                                : P.halo_fdy == 2 ? reinterpret_cast<void *>(hwgrad_kernel<2>)
+                                                  : reinterpret_cast<void *>(hwgrad_kernel<0>),
+                                args));
   GLP_LAUNCH_CHECK("hwgrad_kernel");
   return GLP_OK;
 }
 
-glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st) {
-  if (P.halo) return run_wgrad_halo(P, ws, st);
+// dy: the fp32 dy tensor, used only by fused-dy halo plans (which pack nothing for the filter
+// gradient); every other plan reads the packed dy in the workspace.
+glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const float *dy = nullptr) {
+  if (P.halo) return run_wgrad_halo(P, ws, st, dy);
   const glp_conv_desc_s &d = P.dxg;
   const PassPlan &pp = P.wgrad;
   const void *xpk = ws + P.off_xpk, *dypk = ws + P.off_dypk;
@@ -1108,14 +1170,15 @@ glp_status_t tc_fwd(glp_plan_s &P, const float *x, const BrIn &w, const BrIn &b,
 glp_status_t tc_bwd(glp_plan_s &P, const float *x, const BrIn &dy, const BrIn &w, float *dx,
                     const BrOut &dw, const BrOut &db, bool with_db, int accumulate, uint8_t *ws,
                     cudaStream_t st) {
-  glp_status_t s = launch_pack_dy(P, dy, ws, with_db, st);
-  if (s) return s;
+  glp_status_t s = GLP_OK;
+  if (!P.halo_fdy || dx)   // fused-dy plans pack dy only for the backward-data pass
+    if ((s = launch_pack_dy(P, dy, ws, with_db, st))) return s;
   if (dx) {
     if ((s = run_pack_w_dgrad(P, w, ws, st))) return s;
     if ((s = run_dgrad_gemm(P, dx, ws, st))) return s;
   }
   if ((s = launch_pack_x(P, x, ws + P.off_xpk, st))) return s;
-  if ((s = run_wgrad_gemm(P, ws, st))) return s;
+  if ((s = run_wgrad_gemm(P, ws, st, dy.p[0]))) return s;
   return run_wgrad_reduce(P, dw, with_db ? &db : nullptr, accumulate, ws, st);
 }
 
@@ -1359,6 +1422,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
+  if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
@@ -1441,6 +1505,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
                          : align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = (int)cdiv((long long)c.N * dy_hw, P->pack_block ? PACK_PT : PACKW_ROWS);
+    if (P->halo_fdy) P->db_rows = P->hw.splits;   // one db partial per filter-gradient CTA
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;
@@ -1506,6 +1571,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->math = P->math;
   I->wgrad_halo = P->halo;
   I->fwd_halo = P->hfwd;
+  I->wgrad_fused_dy = P->halo_fdy ? 1 : 0;
   if (P->hfwd) {
     I->grid_fwd = P->hf_grid;
     I->tile_n_fwd = P->hf.bn;
@@ -1622,8 +1688,8 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
     }
     const BrOut dbt = br_out(*P, 1, &dbg);
     if ((s = launch_pack_x(*P, x + o.x, wsb + P->off_xpk, st)) ||
-        (s = launch_pack_dy(*P, br_in1(dy + o.y), wsb, db != nullptr, st)) ||
-        (s = run_wgrad_gemm(*P, wsb, st)) ||
+        (!P->halo_fdy && (s = launch_pack_dy(*P, br_in1(dy + o.y), wsb, db != nullptr, st))) ||
+        (s = run_wgrad_gemm(*P, wsb, st, dy + o.y)) ||
         (s = run_wgrad_reduce(*P, br_out(*P, 1, &dwg), db ? &dbt : nullptr, accumulate ? 1 : 0, wsb, st)))
       return s;
   }
@@ -1682,8 +1748,13 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
     uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
     switch (what) {
       case GLP_PACK_X: s = launch_pack_x(*P, src + o.x, wsb + P->off_xpk, st); break;
-      case GLP_PACK_DY: s = launch_pack_dy(*P, br_in1(src + o.y), wsb, false, st); break;
-      case GLP_PACK_DY_DB: s = launch_pack_dy(*P, br_in1(src + o.y), wsb, true, st); break;
+      case GLP_PACK_DY:
+      case GLP_PACK_DY_DB:
+        if (P->halo_fdy)   // recorded only: the filter gradient reads it, bwd_data packs it
+          record_dy(*P, wsb, src + o.y);
+        else
+          s = launch_pack_dy(*P, br_in1(src + o.y), wsb, what == GLP_PACK_DY_DB, st);
+        break;
       case GLP_PACK_W_FWD: s = run_pack_w_fwd(*P, br_in1(src + o.w), wsb, st); break;
       case GLP_PACK_W_BWD_DATA: s = run_pack_w_dgrad(*P, br_in1(src + o.w), wsb, st); break;
     }
@@ -1714,8 +1785,14 @@ glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_byt
   if ((s = validate_ptrs({dx}))) return s;
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
-    if ((s = run_dgrad_gemm(*P, dx + o.x, static_cast<uint8_t *>(ws) + o.ws,
-                            static_cast<cudaStream_t>(stream))))
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
+    if (P->halo_fdy) {   // dy was only recorded by glp_stage_pack: pack it now for dgrad
+      const float *dy = recorded_dy(*P, wsb);
+      if (!dy) return fail(GLP_ERR_INVALID_VALUE, "bwd_data: glp_stage_pack(GLP_PACK_DY*) first");
+      if ((s = launch_pack_dy(*P, br_in1(dy), wsb, false, static_cast<cudaStream_t>(stream))))
+        return s;
+    }
+    if ((s = run_dgrad_gemm(*P, dx + o.x, wsb, static_cast<cudaStream_t>(stream))))
       return s;
   }
   return GLP_OK;
@@ -1724,10 +1801,12 @@ glp_status_t glp_stage_bwd_data(glp_plan_t P, float *dx, void *ws, size_t ws_byt
 glp_status_t glp_stage_bwd_filter(glp_plan_t P, void *ws, size_t ws_bytes, glp_stream_t stream) {
   glp_status_t s = stage_check(P, ws, ws_bytes);
   if (s) return s;
-  for (int g = 0; g < P->groups; ++g)
-    if ((s = run_wgrad_gemm(*P, static_cast<uint8_t *>(ws) + goff(P, g).ws,
-                            static_cast<cudaStream_t>(stream))))
+  for (int g = 0; g < P->groups; ++g) {
+    uint8_t *wsb = static_cast<uint8_t *>(ws) + goff(P, g).ws;
+    if ((s = run_wgrad_gemm(*P, wsb, static_cast<cudaStream_t>(stream),
+                            P->halo_fdy ? recorded_dy(*P, wsb) : nullptr)))
       return s;
+  }
   return GLP_OK;
 }
 
@@ -2061,10 +2140,11 @@ glp_status_t glp_pool_conv_bwd(glp_pool_t Q, const float *x, const float *dy, co
     cudaStream_t si = Q->streams[i];
     const float *xn = x + n * xs, *dyn = dy + n * ys;
     if (tc) {
-      if ((s = launch_pack_dy(P1, br_in1(dyn), wsi, db != nullptr, si))) return s;
+      if ((!P1.halo_fdy || dx) && (s = launch_pack_dy(P1, br_in1(dyn), wsi, db != nullptr, si)))
+        return s;
       if (dx && (s = run_dgrad_gemm(P1, dx + n * xs, wsi, si))) return s;
       const BrOut dbo = br_out(P1, 1, &dbi);
-      if ((s = launch_pack_x(P1, xn, wsi + P1.off_xpk, si)) || (s = run_wgrad_gemm(P1, wsi, si)) ||
+      if ((s = launch_pack_x(P1, xn, wsi + P1.off_xpk, si)) || (s = run_wgrad_gemm(P1, wsi, si, dyn)) ||
           (s = run_wgrad_reduce(P1, br_out(P1, 1, &dwi), db ? &dbo : nullptr, 1, wsi, si)))
         return s;
     } else {

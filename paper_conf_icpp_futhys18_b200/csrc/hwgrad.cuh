@@ -22,11 +22,16 @@
 // CTA = 192 threads: warps 0-3 epilogue, warp 4 TMA producer, warp 5 TMEM owner + MMA issuer.
 #pragma once
 #include "common.cuh"
+#include <cuda_bf16.h>
+
 #include "ptx.cuh"
 
 namespace glp {
 
 constexpr int HW_THREADS = 192;
+// fused-dy variant with NCG groups of 4 dy-building warps (warps 0-3, then 6-9, 10-13): group g
+// builds k-blocks kb0 + g, kb0 + g + NCG, ... so NCG k-blocks' loads are in flight at once
+__host__ __device__ constexpr int hw_threads(int ncg) { return ncg > 1 ? 192 + 128 * (ncg - 1) : 192; }
 constexpr int HW_BKP = 128;   // pixel rows (K) per k-block
 
 struct HwgradParams {
@@ -45,11 +50,24 @@ struct HwgradParams {
   float *part;        // [splits][mpad][ld] fp32
   int mpad, ld;
   int dbg_skip;       // diagnostics (GLP_DEBUG_SKIP): bit0 skip x' loads, bit1 dy loads, bit2 MMAs
+  // fused-dy variant (FDY): warps 0-3 build the dy operand of every k-block from the fp32 NCHW
+  // tensor themselves (round to bf16, swizzled smem stores) and emit the db partials, so the
+  // separate dy pack (read 4 B + write 2 B per element, then re-read 2 B here) disappears
+  const float *dy;    // NCHW fp32 (channel stride ho*wo, image stride dy_c*ho*wo)
+  int dy_c, ho, wo;   // channels per image of the dy tensor; valid output region
+  int rows;           // N * H' * W' (flattened padded grid)
+  FastDiv div_img, div_w;   // H' * W', W'
+  float *db_part;     // [splits][co]: this CTA's db partial (fixed order)
+  unsigned int *db_tickets;   // reduce_db's completion tickets (armed here: no dy pack runs)
+  int n_tickets;
 };
 
-__global__ void __launch_bounds__(HW_THREADS, 1)
+template <int NCG>   // 0: dy packed in the workspace (TMA); 2 or 3: fused dy, NCG builder groups
+__global__ void __launch_bounds__(hw_threads(NCG), 1)
     hwgrad_kernel(const __grid_constant__ HwgradParams p, const __grid_constant__ CUtensorMap tmapX,
                   const __grid_constant__ CUtensorMap tmapDy) {
+  constexpr bool FDY = NCG > 0;
+  constexpr int MAXG = NCG == 3 ? 3 : 4;   // 32-channel groups a builder thread holds (bn <= 32*MAXG)
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -66,7 +84,7 @@ __global__ void __launch_bounds__(HW_THREADS, 1)
   const int lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S_; ++s) {
-      mbar_init(full(s), 1);
+      mbar_init(full(s), FDY ? 5 : 1);   // FDY: + one arrival per warp of the building group
       mbar_init(empty(s), 1);
     }
     mbar_init(tfull, 1);
@@ -78,7 +96,7 @@ __global__ void __launch_bounds__(HW_THREADS, 1)
   }
   if (warp == 4 && lane == 0) {
     tma_prefetch(&tmapX);
-    tma_prefetch(&tmapDy);
+    if (!FDY) tma_prefetch(&tmapDy);
   }
   tc_fence_before();
   __syncthreads();
@@ -93,7 +111,7 @@ __global__ void __launch_bounds__(HW_THREADS, 1)
     // ===================================== producer ========================================
     int rs = 0;
     uint32_t rph = 0;
-    const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+    const bool la = !(p.dbg_skip & 1), lb = !FDY && !(p.dbg_skip & 2);
     const int nb = (p.bn + 63) / 64;
     const uint32_t tx = (la ? (uint32_t)(p.halo_rows * 128) : 0u) + (lb ? (uint32_t)p.b_bytes : 0u);
     for (int kb = kb0; kb < kb1; ++kb) {
@@ -141,6 +159,106 @@ __global__ void __launch_bounds__(HW_THREADS, 1)
     mma_commit_e<1>(tfull);
     __syncwarp();
   } else {
+    if (FDY) {
+      // ============================ dy operand + db partials (warps 0-3) =====================
+      // thread t = pixel row t of the k-block (q = kb*128 + t on the padded grid); for each group
+      // of 32 channels: 32 coalesced loads (lanes = consecutive pixels of one channel plane),
+      // a transposing butterfly that leaves channel 32g+lane's sum over the warp's 32 pixels in
+      // lane `lane` (added to dbacc[g] in k-block order: a fixed order), then RNE to bf16 and
+      // four 16-byte swizzled stores into the MN-major SW128 atoms of the stage's B region.
+      // group 0 = warps 0-3, group g >= 1 = warps 6+4(g-1) .. 9+4(g-1); group g builds k-blocks
+      // kb0 + g, kb0 + g + NCG, ...
+      const int grp = warp >= 6 ? (warp - 6) / 4 + 1 : 0;
+      const int t = threadIdx.x - (grp ? 192 + 128 * (grp - 1) : 0);
+      if (u == 0 && grp == 0)
+        for (int i = t; i < p.n_tickets; i += 128) p.db_tickets[i] = 0u;
+      const int ngrp = (p.bn + 31) / 32;   // <= MAXG (plan)
+      const size_t hw = (size_t)p.ho * p.wo;
+      float dbacc[MAXG];
+#pragma unroll
+      for (int g = 0; g < MAXG; ++g) dbacc[g] = 0.f;
+      for (int kb = kb0 + grp; kb < kb1; kb += NCG) {
+        const int rs = (kb - kb0) % S_;
+        const uint32_t rph = (uint32_t)(((kb - kb0) / S_) & 1);
+        const int q = kb * HW_BKP + t;
+        uint32_t n = 0, rem = 0, h = 0, w = 0;
+        p.div_img.divmod((uint32_t)min(q, p.rows - 1), n, rem);
+        p.div_w.divmod(rem, h, w);
+        const bool ok = q < p.rows && (int)h < p.ho && (int)w < p.wo;
+        const float *src = p.dy + ((size_t)n * p.dy_c * p.ho + h) * p.wo + w;
+        // every load of the k-block in flight before anything waits (registers, not smem: the
+        // stage need not be free yet)
+        float v[MAXG][32];
+#pragma unroll
+        for (int g = 0; g < MAXG; ++g)
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const int co = g * 32 + j;
+            v[g][j] = (ok && g < ngrp && co < p.co) ? __ldg(src + (size_t)co * hw) : 0.f;
+          }
+        mbar_wait(empty(rs), rph ^ 1u);
+        const uint32_t sB = base + (uint32_t)rs * stage_bytes + (uint32_t)p.a_bytes;
+#pragma unroll
+        for (int g = 0; g < MAXG; ++g) {
+          if (g >= ngrp) break;
+          float tt[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) tt[j] = v[g][j];
+#pragma unroll
+          for (int wdt = 16; wdt >= 1; wdt >>= 1) {
+            const bool up = (lane & wdt) != 0;
+#pragma unroll
+            for (int j = 0; j < wdt; ++j) {
+              const float send = up ? tt[j] : tt[j + wdt];
+              const float keep = up ? tt[j + wdt] : tt[j];
+              tt[j] = keep + __shfl_xor_sync(0xffffffffu, send, wdt);
+            }
+          }
+          dbacc[g] += tt[0];
+#pragma unroll
+          for (int c = 0; c < 4; ++c) {
+            const int co0 = g * 32 + c * 8;
+            if (co0 >= p.bn) break;
+            __nv_bfloat162 a = __floats2bfloat162_rn(v[g][c * 8], v[g][c * 8 + 1]);
+            __nv_bfloat162 b = __floats2bfloat162_rn(v[g][c * 8 + 2], v[g][c * 8 + 3]);
+            __nv_bfloat162 cc = __floats2bfloat162_rn(v[g][c * 8 + 4], v[g][c * 8 + 5]);
+            __nv_bfloat162 d = __floats2bfloat162_rn(v[g][c * 8 + 6], v[g][c * 8 + 7]);
+            const uint32_t atom = (uint32_t)(co0 >> 6), ch = (uint32_t)((co0 & 63) >> 3);
+            const uint32_t addr = sB + atom * (uint32_t)(HW_BKP * 128) + (uint32_t)t * 128u +
+                                  ((ch ^ (uint32_t)(t & 7)) << 4);
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr),
+                         "r"(*reinterpret_cast<uint32_t *>(&a)), "r"(*reinterpret_cast<uint32_t *>(&b)),
+                         "r"(*reinterpret_cast<uint32_t *>(&cc)), "r"(*reinterpret_cast<uint32_t *>(&d))
+                         : "memory");
+          }
+        }
+        fence_proxy_async_smem();   // generic-proxy smem writes -> visible to tcgen05.mma
+        __syncwarp();
+        if (lane == 0) mbar_arrive(full(rs));
+      }
+      // db partial of this CTA's pixel range: warps 0..3 in order (fixed), one row per CTA
+      const uint32_t sred = (bars + 8u * (2 * S_ + 2) + 15u) & ~15u;   // 4*NCG x 256 floats
+      float *red = reinterpret_cast<float *>(smem_raw + (sred - raw));
+      const int slot = grp * 4 + (warp & 3);   // a fixed slot per warp (4 per group)
+#pragma unroll
+      for (int g = 0; g < MAXG; ++g)
+        if (g < ngrp) red[slot * 256 + g * 32 + lane] = dbacc[g];
+      named_bar_sync(1, 128 * NCG);
+      if (grp == 0) {
+        for (int co = t; co < p.co; co += 128) {
+          float tot = 0.f;   // groups in order, each the sum of its 4 warps in order
+#pragma unroll
+          for (int gg = 0; gg < NCG; ++gg) {
+            float a = 0.f;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) a += red[(gg * 4 + k) * 256 + co];
+            tot += a;
+          }
+          p.db_part[(size_t)u * p.co + co] = tot;
+        }
+      }
+    }
+    if (!FDY || warp < 4) {   // groups >= 1 have no epilogue role (TMEM lanes: warps 0-3)
     // ===================================== epilogue ========================================
     mbar_wait(tfull, 0);
     tc_fence_after();
@@ -170,6 +288,7 @@ __global__ void __launch_bounds__(HW_THREADS, 1)
             if (q < lim) dst[c0 + q] = empty_range ? 0.f : __uint_as_float(v[q]);
         }
       }
+    }
     }
   }
   pdl_launch_dependents();

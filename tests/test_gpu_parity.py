@@ -265,6 +265,7 @@ HALO_SHAPES = [
     ("caffenet_conv1_s4", 2, 3, 67, 67, 96, 11, 4, 0),
     ("s2d_c12_k5_s2", 3, 12, 20, 21, 40, 5, 2, 2),             # 9 taps, C_o = 40 (one B atom)
     ("s2d_c16_k3_s2", 2, 16, 17, 15, 24, 3, 2, 1),             # 4 taps, no duplicate
+    ("s2d_co112_k3_s2", 2, 16, 17, 15, 112, 3, 2, 1),          # C_o in (96, 128]: 2 dy builder groups
 ]
 
 
@@ -304,6 +305,40 @@ def test_halo_wgrad_random_and_invariant(shape):
         assert np.abs(runs[0][k] - e).max() / np.abs(e).max() <= 1e-4, k
         for other in runs[1:]:
             np.testing.assert_array_equal(other[k], runs[0][k], err_msg=k)
+
+
+@pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
+def test_halo_wgrad_fused_dy(shape, monkeypatch):
+    """Fused-dy halo filter gradient (hwgrad_kernel<true>: the CTA's own warps build the dy
+    operand from fp32 NCHW with the pack's RNE rounding, and emit the db partials): dW bitwise
+    equal to the packed-dy kernel (GLP_HALO_FDY=0: same operand bits, same MMA order), db within
+    fp32 summation-order noise of it; the staged calls (GLP_PACK_DY_DB only records dy,
+    bwd_data packs it lazily) bitwise equal to the composed calls."""
+    d = _data(shape, seed=49)
+    layer = _layer(shape, "bf16")
+    assert layer.info.wgrad_fused_dy == 1
+    ref = _run(layer, d)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    dx = torch.empty(layer.x_shape, device=DEV)
+    dw = torch.empty(layer.w_shape, device=DEV)
+    db = torch.empty(layer.geom.Co, device=DEV)
+    layer.stage_pack(glp.GLP_PACK_X, t["x"])
+    layer.stage_pack(glp.GLP_PACK_DY_DB, t["dy"])
+    layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
+    layer.stage_bwd_filter()
+    layer.stage_reduce(dw, db)
+    layer.stage_bwd_data(dx)
+    torch.cuda.synchronize()
+    for k, v in (("dx", dx), ("dw", dw), ("db", db)):
+        np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=k)
+    monkeypatch.setenv("GLP_HALO_FDY", "0")
+    layer0 = _layer(shape, "bf16")
+    assert layer0.info.wgrad_fused_dy == 0 and layer0.info.wgrad_halo == 1
+    got0 = _run(layer0, d)
+    np.testing.assert_array_equal(got0["dw"], ref["dw"])
+    np.testing.assert_array_equal(got0["dx"], ref["dx"])
+    scale = np.abs(d["dy"].astype(np.float64)).sum(axis=(0, 2, 3))
+    assert np.all(np.abs(got0["db"].astype(np.float64) - ref["db"]) <= 1e-6 * scale)
 
 
 @pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])

@@ -71,7 +71,13 @@ def main(rnd, rep, launches=None, workload=4, math="bf16"):
     flops = {l.name: l.flops_per_pass() for l in config(workload)}
     outdir = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(outdir, exist_ok=True)
-    rows = [d for d in raw_rows(rep) if "igemm" in d["Kernel Name"][1] or "hwgrad" in d["Kernel Name"][1]]
+    rows = [d for d in raw_rows(rep) if any(k in d["Kernel Name"][1] for k in ("igemm", "hwgrad", "hfwd"))]
+    # the capture may hold more than one step: take the last one that starts with conv1's forward
+    starts = [i for i, d in enumerate(rows) if "hfwd" in d["Kernel Name"][1]]
+    if starts and len(rows) - starts[-1] < len(ORDER):
+        starts = starts[:-1]
+    if starts:
+        rows = rows[starts[-1]:starts[-1] + len(ORDER)]
     lines = [f"ncu --set full --clock-control none (cold cache, one launch at a time) of the GEMM "
              f"launches of one CaffeNet b256 {math} step; report {os.path.basename(rep)}",
              f"{'layer':15s} {'pass':10s} {'kernel':28s} {'us':>7s} {'TF/s':>6s} {'DRAM MB':>8s} "

@@ -353,6 +353,7 @@ struct glp_plan_s {
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
   int allow_hfwd = 1;  // GLP_HFWD=0: im2col forward for space-to-depth layers (A/B runs)
   int allow_fdy = 1;   // GLP_HALO_FDY=0: halo filter gradient on the packed dy (A/B runs)
+  int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -514,7 +515,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     // CTA pairs split the MN-major B tile into halves of whole swizzle atoms: when the 128-byte
     // atom (64 bf16) does not divide bn/2 but the 64-byte one does (C_o = 384 -> bn 192), use
     // 64-byte rows so the pair still forms
-    const int bnw = choose_bn(d.Co);
+    const int bnw = P.wgrad_bn > 0 ? P.wgrad_bn : choose_bn(d.Co);
     if (pp.a_tma && elem == 2 && P.wgrad_cg2 && pp.krow == 128 && (bnw / 2) % 64 != 0 &&
         (bnw / 2) % 32 == 0 && (long long)tapsx * Cpx > 128)
       pp.krow = 64;
@@ -541,7 +542,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
     pp.Ng = d.Co;
     pp.Kpad = d.N * d.Ho * d.Wo;
     pp.kb_total = (int)cdiv(pp.Kpad, BKP);
-    pp.bn = choose_bn(d.Co);
+    pp.bn = P.wgrad_bn > 0 ? P.wgrad_bn : choose_bn(d.Co);
     pp.bn_smem = (int)rup(pp.bn, EPA);
   }
   pp.m_tiles = (int)cdiv(pp.M, 128);
@@ -1423,6 +1424,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
+  if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));

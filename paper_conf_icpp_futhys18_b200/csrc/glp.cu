@@ -865,6 +865,14 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
   if (P.s2d && P.s2d * P.s2d * d.C <= S2DW_MAXC && P.Cpx <= S2DW_MAXC && !P.s2d_block) {
     const long long px = (long long)d.N * P.dxg.H * P.dxg.W;
     const dim3 grid((unsigned)cdiv(px, 128));
+    if (P.s2d == 4 && d.C == 3) {   // CaffeNet conv1: compile-time geometry
+      if (P.elem == 2)
+        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<2, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      else
+        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<4, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      GLP_LAUNCH_CHECK("pack_s2d_warp_t");
+      return GLP_OK;
+    }
     if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<2>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
     else

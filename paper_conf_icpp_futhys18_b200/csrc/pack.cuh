@@ -432,6 +432,85 @@ __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x
   }
 }
 
+// Compile-time (S, C) form of pack_s2d_warp (CaffeNet conv1: S = 4, C = 3): the generic kernel
+// was issue-bound (ncu: stall not_selected / math / wait, 69 M instructions for 264 MB) on its
+// per-channel counter and bounds logic; here one row pointer per (dh, c), one column test per dw,
+// and the loop fully unrolled.
+template <int ELEM, int S, int C>
+__global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__ x, void *__restrict__ dst,
+                                                       int N, int H, int W, int P, int Hs, int Ws,
+                                                       int Cps, int src_c) {
+  constexpr int NC = S * S * C;
+  constexpr int RB = S2DW_MAXC * ELEM + 16;
+  __shared__ __align__(16) uint8_t slab[4][32 * RB];
+  pdl_launch_dependents();
+  pdl_wait();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long total = (long long)N * Hs * Ws;
+  const long long q0 = ((long long)blockIdx.x * 4 + warp) * 32;
+  if (q0 >= total) return;
+  const long long q = q0 + lane;
+  const bool ok = q < total;
+  int n = 0, hs = 0, ws = 0;
+  if (ok) {
+    n = (int)(q / ((long long)Hs * Ws));
+    const int r = (int)(q - (long long)n * Hs * Ws);
+    hs = r / Ws;
+    ws = r - hs * Ws;
+  }
+  const float *xb = x + (size_t)n * src_c * H * W;
+  float v[NC];
+  bool cok[S];
+#pragma unroll
+  for (int dw = 0; dw < S; ++dw) {
+    const int iw = S * ws + dw - P;
+    cok[dw] = iw >= 0 && iw < W;
+  }
+#pragma unroll
+  for (int dh = 0; dh < S; ++dh) {
+    const int ih = S * hs + dh - P;
+    const bool rok = ok && ih >= 0 && ih < H;
+#pragma unroll
+    for (int c = 0; c < C; ++c) {
+      const float *row = xb + ((size_t)c * H + (rok ? ih : 0)) * W + (S * ws - P);
+#pragma unroll
+      for (int dw = 0; dw < S; ++dw)
+        v[(dh * S + dw) * C + c] = (rok && cok[dw]) ? __ldg(row + dw) : 0.f;
+    }
+  }
+  uint8_t *rowp = slab[warp] + lane * RB;
+#pragma unroll
+  for (int j = 0; j < S2DW_MAXC; j += 8) {
+    if (j >= Cps) break;
+    float u[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) u[k] = (j + k < NC) ? v[(j + k < NC) ? j + k : 0] : 0.f;
+    if (ELEM == 2) {
+      __nv_bfloat162 a = __floats2bfloat162_rn(u[0], u[1]), b = __floats2bfloat162_rn(u[2], u[3]);
+      __nv_bfloat162 cq = __floats2bfloat162_rn(u[4], u[5]), d = __floats2bfloat162_rn(u[6], u[7]);
+      *reinterpret_cast<uint4 *>(rowp + j * 2) =
+          make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
+                     *reinterpret_cast<uint32_t *>(&cq), *reinterpret_cast<uint32_t *>(&d));
+    } else {
+      *reinterpret_cast<uint4 *>(rowp + j * 4) =
+          make_uint4(f32_to_tf32_rna(u[0]), f32_to_tf32_rna(u[1]), f32_to_tf32_rna(u[2]),
+                     f32_to_tf32_rna(u[3]));
+      *reinterpret_cast<uint4 *>(rowp + j * 4 + 16) =
+          make_uint4(f32_to_tf32_rna(u[4]), f32_to_tf32_rna(u[5]), f32_to_tf32_rna(u[6]),
+                     f32_to_tf32_rna(u[7]));
+    }
+  }
+  __syncwarp();
+  const int cpr = Cps * ELEM / 16;
+  uint8_t *out = static_cast<uint8_t *>(dst) + (size_t)q0 * Cps * ELEM;
+  const int nrows = (int)min(32LL, total - q0);
+  for (int k = lane; k < nrows * cpr; k += 32) {
+    const int r = k / cpr, ch = k - r * cpr;
+    *reinterpret_cast<uint4 *>(out + (size_t)k * 16) =
+        *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+  }
+}
+
 // Forward B operand in the space-to-depth geometry: Wp[co][t'*Cps + c'], t' = kh'*Ks + kw',
 // c' = (dh*S + dw)*C + c, value W[co][c][S*kh'+dh][S*kw'+dw] (0 past the K x K window).
 template <int ELEM>

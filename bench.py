@@ -237,7 +237,12 @@ class LayerState:
                         lg.dw(idx), lg.db(idx)) for j, lg in enumerate(leaf_grads)]
 
     def launches(self):
+        """Kernels this unit launches per timed step: pack x, W pack(s), fwd GEMM, dy pack, dgrad
+        GEMM, filter-gradient GEMM, dW and db reductions; a fused-dy plan (data-fed halo layer)
+        launches no dy pack."""
         base = 9 if self.dx is not None else 7
+        if self.dx is None and self.conv.info.wgrad_fused_dy:
+            base -= 1
         return base if self.leaves is None else base - 4 + 6 * len(self.leaves)
 
     # the step's kernel groups (one C call each; see step())

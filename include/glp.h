@@ -164,7 +164,8 @@ typedef enum {
   GLP_PACK_DY = 1,         /* dy NCHW fp32 -> packed NHWC operand                              */
   GLP_PACK_DY_DB = 2,      /* as GLP_PACK_DY, plus the fixed-order partial sums of db          */
   GLP_PACK_W_FWD = 3,      /* W -> forward B operand [C_o][(kh,kw,ci)]                         */
-  GLP_PACK_W_BWD_DATA = 4  /* W -> backward-data B operand [C_i][(kh,kw,co)]                   */
+  GLP_PACK_W_BWD_DATA = 4, /* W -> backward-data B operand [C_i][(kh,kw,co)]                   */
+  GLP_PACK_W_BOTH = 5      /* both weight operands in one pass over W (same bits as 3 + 4)       */
 } glp_pack_t;
 glp_status_t glp_stage_pack(glp_plan_t plan, glp_pack_t what, const float *src, void *ws,
                             size_t ws_bytes, glp_stream_t stream);

@@ -924,6 +924,32 @@ glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStr
   return GLP_OK;
 }
 
+// Both weight operands in one kernel (single layers without space-to-depth, taps <= 25); the
+// separate packs otherwise.  Same operand bits either way.
+glp_status_t run_pack_w_both(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  if (P.s2d || w.n > 1 || P.taps > PWB_MAXT) {
+    glp_status_t s = run_pack_w_fwd(P, w, ws, st);
+    return s ? s : run_pack_w_dgrad(P, w, ws, st);
+  }
+  const size_t smem = (size_t)32 * (32 * P.taps + 1) * 4;
+  static bool attr_set[2] = {false, false};
+  void *fn = P.elem == 2 ? reinterpret_cast<void *>(pack_w_both<2>) : reinterpret_cast<void *>(pack_w_both<4>);
+  if (!attr_set[P.elem == 2]) {
+    GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 32 * (32 * PWB_MAXT + 1) * 4));
+    attr_set[P.elem == 2] = true;
+  }
+  const dim3 grid((unsigned)cdiv(std::max(P.Cpx, d.C), 32), (unsigned)cdiv(P.Cop, 32), 2);
+  void *wp = ws + P.off_wpk, *wt = ws + P.off_wtpk;
+  const int flip = P.dgrad.a_tma;
+  if (P.elem == 2)
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<2>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip));
+  else
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<4>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip));
+  GLP_LAUNCH_CHECK("pack_w_both");
+  return GLP_OK;
+}
+
 // output table of a call: n = 1 -> every channel in p[0]; fused group -> the plan's branches
 BrOut br_out(const glp_plan_s &P, int n, float *const *ptrs) {
   BrOut t;
@@ -1752,7 +1778,7 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
   if (s) return s;
   if ((s = validate_ptrs({src}))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (what < GLP_PACK_X || what > GLP_PACK_W_BWD_DATA) return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
+  if (what < GLP_PACK_X || what > GLP_PACK_W_BOTH) return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
     uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
@@ -1767,6 +1793,7 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
         break;
       case GLP_PACK_W_FWD: s = run_pack_w_fwd(*P, br_in1(src + o.w), wsb, st); break;
       case GLP_PACK_W_BWD_DATA: s = run_pack_w_dgrad(*P, br_in1(src + o.w), wsb, st); break;
+      case GLP_PACK_W_BOTH: s = run_pack_w_both(*P, br_in1(src + o.w), wsb, st); break;
     }
     if (s) return s;
   }
@@ -1908,6 +1935,7 @@ glp_status_t glp_stage_pack_group(glp_plan_t P, glp_pack_t what, const float *co
     case GLP_PACK_DY_DB: return launch_pack_dy(*P, t, wsb, true, st);
     case GLP_PACK_W_FWD: return run_pack_w_fwd(*P, t, wsb, st);
     case GLP_PACK_W_BWD_DATA: return run_pack_w_dgrad(*P, t, wsb, st);
+    case GLP_PACK_W_BOTH: return run_pack_w_both(*P, t, wsb, st);
     default: break;
   }
   return fail(GLP_ERR_INVALID_VALUE, "unknown pack kind");

@@ -619,4 +619,58 @@ __global__ void __launch_bounds__(256) pack_w_dgrad_rows(const float *__restrict
   }
 }
 
+// Both weight operands in one pass over W (GLP_PACK_W_BOTH): block (ci tile of 32, co tile of 32)
+// stages W[co][ci][0..taps) for its 32 x 32 (co, ci) pairs (each co contributes one contiguous run
+// of 32*taps floats: coalesced), then writes the forward operand Wp[co][t*Cp + ci] (32 consecutive
+// ci per (co, t)) and the backward-data operand Wt[ci][t'*Cop + co] (32 consecutive co per (ci, t),
+// t' = taps-1-t when flipped).  Tiles cover ci < Cp and co < Cop, so the channel padding is written
+// as zeros here; blockIdx.z == 1 zero-fills the K tails past taps*Cp / taps*Cop.  Values are the
+// same rounding of the same fp32 as the separate packs (bitwise identical operands).
+constexpr int PWB_MAXT = 25;   // taps (<= 5x5) that fit the stage: 32 x (32*25 + 1) floats = 100 KB
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_w_both(const float *__restrict__ w, void *__restrict__ wp,
+                                                   void *__restrict__ wt, int Co, int C, int taps,
+                                                   int Cp, int Cop, int Kpf, int Kpd, int flip) {
+  extern __shared__ float stg[];   // [32 co][32*taps + 1]
+  pdl_launch_dependents();
+  pdl_wait();
+  const int ld = 32 * taps + 1;
+  const int ci0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
+  if (blockIdx.z == 1) {   // K tails (t >= taps) of both operands
+    for (int i = threadIdx.x; i < 32 * (Kpf - taps * Cp); i += 256) {
+      const int r = i / (Kpf - taps * Cp), k = taps * Cp + i % (Kpf - taps * Cp);
+      if (blockIdx.x == 0 && co0 + r < Co) PackOut<ELEM>::store1(wp, (size_t)(co0 + r) * Kpf + k, 0.f);
+    }
+    for (int i = threadIdx.x; i < 32 * (Kpd - taps * Cop); i += 256) {
+      const int r = i / (Kpd - taps * Cop), k = taps * Cop + i % (Kpd - taps * Cop);
+      if (blockIdx.y == 0 && ci0 + r < C) PackOut<ELEM>::store1(wt, (size_t)(ci0 + r) * Kpd + k, 0.f);
+    }
+    return;
+  }
+  const int run = 32 * taps;
+  for (int i = threadIdx.x; i < 32 * run; i += 256) {
+    const int r = i / run, e = i - r * run;   // co row r, element e = ci_l*taps + t
+    const int co = co0 + r, ci = ci0 + e / taps;
+    stg[r * ld + e] = (co < Co && ci < C) ? __ldg(w + ((size_t)co * C + ci) * taps + (e % taps)) : 0.f;
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wr = threadIdx.x >> 5;
+  // forward: rows co (< Co), for each t: 32 consecutive ci (lane)
+  for (int r = wr; r < 32; r += 8) {
+    const int co = co0 + r;
+    if (co >= Co || ci0 + lane >= Cp) continue;
+    for (int t = 0; t < taps; ++t)
+      PackOut<ELEM>::store1(wp, (size_t)co * Kpf + (size_t)t * Cp + ci0 + lane, stg[r * ld + lane * taps + t]);
+  }
+  // backward-data: rows ci (< C), for each t: 32 consecutive co (lane); padding co >= Co -> 0
+  for (int c = wr; c < 32; c += 8) {
+    const int ci = ci0 + c;
+    if (ci >= C || co0 + lane >= Cop) continue;
+    for (int t = 0; t < taps; ++t) {
+      const int tt = flip ? taps - 1 - t : t;
+      PackOut<ELEM>::store1(wt, (size_t)ci * Kpd + (size_t)tt * Cop + co0 + lane, stg[lane * ld + c * taps + t]);
+    }
+  }
+}
+
 }  // namespace glp

@@ -605,3 +605,32 @@ def test_tree_exchange_bitwise_invariant_emulated_ranks():
             np.testing.assert_array_equal(ref, full.astype(np.float32))
         else:
             assert np.abs(ref - full).max() / np.abs(full).max() <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[4], SHAPES[5], SHAPES[6], SHAPES[1], SHAPES[9]],
+                         ids=lambda s: s[0])
+def test_pack_w_both_equals_separate(shape, math):
+    """GLP_PACK_W_BOTH (both weight operands from one pass over W) writes the same operand bits
+    as GLP_PACK_W_FWD + GLP_PACK_W_BWD_DATA: the staged forward and backward-data outputs are
+    bitwise equal (channel padding C, C_o % 32 != 0, 1x1 / 3x3 / 5x5 taps)."""
+    d = _data(shape, seed=51)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    outs = []
+    for both in (False, True):
+        layer = _layer(shape, math)
+        y = torch.empty(layer.y_shape, device=DEV)
+        dx = torch.empty(layer.x_shape, device=DEV)
+        layer.stage_pack(glp.GLP_PACK_X, t["x"])
+        if both:
+            layer.stage_pack(glp.GLP_PACK_W_BOTH, t["w"])
+        else:
+            layer.stage_pack(glp.GLP_PACK_W_FWD, t["w"])
+            layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
+        layer.stage_fwd(t["b"], y)
+        layer.stage_pack(glp.GLP_PACK_DY, t["dy"])
+        layer.stage_bwd_data(dx)
+        torch.cuda.synchronize()
+        outs.append((y.cpu().numpy(), dx.cpu().numpy()))
+    np.testing.assert_array_equal(outs[1][0], outs[0][0])
+    np.testing.assert_array_equal(outs[1][1], outs[0][1])

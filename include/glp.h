@@ -82,6 +82,8 @@ typedef struct {
                             dy itself: glp_stage_pack(GLP_PACK_DY*) then only records the dy
                             pointer for this workspace (it must stay valid until the filter-gradient
                             and backward-data stages have run; the backward-data stage packs it) */
+  int dgrad_halo;        /* 1: backward-data by the shared-halo kernel (unit stride: a 4-D TMA halo
+                            of the packed dy per 64-channel block, tap operands by row shift)     */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

@@ -24,6 +24,7 @@
 #include "common.cuh"
 #include "hwgrad.cuh"
 #include "hfwd.cuh"
+#include "hdgrad.cuh"
 #include "igemm.cuh"
 #include "pack.cuh"
 #include "simt.cuh"
@@ -332,6 +333,9 @@ struct glp_plan_s {
   // halo forward (hfwd.cuh) for the same space-to-depth layers: x' staged once per tile for all
   // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
   int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
+  int hdg = 0;         // halo backward-data (hdgrad.cuh) for unit-stride layers where it pays
+  HdgradParams hd{};
+  int hd_grid = 0, hd_smem = 0;
   int hfwd = 0;
   HfwdParams hf{};
   int hf_grid = 0, hf_smem = 0, hf_regs = 0;
@@ -353,6 +357,7 @@ struct glp_plan_s {
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
   int allow_hfwd = 1;  // GLP_HFWD=0: im2col forward for space-to-depth layers (A/B runs)
   int allow_fdy = 1;   // GLP_HALO_FDY=0: halo filter gradient on the packed dy (A/B runs)
+  int allow_hdg = 1;   // GLP_HDGRAD=0: im2col backward-data everywhere (A/B runs); 2 = force where legal
   int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
@@ -439,6 +444,70 @@ glp_status_t plan_halo(glp_plan_s &P) {
   P.hw_regs = fa.numRegs;
   P.halo = 1;
   P.halo_fdy = ncg;
+  return GLP_OK;
+}
+
+// Halo backward-data (hdgrad.cuh): unit stride, square kernel, bf16, the flipped-tap Wt of the
+// im2col-TMA dgrad, 64-channel blocks of C_o, and a tile geometry (R output rows padded to a pitch
+// of WQ >= W + K - 1 pixels, R*WQ = 128) that wastes at most 30 % of the rows.  Used when the
+// im2col A traffic dominates: >= 9 taps and C_i <= 128 (each A byte feeds few columns).
+glp_status_t plan_hdgrad(glp_plan_s &P) {
+  P.hdg = 0;
+  const glp_conv_desc_s &d = P.d;
+  if (!P.allow_hdg || P.elem != 2 || d.nbr > 1 || d.Sh != 1 || d.Sw != 1 || d.Kh != d.Kw ||
+      d.Ph != d.Pw || d.Ph > d.Kh - 1 || !P.dgrad.a_tma || P.Cop % 64 != 0)
+    return GLP_OK;
+  const int K = d.Kh, taps = K * K;
+  int WQ = 8;
+  while (WQ < d.W + K - 1) WQ *= 2;
+  if (WQ > 128) return GLP_OK;
+  const int R = 128 / WQ;
+  const int tiles_img = (int)cdiv(d.H, R);
+  const double junk = (double)tiles_img * R * WQ / ((double)d.H * d.W);
+  const int bn = (int)rup(d.C, 16);
+  if (P.allow_hdg != 2 && (junk > 1.3 || taps < 9 || bn > 128)) return GLP_OK;
+  if (bn > 256 || (bn / 2) % 16 != 0) return GLP_OK;   // CTA pairs: half of B per CTA, N % 32
+  HdgradParams &h = P.hd;
+  memset(&h, 0, sizeof(h));
+  h.K = K;
+  h.Q = K - 1 - d.Ph;
+  h.WQ = WQ;
+  h.R = R;
+  h.H = d.H;
+  h.W = d.W;
+  h.Ho = d.Ho;
+  h.Wo = d.Wo;
+  h.N = d.N;
+  h.tiles_img = tiles_img;
+  h.units = (int)cdiv((long long)d.N * tiles_img, 2);
+  h.ncb = P.Cop / 64;
+  h.cop = P.Cop;
+  h.bn = bn;
+  h.ci = d.C;
+  h.acc_cols = (int)rup(bn, 32);
+  int tc = 32;
+  while (tc < 2 * h.acc_cols) tc *= 2;
+  h.tmem_cols = tc;
+  h.a_bytes = (int)rup((long long)(R + K - 1) * WQ * 128, 1024);
+  h.b_tap_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
+  h.a_stages = 3;
+  const int fixed = 1024 + h.a_stages * h.a_bytes + 8 * 64 + 16;
+  // as many taps per B stage as keep >= 4 stages (the issuer's barrier round trip costs more than
+  // the 8 MMAs of one tap)
+  h.b_taps = 1;
+  while (h.b_taps < taps && (P.smem_cap - fixed) / ((h.b_taps + 1) * h.b_tap_bytes) >= 4) ++h.b_taps;
+  h.b_bytes = h.b_taps * h.b_tap_bytes;
+  h.b_stages = std::min(8, (P.smem_cap - fixed) / h.b_bytes);
+  if (h.b_stages < 3) return GLP_OK;
+  P.hd_smem = 1024 + h.a_stages * h.a_bytes + h.b_stages * h.b_bytes +
+              8 * (2 * h.a_stages + 2 * h.b_stages + 4) + 16;
+  long long pairs = std::min<long long>(h.units, P.sm_count / 2);
+  if (P.s_override > 0)
+    pairs = std::max(1LL, std::min(pairs, cdiv((long long)P.s_override * tiles_img, 2)));
+  P.hd_grid = (int)(2 * pairs);
+  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hdgrad_kernel),
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  P.hdg = 1;
   return GLP_OK;
 }
 
@@ -933,12 +1002,9 @@ glp_status_t run_pack_w_both(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStre
     return s ? s : run_pack_w_dgrad(P, w, ws, st);
   }
   const size_t smem = (size_t)32 * (32 * P.taps + 1) * 4;
-  static bool attr_set[2] = {false, false};
+  // the attribute is per device: set on every call (a host-side driver call, no launch)
   void *fn = P.elem == 2 ? reinterpret_cast<void *>(pack_w_both<2>) : reinterpret_cast<void *>(pack_w_both<4>);
-  if (!attr_set[P.elem == 2]) {
-    GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 32 * (32 * PWB_MAXT + 1) * 4));
-    attr_set[P.elem == 2] = true;
-  }
+  GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 32 * (32 * PWB_MAXT + 1) * 4));
   const dim3 grid((unsigned)cdiv(std::max(P.Cpx, d.C), 32), (unsigned)cdiv(P.Cop, 32), 2);
   void *wp = ws + P.off_wpk, *wt = ws + P.off_wtpk;
   const int flip = P.dgrad.a_tma;
@@ -1072,7 +1138,58 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);
 }
 
+glp_status_t encode_4d_nhwc(CUtensorMap *map, const void *ptr, int cpitch, int W, int H, int N,
+                            uint32_t box_w, uint32_t box_h) {
+  cuuint64_t dims[4] = {(cuuint64_t)cpitch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+  cuuint64_t strides[3] = {(cuuint64_t)cpitch * 2, (cuuint64_t)W * cpitch * 2,
+                           (cuuint64_t)H * W * cpitch * 2};
+  cuuint32_t box[4] = {64u, box_w, box_h, 1u};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void *>(ptr), dims,
+                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled (4d) failed (" + std::to_string((int)r) + ")");
+  return GLP_OK;
+}
+
+glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
+  const glp_conv_desc_s &d = P.d;
+  CUtensorMap mapDy, mapW;
+  glp_status_t s = cached_maps(P, 1, ws, mapDy, mapW, [&](CUtensorMap &Dy, CUtensorMap &Wm) {
+    glp_status_t r = encode_4d_nhwc(&Dy, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
+                                    (uint32_t)P.hd.WQ, (uint32_t)(P.hd.R + P.hd.K - 1));
+    if (r) return r;
+    return encode_2d(&Wm, 2, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
+                     (uint64_t)P.dgrad.Kpad * 2, 64u, (uint32_t)(P.hd.bn / 2), CU_TENSOR_MAP_SWIZZLE_128B);
+  });
+  if (s) return s;
+  HdgradParams p = P.hd;
+  p.out = dx;
+  p.out_c = P.x_img_c;
+  p.dbg_skip = P.dbg_skip;
+  cudaLaunchConfig_t cfg;
+  memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3((unsigned)P.hd_grid);
+  cfg.blockDim = dim3(HD_THREADS);
+  cfg.dynamicSmemBytes = (size_t)P.hd_smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = P.pdl ? 2 : 1;
+  void *args[] = {&p, &mapDy, &mapW};
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hdgrad_kernel), args));
+  GLP_LAUNCH_CHECK("hdgrad_kernel");
+  return GLP_OK;
+}
+
 glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
+  if (P.hdg) return run_dgrad_halo(P, dx, ws, st);
   const glp_conv_desc_s &d = P.d;
   const PassPlan &pp = P.dgrad;
   void *wtpk = ws + P.off_wtpk;
@@ -1458,6 +1575,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
+  if (const char *e = getenv("GLP_HDGRAD")) P->allow_hdg = atoi(e);
   if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
@@ -1524,7 +1642,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
       if (cur != device) cudaSetDevice(cur);
       return s;
     }
-    if ((s = plan_halo(*P)) || (s = plan_hfwd(*P))) {
+    if ((s = plan_halo(*P)) || (s = plan_hfwd(*P)) || (s = plan_hdgrad(*P))) {
       delete P;
       if (cur != device) cudaSetDevice(cur);
       return s;
@@ -1608,6 +1726,13 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->wgrad_halo = P->halo;
   I->fwd_halo = P->hfwd;
   I->wgrad_fused_dy = P->halo_fdy ? 1 : 0;
+  I->dgrad_halo = P->hdg;
+  if (P->hdg) {
+    I->grid_bwd_data = P->hd_grid;
+    I->tile_n_bwd_data = P->hd.bn;
+    I->stages_bwd_data = P->hd.b_stages;
+    I->tiles_bwd_data = P->hd.units;
+  }
   if (P->hfwd) {
     I->grid_fwd = P->hf_grid;
     I->tile_n_fwd = P->hf.bn;

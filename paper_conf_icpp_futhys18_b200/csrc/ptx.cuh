@@ -151,6 +151,23 @@ __device__ __forceinline__ void tma_load_2d_e(uint32_t dst, const CUtensorMap *m
                "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
                : "memory");
 }
+// 4-D tiled load (coordinates may be negative / past the end: out-of-bounds elements are zero)
+__device__ __forceinline__ void tma_load_4d_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                              int c0, int c1, int c2, int c3) {
+  asm volatile(GLP_ELECT
+               "@P_e cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+               " [%0], [%1, {%3, %4, %5, %6}], [%2];\n\t}" ::"r"(dst),
+               "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_4d_cg2_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                                  int c0, int c1, int c2, int c3) {
+  asm volatile(GLP_ELECT
+               "@P_e cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+               " [%0], [%1, {%3, %4, %5, %6}], [%2];\n\t}" ::"r"(dst),
+               "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
 __device__ __forceinline__ void tma_load_im2col_4d_e(uint32_t dst, const CUtensorMap *map,
                                                      uint32_t bar, int c, int w, int h, int n,
                                                      uint16_t off_w, uint16_t off_h) {

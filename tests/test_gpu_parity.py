@@ -634,3 +634,45 @@ def test_pack_w_both_equals_separate(shape, math):
         outs.append((y.cpu().numpy(), dx.cpu().numpy()))
     np.testing.assert_array_equal(outs[1][0], outs[0][0])
     np.testing.assert_array_equal(outs[1][1], outs[0][1])
+
+
+# unit-stride layers for the shared-halo backward-data kernel (hdgrad.cuh); GLP_HDGRAD=2 forces it
+# where the cost model would keep the im2col kernel (small images waste more padded rows)
+HDG_SHAPES = [
+    ("caffenet_conv2_b2", 2, 96, 27, 27, 256, 5, 1, 2),     # the model's own choice; odd unit count
+    ("k3p1_ragged", 3, 64, 11, 13, 64, 3, 1, 1),            # 3 images x 2 tiles: ragged pair unit
+    ("k3p0", 2, 32, 10, 12, 64, 3, 1, 0),                   # dy smaller than dx: halo offset Q = 2
+    ("k5p1", 2, 32, 9, 9, 128, 5, 1, 1),                    # asymmetric halo (Q = 3)
+]
+
+
+@pytest.mark.parametrize("shape", HDG_SHAPES, ids=lambda s: s[0])
+def test_halo_dgrad(shape, monkeypatch):
+    """Shared-halo backward-data (4-D TMA halo of the packed dy per 64-channel block, flipped taps by
+    row shift, CTA pairs with M = 256 MMAs): bit-exact on integer data, within 1e-4
+    of the rounding-emulated oracle and 2e-2 of the fp64 oracle on random data, bitwise invariant
+    across samples-in-flight overrides."""
+    monkeypatch.setenv("GLP_HDGRAD", "2")
+    layer = _layer(shape, "bf16")
+    assert layer.info.dgrad_halo == 1
+    d = _data(shape, exact=True, seed=53)
+    got = _run(layer, d)
+    ref = _oracle(d, shape[7], shape[8])
+    np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32))
+    d = _data(shape, seed=54)
+    runs = [_run(_layer(shape, "bf16", S), d)["dx"] for S in (0, 1, 0)]
+    ref = _oracle(d, shape[7], shape[8])["dx"]
+    emu = _oracle(d, shape[7], shape[8], x=EMU["bf16"](d["x"]), w=EMU["bf16"](d["w"]),
+                  dy=EMU["bf16"](d["dy"]))["dx"]
+    assert np.abs(runs[0] - ref).max() / np.abs(ref).max() <= TOL["bf16"]
+    assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= 1e-4
+    for other in runs[1:]:
+        np.testing.assert_array_equal(other, runs[0])
+
+
+def test_halo_dgrad_model_choice():
+    """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) and
+    keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would be junk)."""
+    assert _layer(HDG_SHAPES[0], "bf16").info.dgrad_halo == 1
+    assert _layer(SHAPES[6], "bf16").info.dgrad_halo == 0
+    assert _layer(HDG_SHAPES[0], "tf32").info.dgrad_halo == 0

@@ -283,6 +283,21 @@ class LayerState:
         return self.host, self.t
 
 
+def kernel_name(states, rec):
+    """The library kernel that ran a unit's pass (from the plan info: halo forms where chosen)."""
+    for s in states:
+        if s.name != rec["layer"]:
+            continue
+        info = s.conv.info
+        if rec["pass"] == "fwd" and getattr(info, "fwd_halo", 0):
+            return "hfwd_kernel"
+        if rec["pass"] == "bwd_data" and getattr(info, "dgrad_halo", 0):
+            return "hdgrad_kernel"
+        if rec["pass"] == "bwd_filter" and getattr(info, "wgrad_halo", 0):
+            return "hwgrad_kernel"
+    return "igemm_kernel"
+
+
 def set_exact_data(states):
     """--exact-data: every unit's inputs replaced by the integer variant of its seeded draws."""
     import torch
@@ -716,7 +731,7 @@ def run_glp(args, ws, rank, local):
             traffic = None
     roofline = {"bound": "tensor", "achieved": dom["tflops"], "peak": round(peak_tf, 1),
                 "unit": "TFLOP/s", "frac": round(dom["tflops"] / peak_tf, 4), "traffic": traffic,
-                "kernel": f"igemm_kernel {dom['layer']} {dom['pass']}",
+                "kernel": f"{kernel_name(states, dom)} {dom['layer']} {dom['pass']}",
                 "peak_source": peaks["source"] + (" bf16 sustained" if args.math == "bf16"
                                                   else " bf16 sustained x 1.1/2.25 (tf32)"),
                 "share_of_step": round(dom["total_us"] / 1e3 / ms, 4),

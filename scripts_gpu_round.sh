@@ -17,7 +17,7 @@ timeout -s KILL 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dr
 echo "launch rc=$?"
 python tools/launch_table.py gpurun_out/launch_${TAGN}.csv 2>&1 | tail -50
 if [ -z "$NOFULL" ]; then
-  timeout -s KILL 1200 ncu --set full --clock-control none --import-source on -k "regex:igemm|hwgrad|hfwd" -s ${SKIP:-0} -c ${CNT:-30} \
+  timeout -s KILL 1200 ncu --set full --clock-control none --import-source on -k "regex:igemm|hwgrad|hfwd|hdgrad" -s ${SKIP:-0} -c ${CNT:-30} \
     -o gpurun_out/prof_${TAGN} -f python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e --no-graph --serial > gpurun_out/ncu_full_${TAGN}.log 2>&1
   echo "full rc=$?"; tail -3 gpurun_out/ncu_full_${TAGN}.log
 fi

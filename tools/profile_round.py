@@ -71,7 +71,7 @@ def main(rnd, rep, launches=None, workload=4, math="bf16"):
     flops = {l.name: l.flops_per_pass() for l in config(workload)}
     outdir = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(outdir, exist_ok=True)
-    rows = [d for d in raw_rows(rep) if any(k in d["Kernel Name"][1] for k in ("igemm", "hwgrad", "hfwd"))]
+    rows = [d for d in raw_rows(rep) if any(k in d["Kernel Name"][1] for k in ("igemm", "hwgrad", "hfwd", "hdgrad"))]
     # the capture may hold more than one step: take the last one that starts with conv1's forward
     starts = [i for i, d in enumerate(rows) if "hfwd" in d["Kernel Name"][1]]
     if starts and len(rows) - starts[-1] < len(ORDER):

@@ -232,13 +232,14 @@ int choose_bn(int n) {
 // two work units per slot (measured: for the large CaffeNet layers smaller tiles cost more in
 // A re-reads and per-k-block overhead than the last-round quantisation they save).  Below that,
 // time ~ rounds * (k-block MMA cycles ~ 2*bn, floored by the issue loop) picks the tile.
-void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, int &cg_out) {
+void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, int &cg_out,
+                    int min_units = 2) {
   const int bn0 = choose_bn(n);
   const int cg0 = cg2_ok ? 2 : 1;
   bn_out = bn0;
   cg_out = cg0;
   const long long units0 = cdiv(M, 128LL * cg0) * cdiv(n, bn0);
-  if (units0 >= 2LL * (sm_count / cg0)) return;
+  if (units0 >= (long long)min_units * (sm_count / cg0)) return;
   double best_c = 1e300;
   for (int cg = cg0; cg >= 1; --cg) {
     const long long m_units = cdiv(M, 128LL * cg);
@@ -359,6 +360,7 @@ struct glp_plan_s {
   int allow_fdy = 1;   // GLP_HALO_FDY=0: halo filter gradient on the packed dy (A/B runs)
   int allow_hdg = 1;   // GLP_HDGRAD=0: im2col backward-data everywhere (A/B runs); 2 = force where legal
   int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
+  int tile_units = 2;  // GLP_TILE_UNITS=u: fwd/dgrad tile model applies below u units per slot
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -622,7 +624,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const bool wg_cg2 = P.wgrad_cg2 && (pp.bn / 2) % EPA == 0;   // MN-major B halves: whole atoms
   if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && (mode != MODE_WGRAD || wg_cg2)) pp.cg = 2;
   if (mode != MODE_WGRAD && P.bn_model) {
-    choose_tile_mn(pp.Ng, pp.M, pp.cg == 2, P.sm_count, pp.bn, pp.cg);
+    choose_tile_mn(pp.Ng, pp.M, pp.cg == 2, P.sm_count, pp.bn, pp.cg, P.tile_units);
     pp.bn_smem = pp.bn;
   }
   if (pp.cg == 2) pp.bn_smem = pp.bn / 2;
@@ -1577,6 +1579,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
   if (const char *e = getenv("GLP_HDGRAD")) P->allow_hdg = atoi(e);
   if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
+  if (const char *e = getenv("GLP_TILE_UNITS")) P->tile_units = atoi(e);
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));

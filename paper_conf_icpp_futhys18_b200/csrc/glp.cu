@@ -526,7 +526,7 @@ glp_status_t plan_hfwd(glp_plan_s &P) {
   const int bn = (int)rup(x.Co, 16);
   const int shift_max = (Ks - 1) * x.W + (Ks - 1);
   const int halo_rows = 128 + shift_max;
-  if (bn > 256 || halo_rows > 256) return GLP_OK;
+  if (bn > 256 || (bn / 2) % 8 != 0 || halo_rows > 256) return GLP_OK;   // pairs: bn/2 per CTA
   HfwdParams &h = P.hf;
   memset(&h, 0, sizeof(h));
   h.taps = T;
@@ -539,7 +539,7 @@ glp_status_t plan_hfwd(glp_plan_s &P) {
   h.tmem_cols = tc;
   h.halo_rows = halo_rows;
   h.a_bytes = (int)rup((long long)halo_rows * 128, 1024);
-  h.b_tap_bytes = (int)rup((long long)bn * 128, 1024);
+  h.b_tap_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
   h.bias_floats = (int)rup(bn, 4);
   const int fixed = 1024 + T * h.b_tap_bytes + 16 + 16 + 4 * h.bias_floats + 8 * 8;
   h.stages = std::min(6, (P.smem_cap - fixed - 8 * 2 * 6) / h.a_bytes);
@@ -548,15 +548,16 @@ glp_status_t plan_hfwd(glp_plan_s &P) {
   if (rows >= (1LL << 31) - 256) return GLP_OK;
   h.rows = (int)rows;
   h.tiles = (int)cdiv(rows, 128);
+  h.units = (int)cdiv(h.tiles, 2);
   h.div_img = FastDiv((uint32_t)(x.H * x.W));
   h.div_w = FastDiv((uint32_t)x.W);
   h.ho = P.d.Ho;
   h.wo = P.d.Wo;
   P.hf_smem = fixed + 8 * (2 * h.stages + 6) + h.stages * h.a_bytes;
-  long long grid = std::min<long long>(h.tiles, P.sm_count);
+  long long pairs = std::min<long long>(h.units, P.sm_count / 2);
   if (P.s_override > 0)   // test override: only the tiles of S samples in flight at once
-    grid = std::max(1LL, std::min(grid, cdiv((long long)P.s_override * x.H * x.W, 128)));
-  P.hf_grid = (int)grid;
+    pairs = std::max(1LL, std::min(pairs, cdiv((long long)P.s_override * x.H * x.W, 256)));
+  P.hf_grid = (int)(2 * pairs);
   GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hfwd_kernel),
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
@@ -1085,7 +1086,7 @@ glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
                                64u, (uint32_t)P.hf.halo_rows, CU_TENSOR_MAP_SWIZZLE_128B);
     if (r) return r;
     return encode_2d(&Wm, 2, ws + P.off_wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co,
-                     (uint64_t)P.fwd.Kpad * 2, 64u, (uint32_t)P.hf.bn, CU_TENSOR_MAP_SWIZZLE_128B);
+                     (uint64_t)P.fwd.Kpad * 2, 64u, (uint32_t)(P.hf.bn / 2), CU_TENSOR_MAP_SWIZZLE_128B);
   });
   if (s) return s;
   HfwdParams p = P.hf;
@@ -1100,11 +1101,15 @@ glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   cfg.blockDim = dim3(HF_THREADS);
   cfg.dynamicSmemBytes = (size_t)P.hf_smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = P.pdl ? 1 : 0;
+  cfg.numAttrs = P.pdl ? 2 : 1;
   void *args[] = {&p, &mapX, &mapW};
   GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hfwd_kernel), args));
   GLP_LAUNCH_CHECK("hfwd_kernel");
@@ -1740,7 +1745,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
     I->grid_fwd = P->hf_grid;
     I->tile_n_fwd = P->hf.bn;
     I->stages_fwd = P->hf.stages;
-    I->tiles_fwd = P->hf.tiles;
+    I->tiles_fwd = P->hf.units;
   }
   return GLP_OK;
 }

@@ -15,9 +15,13 @@
 // per CTA and stays resident.  L2 reads per tile: ~31 KB instead of ~200 KB.  Rows of the padded
 // grid outside H_o x W_o are computed and dropped (CaffeNet conv1: 57^2 / 55^2 = 7 % extra MMA).
 //
-// Persistent: tile t -> CTA t mod grid (the paper's round-robin dispatch, P171).  CTA = 192
-// threads: warps 0-3 epilogue (TMEM -> bias -> NCHW fp32), warp 4 TMA producer, warp 5 TMEM
-// owner + MMA issuer; two TMEM accumulators so the epilogue of tile i overlaps tile i+1.
+// CTA pairs (cluster of 2, tcgen05.mma.cta_group::2, M = 256): pair unit u covers tiles 2u and
+// 2u + 1, one per CTA; each CTA keeps half of W' (bn/2 rows per tap) resident and stages its own
+// tile's halo; the leader issues the MMAs for both (a single CTA ran M = 128, N = 96 MMAs at ~80
+// cycles against ~56 per SM for the pair).  Persistent: unit u -> pair u mod (grid/2) (the paper's
+// round-robin dispatch, P171).  CTA = 192 threads: warps 0-3 epilogue (TMEM -> bias -> NCHW fp32),
+// warp 4 TMA producer, warp 5 TMEM owner + MMA issuer (leader); two TMEM accumulators so the
+// epilogue of unit i overlaps unit i+1.
 #pragma once
 #include "common.cuh"
 #include "ptx.cuh"
@@ -36,9 +40,10 @@ struct HfwdParams {
   int tmem_cols;           // allocation (power of two >= 2 * acc_cols)
   int halo_rows;           // 128 + max shift
   int a_bytes;             // one halo stage (1024-aligned)
-  int b_tap_bytes;         // one tap's B block: bn rows x 128 B (1024-aligned)
+  int b_tap_bytes;         // one tap's B block of this CTA: bn/2 rows x 128 B (1024-aligned)
   int stages;
   int tiles;               // ceil(rows / 128)
+  int units;               // ceil(tiles / 2): CTA-pair work units
   int rows;                // N * H' * W'
   FastDiv div_img, div_w;  // H' * W', W'
   int ho, wo;              // valid output region of each H' x W' image
@@ -71,60 +76,69 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
       reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
   const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0);
   const int lane = threadIdx.x & 31;
+  const uint32_t rank = blockIdx.x & 1u;   // CTA in the pair
+  const bool leader = rank == 0;
   if (threadIdx.x == 0) {
+    // full / bfull: armed by the leader only (both CTAs' bytes); empty / tfull: one multicast
+    // commit; tempty: the 8 epilogue warps of both CTAs arrive on the leader's barrier
     for (int s = 0; s < S_; ++s) {
       mbar_init(full(s), 1);
       mbar_init(empty(s), 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(tfull(a), 1);
-      mbar_init(tempty(a), 4);
+      mbar_init(tempty(a), 8);
     }
     mbar_init(bfull, 1);
     fence_mbar_init();
   }
   if (warp == 5) {
-    tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
-    tmem_relinquish();
+    tmem_alloc_cg<2>(tmem_slot, (uint32_t)p.tmem_cols);
+    tmem_relinquish_cg<2>();
   }
   if (warp == 4 && lane == 0) {
     tma_prefetch(&tmapX);
     tma_prefetch(&tmapW);
   }
   tc_fence_before();
-  __syncthreads();
+  cluster_sync();
   tc_fence_after();
   pdl_wait();
   const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);
+  const int unit0 = (int)(blockIdx.x >> 1), ustep = (int)(gridDim.x >> 1);
 
   if (warp == 4) {
     // ===================================== producer ========================================
-    // B once: tap t's K slice [t*64, t*64 + 64) of W' (bn rows, rows >= C_o zero-filled)
-    mbar_arrive_expect_tx_e(bfull, (uint32_t)(p.taps * p.bn * 128));
+    // B once: this CTA's half (rows rank*bn/2 ...) of tap t's K slice [t*64, t*64 + 64) of W'
+    // (rows >= C_o zero-filled); completes on the leader's barrier
+    const int half = p.bn / 2;
+    if (leader) mbar_arrive_expect_tx_e(bfull, (uint32_t)(2 * p.taps * half * 128));
     for (int t = 0; t < p.taps; ++t)
-      tma_load_2d_e(sB + (uint32_t)(t * p.b_tap_bytes), &tmapW, bfull, t * 64, 0);
+      tma_load_2d_cg2_e(sB + (uint32_t)(t * p.b_tap_bytes), &tmapW, mapa_shared(bfull, 0), t * 64,
+                        (int)rank * half);
     const bool la = !(p.dbg_skip & 1);
-    const uint32_t tx = la ? (uint32_t)(p.halo_rows * 128) : 0u;
+    const uint32_t tx = la ? (uint32_t)(2 * p.halo_rows * 128) : 0u;
     int rs = 0;
     uint32_t rph = 0;
-    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
+    for (int u = unit0; u < p.units; u += ustep) {
+      const int tile = 2 * u + (int)rank;   // past the last tile: rows past the end -> zeros
       mbar_wait(empty(rs), rph ^ 1u);
       const uint32_t sA = sA0 + (uint32_t)(rs * p.a_bytes);
-      mbar_arrive_expect_tx_e(full(rs), tx);
-      if (la) tma_load_2d_e(sA, &tmapX, full(rs), 0, tile * 128);   // rows past the end: zeros
+      if (leader) mbar_arrive_expect_tx_e(full(rs), tx);
+      if (la) tma_load_2d_cg2_e(sA, &tmapX, mapa_shared(full(rs), 0), 0, tile * 128);
       if (++rs == S_) {
         rs = 0;
         rph ^= 1u;
       }
     }
-  } else if (warp == 5) {
+  } else if (warp == 5 && leader) {
     // ===================================== MMA issuer ======================================
-    const uint32_t idesc = make_idesc(1u, 0u, 0u, 128u, (uint32_t)p.bn);
+    const uint32_t idesc = make_idesc(1u, 0u, 0u, 256u, (uint32_t)p.bn);
     mbar_wait(bfull, 0);
     int rs = 0;
     uint32_t rph = 0, it = 0;
     const bool skip_mma = (p.dbg_skip & 4) != 0;
-    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x, ++it) {
+    for (int u = unit0; u < p.units; u += ustep, ++it) {
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
       mbar_wait(tempty(a), aph ^ 1u);
       tc_fence_after();
@@ -138,17 +152,17 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
         // advance the start by 32 bytes (2 descriptor units)
         const uint64_t da = make_sdesc(sA + (uint32_t)p.shift[t] * 128u, 16u, 1024u, 2u);
         const uint64_t db = make_sdesc(sB + (uint32_t)(t * p.b_tap_bytes), 16u, 1024u, 2u);
-        mma_kblock_e<0, 1, 4, 2>(d, da, db, idesc, t > 0 ? 1u : 0u);
+        mma_kblock_e<0, 2, 4, 2>(d, da, db, idesc, t > 0 ? 1u : 0u);
       }
-      mma_commit_e<1>(empty(rs));
-      mma_commit_e<1>(tfull(a));
+      mma_commit_e<2>(empty(rs));
+      mma_commit_e<2>(tfull(a));
       if (++rs == S_) {
         rs = 0;
         rph ^= 1u;
       }
     }
     __syncwarp();
-  } else {
+  } else if (warp < 4) {
     // ===================================== epilogue ========================================
     const int row = warp * 32 + lane;
     for (int i = row; i < p.bias_floats; i += 128)
@@ -156,10 +170,11 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
     named_bar_sync(1, 128);
     const size_t plane = (size_t)p.out_hw;
     uint32_t it = 0;
-    for (int tile = blockIdx.x; tile < p.tiles; tile += gridDim.x, ++it) {
+    for (int u = unit0; u < p.units; u += ustep, ++it) {
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
       mbar_wait(tfull(a), aph);
       tc_fence_after();
+      const int tile = 2 * u + (int)rank;
       const int q = tile * 128 + row;
       uint32_t n = 0, rem = 0, h = 0, w = 0;
       p.div_img.divmod((uint32_t)min(q, p.rows - 1), n, rem);
@@ -208,14 +223,14 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive_relaxed(tempty(a));
+      if (lane == 0) mbar_arrive_cluster_relaxed(mapa_shared(tempty(a), 0));
     }
   }
   pdl_launch_dependents();
   tc_fence_before();
-  __syncthreads();
+  cluster_sync();
   tc_fence_after();
-  if (warp == 5) tmem_dealloc(tmem_base, (uint32_t)p.tmem_cols);
+  if (warp == 5) tmem_dealloc_cg<2>(tmem_base, (uint32_t)p.tmem_cols);
 }
 
 }  // namespace glp

@@ -358,6 +358,7 @@ struct glp_plan_s {
   int allow_halo = 1;  // GLP_HALO=0: im2col filter gradient for space-to-depth layers (A/B runs)
   int allow_hfwd = 1;  // GLP_HFWD=0: im2col forward for space-to-depth layers (A/B runs)
   int allow_fdy = 1;   // GLP_HALO_FDY=0: halo filter gradient on the packed dy (A/B runs)
+  int fdy_ncg = 0;     // GLP_FDY_NCG=1|2|3: force the fused-dy builder variant (A/B runs)
   int allow_hdg = 1;   // GLP_HDGRAD=0: im2col backward-data everywhere (A/B runs); 2 = force where legal
   int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
   int tile_units = 2;  // GLP_TILE_UNITS=u: fwd/dgrad tile model applies below u units per slot
@@ -425,9 +426,22 @@ glp_status_t plan_halo(glp_plan_s &P) {
   h.ld = bn;
   // fused dy (single layers): the filter gradient builds its dy operand from the fp32 tensor
   const int fdy = (P.allow_fdy && P.d.nbr <= 1 && bn <= 128 && rows < (1LL << 31) - 256) ? 1 : 0;
-  // builder groups: 3 when a thread's channels fit 3 x 32 registers groups (C_o <= 96), else 2
-  const int ncg = fdy ? (bn <= 96 ? 3 : 2) : 0;
-  const int red_bytes = fdy ? 4 * ncg * 256 * 4 + 16 : 0;   // db partial staging
+  // builders: register-staged groups, 3 when a thread's channels fit 3 x 32 registers (C_o <= 96),
+  // else 2.  GLP_FDY_NCG=1 selects one group with a cp.async landing zone (2 x 128 pixels x bn
+  // fp32, which also holds the db staging afterwards; only 2 pipeline stages fit beside it):
+  // measured 171 us against 128 us for CaffeNet conv1.  GLP_FDY_NCG=2|3 forces the group count.
+  int ncg = 0;
+  int red_bytes = 0;
+  if (fdy) {
+    const int land = 2 * bn * 128 * 4 + 16;
+    if (P.fdy_ncg == 1 && (P.smem_cap - 2048 - land) / stage >= 2) {   // measured slower: opt-in
+      ncg = 1;
+      red_bytes = land;
+    } else {
+      ncg = P.fdy_ncg == 2 ? 2 : (P.fdy_ncg == 3 ? 3 : (bn <= 96 ? 3 : 2));
+      red_bytes = 4 * ncg * 256 * 4 + 16;
+    }
+  }
   h.stages = std::min(8, (P.smem_cap - 2048 - red_bytes) / stage);
   if (h.stages < 2) return GLP_OK;
   h.ho = P.d.Ho;
@@ -439,6 +453,7 @@ glp_status_t plan_halo(glp_plan_s &P) {
   P.hw_smem = 1024 + h.stages * stage + 8 * (2 * h.stages + 2) + 16 + red_bytes;
   const void *fn = ncg == 3 ? reinterpret_cast<const void *>(hwgrad_kernel<3>)
                  : ncg == 2 ? reinterpret_cast<const void *>(hwgrad_kernel<2>)
+                 : ncg == 1 ? reinterpret_cast<const void *>(hwgrad_kernel<1>)
                             : reinterpret_cast<const void *>(hwgrad_kernel<0>);
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
@@ -1261,6 +1276,7 @@ glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
   void *args[] = {&p, &mapX, &mapDy};
   GLP_CUDA(cudaLaunchKernelExC(&cfg, P.halo_fdy == 3 ? reinterpret_cast<void *>(hwgrad_kernel<3>)
                                 : P.halo_fdy == 2 ? reinterpret_cast<void *>(hwgrad_kernel<2>)
+                                : P.halo_fdy == 1 ? reinterpret_cast<void *>(hwgrad_kernel<1>)
                                                   : reinterpret_cast<void *>(hwgrad_kernel<0>),
                                 args));
   GLP_LAUNCH_CHECK("hwgrad_kernel");
@@ -1582,6 +1598,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
   if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
   if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
+  if (const char *e = getenv("GLP_FDY_NCG")) P->fdy_ncg = atoi(e);
   if (const char *e = getenv("GLP_HDGRAD")) P->allow_hdg = atoi(e);
   if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
   if (const char *e = getenv("GLP_TILE_UNITS")) P->tile_units = atoi(e);

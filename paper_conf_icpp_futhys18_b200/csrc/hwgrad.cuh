@@ -31,6 +31,8 @@ namespace glp {
 constexpr int HW_THREADS = 192;
 // fused-dy variant with NCG groups of 4 dy-building warps (warps 0-3, then 6-9, 10-13): group g
 // builds k-blocks kb0 + g, kb0 + g + NCG, ... so NCG k-blocks' loads are in flight at once
+// NCG = 1: one builder group (warps 0-3) whose loads land in shared memory by cp.async (two fp32
+// landing buffers of 128 pixels x bn channels), so the loads in flight are not bounded by registers
 __host__ __device__ constexpr int hw_threads(int ncg) { return ncg > 1 ? 192 + 128 * (ncg - 1) : 192; }
 constexpr int HW_BKP = 128;   // pixel rows (K) per k-block
 
@@ -62,12 +64,14 @@ struct HwgradParams {
   int n_tickets;
 };
 
-template <int NCG>   // 0: dy packed in the workspace (TMA); 2 or 3: fused dy, NCG builder groups
+template <int NCG>   // 0: dy packed in the workspace (TMA); 1: fused dy through a cp.async landing
+                     // zone; 2 or 3: fused dy, NCG register-staged builder groups
 __global__ void __launch_bounds__(hw_threads(NCG), 1)
     hwgrad_kernel(const __grid_constant__ HwgradParams p, const __grid_constant__ CUtensorMap tmapX,
                   const __grid_constant__ CUtensorMap tmapDy) {
   constexpr bool FDY = NCG > 0;
   constexpr int MAXG = NCG == 3 ? 3 : 4;   // 32-channel groups a builder thread holds (bn <= 32*MAXG)
+  static_assert(NCG != 1 || MAXG == 4, "landing-zone builders: bn <= 128");
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -177,6 +181,79 @@ __global__ void __launch_bounds__(hw_threads(NCG), 1)
       float dbacc[MAXG];
 #pragma unroll
       for (int g = 0; g < MAXG; ++g) dbacc[g] = 0.f;
+      if constexpr (NCG == 1) {
+        // landing zones after the db staging area: [2][bn][128] fp32 (thread t = pixel column t)
+        const uint32_t sland = (bars + 8u * (2 * S_ + 2) + 15u) & ~15u;   // db staging reuses it
+        const uint32_t lbytes = (uint32_t)p.bn * 128u * 4u;
+        auto issue = [&](int kb, uint32_t buf) {
+          const int q = kb * HW_BKP + t;
+          uint32_t n = 0, rem = 0, h = 0, w = 0;
+          p.div_img.divmod((uint32_t)min(q, p.rows - 1), n, rem);
+          p.div_w.divmod(rem, h, w);
+          const bool ok = q < p.rows && (int)h < p.ho && (int)w < p.wo;
+          const float *src = p.dy + ((size_t)n * p.dy_c * p.ho + h) * p.wo + w;
+          const uint32_t dst = sland + buf * lbytes + (uint32_t)t * 4u;
+          for (int co = 0; co < p.bn; ++co)
+            cp_async4(dst + (uint32_t)co * 512u, ok && co < p.co ? src + (size_t)co * hw : p.dy,
+                      ok && co < p.co);
+          cp_async_commit();
+        };
+        if (kb0 < kb1) issue(kb0, 0u);
+        uint32_t cur = 0;
+        for (int kb = kb0; kb < kb1; ++kb, cur ^= 1u) {
+          const int rs = (kb - kb0) % S_;
+          const uint32_t rph = (uint32_t)(((kb - kb0) / S_) & 1);
+          if (kb + 1 < kb1) {
+            issue(kb + 1, cur ^ 1u);
+            cp_async_wait<1>();
+          } else {
+            cp_async_wait<0>();
+          }
+          mbar_wait(empty(rs), rph ^ 1u);
+          const uint32_t sB = base + (uint32_t)rs * stage_bytes + (uint32_t)p.a_bytes;
+          const float *lv = reinterpret_cast<const float *>(smem_raw + (sland + cur * lbytes - raw)) + t;
+#pragma unroll
+          for (int g = 0; g < MAXG; ++g) {
+            if (g >= ngrp) break;
+            float v[32];
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = lv[(g * 32 + j) * 128];
+            float tt[32];
+#pragma unroll
+            for (int j = 0; j < 32; ++j) tt[j] = v[j];
+#pragma unroll
+            for (int wdt = 16; wdt >= 1; wdt >>= 1) {
+              const bool up = (lane & wdt) != 0;
+#pragma unroll
+              for (int j = 0; j < wdt; ++j) {
+                const float send = up ? tt[j] : tt[j + wdt];
+                const float keep = up ? tt[j + wdt] : tt[j];
+                tt[j] = keep + __shfl_xor_sync(0xffffffffu, send, wdt);
+              }
+            }
+            dbacc[g] += tt[0];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+              const int co0 = g * 32 + c * 8;
+              if (co0 >= p.bn) break;
+              __nv_bfloat162 a = __floats2bfloat162_rn(v[c * 8], v[c * 8 + 1]);
+              __nv_bfloat162 b = __floats2bfloat162_rn(v[c * 8 + 2], v[c * 8 + 3]);
+              __nv_bfloat162 cc = __floats2bfloat162_rn(v[c * 8 + 4], v[c * 8 + 5]);
+              __nv_bfloat162 d = __floats2bfloat162_rn(v[c * 8 + 6], v[c * 8 + 7]);
+              const uint32_t atom = (uint32_t)(co0 >> 6), ch = (uint32_t)((co0 & 63) >> 3);
+              const uint32_t addr = sB + atom * (uint32_t)(HW_BKP * 128) + (uint32_t)t * 128u +
+                                    ((ch ^ (uint32_t)(t & 7)) << 4);
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr),
+                           "r"(*reinterpret_cast<uint32_t *>(&a)), "r"(*reinterpret_cast<uint32_t *>(&b)),
+                           "r"(*reinterpret_cast<uint32_t *>(&cc)), "r"(*reinterpret_cast<uint32_t *>(&d))
+                           : "memory");
+            }
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(full(rs));
+        }
+      } else
       for (int kb = kb0 + grp; kb < kb1; kb += NCG) {
         const int rs = (kb - kb0) % S_;
         const uint32_t rph = (uint32_t)(((kb - kb0) / S_) & 1);
@@ -239,6 +316,7 @@ __global__ void __launch_bounds__(hw_threads(NCG), 1)
       // db partial of this CTA's pixel range: warps 0..3 in order (fixed), one row per CTA
       const uint32_t sred = (bars + 8u * (2 * S_ + 2) + 15u) & ~15u;   // 4*NCG x 256 floats
       float *red = reinterpret_cast<float *>(smem_raw + (sred - raw));
+      if (NCG == 1) named_bar_sync(1, 128);   // the landing zone is done before it holds db
       const int slot = grp * 4 + (warp & 3);   // a fixed slot per warp (4 per group)
 #pragma unroll
       for (int g = 0; g < MAXG; ++g)

@@ -92,6 +92,12 @@ __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, bool v
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n)
                : "memory");
 }
+// 4-byte cp.async (L1-allocating .ca: the only form for sizes < 16); zero-fills when !valid
+__device__ __forceinline__ void cp_async4(uint32_t dst, const void *src, bool valid) {
+  const uint32_t n = valid ? 4u : 0u;
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst), "l"(src), "r"(n)
+               : "memory");
+}
 // Arrive on `bar` when every cp.async previously issued by this thread has completed; noinc:
 // the arrival counts against the barrier's expected count (no pending-count increment).
 // Same completion mechanism as CUTLASS's sm100 cp.async mainloop (cpasync_barrier_arrive).

@@ -676,3 +676,19 @@ def test_halo_dgrad_model_choice():
     assert _layer(HDG_SHAPES[0], "bf16").info.dgrad_halo == 1
     assert _layer(SHAPES[6], "bf16").info.dgrad_halo == 0
     assert _layer(HDG_SHAPES[0], "tf32").info.dgrad_halo == 0
+
+
+@pytest.mark.parametrize("ncg", ["1", "2"])
+def test_halo_wgrad_fused_dy_variants(ncg, monkeypatch):
+    """The other fused-dy builder variants (GLP_FDY_NCG=1: cp.async landing zone; 2: two register
+    groups) give the same dW bits as the default and db within summation-order noise."""
+    shape = HALO_SHAPES[1]
+    d = _data(shape, seed=55)
+    ref = _run(_layer(shape, "bf16"), d)
+    monkeypatch.setenv("GLP_FDY_NCG", ncg)
+    layer = _layer(shape, "bf16")
+    assert layer.info.wgrad_fused_dy == 1
+    got = _run(layer, d)
+    np.testing.assert_array_equal(got["dw"], ref["dw"])
+    scale = np.abs(d["dy"].astype(np.float64)).sum(axis=(0, 2, 3))
+    assert np.all(np.abs(got["db"].astype(np.float64) - ref["db"]) <= 1e-6 * scale)

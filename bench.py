@@ -556,7 +556,7 @@ def run_glp(args, ws, rank, local):
     fstreams = [None] + [torch.cuda.Stream(device=dev) for _ in range(width - 1)]
     gstreams = [torch.cuda.Stream(device=dev) for _ in range(width)]
 
-    def step(ev=None, concurrent=None):
+    def step(ev=None, concurrent=None, with_exchange=True):
         """One training step of every layer's hot path.  concurrent (default: not timing kernels):
         the stream DAG of a real network's step -- per DAG level, each unit's forward chain and
         backward-data chain on its own stream (one level = independent layers; the main stream
@@ -600,7 +600,8 @@ def run_glp(args, ws, rank, local):
                 if ev is not None:
                     ev[i][5].record(stream)
                 s.reduce()
-            exchange()
+            if with_exchange:
+                exchange()
             return
         fs = [stream] + fstreams[1:]
         side_w.wait_stream(stream)
@@ -655,24 +656,28 @@ def run_glp(args, ws, rank, local):
         stream.wait_stream(side_w)
         for g in gstreams:
             stream.wait_stream(g)
-        exchange()
+        if with_exchange:
+            exchange()
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     if G > 1:
         dist.barrier()
-    use_graph = (not args.no_graph) and G == 1
+    use_graph = not args.no_graph
     evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(6)] for _ in states]
            for _ in range(args.steps)]
     if use_graph:
         # The whole step (every pack, GEMM and reduction launch of all layers) recorded once and
-        # replayed: no per-launch host work and minimal gaps between kernels.
+        # replayed: no per-launch host work and minimal gaps between kernels.  The gradient
+        # exchange (NCCL all_reduce, or the tree's point-to-point) stays outside the graph and is
+        # issued after each replay on the same stream.
         g_step = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g_step):
-            step(concurrent=not args.serial)
+            step(concurrent=not args.serial, with_exchange=False)
         for _ in range(max(1, args.warmup)):
             g_step.replay()
+            exchange()
     clocks = ClockSampler(local) if rank == 0 else None
     if clocks:
         clocks.start()
@@ -684,6 +689,7 @@ def run_glp(args, ws, rank, local):
     for k in range(args.steps):
         if use_graph:
             g_step.replay()
+            exchange()
         else:
             step(evs[k])
     t1.record(stream)

@@ -93,14 +93,6 @@ struct IgemmParams {
                                 //   [3] producer waits on empty
   int dbg_skip;          // diagnostics only (GLP_DEBUG_SKIP): bit0 skip A loads, bit1 skip B
                          // loads, bit2 skip MMAs — results are garbage, timings isolate stages
-  // pipelined pack (GLP_PIPE; fwd/dgrad with the im2col TMA): per-128-row-chunk progress counters
-  // of the packed source, polled before a tile's loads; the last CTA resets them.  nullptr: the
-  // pack completed before this kernel started (stream order).
-  unsigned int *prog;
-  unsigned int *prog_done;
-  int prog_target;       // work items per chunk (32-channel blocks of the pack)
-  int prog_nchunks;
-  int prog_kh;           // rows of the gather window (K_h)
 };
 
 }  // namespace glp

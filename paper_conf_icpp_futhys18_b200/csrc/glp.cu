@@ -303,14 +303,6 @@ struct MapCache {
   };
   DyRec dyrec[16];
   int dy_next = 0;
-  // pipelined packs: per workspace, counters zeroed once (init) and a pack launched but not yet
-  // consumed by its GEMM (pending x / dy)
-  struct PipeRec {
-    const void *ws = nullptr;
-    bool init = false, pend_x = false, pend_dy = false;
-  };
-  PipeRec pipe[16];
-  int pipe_next = 0;
   std::mutex mu;
   MapCache() = default;
   MapCache(const MapCache &) {}
@@ -370,9 +362,6 @@ struct glp_plan_s {
   int allow_hdg = 1;   // GLP_HDGRAD=0: im2col backward-data everywhere (A/B runs); 2 = force where legal
   int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
   int tile_units = 2;  // GLP_TILE_UNITS=u: fwd/dgrad tile model applies below u units per slot
-  int pipe = 0;        // GLP_PIPE=1: pipelined activation packs (progress counters + PDL consumer)
-  size_t off_prog = 0, sz_prog = 0;   // [x counters + done | dy counters + done]
-  int prog_chunks_x = 0, prog_chunks_dy = 0;
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -801,8 +790,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
 
 template <int MODE>
 glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
-                          const CUtensorMap &mapB, const CUtensorMap &mapA, cudaStream_t st,
-                          bool pdl = false) {
+                          const CUtensorMap &mapB, const CUtensorMap &mapA, cudaStream_t st) {
   void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg);
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof(cfg));
@@ -818,7 +806,7 @@ glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmPa
   attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = (P.pdl || pdl) ? 2 : 1;
+  cfg.numAttrs = P.pdl ? 2 : 1;
   void *args[] = {const_cast<IgemmParams *>(&p), const_cast<CUtensorMap *>(&mapB),
                   const_cast<CUtensorMap *>(&mapA)};
   GLP_CUDA(cudaLaunchKernelExC(&cfg, fn, args));
@@ -1103,76 +1091,6 @@ const float *recorded_dy(glp_plan_s &P, const void *ws) {
   return nullptr;
 }
 
-MapCache::PipeRec &pipe_rec_locked(glp_plan_s &P, const void *ws) {
-  for (auto &r : P.maps.pipe)
-    if (r.ws == ws) return r;
-  auto &r = P.maps.pipe[P.maps.pipe_next];
-  P.maps.pipe_next = (P.maps.pipe_next + 1) % 16;
-  r = MapCache::PipeRec{};
-  r.ws = ws;
-  return r;
-}
-bool pipe_ok_x(const glp_plan_s &P) {
-  return P.pipe && !P.s2d && !P.hfwd && P.fwd.a_tma && P.d.nbr <= 1 && !P.pack_block &&
-         P.Cpx * P.elem > 32;
-}
-bool pipe_ok_dy(const glp_plan_s &P) {
-  return P.pipe && !P.halo && !P.hdg && P.dgrad.a_tma && P.d.nbr <= 1 && !P.pack_block &&
-         P.Cop * P.elem > 32;
-}
-// Pipelined activation pack (which 0: x for the forward, 1: dy for the backward-data pass): the
-// persistent pack_act_pipe publishes per-chunk progress; the next GEMM of this workspace polls it.
-glp_status_t launch_pack_pipe(glp_plan_s &P, const float *src, uint8_t *ws, int which, bool with_db,
-                              cudaStream_t st) {
-  const glp_conv_desc_s &d = P.d;
-  unsigned int *prog = reinterpret_cast<unsigned int *>(ws + P.off_prog) +
-                       (which ? P.prog_chunks_x + 1 : 0);
-  const int chunks = which ? P.prog_chunks_dy : P.prog_chunks_x;
-  bool clear_all = false, clear_one = false;
-  {
-    std::lock_guard<std::mutex> lk(P.maps.mu);
-    auto &r = pipe_rec_locked(P, ws);
-    clear_all = !r.init;
-    clear_one = which ? r.pend_dy : r.pend_x;   // a pack its GEMM never consumed: dirty counters
-    r.init = true;
-    if (which) r.pend_dy = true;
-    else r.pend_x = true;
-  }
-  if (clear_all) GLP_CUDA(cudaMemsetAsync(ws + P.off_prog, 0, P.sz_prog, st));
-  else if (clear_one) GLP_CUDA(cudaMemsetAsync(prog, 0, (size_t)(chunks + 1) * 4, st));
-  const int C = which ? d.Co : d.C, HW = which ? d.Ho * d.Wo : d.H * d.W;
-  const int Cp = which ? P.Cop : P.Cpx, img_c = which ? P.y_img_c : P.x_img_c;
-  float *dbp = (which && with_db) ? reinterpret_cast<float *>(ws + P.off_dbpart) : nullptr;
-  unsigned int *tickets = dbp ? db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.db_rows).tickets : nullptr;
-  const int nt = (int)cdiv(d.Co, 32);
-  const long long items = (long long)chunks * cdiv(Cp, 32);
-  const dim3 grid((unsigned)std::min<long long>(items, P.sm_count));
-  if (P.elem == 2)
-    GLP_CUDA(launch_pdl(P.pdl, pack_act_pipe<2>, grid, dim3(128), 0, st, src, (void *)(ws + (which ? P.off_dypk : P.off_xpk)), d.N, C, HW, Cp, dbp, tickets, nt, 1, 1, HW, 0, Cp, C, img_c, prog));
-  else
-    GLP_CUDA(launch_pdl(P.pdl, pack_act_pipe<4>, grid, dim3(128), 0, st, src, (void *)(ws + (which ? P.off_dypk : P.off_xpk)), d.N, C, HW, Cp, dbp, tickets, nt, 1, 1, HW, 0, Cp, C, img_c, prog));
-  GLP_LAUNCH_CHECK("pack_act_pipe");
-  return GLP_OK;
-}
-// The GEMM consuming a pending pipelined pack: progress pointers into p, returns true (launch it
-// with programmatic dependent launch).  No pending pack: false.
-bool take_pipe(glp_plan_s &P, uint8_t *ws, int which, IgemmParams &p, int kh) {
-  {
-    std::lock_guard<std::mutex> lk(P.maps.mu);
-    auto &r = pipe_rec_locked(P, ws);
-    bool &pend = which ? r.pend_dy : r.pend_x;
-    if (!pend) return false;
-    pend = false;
-  }
-  const int chunks = which ? P.prog_chunks_dy : P.prog_chunks_x;
-  p.prog = reinterpret_cast<unsigned int *>(ws + P.off_prog) + (which ? P.prog_chunks_x + 1 : 0);
-  p.prog_done = p.prog + chunks;
-  p.prog_nchunks = chunks;
-  p.prog_target = (int)cdiv(which ? P.Cop : P.Cpx, 32);
-  p.prog_kh = kh;
-  return true;
-}
-
 glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t *ws,
                           cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
@@ -1239,8 +1157,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   p.bias_floats = pp.bias_floats;
   p.out_c = P.y_img_c;   // channels per image of y (the whole tensor for a conv group)
   p.out_hw = d.Ho * d.Wo;
-  const bool piped = pp.a_tma && take_pipe(P, ws, 0, p, d.Kh);
-  return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st, piped);
+  return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);
 }
 
 glp_status_t encode_4d_nhwc(CUtensorMap *map, const void *ptr, int cpitch, int W, int H, int N,
@@ -1316,8 +1233,7 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   p.out = dx;
   p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
   p.out_hw = d.H * d.W;
-  const bool piped = pp.a_tma && take_pipe(P, ws, 1, p, d.Kh);
-  return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st, piped);
+  return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
 }
 
 glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const float *dy) {
@@ -1686,7 +1602,6 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   if (const char *e = getenv("GLP_HDGRAD")) P->allow_hdg = atoi(e);
   if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
   if (const char *e = getenv("GLP_TILE_UNITS")) P->tile_units = atoi(e);
-  if (const char *e = getenv("GLP_PIPE")) P->pipe = atoi(e) != 0;
   if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
   if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
@@ -1778,13 +1693,9 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     P->off_wtpk = P->off_wpk + P->sz_wpk;   // own region: both weight packs can live at once
     P->off_part = P->off_wtpk + P->sz_wtpk;
     P->off_dbpart = P->off_part + P->sz_part;
-    P->prog_chunks_x = (int)cdiv((long long)c.N * c.H * c.W, PIPE_ROWS);
-    P->prog_chunks_dy = (int)cdiv((long long)c.N * c.Ho * c.Wo, PIPE_ROWS);
-    P->sz_prog = align1k((size_t)(P->prog_chunks_x + 1 + P->prog_chunks_dy + 1) * 4);
-    P->off_prog = P->off_dbpart + P->sz_dbpart;
     P->ws_fwd = P->off_wpk + P->sz_wpk;
     P->ws_dgrad = P->off_wtpk + P->sz_wtpk;
-    P->ws_wgrad = P->off_prog + P->sz_prog;
+    P->ws_wgrad = P->off_dbpart + P->sz_dbpart;
     P->ws_bwd = P->ws_wgrad;
     const long long slots = (long long)P->sm_count * P->fwd.ctas_per_sm;
     const long long per = (long long)d->Ho * d->Wo * P->fwd.n_tiles;  // pixels*n_tiles per sample
@@ -2022,16 +1933,11 @@ glp_status_t glp_stage_pack(glp_plan_t P, glp_pack_t what, const float *src, voi
     const GOff o = goff(P, g);
     uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
     switch (what) {
-      case GLP_PACK_X:
-        if (pipe_ok_x(*P)) s = launch_pack_pipe(*P, src + o.x, wsb, 0, false, st);
-        else s = launch_pack_x(*P, src + o.x, wsb + P->off_xpk, st);
-        break;
+      case GLP_PACK_X: s = launch_pack_x(*P, src + o.x, wsb + P->off_xpk, st); break;
       case GLP_PACK_DY:
       case GLP_PACK_DY_DB:
         if (P->halo_fdy)   // recorded only: the filter gradient reads it, bwd_data packs it
           record_dy(*P, wsb, src + o.y);
-        else if (pipe_ok_dy(*P))
-          s = launch_pack_pipe(*P, src + o.y, wsb, 1, what == GLP_PACK_DY_DB, st);
         else
           s = launch_pack_dy(*P, br_in1(src + o.y), wsb, what == GLP_PACK_DY_DB, st);
         break;

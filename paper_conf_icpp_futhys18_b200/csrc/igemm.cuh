@@ -156,7 +156,7 @@ __global__ void __launch_bounds__(288, 1)
   tc_fence_after();
   // prologue done (barriers, TMEM, descriptor prefetch): wait for the previous kernel's results
   // before touching global memory
-  if (p.prog == nullptr) pdl_wait();   // pipelined: rows are awaited per tile instead
+  pdl_wait();
   const uint32_t tmem_base = __shfl_sync(0xffffffffu, *tmem_slot_ptr, 0);   // warp-uniform
 
   // work units: CG1 = one 128-row tile; CG2 = a pair of 128-row tiles (one per CTA)
@@ -200,32 +200,6 @@ __global__ void __launch_bounds__(288, 1)
             g.div_w.divmod(rem, oh, ow);
             h_t = (int)oh * g.im_sh - g.im_ph;
             w_t = (int)ow * g.im_sw - g.im_pw;
-            if (p.prog != nullptr) {
-              // wait until the pack has published every source row this tile's window touches
-              uint32_t nb, remb, ohb, owb;
-              g.div_hw.divmod((uint32_t)min(m0 + C::BM - 1, p.M - 1), nb, remb);
-              g.div_w.divmod(remb, ohb, owb);
-              const int hlo = min(max(h_t, 0), g.src_h - 1);
-              const int hhi = min(max((int)ohb * g.im_sh - g.im_ph + p.prog_kh - 1, 0), g.src_h - 1);
-              const long long img = (long long)g.src_h * g.src_w;
-              const long long r0 = (long long)n_t * img + (long long)hlo * g.src_w;
-              const long long r1 = (long long)nb * img + (long long)hhi * g.src_w + g.src_w - 1;
-              const int c0 = (int)(r0 / 128), c1 = min((int)(r1 / 128), p.prog_nchunks - 1);
-              if (lane == 0) {
-                for (int c = c0; c <= c1; ++c) {
-                  unsigned int v;
-                  long long spins = 0;
-                  do {
-                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.prog + c) : "memory");
-                    if (v >= (unsigned)p.prog_target) break;
-                    __nanosleep(64);
-                  } while (++spins < (1LL << 26));
-                  if (spins >= (1LL << 26)) __trap();   // a lost producer: fail, never hang
-                }
-                asm volatile("fence.proxy.async.global;" ::: "memory");
-              }
-              __syncwarp();
-            }
           } else {
 #pragma unroll
             for (int a = 0; a < NA; ++a) {
@@ -696,16 +670,6 @@ __global__ void __launch_bounds__(288, 1)
   else __syncthreads();
   tc_fence_after();
   if (warp == 8) tmem_dealloc_cg<CG>(tmem_base, (uint32_t)p.tmem_cols);
-  if (p.prog != nullptr) {
-    // the last CTA out resets the progress counters for the next pipelined pack
-    // (__syncthreads_or broadcasts the flag: no static shared memory next to the 227 KB dynamic)
-    const int s_last = __syncthreads_or(threadIdx.x == 0 && atomicAdd(p.prog_done, 1u) == gridDim.x - 1);
-    if (s_last) {
-      for (int c = threadIdx.x; c < p.prog_nchunks; c += blockDim.x) p.prog[c] = 0u;
-      if (threadIdx.x == 0) *p.prog_done = 0u;
-      __threadfence();
-    }
-  }
 }
 
 }  // namespace glp

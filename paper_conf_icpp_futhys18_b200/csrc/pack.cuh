@@ -155,15 +155,24 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
 // (32-row tile, channel), the 32 rows summed by a fixed transposing butterfly (lane c ends with
 // channel c's sum).  grid (ceil(Cw/32), ceil(N*HWd/256)), 256 threads.
 constexpr int PACKW_ROWS = 32;
-// One warp's unit of the warp-tiled pack: destination rows [q0, q0 + 32) x channels [c0, c0 + 32)
-// (slab: this warp's 32 x (32*ELEM + 16)-byte staging area).
 template <int ELEM>
-__device__ __forceinline__ void pack_act_unit(const float *__restrict__ src, void *__restrict__ dst,
-                                              long long q0, int c0, long long total, int C, int HW,
-                                              int Cp, float *__restrict__ db_part, int Ws, int Wd,
-                                              int HWd, int co_off, int Cw, int db_ld, int src_c,
-                                              uint8_t *slab, int lane) {
+__global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ src,
+                                                     void *__restrict__ dst, int N, int C, int HW,
+                                                     int Cp, float *__restrict__ db_part,
+                                                     unsigned int *__restrict__ tickets,
+                                                     int n_tickets, int Ws, int Wd, int HWd,
+                                                     int co_off, int Cw, int db_ld, int src_c) {
   constexpr int RB = 32 * ELEM + 16;                    // smem bytes per staged row (+16 pad)
+  __shared__ __align__(16) uint8_t slab[8][32 * RB];
+  pdl_launch_dependents();
+  pdl_wait();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c0 = blockIdx.x * 32;
+  const long long q0 = ((long long)blockIdx.y * 8 + warp) * PACKW_ROWS;
+  const long long total = (long long)N * HWd;
+  if (tickets != nullptr && (blockIdx.x | blockIdx.y) == 0)
+    for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
+  if (q0 >= total) return;
   // this lane's row -> source (n, pixel)
   const long long q = q0 + lane;
   bool ok = q < total;
@@ -204,7 +213,7 @@ __device__ __forceinline__ void pack_act_unit(const float *__restrict__ src, voi
       db_part[(size_t)(q0 / PACKW_ROWS) * db_ld + co_off + c0 + lane] = t[0];
   }
   // round + pack this lane's row, stage it in the warp's slab
-  uint8_t *row = slab + lane * RB;
+  uint8_t *row = slab[warp] + lane * RB;
 #pragma unroll
   for (int j = 0; j < 32; j += 8) {
     uint4 u0, u1;
@@ -232,70 +241,10 @@ __device__ __forceinline__ void pack_act_unit(const float *__restrict__ src, voi
     const long long qr = q0 + r;
     const int c = c0 + ch * (16 / ELEM);
     if (qr < total && c < Cw) {
-      const uint4 val = *reinterpret_cast<const uint4 *>(slab + r * RB + ch * 16);
+      const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
       *reinterpret_cast<uint4 *>(static_cast<uint8_t *>(dst) +
                                  ((size_t)qr * Cp + co_off + c) * ELEM) = val;
     }
-  }
-  __syncwarp();   // the slab is reused by the warp's next unit
-}
-
-template <int ELEM>
-__global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ src,
-                                                     void *__restrict__ dst, int N, int C, int HW,
-                                                     int Cp, float *__restrict__ db_part,
-                                                     unsigned int *__restrict__ tickets,
-                                                     int n_tickets, int Ws, int Wd, int HWd,
-                                                     int co_off, int Cw, int db_ld, int src_c) {
-  constexpr int RB = 32 * ELEM + 16;
-  __shared__ __align__(16) uint8_t slab[8][32 * RB];
-  pdl_launch_dependents();
-  pdl_wait();
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int c0 = blockIdx.x * 32;
-  const long long q0 = ((long long)blockIdx.y * 8 + warp) * PACKW_ROWS;
-  const long long total = (long long)N * HWd;
-  if (tickets != nullptr && (blockIdx.x | blockIdx.y) == 0)
-    for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
-  if (q0 >= total) return;
-  pack_act_unit<ELEM>(src, dst, q0, c0, total, C, HW, Cp, db_part, Ws, Wd, HWd, co_off, Cw, db_ld,
-                      src_c, slab[warp], lane);
-}
-
-// Pipelined form (GLP_PIPE): a persistent grid of 4-warp blocks (10 KB of smem, so each SM keeps
-// room for the persistent GEMM that consumes the packed rows) walks work items (row chunk of 128
-// rows, 32-channel block) in chunk-major order and publishes each finished item on its chunk's
-// counter with a release add; the consumer GEMM, launched with programmatic dependent launch,
-// polls the counters of the rows a tile needs (acquire) instead of waiting for the whole pack.
-constexpr int PIPE_ROWS = 128;   // rows per progress chunk (4 warps x 32)
-template <int ELEM>
-__global__ void __launch_bounds__(128) pack_act_pipe(const float *__restrict__ src,
-                                                     void *__restrict__ dst, int N, int C, int HW,
-                                                     int Cp, float *__restrict__ db_part,
-                                                     unsigned int *__restrict__ tickets,
-                                                     int n_tickets, int Ws, int Wd, int HWd,
-                                                     int co_off, int Cw, int db_ld, int src_c,
-                                                     unsigned int *__restrict__ prog) {
-  constexpr int RB = 32 * ELEM + 16;
-  __shared__ __align__(16) uint8_t slab[4][32 * RB];
-  pdl_launch_dependents();
-  pdl_wait();
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long total = (long long)N * HWd;
-  const int gx = (Cw + 31) / 32;
-  const long long chunks = (total + PIPE_ROWS - 1) / PIPE_ROWS;
-  if (tickets != nullptr && blockIdx.x == 0)
-    for (int i = threadIdx.x; i < n_tickets; i += blockDim.x) tickets[i] = 0u;
-  for (long long it = blockIdx.x; it < chunks * gx; it += gridDim.x) {
-    const long long chunk = it / gx;
-    const int cb = (int)(it - chunk * gx);
-    const long long q0 = chunk * PIPE_ROWS + warp * PACKW_ROWS;
-    if (q0 < total)
-      pack_act_unit<ELEM>(src, dst, q0, cb * 32, total, C, HW, Cp, db_part, Ws, Wd, HWd, co_off,
-                          Cw, db_ld, src_c, slab[warp], lane);
-    __syncthreads();   // every warp's stores of the item precede the release below
-    if (threadIdx.x == 0)
-      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(prog + chunk) : "memory");
   }
 }
 

@@ -692,36 +692,3 @@ def test_halo_wgrad_fused_dy_variants(ncg, monkeypatch):
     np.testing.assert_array_equal(got["dw"], ref["dw"])
     scale = np.abs(d["dy"].astype(np.float64)).sum(axis=(0, 2, 3))
     assert np.all(np.abs(got["db"].astype(np.float64) - ref["db"]) <= 1e-6 * scale)
-
-
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
-@pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[5], SHAPES[6], ("cifar_conv2", 3, 32, 16, 16, 32, 5, 1, 2)],
-                         ids=lambda s: s[0])
-def test_pipelined_packs(shape, math, monkeypatch):
-    """GLP_PIPE=1: the staged activation packs publish per-chunk progress and the consuming
-    forward / backward-data GEMMs (programmatic dependent launch) poll it per tile.  Outputs are
-    bitwise the non-pipelined composed results, on repeated steps (counters reset by the GEMM)
-    and when a pack is issued twice before its GEMM (dirty counters cleared)."""
-    d = _data(shape, seed=57)
-    ref = _run(_layer(shape, math), d)
-    monkeypatch.setenv("GLP_PIPE", "1")
-    layer = _layer(shape, math)
-    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
-    for rep in range(3):
-        y = torch.full(layer.y_shape, float("nan"), device=DEV)
-        dx = torch.full(layer.x_shape, float("nan"), device=DEV)
-        dw = torch.full(layer.w_shape, float("nan"), device=DEV)
-        db = torch.full((layer.geom.Co,), float("nan"), device=DEV)
-        layer.stage_pack(glp.GLP_PACK_X, t["x"])
-        if rep == 2:
-            layer.stage_pack(glp.GLP_PACK_X, t["x"])   # unconsumed pack: counters cleared
-        layer.stage_pack(glp.GLP_PACK_W_FWD, t["w"])
-        layer.stage_fwd(t["b"], y)
-        layer.stage_pack(glp.GLP_PACK_DY_DB, t["dy"])
-        layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
-        layer.stage_bwd_data(dx)
-        layer.stage_bwd_filter()
-        layer.stage_reduce(dw, db)
-        torch.cuda.synchronize()
-        for k, v in (("y", y), ("dx", dx), ("dw", dw), ("db", db)):
-            np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=f"rep {rep} {k}")

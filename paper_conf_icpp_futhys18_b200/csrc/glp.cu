@@ -508,11 +508,14 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   h.a_bytes = (int)rup((long long)(R + K - 1) * WQ * 128, 1024);
   h.b_tap_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
   h.a_stages = 3;
+  if (const char *e = getenv("GLP_HD_ASTAGES")) h.a_stages = std::max(2, atoi(e));   // A/B runs
   const int fixed = 1024 + h.a_stages * h.a_bytes + 8 * 64 + 16;
   // as many taps per B stage as keep >= 4 stages (the issuer's barrier round trip costs more than
   // the 8 MMAs of one tap)
+  int min_bst = 4;
+  if (const char *e = getenv("GLP_HD_BSTAGES")) min_bst = std::max(2, atoi(e));   // A/B runs
   h.b_taps = 1;
-  while (h.b_taps < taps && (P.smem_cap - fixed) / ((h.b_taps + 1) * h.b_tap_bytes) >= 4) ++h.b_taps;
+  while (h.b_taps < taps && (P.smem_cap - fixed) / ((h.b_taps + 1) * h.b_tap_bytes) >= min_bst) ++h.b_taps;
   h.b_bytes = h.b_taps * h.b_tap_bytes;
   h.b_stages = std::min(8, (P.smem_cap - fixed) / h.b_bytes);
   if (h.b_stages < 3) return GLP_OK;

@@ -28,7 +28,7 @@
 
 namespace glp {
 
-constexpr int HF_THREADS = 192;
+constexpr int HF_THREADS = 320;   // + warps 6-9: a second epilogue group (alternate 32-column chunks)
 constexpr int HF_MAXTAPS = 16;
 
 struct HfwdParams {
@@ -87,7 +87,7 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(tfull(a), 1);
-      mbar_init(tempty(a), 8);
+      mbar_init(tempty(a), 16);   // 8 epilogue warps per CTA, both CTAs
     }
     mbar_init(bfull, 1);
     fence_mbar_init();
@@ -162,12 +162,16 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
       }
     }
     __syncwarp();
-  } else if (warp < 4) {
+  } else if (warp < 4 || warp >= 6) {
     // ===================================== epilogue ========================================
-    const int row = warp * 32 + lane;
-    for (int i = row; i < p.bias_floats; i += 128)
+    // two groups of 4 warps (0-3 and 6-9): warp w drains TMEM lanes 32*(w % 4)..+31; group 0 takes
+    // the 32-column chunks 0, 2, 4, ..., group 1 the odd ones, so twice the stores are in flight
+    const int grp = warp >= 6 ? 1 : 0;
+    const int quad = warp & 3;
+    const int row = quad * 32 + lane;
+    for (int i = row + 128 * grp; i < p.bias_floats; i += 256)
       sts_f32(sbias + 4u * (uint32_t)i, (p.bias != nullptr && i < p.co) ? __ldg(p.bias + i) : 0.f);
-    named_bar_sync(1, 128);
+    named_bar_sync(1, 256);
     const size_t plane = (size_t)p.out_hw;
     uint32_t it = 0;
     for (int u = unit0; u < p.units; u += ustep, ++it) {
@@ -181,7 +185,7 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
       p.div_w.divmod(rem, h, w);
       const bool mv = q < p.rows && (int)h < p.ho && (int)w < p.wo && !(p.dbg_skip & 8);
       float *ob = p.out + (size_t)n * p.out_c * plane + (size_t)h * p.wo + w;
-      const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
+      const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + a * (uint32_t)p.acc_cols;
       auto store_chunk = [&](int c0, uint32_t (&v)[32]) {
         if (!mv) return;
         const int lim = min(32, p.co - c0);
@@ -205,21 +209,11 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
             if (k < lim) o[(size_t)k * plane] = __uint_as_float(v[k]) + lds_f32(sbias + 4u * (uint32_t)(c0 + k));
         }
       };
-      // software-pipelined TMEM drain (next chunk's load in flight while this one is stored)
-      uint32_t va[32], vb[32];
-      tmem_ld32(taddr, va);
-      tmem_wait_ld_dep(va);
-      for (int c0 = 0; c0 < p.bn; c0 += 64) {
-        const bool hb = c0 + 32 < p.bn;
-        if (hb) tmem_ld32(taddr + (uint32_t)(c0 + 32), vb);
+      uint32_t va[32];
+      for (int c0 = 32 * grp; c0 < p.bn; c0 += 64) {
+        tmem_ld32(taddr + (uint32_t)c0, va);
+        tmem_wait_ld_dep(va);
         store_chunk(c0, va);
-        if (hb) {
-          tmem_wait_ld_dep(vb);
-          const bool ha = c0 + 64 < p.bn;
-          if (ha) tmem_ld32(taddr + (uint32_t)(c0 + 64), va);
-          store_chunk(c0 + 32, vb);
-          if (ha) tmem_wait_ld_dep(va);
-        }
       }
       tc_fence_before();
       __syncwarp();

@@ -43,7 +43,8 @@ def parse_args():
     p.add_argument("--warmup", type=int, default=10)
     p.add_argument("--impl", choices=["glp", "reference"], default="glp")
     p.add_argument("--workload", type=int, default=4, help="BASELINE.json config index 1..5")
-    p.add_argument("--math", choices=["bf16", "tf32"], default="bf16")
+    p.add_argument("--math", choices=["fp32", "bf16", "tf32"], default="fp32",
+                   help="fp32 = 3xTF32 on tcgen05 (fp32-accurate, the paper's FP32 arithmetic)")
     p.add_argument("--scaling", choices=["weak", "strong"], default="weak")
     p.add_argument("--scheme", choices=["persistent", "pool"], default="persistent",
                    help="pool: the paper's prior-art scheme (per-sample kernels round-robin over a "
@@ -727,7 +728,8 @@ def run_glp(args, ws, rank, local):
         dump_units(states, args.dump, args.workload, args.math)
     peaks = load_peaks()
     dom = max(kern, key=lambda r: r["total_us"])
-    peak_tf = peaks["bf16_tflops_sustained"] * (1.0 if args.math == "bf16" else NOMINAL_TF32_OVER_BF16)
+    peak_tf = peaks["bf16_tflops_sustained"] * {"bf16": 1.0, "tf32": NOMINAL_TF32_OVER_BF16,
+                                                "fp32": NOMINAL_TF32_OVER_BF16 / 3}[args.math]
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):

@@ -53,9 +53,16 @@ typedef enum {
 } glp_status_t;
 
 typedef enum {
-  GLP_MATH_FP32 = 0, /* fp32 CUDA-core direct convolution; normwise error <= 1e-5           */
+  /* fp32-accurate (normwise error <= 1e-5, the paper's FP32 sgemm arithmetic, P173/P314): 3xTF32
+   * on tcgen05.  The packs split every operand v into hi = rna_tf32(v) and lo = rna_tf32(v - hi)
+   * (two planes); each k-step issues hi*hi, hi*lo, lo*hi kind::tf32 MMAs, in that fixed order,
+   * into one fp32 TMEM accumulator (SURVEY §8(c) "3xTF32 hi/lo split", §7.1 phase 9). */
+  GLP_MATH_FP32 = 0,
   GLP_MATH_TF32 = 1, /* tcgen05 kind::tf32 (operands RNA-rounded in the pack), fp32 accumulate */
-  GLP_MATH_BF16 = 2  /* tcgen05 kind::f16 with bf16 operands (RNE), fp32 accumulate           */
+  GLP_MATH_BF16 = 2, /* tcgen05 kind::f16 with bf16 operands (RNE), fp32 accumulate           */
+  /* fp32 CUDA-core direct convolution (one thread per output, fixed K order): the accuracy
+   * anchor the tests compare the tensor-core modes with; no staged API, no fused groups. */
+  GLP_MATH_FP32_SIMT = 3
 } glp_math_t;
 
 typedef struct glp_conv_desc_s *glp_conv_desc_t;
@@ -160,7 +167,7 @@ glp_status_t glp_conv_bwd(glp_plan_t plan, const float *x, const float *dy, cons
  * forward W, backward-data W, partials), so stages that touch disjoint regions may run on
  * different streams when the caller orders them with events (e.g. both weight packs up front,
  * the filter-gradient GEMM + reduce beside the next layer's backward-data work).
- * FP32 plans return GLP_ERR_NOT_SUPPORTED. */
+ * GLP_MATH_FP32_SIMT plans return GLP_ERR_NOT_SUPPORTED. */
 typedef enum {
   GLP_PACK_X = 0,          /* x  NCHW fp32 -> packed NHWC operand (rounded to the math mode)  */
   GLP_PACK_DY = 1,         /* dy NCHW fp32 -> packed NHWC operand                              */
@@ -200,7 +207,7 @@ glp_status_t glp_stage_reduce(glp_plan_t plan, float *dw, float *db, int accumul
  * y/dy [N][sum C_out][H_o][W_o]); the *_group calls below take one pointer per branch instead.
  * 1 <= n_branches <= 4.  Tensor-core plans require every branch but the last to have C_out a
  * multiple of 8 (BF16) / 4 (TF32) (GLP_ERR_NOT_SUPPORTED from glp_plan otherwise); the *_group
- * calls return GLP_ERR_NOT_SUPPORTED for GLP_MATH_FP32 plans.  Same ownership, workspace sizes
+ * calls return GLP_ERR_NOT_SUPPORTED for GLP_MATH_FP32_SIMT plans.  Same ownership, workspace sizes
  * (info.ws_*) and error behaviour as the single-tensor calls; results are bitwise identical to the
  * single-tensor calls on the concatenated tensors. */
 glp_status_t glp_conv_group_desc_create(glp_conv_desc_t *out, int N, int C_in, int H, int W,

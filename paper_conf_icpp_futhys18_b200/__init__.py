@@ -19,8 +19,10 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 # GLP_LIB overrides the in-tree library (A/B runs of two builds on one box)
 LIB_PATH = os.environ.get("GLP_LIB") or os.path.join(PKG, "libglp.so")
 
-GLP_MATH_FP32, GLP_MATH_TF32, GLP_MATH_BF16 = 0, 1, 2
-MATH = {"fp32": GLP_MATH_FP32, "tf32": GLP_MATH_TF32, "bf16": GLP_MATH_BF16}
+# fp32 = 3xTF32 on tcgen05 (fp32-accurate); fp32_simt = the CUDA-core accuracy anchor
+GLP_MATH_FP32, GLP_MATH_TF32, GLP_MATH_BF16, GLP_MATH_FP32_SIMT = 0, 1, 2, 3
+MATH = {"fp32": GLP_MATH_FP32, "tf32": GLP_MATH_TF32, "bf16": GLP_MATH_BF16,
+        "fp32_simt": GLP_MATH_FP32_SIMT}
 
 _c_int, _c_size, _vp, _dbl = ctypes.c_int, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_double
 

@@ -25,6 +25,14 @@ struct FastDiv {
 
 enum ConvMode : int { MODE_FWD = 0, MODE_DGRAD = 1, MODE_WGRAD = 2 };
 
+// Diagnostic work-skipping (timing isolation of pipeline stages, wrong results) exists only in
+// -DGLP_DIAG builds; the product library compiles every test to a constant false.
+#ifdef GLP_DIAG
+#define GLP_SKIP(p, bit) ((((p).dbg_skip) & (bit)) != 0)
+#else
+#define GLP_SKIP(p, bit) false
+#endif
+
 // Geometry of the activation gather (im2col never materialised).  The "pixel space" is the
 // GEMM's pixel dimension: y pixels for fwd (M) and wgrad (K), dx pixels for dgrad (M).
 struct Gather {
@@ -88,11 +96,16 @@ struct IgemmParams {
   int part_mpad;         // wgrad partial rows per split (m_tiles * 128)
   int a_tma;             // 1: A operand by im2col TMA (one thread); 0: cp.async gather
   int ksub;              // k-blocks per pipeline stage (1 or 2; cp.async path: 1)
+  long long lo_off_a;    // 3xTF32: byte offset from the packed A source's hi plane to its lo plane
+  int chunk_kb;          // 3xTF32: k-blocks per TMEM accumulation chunk (summed in fp32 registers)
+#ifdef GLP_DIAG
   unsigned long long *dbg_clk;  // diagnostics only (GLP_DEBUG_CLK): per-CTA cycle counters
                                 //   [0] MMA loop total [1] MMA waits on full [2] MMA waits on tempty
                                 //   [3] producer waits on empty
-  int dbg_skip;          // diagnostics only (GLP_DEBUG_SKIP): bit0 skip A loads, bit1 skip B
-                         // loads, bit2 skip MMAs — results are garbage, timings isolate stages
+#endif
+  int dbg_skip;          // diagnostics builds only (-DGLP_DIAG, GLP_DEBUG_SKIP): bit0 skip A loads,
+                         // bit1 skip B loads, bit2 skip MMAs — results are garbage, timings isolate
+                         // stages.  Product builds compile every GLP_SKIP test to false.
 };
 
 }  // namespace glp

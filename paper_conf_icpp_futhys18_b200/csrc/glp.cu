@@ -107,6 +107,8 @@ struct PassPlan {
   int cg = 1, m_units = 0;          // CTAs per MMA (tcgen05 cta_group); work units along M
   int ksub = 1;                     // k-blocks per pipeline stage
   int bias_floats = 0;              // forward: floats of the epilogue's smem bias stage
+  int threads = 288;                // CTA size (3xTF32: 512, eight epilogue warps)
+  int chunk_kb = 0;                 // 3xTF32: k-blocks per TMEM accumulation chunk
 };
 
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -192,24 +194,25 @@ glp_status_t encode_im2col(CUtensorMap *map, int elem, const void *ptr, int cpit
   return GLP_OK;
 }
 
-template <int MODE, int ELEM, int KROW, int CG>
+template <int MODE, int ELEM, int KROW, int CG, int X3>
 void *kernel_ptr() {
-  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM, KROW, CG>);
+  return reinterpret_cast<void *>(&igemm_kernel<MODE, ELEM, KROW, CG, X3>);
 }
 template <int MODE, int CG>
-void *igemm_ptr_m(int elem, int krow) {
-  if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128, CG>() : kernel_ptr<MODE, 2, 64, CG>();
-  return kernel_ptr<MODE, 4, 128, CG>();
+void *igemm_ptr_m(int elem, int krow, int x3) {
+  if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128, CG, 0>() : kernel_ptr<MODE, 2, 64, CG, 0>();
+  return x3 ? kernel_ptr<MODE, 4, 128, CG, 1>() : kernel_ptr<MODE, 4, 128, CG, 0>();
 }
-void *igemm_ptr(int mode, int elem, int krow, int cg) {
+// x3: the 3xTF32 variant (GLP_MATH_FP32: hi/lo operand planes, three MMAs per k-step)
+void *igemm_ptr(int mode, int elem, int krow, int cg, int x3) {
   if (cg == 2) {
-    if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 2>(elem, krow);
-    if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 2>(elem, krow);
-    return igemm_ptr_m<MODE_WGRAD, 2>(elem, krow);
+    if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 2>(elem, krow, x3);
+    if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 2>(elem, krow, x3);
+    return igemm_ptr_m<MODE_WGRAD, 2>(elem, krow, x3);
   }
-  if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 1>(elem, krow);
-  if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 1>(elem, krow);
-  return igemm_ptr_m<MODE_WGRAD, 1>(elem, krow);
+  if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 1>(elem, krow, x3);
+  if (mode == MODE_DGRAD) return igemm_ptr_m<MODE_DGRAD, 1>(elem, krow, x3);
+  return igemm_ptr_m<MODE_WGRAD, 1>(elem, krow, x3);
 }
 
 CUtensorMapSwizzle swz_kmajor(int krow) {
@@ -262,9 +265,11 @@ void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, 
 // Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
 // (constants, never the queried device or S), so the fp32 summation order is a function of the
 // shape alone (convergence invariance, P264).
-int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem, int cg) {
+int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem, int cg,
+                  int x3) {
   const double sm = 148.0 / cg;   // concurrent work units (CTA pairs for cg = 2)
-  const double kb_s = (elem == 2 ? 2.0 : 4.0) * std::max(bn, 96) / 1.8e9;  // seconds per k-block
+  // seconds per k-block (3xTF32: three MMAs per k-step)
+  const double kb_s = (elem == 2 ? 2.0 : 4.0) * (x3 ? 3.0 : 1.0) * std::max(bn, 96) / 1.8e9;
   const double bw = 6.0e12;
   int best = 1;
   double best_t = 1e30;
@@ -291,7 +296,7 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
 struct MapCache {
   struct Entry {
     const void *ws = nullptr;
-    CUtensorMap a, b;
+    CUtensorMap a, b, a2, b2;   // a2, b2: the lo planes of a 3xTF32 plan
   };
   Entry e[3][8];
   int next[3] = {0, 0, 0};
@@ -313,6 +318,8 @@ struct glp_plan_s {
   glp_conv_desc_s d;
   MapCache maps;
   int device = 0, math = 0, elem = 4, sm_count = 148, s_override = 0;
+  int simt = 0;   // GLP_MATH_FP32_SIMT: the CUDA-core direct convolution (accuracy anchor)
+  int x3 = 0;     // GLP_MATH_FP32: 3xTF32 on tcgen05 (hi/lo operand planes)
   int Cp = 0, Cop = 0, taps = 0;
   // Geometry of the x operand as the forward and filter-gradient passes see it: the layer itself,
   // or its space-to-depth form (s2d = stride S > 1: stride 1, ceil(K/S) taps, S*S*C channels).
@@ -346,6 +353,8 @@ struct glp_plan_s {
   // workspace layout
   size_t off_xpk = 0, off_dypk = 0, off_wpk = 0, off_wtpk = 0, off_part = 0, off_dbpart = 0;
   size_t sz_xpk = 0, sz_dypk = 0, sz_wpk = 0, sz_wtpk = 0, sz_part = 0, sz_dbpart = 0;
+  // 3xTF32: byte offset from each packed operand's hi plane to its lo plane (0: one plane)
+  long long lo_xpk = 0, lo_dypk = 0, lo_wpk = 0, lo_wtpk = 0;
   int db_rows = 0;
   size_t ws_fwd = 0, ws_dgrad = 0, ws_wgrad = 0, ws_bwd = 0;
   double plan_us = 0;
@@ -651,15 +660,19 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.m_units = (int)cdiv(pp.m_tiles, pp.cg);
   if (mode == MODE_WGRAD) {
     pp.splits = choose_splits(pp.m_units * pp.n_tiles, pp.kb_total, pp.bn,
-                              pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg);
+                              pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg, P.x3);
     pp.kb_per_split = (int)cdiv(pp.kb_total, pp.splits);
     pp.splits = (int)cdiv(pp.kb_total, pp.kb_per_split);
   } else {
     pp.splits = 1;
     pp.kb_per_split = pp.kb_total;
   }
-  const int a_bytes = mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow;
-  const int b_row = mode == MODE_WGRAD ? BKP * elem : pp.krow;
+  const int planes = P.x3 ? 2 : 1;   // 3xTF32: hi and lo plane of every operand in the stage
+  // 3xTF32 accumulation chunk (shape-only constant: 16 k-blocks = K 512): bounds the error of the
+  // tensor core's round-toward-zero accumulation to ~1e-6 normwise
+  pp.chunk_kb = P.x3 ? 16 : 0;
+  const int a_bytes = planes * (mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow);
+  const int b_row = planes * (mode == MODE_WGRAD ? BKP * elem : pp.krow);
   // forward: the bias vector is staged once per CTA in smem (every column a tile can touch)
   pp.bias_floats = (mode == MODE_FWD) ? (int)rup((long long)pp.n_tiles * pp.bn, 32) + 32 : 0;
   const int budget = P.smem_cap - 1024 - 1024 - 4 * pp.bias_floats;   // alignment slack; barriers, TMEM slot
@@ -686,7 +699,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16 + 16 + 4 * pp.bias_floats;
   pp.tiles = pp.m_units * pp.n_tiles * pp.splits;   // work units (tile pairs for cg = 2)
 
-  void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg);
+  void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg, P.x3);
   // The attribute is per function (not per plan): always allow the largest tile of any plan.
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
@@ -695,11 +708,12 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   // TMEM term: the CUDA runtime admits one TMEM-allocating (tcgen05) CTA per SM regardless of
   // the columns it asks for (measured with tools/occ_probe2.cu; R16), so the record
   // charges the whole per-SM TMEM to each CTA.
-  glp_kernel_attr_t ka{IGEMM_THREADS, fa.numRegs, pp.smem + (int)fa.sharedSizeBytes,
+  pp.threads = igemm_threads(P.x3);
+  glp_kernel_attr_t ka{pp.threads, fa.numRegs, pp.smem + (int)fa.sharedSizeBytes,
                        L.tmem_cols_per_sm > 0 ? L.tmem_cols_per_sm : pp.tmem_cols};
   pp.ctas_per_sm = ctas_per_sm_closed_form(L, ka);
   int rt = 0;
-  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, IGEMM_THREADS, pp.smem));
+  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rt, fn, pp.threads, pp.smem));
   pp.ctas_runtime = rt;
   if (pp.ctas_per_sm < 1) return fail(GLP_ERR_INTERNAL, "kernel does not fit on an SM");
   const int slots = P.sm_count * pp.ctas_per_sm / pp.cg;   // resident work-unit slots
@@ -716,6 +730,12 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.grid = std::max(1, grid) * pp.cg;   // CTAs (pairs are clusters of 2)
   return GLP_OK;
 }
+
+// The tensor maps of one pass: A (activation gather), B (dense operand) and, for 3xTF32 plans,
+// the same two over the lo planes.
+struct Maps {
+  CUtensorMap a, b, a2, b2;
+};
 
 glp_status_t validate_ptrs(std::initializer_list<const void *> ps) {
   for (const void *p : ps) {
@@ -767,8 +787,12 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   }
   g.cbs = g.cp / (pp.krow / P.elem);
   p.a_tma = pp.a_tma;
+  p.lo_off_a = (mode == MODE_DGRAD) ? P.lo_dypk : P.lo_xpk;
+  p.chunk_kb = pp.chunk_kb;
+#ifdef GLP_DIAG
   p.dbg_skip = P.dbg_skip;
   p.dbg_clk = P.dbg_clk;
+#endif
   g.div_hw = FastDiv((uint32_t)g.pix_hw);
   g.div_w = FastDiv((uint32_t)g.pix_w);
   g.div_cp = FastDiv((uint32_t)g.cp);
@@ -793,12 +817,12 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
 
 template <int MODE>
 glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
-                          const CUtensorMap &mapB, const CUtensorMap &mapA, cudaStream_t st) {
-  void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg);
+                          const Maps &m, cudaStream_t st) {
+  void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg, P.x3);
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof(cfg));
   cfg.gridDim = dim3((unsigned)pp.grid);
-  cfg.blockDim = dim3(IGEMM_THREADS);
+  cfg.blockDim = dim3((unsigned)pp.threads);
   cfg.dynamicSmemBytes = (size_t)pp.smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[2];
@@ -810,8 +834,11 @@ glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmPa
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = P.pdl ? 2 : 1;
-  void *args[] = {const_cast<IgemmParams *>(&p), const_cast<CUtensorMap *>(&mapB),
-                  const_cast<CUtensorMap *>(&mapA)};
+  // single-plane plans pass their hi maps again in the lo slots (never read)
+  const CUtensorMap &b2 = P.x3 ? m.b2 : m.b, &a2 = P.x3 ? m.a2 : m.a;
+  void *args[] = {const_cast<IgemmParams *>(&p), const_cast<CUtensorMap *>(&m.b),
+                  const_cast<CUtensorMap *>(&m.a), const_cast<CUtensorMap *>(&b2),
+                  const_cast<CUtensorMap *>(&a2)};
   GLP_CUDA(cudaLaunchKernelExC(&cfg, fn, args));
   GLP_LAUNCH_CHECK("igemm_kernel");
   return GLP_OK;
@@ -854,9 +881,10 @@ DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
   return a;
 }
 
-glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, int C, int HW,
-                             int Cp, float *db_part, cudaStream_t st, int Ws = 1, int Wd = 1,
-                             int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1,
+// lo: byte offset of dst's lo plane (3xTF32 plans: the region's lo_* offset; 0 otherwise)
+glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, long long lo, int C,
+                             int HW, int Cp, float *db_part, cudaStream_t st, int Ws = 1,
+                             int Wd = 1, int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1,
                              int img_c = -1) {
   if (HWd < 0) HWd = HW;   // default: dense destination (Ws == Wd)
   if (img_c < 0) img_c = C;   // default: the source holds exactly C channels per image
@@ -865,8 +893,8 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
   if (db_part == nullptr && Cp * P.elem <= 32 && Ws == Wd && co_off == 0 && Cw == Cp) {
     const size_t n = (size_t)P.d.N * HW;
     const int g = (int)std::min<size_t>(cdiv((long long)n, 256), 148 * 32);
-    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c));
-    else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<4>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c));
+    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<2>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c, 0LL));
+    else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc_small<4>, dim3(g), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, img_c, lo));
     GLP_LAUNCH_CHECK("pack_nchw_to_nhwc_small");
     return GLP_OK;
   }
@@ -875,14 +903,14 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, i
   const int nt = (int)cdiv(P.d.Co, 32);
   if (!P.pack_block) {   // warp-tiled pack (default)
     dim3 gw((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, 8 * PACKW_ROWS));
-    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<2>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
-    else GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<4>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
+    if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<2>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c, 0LL));
+    else GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<4>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c, lo));
     GLP_LAUNCH_CHECK("pack_act_warp");
     return GLP_OK;
   }
   dim3 grid((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, PACK_PT));
-  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
-  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c));
+  if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<2>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c, 0LL));
+  else GLP_CUDA(launch_pdl(P.pdl, pack_nchw_to_nhwc<4>, dim3(grid), dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c, lo));
   GLP_LAUNCH_CHECK("pack_nchw_to_nhwc");
   return GLP_OK;
 }
@@ -898,12 +926,12 @@ glp_status_t launch_pack_dy(const glp_plan_s &P, const BrIn &dy, uint8_t *ws, bo
   const int Ws = P.halo ? d.Wo : 1, Wd = P.halo ? P.dxg.W : 1;
   const int HWd = P.halo ? P.dxg.H * P.dxg.W : -1;
   if (dy.n <= 1)
-    return launch_pack_act(P, dy.p[0], ws + P.off_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
+    return launch_pack_act(P, dy.p[0], ws + P.off_dypk, P.lo_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
                            HWd, 0, -1, -1, P.y_img_c);
   for (int b = 0; b < dy.n; ++b) {
     const int off = d.br_off[b], cb = d.br_off[b + 1] - off;
     const int cw = (b == dy.n - 1) ? P.Cop - off : cb;
-    glp_status_t s = launch_pack_act(P, dy.p[b], ws + P.off_dypk, cb, d.Ho * d.Wo, P.Cop, dbp, st,
+    glp_status_t s = launch_pack_act(P, dy.p[b], ws + P.off_dypk, P.lo_dypk, cb, d.Ho * d.Wo, P.Cop, dbp, st,
                                      Ws, Wd, HWd, off, cw, d.Co);
     if (s) return s;
   }
@@ -919,21 +947,22 @@ glp_status_t run_pack_w_fwd_one(glp_plan_s &P, const float *w, int co_off, int C
   d.Co = Co;   // rows [co_off, co_off + Co) of the forward B operand
   void *wpk = ws + P.off_wpk + (size_t)co_off * P.fwd.Kpad * P.elem;
   const size_t wn = (size_t)d.Co * P.fwd.Kpad;
+  const long long lo = P.lo_wpk;
   if (P.s2d) {
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<2>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<2>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<4>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<4>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad, lo));
   } else if ((size_t)d.C * P.taps * 4 <= 48 * 1024) {
     const size_t sm = (size_t)d.C * P.taps * 4;
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<2>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<2>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<4>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_rows<4>, dim3((unsigned)d.Co), dim3(256), sm, st, w, wpk, d.C, P.taps, P.Cpx, P.fwd.Kpad, lo));
   } else if (P.elem == 2) {
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<2>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad));
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<2>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad, 0LL));
   } else {
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<4>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad));
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd<4>, dim3(dim3((unsigned)cdiv(P.fwd.Kpad, 256), (unsigned)d.Co)), dim3(256), 0, st, w, wpk, d.Co, d.C, P.taps, P.Cpx, P.fwd.Kpad, lo));
   }
   GLP_LAUNCH_CHECK("pack_w_fwd");
   return GLP_OK;
@@ -957,16 +986,16 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
     const dim3 grid((unsigned)cdiv(px, 128));
     if (P.s2d == 4 && d.C == 3) {   // CaffeNet conv1: compile-time geometry
       if (P.elem == 2)
-        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<2, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<2, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
       else
-        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<4, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<4, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
       GLP_LAUNCH_CHECK("pack_s2d_warp_t");
       return GLP_OK;
     }
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<2>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<2>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<4>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<4>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
     GLP_LAUNCH_CHECK("pack_s2d_warp");
     return GLP_OK;
   }
@@ -979,14 +1008,14 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
     const int rows = d.N * P.dxg.H;
     dim3 grid((unsigned)std::min(rows, P.sm_count * std::max(1, P.s2d_blocks)));
     if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
     GLP_LAUNCH_CHECK("pack_s2d");
     return GLP_OK;
   }
-  return launch_pack_act(P, x, dst, d.C, d.H * d.W, P.Cpx, nullptr, st, 1, 1, -1, 0, -1, -1,
-                         P.x_img_c);
+  return launch_pack_act(P, x, dst, P.lo_xpk, d.C, d.H * d.W, P.Cpx, nullptr, st, 1, 1, -1, 0, -1,
+                         -1, P.x_img_c);
 }
 
 glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStream_t st) {
@@ -1002,13 +1031,13 @@ glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStr
     const size_t sm = (size_t)co * P.taps * 4;
     if (sm <= 48 * 1024) {
       if (P.elem == 2)
-        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<2>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<2>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, 0LL));
       else
-        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<4>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<4>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, P.lo_wtpk));
     } else if (P.elem == 2)
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, P.lo_wtpk));
     GLP_LAUNCH_CHECK("pack_w_dgrad");
   }
   return GLP_OK;
@@ -1030,9 +1059,9 @@ glp_status_t run_pack_w_both(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStre
   void *wp = ws + P.off_wpk, *wt = ws + P.off_wtpk;
   const int flip = P.dgrad.a_tma;
   if (P.elem == 2)
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<2>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip));
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<2>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip, 0LL, 0LL));
   else
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<4>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip));
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<4>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip, P.lo_wpk, P.lo_wtpk));
   GLP_LAUNCH_CHECK("pack_w_both");
   return GLP_OK;
 }
@@ -1054,24 +1083,26 @@ BrOut br_out(const glp_plan_s &P, int n, float *const *ptrs) {
 }
 
 template <typename F>
-glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, CUtensorMap &a, CUtensorMap &b,
-                         F encode) {
+glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, Maps &m, F encode) {
   std::lock_guard<std::mutex> lk(P.maps.mu);
   for (auto &e : P.maps.e[pass])
     if (e.ws == ws) {
-      a = e.a;
-      b = e.b;
+      m.a = e.a;
+      m.b = e.b;
+      m.a2 = e.a2;
+      m.b2 = e.b2;
       return GLP_OK;
     }
-  memset(&a, 0, sizeof(a));
-  memset(&b, 0, sizeof(b));
-  glp_status_t s = encode(a, b);
+  memset(&m, 0, sizeof(m));
+  glp_status_t s = encode(m);
   if (s) return s;
   auto &e = P.maps.e[pass][P.maps.next[pass]];
   P.maps.next[pass] = (P.maps.next[pass] + 1) % 8;
   e.ws = ws;
-  e.a = a;
-  e.b = b;
+  e.a = m.a;
+  e.b = m.b;
+  e.a2 = m.a2;
+  e.b2 = m.b2;
   return GLP_OK;
 }
 
@@ -1098,15 +1129,16 @@ glp_status_t run_fwd_halo(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
                           cudaStream_t st) {
   const glp_conv_desc_s &d = P.dxg;
   const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x'
-  CUtensorMap mapX, mapW;
-  glp_status_t s = cached_maps(P, 0, ws, mapX, mapW, [&](CUtensorMap &X, CUtensorMap &Wm) {
-    glp_status_t r = encode_2d(&X, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
+  Maps m;
+  glp_status_t s = cached_maps(P, 0, ws, m, [&](Maps &q) {
+    glp_status_t r = encode_2d(&q.a, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
                                64u, (uint32_t)P.hf.halo_rows, CU_TENSOR_MAP_SWIZZLE_128B);
     if (r) return r;
-    return encode_2d(&Wm, 2, ws + P.off_wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co,
+    return encode_2d(&q.b, 2, ws + P.off_wpk, (uint64_t)P.fwd.Kpad, (uint64_t)d.Co,
                      (uint64_t)P.fwd.Kpad * 2, 64u, (uint32_t)(P.hf.bn / 2), CU_TENSOR_MAP_SWIZZLE_128B);
   });
   if (s) return s;
+  CUtensorMap &mapX = m.a, &mapW = m.b;
   HfwdParams p = P.hf;
   p.out = y.p[0];
   p.bias = b.p[0];
@@ -1141,15 +1173,22 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   const PassPlan &pp = P.fwd;
   void *xpk = ws + P.off_xpk, *wpk = ws + P.off_wpk;
   const int BK = pp.krow / P.elem;
-  CUtensorMap mapB, mapA;
-  glp_status_t s = cached_maps(P, 0, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
-    glp_status_t r = encode_2d(&B, P.elem, wpk, (uint64_t)pp.Kpad, (uint64_t)d.Co,
-                               (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
-                               swz_kmajor(pp.krow));
-    if (r || !pp.a_tma) return r;
-    if ((r = get_encode_im2col())) return r;
-    return encode_im2col(&A, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
-                         d.Ph - (d.Kh - 1), BK, 128, d.Sw, d.Sh, swz_kmajor(pp.krow));
+  Maps m;
+  glp_status_t s = cached_maps(P, 0, ws, m, [&](Maps &q) {
+    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
+      const long long lw = pl ? P.lo_wpk : 0, lx = pl ? P.lo_xpk : 0;
+      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<uint8_t *>(wpk) + lw,
+                                 (uint64_t)pp.Kpad, (uint64_t)d.Co, (uint64_t)pp.Kpad * P.elem,
+                                 (uint32_t)BK, (uint32_t)pp.bn_smem, swz_kmajor(pp.krow));
+      if (r) return r;
+      if (!pp.a_tma) continue;
+      if ((r = get_encode_im2col())) return r;
+      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<uint8_t *>(xpk) + lx, P.Cpx, d.W,
+                        d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1), d.Ph - (d.Kh - 1), BK, 128,
+                        d.Sw, d.Sh, swz_kmajor(pp.krow));
+      if (r) return r;
+    }
+    return GLP_OK;
   });
   if (s) return s;
   IgemmParams p = make_params(P, pp, MODE_FWD, xpk);
@@ -1160,7 +1199,7 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   p.bias_floats = pp.bias_floats;
   p.out_c = P.y_img_c;   // channels per image of y (the whole tensor for a conv group)
   p.out_hw = d.Ho * d.Wo;
-  return launch_igemm<MODE_FWD>(P, pp, p, mapB, mapA, st);
+  return launch_igemm<MODE_FWD>(P, pp, p, m, st);
 }
 
 glp_status_t encode_4d_nhwc(CUtensorMap *map, const void *ptr, int cpitch, int W, int H, int N,
@@ -1179,15 +1218,16 @@ glp_status_t encode_4d_nhwc(CUtensorMap *map, const void *ptr, int cpitch, int W
 
 glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
   const glp_conv_desc_s &d = P.d;
-  CUtensorMap mapDy, mapW;
-  glp_status_t s = cached_maps(P, 1, ws, mapDy, mapW, [&](CUtensorMap &Dy, CUtensorMap &Wm) {
-    glp_status_t r = encode_4d_nhwc(&Dy, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
+  Maps m;
+  glp_status_t s = cached_maps(P, 1, ws, m, [&](Maps &q) {
+    glp_status_t r = encode_4d_nhwc(&q.a, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
                                     (uint32_t)P.hd.WQ, (uint32_t)(P.hd.R + P.hd.K - 1));
     if (r) return r;
-    return encode_2d(&Wm, 2, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
+    return encode_2d(&q.b, 2, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
                      (uint64_t)P.dgrad.Kpad * 2, 64u, (uint32_t)(P.hd.bn / 2), CU_TENSOR_MAP_SWIZZLE_128B);
   });
   if (s) return s;
+  CUtensorMap &mapDy = m.a, &mapW = m.b;
   HdgradParams p = P.hd;
   p.out = dx;
   p.out_c = P.x_img_c;
@@ -1220,23 +1260,30 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   void *wtpk = ws + P.off_wtpk;
   const void *dypk = ws + P.off_dypk;
   const int BK = pp.krow / P.elem;
-  CUtensorMap mapB, mapA;
-  glp_status_t s = cached_maps(P, 1, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
-    glp_status_t r = encode_2d(&B, P.elem, wtpk, (uint64_t)pp.Kpad, (uint64_t)d.C,
-                               (uint64_t)pp.Kpad * P.elem, (uint32_t)BK, (uint32_t)pp.bn_smem,
-                               swz_kmajor(pp.krow));
-    if (r || !pp.a_tma) return r;
-    // dx pixel (h, w) reads dy at (h - (Kh-1-Ph) + kh', w - (Kw-1-Pw) + kw') with kh' = Kh-1-kh
-    if ((r = get_encode_im2col())) return r;
-    return encode_im2col(&A, P.elem, dypk, P.Cop, d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw),
-                         -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK, 128, 1, 1, swz_kmajor(pp.krow));
+  Maps m;
+  glp_status_t s = cached_maps(P, 1, ws, m, [&](Maps &q) {
+    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
+      const long long lw = pl ? P.lo_wtpk : 0, ld = pl ? P.lo_dypk : 0;
+      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<uint8_t *>(wtpk) + lw,
+                                 (uint64_t)pp.Kpad, (uint64_t)d.C, (uint64_t)pp.Kpad * P.elem,
+                                 (uint32_t)BK, (uint32_t)pp.bn_smem, swz_kmajor(pp.krow));
+      if (r) return r;
+      if (!pp.a_tma) continue;
+      // dx pixel (h, w) reads dy at (h - (Kh-1-Ph) + kh', w - (Kw-1-Pw) + kw') with kh' = Kh-1-kh
+      if ((r = get_encode_im2col())) return r;
+      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<const uint8_t *>(dypk) + ld, P.Cop,
+                        d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw), -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK,
+                        128, 1, 1, swz_kmajor(pp.krow));
+      if (r) return r;
+    }
+    return GLP_OK;
   });
   if (s) return s;
   IgemmParams p = make_params(P, pp, MODE_DGRAD, dypk);
   p.out = dx;
   p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
   p.out_hw = d.H * d.W;
-  return launch_igemm<MODE_DGRAD>(P, pp, p, mapB, mapA, st);
+  return launch_igemm<MODE_DGRAD>(P, pp, p, m, st);
 }
 
 glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const float *dy) {
@@ -1245,15 +1292,16 @@ glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
     return fail(GLP_ERR_INVALID_VALUE, "filter gradient: no dy recorded for this workspace "
                                        "(glp_stage_pack(GLP_PACK_DY*) first)");
   const uint64_t rows = (uint64_t)d.N * d.H * d.W;   // flat padded grid of x' and dy
-  CUtensorMap mapX, mapDy;
-  glp_status_t s = cached_maps(P, 2, ws, mapX, mapDy, [&](CUtensorMap &X, CUtensorMap &Dy) {
-    glp_status_t r = encode_2d(&X, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
+  Maps m;
+  glp_status_t s = cached_maps(P, 2, ws, m, [&](Maps &q) {
+    glp_status_t r = encode_2d(&q.a, 2, ws + P.off_xpk, (uint64_t)P.Cpx, rows, (uint64_t)P.Cpx * 2,
                                64u, (uint32_t)P.hw.halo_rows, CU_TENSOR_MAP_SWIZZLE_128B);
     if (r) return r;
-    return encode_2d(&Dy, 2, ws + P.off_dypk, (uint64_t)P.Cop, rows, (uint64_t)P.Cop * 2, 64u,
+    return encode_2d(&q.b, 2, ws + P.off_dypk, (uint64_t)P.Cop, rows, (uint64_t)P.Cop * 2, 64u,
                      (uint32_t)HW_BKP, CU_TENSOR_MAP_SWIZZLE_128B);
   });
   if (s) return s;
+  CUtensorMap &mapX = m.a, &mapDy = m.b;
   HwgradParams p = P.hw;
   p.part = reinterpret_cast<float *>(ws + P.off_part);
   p.dbg_skip = P.dbg_skip;
@@ -1295,20 +1343,28 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
   const void *xpk = ws + P.off_xpk, *dypk = ws + P.off_dypk;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
   const int BKP = 128 / P.elem, EPA = pp.krow / P.elem;
-  CUtensorMap mapB, mapA;
-  glp_status_t s = cached_maps(P, 2, ws, mapA, mapB, [&](CUtensorMap &A, CUtensorMap &B) {
-    glp_status_t r = encode_2d(&B, P.elem, dypk, (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
-                               (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
-                               swz_mnmajor(P.elem, pp.krow));
-    if (r || !pp.a_tma) return r;
-    if ((r = get_encode_im2col())) return r;
-    return encode_im2col(&A, P.elem, xpk, P.Cpx, d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1),
-                         d.Ph - (d.Kh - 1), EPA, BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
+  Maps m;
+  glp_status_t s = cached_maps(P, 2, ws, m, [&](Maps &q) {
+    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
+      const long long ld = pl ? P.lo_dypk : 0, lx = pl ? P.lo_xpk : 0;
+      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<const uint8_t *>(dypk) + ld,
+                                 (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
+                                 (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
+                                 swz_mnmajor(P.elem, pp.krow));
+      if (r) return r;
+      if (!pp.a_tma) continue;
+      if ((r = get_encode_im2col())) return r;
+      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<const uint8_t *>(xpk) + lx, P.Cpx,
+                        d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1), d.Ph - (d.Kh - 1), EPA,
+                        BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
+      if (r) return r;
+    }
+    return GLP_OK;
   });
   if (s) return s;
   IgemmParams p = make_params(P, pp, MODE_WGRAD, xpk);
   p.out = part;
-  return launch_igemm<MODE_WGRAD>(P, pp, p, mapB, mapA, st);
+  return launch_igemm<MODE_WGRAD>(P, pp, p, m, st);
 }
 
 glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw, const BrOut *db, int accumulate,
@@ -1554,7 +1610,8 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
 glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t math, int S) {
   if (!out || !d) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
   *out = nullptr;
-  if (math != GLP_MATH_FP32 && math != GLP_MATH_TF32 && math != GLP_MATH_BF16)
+  if (math != GLP_MATH_FP32 && math != GLP_MATH_TF32 && math != GLP_MATH_BF16 &&
+      math != GLP_MATH_FP32_SIMT)
     return fail(GLP_ERR_INVALID_VALUE, "unknown math mode");
   if (S < 0) return fail(GLP_ERR_INVALID_VALUE, "samples_in_flight < 0");
   const auto t0 = std::chrono::steady_clock::now();
@@ -1588,6 +1645,8 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->device = device;
   P->math = (int)math;
   P->elem = (math == GLP_MATH_BF16) ? 2 : 4;
+  P->simt = (math == GLP_MATH_FP32_SIMT) ? 1 : 0;
+  P->x3 = (math == GLP_MATH_FP32) ? 1 : 0;
   P->sm_count = prop.multiProcessorCount;
   P->s_override = S;
   if (const char *e = getenv("GLP_CTA_GROUP")) P->allow_cg2 = (atoi(e) != 1);
@@ -1623,7 +1682,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->dxg = *d;
   P->Cpx = P->Cp;
   P->tapsx = P->taps;
-  if (math != GLP_MATH_FP32 && d->Sh == d->Sw && d->Sh > 1 && d->Kh == d->Kw && d->Ph == d->Pw &&
+  if (!P->simt && d->Sh == d->Sw && d->Sh > 1 && d->Kh == d->Kw && d->Ph == d->Pw &&
       d->Kh >= d->Sh) {
     const int S2 = d->Sh, Ks = (int)cdiv(d->Kh, S2), cs = S2 * S2 * d->C;
     const int cps = (int)rup(cs, 32);
@@ -1652,7 +1711,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   L.smem_reserved_per_cta = (int)prop.reservedSharedMemPerBlock;
 
   glp_status_t s = GLP_OK;
-  if (d->nbr > 1 && math != GLP_MATH_FP32) {
+  if (d->nbr > 1 && !P->simt) {
     // a branch's packed channels start on a 16-byte chunk of the pitch (8 bf16 / 4 tf32)
     const int ch = 16 / P->elem;
     for (int b = 1; b < d->nbr; ++b)
@@ -1663,7 +1722,7 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
                                                std::to_string(ch) + " == 0");
       }
   }
-  if (math != GLP_MATH_FP32) {
+  if (!P->simt) {
     if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
         (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {
       delete P;
@@ -1677,12 +1736,24 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
     }
     const glp_conv_desc_s &c = *d;
     // x region: the forward/filter-gradient operand, or the direct packing of glp_debug_im2col
-    P->sz_xpk = align1k(std::max((size_t)c.N * c.H * c.W * P->Cp,
-                                 (size_t)c.N * P->dxg.H * P->dxg.W * P->Cpx) * P->elem);
+    // every packed operand region holds one plane, or (3xTF32) its hi plane then its lo plane
+    const size_t pl_x = align1k(std::max((size_t)c.N * c.H * c.W * P->Cp,
+                                         (size_t)c.N * P->dxg.H * P->dxg.W * P->Cpx) * P->elem);
     const size_t dy_hw = P->halo ? (size_t)P->dxg.H * P->dxg.W : (size_t)c.Ho * c.Wo;
-    P->sz_dypk = align1k((size_t)c.N * dy_hw * P->Cop * P->elem);
-    P->sz_wpk = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
-    P->sz_wtpk = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
+    const size_t pl_dy = align1k((size_t)c.N * dy_hw * P->Cop * P->elem);
+    const size_t pl_w = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
+    const size_t pl_wt = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
+    const size_t planes = P->x3 ? 2 : 1;
+    P->sz_xpk = planes * pl_x;
+    P->sz_dypk = planes * pl_dy;
+    P->sz_wpk = planes * pl_w;
+    P->sz_wtpk = planes * pl_wt;
+    if (P->x3) {
+      P->lo_xpk = (long long)pl_x;
+      P->lo_dypk = (long long)pl_dy;
+      P->lo_wpk = (long long)pl_w;
+      P->lo_wtpk = (long long)pl_wt;
+    }
     P->sz_part = P->halo ? align1k((size_t)P->hw.splits * P->hw.mpad * P->hw.ld * 4)
                          : align1k((size_t)P->wgrad.splits * P->wgrad.m_units * P->wgrad.cg * 128 *
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
@@ -1741,7 +1812,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->stages_fwd = P->fwd.stages;
   I->stages_bwd_data = P->dgrad.stages;
   I->stages_bwd_filter = P->halo ? P->hw.stages : P->wgrad.stages;
-  I->splits_wgrad = P->math == GLP_MATH_FP32 ? P->simt_splits : P->halo ? P->hw.splits : P->wgrad.splits;
+  I->splits_wgrad = P->simt ? P->simt_splits : P->halo ? P->hw.splits : P->wgrad.splits;
   I->tiles_fwd = P->fwd.tiles;
   I->tiles_bwd_data = P->dgrad.tiles;
   I->tiles_bwd_filter = P->halo ? P->hw.splits : P->wgrad.tiles;
@@ -1772,9 +1843,9 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
 
 glp_status_t glp_plan_kernel_attr(glp_plan_t P, int which, glp_kernel_attr_t *a, int *model, int *rt) {
   if (!P || !a || !model || !rt || which < 0 || which > 2) return fail(GLP_ERR_INVALID_VALUE, "bad argument");
-  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no persistent kernel");
+  if (P->simt) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no persistent kernel");
   const PassPlan &pp = which == 0 ? P->fwd : which == 1 ? P->dgrad : P->wgrad;
-  *a = glp_kernel_attr_t{IGEMM_THREADS, pp.regs, pp.smem, pp.tmem_cols};
+  *a = glp_kernel_attr_t{pp.threads, pp.regs, pp.smem, pp.tmem_cols};
   *model = pp.ctas_per_sm;
   *rt = pp.ctas_runtime;
   return GLP_OK;
@@ -1817,11 +1888,11 @@ glp_status_t glp_conv_fwd(glp_plan_t P, const float *x, const float *w, const fl
   if (b && (reinterpret_cast<uintptr_t>(b) % 4)) return fail(GLP_ERR_INVALID_VALUE, "bias misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  if (!P->simt && (s = get_encode())) return s;
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
     float *yg = y + o.y;
-    if (P->math == GLP_MATH_FP32) {
+    if (P->simt) {
       const size_t n = (size_t)P->d.N * P->d.Co * P->d.Ho * P->d.Wo;
       simt_fwd<<<ew_grid(n), 256, 0, st>>>(geomP(*P), x + o.x, w + o.w, offc(b, o.b), yg);
       GLP_LAUNCH_CHECK("simt_fwd");
@@ -1840,10 +1911,10 @@ glp_status_t glp_conv_bwd_data(glp_plan_t P, const float *dy, const float *w, fl
   if (s) return s;
   if ((s = check_ws(P, ws, ws_bytes, P->ws_dgrad))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  if (!P->simt && (s = get_encode())) return s;
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
-    if (P->math == GLP_MATH_FP32) {
+    if (P->simt) {
       const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
       simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geomP(*P), dy + o.y, w + o.w, dx + o.x);
       GLP_LAUNCH_CHECK("simt_dgrad");
@@ -1866,12 +1937,12 @@ glp_status_t glp_conv_bwd_filter(glp_plan_t P, const float *x, const float *dy, 
   if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_wgrad))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  if (!P->simt && (s = get_encode())) return s;
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
     uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
     float *dwg = dw + o.w, *dbg = offm(db, o.b);
-    if (P->math == GLP_MATH_FP32) {
+    if (P->simt) {
       if ((s = run_wgrad_simt(*P, x + o.x, dy + o.y, dwg, dbg, accumulate ? 1 : 0, wsb, st))) return s;
       continue;
     }
@@ -1895,12 +1966,12 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
   if (db && (reinterpret_cast<uintptr_t>(db) % 4)) return fail(GLP_ERR_INVALID_VALUE, "db misaligned");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_bwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (P->math != GLP_MATH_FP32 && (s = get_encode())) return s;
+  if (!P->simt && (s = get_encode())) return s;
   for (int g = 0; g < P->groups; ++g) {
     const GOff o = goff(P, g);
     uint8_t *wsb = static_cast<uint8_t *>(ws) + o.ws;
     float *dwg = dw + o.w, *dbg = offm(db, o.b);
-    if (P->math == GLP_MATH_FP32) {
+    if (P->simt) {
       if (dx) {
         const size_t n = (size_t)P->d.N * P->d.C * P->d.H * P->d.W;
         simt_dgrad<<<ew_grid(n), 256, 0, st>>>(geomP(*P), dy + o.y, w + o.w, dx + o.x);
@@ -1919,7 +1990,7 @@ glp_status_t glp_conv_bwd(glp_plan_t P, const float *x, const float *dy, const f
 
 static glp_status_t stage_check(glp_plan_t P, void *ws, size_t ws_bytes) {
   if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
-  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "staged API needs a tensor-core plan");
+  if (P->simt) return fail(GLP_ERR_NOT_SUPPORTED, "staged API needs a tensor-core plan");
   glp_status_t s = check_ws(P, ws, ws_bytes, P->ws_bwd);
   if (s) return s;
   return get_encode();
@@ -2028,7 +2099,7 @@ static glp_status_t group_tables(glp_plan_t P, const float *const *in, BrIn &t, 
 }
 static glp_status_t group_check(glp_plan_t P, void *ws, size_t ws_bytes, size_t need) {
   if (!P) return fail(GLP_ERR_INVALID_VALUE, "plan is NULL");
-  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "fused groups need a tensor-core plan");
+  if (P->simt) return fail(GLP_ERR_NOT_SUPPORTED, "fused groups need a tensor-core plan");
   glp_status_t s = check_ws(P, ws, ws_bytes, need);
   if (s) return s;
   return get_encode();
@@ -2126,12 +2197,13 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   if (s) return s;
   if (n < 0 || n >= P->d.N) return fail(GLP_ERR_INVALID_VALUE, "sample index out of range");
   if (P->groups > 1) return fail(GLP_ERR_NOT_SUPPORTED, "debug im2col of a grouped layer");
-  if (P->math == GLP_MATH_FP32) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no packed operand");
+  if (P->simt) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no packed operand");
   if ((s = check_ws(P, ws, ws_bytes, P->ws_fwd))) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   void *xpk = wsb + P->off_xpk;
-  if ((s = launch_pack_act(*P, x, xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st))) return s;
+  if ((s = launch_pack_act(*P, x, xpk, P->lo_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st)))
+    return s;
   // the direct (non space-to-depth) gather geometry of the layer
   glp_plan_s Q = *P;
   Q.s2d = 0;
@@ -2213,7 +2285,7 @@ glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t d, int device, glp
   glp_device_limits_b200(&L);
   glp_kernel_attr_t ka{256, 0, 0, 0};
   int blocks = (int)std::max<long long>(1, cdiv((long long)Q->d1.Co * Q->d1.Ho * Q->d1.Wo, 256));
-  if (math != GLP_MATH_FP32) {
+  if (math != GLP_MATH_FP32_SIMT) {
     int m = 0, r = 0;
     glp_plan_kernel_attr(Q->plan1, 0, &ka, &m, &r);
     blocks = Q->plan1->fwd.grid;
@@ -2274,7 +2346,7 @@ glp_status_t glp_pool_conv_fwd(glp_pool_t Q, const float *x, const float *w, con
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   const glp_conv_desc_s &d = Q->d1;
   const size_t xs = (size_t)d.C * d.H * d.W, ys = (size_t)d.Co * d.Ho * d.Wo;
-  const bool tc = Q->math != GLP_MATH_FP32;
+  const bool tc = Q->math != GLP_MATH_FP32_SIMT;
   if ((s = pool_fork(Q, st))) return s;
   // internal calls: per-sample slices are only 4-byte aligned (e.g. 3 x 227 x 227 floats)
   glp_plan_s &P1 = *Q->plan1;
@@ -2313,7 +2385,7 @@ glp_status_t glp_pool_conv_bwd(glp_pool_t Q, const float *x, const float *dy, co
   const size_t xs = (size_t)d.C * d.H * d.W, ys = (size_t)d.Co * d.Ho * d.Wo;
   const size_t wsz = (size_t)d.Co * d.C * d.Kh * d.Kw;
   float *acc = reinterpret_cast<float *>(wsb + (size_t)Q->S * Q->slot_ws);
-  const bool tc = Q->math != GLP_MATH_FP32;
+  const bool tc = Q->math != GLP_MATH_FP32_SIMT;
   if ((s = pool_fork(Q, st))) return s;
   // The paper's concurrent streams would all accumulate (beta = 1) into one dW and race
   // (P262-264); each stream here owns an accumulator, summed in stream order at the join.

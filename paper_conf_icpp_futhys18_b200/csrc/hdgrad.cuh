@@ -118,7 +118,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
 
   if (warp == 4) {
     // ===================================== producer ========================================
-    const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+    const bool la = !GLP_SKIP(p, 1), lb = !GLP_SKIP(p, 2);
     const int half = p.bn / 2;
     int as = 0, bs = 0;
     uint32_t aph = 0, bph = 0;
@@ -155,7 +155,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
   } else if (warp == 5 && leader) {
     // ===================================== MMA issuer ======================================
     const uint32_t idesc = make_idesc(1u, 0u, 0u, 256u, (uint32_t)p.bn);
-    const bool skip_mma = (p.dbg_skip & 4) != 0;
+    const bool skip_mma = GLP_SKIP(p, 4);
     int as = 0, bs = 0;
     uint32_t aph = 0, bph = 0, it = 0;
     for (int u = unit0; u < p.units; u += ustep, ++it) {
@@ -179,7 +179,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
           for (int j = 0; j < nsub; ++j) {
             // (diagnostics, GLP_DEBUG_SKIP bit 5: drop the kw row shift, i.e. only 8-row-aligned
             // starts; results wrong — isolates the cost of misaligned operand starts)
-            const uint64_t sh = (uint64_t)((kh * p.WQ + ((p.dbg_skip & 32) ? 0 : kw)) * 8);
+            const uint64_t sh = (uint64_t)((kh * p.WQ + (GLP_SKIP(p, 32) ? 0 : kw)) * 8);
             const uint64_t db = db0 + (uint64_t)(j * (p.b_tap_bytes >> 4));
             const uint32_t acc = (cb | t0 | j) ? 1u : 0u;
             if (!skip_mma || (cb | t0 | j) == 0) mma_kblock_e<0, 2, 4, 2>(d0, da0 + sh, db, idesc, acc);
@@ -218,7 +218,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
         const int tile = 2 * u + my_tile_of_unit_offset;
         const int n = tile / p.tiles_img, r0 = (tile - n * p.tiles_img) * p.R;
         const int h = r0 + rr;
-        const bool mv = tile < total_tiles && h < p.H && ww < p.W && !(p.dbg_skip & 8);
+        const bool mv = tile < total_tiles && h < p.H && ww < p.W && !GLP_SKIP(p, 8);
         float *ob = p.out + (size_t)n * p.out_c * plane + (size_t)h * p.W + ww;
         const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
         for (int c0 = 0; c0 < p.bn; c0 += 32) {

@@ -116,7 +116,7 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
     for (int t = 0; t < p.taps; ++t)
       tma_load_2d_cg2_e(sB + (uint32_t)(t * p.b_tap_bytes), &tmapW, mapa_shared(bfull, 0), t * 64,
                         (int)rank * half);
-    const bool la = !(p.dbg_skip & 1);
+    const bool la = !GLP_SKIP(p, 1);
     const uint32_t tx = la ? (uint32_t)(2 * p.halo_rows * 128) : 0u;
     int rs = 0;
     uint32_t rph = 0;
@@ -137,7 +137,7 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
     mbar_wait(bfull, 0);
     int rs = 0;
     uint32_t rph = 0, it = 0;
-    const bool skip_mma = (p.dbg_skip & 4) != 0;
+    const bool skip_mma = GLP_SKIP(p, 4);
     for (int u = unit0; u < p.units; u += ustep, ++it) {
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
       mbar_wait(tempty(a), aph ^ 1u);
@@ -183,7 +183,7 @@ __global__ void __launch_bounds__(HF_THREADS, 1)
       uint32_t n = 0, rem = 0, h = 0, w = 0;
       p.div_img.divmod((uint32_t)min(q, p.rows - 1), n, rem);
       p.div_w.divmod(rem, h, w);
-      const bool mv = q < p.rows && (int)h < p.ho && (int)w < p.wo && !(p.dbg_skip & 8);
+      const bool mv = q < p.rows && (int)h < p.ho && (int)w < p.wo && !GLP_SKIP(p, 8);
       float *ob = p.out + (size_t)n * p.out_c * plane + (size_t)h * p.wo + w;
       const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + a * (uint32_t)p.acc_cols;
       auto store_chunk = [&](int c0, uint32_t (&v)[32]) {

@@ -115,7 +115,7 @@ __global__ void __launch_bounds__(hw_threads(NCG), 1)
     // ===================================== producer ========================================
     int rs = 0;
     uint32_t rph = 0;
-    const bool la = !(p.dbg_skip & 1), lb = !FDY && !(p.dbg_skip & 2);
+    const bool la = !GLP_SKIP(p, 1), lb = !FDY && !GLP_SKIP(p, 2);
     const int nb = (p.bn + 63) / 64;
     const uint32_t tx = (la ? (uint32_t)(p.halo_rows * 128) : 0u) + (lb ? (uint32_t)p.b_bytes : 0u);
     for (int kb = kb0; kb < kb1; ++kb) {
@@ -144,7 +144,7 @@ __global__ void __launch_bounds__(hw_threads(NCG), 1)
       const uint32_t sA = base + (uint32_t)rs * stage_bytes, sB = sA + (uint32_t)p.a_bytes;
       // B: dy MN-major, 64-channel SW128 atoms of HW_BKP rows (LBO = one atom column)
       const uint64_t db = make_sdesc(sB, HW_BKP * 128u, 1024u, 2u);
-      for (int j = 0; j < p.n_acc && !(p.dbg_skip & 4); ++j) {
+      for (int j = 0; j < p.n_acc && !GLP_SKIP(p, 4); ++j) {
         const uint32_t sa = sA + (uint32_t)p.shift_a[j] * 128u;
         const uint64_t da =
             make_sdesc(sa, (uint32_t)(p.shift_b[j] - p.shift_a[j]) * 128u, 1024u, 2u);

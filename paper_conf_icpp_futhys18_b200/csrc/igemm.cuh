@@ -30,10 +30,10 @@
 
 namespace glp {
 
-constexpr int IGEMM_THREADS = 288;
-#ifndef GLP_TMA_WARP
-#define GLP_TMA_WARP 4
-#endif
+constexpr int IGEMM_THREADS = 288;      // 4 epilogue warps, 4 producer warps, 1 MMA warp
+constexpr int IGEMM_X3_THREADS = 512;   // 3xTF32: 8 epilogue warps, 4 producer, 1 MMA, 3 idle
+constexpr int X3_EPI_REGS = 192, X3_OTHER_REGS = 64;   // setmaxnreg split (sum = 2 x 128 regs)
+__host__ __device__ constexpr int igemm_threads(int x3) { return x3 ? IGEMM_X3_THREADS : IGEMM_THREADS; }
 
 template <int ELEM, int KROW>
 struct TileCfg {
@@ -97,16 +97,38 @@ __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS,
 // CG = 1: one CTA per 128-row tile.  CG = 2: CTA pairs (cluster of 2) run tcgen05.mma.cta_group::2
 // with M = 256: each CTA loads its own 128 A rows and half of the B tile (p.bn_smem = BN/2), the
 // pair leader issues the MMAs for both SMs and multicasts its commits (A by TMA only).
-template <int MODE, int ELEM, int KROW, int CG>
-__global__ void __launch_bounds__(288, 1)
+//
+// X3 = 1 (GLP_MATH_FP32, ELEM 4, KROW 128): 3xTF32.  Every operand has a hi and a lo plane (the
+// packs write hi = rna(v) and lo = rna(v - hi)); a k-block slot holds [A_hi | A_lo] and
+// [B_hi | B_lo] (each plane in the single-plane layout), the producer loads both planes (tmapA2 /
+// tmapB2 = the lo planes), and the MMA issuer runs hi*hi, hi*lo, lo*hi per k-step into the same
+// TMEM accumulator (mma_kblock_x3_e).
+// The tensor core rounds every MMA's fp32 result toward zero (measured: the normwise error of one
+// accumulator grows linearly with K, ~2^-25 of the accumulator per MMA), so a 3xTF32 tile does not
+// accumulate its whole K range in TMEM: the k-blocks are cut into chunks of p.chunk_kb (a function
+// of the shape only), each chunk accumulated from zero in one of two TMEM buffers, and the 8
+// epilogue warps add the chunks in fp32 (round-to-nearest) in registers -- the row's running sum,
+// half of the tile's columns per warp (warp w: TMEM lanes 32*(w%4), columns half w/4) -- then
+// store the sum.  The buffers alternate chunk by chunk across tiles, so the MMA issuer never
+// waits for the final stores.
+template <int MODE, int ELEM, int KROW, int CG, int X3>
+__global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
     igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB,
-                 const __grid_constant__ CUtensorMap tmapA) {
+                 const __grid_constant__ CUtensorMap tmapA, const __grid_constant__ CUtensorMap tmapB2,
+                 const __grid_constant__ CUtensorMap tmapA2) {
   using C = TileCfg<ELEM, KROW>;
-  constexpr uint32_t A_BYTES = C::a_bytes(MODE);
+  static_assert(!X3 || (ELEM == 4 && KROW == 128), "3xTF32 uses 128-byte tf32 rows");
+  constexpr int EW = X3 ? 8 : 4;    // epilogue warps 0 .. EW-1
+  constexpr int PW = EW;            // producer warps PW .. PW+3 (TMA: warp PW alone)
+  constexpr int MW = EW + 4;        // TMEM allocator + MMA issuer
+  constexpr uint32_t PL = X3 ? 2u : 1u;                 // operand planes (hi, lo)
+  constexpr uint32_t A_BYTES1 = C::a_bytes(MODE);       // one plane of one k-block's A
+  constexpr uint32_t A_BYTES = PL * A_BYTES1;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
-  const uint32_t b_bytes = (uint32_t)p.bn_smem * C::b_row_bytes(MODE);
+  const uint32_t b_bytes1 = (uint32_t)p.bn_smem * C::b_row_bytes(MODE);
+  const uint32_t b_bytes = PL * b_bytes1;
   // a stage holds p.ksub consecutive k-blocks: [A_0 .. A_ks-1 | B_0 .. B_ks-1] (ksub = 2 halves
   // the barrier round trips per MMA; the cp.async path always uses ksub = 1)
   const uint32_t stage_bytes = (uint32_t)p.ksub * (A_BYTES + b_bytes);
@@ -138,17 +160,21 @@ __global__ void __launch_bounds__(288, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(tfull(a), 1);         // tcgen05.commit after the last k-block of a tile
-      mbar_init(tempty(a), 4 * CG);   // one arrival per epilogue warp (of both CTAs for CG2)
+      mbar_init(tempty(a), EW * CG);  // one arrival per epilogue warp (of both CTAs for CG2)
     }
     fence_mbar_init();
   }
-  if (warp == 8) {
+  if (warp == MW) {
     tmem_alloc_cg<CG>(tmem_slot, (uint32_t)p.tmem_cols);
     tmem_relinquish_cg<CG>();
   }
-  if (warp == 4 && lane == 0) {
+  if (warp == PW && lane == 0) {
     tma_prefetch(&tmapB);
     if (a_tma) tma_prefetch(&tmapA);
+    if (X3) {
+      tma_prefetch(&tmapB2);
+      if (a_tma) tma_prefetch(&tmapA2);
+    }
   }
   tc_fence_before();
   if (CG == 2) cluster_sync();
@@ -165,19 +191,26 @@ __global__ void __launch_bounds__(288, 1)
   const int ustep = (CG == 2) ? (int)(gridDim.x >> 1) : (int)gridDim.x;
   const Gather &g = p.g;
 
-  if (warp >= 4 && warp < 8) {
+  // 3xTF32: the epilogue warpgroups (warps 0-7) hold the chunk sums in registers: they raise their
+  // register budget, the other two warpgroups lower theirs (setmaxnreg at the top of each role
+  // branch, so ptxas allocates each branch with its own budget)
+  if (warp >= EW) {
+  if constexpr (X3) asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(X3_OTHER_REGS));
+  if (warp < PW + 4) {
     // ===================================== producers =======================================
-    const int pt = threadIdx.x - 128;
+    const int pt = threadIdx.x - 32 * PW;
     if (a_tma) {
-      if (warp == GLP_TMA_WARP) {   // one converged warp; each TMA / arrive is issued by an elected lane
+      if (warp == PW) {   // one converged warp; each TMA / arrive is issued by an elected lane
         int rs = 0;          // ring slot and its phase, advanced incrementally
         uint32_t rph = 0;
         uint32_t stg_addr = base;   // shared address of ring slot rs
         const int KS = p.ksub, cbs = g.cbs, KW = g.kw;
-        const bool la = !(p.dbg_skip & 1), lb = !(p.dbg_skip & 2);
+        const bool la = !GLP_SKIP(p, 1), lb = !GLP_SKIP(p, 2);
         const uint32_t kb_tx = (la ? A_BYTES : 0u) + (lb ? b_bytes : 0u);
         const uint32_t sB_off = (uint32_t)KS * A_BYTES;
+#ifdef GLP_DIAG
         long long c_empty = 0;
+#endif
         for (int tile = unit0; tile < total_tiles; tile += ustep) {
           int m_tile, n_tile, split;
           decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
@@ -221,9 +254,13 @@ __global__ void __launch_bounds__(288, 1)
           int kh = 0, kw = 0, cb = 0;       // fwd/dgrad K position (tap (kh, kw), channel block)
           for (int kbs = kb0; kbs < kb1; kbs += KS) {
             const int s = rs;
+#ifdef GLP_DIAG
             long long c0 = (p.dbg_clk != nullptr) ? clock64() : 0;
+#endif
             mbar_wait(empty(s), rph ^ 1u);
+#ifdef GLP_DIAG
             if (p.dbg_clk != nullptr) c_empty += clock64() - c0;
+#endif
             const int nsub = min(KS, kb1 - kbs);
             const uint32_t stg = stg_addr;
             const uint32_t tx = (uint32_t)nsub * kb_tx;
@@ -250,17 +287,21 @@ __global__ void __launch_bounds__(288, 1)
               const uint32_t sA = stg + (uint32_t)sub * A_BYTES;
               const uint32_t sB = stg + sB_off + (uint32_t)sub * b_bytes;
               if (MODE != MODE_WGRAD) {
-                if (la) {
-                  if (CG == 1)
-                    tma_load_im2col_4d_e(sA, &tmapA, bar, cb * C::BK, w_t, h_t, (int)n_t,
-                                         (uint16_t)kw, (uint16_t)kh);
-                  else
-                    tma_load_im2col_4d_cg2_e(sA, &tmapA, bar, cb * C::BK, w_t, h_t, (int)n_t,
-                                             (uint16_t)kw, (uint16_t)kh);
-                }
-                if (lb) {
-                  if (CG == 1) tma_load_2d_e(sB, &tmapB, bar, kb * C::BK, nb0);
-                  else tma_load_2d_cg2_e(sB, &tmapB, bar, kb * C::BK, nb0);
+#pragma unroll
+                for (uint32_t pl = 0; pl < PL; ++pl) {
+                  const CUtensorMap *mA = pl ? &tmapA2 : &tmapA, *mB = pl ? &tmapB2 : &tmapB;
+                  if (la) {
+                    if (CG == 1)
+                      tma_load_im2col_4d_e(sA + pl * A_BYTES1, mA, bar, cb * C::BK, w_t, h_t,
+                                           (int)n_t, (uint16_t)kw, (uint16_t)kh);
+                    else
+                      tma_load_im2col_4d_cg2_e(sA + pl * A_BYTES1, mA, bar, cb * C::BK, w_t, h_t,
+                                               (int)n_t, (uint16_t)kw, (uint16_t)kh);
+                  }
+                  if (lb) {
+                    if (CG == 1) tma_load_2d_e(sB + pl * b_bytes1, mB, bar, kb * C::BK, nb0);
+                    else tma_load_2d_cg2_e(sB + pl * b_bytes1, mB, bar, kb * C::BK, nb0);
+                  }
                 }
                 if (++cb == cbs) {
                   cb = 0;
@@ -274,32 +315,39 @@ __global__ void __launch_bounds__(288, 1)
                 g.div_hw.divmod((uint32_t)(kb * C::BKP), n, rem);
                 g.div_w.divmod(rem, oh, ow);
                 const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
-                if (la) {
 #pragma unroll
-                  for (int a = 0; a < NA; ++a) {
-                    if (CG == 1)
-                      tma_load_im2col_4d_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, bar, ac[a], w0,
-                                           h0, (int)n, akw[a], akh[a]);
-                    else
-                      tma_load_im2col_4d_cg2_e(sA + (uint32_t)a * C::MN_LBO, &tmapA, bar, ac[a],
-                                               w0, h0, (int)n, akw[a], akh[a]);
+                for (uint32_t pl = 0; pl < PL; ++pl) {
+                  const CUtensorMap *mA = pl ? &tmapA2 : &tmapA, *mB = pl ? &tmapB2 : &tmapB;
+                  const uint32_t pA = sA + pl * A_BYTES1, pB = sB + pl * b_bytes1;
+                  if (la) {
+#pragma unroll
+                    for (int a = 0; a < NA; ++a) {
+                      if (CG == 1)
+                        tma_load_im2col_4d_e(pA + (uint32_t)a * C::MN_LBO, mA, bar, ac[a], w0,
+                                             h0, (int)n, akw[a], akh[a]);
+                      else
+                        tma_load_im2col_4d_cg2_e(pA + (uint32_t)a * C::MN_LBO, mA, bar, ac[a],
+                                                 w0, h0, (int)n, akw[a], akh[a]);
+                    }
                   }
-                }
-                if (lb) {
-                  for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
-                    if (CG == 1)
-                      tma_load_2d_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, bar, nb0 + a * C::EPA,
-                                    kb * C::BKP);
-                    else
-                      tma_load_2d_cg2_e(sB + (uint32_t)a * C::MN_LBO, &tmapB, bar,
-                                        nb0 + a * C::EPA, kb * C::BKP);
+                  if (lb) {
+                    for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
+                      if (CG == 1)
+                        tma_load_2d_e(pB + (uint32_t)a * C::MN_LBO, mB, bar, nb0 + a * C::EPA,
+                                      kb * C::BKP);
+                      else
+                        tma_load_2d_cg2_e(pB + (uint32_t)a * C::MN_LBO, mB, bar,
+                                          nb0 + a * C::EPA, kb * C::BKP);
+                    }
                   }
                 }
               }
             }
           }
         }
+#ifdef GLP_DIAG
         if (p.dbg_clk != nullptr && lane == 0) p.dbg_clk[blockIdx.x * 4 + 3] = c_empty;
+#endif
       }
     } else if (KROW == 128 && CG == 1) {
       // -------- cp.async gather (SWIZZLE_128B layouts only) --------
@@ -350,6 +398,7 @@ __global__ void __launch_bounds__(288, 1)
             if (pt == 0) {
               mbar_arrive_expect_tx(full(s), b_bytes);
               tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
+              if (X3) tma_load_2d(sB + b_bytes1, &tmapB2, full(s), kb * C::BK, n0);
             }
             const bool kv = (int)t < g.taps;
 #pragma unroll
@@ -379,6 +428,7 @@ __global__ void __launch_bounds__(288, 1)
                 src += ((size_t)(pbase[i] + (uint32_t)(ih * g.src_w + iw)) * (uint32_t)g.src_cp + c) *
                        ELEM;
               cp_async16(sA + dst0 + (uint32_t)i * 2048u, src, ok);
+              if (X3) cp_async16(sA + A_BYTES1 + dst0 + (uint32_t)i * 2048u, src + p.lo_off_a, ok);
             }
             cp_async_mbar_arrive_noinc(full(s));
             c += C::BK;
@@ -410,9 +460,10 @@ __global__ void __launch_bounds__(288, 1)
             const uint32_t sA = base + (uint32_t)s * stage_bytes, sB = sA + A_BYTES;
             if (pt == 0) {
               mbar_arrive_expect_tx(full(s), b_bytes);
-              for (int a = 0; a < p.bn_smem / C::EPA; ++a)
-                tma_load_2d(sB + (uint32_t)a * C::MN_LBO, &tmapB, full(s), n0 + a * C::EPA,
-                            kb * C::BKP);
+              for (uint32_t pl = 0; pl < PL; ++pl)
+                for (int a = 0; a < p.bn_smem / C::EPA; ++a)
+                  tma_load_2d(sB + pl * b_bytes1 + (uint32_t)a * C::MN_LBO, pl ? &tmapB2 : &tmapB,
+                              full(s), n0 + a * C::EPA, kb * C::BKP);
             }
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
@@ -436,13 +487,14 @@ __global__ void __launch_bounds__(288, 1)
                 dst = sA + dcol + (uint32_t)(r >> 2) * 512u + (uint32_t)(r & 3) * 128u +
                       (uint32_t)((((jj >> 1) ^ (r & 3)) << 5) | ((jj & 1) << 4));
               cp_async16(dst, src, ok);
+              if (X3) cp_async16(dst + A_BYTES1, src + p.lo_off_a, ok);
             }
             cp_async_mbar_arrive_noinc(full(s));
           }
         }
       }
     }
-  } else if (warp == 8) {
+  } else if (warp == MW) {
     // ===================================== MMA issuer ======================================
     if (leader) {   // whole warp runs the loop; each tcgen05 op is issued by an elected lane
       constexpr uint32_t fmt = (ELEM == 2) ? 1u : 2u;  // BF16 : TF32
@@ -461,13 +513,69 @@ __global__ void __launch_bounds__(288, 1)
         db0 = make_sdesc(base + (uint32_t)p.ksub * A_BYTES, 16u, C::K_SBO, C::K_LAYOUT);
       }
       const uint64_t stage16 = stage_bytes >> 4, b16 = b_bytes >> 4;
+      const uint64_t alo16 = A_BYTES1 >> 4, blo16 = b_bytes1 >> 4;   // lo planes (X3)
       const int KS = p.ksub, kb_total = p.kb_total, kb_per_split = p.kb_per_split;
-      const bool skip_mma = (p.dbg_skip & 4) != 0;
+      const bool skip_mma = GLP_SKIP(p, 4);
       int rs = 0;
       uint32_t rph = 0, it = 0;
       uint64_t da = da0, db = db0;   // descriptors of ring slot rs
+#ifdef GLP_DIAG
       const bool clk = p.dbg_clk != nullptr;
+#else
+      constexpr bool clk = false;
+#endif
       long long c_t0 = clk ? clock64() : 0, c_full = 0, c_te = 0;
+      (void)c_t0;
+      if constexpr (X3) {
+        // 3xTF32: chunks of p.chunk_kb k-blocks, each accumulated from zero into TMEM buffer
+        // (chunk count & 1); the epilogue sums the chunks of a tile in fp32 registers
+        const int CK = p.chunk_kb;
+        uint32_t gch = 0;   // chunks started by this CTA
+        for (int tile = unit0; tile < total_tiles; tile += ustep) {
+          int m_tile, n_tile, split;
+          decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+          int kb0 = 0, kb1 = kb_total;
+          if (MODE == MODE_WGRAD) {
+            kb0 = split * kb_per_split;
+            kb1 = min(kb0 + kb_per_split, kb_total);
+          }
+          uint32_t acc = 0, d = tmem_base, cur = 0;
+          int next_chunk = kb0;   // first k-block of the next chunk
+          for (int kbs = kb0; kbs < kb1; kbs += KS) {
+            mbar_wait(full(rs), rph);
+            tc_fence_after();
+            const int nsub = min(KS, kb1 - kbs);
+#pragma unroll
+            for (int sub = 0; sub < 4; ++sub) {
+              if (sub >= nsub) break;
+              if (kbs + sub == next_chunk) {   // chunk boundary: publish the finished chunk
+                if (next_chunk != kb0) mma_commit_e<CG>(tfull(cur));
+                cur = gch & 1u;
+                mbar_wait(tempty(cur), ((gch >> 1) & 1u) ^ 1u);
+                tc_fence_after();
+                ++gch;
+                d = tmem_base + cur * (uint32_t)p.acc_cols;
+                acc = 0;
+                next_chunk += CK;
+              }
+              mma_kblock_x3_e<CG, KSTEPS, DSTEP>(d, da + (uint64_t)(sub * (A_BYTES >> 4)),
+                                                db + (uint64_t)sub * b16, alo16, blo16, idesc, acc);
+              acc = 1;
+            }
+            mma_commit_e<CG>(empty(rs));
+            if (++rs == S_) {
+              rs = 0;
+              rph ^= 1u;
+              da = da0;
+              db = db0;
+            } else {
+              da += stage16;
+              db += stage16;
+            }
+          }
+          mma_commit_e<CG>(tfull(cur));
+        }
+      } else
       for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
         int m_tile, n_tile, split;
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
@@ -510,23 +618,27 @@ __global__ void __launch_bounds__(288, 1)
         }
         mma_commit_e<CG>(tfull(a));
       }
+#ifdef GLP_DIAG
       if (clk && lane == 0) {
         p.dbg_clk[blockIdx.x * 4 + 0] = clock64() - c_t0;
         p.dbg_clk[blockIdx.x * 4 + 1] = c_full;
         p.dbg_clk[blockIdx.x * 4 + 2] = c_te;
       }
+#endif
     }
     __syncwarp();
+  }
   } else {
+    if constexpr (X3) asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(X3_EPI_REGS));
     // ===================================== epilogue ========================================
-    const int row = warp * 32 + lane;
+    const int row = warp * 32 + lane;   // (X3: warps 4-7 repeat the TMEM lanes of warps 0-3)
     uint32_t it = 0;
     // the whole bias vector staged once in shared memory after the barriers (16-byte aligned,
     // p.bias_floats >= every column a tile can touch, zero past N): the per-chunk global bias
     // load had its latency exposed in every chunk of every tile (ncu: STS waiting on LDG)
     const uint32_t sbias = (tmem_slot + 16u + 15u) & ~15u;
     if (MODE == MODE_FWD) {
-      for (int i = row; i < p.bias_floats; i += 128) {
+      for (int i = row; i < p.bias_floats; i += 32 * EW) {
         float bv = 0.f;
         if (i < p.N) {
           if (p.ybr.n > 1) {
@@ -538,23 +650,140 @@ __global__ void __launch_bounds__(288, 1)
         }
         sts_f32(sbias + 4u * (uint32_t)i, bv);
       }
-      named_bar_sync(1, 128);
+      named_bar_sync(1, 32 * EW);
     }
+    if constexpr (X3) {
+      // ---- 3xTF32: sum the tile's chunks in fp32 registers, then store ----
+      const int q = warp & 3, hf = warp >> 2;          // TMEM lane quadrant, column half
+      const int r = q * 32 + lane;                     // accumulator row of this thread
+      const int H0 = min(p.bn, ((p.bn + 1) / 2 + 31) & ~31);
+      const int c_lo = hf ? H0 : 0, c_hi = hf ? p.bn : H0;   // <= 128 columns, c_lo % 32 == 0
+      const int CK = p.chunk_kb;
+      uint32_t gch = 0;
+      float S[128];
+      for (int tile = unit0; tile < total_tiles; tile += ustep) {
+        int m_tile, n_tile, split;
+        decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
+        int kb0 = 0, kb1 = p.kb_total;
+        if (MODE == MODE_WGRAD) {
+          kb0 = split * p.kb_per_split;
+          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+        }
+        const int nch = (kb1 - kb0 + CK - 1) / CK;
+        for (int ch = 0; ch < nch; ++ch, ++gch) {
+          const uint32_t b = gch & 1u;
+          mbar_wait(tfull(b), (gch >> 1) & 1u);
+          tc_fence_after();
+          const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + b * (uint32_t)p.acc_cols;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            if (c_lo + 32 * j < c_hi) {
+              uint32_t v[32];
+              tmem_ld32(taddr + (uint32_t)(c_lo + 32 * j), v);
+              tmem_wait_ld_dep(v);
+              if (ch == 0) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) S[32 * j + i] = __uint_as_float(v[i]);
+              } else {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) S[32 * j + i] += __uint_as_float(v[i]);
+              }
+            }
+          }
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {   // chunk buffer drained: one arrival per warp (on the pair leader)
+            if (CG == 1) mbar_arrive_relaxed(tempty(b));
+            else mbar_arrive_cluster_relaxed(mapa_shared(tempty(b), 0));
+          }
+        }
+        const int m = (m_tile * CG + (int)rank) * C::BM + r;
+        const int n0 = n_tile * p.bn;
+        if (m >= p.M || GLP_SKIP(p, 8)) continue;
+        if (MODE != MODE_WGRAD) {
+          uint32_t n, pimg;
+          g.div_hw.divmod((uint32_t)m, n, pimg);
+          const size_t plane = (size_t)p.out_hw;
+          // columns [c_lo, c_lo + lim) of this tile exist; lanes are 32 consecutive pixels, so
+          // each store writes one channel's 128-byte pixel run; the pointer steps one plane
+          const int lim = min(c_hi, p.N - n0) - c_lo;
+          const uint32_t sb = sbias + 4u * (uint32_t)(n0 + c_lo);
+          if (MODE == MODE_FWD && p.ybr.n > 1) {   // fused sibling group: per-branch tensors
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (32 * j + i < lim)
+                  *p.ybr.at(n0 + c_lo + 32 * j + i, n, plane, pimg) =
+                      S[32 * j + i] + lds_f32(sb + 4u * (uint32_t)(32 * j + i));
+          } else {
+            float *o = p.out + (size_t)n * p.out_c * plane + pimg + (size_t)(n0 + c_lo) * plane;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              if (32 * j + 32 <= lim) {
+#pragma unroll
+                for (int i = 0; i < 32; i += 4) {
+                  float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
+                  if (MODE == MODE_FWD) b4 = lds_f32x4(sb + 4u * (uint32_t)(32 * j + i));
+                  o[0] = S[32 * j + i] + b4.x;
+                  o += plane;
+                  o[0] = S[32 * j + i + 1] + b4.y;
+                  o += plane;
+                  o[0] = S[32 * j + i + 2] + b4.z;
+                  o += plane;
+                  o[0] = S[32 * j + i + 3] + b4.w;
+                  o += plane;
+                }
+              } else if (32 * j < lim) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  if (32 * j + i < lim)
+                    o[0] = S[32 * j + i] +
+                           ((MODE == MODE_FWD) ? lds_f32(sb + 4u * (uint32_t)(32 * j + i)) : 0.f);
+                  o += plane;
+                }
+              }
+            }
+          }
+        } else {
+          float *dst = p.out + ((size_t)split * p.part_mpad + (size_t)m) * p.part_ld + n0;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const int c = c_lo + 32 * j;
+            if (c + 32 <= c_hi) {
+#pragma unroll
+              for (int i = 0; i < 32; i += 4)
+                *reinterpret_cast<float4 *>(dst + c + i) =
+                    make_float4(S[32 * j + i], S[32 * j + i + 1], S[32 * j + i + 2], S[32 * j + i + 3]);
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (c + i < c_hi) dst[c + i] = S[32 * j + i];
+            }
+          }
+        }
+      }
+    } else {
+#ifdef GLP_DIAG
     const bool clk = p.dbg_clk != nullptr && warp == 0;
+#else
+    constexpr bool clk = false;
+#endif
     long long e_t0 = clk ? clock64() : 0, e_wait = 0, e_ld = 0;
+    (void)e_t0;
     for (int tile = unit0; tile < total_tiles; tile += ustep, ++it) {
       int m_tile, n_tile, split;
       decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
       const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
       long long c0 = clk ? clock64() : 0;
       // plain try_wait (suspends in hardware); GLP_DEBUG_SKIP bit 16 selects a nanosleep back-off
-      if (p.dbg_skip & 16) mbar_wait_sleep(tfull(a), aph);
+      if (GLP_SKIP(p, 16)) mbar_wait_sleep(tfull(a), aph);
       else mbar_wait(tfull(a), aph);
       if (clk) e_wait += clock64() - c0;
       tc_fence_after();
       const int m = (m_tile * CG + (int)rank) * C::BM + row;
       const int n0 = n_tile * p.bn;
-      const bool mv = m < p.M && !(p.dbg_skip & 8);
+      const bool mv = m < p.M && !GLP_SKIP(p, 8);
       const uint32_t taddr = tmem_base + ((uint32_t)(warp * 32) << 16) + a * (uint32_t)p.acc_cols;
       if (MODE != MODE_WGRAD) {
         uint32_t n, pimg;
@@ -656,11 +885,14 @@ __global__ void __launch_bounds__(288, 1)
         else mbar_arrive_cluster_relaxed(mapa_shared(tempty(a), 0));
       }
     }
+#ifdef GLP_DIAG
     if (clk && lane == 0) {
       p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 0] = clock64() - e_t0;
       p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 1] = e_wait;
       p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 2] = e_ld;
       p.dbg_clk[gridDim.x * 4 + blockIdx.x * 4 + 3] = it;
+    }
+#endif
     }
   }
   // all tiles done: the next kernel may start launching into the teardown
@@ -669,7 +901,7 @@ __global__ void __launch_bounds__(288, 1)
   if (CG == 2) cluster_sync();
   else __syncthreads();
   tc_fence_after();
-  if (warp == 8) tmem_dealloc_cg<CG>(tmem_base, (uint32_t)p.tmem_cols);
+  if (warp == MW) tmem_dealloc_cg<CG>(tmem_base, (uint32_t)p.tmem_cols);
 }
 
 }  // namespace glp

@@ -13,32 +13,51 @@
 
 namespace glp {
 
+// 3xTF32 (GLP_MATH_FP32): the packs of a tf32 operand also write its lo plane, `lo` bytes past
+// the hi plane (lo = 0: single plane).  Plane 0 = hi = rna(v); plane 1 = lo = rna(v - hi), the
+// fp32 subtraction being exact (SURVEY §8(c) "3xTF32 hi/lo split"; oracle.split_3xtf32).
+__device__ __forceinline__ uint32_t tf32_plane(float v, int pl) {
+  const uint32_t hi = f32_to_tf32_rna(v);
+  return pl ? f32_to_tf32_rna(v - __uint_as_float(hi)) : hi;
+}
+
 template <int ELEM>
 struct PackOut;
 template <>
 struct PackOut<2> {
   __device__ __forceinline__ static void store4(void *dst, size_t idx, float a, float b, float c,
-                                                float d) {
+                                                float d, long long = 0) {
     __nv_bfloat162 lo = __floats2bfloat162_rn(a, b), hi = __floats2bfloat162_rn(c, d);
     uint2 u;
     u.x = *reinterpret_cast<uint32_t *>(&lo);
     u.y = *reinterpret_cast<uint32_t *>(&hi);
     *reinterpret_cast<uint2 *>(static_cast<__nv_bfloat16 *>(dst) + idx) = u;
   }
-  __device__ __forceinline__ static void store1(void *dst, size_t idx, float a) {
+  __device__ __forceinline__ static void store1(void *dst, size_t idx, float a, long long = 0) {
     static_cast<__nv_bfloat16 *>(dst)[idx] = __float2bfloat16_rn(a);
   }
 };
 template <>
 struct PackOut<4> {
   __device__ __forceinline__ static void store4(void *dst, size_t idx, float a, float b, float c,
-                                                float d) {
+                                                float d, long long lo = 0) {
     uint4 u = make_uint4(f32_to_tf32_rna(a), f32_to_tf32_rna(b), f32_to_tf32_rna(c),
                          f32_to_tf32_rna(d));
     *reinterpret_cast<uint4 *>(static_cast<float *>(dst) + idx) = u;
+    if (lo) {
+      uint4 l = make_uint4(f32_to_tf32_rna(a - __uint_as_float(u.x)),
+                           f32_to_tf32_rna(b - __uint_as_float(u.y)),
+                           f32_to_tf32_rna(c - __uint_as_float(u.z)),
+                           f32_to_tf32_rna(d - __uint_as_float(u.w)));
+      *reinterpret_cast<uint4 *>(static_cast<uint8_t *>(dst) + lo + idx * 4) = l;
+    }
   }
-  __device__ __forceinline__ static void store1(void *dst, size_t idx, float a) {
-    static_cast<uint32_t *>(dst)[idx] = f32_to_tf32_rna(a);
+  __device__ __forceinline__ static void store1(void *dst, size_t idx, float a, long long lo = 0) {
+    const uint32_t h = f32_to_tf32_rna(a);
+    static_cast<uint32_t *>(dst)[idx] = h;
+    if (lo)
+      *reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(dst) + lo + idx * 4) =
+          f32_to_tf32_rna(a - __uint_as_float(h));
   }
 };
 
@@ -62,7 +81,8 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
                                                          int HW, int Cp, float *__restrict__ db_part,
                                                          unsigned int *__restrict__ tickets,
                                                          int n_tickets, int Ws, int Wd, int HWd,
-                                                         int co_off, int Cw, int db_ld, int src_c) {
+                                                         int co_off, int Cw, int db_ld, int src_c,
+                                                         long long lo_off) {
   // src_c: channels per image of the source tensor (> C when packing one group's channel slice).
   // (co_off, Cw, db_ld): this call writes destination channels [co_off, co_off + Cw) of rows with
   // pitch Cp (source channels 0..C-1, zeros past C) and db_part columns co_off + c of width db_ld —
@@ -140,7 +160,7 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
 #pragma unroll
       for (int u = 0; u < CPT; u += 4)
         PackOut<ELEM>::store4(dst, o + u, tile[cl + u][pp], tile[cl + u + 1][pp],
-                              tile[cl + u + 2][pp], tile[cl + u + 3][pp]);
+                              tile[cl + u + 2][pp], tile[cl + u + 3][pp], lo_off);
     }
   }
 }
@@ -161,7 +181,8 @@ __global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ s
                                                      int Cp, float *__restrict__ db_part,
                                                      unsigned int *__restrict__ tickets,
                                                      int n_tickets, int Ws, int Wd, int HWd,
-                                                     int co_off, int Cw, int db_ld, int src_c) {
+                                                     int co_off, int Cw, int db_ld, int src_c,
+                                                     long long lo_off) {
   constexpr int RB = 32 * ELEM + 16;                    // smem bytes per staged row (+16 pad)
   __shared__ __align__(16) uint8_t slab[8][32 * RB];
   pdl_launch_dependents();
@@ -212,39 +233,44 @@ __global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ s
     if (c0 + lane < C)
       db_part[(size_t)(q0 / PACKW_ROWS) * db_ld + co_off + c0 + lane] = t[0];
   }
-  // round + pack this lane's row, stage it in the warp's slab
+  // round + pack this lane's row, stage it in the warp's slab; 3xTF32 (lo_off != 0) stages and
+  // writes the hi plane, then the lo plane through the same slab
   uint8_t *row = slab[warp] + lane * RB;
+  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;
+  for (int pl = 0; pl < planes; ++pl) {
 #pragma unroll
-  for (int j = 0; j < 32; j += 8) {
-    uint4 u0, u1;
-    if (ELEM == 2) {
-      __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
-      __nv_bfloat162 c = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
-      u0 = make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
-                      *reinterpret_cast<uint32_t *>(&c), *reinterpret_cast<uint32_t *>(&d));
-      *reinterpret_cast<uint4 *>(row + j * 2) = u0;
-    } else {
-      u0 = make_uint4(f32_to_tf32_rna(v[j]), f32_to_tf32_rna(v[j + 1]), f32_to_tf32_rna(v[j + 2]),
-                      f32_to_tf32_rna(v[j + 3]));
-      u1 = make_uint4(f32_to_tf32_rna(v[j + 4]), f32_to_tf32_rna(v[j + 5]), f32_to_tf32_rna(v[j + 6]),
-                      f32_to_tf32_rna(v[j + 7]));
-      *reinterpret_cast<uint4 *>(row + j * 4) = u0;
-      *reinterpret_cast<uint4 *>(row + j * 4 + 16) = u1;
+    for (int j = 0; j < 32; j += 8) {
+      uint4 u0, u1;
+      if (ELEM == 2) {
+        __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
+        __nv_bfloat162 c = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
+        u0 = make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
+                        *reinterpret_cast<uint32_t *>(&c), *reinterpret_cast<uint32_t *>(&d));
+        *reinterpret_cast<uint4 *>(row + j * 2) = u0;
+      } else {
+        u0 = make_uint4(tf32_plane(v[j], pl), tf32_plane(v[j + 1], pl), tf32_plane(v[j + 2], pl),
+                        tf32_plane(v[j + 3], pl));
+        u1 = make_uint4(tf32_plane(v[j + 4], pl), tf32_plane(v[j + 5], pl), tf32_plane(v[j + 6], pl),
+                        tf32_plane(v[j + 7], pl));
+        *reinterpret_cast<uint4 *>(row + j * 4) = u0;
+        *reinterpret_cast<uint4 *>(row + j * 4 + 16) = u1;
+      }
     }
-  }
-  __syncwarp();
-  // write back: chunk k of the 32-row slab -> row k / CPR, 16-byte chunk k % CPR
-  constexpr int CPR = 32 * ELEM / 16;                   // 16-byte chunks per row (4 bf16, 8 tf32)
+    __syncwarp();
+    // write back: chunk k of the 32-row slab -> row k / CPR, 16-byte chunk k % CPR
+    constexpr int CPR = 32 * ELEM / 16;                   // 16-byte chunks per row (4 bf16, 8 tf32)
+    uint8_t *dpl = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0);
 #pragma unroll
-  for (int i = 0; i < CPR; ++i) {
-    const int k = i * 32 + lane, r = k / CPR, ch = k % CPR;
-    const long long qr = q0 + r;
-    const int c = c0 + ch * (16 / ELEM);
-    if (qr < total && c < Cw) {
-      const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
-      *reinterpret_cast<uint4 *>(static_cast<uint8_t *>(dst) +
-                                 ((size_t)qr * Cp + co_off + c) * ELEM) = val;
+    for (int i = 0; i < CPR; ++i) {
+      const int k = i * 32 + lane, r = k / CPR, ch = k % CPR;
+      const long long qr = q0 + r;
+      const int c = c0 + ch * (16 / ELEM);
+      if (qr < total && c < Cw) {
+        const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+        *reinterpret_cast<uint4 *>(dpl + ((size_t)qr * Cp + co_off + c) * ELEM) = val;
+      }
     }
+    __syncwarp();
   }
 }
 
@@ -252,7 +278,8 @@ __global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ s
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__restrict__ src,
                                                                void *__restrict__ dst, int N, int C,
-                                                               int HW, int Cp, int src_c) {
+                                                               int HW, int Cp, int src_c,
+                                                               long long lo_off) {
   pdl_launch_dependents();
   pdl_wait();
   const size_t total = (size_t)N * HW;
@@ -264,7 +291,7 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc_small(const float *__re
       float a[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) a[u] = (c + u < C) ? __ldg(s + (size_t)(c + u) * HW) : 0.f;
-      PackOut<ELEM>::store4(dst, i * Cp + c, a[0], a[1], a[2], a[3]);
+      PackOut<ELEM>::store4(dst, i * Cp + c, a[0], a[1], a[2], a[3], lo_off);
     }
   }
 }
@@ -283,7 +310,7 @@ constexpr int S2D_LD = 12;   // staged source floats per thread per row (S*C*W <
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, void *__restrict__ dst,
                                                 int N, int C, int H, int W, int S, int P, int Hs,
-                                                int Ws, int Cps, int src_c) {
+                                                int Ws, int Cps, int src_c, long long lo_off) {
   extern __shared__ float rows[];   // [S*C][W] source rows (row r = dh*C + c)
   constexpr int CH = 16 / ELEM;     // channels per 16-byte chunk
   pdl_launch_dependents();
@@ -348,7 +375,7 @@ __global__ void __launch_bounds__(256) pack_s2d(const float *__restrict__ x, voi
 #pragma unroll
       for (int u = 0; u < CH; u += 4)
         PackOut<ELEM>::store4(dst, (obase + ws) * Cps + j * CH + u, o[u], o[u + 1], o[u + 2],
-                              o[u + 3]);
+                              o[u + 3], lo_off);
     }
     __syncthreads();
   }
@@ -365,7 +392,7 @@ constexpr int S2DW_MAXC = 64;
 template <int ELEM>
 __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x, void *__restrict__ dst,
                                                      int N, int C, int H, int W, int S, int P, int Hs,
-                                                     int Ws, int Cps, int src_c) {
+                                                     int Ws, int Cps, int src_c, long long lo_off) {
   constexpr int RB = S2DW_MAXC * ELEM + 16;            // slab bytes per staged row (+16 pad)
   __shared__ __align__(16) uint8_t slab[4][32 * RB];
   pdl_launch_dependents();
@@ -402,33 +429,37 @@ __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x
     }
   }
   uint8_t *row = slab[warp] + lane * RB;
+  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;   // 3xTF32: hi plane, then lo plane
+  for (int pl = 0; pl < planes; ++pl) {
 #pragma unroll
-  for (int j = 0; j < S2DW_MAXC; j += 8) {
-    if (j >= Cps) break;
-    if (ELEM == 2) {
-      __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
-      __nv_bfloat162 cq = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
-      *reinterpret_cast<uint4 *>(row + j * 2) =
-          make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
-                     *reinterpret_cast<uint32_t *>(&cq), *reinterpret_cast<uint32_t *>(&d));
-    } else {
-      *reinterpret_cast<uint4 *>(row + j * 4) =
-          make_uint4(f32_to_tf32_rna(v[j]), f32_to_tf32_rna(v[j + 1]), f32_to_tf32_rna(v[j + 2]),
-                     f32_to_tf32_rna(v[j + 3]));
-      *reinterpret_cast<uint4 *>(row + j * 4 + 16) =
-          make_uint4(f32_to_tf32_rna(v[j + 4]), f32_to_tf32_rna(v[j + 5]), f32_to_tf32_rna(v[j + 6]),
-                     f32_to_tf32_rna(v[j + 7]));
+    for (int j = 0; j < S2DW_MAXC; j += 8) {
+      if (j >= Cps) break;
+      if (ELEM == 2) {
+        __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
+        __nv_bfloat162 cq = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
+        *reinterpret_cast<uint4 *>(row + j * 2) =
+            make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
+                       *reinterpret_cast<uint32_t *>(&cq), *reinterpret_cast<uint32_t *>(&d));
+      } else {
+        *reinterpret_cast<uint4 *>(row + j * 4) =
+            make_uint4(tf32_plane(v[j], pl), tf32_plane(v[j + 1], pl), tf32_plane(v[j + 2], pl),
+                       tf32_plane(v[j + 3], pl));
+        *reinterpret_cast<uint4 *>(row + j * 4 + 16) =
+            make_uint4(tf32_plane(v[j + 4], pl), tf32_plane(v[j + 5], pl), tf32_plane(v[j + 6], pl),
+                       tf32_plane(v[j + 7], pl));
+      }
     }
-  }
-  __syncwarp();
-  // the warp's rows q0 .. q0+31 are contiguous in dst: chunk k -> row k / cpr, chunk k % cpr
-  const int cpr = Cps * ELEM / 16;
-  uint8_t *out = static_cast<uint8_t *>(dst) + (size_t)q0 * Cps * ELEM;
-  const int nrows = (int)min(32LL, total - q0);
-  for (int k = lane; k < nrows * cpr; k += 32) {
-    const int r = k / cpr, ch = k - r * cpr;
-    *reinterpret_cast<uint4 *>(out + (size_t)k * 16) =
-        *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+    __syncwarp();
+    // the warp's rows q0 .. q0+31 are contiguous in dst: chunk k -> row k / cpr, chunk k % cpr
+    const int cpr = Cps * ELEM / 16;
+    uint8_t *out = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0) + (size_t)q0 * Cps * ELEM;
+    const int nrows = (int)min(32LL, total - q0);
+    for (int k = lane; k < nrows * cpr; k += 32) {
+      const int r = k / cpr, ch = k - r * cpr;
+      *reinterpret_cast<uint4 *>(out + (size_t)k * 16) =
+          *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+    }
+    __syncwarp();
   }
 }
 
@@ -439,7 +470,7 @@ __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x
 template <int ELEM, int S, int C>
 __global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__ x, void *__restrict__ dst,
                                                        int N, int H, int W, int P, int Hs, int Ws,
-                                                       int Cps, int src_c) {
+                                                       int Cps, int src_c, long long lo_off) {
   constexpr int NC = S * S * C;
   constexpr int RB = S2DW_MAXC * ELEM + 16;
   __shared__ __align__(16) uint8_t slab[4][32 * RB];
@@ -479,35 +510,39 @@ __global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__
     }
   }
   uint8_t *rowp = slab[warp] + lane * RB;
+  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;   // 3xTF32: hi plane, then lo plane
+  for (int pl = 0; pl < planes; ++pl) {
 #pragma unroll
-  for (int j = 0; j < S2DW_MAXC; j += 8) {
-    if (j >= Cps) break;
-    float u[8];
+    for (int j = 0; j < S2DW_MAXC; j += 8) {
+      if (j >= Cps) break;
+      float u[8];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) u[k] = (j + k < NC) ? v[(j + k < NC) ? j + k : 0] : 0.f;
-    if (ELEM == 2) {
-      __nv_bfloat162 a = __floats2bfloat162_rn(u[0], u[1]), b = __floats2bfloat162_rn(u[2], u[3]);
-      __nv_bfloat162 cq = __floats2bfloat162_rn(u[4], u[5]), d = __floats2bfloat162_rn(u[6], u[7]);
-      *reinterpret_cast<uint4 *>(rowp + j * 2) =
-          make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
-                     *reinterpret_cast<uint32_t *>(&cq), *reinterpret_cast<uint32_t *>(&d));
-    } else {
-      *reinterpret_cast<uint4 *>(rowp + j * 4) =
-          make_uint4(f32_to_tf32_rna(u[0]), f32_to_tf32_rna(u[1]), f32_to_tf32_rna(u[2]),
-                     f32_to_tf32_rna(u[3]));
-      *reinterpret_cast<uint4 *>(rowp + j * 4 + 16) =
-          make_uint4(f32_to_tf32_rna(u[4]), f32_to_tf32_rna(u[5]), f32_to_tf32_rna(u[6]),
-                     f32_to_tf32_rna(u[7]));
+      for (int k = 0; k < 8; ++k) u[k] = (j + k < NC) ? v[(j + k < NC) ? j + k : 0] : 0.f;
+      if (ELEM == 2) {
+        __nv_bfloat162 a = __floats2bfloat162_rn(u[0], u[1]), b = __floats2bfloat162_rn(u[2], u[3]);
+        __nv_bfloat162 cq = __floats2bfloat162_rn(u[4], u[5]), d = __floats2bfloat162_rn(u[6], u[7]);
+        *reinterpret_cast<uint4 *>(rowp + j * 2) =
+            make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
+                       *reinterpret_cast<uint32_t *>(&cq), *reinterpret_cast<uint32_t *>(&d));
+      } else {
+        *reinterpret_cast<uint4 *>(rowp + j * 4) =
+            make_uint4(tf32_plane(u[0], pl), tf32_plane(u[1], pl), tf32_plane(u[2], pl),
+                       tf32_plane(u[3], pl));
+        *reinterpret_cast<uint4 *>(rowp + j * 4 + 16) =
+            make_uint4(tf32_plane(u[4], pl), tf32_plane(u[5], pl), tf32_plane(u[6], pl),
+                       tf32_plane(u[7], pl));
+      }
     }
-  }
-  __syncwarp();
-  const int cpr = Cps * ELEM / 16;
-  uint8_t *out = static_cast<uint8_t *>(dst) + (size_t)q0 * Cps * ELEM;
-  const int nrows = (int)min(32LL, total - q0);
-  for (int k = lane; k < nrows * cpr; k += 32) {
-    const int r = k / cpr, ch = k - r * cpr;
-    *reinterpret_cast<uint4 *>(out + (size_t)k * 16) =
-        *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+    __syncwarp();
+    const int cpr = Cps * ELEM / 16;
+    uint8_t *out = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0) + (size_t)q0 * Cps * ELEM;
+    const int nrows = (int)min(32LL, total - q0);
+    for (int k = lane; k < nrows * cpr; k += 32) {
+      const int r = k / cpr, ch = k - r * cpr;
+      *reinterpret_cast<uint4 *>(out + (size_t)k * 16) =
+          *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+    }
+    __syncwarp();
   }
 }
 
@@ -515,7 +550,7 @@ __global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__
 // c' = (dh*S + dw)*C + c, value W[co][c][S*kh'+dh][S*kw'+dw] (0 past the K x K window).
 template <int ELEM>
 __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ out, int Co, int C,
-                               int K, int S, int Ks, int Cps, int Kpad) {
+                               int K, int S, int Ks, int Cps, int Kpad, long long lo_off) {
   pdl_launch_dependents();
   pdl_wait();
   const size_t total = (size_t)Co * Kpad;
@@ -529,7 +564,7 @@ __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ o
       const int kh = S * khs + dh, kw = S * kws + dw;
       if (kh < K && kw < K) v = __ldg(w + (((size_t)co * C + c) * K + kh) * K + kw);
     }
-    PackOut<ELEM>::store1(out, i, v);
+    PackOut<ELEM>::store1(out, i, v, lo_off);
   }
 }
 
@@ -538,14 +573,15 @@ __global__ void pack_w_fwd_s2d(const float *__restrict__ w, void *__restrict__ o
 // spent most of its time in 64-bit divisions).
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_fwd(const float *__restrict__ w, void *__restrict__ out,
-                                                  int Co, int C, int taps, int Cp, int Kpad) {
+                                                  int Co, int C, int taps, int Cp, int Kpad,
+                                                  long long lo_off) {
   pdl_launch_dependents();
   pdl_wait();
   const int co = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= Kpad) return;
   const int t = k / Cp, c = k - t * Cp;
   const float v = (t < taps && c < C) ? __ldg(w + ((size_t)co * C + c) * taps + t) : 0.f;
-  PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v);
+  PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v, lo_off);
 }
 
 // W [Co][C][Kh][Kw] -> backward-data B operand Wt[ci][tap*Cop + co] (row length Kpad).
@@ -557,7 +593,8 @@ __global__ void __launch_bounds__(256) pack_w_fwd(const float *__restrict__ w, v
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w, void *__restrict__ out,
                                                     int Co, int C, int taps, int Cop, int Kpad,
-                                                    int flip, int co_off, int co_lo, int co_hi) {
+                                                    int flip, int co_off, int co_lo, int co_hi,
+                                                    long long lo_off) {
   pdl_launch_dependents();
   pdl_wait();
   const int ci = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
@@ -568,7 +605,7 @@ __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w,
   const float v = (t < taps && cb < Co)
                       ? __ldg(w + ((size_t)cb * C + ci) * taps + (flip ? taps - 1 - t : t))
                       : 0.f;
-  PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
+  PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v, lo_off);
 }
 
 // Row-staged weight packs (default when a staged row fits 48 KB of shared memory).  The element-
@@ -579,7 +616,8 @@ __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w,
 // Forward: block co stages W[co][0..C*taps) and writes Wp[co][t*Cp + c].
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_fwd_rows(const float *__restrict__ w, void *__restrict__ out,
-                                                       int C, int taps, int Cp, int Kpad) {
+                                                       int C, int taps, int Cp, int Kpad,
+                                                       long long lo_off) {
   extern __shared__ float srow[];
   pdl_launch_dependents();
   pdl_wait();
@@ -590,7 +628,7 @@ __global__ void __launch_bounds__(256) pack_w_fwd_rows(const float *__restrict__
   for (int k = threadIdx.x; k < Kpad; k += 256) {
     const int t = k / Cp, c = k - t * Cp;
     const float v = (t < taps && c < C) ? srow[c * taps + t] : 0.f;
-    PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v);
+    PackOut<ELEM>::store1(out, (size_t)co * Kpad + k, v, lo_off);
   }
 }
 
@@ -600,7 +638,8 @@ __global__ void __launch_bounds__(256) pack_w_fwd_rows(const float *__restrict__
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_dgrad_rows(const float *__restrict__ w, void *__restrict__ out,
                                                          int Co, int C, int taps, int Cop, int Kpad,
-                                                         int flip, int co_off, int co_lo, int co_hi) {
+                                                         int flip, int co_off, int co_lo, int co_hi,
+                                                         long long lo_off) {
   extern __shared__ float srow[];   // [Co][taps]
   pdl_launch_dependents();
   pdl_wait();
@@ -615,7 +654,7 @@ __global__ void __launch_bounds__(256) pack_w_dgrad_rows(const float *__restrict
     if (t < taps && (co < co_lo || co >= co_hi)) continue;   // another branch's channels
     const int cb = co - co_off;
     const float v = (t < taps && cb < Co) ? srow[cb * taps + (flip ? taps - 1 - t : t)] : 0.f;
-    PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v);
+    PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v, lo_off);
   }
 }
 
@@ -630,7 +669,8 @@ constexpr int PWB_MAXT = 25;   // taps (<= 5x5) that fit the stage: 32 x (32*25 
 template <int ELEM>
 __global__ void __launch_bounds__(256) pack_w_both(const float *__restrict__ w, void *__restrict__ wp,
                                                    void *__restrict__ wt, int Co, int C, int taps,
-                                                   int Cp, int Cop, int Kpf, int Kpd, int flip) {
+                                                   int Cp, int Cop, int Kpf, int Kpd, int flip,
+                                                   long long lo_p, long long lo_t) {
   extern __shared__ float stg[];   // [32 co][32*taps + 1]
   pdl_launch_dependents();
   pdl_wait();
@@ -639,11 +679,11 @@ __global__ void __launch_bounds__(256) pack_w_both(const float *__restrict__ w, 
   if (blockIdx.z == 1) {   // K tails (t >= taps) of both operands
     for (int i = threadIdx.x; i < 32 * (Kpf - taps * Cp); i += 256) {
       const int r = i / (Kpf - taps * Cp), k = taps * Cp + i % (Kpf - taps * Cp);
-      if (blockIdx.x == 0 && co0 + r < Co) PackOut<ELEM>::store1(wp, (size_t)(co0 + r) * Kpf + k, 0.f);
+      if (blockIdx.x == 0 && co0 + r < Co) PackOut<ELEM>::store1(wp, (size_t)(co0 + r) * Kpf + k, 0.f, lo_p);
     }
     for (int i = threadIdx.x; i < 32 * (Kpd - taps * Cop); i += 256) {
       const int r = i / (Kpd - taps * Cop), k = taps * Cop + i % (Kpd - taps * Cop);
-      if (blockIdx.y == 0 && ci0 + r < C) PackOut<ELEM>::store1(wt, (size_t)(ci0 + r) * Kpd + k, 0.f);
+      if (blockIdx.y == 0 && ci0 + r < C) PackOut<ELEM>::store1(wt, (size_t)(ci0 + r) * Kpd + k, 0.f, lo_t);
     }
     return;
   }
@@ -660,7 +700,7 @@ __global__ void __launch_bounds__(256) pack_w_both(const float *__restrict__ w, 
     const int co = co0 + r;
     if (co >= Co || ci0 + lane >= Cp) continue;
     for (int t = 0; t < taps; ++t)
-      PackOut<ELEM>::store1(wp, (size_t)co * Kpf + (size_t)t * Cp + ci0 + lane, stg[r * ld + lane * taps + t]);
+      PackOut<ELEM>::store1(wp, (size_t)co * Kpf + (size_t)t * Cp + ci0 + lane, stg[r * ld + lane * taps + t], lo_p);
   }
   // backward-data: rows ci (< C), for each t: 32 consecutive co (lane); padding co >= Co -> 0
   for (int c = wr; c < 32; c += 8) {
@@ -668,7 +708,7 @@ __global__ void __launch_bounds__(256) pack_w_both(const float *__restrict__ w, 
     if (ci >= C || co0 + lane >= Cop) continue;
     for (int t = 0; t < taps; ++t) {
       const int tt = flip ? taps - 1 - t : t;
-      PackOut<ELEM>::store1(wt, (size_t)ci * Kpd + (size_t)tt * Cop + co0 + lane, stg[lane * ld + c * taps + t]);
+      PackOut<ELEM>::store1(wt, (size_t)ci * Kpd + (size_t)tt * Cop + co0 + lane, stg[lane * ld + c * taps + t], lo_t);
     }
   }
 }

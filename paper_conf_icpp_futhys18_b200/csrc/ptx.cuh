@@ -260,6 +260,39 @@ __device__ __forceinline__ void mma_kblock_e(uint32_t d_tmem, uint64_t adesc, ui
 #undef GLP_MMA_I
 #undef GLP_MMA_HEAD
 }
+// 3xTF32 k-block (GLP_MATH_FP32): every operand is a hi plane and a lo plane (hi = rna(v),
+// lo = rna(v - hi)) at byte offsets 16*alo16 (A) / 16*blo16 (B) from the hi plane.  Per k-step
+// three kind::tf32 MMAs accumulate, in this fixed order, hi*hi, hi*lo and lo*hi into the same
+// TMEM accumulator (lo*lo, below 2^-22 of a product, is dropped).  NSTEP k-steps advanced by STEP
+// 16-byte units, all in one instruction block; `accumulate` applies to the first MMA only.
+template <int CG, int NSTEP, int STEP>
+__device__ __forceinline__ void mma_kblock_x3_e(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
+                                                uint64_t alo16, uint64_t blo16, uint32_t idesc,
+                                                uint32_t accumulate) {
+  static_assert(NSTEP == 4, "3xTF32 k-block = 4 k-steps of K = 8");
+#define GLP_X3_HEAD                                                                     \
+  "{\n\t.reg .pred P_e, p, q;\n\t.reg .b64 a, b, al, bl;\n\t"                           \
+  "elect.sync _|P_e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\tsetp.eq.b32 q, %3, %3;\n\t" \
+  "mov.b64 a, %1;\n\tmov.b64 b, %2;\n\t"
+#define GLP_X3_STEP(CGS, P)                                                             \
+  "add.s64 al, a, %5;\n\tadd.s64 bl, b, %6;\n\t"                                        \
+  "@P_e tcgen05.mma.cta_group::" CGS ".kind::tf32 [%0], a, b, %3, " P ";\n\t"           \
+  "@P_e tcgen05.mma.cta_group::" CGS ".kind::tf32 [%0], a, bl, %3, q;\n\t"              \
+  "@P_e tcgen05.mma.cta_group::" CGS ".kind::tf32 [%0], al, b, %3, q;\n\t"
+#define GLP_X3_ADV "add.s64 a, a, %7;\n\tadd.s64 b, b, %7;\n\t"
+#define GLP_X3_K4(CGS)                                                                  \
+  asm volatile(GLP_X3_HEAD GLP_X3_STEP(CGS, "p") GLP_X3_ADV GLP_X3_STEP(CGS, "q")      \
+               GLP_X3_ADV GLP_X3_STEP(CGS, "q") GLP_X3_ADV GLP_X3_STEP(CGS, "q") "}"   \
+               ::"r"(d_tmem), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate),      \
+               "l"(alo16), "l"(blo16), "n"(STEP) : "memory")
+  if (CG == 1) GLP_X3_K4("1");
+  else GLP_X3_K4("2");
+#undef GLP_X3_K4
+#undef GLP_X3_ADV
+#undef GLP_X3_STEP
+#undef GLP_X3_HEAD
+}
+
 template <int CG>
 __device__ __forceinline__ void mma_commit_e(uint32_t bar) {
   if (CG == 1)

@@ -15,8 +15,9 @@ from glp_workloads import gen_custom
 
 pytestmark = pytest.mark.gpu
 DEV = torch.device("cuda:0")
-TOL = {"fp32": 1e-5, "tf32": 2e-2, "bf16": 2e-2}
-EMU = {"tf32": oracle.round_tf32_rna, "bf16": oracle.round_bf16_rne}
+TOL = {"fp32": 1e-5, "fp32_simt": 1e-5, "tf32": 2e-2, "bf16": 2e-2}
+# the operand each tensor-core mode's MMA sees (3xTF32: the hi plane for layout checks)
+EMU = {"tf32": oracle.round_tf32_rna, "bf16": oracle.round_bf16_rne, "fp32": oracle.round_tf32_rna}
 
 # name, N, C, H, W, Co, K, S, P  — several M tiles, ragged tails, odd geometry
 SHAPES = [
@@ -68,7 +69,7 @@ def _layer(shape, math, S=0):
     return glp.ConvLayer(N, C, H, W, Co, K, St, P, math=math, samples_in_flight=S)
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
 def test_parity_random(shape, math):
     d = _data(shape)
@@ -79,20 +80,36 @@ def test_parity_random(shape, math):
     assert all(e <= TOL[math] for e in errs.values()), errs
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
 def test_parity_rounding_emulated(shape, math):
     """Oracle on the operands rounded exactly as the pack step defines (oracle.round_*):
-    catches indexing bugs that the 2e-2 tolerance would hide."""
+    catches indexing bugs that the 2e-2 tolerance would hide.  3xTF32: the oracle of the three
+    products the MMAs form, hi*hi + hi*lo + lo*hi with (hi, lo) = oracle.split_3xtf32 (each
+    pass is linear in each operand, so the sum of three oracle calls), at 1e-6."""
     d = _data(shape, seed=5)
     got = _run(_layer(shape, math), d)
-    r = EMU[math]
-    ref = _oracle(d, shape[7], shape[8], x=r(d["x"]), w=r(d["w"]), dy=r(d["dy"]))
+    S, P = shape[7], shape[8]
+    if math == "fp32":
+        sp = {k: oracle.split_3xtf32(d[k]) for k in ("x", "w", "dy")}
+        parts = [_oracle(d, S, P, x=sp["x"][i], w=sp["w"][j], dy=sp["dy"][i])
+                 for i, j in ((0, 0), (0, 1), (1, 0))]
+        # dW pairs x with dy: its three products are (hi,hi), (hi,lo), (lo,hi) of (x, dy)
+        pw = [_oracle(d, S, P, x=sp["x"][i], dy=sp["dy"][j])["dw"] for i, j in ((0, 0), (0, 1), (1, 0))]
+        ref = {k: parts[0][k] + parts[1][k] + parts[2][k] for k in ("y", "dx")}
+        ref["y"] -= 2 * d["b"].astype(np.float64)[None, :, None, None]   # bias counted once
+        ref["dw"] = pw[0] + pw[1] + pw[2]
+        ref["db"] = parts[0]["db"]
+        bar = 5e-6   # chunked fp32 accumulation of truncating MMAs (DESIGN.md "3xTF32")
+    else:
+        r = EMU[math]
+        ref = _oracle(d, S, P, x=r(d["x"]), w=r(d["w"]), dy=r(d["dy"]))
+        bar = 1e-4
     errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
-    assert all(e <= 1e-4 for e in errs.values()), errs
+    assert all(e <= bar for e in errs.values()), errs
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
 def test_exact_integer_bitexact(shape, math):
     """Integer data in [-2,2]: every partial sum is an exact integer < 2^24 in fp32/TF32/BF16,
@@ -105,7 +122,7 @@ def test_exact_integer_bitexact(shape, math):
         np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
 @pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[2], SHAPES[5], SHAPES[6]], ids=lambda s: s[0])
 def test_samples_in_flight_invariance(shape, math):
     """Convergence invariance (P264): outputs bitwise identical for every S and on rerun."""
@@ -121,7 +138,7 @@ def test_samples_in_flight_invariance(shape, math):
         np.testing.assert_array_equal(again[k], base[k])
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", [SHAPES[1], SHAPES[2], SHAPES[3], SHAPES[6]], ids=lambda s: s[0])
 def test_im2col_layout_bitexact(shape, math):
     """glp_debug_im2col (the producer's own gather math on the packed operand) equals the
@@ -153,7 +170,7 @@ def test_accumulate_flag():
     np.testing.assert_array_equal(db.cpu().numpy(), (d["dy"].astype(np.float64).sum((0, 2, 3)) + 1).astype(np.float32))
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 def test_combined_bwd_equals_separate(math):
     shape = SHAPES[5]
     d = _data(shape, seed=8)
@@ -170,7 +187,7 @@ def test_combined_bwd_equals_separate(math):
     np.testing.assert_array_equal(db.cpu().numpy(), sep["db"])
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 def test_analyzer_matches_occupancy_api(math):
     """The re-derived analyzer's CTAs/SM for every shipped kernel equals the CUDA occupancy API."""
     for shape in SHAPES:
@@ -196,7 +213,7 @@ def test_error_paths_on_device():
     assert rc == 1  # misaligned
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 def test_staged_equals_composed(math):
     """Staged calls (pack once, GEMMs, reduce) are bitwise identical to the composed calls."""
     shape = SHAPES[6]
@@ -221,7 +238,7 @@ def test_staged_equals_composed(math):
         np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=k)
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[2], SHAPES[5], SHAPES[6]], ids=lambda s: s[0])
 def test_single_cta_mma_path(shape, math, monkeypatch):
     """GLP_CTA_GROUP=1 forces single-CTA tcgen05 MMAs (no CTA pairs): still bit-exact on integer
@@ -240,7 +257,7 @@ def test_single_cta_mma_path(shape, math, monkeypatch):
         np.testing.assert_array_equal(one[k], two[k], err_msg=k)
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", [("c64_k3", 2, 64, 8, 8, 128, 3, 1, 1),
                                    ("c64_k3_n256", 2, 64, 8, 8, 256, 3, 1, 1),
                                    ("c96_k5", 2, 96, 9, 9, 256, 5, 1, 2),
@@ -418,7 +435,7 @@ def _group_run(layer, x, ws, bs, dys, staged=False):
     return {"y": c(ys), "dx": dx.cpu().numpy(), "dw": c(dws), "db": c(dbs)}
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("g", GROUPS, ids=lambda g: g[0])
 def test_group_exact_vs_oracle(g, math):
     """A fused group equals the oracle of each branch bit for bit on integer data (y_b, dW_b,
@@ -473,7 +490,7 @@ def test_group_rejects_misaligned_branch():
 POOL_SHAPES = [SHAPES[0], SHAPES[2], SHAPES[6], ("k5_ragged", 5, 24, 11, 13, 40, 5, 1, 2)]
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
 @pytest.mark.parametrize("shape", POOL_SHAPES, ids=lambda s: s[0])
 def test_stream_pool_comparator(shape, math):
     """The paper's per-sample stream pool (prior-art comparator): forward and backward-data are
@@ -533,7 +550,7 @@ def _grouped_oracle(d, S, P, G):
             "dw": np.concatenate(out["dw"], 0), "db": dy.astype(np.float64).sum(axis=(0, 2, 3))}
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
 @pytest.mark.parametrize("shape", GROUPED, ids=lambda s: s[0])
 def test_grouped_conv(shape, math):
     """Grouped convolution equals the oracle of each group: bit-exact on integer data (every
@@ -552,7 +569,7 @@ def test_grouped_conv(shape, math):
                 np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
             else:
                 assert np.abs(got[k] - ref[k]).max() / np.abs(ref[k]).max() <= TOL[math], k
-    if math != "fp32":
+    if math != "fp32_simt":
         t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
         y = torch.empty(layer.y_shape, device=DEV)
         dx = torch.empty(layer.x_shape, device=DEV)
@@ -607,7 +624,7 @@ def test_tree_exchange_bitwise_invariant_emulated_ranks():
             assert np.abs(ref - full).max() / np.abs(full).max() <= TOL["bf16"]
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[4], SHAPES[5], SHAPES[6], SHAPES[1], SHAPES[9]],
                          ids=lambda s: s[0])
 def test_pack_w_both_equals_separate(shape, math):
@@ -692,3 +709,20 @@ def test_halo_wgrad_fused_dy_variants(ncg, monkeypatch):
     np.testing.assert_array_equal(got["dw"], ref["dw"])
     scale = np.abs(d["dy"].astype(np.float64)).sum(axis=(0, 2, 3))
     assert np.all(np.abs(got["db"].astype(np.float64) - ref["db"]) <= 1e-6 * scale)
+
+
+LONG_K = [("caffenet_conv2", 2, 96, 27, 27, 256, 5, 1, 2),    # dgrad K = 6400, fwd K = 2400
+          ("caffenet_conv4", 2, 384, 13, 13, 384, 3, 1, 1),   # K = 3456 both ways
+          ("gnet_conv_4", 3, 192, 7, 7, 384, 3, 1, 1)]
+
+
+@pytest.mark.parametrize("shape", LONG_K, ids=lambda s: s[0])
+def test_fp32_long_reductions(shape):
+    """GLP_MATH_FP32 (3xTF32) at the paper's longest reductions: the tensor core truncates each
+    MMA's fp32 result, so the error of one TMEM accumulator grows with K; the chunked fp32 register
+    accumulation keeps every output within the 1e-5 normwise bar (BASELINE.json north_star)."""
+    d = _data(shape, seed=91)
+    got = _run(_layer(shape, "fp32"), d)
+    ref = _oracle(d, shape[7], shape[8])
+    errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
+    assert all(e <= TOL["fp32"] for e in errs.values()), errs

@@ -32,6 +32,8 @@ sys.path.insert(0, ROOT)
 from glp_workloads import CONFIG_NAMES, LEVELS, SIBLINGS, config, gen_layer  # noqa: E402
 
 METRIC = "conv fwd+bwd images/sec"
+# the arithmetic each --math mode computes in (fp32 = 3xTF32 on tcgen05: fp32-accurate)
+DTYPE = {"fp32": "fp32 (3xtf32)", "tf32": "tf32", "bf16": "bf16"}
 UNIT = "images/s"
 NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25   # B200_PROFILING.md nominal dense ratio
 
@@ -45,7 +47,9 @@ def parse_args():
     p.add_argument("--workload", type=int, default=4, help="BASELINE.json config index 1..5")
     p.add_argument("--math", choices=["fp32", "bf16", "tf32"], default="fp32",
                    help="fp32 = 3xTF32 on tcgen05 (fp32-accurate, the paper's FP32 arithmetic)")
-    p.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    p.add_argument("--scaling", choices=["weak", "strong"], default="strong",
+                   help="strong (default, the BASELINE.json cfg4 wording): the config's global batch "
+                        "sharded over the GPUs; weak: the config batch on every GPU")
     p.add_argument("--scheme", choices=["persistent", "pool"], default="persistent",
                    help="pool: the paper's prior-art scheme (per-sample kernels round-robin over a "
                         "stream pool sized by Eq. 7) as a comparator; 1 GPU")
@@ -63,6 +67,11 @@ def parse_args():
                    help="run sibling layers that share an input (GoogLeNet 5b 1x1 branches) as "
                         "separate layers instead of one fused group")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-extra-modes", action="store_true",
+                   help="skip the bf16 / tf32 lines measured beside the fp32 headline (1 GPU)")
+    p.add_argument("--dry-run", action="store_true",
+                   help="(tests) launcher plumbing only: start the ranks, form a gloo process group "
+                        "on CPU, all-reduce one tensor and print the line's n_gpus; no GPU work")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=5)
     p.add_argument("--serial", action="store_true",
@@ -224,6 +233,11 @@ class LayerState:
         self.db = grads.db(idx)
         self.flops = float(self.layer.with_batch(n_local).flops_per_pass())
         self.leaves = None
+        self.idx = idx
+
+    def grad_idxs(self):
+        """Slots of the flat dW||db buffer this unit writes (its all-reduce bucket)."""
+        return [self.idx]
 
     def use_leaves(self, leaf_grads, idx, math, dev):
         """Deterministic exchange: the filter gradient per batch leaf of this rank (one plan for
@@ -381,6 +395,10 @@ class GroupState:
         self.dws = [grads.dw(i) for i in idxs]
         self.dbs = [grads.db(i) for i in idxs]
         self.flops = float(sum(m.with_batch(n_local).flops_per_pass() for m in members))
+        self.idxs = list(idxs)
+
+    def grad_idxs(self):
+        return self.idxs
 
     def launches(self):
         nb = len(self.members)   # per-branch packs of W (x2) and dy
@@ -479,19 +497,10 @@ def run_pool(args):
         "tflops_step": round(step_flops / (ms * 1e-3) / 1e12, 1)}), flush=True)
 
 
-def run_glp(args, ws, rank, local):
-    import numpy as np
-    import torch
-    import torch.distributed as dist
-    import paper_conf_icpp_futhys18_b200 as glp
-
-    dev = torch.device("cuda", local)
-    torch.cuda.set_device(dev)
-    if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
-    from paper_conf_icpp_futhys18_b200.dist import FlatGrads, shard_range
+def build_states(args, math, G, rank, dev, grads):
+    """Plans, seeded inputs and outputs of every unit of the workload at this rank's batch."""
+    from paper_conf_icpp_futhys18_b200.dist import shard_range
     layers = config(args.workload)
-    G = ws
     shards = [shard_range(l.N, rank, G) for l in layers]
     if args.scaling == "strong":
         n_local = [b - a for a, b in shards]
@@ -499,9 +508,6 @@ def run_glp(args, ws, rank, local):
     else:
         n_local = [l.N for l in layers]
         n_global = [l.N * G for l in layers]
-    grads = FlatGrads([l.w_shape for l in layers], device=dev)
-    flat = grads.buf
-    nparams = grads.numel
     groups = [] if args.no_fuse else SIBLINGS.get(args.workload, [])
     in_group = {name: gi for gi, g in enumerate(groups) for name in g}
     states = []
@@ -510,69 +516,77 @@ def run_glp(args, ws, rank, local):
         shard = shards[i] if args.scaling == "strong" and G > 1 else None
         gi = in_group.get(l.name)
         if gi is None:
-            states.append(LayerState(l, nl, ng, shard, args.math, dev, grads, i))
+            states.append(LayerState(l, nl, ng, shard, math, dev, grads, i))
         elif gi not in done_groups:
             if shard is not None:
                 raise SystemExit("fused groups with strong scaling: use --no-fuse")
             done_groups.add(gi)
             idxs = [j for j, m in enumerate(layers) if m.name in groups[gi]]
-            states.append(GroupState([layers[j] for j in idxs], nl, ng, args.math, dev, grads,
-                                     idxs))
-    if args.exact_data:
-        set_exact_data(states)
-    stream = torch.cuda.current_stream()
+            states.append(GroupState([layers[j] for j in idxs], nl, ng, math, dev, grads, idxs))
+    return layers, states, n_local
 
-    tree = None
-    if args.exchange == "tree":
-        from paper_conf_icpp_futhys18_b200.dist import TreeAllreduce, rank_leaves
-        my_leaves = rank_leaves(rank, G)
-        if any(not isinstance(s, LayerState) for s in states) or n_local[0] % len(my_leaves):
-            raise SystemExit("--exchange tree: single layers and a leaf-divisible batch only")
-        leaf_grads = [FlatGrads([l.w_shape for l in layers], device=dev) for _ in my_leaves]
-        for i, s in enumerate(states):
-            s.use_leaves(leaf_grads, i, args.math, dev)
-        tree = TreeAllreduce()
 
-    def exchange():
-        if tree is not None:
-            flat.copy_(tree([lg.buf for lg in leaf_grads]))
-        elif G > 1:
-            grads.allreduce()
-
-    # network DAG levels (units of one level are independent: concurrent streams, the GLP4NN idea
-    # of concurrent kernels applied to a real step's independent layers); default: a chain
+def dag_levels(args, states):
+    """Network DAG levels of the workload's units (glp_workloads.LEVELS; default: a chain)."""
     lv = None if args.chain else LEVELS.get(args.workload)
-    if lv:
-        where = {name: k for k, names in enumerate(lv) for name in names}
-        unit_level = [where[(s.members[0] if isinstance(s, GroupState) else s.layer).name]
-                      for s in states]
-        levels = [[i for i, u in enumerate(unit_level) if u == k] for k in range(len(lv))]
-        levels = [l for l in levels if l]
-    else:
-        levels = [[i] for i in range(len(states))]
-    width = max(len(l) for l in levels)
-    side_w = torch.cuda.Stream(device=dev)   # weight packs (weights are known at step start)
-    # per slot of a level: a forward/backward-data stream (slot 0 = the main stream) and a
-    # filter-gradient stream (wgrad GEMM + dW/db reduction)
-    fstreams = [None] + [torch.cuda.Stream(device=dev) for _ in range(width - 1)]
-    gstreams = [torch.cuda.Stream(device=dev) for _ in range(width)]
+    if not lv:
+        return [[i] for i in range(len(states))]
+    where = {name: k for k, names in enumerate(lv) for name in names}
+    unit_level = [where[(s.members[0] if isinstance(s, GroupState) else s.layer).name]
+                  for s in states]
+    levels = [[i for i, u in enumerate(unit_level) if u == k] for k in range(len(lv))]
+    return [l for l in levels if l]
 
-    def step(ev=None, concurrent=None, with_exchange=True):
-        """One training step of every layer's hot path.  concurrent (default: not timing kernels):
-        the stream DAG of a real network's step -- per DAG level, each unit's forward chain and
-        backward-data chain on its own stream (one level = independent layers; the main stream
-        for a chain); both weight packs of every unit on side stream W at step start; each unit's
-        filter-gradient GEMM + reductions on a G stream as soon as its dy is packed (they overlap
-        the next level's backward-data work, which does not depend on them); everything is
-        joined before the step ends.  Serial (ev given): everything on the main stream, in order,
-        with CUDA events around each GEMM for the per-kernel attribution."""
+
+class Step:
+    """One training step of every unit's hot path, issued as the stream DAG of a real network's
+    step (or serially, with CUDA events around each GEMM, for the per-kernel attribution).
+
+    Gradient exchange (G > 1, BJ.ns (4)): 'nccl' = every unit's dW||db bucket is
+    all-reduced (SUM, NCCL over NVLink) on its filter-gradient stream as soon as that unit's
+    filter-gradient GEMM and reductions are done -- in reverse layer order, overlapping the
+    remaining backward-data work of the earlier layers; the step ends when every bucket has
+    arrived.  'tree' = the deterministic exchange (NEXT-2) after the step."""
+
+    def __init__(self, args, states, grads, G, dev, tree=None, leaf_grads=None):
+        import torch
+        self.args, self.states, self.grads, self.G = args, states, grads, G
+        self.tree, self.leaf_grads = tree, leaf_grads
+        self.levels = dag_levels(args, states)
+        self.width = max(len(l) for l in self.levels)
+        self.side_w = torch.cuda.Stream(device=dev)   # weight packs (known at step start)
+        self.fstreams = [None] + [torch.cuda.Stream(device=dev) for _ in range(self.width - 1)]
+        self.gstreams = [torch.cuda.Stream(device=dev) for _ in range(self.width)]
+        self.bucketed = G > 1 and tree is None
+        self.works = []
+
+    def _bucket(self, s, g):
+        """All-reduce this unit's gradient bucket(s) on stream g (after its reductions)."""
+        if not self.bucketed:
+            return
+        import torch
+        import torch.distributed as dist
+        with torch.cuda.stream(g):
+            self.works.append(dist.all_reduce(self.grads.bucket(s.grad_idxs()),
+                                              op=dist.ReduceOp.SUM, async_op=True))
+
+    def exchange_tail(self):
+        """Join the exchange: bucketed all-reduces (already in flight) or the tree."""
+        if self.tree is not None:
+            self.grads.buf.copy_(self.tree([lg.buf for lg in self.leaf_grads]))
+        for w in self.works:
+            w.wait()   # the current stream waits for the collective
+        self.works = []
+
+    def __call__(self, ev=None, concurrent=None, with_exchange=True):
+        import torch
+        states = self.states
         stream = torch.cuda.current_stream()   # the capture stream while a graph is recorded
         conc = (ev is None) if concurrent is None else concurrent
 
         def mark(e):
             # attribution runs: a GPU-side spin before each start event keeps the stream busy while
             # the host enqueues the event and the kernel, so the interval holds the kernel only
-            # (without it, host launch latency of small kernels leaked into their timings)
             torch.cuda._sleep(40000)
             e.record(stream)
 
@@ -601,10 +615,13 @@ def run_glp(args, ws, rank, local):
                 if ev is not None:
                     ev[i][5].record(stream)
                 s.reduce()
+                if with_exchange:
+                    self._bucket(s, stream)
             if with_exchange:
-                exchange()
+                self.exchange_tail()
             return
-        fs = [stream] + fstreams[1:]
+        fs = [stream] + self.fstreams[1:]
+        side_w, gstreams = self.side_w, self.gstreams
         side_w.wait_stream(stream)
         for g in gstreams:
             g.wait_stream(stream)
@@ -629,7 +646,7 @@ def run_glp(args, ws, rank, local):
             for k in range(1, n):
                 stream.wait_stream(fs[k])
 
-        for lvl in levels:
+        for lvl in self.levels:
             fork(len(lvl))
             for k, i in enumerate(lvl):
                 s, f = states[i], fs[k]
@@ -638,7 +655,7 @@ def run_glp(args, ws, rank, local):
                     f.wait_event(ew_f[i])
                     s.fwd(f)
             join(len(lvl))
-        for lvl in reversed(levels):
+        for lvl in reversed(self.levels):
             fork(len(lvl))
             for k, i in enumerate(lvl):
                 s, f, g = states[i], fs[k], gstreams[k]
@@ -650,6 +667,8 @@ def run_glp(args, ws, rank, local):
                     with torch.cuda.stream(g):
                         s.bwd_filter(g)
                         s.reduce(g)
+                    if with_exchange:
+                        self._bucket(s, g)
                     if s.dx is not None:
                         f.wait_event(ew_b[i])
                         s.bwd_data(f)
@@ -658,63 +677,122 @@ def run_glp(args, ws, rank, local):
         for g in gstreams:
             stream.wait_stream(g)
         if with_exchange:
-            exchange()
+            self.exchange_tail()
+
+
+def time_steps(step_fn, steps, stream):
+    """Device time of `steps` calls of step_fn (CUDA events on `stream`), ms per step."""
+    import torch
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t0.record(stream)
+    for _ in range(steps):
+        step_fn()
+    t1.record(stream)
+    torch.cuda.synchronize()
+    return t0.elapsed_time(t1) / steps
+
+
+def quick_mode(args, math, G, rank, dev):
+    """Images/s of the same workload in another math mode (1 GPU, CUDA-graph replay): the
+    bf16 / tf32 lines reported beside the fp32 headline."""
+    import torch
+    from paper_conf_icpp_futhys18_b200.dist import FlatGrads
+    layers = config(args.workload)
+    grads = FlatGrads([l.w_shape for l in layers], device=dev)
+    _, states, n_local = build_states(args, math, G, rank, dev, grads)
+    step = Step(args, states, grads, G, dev)
+    for _ in range(max(3, args.warmup)):
+        step()
+    g_step = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g_step):
+        step(concurrent=not args.serial, with_exchange=False)
+    for _ in range(3):
+        g_step.replay()
+    ms = time_steps(g_step.replay, args.steps, torch.cuda.current_stream())
+    out = {"value": round(n_local[0] / (ms / 1e3), 1), "ms_per_step": round(ms, 4),
+           "dtype": math, "launch": "cuda_graph"}
+    del g_step, step, states
+    torch.cuda.empty_cache()
+    return out
+
+
+def run_glp(args, ws, rank, local):
+    import torch
+    import torch.distributed as dist
+
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    G = ws
+    if G > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_icpp_futhys18_b200.dist import FlatGrads
+    layers = config(args.workload)
+    grads = FlatGrads([l.w_shape for l in layers], device=dev)
+    flat = grads.buf
+    nparams = grads.numel
+    layers, states, n_local = build_states(args, args.math, G, rank, dev, grads)
+    if args.exact_data:
+        set_exact_data(states)
+    stream = torch.cuda.current_stream()
+
+    tree, leaf_grads = None, None
+    if args.exchange == "tree":
+        from paper_conf_icpp_futhys18_b200.dist import TreeAllreduce, rank_leaves
+        my_leaves = rank_leaves(rank, G)
+        if any(not isinstance(s, LayerState) for s in states) or n_local[0] % len(my_leaves):
+            raise SystemExit("--exchange tree: single layers and a leaf-divisible batch only")
+        leaf_grads = [FlatGrads([l.w_shape for l in layers], device=dev) for _ in my_leaves]
+        for i, s in enumerate(states):
+            s.use_leaves(leaf_grads, i, args.math, dev)
+        tree = TreeAllreduce()
+    step = Step(args, states, grads, G, dev, tree, leaf_grads)
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     if G > 1:
         dist.barrier()
-    use_graph = not args.no_graph
+    # One GPU: the whole step (every pack, GEMM and reduction launch of all layers) is recorded
+    # once as a CUDA graph and replayed.  G > 1: the step is issued eagerly so that each unit's
+    # gradient bucket is all-reduced (NCCL) as soon as it is ready, overlapping the rest of the
+    # backward (NCCL collectives are not captured into the graph).
+    use_graph = not args.no_graph and G == 1 and tree is None
     evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(6)] for _ in states]
            for _ in range(args.steps)]
     if use_graph:
-        # The whole step (every pack, GEMM and reduction launch of all layers) recorded once and
-        # replayed: no per-launch host work and minimal gaps between kernels.  The gradient
-        # exchange (NCCL all_reduce, or the tree's point-to-point) stays outside the graph and is
-        # issued after each replay on the same stream.
         g_step = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g_step):
             step(concurrent=not args.serial, with_exchange=False)
         for _ in range(max(1, args.warmup)):
             g_step.replay()
-            exchange()
+        run_one = g_step.replay
+    else:
+        def run_one():
+            step(concurrent=not args.serial)
     clocks = ClockSampler(local) if rank == 0 else None
     if clocks:
         clocks.start()
-    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    torch.cuda.synchronize()
     if G > 1:
+        torch.cuda.synchronize()
         dist.barrier()
-    t0.record(stream)
-    for k in range(args.steps):
-        if use_graph:
-            g_step.replay()
-            exchange()
-        else:
-            step(evs[k])
-    t1.record(stream)
-    torch.cuda.synchronize()
+    ms_per_step = time_steps(run_one, args.steps, stream)
     if G > 1:
         dist.barrier()
     clk = clocks.stop() if clocks else None
-    ms = t0.elapsed_time(t1)
     if G > 1:
-        tt = torch.tensor([ms], device=dev)
+        tt = torch.tensor([ms_per_step], device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
-    ms_per_step = ms / args.steps
-    images_per_step = n_local[0] * G
+        ms_per_step = float(tt.item())
+    images_per_step = sum(n_local[:1]) * G if args.scaling == "weak" else layers[0].N
     value = images_per_step / (ms_per_step / 1e3)
 
-    if use_graph:
-        # per-kernel attribution: events cannot time nodes inside a graph, so the same step runs
-        # K more times eagerly with CUDA events around each GEMM on the launching stream (kernel
-        # durations do not depend on how the launches were issued)
-        for k in range(args.steps):
-            step(evs[k], concurrent=False)
-        torch.cuda.synchronize()
-    # per-kernel live timings (CUDA events on the launching stream)
+    # per-kernel attribution: events cannot time nodes inside a graph, so the same step runs K
+    # more times eagerly and serially with CUDA events around each GEMM on the launching stream
+    # (kernel durations do not depend on how the launches were issued)
+    for k in range(args.steps):
+        step(evs[k], concurrent=False, with_exchange=False)
+    torch.cuda.synchronize()
     kern = []
     for i, s in enumerate(states):
         for name, a, b in (("fwd", 0, 1), ("bwd_data", 2, 3), ("bwd_filter", 4, 5)):
@@ -726,29 +804,11 @@ def run_glp(args, ws, rank, local):
                          "total_us": sum(us), "tflops": round(s.flops / (avg * 1e-6) / 1e12, 1)})
     if args.dump and rank == 0:
         dump_units(states, args.dump, args.workload, args.math)
-    peaks = load_peaks()
-    dom = max(kern, key=lambda r: r["total_us"])
-    peak_tf = peaks["bf16_tflops_sustained"] * {"bf16": 1.0, "tf32": NOMINAL_TF32_OVER_BF16,
-                                                "fp32": NOMINAL_TF32_OVER_BF16 / 3}[args.math]
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tpath):
-        try:
-            traffic = json.load(open(tpath)).get(f"{args.workload}/{dom['layer']}/{dom['pass']}/{args.math}")
-        except Exception:
-            traffic = None
-    roofline = {"bound": "tensor", "achieved": dom["tflops"], "peak": round(peak_tf, 1),
-                "unit": "TFLOP/s", "frac": round(dom["tflops"] / peak_tf, 4), "traffic": traffic,
-                "kernel": f"{kernel_name(states, dom)} {dom['layer']} {dom['pass']}",
-                "peak_source": peaks["source"] + (" bf16 sustained" if args.math == "bf16"
-                                                  else " bf16 sustained x 1.1/2.25 (tf32)"),
-                "share_of_step": round(dom["total_us"] / 1e3 / ms, 4),
-                # context: the same kernel against the burst (one-shot) cuBLAS figure
-                "frac_of_burst_peak": round(dom["tflops"] / (peaks["bf16_tflops"] * (
-                    1.0 if args.math == "bf16" else NOMINAL_TF32_OVER_BF16)), 4)}
+    roofline = make_roofline(args, states, kern, ms_per_step)
     step_flops = sum(s.flops * (3 if s.dx is not None else 2) for s in states)
 
-    # end-to-end: pinned host buffers -> device every step, dW||db back every step
+    # end-to-end through the public API: pinned host buffers -> device every step (each unit's
+    # x, dy, W, b), the step, and dW||db back to the host every step
     e2e = None
     if not args.no_e2e:
         host_pinned = [{k: v.pin_memory() for k, v in s.host.items()} for s in states]
@@ -760,24 +820,25 @@ def run_glp(args, ws, rank, local):
         torch.cuda.synchronize()
         if G > 1:
             dist.barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(ke):
+
+        def e2e_step():
             for s, hp in zip(states, host_pinned):
                 for k2, v in hp.items():
                     s.t[k2].copy_(v, non_blocking=True)
             step()
             out_host.copy_(flat, non_blocking=True)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        ems = e0.elapsed_time(e1)
+        ems = time_steps(e2e_step, ke, stream)
         if G > 1:
             tt = torch.tensor([ems], device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ems = float(tt.item())
-        e2e = {"value": round(images_per_step / (ems / ke / 1e3), 1), "unit": UNIT,
+        e2e = {"value": round(images_per_step / (ems / 1e3), 1), "unit": UNIT,
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": round(ems / ke, 3), "steps": ke}
+               "ms_per_step": round(ems, 3), "steps": ke}
+
+    modes = None
+    if G == 1 and not args.no_extra_modes:
+        modes = {m: quick_mode(args, m, G, rank, dev) for m in ("bf16", "tf32") if m != args.math}
 
     cpu = None
     if rank == 0 and G == 1 and not args.no_cpu_baseline:
@@ -790,15 +851,18 @@ def run_glp(args, ws, rank, local):
             dist.destroy_process_group()
         return
     info0 = [s.conv.info for s in states]
+    knobs = {k: v for k, v in os.environ.items() if k.startswith("GLP_")}
     line = {
         "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": G,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
-        "dtype": args.math, "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
+        "dtype": DTYPE[args.math], "data": "synthetic (seeded, Table 5 shapes; glp_workloads)",
         "config": {"workload": CONFIG_NAMES[args.workload], "model": "conv layers only",
                    "global_batch": images_per_step, "per_gpu_batch": n_local[0],
                    "layers": [s.name for s in states], "math": args.math,
-                   "parallelism": f"dp{G}", "exchange": args.exchange, "l2": "inputs larger than L2 (step working set "
+                   "parallelism": f"dp{G}", "exchange": args.exchange + (
+                       " (per-unit buckets overlapped with the backward)" if step.bucketed else ""),
+                   "l2": "inputs larger than L2 (step working set "
                    f"{sum(v.numel() * 4 for s in states for v in s.t.values()) / 1e9:.2f} GB)",
                    "step_gflop": round(step_flops / 1e9, 1),
                    "samples_in_flight": [i.samples_in_flight for i in info0],
@@ -806,17 +870,50 @@ def run_glp(args, ws, rank, local):
         "tflops_step": round(step_flops / (ms_per_step * 1e-3) / 1e12, 1),
         "roofline": roofline,
         "kernels": [{k: r[k] for k in ("layer", "pass", "avg_us", "tflops")} for r in kern],
+        "modes": modes,
         "cpu_baseline": cpu,
         "clocks": clk,
         "e2e": e2e,
         "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
         "launch": ("cuda_graph" if use_graph else "eager") +
-                  ("" if (args.serial or not use_graph) else
-                   f" (step DAG: {len(levels)} levels, up to {width} concurrent units)"),
+                  ("" if args.serial else
+                   f" (step DAG: {len(step.levels)} levels, up to {step.width} concurrent units)"),
+        "env_knobs": knobs,
     }
     print(json.dumps(line), flush=True)
     if G > 1:
         dist.destroy_process_group()
+
+
+def make_roofline(args, states, kern, ms_per_step):
+    """Roofline of the dominant kernel (largest share of the step): achieved = its algorithmic
+    flops per launch / its live CUDA-event duration; peak = the measured burst bf16 figure of
+    MEASURED_PEAKS.json (the kernel is event-timed alone, in a sub-second region) times the
+    guide's nominal ratio for the kernel's dtype (tf32: 1.1/2.25; 3xTF32: three tf32 MMAs per
+    fp32-equivalent flop, /3).  The sustained figure is given as context."""
+    peaks = load_peaks()
+    dom = max(kern, key=lambda r: r["total_us"])
+    ratio = {"bf16": 1.0, "tf32": NOMINAL_TF32_OVER_BF16, "fp32": NOMINAL_TF32_OVER_BF16 / 3}[args.math]
+    peak_tf = peaks["bf16_tflops"] * ratio
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get(f"{args.workload}/{dom['layer']}/{dom['pass']}/{args.math}")
+        except Exception:
+            traffic = None
+    src = {"bf16": " bf16 burst", "tf32": " bf16 burst x 1.1/2.25 (tf32)",
+           "fp32": " bf16 burst x 1.1/2.25 / 3 (3xTF32: three tf32 MMAs per flop)"}[args.math]
+    out = {"bound": "tensor", "achieved": dom["tflops"], "peak": round(peak_tf, 1),
+           "unit": "TFLOP/s", "frac": round(dom["tflops"] / peak_tf, 4), "traffic": traffic,
+           "kernel": f"{kernel_name(states, dom)} {dom['layer']} {dom['pass']}",
+           "peak_source": peaks["source"] + src,
+           "share_of_step": round(dom["total_us"] / 1e3 / (ms_per_step * args.steps), 4),
+           "frac_of_sustained_peak": round(dom["tflops"] / (peaks["bf16_tflops_sustained"] * ratio), 4)}
+    if args.math == "fp32":
+        # the same kernel against the tensor pipe's nominal tf32 rate (1.1 PF/s dense, /3)
+        out["frac_of_nominal_tf32"] = round(dom["tflops"] / (1100.0 / 3), 4)
+    return out
 
 
 # ------------------------------------------------------------------------- CPU oracle --------
@@ -930,14 +1027,56 @@ def run_reference(args, ws, rank):
     print(json.dumps(line), flush=True)
 
 
+def free_port() -> int:
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def relaunch(args) -> int:
+    """`python bench.py --gpus N` (N > 1) outside torchrun: start the N ranks ourselves (one
+    process per GPU) with torch.distributed.run on 127.0.0.1; rank 0 prints the line."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+           "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def dry_run(ws, rank):
+    """Launcher plumbing check on CPU (gloo): every rank contributes 1, rank 0 prints the count."""
+    import torch
+    import torch.distributed as dist
+    if ws > 1:
+        dist.init_process_group("gloo")
+    t = torch.ones(1)
+    if ws > 1:
+        dist.all_reduce(t)
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "n_gpus": ws, "ranks_seen": int(t.item()),
+                          "dry_run": True}), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
 def main():
     args = parse_args()
     ws, rank, local = dist_env()
-    if ws != args.gpus and ws > 1:
-        print(f"warning: WORLD_SIZE={ws} but --gpus {args.gpus}", file=sys.stderr)
     if args.impl == "reference":
         run_reference(args, ws, rank)
         return
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(relaunch(args))
+    if ws != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}: refusing to run a different "
+                 "number of ranks than asked")
+    if args.dry_run:
+        dry_run(ws, rank)
+        return
+    import torch
+    if torch.cuda.device_count() < (local + 1):
+        sys.exit(f"bench.py: rank {rank} needs cuda:{local} but {torch.cuda.device_count()} "
+                 "CUDA device(s) are visible (there is no CPU fallback)")
     if args.scheme == "pool":
         if rank == 0:
             run_pool(args)

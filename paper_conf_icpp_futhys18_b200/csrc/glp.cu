@@ -1417,10 +1417,10 @@ glp_status_t tc_bwd(glp_plan_s &P, const float *x, const BrIn &dy, const BrIn &w
 }
 
 // out = a + b elementwise (one IEEE fp32 add per element: commutative, so a tree of these is
-// bitwise independent of which rank holds which operand).
-__global__ void __launch_bounds__(256) sum2_kernel(const float *__restrict__ a,
-                                                   const float *__restrict__ b,
-                                                   float *__restrict__ out, size_t n) {
+// bitwise independent of which rank holds which operand).  out may alias a or b (the tree adds
+// in place), so no pointer is __restrict__.
+__global__ void __launch_bounds__(256) sum2_kernel(const float *a, const float *b, float *out,
+                                                   size_t n) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n;
        i += (size_t)gridDim.x * blockDim.x)
     out[i] = a[i] + b[i];

@@ -51,6 +51,14 @@ class FlatGrads:
         s = self.slots[i]
         return self.buf[s.b_off:s.b_off + s.co]
 
+    def bucket(self, idxs):
+        """The contiguous slice [dW_i | db_i | ... ] of the slots `idxs` (consecutive): one unit's
+        all-reduce bucket, issued as soon as that unit's filter gradient is reduced (bench.py
+        overlaps the buckets with the remaining backward, in reverse layer order)."""
+        lo = self.slots[min(idxs)].w_off
+        hi = max(self.slots[j].b_off + self.slots[j].co for j in idxs)
+        return self.buf[lo:hi]
+
     def allreduce(self, group=None):
         import torch.distributed as dist
         if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
@@ -126,13 +134,15 @@ class TreeAllreduce:
         if not (dist.is_available() and dist.is_initialized()):
             return acc
         world = dist.get_world_size(self.group)
-        rank = dist.get_rank(self.group)
+        rank = dist.get_rank(self.group)   # rank within the group
         recv = acc.clone()
         d = 1
         while d < world:
             partner = rank ^ d
-            ops = [dist.P2POp(dist.isend, acc, partner, self.group),
-                   dist.P2POp(dist.irecv, recv, partner, self.group)]
+            # P2POp takes the peer's GLOBAL rank: map the group rank (identity for the default group)
+            peer = partner if self.group is None else dist.get_global_rank(self.group, partner)
+            ops = [dist.P2POp(dist.isend, acc, peer, self.group),
+                   dist.P2POp(dist.irecv, recv, peer, self.group)]
             for r in dist.batch_isend_irecv(ops):
                 r.wait()
             if rank < partner:

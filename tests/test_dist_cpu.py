@@ -155,3 +155,73 @@ def test_leaf_partition():
         rank_leaves(0, 3)
     with pytest.raises(ValueError):
         leaf_range(100, 0)
+
+
+def _bucket_worker(rank, world, port, q):
+    """bench.py's overlapped exchange: one all_reduce per unit bucket, issued in reverse layer
+    order, must give the same buffer as the single whole-buffer all_reduce."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    shapes = [(4, 3, 3, 3), (6, 4, 1, 1), (5, 6, 5, 5)]
+    a, b = FlatGrads(shapes), FlatGrads(shapes)
+    g = torch.Generator().manual_seed(100 + rank)
+    a.buf.copy_(torch.randn(a.numel, generator=g))
+    b.buf.copy_(a.buf)
+    a.allreduce()
+    works = [dist.all_reduce(b.bucket([i]), async_op=True) for i in reversed(range(len(shapes)))]
+    for w in works:
+        w.wait()
+    q.put((rank, a.buf.numpy().copy(), b.buf.numpy().copy(),
+           b.bucket([1, 2]).numel() == b.numel - (4 * 27 + 4)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_bucketed_allreduce_equals_flat():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bucket_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for _, flat, buck, ok in res:
+        assert ok
+        np.testing.assert_array_equal(flat, buck)   # two-operand fp32 sums: bitwise
+    np.testing.assert_array_equal(res[0][1], res[1][1])
+
+
+def _subgroup_tree_worker(rank, world, port, q):
+    """TreeAllreduce on a subgroup whose group ranks differ from the global ranks (global ranks
+    1 and 3 of 4 form the group): the partner must be mapped to its global rank."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    grp = dist.new_group([1, 3])
+    if rank in (1, 3):
+        gr = dist.get_rank(grp)
+        parts = _leaf_parts()
+        mine = [torch.from_numpy(parts[j].copy()) for j in rank_leaves(gr, 2)]
+        out = TreeAllreduce(group=grp)(mine)
+        q.put((rank, out.numpy().copy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_tree_allreduce_on_subgroup():
+    ref = tree_sum([torch.from_numpy(p.copy()) for p in _leaf_parts()],
+                   lambda a, b, o: torch.add(a, b, out=o)).numpy()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_subgroup_tree_worker, args=(r, 4, port, q)) for r in range(4)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(timeout=60)
+    assert sorted(res) == [1, 3]
+    for r in res:
+        np.testing.assert_array_equal(res[r], ref)

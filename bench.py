@@ -1070,6 +1070,10 @@ def main():
     if ws != args.gpus:
         sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}: refusing to run a different "
                  "number of ranks than asked")
+    diag = sorted(k for k in os.environ if k.startswith("GLP_DEBUG"))
+    if diag:
+        sys.exit(f"bench.py: diagnostic knob(s) {diag} set: they skip work in -DGLP_DIAG builds, so "
+                 "no throughput is printed (unset them)")
     if args.dry_run:
         dry_run(ws, rank)
         return

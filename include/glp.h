@@ -133,6 +133,36 @@ glp_status_t glp_conv_desc_destroy(glp_conv_desc_t desc);
  * P264: outputs must be bitwise identical for every S). */
 glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t desc, int device, glp_math_t math,
                       int samples_in_flight);
+/* Plan options: choices between alternative kernels / tilings of the SAME computation.  Every
+ * option value gives bitwise the same outputs as the default for a given (shape, math mode)
+ * (the GEMMs have no K split but the wgrad one, whose split count and order are shape-only; each
+ * alternative is tested for bitwise equality), so the options only move time.  They exist for
+ * tests and A/B measurements; the library reads no environment variables (diagnostic builds,
+ * -DGLP_DIAG, add work-skipping timing hooks and never ship).  glp_plan == glp_plan_ex with the
+ * defaults of glp_plan_options_default. */
+typedef struct {
+  int cta_pairs;          /* 1: tcgen05 cta_group::2 CTA pairs where they apply; 0: single-CTA MMAs */
+  int wgrad_cta_pairs;    /* 1: CTA pairs for the filter gradient too; 0: not                      */
+  int halo_wgrad;         /* 1: shared-halo filter gradient for space-to-depth layers; 0: im2col   */
+  int halo_fwd;           /* 1: shared-halo forward for space-to-depth layers; 0: im2col           */
+  int halo_dgrad;         /* 1: shared-halo backward-data where the cost model picks it; 0: never;
+                             2: wherever legal                                                     */
+  int fused_dy;           /* 1: the halo filter gradient builds its dy operand from fp32 dy; 0: it
+                             reads the packed dy                                                   */
+  int fused_dy_builders;  /* 0: model; 1: cp.async landing zone; 2 or 3: register builder groups   */
+  int max_kblocks_per_stage; /* 1..4 (k-blocks per pipeline stage cap; 4 = default)                */
+  int wgrad_tile_n;       /* 0: model; else the filter-gradient N tile (multiple of 16, <= 256)    */
+  int tile_units;         /* fwd/dgrad tile model applies below this many work units per slot (2)  */
+  int bn_model;           /* 1: fwd/dgrad N-tile model for small grids; 0: always the default tile */
+  int pack_block;         /* 0: warp-tiled activation pack; 1: block-tiled                         */
+  int s2d_block;          /* 0: warp-per-32-pixel space-to-depth pack; 1: block-persistent          */
+  int smem_cap;           /* dynamic shared memory budget of the persistent GEMMs, bytes (232448)  */
+  int pdl;                /* 1: programmatic dependent launch between the plan's kernels; 0: not   */
+} glp_plan_options_t;
+glp_status_t glp_plan_options_default(glp_plan_options_t *opts);
+/* opts may be NULL (defaults).  GLP_ERR_INVALID_VALUE for an out-of-range option. */
+glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t desc, int device, glp_math_t math,
+                         int samples_in_flight, const glp_plan_options_t *opts);
 glp_status_t glp_plan_get_info(glp_plan_t plan, glp_plan_info_t *info);
 glp_status_t glp_plan_destroy(glp_plan_t plan);
 

@@ -53,6 +53,28 @@ class KernelAttr(ctypes.Structure):
     _fields_ = [("threads", _c_int), ("regs", _c_int), ("smem_bytes", _c_int), ("tmem_cols", _c_int)]
 
 
+class PlanOptions(ctypes.Structure):
+    """glp_plan_options_t: alternative kernels / tilings of the same computation (bitwise-equal
+    outputs; tests and A/B measurements only)."""
+    _fields_ = [("cta_pairs", _c_int), ("wgrad_cta_pairs", _c_int), ("halo_wgrad", _c_int),
+                ("halo_fwd", _c_int), ("halo_dgrad", _c_int), ("fused_dy", _c_int),
+                ("fused_dy_builders", _c_int), ("max_kblocks_per_stage", _c_int),
+                ("wgrad_tile_n", _c_int), ("tile_units", _c_int), ("bn_model", _c_int),
+                ("pack_block", _c_int), ("s2d_block", _c_int), ("smem_cap", _c_int), ("pdl", _c_int)]
+
+
+def plan_options(**kw) -> PlanOptions:
+    """The library defaults (glp_plan_options_default) with the given fields replaced."""
+    o = PlanOptions()
+    _ck(lib().glp_plan_options_default(ctypes.byref(o)), "glp_plan_options_default")
+    names = {f for f, _ in PlanOptions._fields_}
+    for k, v in kw.items():
+        if k not in names:
+            raise ValueError(f"unknown plan option {k!r}")
+        setattr(o, k, int(v))
+    return o
+
+
 # every symbol include/glp.h declares (checked by tests/test_abi.py)
 EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_destroy", "glp_plan",
            "glp_plan_get_info", "glp_plan_destroy", "glp_conv_fwd", "glp_conv_bwd_data",
@@ -63,7 +85,8 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_stage_bwd_filter", "glp_stage_reduce", "glp_conv_group_desc_create",
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
            "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
-           "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups", "glp_sum2"]
+           "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups", "glp_sum2",
+           "glp_plan_ex", "glp_plan_options_default"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA, GLP_PACK_W_BOTH = 0, 1, 2, 3, 4, 5
 
@@ -95,6 +118,8 @@ def lib():
         L.glp_conv_desc_get_output.argtypes = [_vp, P(_c_int), P(_c_int)]
         L.glp_conv_desc_destroy.argtypes = [_vp]
         L.glp_plan.argtypes = [P(_vp), _vp, _c_int, _c_int, _c_int]
+        L.glp_plan_ex.argtypes = [P(_vp), _vp, _c_int, _c_int, _c_int, P(PlanOptions)]
+        L.glp_plan_options_default.argtypes = [P(PlanOptions)]
         L.glp_plan_get_info.argtypes = [_vp, P(PlanInfo)]
         L.glp_plan_destroy.argtypes = [_vp]
         L.glp_conv_fwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
@@ -169,6 +194,26 @@ def _ptr(t):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
 
 
+def _checked(t, shape, device, name, nullable=False):
+    """Pointer of a tensor the kernels will read or write: fp32, contiguous, on the plan's CUDA
+    device, exactly `shape` (the kernels index N*C*H*W floats from the pointer, so anything else
+    would read or write past the allocation).  Raises ValueError before any library call."""
+    if t is None:
+        if nullable:
+            return None
+        raise ValueError(f"{name}: tensor required")
+    import torch
+    if t.dtype != torch.float32:
+        raise ValueError(f"{name}: dtype {t.dtype}, expected torch.float32")
+    if not t.is_cuda or t.device.index != device:
+        raise ValueError(f"{name}: on {t.device}, expected cuda:{device}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: not contiguous")
+    if tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name}: shape {tuple(t.shape)}, expected {tuple(shape)}")
+    return ctypes.c_void_p(t.data_ptr())
+
+
 def _ptrs(ts):
     """Pointer array (const float *const *) of a list of tensors (None entries -> NULL); the
     array object must stay alive for the duration of the call."""
@@ -176,6 +221,20 @@ def _ptrs(ts):
         return None
     arr = (ctypes.c_void_p * len(ts))(*[(None if t is None else t.data_ptr()) for t in ts])
     return ctypes.cast(arr, ctypes.c_void_p), arr
+
+
+def _checked_list(ts, shapes, device, name, nullable=False, entries_nullable=False):
+    """Pointer array of per-branch tensors, each checked as _checked (None entries allowed only
+    where the library allows them, e.g. a branch without bias)."""
+    if ts is None:
+        if nullable:
+            return None
+        raise ValueError(f"{name}: list required")
+    if len(ts) != len(shapes):
+        raise ValueError(f"{name}: {len(ts)} tensors for {len(shapes)} branches")
+    for i, (t, sh) in enumerate(zip(ts, shapes)):
+        _checked(t, sh, device, f"{name}[{i}]", nullable=entries_nullable)
+    return _ptrs(ts)
 
 
 def _stream(stream):
@@ -186,7 +245,9 @@ def _stream(stream):
 
 def sum2(a, b, out, stream=None):
     """out = a + b (fp32 CUDA tensors of equal size): the deterministic tree's add (glp_sum2)."""
-    _ck(lib().glp_sum2(_ptr(a), _ptr(b), _ptr(out), a.numel(), _stream(stream)), "glp_sum2")
+    dev = a.device.index if a.is_cuda else -1
+    pa, pb, po = (_checked(t, tuple(a.shape), dev, n) for t, n in ((a, "a"), (b, "b"), (out, "out")))
+    _ck(lib().glp_sum2(pa, pb, po, a.numel(), _stream(stream)), "glp_sum2")
     return out
 
 
@@ -212,7 +273,8 @@ class ConvLayer:
     ``stream`` (default: torch's current stream) without synchronising."""
 
     def __init__(self, N, C, H, W, Co, K, stride=1, pad=0, math="bf16", device=0,
-                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None, branches=None, groups=1):
+                 samples_in_flight=0, Kw=None, stride_w=None, pad_w=None, branches=None, groups=1,
+                 options=None):
         import torch
         self.groups = int(groups)
         self.branches = None if branches is None else [int(c) for c in branches]
@@ -240,8 +302,11 @@ class ConvLayer:
         self.math = MATH[math] if isinstance(math, str) else int(math)
         self.device = int(device)
         self._plan = _vp()
-        _ck(L.glp_plan(ctypes.byref(self._plan), self._desc, self.device, self.math,
-                       int(samples_in_flight)), "glp_plan")
+        opts = options if isinstance(options, PlanOptions) or options is None \
+            else plan_options(**options)
+        _ck(L.glp_plan_ex(ctypes.byref(self._plan), self._desc, self.device, self.math,
+                          int(samples_in_flight), None if opts is None else ctypes.byref(opts)),
+            "glp_plan_ex")
         self.info = PlanInfo()
         _ck(L.glp_plan_get_info(self._plan, ctypes.byref(self.info)), "glp_plan_get_info")
         nbytes = max(self.info.ws_fwd, self.info.ws_bwd_data, self.info.ws_bwd_filter,
@@ -275,41 +340,59 @@ class ConvLayer:
                 "tmem_cols": a.tmem_cols, "model": m.value, "runtime": r.value}
 
     # compute
+    # tensor checks (shape, dtype, device, contiguity) before any library call
+    def _x(self, t, name="x"):
+        return _checked(t, self.x_shape, self.device, name)
+
+    def _y(self, t, name="y"):
+        return _checked(t, self.y_shape, self.device, name)
+
+    def _w(self, t, name="w"):
+        return _checked(t, self.w_shape, self.device, name)
+
+    def _b(self, t, name="b"):
+        return _checked(t, (self.geom.Co,), self.device, name, nullable=True)
+
     def fwd(self, x, w, b, y, stream=None):
-        _ck(lib().glp_conv_fwd(self._plan, _ptr(x), _ptr(w), _ptr(b), _ptr(y),
+        _ck(lib().glp_conv_fwd(self._plan, self._x(x), self._w(w), self._b(b), self._y(y),
                                ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_conv_fwd")
         return y
 
     def bwd_data(self, dy, w, dx, stream=None):
-        _ck(lib().glp_conv_bwd_data(self._plan, _ptr(dy), _ptr(w), _ptr(dx),
+        _ck(lib().glp_conv_bwd_data(self._plan, self._y(dy, "dy"), self._w(w), self._x(dx, "dx"),
                                     ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_conv_bwd_data")
         return dx
 
     def bwd_filter(self, x, dy, dw, db=None, accumulate=False, stream=None):
-        _ck(lib().glp_conv_bwd_filter(self._plan, _ptr(x), _ptr(dy), _ptr(dw), _ptr(db),
-                                      int(bool(accumulate)), ctypes.c_void_p(self.ws_ptr),
-                                      self.ws_bytes, _stream(stream)), "glp_conv_bwd_filter")
+        _ck(lib().glp_conv_bwd_filter(self._plan, self._x(x), self._y(dy, "dy"), self._w(dw, "dw"),
+                                      self._b(db, "db"), int(bool(accumulate)),
+                                      ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_conv_bwd_filter")
         return dw, db
 
     def bwd(self, x, dy, w, dx, dw, db=None, accumulate=False, stream=None):
-        _ck(lib().glp_conv_bwd(self._plan, _ptr(x), _ptr(dy), _ptr(w), _ptr(dx), _ptr(dw),
-                               _ptr(db), int(bool(accumulate)), ctypes.c_void_p(self.ws_ptr),
-                               self.ws_bytes, _stream(stream)), "glp_conv_bwd")
+        pdx = None if dx is None else self._x(dx, "dx")
+        _ck(lib().glp_conv_bwd(self._plan, self._x(x), self._y(dy, "dy"), self._w(w), pdx,
+                               self._w(dw, "dw"), self._b(db, "db"), int(bool(accumulate)),
+                               ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
+            "glp_conv_bwd")
         return dx, dw, db
 
     # staged execution (include/glp.h "staged execution"): one C call per kernel group
     def stage_pack(self, what, src, stream=None):
-        _ck(lib().glp_stage_pack(self._plan, int(what), _ptr(src), ctypes.c_void_p(self.ws_ptr),
+        shape = {GLP_PACK_X: self.x_shape, GLP_PACK_DY: self.y_shape, GLP_PACK_DY_DB: self.y_shape}
+        p = _checked(src, shape.get(int(what), self.w_shape), self.device, "src")
+        _ck(lib().glp_stage_pack(self._plan, int(what), p, ctypes.c_void_p(self.ws_ptr),
                                  self.ws_bytes, _stream(stream)), "glp_stage_pack")
 
     def stage_fwd(self, b, y, stream=None):
-        _ck(lib().glp_stage_fwd(self._plan, _ptr(b), _ptr(y), ctypes.c_void_p(self.ws_ptr),
+        _ck(lib().glp_stage_fwd(self._plan, self._b(b), self._y(y), ctypes.c_void_p(self.ws_ptr),
                                 self.ws_bytes, _stream(stream)), "glp_stage_fwd")
 
     def stage_bwd_data(self, dx, stream=None):
-        _ck(lib().glp_stage_bwd_data(self._plan, _ptr(dx), ctypes.c_void_p(self.ws_ptr),
+        _ck(lib().glp_stage_bwd_data(self._plan, self._x(dx, "dx"), ctypes.c_void_p(self.ws_ptr),
                                      self.ws_bytes, _stream(stream)), "glp_stage_bwd_data")
 
     def stage_bwd_filter(self, stream=None):
@@ -317,7 +400,8 @@ class ConvLayer:
                                        _stream(stream)), "glp_stage_bwd_filter")
 
     def stage_reduce(self, dw, db=None, accumulate=False, stream=None):
-        _ck(lib().glp_stage_reduce(self._plan, _ptr(dw), _ptr(db), int(bool(accumulate)),
+        _ck(lib().glp_stage_reduce(self._plan, self._w(dw, "dw"), self._b(db, "db"),
+                                   int(bool(accumulate)),
                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_stage_reduce")
 
@@ -329,42 +413,67 @@ class ConvLayer:
         g = self.geom
         return [(c, g.C, g.Kh, g.Kw) for c in self.branches]
 
+    def _brw(self):
+        return self.branch_w_shapes()
+
+    def _bry(self):
+        return self.branch_y_shapes()
+
+    def _brb(self):
+        return [(c,) for c in self.branches]
+
     def group_fwd(self, x, ws, bs, ys, stream=None):
-        (pw, _a), (py, _b) = _ptrs(ws), _ptrs(ys)
-        pb = _ptrs(bs)
-        _ck(lib().glp_conv_group_fwd(self._plan, _ptr(x), pw, None if pb is None else pb[0], py,
+        dv = self.device
+        (pw, _a) = _checked_list(ws, self._brw(), dv, "w")
+        (py, _b) = _checked_list(ys, self._bry(), dv, "y")
+        pb = _checked_list(bs, self._brb(), dv, "b", nullable=True, entries_nullable=True)
+        _ck(lib().glp_conv_group_fwd(self._plan, self._x(x), pw, None if pb is None else pb[0], py,
                                      ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_conv_group_fwd")
         return ys
 
     def group_bwd(self, x, dys, ws, dx, dws, dbs=None, accumulate=False, stream=None):
-        (pdy, _a), (pw, _b), (pdw, _c) = _ptrs(dys), _ptrs(ws), _ptrs(dws)
-        pdb = _ptrs(dbs)
-        _ck(lib().glp_conv_group_bwd(self._plan, _ptr(x), pdy, pw, _ptr(dx), pdw,
+        dv = self.device
+        (pdy, _a) = _checked_list(dys, self._bry(), dv, "dy")
+        (pw, _b) = _checked_list(ws, self._brw(), dv, "w")
+        (pdw, _c) = _checked_list(dws, self._brw(), dv, "dw")
+        pdb = _checked_list(dbs, self._brb(), dv, "db", nullable=True)
+        pdx = None if dx is None else self._x(dx, "dx")
+        _ck(lib().glp_conv_group_bwd(self._plan, self._x(x), pdy, pw, pdx, pdw,
                                      None if pdb is None else pdb[0], int(bool(accumulate)),
                                      ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_conv_group_bwd")
         return dx, dws, dbs
 
     def stage_pack_group(self, what, srcs, stream=None):
-        p, _a = _ptrs(srcs)
+        dv = self.device
+        if int(what) == GLP_PACK_X:
+            p, _a = _checked_list(srcs, [self.x_shape], dv, "src")
+        elif int(what) in (GLP_PACK_DY, GLP_PACK_DY_DB):
+            p, _a = _checked_list(srcs, self._bry(), dv, "src")
+        else:
+            p, _a = _checked_list(srcs, self._brw(), dv, "src")
         _ck(lib().glp_stage_pack_group(self._plan, int(what), p, ctypes.c_void_p(self.ws_ptr),
                                        self.ws_bytes, _stream(stream)), "glp_stage_pack_group")
 
     def stage_fwd_group(self, bs, ys, stream=None):
-        pb, (py, _a) = _ptrs(bs), _ptrs(ys)
+        pb = _checked_list(bs, self._brb(), self.device, "b", nullable=True, entries_nullable=True)
+        (py, _a) = _checked_list(ys, self._bry(), self.device, "y")
         _ck(lib().glp_stage_fwd_group(self._plan, None if pb is None else pb[0], py,
                                       ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_stage_fwd_group")
 
     def stage_reduce_group(self, dws, dbs=None, accumulate=False, stream=None):
-        (pdw, _a), pdb = _ptrs(dws), _ptrs(dbs)
+        (pdw, _a) = _checked_list(dws, self._brw(), self.device, "dw")
+        pdb = _checked_list(dbs, self._brb(), self.device, "db", nullable=True)
         _ck(lib().glp_stage_reduce_group(self._plan, pdw, None if pdb is None else pdb[0],
                                          int(bool(accumulate)), ctypes.c_void_p(self.ws_ptr),
                                          self.ws_bytes, _stream(stream)), "glp_stage_reduce_group")
 
     def debug_im2col(self, x, n, col, stream=None):
-        _ck(lib().glp_debug_im2col(self._plan, _ptr(x), int(n), _ptr(col),
+        g = self.geom
+        pcol = _checked(col, (g.C * g.Kh * g.Kw, self.Ho * self.Wo), self.device, "col")
+        _ck(lib().glp_debug_im2col(self._plan, self._x(x), int(n), pcol,
                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_debug_im2col")
         return col
@@ -400,20 +509,30 @@ class StreamPool:
             "glp_pool_get_info")
         self.n_streams, self.eq7_bound = ns.value, eq7.value
         nbytes = wsb.value + 1024
+        self.device = int(device)
+        g = self.geom
+        Ho, Wo = (H + 2 * pad - K) // stride + 1, (W + 2 * pad - K) // stride + 1
+        self._shapes = {"x": (N, C, H, W), "y": (N, Co, Ho, Wo), "w": (Co, C, K, K), "b": (Co,)}
         self._ws_buf = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{int(device)}")
         off = (-self._ws_buf.data_ptr()) % 1024
         self.ws_ptr = self._ws_buf.data_ptr() + off
         self.ws_bytes = nbytes - off
 
+    def _c(self, t, kind, name, nullable=False):
+        return _checked(t, self._shapes[kind], self.device, name, nullable)
+
     def fwd(self, x, w, b, y, stream=None):
-        _ck(lib().glp_pool_conv_fwd(self._pool, _ptr(x), _ptr(w), _ptr(b), _ptr(y),
+        _ck(lib().glp_pool_conv_fwd(self._pool, self._c(x, "x", "x"), self._c(w, "w", "w"),
+                                    self._c(b, "b", "b", True), self._c(y, "y", "y"),
                                     ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_pool_conv_fwd")
         return y
 
     def bwd(self, x, dy, w, dx, dw, db=None, stream=None):
-        _ck(lib().glp_pool_conv_bwd(self._pool, _ptr(x), _ptr(dy), _ptr(w), _ptr(dx), _ptr(dw),
-                                    _ptr(db), ctypes.c_void_p(self.ws_ptr), self.ws_bytes,
+        _ck(lib().glp_pool_conv_bwd(self._pool, self._c(x, "x", "x"), self._c(dy, "y", "dy"),
+                                    self._c(w, "w", "w"), self._c(dx, "x", "dx", True),
+                                    self._c(dw, "w", "dw"), self._c(db, "b", "db", True),
+                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes,
                                     _stream(stream)), "glp_pool_conv_bwd")
         return dx, dw, db
 

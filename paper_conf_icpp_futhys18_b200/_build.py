@@ -22,17 +22,28 @@ def stale() -> bool:
     return any(os.path.getmtime(s) > t for s in SOURCES)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
-        return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *FLAGS, "-o", tmp, os.path.join(PKG, "csrc", "glp.cu")]
+DIAG_LIB = os.path.join(PKG, "libglp_diag.so")
+
+
+def build(force: bool = False, verbose: bool = False, diag: bool = False) -> str:
+    """libglp.so (the product), or with diag=True libglp_diag.so: the same sources compiled with
+    -DGLP_DIAG, which adds the work-skipping / cycle-counter hooks of tools/stage_probe.py and
+    tools/clk_probe.py (GLP_DEBUG_* environment variables; results are wrong in skip modes).  The
+    diagnostic library is never loaded unless GLP_LIB points at it."""
+    lib = DIAG_LIB if diag else LIB
+    if not force and os.path.exists(lib) and not any(
+            os.path.getmtime(s) > os.path.getmtime(lib) for s in SOURCES):
+        return lib
+    tmp = lib + f".tmp{os.getpid()}"
+    cmd = [NVCC, *FLAGS, *(["-DGLP_DIAG"] if diag else []), "-o", tmp,
+           os.path.join(PKG, "csrc", "glp.cu")]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force=True, verbose=True))
+    import sys
+    print(build(force=True, verbose=True, diag="--diag" in sys.argv))

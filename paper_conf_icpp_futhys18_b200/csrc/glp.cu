@@ -517,12 +517,16 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   h.a_bytes = (int)rup((long long)(R + K - 1) * WQ * 128, 1024);
   h.b_tap_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
   h.a_stages = 3;
+#ifdef GLP_DIAG
   if (const char *e = getenv("GLP_HD_ASTAGES")) h.a_stages = std::max(2, atoi(e));   // A/B runs
+#endif
   const int fixed = 1024 + h.a_stages * h.a_bytes + 8 * 64 + 16;
   // as many taps per B stage as keep >= 4 stages (the issuer's barrier round trip costs more than
   // the 8 MMAs of one tap)
   int min_bst = 4;
+#ifdef GLP_DIAG
   if (const char *e = getenv("GLP_HD_BSTAGES")) min_bst = std::max(2, atoi(e));   // A/B runs
+#endif
   h.b_taps = 1;
   while (h.b_taps < taps && (P.smem_cap - fixed) / ((h.b_taps + 1) * h.b_tap_bytes) >= min_bst) ++h.b_taps;
   h.b_bytes = h.b_taps * h.b_tap_bytes;
@@ -688,8 +692,10 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
       ++pp.ksub;
   const int stage_bytes = pp.ksub * kb_bytes;
   pp.stages = std::min(8, budget / stage_bytes);
+#ifdef GLP_DIAG
   if (const char *e = getenv("GLP_DEBUG_STAGES"))   // diagnostics: fewer ring stages
     pp.stages = std::max(2, std::min(pp.stages, atoi(e)));
+#endif
   if (pp.stages < 2) return fail(GLP_ERR_INTERNAL, "tile does not fit in smem");
   pp.acc_cols = (int)rup(pp.bn, 32);
   int tc = 32;
@@ -1607,8 +1613,27 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
   return GLP_OK;
 }
 
+glp_status_t glp_plan_options_default(glp_plan_options_t *o) {
+  if (!o) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 2, 1, 0, 0, 232448, 0};
+  return GLP_OK;
+}
+
 glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t math, int S) {
+  return glp_plan_ex(out, d, device, math, S, nullptr);
+}
+
+glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t math, int S,
+                         const glp_plan_options_t *opts) {
   if (!out || !d) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  glp_plan_options_t o;
+  glp_plan_options_default(&o);
+  if (opts) o = *opts;
+  if (o.halo_dgrad < 0 || o.halo_dgrad > 2 || o.fused_dy_builders < 0 || o.fused_dy_builders > 3 ||
+      o.max_kblocks_per_stage < 1 || o.max_kblocks_per_stage > 4 || o.wgrad_tile_n < 0 ||
+      o.wgrad_tile_n > 256 || o.wgrad_tile_n % 16 || o.tile_units < 0 || o.smem_cap < 65536 ||
+      o.smem_cap > 232448)
+    return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
   *out = nullptr;
   if (math != GLP_MATH_FP32 && math != GLP_MATH_TF32 && math != GLP_MATH_BF16 &&
       math != GLP_MATH_FP32_SIMT)
@@ -1649,27 +1674,30 @@ glp_status_t glp_plan(glp_plan_t *out, glp_conv_desc_t d, int device, glp_math_t
   P->x3 = (math == GLP_MATH_FP32) ? 1 : 0;
   P->sm_count = prop.multiProcessorCount;
   P->s_override = S;
-  if (const char *e = getenv("GLP_CTA_GROUP")) P->allow_cg2 = (atoi(e) != 1);
-  if (const char *e = getenv("GLP_KSUB")) {
-    P->ksub_max = std::max(1, std::min(4, atoi(e)));
-    P->allow_ksub2 = P->ksub_max > 1;
-  }
-  if (const char *e = getenv("GLP_WGRAD_CG2")) P->wgrad_cg2 = atoi(e) != 0;
-  if (const char *e = getenv("GLP_PDL")) P->pdl = atoi(e) != 0;
-  if (const char *e = getenv("GLP_BN_MODEL")) P->bn_model = atoi(e) != 0;
-  if (const char *e = getenv("GLP_HALO")) P->allow_halo = atoi(e) != 0;
-  if (const char *e = getenv("GLP_HFWD")) P->allow_hfwd = atoi(e) != 0;
-  if (const char *e = getenv("GLP_HALO_FDY")) P->allow_fdy = atoi(e) != 0;
-  if (const char *e = getenv("GLP_FDY_NCG")) P->fdy_ncg = atoi(e);
-  if (const char *e = getenv("GLP_HDGRAD")) P->allow_hdg = atoi(e);
-  if (const char *e = getenv("GLP_WGRAD_BN")) P->wgrad_bn = atoi(e);
-  if (const char *e = getenv("GLP_TILE_UNITS")) P->tile_units = atoi(e);
-  if (const char *e = getenv("GLP_PACK_BLOCK")) P->pack_block = atoi(e) != 0;
-  if (const char *e = getenv("GLP_S2D_BLOCK")) P->s2d_block = atoi(e) != 0;
-  if (const char *e = getenv("GLP_SMEM_CAP")) P->smem_cap = std::max(65536, std::min(232448, atoi(e)));
-  // diagnostics: GLP_DEBUG_CLK = device address of >= 4 * grid uint64 counters (tools/clk_probe.py)
+  // plan options (include/glp.h glp_plan_options_t): alternative kernels / tilings of the same
+  // computation, bitwise-equal outputs
+  P->allow_cg2 = o.cta_pairs != 0;
+  P->ksub_max = o.max_kblocks_per_stage;
+  P->allow_ksub2 = P->ksub_max > 1;
+  P->wgrad_cg2 = o.wgrad_cta_pairs != 0;
+  P->pdl = o.pdl != 0;
+  P->bn_model = o.bn_model != 0;
+  P->allow_halo = o.halo_wgrad != 0;
+  P->allow_hfwd = o.halo_fwd != 0;
+  P->allow_fdy = o.fused_dy != 0;
+  P->fdy_ncg = o.fused_dy_builders;
+  P->allow_hdg = o.halo_dgrad;
+  P->wgrad_bn = o.wgrad_tile_n;
+  P->tile_units = o.tile_units;
+  P->pack_block = o.pack_block != 0;
+  P->s2d_block = o.s2d_block != 0;
+  P->smem_cap = o.smem_cap;
+#ifdef GLP_DIAG
+  // diagnostic builds only (never the shipped library): GLP_DEBUG_CLK = device address of
+  // >= 4 * grid uint64 counters (tools/clk_probe.py); GLP_DEBUG_SKIP = work-skipping bits
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
   if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 31;
+#endif
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to
   // 32 would multiply the MMA work; those use the 16-byte-chunk cp.async gather.

@@ -1,6 +1,6 @@
 #!/bin/bash
 # GPU-box bench: timed run, ncu launch list, one ncu --set full capture of a top kernel.
-cd "$(dirname "$0")"
+cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 W=${WORKLOAD:-4}
 MATH=${MATH:-bf16}

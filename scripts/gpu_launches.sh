@@ -1,6 +1,6 @@
 #!/bin/bash
 # ncu launch list (time + dram bytes) of 2 serial eager bench steps, and optional full captures
-cd "$(dirname "$0")"
+cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 W=${WORKLOAD:-4}; MATH=${MATH:-bf16}; TAGN=${TAG:-step}
 timeout -s KILL 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \

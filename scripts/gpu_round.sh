@@ -2,10 +2,10 @@
 # Round evidence in one gpurun call: smoke + gpu tests, the default bench line, the reference
 # (oracle) arm, the ncu launch list of one step (time + dram bytes) and ncu --set full captures
 # of every GEMM launch of one step.
-cd "$(dirname "$0")"
+cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 TAGN=${TAG:-round}
-[ -z "$NOCHECK" ] && ./scripts_gpu_check.sh
+[ -z "$NOCHECK" ] && ./scripts/gpu_check.sh
 timeout -s KILL 600 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
 echo "bench rc=$?"; cat gpurun_out/bench_default.json; tail -3 gpurun_out/bench_default.err
 if [ -z "$NOREF" ]; then

@@ -115,3 +115,32 @@ def test_eq7_vs_oracle():
         got = glp.glp_analyze_eq7(lim, threads, smem, blocks)
         exp = A.eq7_bound(A.Kernel(blocks=blocks, threads=threads, smem=smem), dev)
         assert got == exp
+
+
+def test_plan_options_abi():
+    """glp_plan_options_default fills the documented defaults; glp_plan_ex rejects an
+    out-of-range option before touching a device (GLP_ERR_INVALID_VALUE)."""
+    o = glp.plan_options()
+    assert (o.cta_pairs, o.wgrad_cta_pairs, o.halo_wgrad, o.halo_fwd, o.halo_dgrad, o.fused_dy,
+            o.fused_dy_builders, o.max_kblocks_per_stage, o.smem_cap) == (1, 1, 1, 1, 1, 1, 0, 4, 232448)
+    L = glp.lib()
+    d = ctypes.c_void_p()
+    assert L.glp_conv_desc_create(ctypes.byref(d), 2, 3, 8, 8, 4, 3, 3, 1, 1, 1, 1) == 0
+    p = ctypes.c_void_p()
+    for bad in ({"halo_dgrad": 3}, {"max_kblocks_per_stage": 0}, {"wgrad_tile_n": 24},
+                {"smem_cap": 1000}):
+        ob = glp.plan_options(**bad)
+        assert L.glp_plan_ex(ctypes.byref(p), d, 0, glp.GLP_MATH_BF16, 0, ctypes.byref(ob)) == 1
+    with pytest.raises(ValueError):
+        glp.plan_options(no_such_option=1)
+    L.glp_conv_desc_destroy(d)
+
+
+def test_product_library_reads_no_environment():
+    """The shipped library has no getenv: knobs are explicit plan options (glp_plan_ex), and
+    the work-skipping diagnostics exist only in -DGLP_DIAG builds."""
+    blob = open(glp.LIB_PATH, "rb").read()
+    api = (b"GLP_OK", b"GLP_ERR_", b"GLP_PACK", b"GLP_PAC", b"GLP_MATH")   # enum names in messages
+    knobs = sorted(k for k in set(re.findall(rb"GLP_[A-Z][A-Z0-9_]+", blob))
+                   if not k.startswith(api))
+    assert knobs == [], knobs

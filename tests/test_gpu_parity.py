@@ -64,9 +64,11 @@ def _data(shape, exact=False, seed=1):
     return gen_custom(N, C, H, W, Co, K, K, seed, exact=exact, Ho=Ho, Wo=Wo, data_fed=exact and C <= 3)
 
 
-def _layer(shape, math, S=0):
+def _layer(shape, math, S=0, **opts):
+    """opts: plan options (glp_plan_options_t fields) selecting alternative kernels / tilings."""
     _, N, C, H, W, Co, K, St, P = shape
-    return glp.ConvLayer(N, C, H, W, Co, K, St, P, math=math, samples_in_flight=S)
+    return glp.ConvLayer(N, C, H, W, Co, K, St, P, math=math, samples_in_flight=S,
+                         options=opts or None)
 
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])
@@ -240,18 +242,16 @@ def test_staged_equals_composed(math):
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", [SHAPES[0], SHAPES[2], SHAPES[5], SHAPES[6]], ids=lambda s: s[0])
-def test_single_cta_mma_path(shape, math, monkeypatch):
-    """GLP_CTA_GROUP=1 forces single-CTA tcgen05 MMAs (no CTA pairs): still bit-exact on integer
-    data, and equal to the default (paired) plan on random data (same per-element K order)."""
+def test_single_cta_mma_path(shape, math):
+    """Plan option cta_pairs = 0 forces single-CTA tcgen05 MMAs (no CTA pairs): still bit-exact on
+    integer data, and equal to the default (paired) plan on random data (same per-element K order)."""
     d = _data(shape, exact=True, seed=21)
-    monkeypatch.setenv("GLP_CTA_GROUP", "1")
-    got = _run(_layer(shape, math), d)
+    got = _run(_layer(shape, math, cta_pairs=0), d)
     ref = _oracle(d, shape[7], shape[8])
     for k in ref:
         np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
     dr = _data(shape, seed=22)
-    one = _run(_layer(shape, math), dr)
-    monkeypatch.delenv("GLP_CTA_GROUP")
+    one = _run(_layer(shape, math, cta_pairs=0), dr)
     two = _run(_layer(shape, math), dr)
     for k in ("y", "dx"):
         np.testing.assert_array_equal(one[k], two[k], err_msg=k)
@@ -264,13 +264,12 @@ def test_single_cta_mma_path(shape, math, monkeypatch):
                                    ("c256_k3_n384", 2, 256, 7, 7, 384, 3, 1, 1)],
                          ids=lambda s: s[0])
 @pytest.mark.parametrize("cg2", ["0", "1"])
-def test_wgrad_cta_pairs_exact(shape, math, cg2, monkeypatch):
+def test_wgrad_cta_pairs_exact(shape, math, cg2):
     """Filter gradient with and without CTA pairs (cta_group::2, MN-major halves of B; the
     C_o = 384 case switches to 64-byte rows so bn/2 = 96 is whole atoms) is bit-exact on integer
     data, with the split partials reduced at the paired row pitch."""
-    monkeypatch.setenv("GLP_WGRAD_CG2", cg2)
     d = _data(shape, exact=True, seed=41)
-    got = _run(_layer(shape, math), d)
+    got = _run(_layer(shape, math, wgrad_cta_pairs=int(cg2)), d)
     ref = _oracle(d, shape[7], shape[8])
     np.testing.assert_array_equal(got["dw"], ref["dw"].astype(np.float32))
     np.testing.assert_array_equal(got["db"], ref["db"].astype(np.float32))
@@ -287,10 +286,10 @@ HALO_SHAPES = [
 
 
 @pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
-def test_halo_wgrad_exact(shape, monkeypatch):
+def test_halo_wgrad_exact(shape):
     """The shared-halo filter gradient (row-shifted SWIZZLE_128B descriptors over one staged x'
     tile per k-block, dy on the padded grid) is bit-exact on integer data, and so is the
-    backward-data pass that reads the padded dy; GLP_HALO=0 (im2col path) agrees bit for bit."""
+    backward-data pass that reads the padded dy; halo_wgrad = 0 (im2col path) agrees bit for bit."""
     d = _data(shape, exact=True, seed=43)
     ref = _oracle(d, shape[7], shape[8])
     layer = _layer(shape, "bf16")
@@ -298,8 +297,7 @@ def test_halo_wgrad_exact(shape, monkeypatch):
     got = _run(layer, d)
     for k in ("y", "dx", "dw", "db"):
         np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
-    monkeypatch.setenv("GLP_HALO", "0")
-    layer0 = _layer(shape, "bf16")
+    layer0 = _layer(shape, "bf16", halo_wgrad=0)
     assert layer0.info.wgrad_halo == 0
     got0 = _run(layer0, d)
     for k in ("dw", "db", "dx"):
@@ -325,10 +323,10 @@ def test_halo_wgrad_random_and_invariant(shape):
 
 
 @pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
-def test_halo_wgrad_fused_dy(shape, monkeypatch):
+def test_halo_wgrad_fused_dy(shape):
     """Fused-dy halo filter gradient (hwgrad_kernel<true>: the CTA's own warps build the dy
     operand from fp32 NCHW with the pack's RNE rounding, and emit the db partials): dW bitwise
-    equal to the packed-dy kernel (GLP_HALO_FDY=0: same operand bits, same MMA order), db within
+    equal to the packed-dy kernel (fused_dy = 0: same operand bits, same MMA order), db within
     fp32 summation-order noise of it; the staged calls (GLP_PACK_DY_DB only records dy,
     bwd_data packs it lazily) bitwise equal to the composed calls."""
     d = _data(shape, seed=49)
@@ -348,8 +346,7 @@ def test_halo_wgrad_fused_dy(shape, monkeypatch):
     torch.cuda.synchronize()
     for k, v in (("dx", dx), ("dw", dw), ("db", db)):
         np.testing.assert_array_equal(v.cpu().numpy(), ref[k], err_msg=k)
-    monkeypatch.setenv("GLP_HALO_FDY", "0")
-    layer0 = _layer(shape, "bf16")
+    layer0 = _layer(shape, "bf16", fused_dy=0)
     assert layer0.info.wgrad_fused_dy == 0 and layer0.info.wgrad_halo == 1
     got0 = _run(layer0, d)
     np.testing.assert_array_equal(got0["dw"], ref["dw"])
@@ -359,25 +356,24 @@ def test_halo_wgrad_fused_dy(shape, monkeypatch):
 
 
 @pytest.mark.parametrize("shape", HALO_SHAPES, ids=lambda s: s[0])
-def test_halo_fwd_exact(shape, monkeypatch):
+def test_halo_fwd_exact(shape):
     """The shared-halo forward (hfwd.cuh: one staged x' tile per 128 rows of the padded grid,
     row-shifted K-major SWIZZLE_128B descriptors per tap, resident W', invalid padded-grid rows
-    dropped) is bit-exact on integer data, and GLP_HFWD=0 (im2col forward) agrees bit for bit."""
+    dropped) is bit-exact on integer data, and halo_fwd = 0 (im2col forward) agrees bit for bit."""
     d = _data(shape, exact=True, seed=47)
     ref = _oracle(d, shape[7], shape[8])
     layer = _layer(shape, "bf16")
     assert layer.info.fwd_halo == 1
     got = _run(layer, d)
     np.testing.assert_array_equal(got["y"], ref["y"].astype(np.float32))
-    monkeypatch.setenv("GLP_HFWD", "0")
-    layer0 = _layer(shape, "bf16")
+    layer0 = _layer(shape, "bf16", halo_fwd=0)
     assert layer0.info.fwd_halo == 0
     got0 = _run(layer0, d)
     np.testing.assert_array_equal(got0["y"], got["y"])
 
 
 @pytest.mark.parametrize("shape", HALO_SHAPES[:3], ids=lambda s: s[0])
-def test_halo_fwd_random_and_invariant(shape, monkeypatch):
+def test_halo_fwd_random_and_invariant(shape):
     """Random data: y within the bf16 bar of the oracle and 1e-4 of the rounding-emulated oracle,
     bitwise identical across samples-in-flight overrides (grid sizes) and reruns, and equal to
     the im2col forward (same MMA order: taps in order, 4 K=16 steps per 64-channel atom)."""
@@ -390,8 +386,7 @@ def test_halo_fwd_random_and_invariant(shape, monkeypatch):
     assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= 1e-4
     for other in runs[1:]:
         np.testing.assert_array_equal(other, runs[0])
-    monkeypatch.setenv("GLP_HFWD", "0")
-    np.testing.assert_array_equal(_run(_layer(shape, "bf16"), d)["y"], runs[0])
+    np.testing.assert_array_equal(_run(_layer(shape, "bf16", halo_fwd=0), d)["y"], runs[0])
 
 
 # fused sibling groups (include/glp.h): name, N, C, H, W, branches, K, S, P
@@ -653,7 +648,7 @@ def test_pack_w_both_equals_separate(shape, math):
     np.testing.assert_array_equal(outs[1][1], outs[0][1])
 
 
-# unit-stride layers for the shared-halo backward-data kernel (hdgrad.cuh); GLP_HDGRAD=2 forces it
+# unit-stride layers for the shared-halo backward-data kernel (hdgrad.cuh); halo_dgrad = 2 forces it
 # where the cost model would keep the im2col kernel (small images waste more padded rows)
 HDG_SHAPES = [
     ("caffenet_conv2_b2", 2, 96, 27, 27, 256, 5, 1, 2),     # the model's own choice; odd unit count
@@ -664,20 +659,19 @@ HDG_SHAPES = [
 
 
 @pytest.mark.parametrize("shape", HDG_SHAPES, ids=lambda s: s[0])
-def test_halo_dgrad(shape, monkeypatch):
+def test_halo_dgrad(shape):
     """Shared-halo backward-data (4-D TMA halo of the packed dy per 64-channel block, flipped taps by
     row shift, CTA pairs with M = 256 MMAs): bit-exact on integer data, within 1e-4
     of the rounding-emulated oracle and 2e-2 of the fp64 oracle on random data, bitwise invariant
     across samples-in-flight overrides."""
-    monkeypatch.setenv("GLP_HDGRAD", "2")
-    layer = _layer(shape, "bf16")
+    layer = _layer(shape, "bf16", halo_dgrad=2)
     assert layer.info.dgrad_halo == 1
     d = _data(shape, exact=True, seed=53)
     got = _run(layer, d)
     ref = _oracle(d, shape[7], shape[8])
     np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32))
     d = _data(shape, seed=54)
-    runs = [_run(_layer(shape, "bf16", S), d)["dx"] for S in (0, 1, 0)]
+    runs = [_run(_layer(shape, "bf16", S, halo_dgrad=2), d)["dx"] for S in (0, 1, 0)]
     ref = _oracle(d, shape[7], shape[8])["dx"]
     emu = _oracle(d, shape[7], shape[8], x=EMU["bf16"](d["x"]), w=EMU["bf16"](d["w"]),
                   dy=EMU["bf16"](d["dy"]))["dx"]
@@ -696,14 +690,13 @@ def test_halo_dgrad_model_choice():
 
 
 @pytest.mark.parametrize("ncg", ["1", "2"])
-def test_halo_wgrad_fused_dy_variants(ncg, monkeypatch):
-    """The other fused-dy builder variants (GLP_FDY_NCG=1: cp.async landing zone; 2: two register
-    groups) give the same dW bits as the default and db within summation-order noise."""
+def test_halo_wgrad_fused_dy_variants(ncg):
+    """The other fused-dy builder variants (fused_dy_builders = 1: cp.async landing zone; 2: two
+    register groups) give the same dW bits as the default and db within summation-order noise."""
     shape = HALO_SHAPES[1]
     d = _data(shape, seed=55)
     ref = _run(_layer(shape, "bf16"), d)
-    monkeypatch.setenv("GLP_FDY_NCG", ncg)
-    layer = _layer(shape, "bf16")
+    layer = _layer(shape, "bf16", fused_dy_builders=int(ncg))
     assert layer.info.wgrad_fused_dy == 1
     got = _run(layer, d)
     np.testing.assert_array_equal(got["dw"], ref["dw"])
@@ -726,3 +719,30 @@ def test_fp32_long_reductions(shape):
     ref = _oracle(d, shape[7], shape[8])
     errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
     assert all(e <= TOL["fp32"] for e in errs.values()), errs
+
+
+def test_binding_rejects_bad_tensors():
+    """The Python binding checks every tensor before the C call (dtype, device, contiguity and the
+    exact shape the kernels index): a wrong tensor raises ValueError instead of letting the
+    kernels read or write past an allocation."""
+    shape = SHAPES[0]
+    layer = _layer(shape, "bf16")
+    x = torch.zeros(layer.x_shape, device=DEV)
+    w = torch.zeros(layer.w_shape, device=DEV)
+    b = torch.zeros(layer.geom.Co, device=DEV)
+    y = torch.zeros(layer.y_shape, device=DEV)
+    bad = [
+        (x.half(), w, b, y),                                   # dtype
+        (x.cpu(), w, b, y),                                    # device
+        (x.transpose(2, 3), w, b, y),                          # not contiguous
+        (x, w, b, torch.zeros(layer.y_shape[0], layer.y_shape[1] + 1, *layer.y_shape[2:],
+                              device=DEV)),                    # shape
+        (x, w[:, :1].contiguous(), b, y),                      # weight shape
+        (x, w, torch.zeros(layer.geom.Co + 1, device=DEV), y),  # bias shape
+    ]
+    for args in bad:
+        with pytest.raises(ValueError):
+            layer.fwd(*args)
+    layer.fwd(x, w, None, y)   # bias is nullable
+    with pytest.raises(ValueError):
+        layer.bwd_filter(x, y, torch.zeros(1, device=DEV))

@@ -1,6 +1,9 @@
 """Diagnostic: per-CTA cycle split of the igemm issue warps (GLP_DEBUG_CLK): MMA-warp loop
 total, its waits on `full` (data not ready) and `tempty` (epilogue behind), producer waits on
-`empty` (ring full).  Usage: python tools/clk_probe.py layer:pass ..."""
+`empty` (ring full).  Usage: python tools/clk_probe.py layer:pass ...
+Needs the diagnostic library (the product libglp.so has no such hooks):
+    python -m paper_conf_icpp_futhys18_b200._build --diag
+    GLP_LIB=paper_conf_icpp_futhys18_b200/libglp_diag.so python tools/clk_probe.py ..."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch

@@ -1,5 +1,8 @@
 """Diagnostic: time one GEMM stage with A loads / B loads / MMAs selectively skipped
-(GLP_DEBUG_SKIP bits 0/1/2; results are garbage in the skipped modes)."""
+(GLP_DEBUG_SKIP bits 0/1/2; results are garbage in the skipped modes).
+Needs the diagnostic library (the product libglp.so has no such hooks):
+    python -m paper_conf_icpp_futhys18_b200._build --diag
+    GLP_LIB=paper_conf_icpp_futhys18_b200/libglp_diag.so python tools/stage_probe.py ..."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch

@@ -91,6 +91,11 @@ typedef struct {
                             and backward-data stages have run; the backward-data stage packs it) */
   int dgrad_halo;        /* 1: backward-data by the shared-halo kernel (unit stride: a 4-D TMA halo
                             of the packed dy per 64-channel block, tap operands by row shift)     */
+  /* The analyzer's inputs for samples_in_flight, S = glp_analyze_samples_in_flight(s_slot_rows,
+   * s_rows_per_sample, N): the forward kernel's resident GEMM rows (#SM x CTAs/SM of the kernel
+   * glp_plan_kernel_attr(0) describes x 128) and the rows one sample occupies (H_o*W_o, or the
+   * padded grid of the halo forward, x the N tiles). */
+  long long s_slot_rows, s_rows_per_sample;
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */
@@ -314,7 +319,8 @@ glp_status_t glp_analyze_samples_in_flight(int slots, int tiles_per_sample, int 
  * term (R17).  Output floor(min(...)). */
 glp_status_t glp_analyze_eq7(const glp_device_limits_t *lim, const glp_kernel_attr_t *k,
                              int blocks, double t_kernel, double t_launch, int *bound);
-/* Attributes of the shipped kernels for a plan (for the occupancy-API cross-check). which:
+/* Attributes of the kernel the plan launches for a pass (the halo kernel where the plan chose
+ * one; the occupancy-API cross-check and the samples-in-flight inputs). which:
  * 0 = forward, 1 = backward-data, 2 = backward-filter. */
 glp_status_t glp_plan_kernel_attr(glp_plan_t plan, int which, glp_kernel_attr_t *attr,
                                   int *ctas_per_sm_model, int *ctas_per_sm_runtime);

@@ -10,9 +10,10 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 ``paper_conf_icpp_futhys18_b200`` and does not import it.
 
 Parity status per function (see DESIGN.md §Oracle pins):
-  conv_fwd / conv_bwd_data / conv_bwd_filter / im2col  -- pinned (hand cases, torch fp64,
+  conv_fwd / conv_bwd_data / conv_bwd_filter / conv_db / im2col -- pinned (hand cases, torch fp64,
       adjoint identity, finite differences, 1x1 = matmul, batch-sum, floor truncation,
-      im2col+GEMM == direct conv, thread-count invariance)
+      im2col+GEMM == direct conv, thread-count invariance; conv_db == the bwd_filter db bitwise
+      and numpy's sum; absmode == the plain mode bitwise on non-negative operands)
   round_tf32_rna / round_bf16_rne / split_3xtf32          -- pinned (bit patterns, error bound)
   analyzer.*                                              -- pinned (paper worked example P173,
       brute-force MILP enumeration vs closed form)
@@ -50,6 +51,7 @@ def lib():
         L.oracle_conv_bwd_data.argtypes = [i] * 11 + [p, p, p, i]
         L.oracle_conv_bwd_filter.argtypes = [i] * 11 + [p, p, p, p, i]
         L.oracle_im2col.argtypes = [i] * 9 + [p, p]
+        L.oracle_conv_db.argtypes = [i] * 4 + [p, p]
         L.oracle_conv_bwd_filter_at.argtypes = [i] * 11 + [p, p, i, i, i, i]
         L.oracle_conv_bwd_filter_at.restype = ctypes.c_double
         L.oracle_set_threads.argtypes = [i]
@@ -116,6 +118,16 @@ def conv_bwd_filter(x, dy, w_shape, stride=1, pad=0, with_bias=True, absmode=Fal
     db = np.empty((w_shape[0],), np.float64) if with_bias else None
     lib().oracle_conv_bwd_filter(*g, _ptr(x), _ptr(dy), _ptr(dw), _ptr(db), int(absmode))
     return dw, db
+
+
+def conv_db(dy):
+    """P129 bias gradient alone: db[co] = sum_{n,ho,wo} dy[n,co,ho,wo] (fp64), the same loops as
+    conv_bwd_filter's db."""
+    dy = _f32(dy)
+    N, Co, Ho, Wo = dy.shape
+    db = np.empty((Co,), np.float64)
+    lib().oracle_conv_db(N, Co, Ho, Wo, _ptr(dy), _ptr(db))
+    return db
 
 
 def conv_bwd_filter_at(x, dy, w_shape, stride, pad, idx):

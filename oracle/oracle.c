@@ -167,6 +167,18 @@ void oracle_conv_bwd_filter(int N, int C, int H, int W, int Co, int Kh, int Kw, 
   }
 }
 
+/* Bias gradient alone (P129): db[co] = sum_{n,ho,wo} dy[n,co,ho,wo], the same loops as the db
+ * part of oracle_conv_bwd_filter (for full-size checks where the whole dW would be too slow). */
+void oracle_conv_db(int N, int Co, int Ho, int Wo, const float *dy, double *db) {
+#pragma omp parallel for schedule(static)
+  for (int co = 0; co < Co; ++co) {
+    double acc = 0.0;
+    for (int n = 0; n < N; ++n)
+      for (int p = 0; p < Ho * Wo; ++p) acc += (double)dy[((size_t)n * Co + co) * Ho * Wo + p];
+    db[co] = acc;
+  }
+}
+
 /* Caffe im2col of ONE sample (P173 "im2col"): col[(ci*Kh+kh)*Kw+kw][ho*Wo+wo]. Pure data
  * movement, so the output keeps the input's fp32 values exactly. */
 void oracle_im2col(int C, int H, int W, int Kh, int Kw, int Sh, int Sw, int Ph, int Pw,

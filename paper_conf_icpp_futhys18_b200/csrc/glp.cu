@@ -111,6 +111,12 @@ struct PassPlan {
   int chunk_kb = 0;                 // 3xTF32: k-blocks per TMEM accumulation chunk
 };
 
+// Analyzer record of one shipped kernel (Table 2 "profiling input", P194-200): its attributes,
+// the closed-form CTAs/SM (Eqs 4-5 re-derived + the sm_100a limits) and the CUDA occupancy API's.
+struct KAttr {
+  int threads = 0, regs = 0, smem = 0, tmem = 0, model = 0, rt = 0;
+};
+
 using TmapEncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
                                   const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
                                   const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
@@ -338,6 +344,9 @@ struct glp_plan_s {
   int halo = 0;
   HwgradParams hw{};
   int hw_grid = 0, hw_smem = 0, hw_regs = 0;
+  KAttr hw_attr, hd_attr, hf_attr;   // analyzer records of the halo kernels the plan uses
+  glp_device_limits_t lim{};         // the device's per-SM limits (analyzer input)
+  long long s_slot_rows = 0, s_rows_per_sample = 0;   // the analyzer's S inputs (forward kernel)
   // halo forward (hfwd.cuh) for the same space-to-depth layers: x' staged once per tile for all
   // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
   int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
@@ -383,6 +392,26 @@ struct glp_plan_s {
 };
 
 namespace {
+
+// The analyzer's view of a kernel (P167: "kernel analyzer"): attributes from the runtime, CTAs per
+// SM from the closed form over every per-SM limit, cross-checked against the occupancy API.  TMEM:
+// the runtime admits one tcgen05 (TMEM-allocating) CTA per SM whatever its column count (R16), so
+// such a kernel is charged the whole per-SM TMEM.
+glp_status_t analyze_kernel(const glp_plan_s &P, const void *fn, int threads, int dyn_smem,
+                            int tmem_cols, KAttr &k) {
+  cudaFuncAttributes fa;
+  GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
+  k.threads = threads;
+  k.regs = fa.numRegs;
+  k.smem = dyn_smem + (int)fa.sharedSizeBytes;
+  k.tmem = tmem_cols;
+  glp_kernel_attr_t ka{threads, fa.numRegs, k.smem,
+                       (tmem_cols > 0 && P.lim.tmem_cols_per_sm > 0) ? P.lim.tmem_cols_per_sm : tmem_cols};
+  k.model = ctas_per_sm_closed_form(P.lim, ka);
+  GLP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k.rt, fn, threads, dyn_smem));
+  if (k.model < 1) return fail(GLP_ERR_INTERNAL, "kernel does not fit on an SM");
+  return GLP_OK;
+}
 
 // Halo filter gradient (hwgrad.cuh) for space-to-depth layers whose x' rows are one 64-channel
 // bf16 atom and whose tap pairs' accumulators fit TMEM.  Split count: shape-only (a fixed
@@ -465,9 +494,11 @@ glp_status_t plan_halo(glp_plan_s &P) {
                  : ncg == 1 ? reinterpret_cast<const void *>(hwgrad_kernel<1>)
                             : reinterpret_cast<const void *>(hwgrad_kernel<0>);
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
-  cudaFuncAttributes fa;
-  GLP_CUDA(cudaFuncGetAttributes(&fa, fn));
-  P.hw_regs = fa.numRegs;
+  glp_status_t s = analyze_kernel(P, fn, hw_threads(ncg), P.hw_smem, h.tmem_cols, P.hw_attr);
+  if (s) return s;
+  P.hw_regs = P.hw_attr.regs;
+  // grid = the shape-only split count (148 ranges, never the queried device: the reduction order
+  // is fixed); the analyzer's slots (#SM x CTAs/SM) bound how many run at once
   P.halo = 1;
   P.halo_fdy = ncg;
   return GLP_OK;
@@ -534,12 +565,16 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   if (h.b_stages < 3) return GLP_OK;
   P.hd_smem = 1024 + h.a_stages * h.a_bytes + h.b_stages * h.b_bytes +
               8 * (2 * h.a_stages + 2 * h.b_stages + 4) + 16;
-  long long pairs = std::min<long long>(h.units, P.sm_count / 2);
+  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hdgrad_kernel),
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  glp_status_t s = analyze_kernel(P, reinterpret_cast<const void *>(hdgrad_kernel), HD_THREADS,
+                                  P.hd_smem, h.tmem_cols, P.hd_attr);
+  if (s) return s;
+  // persistent grid: the analyzer's resident CTA-pair slots (#SM x CTAs/SM / 2), at most the units
+  long long pairs = std::min<long long>(h.units, (long long)P.sm_count * P.hd_attr.model / 2);
   if (P.s_override > 0)
     pairs = std::max(1LL, std::min(pairs, cdiv((long long)P.s_override * tiles_img, 2)));
   P.hd_grid = (int)(2 * pairs);
-  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hdgrad_kernel),
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   P.hdg = 1;
   return GLP_OK;
 }
@@ -585,15 +620,17 @@ glp_status_t plan_hfwd(glp_plan_s &P) {
   h.ho = P.d.Ho;
   h.wo = P.d.Wo;
   P.hf_smem = fixed + 8 * (2 * h.stages + 6) + h.stages * h.a_bytes;
-  long long pairs = std::min<long long>(h.units, P.sm_count / 2);
+  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hfwd_kernel),
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+  glp_status_t s = analyze_kernel(P, reinterpret_cast<const void *>(hfwd_kernel), HF_THREADS,
+                                  P.hf_smem, h.tmem_cols, P.hf_attr);
+  if (s) return s;
+  P.hf_regs = P.hf_attr.regs;
+  // persistent grid: the analyzer's resident CTA-pair slots, at most the units
+  long long pairs = std::min<long long>(h.units, (long long)P.sm_count * P.hf_attr.model / 2);
   if (P.s_override > 0)   // test override: only the tiles of S samples in flight at once
     pairs = std::max(1LL, std::min(pairs, cdiv((long long)P.s_override * x.H * x.W, 256)));
   P.hf_grid = (int)(2 * pairs);
-  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hfwd_kernel),
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
-  cudaFuncAttributes fa;
-  GLP_CUDA(cudaFuncGetAttributes(&fa, reinterpret_cast<const void *>(hfwd_kernel)));
-  P.hf_regs = fa.numRegs;
   P.hfwd = 1;
   return GLP_OK;
 }
@@ -1738,6 +1775,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
   L.max_blocks_per_sm = prop.maxBlocksPerMultiProcessor;
   L.smem_reserved_per_cta = (int)prop.reservedSharedMemPerBlock;
 
+  P->lim = L;
   glp_status_t s = GLP_OK;
   if (d->nbr > 1 && !P->simt) {
     // a branch's packed channels start on a 16-byte chunk of the pitch (8 bf16 / 4 tf32)
@@ -1799,9 +1837,25 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
     P->ws_dgrad = P->off_wtpk + P->sz_wtpk;
     P->ws_wgrad = P->off_dbpart + P->sz_dbpart;
     P->ws_bwd = P->ws_wgrad;
-    const long long slots = (long long)P->sm_count * P->fwd.ctas_per_sm;
-    const long long per = (long long)d->Ho * d->Wo * P->fwd.n_tiles;  // pixels*n_tiles per sample
-    P->S = (int)std::max(1LL, std::min<long long>(d->N, slots * 128 / std::max(1LL, per)));
+    // Samples in flight (the paper's C_out, Eq. 9 re-derived, R18) through the analyzer: the
+    // forward kernel's resident rows (#SM x CTAs/SM x 128 GEMM rows) over the rows a sample
+    // occupies (H_o*W_o pixels -- the padded x' grid for the halo forward -- times the N tiles)
+    const bool hf = P->hfwd != 0;
+    const int beta = hf ? P->hf_attr.model : P->fwd.ctas_per_sm;
+    P->s_slot_rows = (long long)P->sm_count * beta * 128;
+    P->s_rows_per_sample = hf ? (long long)P->dxg.H * P->dxg.W
+                              : (long long)d->Ho * d->Wo * P->fwd.n_tiles;
+    if (P->s_slot_rows >= (1LL << 31) || P->s_rows_per_sample >= (1LL << 31)) {
+      delete P;
+      if (cur != device) cudaSetDevice(cur);
+      return fail(GLP_ERR_NOT_SUPPORTED, "analyzer inputs exceed 32 bits");
+    }
+    if ((s = glp_analyze_samples_in_flight((int)P->s_slot_rows, (int)P->s_rows_per_sample, d->N,
+                                           &P->S))) {
+      delete P;
+      if (cur != device) cudaSetDevice(cur);
+      return s;
+    }
     if (S > 0) P->S = std::min(S, d->N);
   } else {
     const long long npix = (long long)d->N * d->Ho * d->Wo;
@@ -1854,6 +1908,8 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->fwd_halo = P->hfwd;
   I->wgrad_fused_dy = P->halo_fdy ? 1 : 0;
   I->dgrad_halo = P->hdg;
+  I->s_slot_rows = P->s_slot_rows;
+  I->s_rows_per_sample = P->s_rows_per_sample;
   if (P->hdg) {
     I->grid_bwd_data = P->hd_grid;
     I->tile_n_bwd_data = P->hd.bn;
@@ -1872,6 +1928,16 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
 glp_status_t glp_plan_kernel_attr(glp_plan_t P, int which, glp_kernel_attr_t *a, int *model, int *rt) {
   if (!P || !a || !model || !rt || which < 0 || which > 2) return fail(GLP_ERR_INVALID_VALUE, "bad argument");
   if (P->simt) return fail(GLP_ERR_NOT_SUPPORTED, "SIMT path has no persistent kernel");
+  // the kernel the plan actually launches for the pass: a halo kernel where the plan chose one
+  const KAttr *h = (which == 0 && P->hfwd) ? &P->hf_attr
+                 : (which == 1 && P->hdg) ? &P->hd_attr
+                 : (which == 2 && P->halo) ? &P->hw_attr : nullptr;
+  if (h) {
+    *a = glp_kernel_attr_t{h->threads, h->regs, h->smem, h->tmem};
+    *model = h->model;
+    *rt = h->rt;
+    return GLP_OK;
+  }
   const PassPlan &pp = which == 0 ? P->fwd : which == 1 ? P->dgrad : P->wgrad;
   *a = glp_kernel_attr_t{pp.threads, pp.regs, pp.smem, pp.tmem_cols};
   *model = pp.ctas_per_sm;

@@ -4,11 +4,17 @@ after the timed steps), checked against the oracle on sampled outputs it compute
 (oracle.conv_fwd_at / conv_bwd_data_at / conv_bwd_filter_at) and on db in full.
 
 Bars: integer data (`--exact-data`) -> every sampled element bit-exact; float
-data -> |g - r| <= 2e-2 * max_sampled |r| against the fp64 oracle on the unrounded inputs (the
-north_star bar, normwise over the sample) and |g - r_emu| <= 1e-5 * sum|a||b| against the oracle
-on the operands rounded as the pack step defines (the condition-aware bound of fp32 accumulation
-over exactly rounded products).  Samples always include the first and the last element (the
-ragged last tile) of every tensor.
+data -> |g - r| <= bar * max_sampled |r| against the fp64 oracle on the unrounded inputs (the
+north_star bar, normwise over the sample: 2e-2 for TF32/BF16, 1e-5 for GLP_MATH_FP32 = 3xTF32)
+and |g - r_emu| <= 1e-5 * sum|a||b| against the oracle of the products the MMAs form (operands
+rounded as the pack step defines; 3xTF32: hi*hi + hi*lo + lo*hi of oracle.split_3xtf32) -- the
+condition-aware bound of fp32 accumulation over exactly formed products.  Samples always include
+the first and the last element (the ragged last tile) of every tensor.  db is compared in full
+with oracle.conv_db.
+
+test_fullsize_whole_tensor_exact: CaffeNet conv1-5 at batch 256 (BASELINE.json configs[3]) with
+integer data, every output tensor compared WHOLE and bit for bit with the oracle, in every tensor
+math mode (one oracle pass serves the three modes: the integer draws are the same).
 """
 import json
 import os
@@ -23,6 +29,7 @@ import oracle
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 EMU = {"tf32": oracle.round_tf32_rna, "bf16": oracle.round_bf16_rne}
+BAR = {"bf16": 2e-2, "tf32": 2e-2, "fp32": 1e-5}
 NS = 40   # sampled elements per tensor
 
 
@@ -48,13 +55,36 @@ def _samples(shape, rng):
     return idx
 
 
+def _emu(fn, a, b, math, *rest, **kw):
+    """Oracle value of the products the MMAs form from operands a, b (one element): the rounded
+    operands (TF32 / BF16), or for 3xTF32 hi*hi + hi*lo + lo*hi of the split planes (the oracle
+    is linear in each operand).  `a`, `b` are (array, rounded) pairs prepared by _prep."""
+    if math != "fp32":
+        return fn(a[1], b[1], *rest, **kw)
+    (ah, al), (bh, bl) = a[2], b[2]
+    return fn(ah, bh, *rest, **kw) + fn(ah, bl, *rest, **kw) + fn(al, bh, *rest, **kw)
+
+
+def _prep(v, math):
+    """(fp32 array, rounded operand, (hi, lo) split) of one operand."""
+    if math == "fp32":
+        hi, lo = oracle.split_3xtf32(v)
+        return (v, hi, (hi, lo))
+    return (v, EMU[math](v), None)
+
+
+def _sl(p, *idx):
+    """Slice every member of a _prep triple."""
+    return (p[0][idx], p[1][idx], None if p[2] is None else (p[2][0][idx], p[2][1][idx]))
+
+
 def _check(kind, got, ref, emu, scale, exact, math, what):
     got, ref = np.asarray(got, np.float64), np.asarray(ref, np.float64)
     if exact:
         np.testing.assert_array_equal(got, ref, err_msg=what)
         return
-    bar = 2e-2 * max(np.abs(ref).max(), 1e-30)
-    assert np.abs(got - ref).max() <= bar, (what, np.abs(got - ref).max() / bar * 2e-2)
+    bar = BAR[math] * max(np.abs(ref).max(), 1e-30)
+    assert np.abs(got - ref).max() <= bar, (what, np.abs(got - ref).max() / bar * BAR[math])
     emu, scale = np.asarray(emu, np.float64), np.asarray(scale, np.float64)
     assert np.all(np.abs(got - emu) <= 1e-5 * scale + 1e-30), (
         what, float((np.abs(got - emu) / np.maximum(scale, 1e-30)).max()))
@@ -65,8 +95,7 @@ def _check_unit(tmp, i, u, math, exact, rng):
     x = np.asarray(_load(tmp, i, "x"))
     grp = u["kind"] == "group"
     nb = len(u["Co"])
-    r = EMU[math]
-    xe = r(x)
+    xp = _prep(x, math)
     dx_terms = []
     for b in range(nb):
         sfx = str(b) if grp else ""
@@ -76,7 +105,7 @@ def _check_unit(tmp, i, u, math, exact, rng):
         y = _load(tmp, i, "y" + sfx)
         dw = _load(tmp, i, "dw" + sfx)
         db = _load(tmp, i, "db" + sfx)
-        we, dye = r(w), r(dy)
+        wp, dyp = _prep(w, math), _prep(dy, math)
         Cg, Cog = u["C"] // G, u["Co"][b] // G
         name = f"{u['names'][b]}"
 
@@ -95,7 +124,8 @@ def _check_unit(tmp, i, u, math, exact, rng):
             bg = bias[g * Cog:(g + 1) * Cog]
             g_.append(y[n, co, ho, wo])
             ref.append(oracle.conv_fwd_at(xi, wg, bg, S, P, j))
-            emu.append(oracle.conv_fwd_at(xe[n:n + 1, cs], we[g * Cog:(g + 1) * Cog], bg, S, P, j))
+            emu.append(_emu(oracle.conv_fwd_at, _sl(xp, slice(n, n + 1), cs),
+                            _sl(wp, slice(g * Cog, (g + 1) * Cog)), math, None, S, P, j) + float(bg[j[1]]))
             sc.append(oracle.conv_fwd_at(xi, wg, None, S, P, j, absmode=True) + abs(float(bg[j[1]])))
         _check("y", g_, ref, emu, sc, exact, math, f"{name} y")
         # filter gradient
@@ -107,17 +137,18 @@ def _check_unit(tmp, i, u, math, exact, rng):
             wsh = (Cog, Cg, w.shape[2], w.shape[3])
             g_.append(dw[co, ci, kh, kw])
             ref.append(oracle.conv_bwd_filter_at(x[:, cs], dy[:, os_], wsh, S, P, j))
-            emu.append(oracle.conv_bwd_filter_at(xe[:, cs], dye[:, os_], wsh, S, P, j))
+            emu.append(_emu(oracle.conv_bwd_filter_at, _sl(xp, slice(None), cs),
+                            _sl(dyp, slice(None), os_), math, wsh, S, P, j))
             sc.append(oracle.conv_bwd_filter_at_abs(x[:, cs], dy[:, os_], wsh, S, P, j))
         _check("dw", g_, ref, emu, sc, exact, math, f"{name} dW")
-        # bias gradient in full (plain sum over n, ho, wo)
-        ref = dy.astype(np.float64).sum(axis=(0, 2, 3))
+        # bias gradient in full (the oracle's plain sum over n, ho, wo)
+        ref = oracle.conv_db(dy)
         if exact:
             np.testing.assert_array_equal(np.asarray(db, np.float64), ref, err_msg=f"{name} db")
         else:
             scale = np.abs(dy.astype(np.float64)).sum(axis=(0, 2, 3))
             assert np.all(np.abs(np.asarray(db, np.float64) - ref) <= 1e-5 * scale + 1e-30), name
-        dx_terms.append((w, we, dy, dye, Cg, Cog))
+        dx_terms.append((w, wp, dy, dyp, Cg, Cog))
     if "dx" not in u["arrays"]:
         assert u["data_fed"]   # the data-fed first layer has no backward-data pass (R9)
         return
@@ -126,13 +157,14 @@ def _check_unit(tmp, i, u, math, exact, rng):
     g_, ref, emu, sc = [], [], [], []
     for n, ci, h, ww in idx:
         rr = ee = ss = 0.0
-        for w, we, dy, dye, Cg, Cog in dx_terms:
+        for w, wp, dy, dyp, Cg, Cog in dx_terms:
             g = ci // Cg
             os_ = slice(g * Cog, (g + 1) * Cog)
             j = (0, ci - g * Cg, h, ww)
             xs = (1, Cg) + tuple(dx.shape[2:])
             rr += oracle.conv_bwd_data_at(dy[n:n + 1, os_], w[os_], xs, S, P, j)
-            ee += oracle.conv_bwd_data_at(dye[n:n + 1, os_], we[os_], xs, S, P, j)
+            ee += _emu(oracle.conv_bwd_data_at, _sl(dyp, slice(n, n + 1), os_), _sl(wp, os_), math,
+                       xs, S, P, j)
             ss += oracle.conv_bwd_data_at(dy[n:n + 1, os_], w[os_], xs, S, P, j, absmode=True)
         g_.append(dx[n, ci, h, ww])
         ref.append(rr)
@@ -142,8 +174,10 @@ def _check_unit(tmp, i, u, math, exact, rng):
 
 
 CASES = [(1, "bf16", False), (2, "bf16", False), (3, "bf16", False), (4, "bf16", False),
-         (4, "bf16", True), (4, "tf32", False), (4, "tf32", True), (5, "bf16", False),
-         (5, "bf16", True), (6, "bf16", False), (7, "bf16", True)]
+         (4, "tf32", False), (5, "bf16", False), (5, "bf16", True), (6, "bf16", False),
+         (7, "bf16", True),
+         (1, "fp32", False), (2, "fp32", False), (3, "fp32", False), (4, "fp32", False),
+         (5, "fp32", False), (6, "fp32", False), (7, "fp32", True), (7, "fp32", False)]
 
 
 @pytest.mark.parametrize("case", CASES, ids=lambda c: f"cfg{c[0]}-{c[1]}-{'exact' if c[2] else 'float'}")
@@ -154,3 +188,28 @@ def test_fullsize_sampled_parity(case, tmp_path):
     rng = np.random.Generator(np.random.PCG64(1000 + workload))
     for i, u in enumerate(meta["units"]):
         _check_unit(tmp_path, i, u, math, exact, rng)
+
+
+def test_fullsize_whole_tensor_exact(tmp_path):
+    """CaffeNet conv1-5, batch 256, integer data: bench.py's own plans and graph-replayed step in
+    bf16, tf32 and fp32 (3xTF32); every output tensor (y, dx, dW, db of every layer) equals the
+    whole-tensor oracle bit for bit in every mode."""
+    metas = {m: _bench_dump(tmp_path / m, 4, m, True) for m in ("bf16", "tf32", "fp32")}
+    units = metas["bf16"]["units"]
+    for i, u in enumerate(units):
+        S, P = u["S"], u["P"]
+        x = np.asarray(_load(tmp_path / "bf16", i, "x"))
+        w = np.asarray(_load(tmp_path / "bf16", i, "w"))
+        b = np.asarray(_load(tmp_path / "bf16", i, "b"))
+        dy = np.asarray(_load(tmp_path / "bf16", i, "dy"))
+        for m in ("tf32", "fp32"):   # the same integer draws in every mode
+            for k, v in (("x", x), ("w", w), ("dy", dy)):
+                np.testing.assert_array_equal(np.asarray(_load(tmp_path / m, i, k)), v)
+        ref = {"y": oracle.conv_fwd(x, w, b, S, P)}
+        ref["dw"], ref["db"] = oracle.conv_bwd_filter(x, dy, w.shape, S, P)
+        if not u["data_fed"]:
+            ref["dx"] = oracle.conv_bwd_data(dy, w, x.shape, S, P)
+        for m in ("bf16", "tf32", "fp32"):
+            for k, r in ref.items():
+                np.testing.assert_array_equal(np.asarray(_load(tmp_path / m, i, k)),
+                                              r.astype(np.float32), err_msg=f"{m} {u['names'][0]} {k}")

@@ -54,7 +54,7 @@ def _oracle(d, S, P, x=None, w=None, dy=None):
     y = oracle.conv_fwd(x, w, d["b"], S, P)
     dx = oracle.conv_bwd_data(dy, w, x.shape, S, P)
     dw, _ = oracle.conv_bwd_filter(x, dy, w.shape, S, P)
-    db = d["dy"].astype(np.float64).sum(axis=(0, 2, 3))
+    db = oracle.conv_db(d["dy"])   # db is summed from the unrounded fp32 dy in every mode
     return {"y": y, "dx": dx, "dw": dw, "db": db}
 
 
@@ -191,8 +191,10 @@ def test_combined_bwd_equals_separate(math):
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 def test_analyzer_matches_occupancy_api(math):
-    """The re-derived analyzer's CTAs/SM for every shipped kernel equals the CUDA occupancy API."""
-    for shape in SHAPES:
+    """The re-derived analyzer's CTAs/SM for every shipped kernel (the halo kernels included, where
+    a plan picks them) equals the CUDA occupancy API."""
+    for shape in SHAPES + [("caffenet_conv1_full", 2, 3, 227, 227, 96, 11, 4, 0),
+                           ("caffenet_conv2_b2", 2, 96, 27, 27, 256, 5, 1, 2)]:
         layer = _layer(shape, math)
         for which in range(3):
             a = layer.kernel_attr(which)
@@ -746,3 +748,42 @@ def test_binding_rejects_bad_tensors():
     layer.fwd(x, w, None, y)   # bias is nullable
     with pytest.raises(ValueError):
         layer.bwd_filter(x, y, torch.zeros(1, device=DEV))
+
+
+TABLE5 = [  # every Table 5 layer (P334-355) at its BASELINE.json batch
+    ("lenet_conv1", 64, 1, 28, 28, 20, 5, 1, 0), ("lenet_conv2", 64, 20, 12, 12, 50, 5, 1, 0),
+    ("cifar10_conv1", 100, 3, 32, 32, 32, 5, 1, 2), ("cifar10_conv2", 100, 32, 16, 16, 32, 5, 1, 2),
+    ("cifar10_conv3", 100, 32, 8, 8, 64, 5, 1, 2),
+    ("caffenet_conv1", 256, 3, 227, 227, 96, 11, 4, 0), ("caffenet_conv2", 256, 96, 27, 27, 256, 5, 1, 2),
+    ("caffenet_conv3", 256, 256, 13, 13, 384, 3, 1, 1), ("caffenet_conv4", 256, 384, 13, 13, 384, 3, 1, 1),
+    ("caffenet_conv5", 256, 384, 13, 13, 256, 3, 1, 1),
+    ("googlenet_conv_1", 128, 160, 7, 7, 320, 3, 1, 1), ("googlenet_conv_2", 128, 832, 7, 7, 32, 1, 1, 0),
+    ("googlenet_conv_3", 128, 832, 7, 7, 384, 1, 1, 0), ("googlenet_conv_4", 128, 192, 7, 7, 384, 3, 1, 1),
+    ("googlenet_conv_5", 128, 832, 7, 7, 192, 1, 1, 0), ("googlenet_conv_6", 128, 832, 7, 7, 48, 1, 1, 0),
+]
+
+
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+def test_samples_in_flight_through_analyzer(math):
+    """S (the paper's C_out, Eq. 9 re-derived, P254) of every Table 5 layer's plan equals the
+    oracle analyzer's enumeration on the attributes of the forward kernel the plan launches:
+    CTAs/SM by enumeration over every per-SM limit (TMEM charged whole, R16), resident rows =
+    148 x CTAs/SM x 128, rows per sample = H_o*W_o x N tiles (the padded x' grid for the halo
+    forward), S = largest s <= N with s * rows_per_sample <= resident rows (>= 1)."""
+    from oracle import analyzer as A
+    dev = A.B200()
+    for shape in TABLE5:
+        name, N, C, H, W, Co, K, St, P = shape
+        layer = _layer(shape, math)
+        info = layer.info
+        a = layer.kernel_attr(0)
+        beta = A.ctas_per_sm_enum(a["threads"], a["regs"], a["smem"], 512 if a["tmem_cols"] else 0, dev)
+        slot_rows = dev.n_sm * beta * 128
+        Ho = oracle.out_dim(H, K, St, P)
+        if info.fwd_halo:
+            Ks = -(-K // St)
+            rows = (Ho + Ks - 1) * (Ho + Ks - 1)
+        else:
+            rows = Ho * Ho * -(-Co // info.tile_n_fwd)
+        assert (info.s_slot_rows, info.s_rows_per_sample) == (slot_rows, rows), name
+        assert info.samples_in_flight == A.samples_in_flight_enum(slot_rows, rows, N), name

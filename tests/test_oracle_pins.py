@@ -203,6 +203,47 @@ def test_absmode_bounds():
     assert np.all(np.abs(y) <= ya + 1e-15)
 
 
+def test_absmode_exact_on_nonnegative_operands():
+    """Pin of the condition scale sum|a||b| (the full-size float bar): on non-negative operands
+    |a||b| = ab, so absmode must equal the plain mode BIT FOR BIT (same loops, same order), for
+    every pass and for the one-element forms; and it is invariant under operand sign flips."""
+    N, C, H, W, Co, K, S, P = 2, 4, 9, 11, 5, 3, 2, 1
+    Ho, Wo = oracle.out_dim(H, K, S, P), oracle.out_dim(W, K, S, P)
+    d = gen_custom(N, C, H, W, Co, K, K, 31, Ho=Ho, Wo=Wo)
+    x, w, dy = np.abs(d["x"]), np.abs(d["w"]), np.abs(d["dy"])
+    np.testing.assert_array_equal(oracle.conv_fwd(x, w, None, S, P, absmode=True),
+                                  oracle.conv_fwd(x, w, None, S, P))
+    np.testing.assert_array_equal(oracle.conv_bwd_data(dy, w, x.shape, S, P, absmode=True),
+                                  oracle.conv_bwd_data(dy, w, x.shape, S, P))
+    for a, b in zip(oracle.conv_bwd_filter(x, dy, w.shape, S, P, absmode=True),
+                    oracle.conv_bwd_filter(x, dy, w.shape, S, P)):
+        np.testing.assert_array_equal(a, b)
+    for idx in ((0, 0, 0, 0), (1, 4, Ho - 1, Wo - 1), (1, 2, 1, 3)):
+        assert oracle.conv_fwd_at(x, w, None, S, P, idx, absmode=True) == \
+            oracle.conv_fwd_at(x, w, None, S, P, idx)
+    for idx in ((0, 0, 0, 0), (1, 3, H - 1, W - 1), (0, 2, 4, 5)):
+        assert oracle.conv_bwd_data_at(dy, w, x.shape, S, P, idx, absmode=True) == \
+            oracle.conv_bwd_data_at(dy, w, x.shape, S, P, idx)
+    for idx in ((0, 0, 0, 0), (4, 3, 2, 2), (2, 1, 0, 2)):
+        # the numpy form sums in another order than the C loop: equal to rounding only
+        assert np.isclose(oracle.conv_bwd_filter_at_abs(x, dy, w.shape, S, P, idx),
+                          oracle.conv_bwd_filter_at(x, dy, w.shape, S, P, idx), rtol=1e-14, atol=0)
+    # signs do not matter to the condition scale
+    np.testing.assert_array_equal(oracle.conv_fwd(-d["x"], d["w"], None, S, P, absmode=True),
+                                  oracle.conv_fwd(x, w, None, S, P))
+
+
+def test_conv_db_definition():
+    """conv_db (the bias gradient alone, for full-size checks) equals the db of conv_bwd_filter
+    bitwise (same definition and loops) and numpy's fp64 sum over (n, ho, wo)."""
+    d = gen_custom(3, 4, 9, 9, 6, 3, 3, 32, Ho=9, Wo=9)
+    db = oracle.conv_db(d["dy"])
+    _, db2 = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, 1, 1)
+    np.testing.assert_array_equal(db, db2)
+    np.testing.assert_allclose(db, d["dy"].astype(np.float64).sum(axis=(0, 2, 3)), rtol=1e-13,
+                               atol=1e-15)
+
+
 # ---------------------------------------------------------------- rounding step ------------
 
 def _u(s):

@@ -717,6 +717,34 @@ def quick_mode(args, math, G, rank, dev):
     return out
 
 
+def weak_scaling(args, G, rank, dev):
+    """G > 1: the same step with the config batch on EVERY rank (weak scaling), reported beside the
+    strong-scaling headline; eager steps with the bucketed exchange, max over ranks."""
+    import argparse as _ap
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icpp_futhys18_b200.dist import FlatGrads
+    a = _ap.Namespace(**vars(args))
+    a.scaling = "weak"
+    layers = config(a.workload)
+    grads = FlatGrads([l.w_shape for l in layers], device=dev)
+    _, states, n_local = build_states(a, a.math, G, rank, dev, grads)
+    step = Step(a, states, grads, G, dev)
+    for _ in range(max(3, a.warmup)):
+        step()
+    torch.cuda.synchronize()
+    dist.barrier()
+    ms = time_steps(lambda: step(concurrent=not a.serial), a.steps, torch.cuda.current_stream())
+    tt = torch.tensor([ms], device=dev)
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    ms = float(tt.item())
+    out = {"value": round(n_local[0] * G / (ms / 1e3), 1), "ms_per_step": round(ms, 4),
+           "per_gpu_batch": n_local[0], "global_batch": n_local[0] * G}
+    del step, states
+    torch.cuda.empty_cache()
+    return out
+
+
 def run_glp(args, ws, rank, local):
     import torch
     import torch.distributed as dist
@@ -725,6 +753,9 @@ def run_glp(args, ws, rank, local):
     torch.cuda.set_device(dev)
     G = ws
     if G > 1:
+        # the NCCL communicator lines (ring/tree/NVLS choice over NVLink) go to stderr
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("nccl", device_id=dev)
     from paper_conf_icpp_futhys18_b200.dist import FlatGrads
     layers = config(args.workload)
@@ -836,6 +867,9 @@ def run_glp(args, ws, rank, local):
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "ms_per_step": round(ems, 3), "steps": ke}
 
+    weak = None
+    if G > 1 and args.scaling == "strong" and not args.no_extra_modes:
+        weak = weak_scaling(args, G, rank, dev)
     modes = None
     if G == 1 and not args.no_extra_modes:
         modes = {m: quick_mode(args, m, G, rank, dev) for m in ("bf16", "tf32") if m != args.math}
@@ -871,6 +905,7 @@ def run_glp(args, ws, rank, local):
         "roofline": roofline,
         "kernels": [{k: r[k] for k in ("layer", "pass", "avg_us", "tflops")} for r in kern],
         "modes": modes,
+        "weak_scaling": weak,
         "cpu_baseline": cpu,
         "clocks": clk,
         "e2e": e2e,

@@ -125,20 +125,6 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map
       : "memory");
 }
 
-// im2col-mode TMA over a 4-D NHWC tensor {C, W, H, N}: loads `pixelsPerColumn` pixels starting at
-// base pixel (w, h, n) of the encoded bounding box (traversal wraps rows and images), each pixel
-// read at (w + off_w, h + off_h) with `channelsPerPixel` channels from c; out of bounds -> zeros.
-__device__ __forceinline__ void tma_load_im2col_4d(uint32_t dst, const CUtensorMap *map,
-                                                   uint32_t bar, int c, int w, int h, int n,
-                                                   uint16_t off_w, uint16_t off_h) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(off_w),
-      "h"(off_h)
-      : "memory");
-}
-
 // ------------------------------------------------------------------ warp-converged issue ---
 // Single-lane async ops issued by a converged warp: `elect.sync` inside the instruction block
 // picks one lane, so the operands stay warp-uniform (uniform datapath) and the compiler does not
@@ -155,15 +141,6 @@ __device__ __forceinline__ void tma_load_2d_e(uint32_t dst, const CUtensorMap *m
                "@P_e cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
                " [%0], [%1, {%3, %4}], [%2];\n\t}" ::"r"(dst),
                "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
-               : "memory");
-}
-// 4-D tiled load (coordinates may be negative / past the end: out-of-bounds elements are zero)
-__device__ __forceinline__ void tma_load_4d_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
-                                              int c0, int c1, int c2, int c3) {
-  asm volatile(GLP_ELECT
-               "@P_e cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-               " [%0], [%1, {%3, %4, %5, %6}], [%2];\n\t}" ::"r"(dst),
-               "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
                : "memory");
 }
 __device__ __forceinline__ void tma_load_4d_cg2_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
@@ -201,21 +178,6 @@ __device__ __forceinline__ void tma_load_im2col_4d_cg2_e(uint32_t dst, const CUt
                "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n),
                "h"(off_w), "h"(off_h)
                : "memory");
-}
-// tcgen05.mma (kind selected by KIND: 0 f16, 1 tf32; CG = cta_group) by one elected lane.
-template <int KIND, int CG>
-__device__ __forceinline__ void mma_e(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
-                                      uint32_t idesc, uint32_t accumulate) {
-#define GLP_MMA_E(KINDS, CGS)                                                                  \
-  asm volatile(GLP_ELECT ".reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"                          \
-               "@P_e tcgen05.mma.cta_group::" CGS ".kind::" KINDS " [%0], %1, %2, %3, p;\n\t}" \
-               ::"r"(d_tmem), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)            \
-               : "memory")
-  if (KIND == 0 && CG == 1) GLP_MMA_E("f16", "1");
-  else if (KIND == 0) GLP_MMA_E("f16", "2");
-  else if (CG == 1) GLP_MMA_E("tf32", "1");
-  else GLP_MMA_E("tf32", "2");
-#undef GLP_MMA_E
 }
 // All NSTEP tcgen05.mma of one k-block in one instruction block (one elect, descriptors advanced
 // by STEP 16-byte units per MMA inside the block): the MMA-issuing warp's loop is latency-bound,
@@ -306,12 +268,6 @@ __device__ __forceinline__ void mma_commit_e(uint32_t bar) {
                  : "memory");
 }
 
-// ------------------------------------------------------------------ clusters (CTA pairs) ---
-__device__ __forceinline__ uint32_t cluster_ctarank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
                    : "memory");
@@ -332,30 +288,6 @@ __device__ __forceinline__ void mbar_arrive_relaxed(uint32_t bar) {
 __device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t cluster_bar) {
   asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_bar)
                : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_bar) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_bar)
-               : "memory");
-}
-// 2-SM TMA loads: data lands in the issuing CTA's smem, completion bytes are counted on the
-// mbarrier given by a shared::cluster address (the pair leader's).
-__device__ __forceinline__ void tma_load_2d_cg2(uint32_t dst, const CUtensorMap *map, uint32_t bar,
-                                                int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_im2col_4d_cg2(uint32_t dst, const CUtensorMap *map,
-                                                       uint32_t bar, int c, int w, int h, int n,
-                                                       uint16_t off_w, uint16_t off_h) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.im2col.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(off_w),
-      "h"(off_h)
-      : "memory");
 }
 
 // ------------------------------------------------------------------ tcgen05 --------------
@@ -380,34 +312,6 @@ __device__ __forceinline__ void tmem_dealloc_cg(uint32_t taddr, uint32_t ncols) 
   else
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
 }
-// 2-SM MMA: D (M = 256 across the pair, 128 rows per SM) (+)= A (128 rows per SM) * B (N/2
-// columns per SM); issued by the pair leader only.
-__device__ __forceinline__ void mma_f16_cg2(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
-                                            uint32_t idesc, uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-__device__ __forceinline__ void mma_tf32_cg2(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
-                                             uint32_t idesc, uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-// Arrive on the mbarrier at the same smem offset in every CTA of `mask` when this thread's
-// previously issued tcgen05 ops (both SMs of the pair) have completed.
-__device__ __forceinline__ void mma_commit_cg2_mc(uint32_t bar, uint16_t mask) {
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
-      " [%0], %1;" ::"r"(bar), "h"(mask)
-      : "memory");
-}
 __device__ __forceinline__ void tmem_alloc(uint32_t dst_smem, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(dst_smem),
                "r"(ncols)
@@ -429,31 +333,6 @@ __device__ __forceinline__ void tc_fence_before() {
 }
 __device__ __forceinline__ void tc_fence_after() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-}
-// D[tmem] (+)= A[smem] * B[smem]^T, one CTA, kind::f16 (bf16 operands here) / kind::tf32.
-__device__ __forceinline__ void mma_f16(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
-                                        uint32_t idesc, uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-__device__ __forceinline__ void mma_tf32(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
-                                         uint32_t idesc, uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-// Arrive on an mbarrier when every previously issued tcgen05 op of this thread has completed.
-__device__ __forceinline__ void mma_commit(uint32_t bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                   bar)
-               : "memory");
 }
 __device__ __forceinline__ void tmem_wait_ld() {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");

@@ -29,7 +29,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from glp_workloads import CONFIG_NAMES, LEVELS, SIBLINGS, config, gen_layer  # noqa: E402
+from glp_workloads import CONFIG_NAMES, LEVELS, SHARED, SIBLINGS, config, gen_layer  # noqa: E402
 
 METRIC = "conv fwd+bwd images/sec"
 # the arithmetic each --math mode computes in (fp32 = 3xTF32 on tcgen05: fp32-accurate)
@@ -234,10 +234,26 @@ class LayerState:
         self.flops = float(self.layer.with_batch(n_local).flops_per_pass())
         self.leaves = None
         self.idx = idx
+        # shared parameters (glp_workloads.SHARED): a sharer reads its owner's W and b and adds its
+        # filter gradient to the owner's (accumulate = 1) after the owner's own
+        self.owner = None
+        self.has_sharer = False
+        self.accumulate = False
+        self.shared_keys = set()
+
+    def share_params_of(self, owner):
+        self.owner = owner
+        owner.has_sharer = True
+        self.accumulate = True
+        for k in ("w", "b"):
+            self.t[k] = owner.t[k]
+            self.host[k] = owner.host[k]
+        self.shared_keys = {"w", "b"}
+        self.dw, self.db = owner.dw, owner.db
 
     def grad_idxs(self):
         """Slots of the flat dW||db buffer this unit writes (its all-reduce bucket)."""
-        return [self.idx]
+        return [self.owner.idx if self.owner is not None else self.idx]
 
     def use_leaves(self, leaf_grads, idx, math, dev):
         """Deterministic exchange: the filter gradient per batch leaf of this rank (one plan for
@@ -292,7 +308,7 @@ class LayerState:
 
     def reduce(self, st=None):
         if self.leaves is None:
-            self.conv.stage_reduce(self.dw, self.db, stream=st)
+            self.conv.stage_reduce(self.dw, self.db, accumulate=self.accumulate, stream=st)
 
     def host_inputs(self):
         return self.host, self.t
@@ -326,6 +342,8 @@ def set_exact_data(states):
         else:
             new = gen_layer(s.layer, exact=True, batch=s.n)
         for k, v in new.items():
+            if k in s.shared_keys:   # the owner's parameters (replaced with the owner's draws)
+                continue
             s.host[k] = torch.from_numpy(v)
             s.t[k].copy_(s.host[k])
 
@@ -345,7 +363,8 @@ def dump_units(states, path, workload, math):
              "names": [m.name for m in s.members] if grp else [l.name],
              "N": s.n, "C": l.C, "H": l.H, "W": l.W, "K": l.K, "S": l.S, "P": l.P,
              "groups": l.groups, "data_fed": l.data_fed,
-             "Co": [m.Co for m in s.members] if grp else [l.Co]}
+             "Co": [m.Co for m in s.members] if grp else [l.Co],
+             "shares": None if s.owner is None else s.owner.name}
         arrays = {k: v.cpu().numpy() for k, v in s.t.items()}
         if grp:
             for b in range(len(s.members)):
@@ -396,6 +415,7 @@ class GroupState:
         self.dbs = [grads.db(i) for i in idxs]
         self.flops = float(sum(m.with_batch(n_local).flops_per_pass() for m in members))
         self.idxs = list(idxs)
+        self.owner, self.has_sharer, self.accumulate, self.shared_keys = None, False, False, set()
 
     def grad_idxs(self):
         return self.idxs
@@ -523,6 +543,9 @@ def build_states(args, math, G, rank, dev, grads):
             done_groups.add(gi)
             idxs = [j for j, m in enumerate(layers) if m.name in groups[gi]]
             states.append(GroupState([layers[j] for j in idxs], nl, ng, math, dev, grads, idxs))
+    by_name = {s.name: s for s in states}
+    for sharer, owner in SHARED.get(args.workload, {}).items():
+        by_name[sharer].share_params_of(by_name[owner])
     return layers, states, n_local
 
 
@@ -535,6 +558,9 @@ def dag_levels(args, states):
     unit_level = [where[(s.members[0] if isinstance(s, GroupState) else s.layer).name]
                   for s in states]
     levels = [[i for i, u in enumerate(unit_level) if u == k] for k in range(len(lv))]
+    # within a level, parameter owners are issued before their sharers (the sharer's accumulate=1
+    # reduction waits for the owner's)
+    levels = [sorted(l, key=lambda i: states[i].owner is not None) for l in levels]
     return [l for l in levels if l]
 
 
@@ -561,8 +587,9 @@ class Step:
         self.works = []
 
     def _bucket(self, s, g):
-        """All-reduce this unit's gradient bucket(s) on stream g (after its reductions)."""
-        if not self.bucketed:
+        """All-reduce this unit's gradient bucket(s) on stream g (after its reductions); a parameter
+        owner with a sharer leaves its bucket to the sharer (issued after the accumulation)."""
+        if not self.bucketed or s.has_sharer:
             return
         import torch
         import torch.distributed as dist
@@ -625,7 +652,7 @@ class Step:
         side_w.wait_stream(stream)
         for g in gstreams:
             g.wait_stream(stream)
-        ew_f, ew_b = {}, {}
+        ew_f, ew_b, red_done = {}, {}, {}
         with torch.cuda.stream(side_w):
             for i, s in enumerate(states):
                 s.pack_w_fwd(side_w)
@@ -666,7 +693,11 @@ class Step:
                     g.wait_event(e_dy)
                     with torch.cuda.stream(g):
                         s.bwd_filter(g)
+                        if s.owner is not None:   # accumulate onto the owner's finished gradient
+                            g.wait_event(red_done[id(s.owner)])
                         s.reduce(g)
+                        red_done[id(s)] = torch.cuda.Event()
+                        red_done[id(s)].record(g)
                     if with_exchange:
                         self._bucket(s, g)
                     if s.dx is not None:
@@ -842,7 +873,8 @@ def run_glp(args, ws, rank, local):
     # x, dy, W, b), the step, and dW||db back to the host every step
     e2e = None
     if not args.no_e2e:
-        host_pinned = [{k: v.pin_memory() for k, v in s.host.items()} for s in states]
+        host_pinned = [{k: v.pin_memory() for k, v in s.host.items() if k not in s.shared_keys}
+                       for s in states]
         out_host = torch.empty(nparams, pin_memory=True)
         h2d = sum(v.numel() * 4 for hp in host_pinned for v in hp.values())
         d2h = nparams * 4

@@ -111,6 +111,54 @@ _TABLE: Dict[int, List[Layer]] = {
         _L("caffenet_conv5_g2", 256, 384, 13, 256, 3, 1, 1, 13, False, groups=2)],
 }
 
+
+# the Siamese network of Table 5 (P341-344) with its shared weights: the two
+# towers (conv1, conv2) and (conv1_p, conv2_p) read different images but conv1_p / conv2_p use
+# conv1's / conv2's parameters [ext: Caffe mnist_siamese, param names shared], so their filter
+# gradients accumulate into one diff (Caffe beta = 1; glp_conv_bwd_filter accumulate = 1).  The
+# sharing towers are listed first so that, visited in reverse for the backward, every owner's
+# gradient overwrites before its sharer accumulates.
+_TABLE[8] = [_L("siamese_conv1_p", 64, 1, 28, 20, 5, 1, 0, 24, True),
+             _L("siamese_conv2_p", 64, 20, 12, 50, 5, 1, 0, 8, False),
+             _L("siamese_conv1", 64, 1, 28, 20, 5, 1, 0, 24, True),
+             _L("siamese_conv2", 64, 20, 12, 50, 5, 1, 0, 8, False)]
+
+# GoogLeNet's whole convolution stack at 224 x 224, batch 128 (BASELINE.json
+# configs[4] "synthetic 3x224x224"): conv1 7x7/2, conv2_reduce, conv2 and the nine inception
+# modules (3a-5b: 1x1, 3x3_reduce, 3x3, 5x5_reduce, 5x5, pool_proj) -- 57 convolutions, branch
+# widths from the GoogLeNet prototxt [ext: Szegedy et al. 2015, Table 1]; Table 5 lists 6 of them
+# (P350-355).  Each layer's input is synthesised at its own shape (pooling / concatenation are not
+# on the path).
+_INCEPTION = [  # name, H = W, C_in, [1x1, 3x3_reduce, 3x3, 5x5_reduce, 5x5, pool_proj]
+    ("3a", 28, 192, [64, 96, 128, 16, 32, 32]), ("3b", 28, 256, [128, 128, 192, 32, 96, 64]),
+    ("4a", 14, 480, [192, 96, 208, 16, 48, 64]), ("4b", 14, 512, [160, 112, 224, 24, 64, 64]),
+    ("4c", 14, 512, [128, 128, 256, 24, 64, 64]), ("4d", 14, 512, [112, 144, 288, 32, 64, 64]),
+    ("4e", 14, 528, [256, 160, 320, 32, 128, 128]), ("5a", 7, 832, [256, 160, 320, 32, 128, 128]),
+    ("5b", 7, 832, [384, 192, 384, 48, 128, 128])]
+
+
+def _googlenet_full(N=128):
+    ls = [_L("g_conv1_7x7_s2", N, 3, 224, 64, 7, 2, 3, 112, True),
+          _L("g_conv2_reduce", N, 64, 56, 64, 1, 1, 0, 56, False),
+          _L("g_conv2_3x3", N, 64, 56, 192, 3, 1, 1, 56, False)]
+    for m, hw, cin, (a, b, c, d, e, f) in _INCEPTION:
+        ls += [_L(f"g_{m}_1x1", N, cin, hw, a, 1, 1, 0, hw, False),
+               _L(f"g_{m}_3x3_reduce", N, cin, hw, b, 1, 1, 0, hw, False),
+               _L(f"g_{m}_5x5_reduce", N, cin, hw, d, 1, 1, 0, hw, False),
+               _L(f"g_{m}_pool_proj", N, cin, hw, f, 1, 1, 0, hw, False),
+               _L(f"g_{m}_3x3", N, b, hw, c, 3, 1, 1, hw, False),
+               _L(f"g_{m}_5x5", N, d, hw, e, 5, 1, 2, hw, False)]
+    return ls
+
+
+_TABLE[9] = _googlenet_full()
+
+# Shared-parameter layers: sharer -> owner (same W and b; the sharer's filter gradient is added
+# to the owner's with accumulate = 1 after the owner's own).
+SHARED: Dict[int, Dict[str, str]] = {
+    8: {"siamese_conv1_p": "siamese_conv1", "siamese_conv2_p": "siamese_conv2"},
+}
+
 # Sibling layers that read the same input tensor in the real network and can run as one fused
 # group (include/glp.h "fused sibling groups"): GoogLeNet inception 5b's
 # 1x1, 3x3_reduce and 5x5_reduce branches (Table 5 conv_3, conv_5, conv_6) all read 5b's
@@ -119,6 +167,7 @@ SIBLINGS: Dict[int, List[List[str]]] = {
     5: [["googlenet_conv_3", "googlenet_conv_5", "googlenet_conv_6"]],
     6: [["i5a_1x1", "i5a_3x3_reduce", "i5a_5x5_reduce"],
         ["i5b_1x1", "i5b_3x3_reduce", "i5b_5x5_reduce"]],
+    9: [[f"g_{m}_1x1", f"g_{m}_3x3_reduce", f"g_{m}_5x5_reduce"] for m, *_ in _INCEPTION],
 }
 
 # The network DAG of a workload as levels of layers that are independent of each other in the
@@ -129,6 +178,14 @@ SIBLINGS: Dict[int, List[List[str]]] = {
 # the module input (1x1, 3x3_reduce, 5x5_reduce, pool_proj after the max-pool), then the 3x3 and
 # 5x5 convolutions of the reduced maps.
 LEVELS: Dict[int, List[List[str]]] = {
+    # Siamese: the two towers run side by side (conv2 reads conv1's output in each tower)
+    8: [["siamese_conv1_p", "siamese_conv1"], ["siamese_conv2_p", "siamese_conv2"]],
+    # full GoogLeNet: the stem is a chain; per module, the branches that read the module input,
+    # then the 3x3 and 5x5 convolutions of the reduced maps
+    9: [["g_conv1_7x7_s2"], ["g_conv2_reduce"], ["g_conv2_3x3"]] +
+       [lv for m, *_ in _INCEPTION
+        for lv in ([f"g_{m}_1x1", f"g_{m}_3x3_reduce", f"g_{m}_5x5_reduce", f"g_{m}_pool_proj"],
+                   [f"g_{m}_3x3", f"g_{m}_5x5"])],
     5: [["googlenet_conv_1", "googlenet_conv_2"],
         ["googlenet_conv_3", "googlenet_conv_5", "googlenet_conv_6"],
         ["googlenet_conv_4"]],
@@ -146,6 +203,8 @@ CONFIG_NAMES = {
     5: "googlenet_table5_units_b128",
     6: "googlenet_inception_5a5b_b128",
     7: "caffenet_group2_conv1-5_b256",
+    8: "siamese_lenet_shared_b64",
+    9: "googlenet_full_224_b128",
 }
 
 

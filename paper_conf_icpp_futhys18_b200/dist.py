@@ -40,6 +40,7 @@ class FlatGrads:
             n = s[0] * s[1] * s[2] * s[3]
             self.slots.append(GradSlot(tuple(s), off, off + n, s[0]))
             off += n + s[0]
+            off = (off + 3) // 4 * 4   # every dW starts 16-byte aligned (the library checks)
         self.numel = off
         self.buf = torch.zeros(off, device=device, dtype=dtype or torch.float32)
 

@@ -166,13 +166,18 @@ def _bucket_worker(rank, world, port, q):
     a, b = FlatGrads(shapes), FlatGrads(shapes)
     g = torch.Generator().manual_seed(100 + rank)
     a.buf.copy_(torch.randn(a.numel, generator=g))
+    pad = torch.ones(a.numel, dtype=torch.bool)   # the alignment padding between slots stays 0
+    for sl in a.slots:
+        pad[sl.w_off:sl.b_off + sl.co] = False
+    a.buf[pad] = 0.0
     b.buf.copy_(a.buf)
     a.allreduce()
     works = [dist.all_reduce(b.bucket([i]), async_op=True) for i in reversed(range(len(shapes)))]
     for w in works:
         w.wait()
     q.put((rank, a.buf.numpy().copy(), b.buf.numpy().copy(),
-           b.bucket([1, 2]).numel() == b.numel - (4 * 27 + 4)))
+           b.bucket([1, 2]).numel() == b.slots[2].b_off + b.slots[2].co - b.slots[1].w_off
+           and all(sl.w_off % 4 == 0 for sl in b.slots)))
     dist.barrier()
     dist.destroy_process_group()
 

@@ -90,7 +90,9 @@ def _check(kind, got, ref, emu, scale, exact, math, what):
         what, float((np.abs(got - emu) / np.maximum(scale, 1e-30)).max()))
 
 
-def _check_unit(tmp, i, u, math, exact, rng):
+def _check_unit(tmp, i, u, math, exact, rng, extra=()):
+    """extra: (x, dy) of the units that share this unit's parameters (Siamese towers): their
+    filter gradients accumulate into this unit's dW / db (Caffe beta = 1)."""
     S, P, G = u["S"], u["P"], u["groups"]
     x = np.asarray(_load(tmp, i, "x"))
     grp = u["kind"] == "group"
@@ -128,6 +130,10 @@ def _check_unit(tmp, i, u, math, exact, rng):
                             _sl(wp, slice(g * Cog, (g + 1) * Cog)), math, None, S, P, j) + float(bg[j[1]]))
             sc.append(oracle.conv_fwd_at(xi, wg, None, S, P, j, absmode=True) + abs(float(bg[j[1]])))
         _check("y", g_, ref, emu, sc, exact, math, f"{name} y")
+        if u.get("shares"):   # dW / db are the owner's (checked there, with this unit's share)
+            dx_terms.append((w, wp, dy, dyp, Cg, Cog))
+            continue
+        ext = [(ex, ed, _prep(ex, math), _prep(ed, math)) for ex, ed in extra]
         # filter gradient
         idx = _samples(dw.shape, rng)
         g_, ref, emu, sc = [], [], [], []
@@ -136,17 +142,22 @@ def _check_unit(tmp, i, u, math, exact, rng):
             j = (co - g * Cog, ci, kh, kw)
             wsh = (Cog, Cg, w.shape[2], w.shape[3])
             g_.append(dw[co, ci, kh, kw])
-            ref.append(oracle.conv_bwd_filter_at(x[:, cs], dy[:, os_], wsh, S, P, j))
-            emu.append(_emu(oracle.conv_bwd_filter_at, _sl(xp, slice(None), cs),
-                            _sl(dyp, slice(None), os_), math, wsh, S, P, j))
-            sc.append(oracle.conv_bwd_filter_at_abs(x[:, cs], dy[:, os_], wsh, S, P, j))
+            r_, e_, s_ = 0.0, 0.0, 0.0
+            for xx, dd, xxp, ddp in [(x, dy, xp, dyp)] + ext:
+                r_ += oracle.conv_bwd_filter_at(xx[:, cs], dd[:, os_], wsh, S, P, j)
+                e_ += _emu(oracle.conv_bwd_filter_at, _sl(xxp, slice(None), cs),
+                           _sl(ddp, slice(None), os_), math, wsh, S, P, j)
+                s_ += oracle.conv_bwd_filter_at_abs(xx[:, cs], dd[:, os_], wsh, S, P, j)
+            ref.append(r_)
+            emu.append(e_)
+            sc.append(s_)
         _check("dw", g_, ref, emu, sc, exact, math, f"{name} dW")
         # bias gradient in full (the oracle's plain sum over n, ho, wo)
-        ref = oracle.conv_db(dy)
+        ref = oracle.conv_db(dy) + sum(oracle.conv_db(ed) for _, ed in extra)
         if exact:
             np.testing.assert_array_equal(np.asarray(db, np.float64), ref, err_msg=f"{name} db")
         else:
-            scale = np.abs(dy.astype(np.float64)).sum(axis=(0, 2, 3))
+            scale = sum(np.abs(d_.astype(np.float64)).sum(axis=(0, 2, 3)) for d_ in [dy] + [e for _, e in extra])
             assert np.all(np.abs(np.asarray(db, np.float64) - ref) <= 1e-5 * scale + 1e-30), name
         dx_terms.append((w, wp, dy, dyp, Cg, Cog))
     if "dx" not in u["arrays"]:
@@ -177,7 +188,8 @@ CASES = [(1, "bf16", False), (2, "bf16", False), (3, "bf16", False), (4, "bf16",
          (4, "tf32", False), (5, "bf16", False), (5, "bf16", True), (6, "bf16", False),
          (7, "bf16", True),
          (1, "fp32", False), (2, "fp32", False), (3, "fp32", False), (4, "fp32", False),
-         (5, "fp32", False), (6, "fp32", False), (7, "fp32", True), (7, "fp32", False)]
+         (5, "fp32", False), (6, "fp32", False), (7, "fp32", True), (7, "fp32", False),
+         (8, "bf16", True), (8, "fp32", False), (9, "fp32", False), (9, "bf16", True)]
 
 
 @pytest.mark.parametrize("case", CASES, ids=lambda c: f"cfg{c[0]}-{c[1]}-{'exact' if c[2] else 'float'}")
@@ -186,8 +198,11 @@ def test_fullsize_sampled_parity(case, tmp_path):
     meta = _bench_dump(tmp_path, workload, math, exact)
     assert meta["workload"] == workload and meta["math"] == math
     rng = np.random.Generator(np.random.PCG64(1000 + workload))
-    for i, u in enumerate(meta["units"]):
-        _check_unit(tmp_path, i, u, math, exact, rng)
+    units = meta["units"]
+    for i, u in enumerate(units):
+        extra = [(np.asarray(_load(tmp_path, j, "x")), np.asarray(_load(tmp_path, j, "dy")))
+                 for j, v in enumerate(units) if v.get("shares") == u["names"][0]]
+        _check_unit(tmp_path, i, u, math, exact, rng, extra)
 
 
 def test_fullsize_whole_tensor_exact(tmp_path):

@@ -282,8 +282,9 @@ glp_status_t glp_sum2(const float *a, const float *b, float *out, size_t n, glp_
  * GLP4NN's own scheme (P165-173, Figs 4/6): every layer pass runs as per-sample kernels (batch 1,
  * the sample's im2col+GEMM chain) dispatched round-robin (P171) over a pool of CUDA streams whose
  * size is the paper's Eq. 7 bound for the per-sample forward kernel (P245: thread and shared-
- * memory terms, no launch term, capped by the concurrent-kernel limit C of Eq. 6) or the caller's
- * n_streams (> 0; both capped by N and 64).  Kept to measure what the persistent tile scheduler
+ * memory terms, plus the launch term once glp_pool_set_launch_term has supplied the measured
+ * T_K / T_launch; capped by the concurrent-kernel limit C of Eq. 6) or the caller's n_streams
+ * (> 0; both capped by N and 64).  Kept to measure what the persistent tile scheduler
  * of the glp_conv_* calls buys on B200 (bench.py --scheme pool); not the product path.
  * A pool owns its streams and a per-sample plan; desc must be a single layer (no groups).
  * Calls fork from `stream` (event), run on the pool's streams and join back to `stream`.
@@ -298,6 +299,15 @@ typedef struct glp_pool_s *glp_pool_t;
 glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t desc, int device, glp_math_t math,
                              int n_streams);
 glp_status_t glp_pool_get_info(glp_pool_t pool, int *n_streams, int *eq7_bound, size_t *ws_bytes);
+/* Eq. 7's launch term (P243-245, reading R17): #K_i <= ceil(T_K / T_launch), with T_K the
+ * per-sample forward kernel's duration and T_launch the host launch cost, both measured (us) by
+ * the CUPTI resource tracker (include/glp_tracker.h) in a profiling run of the pool ("profile once",
+ * P173).  Recomputes the Eq. 7 bound with the term and, unless the caller fixed n_streams, resizes
+ * the pool to it (re-query ws_bytes with glp_pool_get_info).  GLP_ERR_INVALID_VALUE unless both
+ * times are positive. */
+glp_status_t glp_pool_set_launch_term(glp_pool_t pool, double t_kernel_us, double t_launch_us);
+/* The pool's Eq. 7 bound without and with the launch term (0 until glp_pool_set_launch_term). */
+glp_status_t glp_pool_get_eq7(glp_pool_t pool, int *without_launch_term, int *with_launch_term);
 glp_status_t glp_pool_conv_fwd(glp_pool_t pool, const float *x, const float *w, const float *b,
                                float *y, void *ws, size_t ws_bytes, glp_stream_t stream);
 /* dx may be NULL (data-fed layer), db may be NULL.  dW, db are overwritten. */

@@ -87,7 +87,7 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
            "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
            "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups", "glp_sum2",
-           "glp_plan_ex", "glp_plan_options_default"]
+           "glp_plan_ex", "glp_plan_options_default", "glp_pool_set_launch_term", "glp_pool_get_eq7"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA, GLP_PACK_W_BOTH = 0, 1, 2, 3, 4, 5
 
@@ -149,6 +149,8 @@ def lib():
         L.glp_pool_conv_fwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_pool_conv_bwd.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _c_size, _vp]
         L.glp_pool_destroy.argtypes = [_vp]
+        L.glp_pool_set_launch_term.argtypes = [_vp, _dbl, _dbl]
+        L.glp_pool_get_eq7.argtypes = [_vp, P(_c_int), P(_c_int)]
         L.glp_conv_desc_set_groups.argtypes = [_vp, _c_int]
         L.glp_sum2.argtypes = [_vp, _vp, _vp, _c_size, _vp]
         _lib = L
@@ -505,19 +507,54 @@ class StreamPool:
         self._pool = _vp()
         _ck(L.glp_pool_create(ctypes.byref(self._pool), self._desc, int(device), self.math,
                               int(n_streams)), "glp_pool_create")
+        self.device = int(device)
+        Ho, Wo = (H + 2 * pad - K) // stride + 1, (W + 2 * pad - K) // stride + 1
+        self._shapes = {"x": (N, C, H, W), "y": (N, Co, Ho, Wo), "w": (Co, C, K, K), "b": (Co,)}
+        self.eq7_launch_bound = 0
+        self.t_kernel_us = self.t_launch_us = None
+        self._sync_info()
+
+    def _sync_info(self):
+        """Pool size, Eq. 7 bounds and workspace (re-read after a recalibration)."""
+        import torch
+        L = lib()
         ns, eq7, wsb = _c_int(), _c_int(), _c_size()
         _ck(L.glp_pool_get_info(self._pool, ctypes.byref(ns), ctypes.byref(eq7), ctypes.byref(wsb)),
             "glp_pool_get_info")
         self.n_streams, self.eq7_bound = ns.value, eq7.value
         nbytes = wsb.value + 1024
-        self.device = int(device)
-        g = self.geom
-        Ho, Wo = (H + 2 * pad - K) // stride + 1, (W + 2 * pad - K) // stride + 1
-        self._shapes = {"x": (N, C, H, W), "y": (N, Co, Ho, Wo), "w": (Co, C, K, K), "b": (Co,)}
-        self._ws_buf = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{int(device)}")
-        off = (-self._ws_buf.data_ptr()) % 1024
-        self.ws_ptr = self._ws_buf.data_ptr() + off
-        self.ws_bytes = nbytes - off
+        if getattr(self, "_ws_nbytes", 0) < nbytes:
+            self._ws_buf = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{self.device}")
+            self._ws_nbytes = nbytes
+            off = (-self._ws_buf.data_ptr()) % 1024
+            self.ws_ptr = self._ws_buf.data_ptr() + off
+            self.ws_bytes = nbytes - off
+
+    def set_launch_term(self, t_kernel_us, t_launch_us):
+        """Eq. 7 with the T_K / T_launch term (glp_pool_set_launch_term)."""
+        _ck(lib().glp_pool_set_launch_term(self._pool, float(t_kernel_us), float(t_launch_us)),
+            "glp_pool_set_launch_term")
+        a, b = _c_int(), _c_int()
+        _ck(lib().glp_pool_get_eq7(self._pool, ctypes.byref(a), ctypes.byref(b)), "glp_pool_get_eq7")
+        self.eq7_launch_bound = b.value
+        self.t_kernel_us, self.t_launch_us = float(t_kernel_us), float(t_launch_us)
+        self._sync_info()
+
+    def calibrate(self, x, w, b, y):
+        """"Profile once" (P173): run the pool's forward once under the CUPTI resource tracker,
+        take T_K = the mean duration of the per-sample forward GEMM kernels and T_launch = the
+        mean duration of the kernel-launch API calls, and apply Eq. 7's launch term.  Returns
+        (T_K us, T_launch us, records of the profiled kernels)."""
+        from .tracker import Tracker
+        with Tracker() as t:
+            self.fwd(x, w, b, y)
+        gemm = [k for k in t.kernels if any(s in k.name for s in ("igemm", "hfwd", "simt_fwd"))]
+        if not gemm or not t.launch_us:
+            raise RuntimeError("resource tracker recorded no forward kernels / launches")
+        tk = sum(k.duration_us for k in gemm) / len(gemm)
+        tl = sum(t.launch_us) / len(t.launch_us)
+        self.set_launch_term(tk, tl)
+        return tk, tl, gemm
 
     def _c(self, t, kind, name, nullable=False):
         return _checked(t, self._shapes[kind], self.device, name, nullable)

@@ -44,6 +44,25 @@ def build(force: bool = False, verbose: bool = False, diag: bool = False) -> str
     return lib
 
 
+TRACKER_LIB = os.path.join(PKG, "libglp_tracker.so")
+CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
+
+
+def build_tracker(force: bool = False) -> str:
+    """libglp_tracker.so: the CUPTI resource tracker (csrc/tracker.cpp, include/glp_tracker.h),
+    host C++ linked against the toolkit's libcupti."""
+    src = [os.path.join(PKG, "csrc", "tracker.cpp"), os.path.join(ROOT, "include", "glp_tracker.h")]
+    if not force and os.path.exists(TRACKER_LIB) and not any(
+            os.path.getmtime(s) > os.path.getmtime(TRACKER_LIB) for s in src):
+        return TRACKER_LIB
+    tmp = TRACKER_LIB + f".tmp{os.getpid()}"
+    lib64 = os.path.join(CUDA, "lib64")
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-shared", "-I", os.path.join(CUDA, "include"),
+                           "-o", tmp, src[0], "-L", lib64, "-lcupti", f"-Wl,-rpath,{lib64}"])
+    os.replace(tmp, TRACKER_LIB)
+    return TRACKER_LIB
+
+
 if __name__ == "__main__":
     import sys
     print(build(force=True, verbose=True, diag="--diag" in sys.argv))

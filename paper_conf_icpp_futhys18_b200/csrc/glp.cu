@@ -2331,6 +2331,11 @@ struct glp_pool_s {
   glp_conv_desc_s d1;            // the per-sample (N = 1) layer
   glp_plan_t plan1 = nullptr;    // its plan (shared by every stream: plans are immutable)
   int N = 0, device = 0, math = 0, S = 1, eq7 = 1;
+  int eq7_launch = 0;           // Eq. 7 bound with the measured T_K / T_launch term (0: not set)
+  int n_streams_req = 0, cap = 1;  // caller's pool size (0 = the Eq. 7 bound); streams created
+  glp_kernel_attr_t ka{};       // the per-sample forward kernel's record (Eq. 7 input)
+  int blocks = 1;
+  double t_kernel = 0, t_launch = 0;
   size_t slot_ws = 0, acc_floats = 0, ws_bytes = 0;
   std::vector<cudaStream_t> streams;
   std::vector<cudaEvent_t> joins;
@@ -2382,19 +2387,23 @@ glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t d, int device, glp
   if (math != GLP_MATH_FP32_SIMT) {
     int m = 0, r = 0;
     glp_plan_kernel_attr(Q->plan1, 0, &ka, &m, &r);
-    blocks = Q->plan1->fwd.grid;
+    blocks = Q->plan1->hfwd ? Q->plan1->hf_grid : Q->plan1->fwd.grid;
   }
+  Q->ka = ka;
+  Q->blocks = blocks;
   int bound = 1;
   glp_analyze_eq7(&L, &ka, blocks, 0.0, 0.0, &bound);
   Q->eq7 = std::max(1, std::min(bound, L.max_concurrent_kernels));
-  Q->S = std::max(1, std::min(n_streams > 0 ? n_streams : Q->eq7, std::min(Q->N, 64)));
+  Q->n_streams_req = n_streams;
+  Q->cap = std::max(1, std::min(Q->N, 64));
+  Q->S = std::max(1, std::min(n_streams > 0 ? n_streams : Q->eq7, Q->cap));
   Q->slot_ws = align1k(std::max<size_t>(Q->plan1->ws_bwd, 1));
   Q->acc_floats = (size_t)rup((long long)d->Co * d->C * d->Kh * d->Kw + d->Co, 64);
   Q->ws_bytes = (size_t)Q->S * Q->slot_ws + align1k((size_t)Q->S * Q->acc_floats * 4);
   int cur = 0;
   cudaGetDevice(&cur);
   if (cur != device) cudaSetDevice(device);
-  for (int i = 0; i < Q->S; ++i) {
+  for (int i = 0; i < Q->cap; ++i) {   // every stream the pool may use after a recalibration
     cudaStream_t st;
     cudaEvent_t ev;
     if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess ||
@@ -2409,6 +2418,29 @@ glp_status_t glp_pool_create(glp_pool_t *out, glp_conv_desc_t d, int device, glp
   cudaEventCreateWithFlags(&Q->fork, cudaEventDisableTiming);
   if (cur != device) cudaSetDevice(cur);
   *out = Q;
+  return GLP_OK;
+}
+
+glp_status_t glp_pool_set_launch_term(glp_pool_t Q, double t_kernel_us, double t_launch_us) {
+  if (!Q || !(t_kernel_us > 0) || !(t_launch_us > 0))
+    return fail(GLP_ERR_INVALID_VALUE, "T_K and T_launch must be positive");
+  glp_device_limits_t L;
+  glp_device_limits_b200(&L);
+  int bound = 1;
+  glp_status_t s = glp_analyze_eq7(&L, &Q->ka, Q->blocks, t_kernel_us, t_launch_us, &bound);
+  if (s) return s;
+  Q->t_kernel = t_kernel_us;
+  Q->t_launch = t_launch_us;
+  Q->eq7_launch = std::max(1, std::min(bound, L.max_concurrent_kernels));
+  Q->S = std::max(1, std::min(Q->n_streams_req > 0 ? Q->n_streams_req : Q->eq7_launch, Q->cap));
+  Q->ws_bytes = (size_t)Q->S * Q->slot_ws + align1k((size_t)Q->S * Q->acc_floats * 4);
+  return GLP_OK;
+}
+
+glp_status_t glp_pool_get_eq7(glp_pool_t Q, int *without_launch_term, int *with_launch_term) {
+  if (!Q) return fail(GLP_ERR_INVALID_VALUE, "pool is NULL");
+  if (without_launch_term) *without_launch_term = Q->eq7;
+  if (with_launch_term) *with_launch_term = Q->eq7_launch;
   return GLP_OK;
 }
 

@@ -18,10 +18,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def built():
     from paper_conf_icpp_futhys18_b200 import _build
     _build.build()
+    _build.build_tracker()
 
 
-def header_functions():
-    src = open(os.path.join(ROOT, "include", "glp.h")).read()
+def header_functions(header="glp.h"):
+    src = open(os.path.join(ROOT, "include", header)).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
     return sorted(set(re.findall(r"\b(glp_[a-z0-9_]+)\s*\(", src)))
 
@@ -144,3 +145,20 @@ def test_product_library_reads_no_environment():
     knobs = sorted(k for k in set(re.findall(rb"GLP_[A-Z][A-Z0-9_]+", blob))
                    if not k.startswith(api))
     assert knobs == [], knobs
+
+
+def test_tracker_exports_every_declared_symbol():
+    """libglp_tracker.so (the CUPTI resource tracker, include/glp_tracker.h) loads and exports
+    every declared call; its record structs match the header's field order."""
+    from paper_conf_icpp_futhys18_b200 import tracker
+    decl = header_functions("glp_tracker.h")
+    assert sorted(tracker.EXPORTS) == decl
+    L = tracker.lib()
+    for name in decl:
+        assert getattr(L, name) is not None
+    src = open(os.path.join(ROOT, "include", "glp_tracker.h")).read()
+    body = re.sub(r"/\*.*?\*/", "", src[src.index("typedef struct {"):src.index("} glp_kernel_record_t;")],
+                  flags=re.S)
+    fields = re.findall(r"\b(name|grid|block|cluster|regs|static_smem|dynamic_smem|queued_ns|"
+                        r"submitted_ns|start_ns|end_ns|stream_id|correlation_id)\b", body)
+    assert fields == [f for f, _ in tracker.KernelRecord._fields_]

@@ -787,3 +787,55 @@ def test_samples_in_flight_through_analyzer(math):
             rows = Ho * Ho * -(-Co // info.tile_n_fwd)
         assert (info.s_slot_rows, info.s_rows_per_sample) == (slot_rows, rows), name
         assert info.samples_in_flight == A.samples_in_flight_enum(slot_rows, rows, N), name
+
+
+def test_resource_tracker_records_plan_kernels():
+    """The CUPTI resource tracker (NEXT-4; P165) records the kernels a call launches with the
+    analyzer's inputs: the forward GEMM's grid, block, cluster, registers and shared memory equal
+    the plan's, and launch-API durations (T_launch) are collected."""
+    from paper_conf_icpp_futhys18_b200.tracker import Tracker
+    shape = SHAPES[6]
+    layer = _layer(shape, "bf16")
+    d = _data(shape, seed=2)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    y = torch.empty(layer.y_shape, device=DEV)
+    layer.fwd(t["x"], t["w"], t["b"], y)
+    torch.cuda.synchronize()
+    with Tracker() as tr:
+        layer.fwd(t["x"], t["w"], t["b"], y)
+    gemm = [k for k in tr.kernels if "igemm_kernel" in k.name]
+    assert len(gemm) == 1, [k.name for k in tr.kernels]
+    k, a = gemm[0], layer.kernel_attr(0)
+    assert (k.grid[0], k.block[0], k.regs) == (layer.info.grid_fwd, a["threads"], a["regs"])
+    assert k.cluster[0] in (1, 2) and k.smem >= a["smem"] and k.duration_us > 0
+    assert any("pack" in r.name for r in tr.kernels)
+    assert len(tr.launch_us) >= 3 and all(v > 0 for v in tr.launch_us)
+
+
+@pytest.mark.parametrize("math", ["bf16", "fp32"])
+def test_pool_eq7_launch_term(math):
+    """The stream-pool comparator profiled once by the resource tracker: T_K (its per-sample
+    forward GEMMs) and T_launch (launch API calls) give the Eq. 7 bound with the launch term
+    (P245) exactly as the oracle's model computes it, the pool resizes to it, and its outputs
+    keep the persistent path's bits."""
+    from oracle import analyzer as A
+    shape = SHAPES[0]
+    _, N, C, H, W, Co, K, S, P = shape
+    d = _data(shape, seed=3)
+    T = lambda a: torch.from_numpy(a).to(DEV)
+    pool = glp.StreamPool(N, C, H, W, Co, K, S, P, math=math)
+    y = torch.empty((N, Co, oracle.out_dim(H, K, S, P), oracle.out_dim(W, K, S, P)), device=DEV)
+    pool.fwd(T(d["x"]), T(d["w"]), T(d["b"]), y)
+    tk, tl, recs = pool.calibrate(T(d["x"]), T(d["w"]), T(d["b"]), y)
+    assert tk > 0 and tl > 0 and len(recs) == N   # one per-sample forward GEMM per sample
+    one = glp.ConvLayer(1, C, H, W, Co, K, S, P, math=math)
+    a = one.kernel_attr(0)
+    kern = A.Kernel(blocks=one.info.grid_fwd, threads=a["threads"], smem=a["smem"],
+                    t_kernel=tk, t_launch=tl)
+    exp = max(1, min(A.eq7_bound(kern, A.B200()), A.B200().C))
+    assert pool.eq7_launch_bound == exp
+    assert pool.n_streams == max(1, min(exp, N, 64))
+    y2 = torch.empty_like(y)
+    pool.fwd(T(d["x"]), T(d["w"]), T(d["b"]), y2)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(y2.cpu().numpy(), _run(_layer(shape, math), d)["y"])

@@ -208,15 +208,17 @@ class ClockSampler:
 # ------------------------------------------------------------------------- GLP arm ------------
 
 class LayerState:
-    def __init__(self, layer, n_local, n_global, shard, math, dev, grads, idx):
+    def __init__(self, layer, n_local, n_global, shard, math, dev, grads, idx, leaves=0):
         import torch
         import paper_conf_icpp_futhys18_b200 as glp
         self.glp = glp
         self.layer = layer
         self.name = layer.name
         self.n = n_local
+        # leaves > 1: a leaf plan (the deterministic exchange: splits never cross a batch leaf)
         self.conv = glp.ConvLayer(n_local, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.S,
-                                  layer.P, math=math, device=dev.index, groups=layer.groups)
+                                  layer.P, math=math, device=dev.index, groups=layer.groups,
+                                  options={"wgrad_leaves": leaves} if leaves > 0 else None)
         if shard is None:
             d = gen_layer(layer, n_global=n_global, batch=n_local)
         else:  # strong scaling: this rank's contiguous slice of the global batch
@@ -255,18 +257,6 @@ class LayerState:
         """Slots of the flat dW||db buffer this unit writes (its all-reduce bucket)."""
         return [self.owner.idx if self.owner is not None else self.idx]
 
-    def use_leaves(self, leaf_grads, idx, math, dev):
-        """Deterministic exchange: the filter gradient per batch leaf of this rank (one plan for
-        the leaf batch), each into its leaf's flat buffer."""
-        glp = self.glp
-        k = len(leaf_grads)
-        nl = self.n // k
-        l = self.layer
-        self.leaf_conv = glp.ConvLayer(nl, l.C, l.H, l.W, l.Co, l.K, l.S, l.P, math=math,
-                                       device=dev.index, groups=l.groups)
-        self.leaves = [(self.t["x"][j * nl:(j + 1) * nl], self.t["dy"][j * nl:(j + 1) * nl],
-                        lg.dw(idx), lg.db(idx)) for j, lg in enumerate(leaf_grads)]
-
     def launches(self):
         """Kernels this unit launches per timed step: pack x, W pack(s), fwd GEMM, dy pack, dgrad
         GEMM, filter-gradient GEMM, dW and db reductions; a fused-dy plan (data-fed halo layer)
@@ -274,7 +264,7 @@ class LayerState:
         base = 9 if self.dx is not None else 7
         if self.dx is None and self.conv.info.wgrad_fused_dy:
             base -= 1
-        return base if self.leaves is None else base - 4 + 6 * len(self.leaves)
+        return base
 
     # the step's kernel groups (one C call each; see step())
     def pack_x(self, st=None):
@@ -296,19 +286,16 @@ class LayerState:
         self.conv.stage_bwd_data(self.dx, stream=st)
 
     def bwd_filter(self, st=None):
-        if self.leaves is None:
-            self.conv.stage_bwd_filter(stream=st)
-            return
-        lc, glp = self.leaf_conv, self.glp
-        for x, dy, dw, db in self.leaves:
-            lc.stage_pack(glp.GLP_PACK_X, x, stream=st)
-            lc.stage_pack(glp.GLP_PACK_DY_DB, dy, stream=st)
-            lc.stage_bwd_filter(stream=st)
-            lc.stage_reduce(dw, db, stream=st)
+        self.conv.stage_bwd_filter(stream=st)
 
     def reduce(self, st=None):
         if self.leaves is None:
             self.conv.stage_reduce(self.dw, self.db, accumulate=self.accumulate, stream=st)
+            return
+        # deterministic exchange: one dW||db per leaf into the leaf buffers (the tree sums them)
+        ex, sl = self.leaves, self.slot
+        flat = ex.leaves.view(-1)
+        self.conv.stage_reduce_leaves(flat[sl.w_off:], flat[sl.b_off:], ex.numel, stream=st)
 
     def host_inputs(self):
         return self.host, self.t
@@ -524,7 +511,7 @@ def run_pool(args):
         "tflops_step": round(step_flops / (ms * 1e-3) / 1e12, 1)}), flush=True)
 
 
-def build_states(args, math, G, rank, dev, grads):
+def build_states(args, math, G, rank, dev, grads, leaves=0):
     """Plans, seeded inputs and outputs of every unit of the workload at this rank's batch."""
     from paper_conf_icpp_futhys18_b200.dist import shard_range
     layers = config(args.workload)
@@ -543,7 +530,7 @@ def build_states(args, math, G, rank, dev, grads):
         shard = shards[i] if args.scaling == "strong" and G > 1 else None
         gi = in_group.get(l.name)
         if gi is None:
-            states.append(LayerState(l, nl, ng, shard, math, dev, grads, i))
+            states.append(LayerState(l, nl, ng, shard, math, dev, grads, i, leaves))
         elif gi not in done_groups:
             if shard is not None:
                 raise SystemExit("fused groups with strong scaling: use --no-fuse")
@@ -581,10 +568,10 @@ class Step:
     remaining backward-data work of the earlier layers; the step ends when every bucket has
     arrived.  'tree' = the deterministic exchange (NEXT-2) after the step."""
 
-    def __init__(self, args, states, grads, G, dev, tree=None, leaf_grads=None):
+    def __init__(self, args, states, grads, G, dev, tree=None):
         import torch
         self.args, self.states, self.grads, self.G = args, states, grads, G
-        self.tree, self.leaf_grads = tree, leaf_grads
+        self.tree = tree
         self.levels = dag_levels(args, states)
         self.width = max(len(l) for l in self.levels)
         self.side_w = torch.cuda.Stream(device=dev)   # weight packs (known at step start)
@@ -607,7 +594,7 @@ class Step:
     def exchange_tail(self):
         """Join the exchange: bucketed all-reduces (already in flight) or the tree."""
         if self.tree is not None:
-            self.grads.buf.copy_(self.tree([lg.buf for lg in self.leaf_grads]))
+            self.tree(self.grads.buf)
         for w in self.works:
             w.wait()   # the current stream waits for the collective
         self.works = []
@@ -800,22 +787,25 @@ def run_glp(args, ws, rank, local):
     grads = FlatGrads([l.w_shape for l in layers], device=dev)
     flat = grads.buf
     nparams = grads.numel
-    layers, states, n_local = build_states(args, args.math, G, rank, dev, grads)
+    tree, n_leaves = None, 0
+    if args.exchange == "tree":
+        from paper_conf_icpp_futhys18_b200.dist import LeafTreeExchange, rank_leaves
+        n_leaves = len(rank_leaves(rank, G))
+        if SIBLINGS.get(args.workload) and not args.no_fuse:
+            raise SystemExit("--exchange tree: single layers only (use --no-fuse)")
+        if SHARED.get(args.workload):
+            raise SystemExit("--exchange tree: no shared-parameter workloads")
+    layers, states, n_local = build_states(args, args.math, G, rank, dev, grads, n_leaves)
     if args.exact_data:
         set_exact_data(states)
     stream = torch.cuda.current_stream()
-
-    tree, leaf_grads = None, None
     if args.exchange == "tree":
-        from paper_conf_icpp_futhys18_b200.dist import TreeAllreduce, rank_leaves
-        my_leaves = rank_leaves(rank, G)
-        if any(not isinstance(s, LayerState) for s in states) or n_local[0] % len(my_leaves):
-            raise SystemExit("--exchange tree: single layers and a leaf-divisible batch only")
-        leaf_grads = [FlatGrads([l.w_shape for l in layers], device=dev) for _ in my_leaves]
-        for i, s in enumerate(states):
-            s.use_leaves(leaf_grads, i, args.math, dev)
-        tree = TreeAllreduce()
-    step = Step(args, states, grads, G, dev, tree, leaf_grads)
+        # the step packs once; each unit's filter gradient reduces per leaf into the exchange's leaf
+        # buffers; the fixed 8-leaf tree (local subtree + top levels across ranks) gives dW||db
+        tree = LeafTreeExchange(grads.numel, n_leaves, dev)
+        for s in states:
+            s.leaves, s.slot = tree, grads.slots[s.idx]
+    step = Step(args, states, grads, G, dev, tree)
 
     for _ in range(args.warmup):
         step()
@@ -826,7 +816,7 @@ def run_glp(args, ws, rank, local):
     # once as a CUDA graph and replayed.  G > 1: the step is issued eagerly so that each unit's
     # gradient bucket is all-reduced (NCCL) as soon as it is ready, overlapping the rest of the
     # backward (NCCL collectives are not captured into the graph).
-    use_graph = not args.no_graph and G == 1 and tree is None
+    use_graph = not args.no_graph and G == 1
     evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(6)] for _ in states]
            for _ in range(args.steps)]
     if use_graph:
@@ -835,7 +825,11 @@ def run_glp(args, ws, rank, local):
             step(concurrent=not args.serial, with_exchange=False)
         for _ in range(max(1, args.warmup)):
             g_step.replay()
-        run_one = g_step.replay
+            step.exchange_tail()
+
+        def run_one():
+            g_step.replay()
+            step.exchange_tail()   # the tree kernel (tree mode); nothing on one GPU otherwise
     else:
         def run_one():
             step(concurrent=not args.serial)

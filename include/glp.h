@@ -163,6 +163,17 @@ typedef struct {
   int s2d_block;          /* 0: warp-per-32-pixel space-to-depth pack; 1: block-persistent          */
   int smem_cap;           /* dynamic shared memory budget of the persistent GEMMs, bytes (232448)  */
   int pdl;                /* 1: programmatic dependent launch between the plan's kernels; 0: not   */
+  int wgrad_leaves;       /* 0 (default): no leaves.  1, 2, 4 or 8: a leaf plan -- the local batch
+                             is this many equal leaves of the global batch's 8 (the deterministic
+                             exchange, NEXT-2).  The filter gradient's splits are chosen for ONE
+                             leaf (as if the 8 leaves shared the device) and never cross a leaf
+                             boundary, so a leaf's partial is the same bits on any rank; the
+                             composed calls and
+                             glp_stage_reduce return the fixed tree (glp_tree_sum) over the leaves,
+                             glp_stage_reduce_leaves the leaves themselves.  Needs N divisible by the
+                             leaves and a leaf's N*H_o*W_o a multiple of the k-block (32 pixels
+                             tf32 / fp32, 64 bf16); tensor-core single-layer plans (no fused
+                             sibling groups).  Changes the split order, hence low bits, vs 1.      */
 } glp_plan_options_t;
 glp_status_t glp_plan_options_default(glp_plan_options_t *opts);
 /* opts may be NULL (defaults).  GLP_ERR_INVALID_VALUE for an out-of-range option. */
@@ -277,6 +288,25 @@ glp_status_t glp_stage_reduce_group(glp_plan_t plan, float *const *dw, float *co
  * out may alias a or b; asynchronous on `stream`).  Since a + b == b + a bitwise, dW is bitwise
  * identical for 1, 2, 4 and 8 ranks. */
 glp_status_t glp_sum2(const float *a, const float *b, float *out, size_t n, glp_stream_t stream);
+/* out (+)= T(parts[0..n)): the balanced binary tree over n = 1, 2, 4 or 8 device arrays of count
+ * floats in index order (level by level, adjacent pairs: ((p0+p1)+(p2+p3))+((p4+p5)+(p6+p7))) --
+ * bitwise the glp_sum2 tree -- in one launch.  accumulate = 1 adds the tree to out.  A rank sums
+ * its contiguous block of leaves with it (a complete subtree of the 8-leaf tree). */
+glp_status_t glp_tree_sum(const float *const *parts, int n, float *out, size_t count,
+                          int accumulate, glp_stream_t stream);
+/* The tree's top levels across ranks over NVLink peer memory: subtrees[r] / outs[r] are rank r's
+ * subtree sum and output buffers as mapped on this device (torch symmetric memory), world = 1, 2,
+ * 4 or 8.  This rank computes the element slice [rank*count/world, (rank+1)*count/world) of
+ * T(subtrees[0..world)) with peer loads and stores it into every rank's output (peer stores).
+ * The caller brackets the call with barriers (every subtree complete before; every slice written
+ * after); then every rank holds bitwise the tree over all leaves, for any world. */
+glp_status_t glp_tree_exchange(const float *const *subtrees, float *const *outs, int world, int rank,
+                               size_t count, glp_stream_t stream);
+/* Leaf plans (wgrad_leaves > 1): the fixed-order reduction of each leaf's split partials, leaf l's
+ * dW (Caffe layout) at dw + l*leaf_stride and db at db + l*leaf_stride (db may be NULL; leaf_stride
+ * in floats, a multiple of 4).  Needs GLP_PACK_DY_DB when db != NULL.  Overwrites. */
+glp_status_t glp_stage_reduce_leaves(glp_plan_t plan, float *dw, float *db, size_t leaf_stride,
+                                     void *ws, size_t ws_bytes, glp_stream_t stream);
 
 /* ---- prior-art comparator: the paper's stream pool --------------------- *
  * GLP4NN's own scheme (P165-173, Figs 4/6): every layer pass runs as per-sample kernels (batch 1,

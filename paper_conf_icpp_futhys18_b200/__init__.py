@@ -61,7 +61,8 @@ class PlanOptions(ctypes.Structure):
                 ("halo_fwd", _c_int), ("halo_dgrad", _c_int), ("fused_dy", _c_int),
                 ("fused_dy_builders", _c_int), ("max_kblocks_per_stage", _c_int),
                 ("wgrad_tile_n", _c_int), ("tile_units", _c_int), ("bn_model", _c_int),
-                ("pack_block", _c_int), ("s2d_block", _c_int), ("smem_cap", _c_int), ("pdl", _c_int)]
+                ("pack_block", _c_int), ("s2d_block", _c_int), ("smem_cap", _c_int), ("pdl", _c_int),
+                ("wgrad_leaves", _c_int)]
 
 
 def plan_options(**kw) -> PlanOptions:
@@ -87,7 +88,8 @@ EXPORTS = ["glp_conv_desc_create", "glp_conv_desc_get_output", "glp_conv_desc_de
            "glp_conv_group_fwd", "glp_conv_group_bwd", "glp_stage_pack_group", "glp_stage_fwd_group",
            "glp_stage_reduce_group", "glp_pool_create", "glp_pool_get_info", "glp_pool_conv_fwd",
            "glp_pool_conv_bwd", "glp_pool_destroy", "glp_conv_desc_set_groups", "glp_sum2",
-           "glp_plan_ex", "glp_plan_options_default", "glp_pool_set_launch_term", "glp_pool_get_eq7"]
+           "glp_plan_ex", "glp_plan_options_default", "glp_pool_set_launch_term", "glp_pool_get_eq7",
+           "glp_tree_sum", "glp_tree_exchange", "glp_stage_reduce_leaves"]
 
 GLP_PACK_X, GLP_PACK_DY, GLP_PACK_DY_DB, GLP_PACK_W_FWD, GLP_PACK_W_BWD_DATA, GLP_PACK_W_BOTH = 0, 1, 2, 3, 4, 5
 
@@ -153,6 +155,9 @@ def lib():
         L.glp_pool_get_eq7.argtypes = [_vp, P(_c_int), P(_c_int)]
         L.glp_conv_desc_set_groups.argtypes = [_vp, _c_int]
         L.glp_sum2.argtypes = [_vp, _vp, _vp, _c_size, _vp]
+        L.glp_tree_sum.argtypes = [_vp, _c_int, _vp, _c_size, _c_int, _vp]
+        L.glp_tree_exchange.argtypes = [_vp, _vp, _c_int, _c_int, _c_size, _vp]
+        L.glp_stage_reduce_leaves.argtypes = [_vp, _vp, _vp, _c_size, _vp, _c_size, _vp]
         _lib = L
     return _lib
 
@@ -240,6 +245,11 @@ def _checked_list(ts, shapes, device, name, nullable=False, entries_nullable=Fal
     return _ptrs(ts)
 
 
+def torch_float32():
+    import torch
+    return torch.float32
+
+
 def _stream(stream):
     import torch
     s = stream if stream is not None else torch.cuda.current_stream()
@@ -252,6 +262,33 @@ def sum2(a, b, out, stream=None):
     pa, pb, po = (_checked(t, tuple(a.shape), dev, n) for t, n in ((a, "a"), (b, "b"), (out, "out")))
     _ck(lib().glp_sum2(pa, pb, po, a.numel(), _stream(stream)), "glp_sum2")
     return out
+
+
+def _addr_array(addrs):
+    arr = (ctypes.c_void_p * len(addrs))(*[int(a) for a in addrs])
+    return ctypes.cast(arr, ctypes.c_void_p), arr
+
+
+def tree_sum(parts, out, accumulate=False, stream=None):
+    """out (+)= the fixed balanced binary tree over 1, 2, 4 or 8 equal fp32 CUDA tensors
+    (glp_tree_sum): bitwise the dist.tree_sum of glp_sum2 adds, in one launch."""
+    dev = out.device.index
+    for k, p in enumerate(parts):
+        _checked(p, tuple(out.shape), dev, f"parts[{k}]")
+    po = _checked(out, tuple(out.shape), dev, "out")
+    pa, _keep = _addr_array([p.data_ptr() for p in parts])
+    _ck(lib().glp_tree_sum(pa, len(parts), po, out.numel(), int(bool(accumulate)), _stream(stream)),
+        "glp_tree_sum")
+    return out
+
+
+def tree_exchange(subtree_ptrs, out_ptrs, rank, count, stream=None):
+    """glp_tree_exchange over peer device addresses (ints, e.g. torch symmetric-memory
+    buffer_ptrs): this rank's slice of the top tree, stored into every rank's output."""
+    ps, _a = _addr_array(subtree_ptrs)
+    po, _b = _addr_array(out_ptrs)
+    _ck(lib().glp_tree_exchange(ps, po, len(subtree_ptrs), int(rank), int(count), _stream(stream)),
+        "glp_tree_exchange")
 
 
 @dataclass
@@ -407,6 +444,17 @@ class ConvLayer:
                                    int(bool(accumulate)),
                                    ctypes.c_void_p(self.ws_ptr), self.ws_bytes, _stream(stream)),
             "glp_stage_reduce")
+
+    def stage_reduce_leaves(self, dw_flat, db_flat, leaf_stride, stream=None):
+        """Leaf plans: leaf l's dW / db at dw_flat / db_flat + l * leaf_stride floats (views into
+        an [L, stride] leaf buffer; glp_stage_reduce_leaves)."""
+        for t, nm in ((dw_flat, "dw"), (db_flat, "db")):
+            if t is not None and (t.dtype != torch_float32() or not t.is_cuda or
+                                  t.device.index != self.device):
+                raise ValueError(f"{nm}: fp32 tensor on cuda:{self.device} required")
+        _ck(lib().glp_stage_reduce_leaves(self._plan, _ptr(dw_flat), _ptr(db_flat), int(leaf_stride),
+                                          ctypes.c_void_p(self.ws_ptr), self.ws_bytes,
+                                          _stream(stream)), "glp_stage_reduce_leaves")
 
     # fused sibling groups (include/glp.h "fused sibling groups"): one tensor per branch
     def branch_y_shapes(self):

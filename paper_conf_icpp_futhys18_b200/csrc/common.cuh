@@ -79,6 +79,8 @@ struct IgemmParams {
   int m_tiles, n_tiles, splits;
   int kb_total;          // k-blocks over the whole K extent
   int kb_per_split;
+  int kb_per_leaf;       // wgrad leaf plans: k-blocks per leaf (0: no leaves)
+  int splits_per_leaf;   // wgrad leaf plans: splits per leaf (0: no leaves)
   int bn;                // N tile (multiple of 16, <= 256)
   int bn_smem;           // rows/cols of B held in smem per stage
   int stages;

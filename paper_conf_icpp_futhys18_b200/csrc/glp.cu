@@ -108,6 +108,7 @@ struct PassPlan {
   int ksub = 1;                     // k-blocks per pipeline stage
   int bias_floats = 0;              // forward: floats of the epilogue's smem bias stage
   int threads = 288;                // CTA size (3xTF32: 512, eight epilogue warps)
+  int kb_per_leaf = 0, splits_per_leaf = 0;   // wgrad leaf plans (deterministic exchange)
   int chunk_kb = 0;                 // 3xTF32: k-blocks per TMEM accumulation chunk
 };
 
@@ -271,8 +272,11 @@ void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, 
 // Shape-only split count of the wgrad reduction over N*H_o*W_o: minimises a fixed cost model
 // (constants, never the queried device or S), so the fp32 summation order is a function of the
 // shape alone (convergence invariance, P264).
+// leaves > 1 (leaf plans): kb_total is ONE leaf's k-blocks and the model assumes `leaves` such
+// leaves share the device (a constant: the global batch's 8 leaves, never the rank's count, so the
+// per-leaf split count is the same on every rank).
 int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int elem, int cg,
-                  int x3) {
+                  int x3, int leaves = 1) {
   const double sm = 148.0 / cg;   // concurrent work units (CTA pairs for cg = 2)
   // seconds per k-block (3xTF32: three MMAs per k-step)
   const double kb_s = (elem == 2 ? 2.0 : 4.0) * (x3 ? 3.0 : 1.0) * std::max(bn, 96) / 1.8e9;
@@ -284,8 +288,8 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
     const int kbps = (int)cdiv(kb_total, s);
     const int real = (int)cdiv(kb_total, kbps);
     if (real != s) continue;
-    const double waves = std::ceil(tiles_mn * (double)s / sm);
-    const double t = waves * (kbps * kb_s + 2e-6) + (double)s * mpad * npad * 8.0 / bw;
+    const double waves = std::ceil(tiles_mn * (double)s * leaves / sm);
+    const double t = waves * (kbps * kb_s + 2e-6) + (double)s * leaves * mpad * npad * 8.0 / bw;
     if (t < best_t * 0.999) {
       best_t = t;
       best = s;
@@ -385,6 +389,12 @@ struct glp_plan_s {
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
   // instead of after it.  GLP_SMEM_CAP (bytes) overrides (A/B runs).
   int smem_cap = 232448;
+  // deterministic exchange: the local batch is `leaves` equal leaves of
+  // the global batch; the filter gradient's splits never cross a leaf, so each leaf's partial is
+  // the same bits on any rank, and the leaves are summed by a fixed binary tree
+  int leaves = 1;
+  int leaf_plan = 0;   // wgrad_leaves > 0: the per-leaf split model (also with one local leaf)
+  size_t off_leaf = 0, sz_leaf = 0, leaf_stride = 0;   // workspace leaf partials (composed calls)
   int pack_block = 0;  // GLP_PACK_BLOCK=1: the block-tiled activation pack (A/B runs)
   int s2d_block = 0;   // GLP_S2D_BLOCK=1: the block-persistent space-to-depth pack (A/B runs)
   unsigned long long *dbg_clk = nullptr;   // GLP_DEBUG_CLK=1: per-CTA cycle counters (diagnostics)
@@ -699,7 +709,20 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   if (pp.cg == 2) pp.bn_smem = pp.bn / 2;
   pp.n_tiles = (int)cdiv(pp.Ng, pp.bn);
   pp.m_units = (int)cdiv(pp.m_tiles, pp.cg);
-  if (mode == MODE_WGRAD) {
+  if (mode == MODE_WGRAD && P.leaf_plan) {
+    // leaf plan: the split count of ONE leaf (its shape only: the same for every rank count)
+    const long long pleaf = (long long)(d.N / P.leaves) * d.Ho * d.Wo;
+    if (d.N % P.leaves || pleaf % BKP)
+      return fail(GLP_ERR_NOT_SUPPORTED, "wgrad leaves: the batch must split into leaves whose "
+                                         "pixel count is a multiple of the k-block");
+    pp.kb_per_leaf = (int)(pleaf / BKP);
+    pp.splits_per_leaf = choose_splits(pp.m_units * pp.n_tiles, pp.kb_per_leaf, pp.bn,
+                                       pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg,
+                                       P.x3, /*leaves of the global batch*/ 8);
+    pp.kb_per_split = (int)cdiv(pp.kb_per_leaf, pp.splits_per_leaf);
+    pp.splits_per_leaf = (int)cdiv(pp.kb_per_leaf, pp.kb_per_split);
+    pp.splits = P.leaves * pp.splits_per_leaf;
+  } else if (mode == MODE_WGRAD) {
     pp.splits = choose_splits(pp.m_units * pp.n_tiles, pp.kb_total, pp.bn,
                               pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg, P.x3);
     pp.kb_per_split = (int)cdiv(pp.kb_total, pp.splits);
@@ -847,6 +870,8 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   p.splits = pp.splits;
   p.kb_total = pp.kb_total;
   p.kb_per_split = pp.kb_per_split;
+  p.kb_per_leaf = pp.kb_per_leaf;
+  p.splits_per_leaf = pp.splits_per_leaf;
   p.bn = pp.bn;
   p.bn_smem = pp.bn_smem;
   p.stages = pp.stages;
@@ -911,16 +936,17 @@ struct DbAux {
   float *part, *part2;
   unsigned int *tickets;
 };
-size_t db_aux_bytes(int rows, int Co) {
-  return align1k((size_t)rows * Co * 4) + align1k((size_t)DB_GROUPS * Co * 4) +
-         align1k((size_t)cdiv(Co, 32) * 4);
+// (leaves: one group-sum slice and one ticket slice per leaf of a leaf plan)
+size_t db_aux_bytes(int rows, int Co, int leaves = 1) {
+  return align1k((size_t)rows * Co * 4) + align1k((size_t)leaves * DB_GROUPS * Co * 4) +
+         align1k((size_t)leaves * cdiv(Co, 32) * 4);
 }
 DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
   DbAux a;
   a.part = reinterpret_cast<float *>(base);
   a.part2 = reinterpret_cast<float *>(base + align1k((size_t)rows * P.d.Co * 4));
   a.tickets = reinterpret_cast<unsigned int *>(base + align1k((size_t)rows * P.d.Co * 4) +
-                                               align1k((size_t)DB_GROUPS * P.d.Co * 4));
+                                               align1k((size_t)P.leaves * DB_GROUPS * P.d.Co * 4));
   return a;
 }
 
@@ -943,7 +969,7 @@ glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, l
   }
   unsigned int *tickets = nullptr;
   if (db_part) tickets = db_aux(P, reinterpret_cast<uint8_t *>(db_part), P.db_rows).tickets;
-  const int nt = (int)cdiv(P.d.Co, 32);
+  const int nt = (int)cdiv(P.d.Co, 32) * P.leaves;   // every leaf's tickets are armed
   if (!P.pack_block) {   // warp-tiled pack (default)
     dim3 gw((unsigned)cdiv(Cw, 32), (unsigned)cdiv((long long)P.d.N * HWd, 8 * PACKW_ROWS));
     if (P.elem == 2) GLP_CUDA(launch_pdl(P.pdl, pack_act_warp<2>, gw, dim3(256), 0, st, src, dst, P.d.N, C, HW, Cp, db_part, tickets, nt, Ws, Wd, HWd, co_off, Cw, db_ld, img_c, 0LL));
@@ -1410,10 +1436,30 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
   return launch_igemm<MODE_WGRAD>(P, pp, p, m, st);
 }
 
-glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw, const BrOut *db, int accumulate,
-                              uint8_t *ws, cudaStream_t st) {
+// leaf_stride > 0 (leaf plans): leaf l's dW / db go to dw / db + l * leaf_stride floats (one
+// reduction per leaf, grid z = leaf); leaf plans called with leaf_stride = 0 reduce into the
+// workspace leaf region and sum the leaves with the fixed tree into dw / db.
+glp_status_t run_tree(const float *const *parts, int n, float *out, size_t count, int accumulate,
+                      cudaStream_t st);
+glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw_in, const BrOut *db_in, int accumulate,
+                              uint8_t *ws, cudaStream_t st, long long leaf_stride = 0) {
   const glp_conv_desc_s &d = P.d;
   float *part = reinterpret_cast<float *>(ws + P.off_part);
+  const int L = P.leaves;
+  BrOut dw = dw_in, dbl;
+  const BrOut *db = db_in;
+  const size_t wsz = (size_t)d.Co * d.C * d.Kh * d.Kw;
+  const bool via_ws = L > 1 && leaf_stride == 0;   // composed call on a leaf plan
+  float *leaf = reinterpret_cast<float *>(ws + P.off_leaf);
+  if (via_ws) {   // leaf l at leaf + l * P.leaf_stride: [dW | db]
+    if (dw_in.n > 1) return fail(GLP_ERR_NOT_SUPPORTED, "leaf plans run single layers");
+    dw = br_out(P, 1, &leaf);
+    float *lb = leaf + wsz;
+    dbl = br_out(P, 1, &lb);
+    if (db_in) db = &dbl;
+    leaf_stride = (long long)P.leaf_stride;
+  }
+  const int acc_red = via_ws ? 0 : accumulate;
   if (P.halo) {
     GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
                         dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32)),
@@ -1422,16 +1468,29 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw, const BrOut *db, i
     GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
   } else
   GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw,
-                      dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32)),
+                      dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32), (unsigned)L),
                       dim3(32, 8), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
                       P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128,
-                      P.wgrad.splits, accumulate, P.s2d, P.dxg.Kw));
+                      P.wgrad.splits / L, acc_red, P.s2d, P.dxg.Kw, leaf_stride));
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
     DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
-    GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), dim3(256), 0,
-                        st, a.part, *db, d.Co, P.db_rows, accumulate, a.part2, a.tickets));
+    GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS, (unsigned)L),
+                        dim3(256), 0, st, a.part, *db, d.Co, P.db_rows / L, acc_red, a.part2,
+                        a.tickets, leaf_stride));
     GLP_LAUNCH_CHECK("reduce_db");
+  }
+  if (via_ws) {   // dW || db = the fixed tree over the leaves (glp_tree_sum order)
+    const float *parts[8];
+    for (int l = 0; l < L; ++l) parts[l] = leaf + (size_t)l * P.leaf_stride;
+    float *out = dw_in.p[0];
+    glp_status_t s = run_tree(parts, L, out, wsz, accumulate, st);
+    if (s) return s;
+    if (db_in) {
+      const float *pb[8];
+      for (int l = 0; l < L; ++l) pb[l] = parts[l] + wsz;
+      if ((s = run_tree(pb, L, db_in->p[0], (size_t)d.Co, accumulate, st))) return s;
+    }
   }
   return GLP_OK;
 }
@@ -1482,6 +1541,69 @@ __global__ void __launch_bounds__(256) pool_sum_slots(const float *__restrict__ 
   }
 }
 
+// ---- deterministic exchange: the fixed binary tree ----
+// Pointer tables by value (kernel parameters): up to 8 leaves / ranks.
+struct Ptr8 {
+  const float *p[8];
+};
+struct MPtr8 {
+  float *p[8];
+};
+
+// out[i] (+)= T(parts[0..n))[i], T = the balanced binary tree over n (a power of two <= 8)
+// operands in index order: level by level, v[k] = v[k] + v[k + w] for k = 0, 2w, ... -- the same
+// fp32 adds, in the same order, as dist.tree_sum over glp_sum2.
+__global__ void __launch_bounds__(256) tree_sum_kernel(const Ptr8 parts, int n, float *out,
+                                                       size_t count, int accumulate) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < count;
+       i += (size_t)gridDim.x * blockDim.x) {
+    float v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = k < n ? __ldg(parts.p[k] + i) : 0.f;
+#pragma unroll
+    for (int w = 1; w < 8; w <<= 1)
+#pragma unroll
+      for (int k = 0; k + w < 8; k += 2 * w)
+        if (k + w < n) v[k] = v[k] + v[k + w];
+    out[i] = accumulate ? out[i] + v[0] : v[0];
+  }
+}
+
+// The top of the tree across ranks over NVLink peer memory (torch symmetric memory): element slice
+// [rank*count/world, (rank+1)*count/world) of T(subtrees[0..world)) -- the rank-ordered subtree
+// sums of every rank, read by peer loads -- is computed by this rank and stored into every rank's
+// output buffer (peer stores), so after a barrier every rank holds the same bits, those of the
+// tree over all leaves.  Plain volatile-free global loads/stores on mapped peer pointers.
+__global__ void __launch_bounds__(256) tree_exchange_kernel(const Ptr8 subtrees, const MPtr8 outs,
+                                                            int world, int rank, size_t count) {
+  const size_t lo = count * (size_t)rank / world, hi = count * (size_t)(rank + 1) / world;
+  for (size_t i = lo + blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < hi;
+       i += (size_t)gridDim.x * blockDim.x) {
+    float v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = k < world ? subtrees.p[k][i] : 0.f;
+#pragma unroll
+    for (int w = 1; w < 8; w <<= 1)
+#pragma unroll
+      for (int k = 0; k + w < 8; k += 2 * w)
+        if (k + w < world) v[k] = v[k] + v[k + w];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (k < world) outs.p[k][i] = v[0];
+  }
+}
+
+glp_status_t run_tree(const float *const *parts, int n, float *out, size_t count, int accumulate,
+                      cudaStream_t st) {
+  if (n < 1 || n > 8 || (n & (n - 1))) return fail(GLP_ERR_INVALID_VALUE, "tree: n must be 1, 2, 4 or 8");
+  if (count == 0) return GLP_OK;
+  Ptr8 t{};
+  for (int k = 0; k < n; ++k) t.p[k] = parts[k];
+  tree_sum_kernel<<<ew_grid(count), 256, 0, st>>>(t, n, out, count, accumulate);
+  GLP_LAUNCH_CHECK("tree_sum_kernel");
+  return GLP_OK;
+}
+
 ConvGeom geomP(const glp_plan_s &P) {
   const glp_conv_desc_s &d = P.d;
   return ConvGeom{d.N, d.C, d.H, d.W, d.Co, d.Kh, d.Kw, d.Sh, d.Sw, d.Ph, d.Pw, d.Ho, d.Wo,
@@ -1505,7 +1627,7 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
     GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
     float *dbs[1] = {db};
     reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), 256, 0, st>>>(
-        a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets);
+        a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets, 0LL);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;
@@ -1652,7 +1774,7 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
 
 glp_status_t glp_plan_options_default(glp_plan_options_t *o) {
   if (!o) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
-  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 2, 1, 0, 0, 232448, 0};
+  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 2, 1, 0, 0, 232448, 0, 0};
   return GLP_OK;
 }
 
@@ -1669,8 +1791,11 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
   if (o.halo_dgrad < 0 || o.halo_dgrad > 2 || o.fused_dy_builders < 0 || o.fused_dy_builders > 3 ||
       o.max_kblocks_per_stage < 1 || o.max_kblocks_per_stage > 4 || o.wgrad_tile_n < 0 ||
       o.wgrad_tile_n > 256 || o.wgrad_tile_n % 16 || o.tile_units < 0 || o.smem_cap < 65536 ||
-      o.smem_cap > 232448)
+      o.smem_cap > 232448 || (o.wgrad_leaves != 0 && o.wgrad_leaves != 1 && o.wgrad_leaves != 2 &&
+                              o.wgrad_leaves != 4 && o.wgrad_leaves != 8))
     return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
+  if (o.wgrad_leaves > 0 && (math == GLP_MATH_FP32_SIMT || d->nbr > 1))
+    return fail(GLP_ERR_NOT_SUPPORTED, "wgrad leaves: tensor-core single-layer plans only");
   *out = nullptr;
   if (math != GLP_MATH_FP32 && math != GLP_MATH_TF32 && math != GLP_MATH_BF16 &&
       math != GLP_MATH_FP32_SIMT)
@@ -1729,6 +1854,12 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
   P->pack_block = o.pack_block != 0;
   P->s2d_block = o.s2d_block != 0;
   P->smem_cap = o.smem_cap;
+  P->leaves = std::max(1, o.wgrad_leaves);
+  P->leaf_plan = o.wgrad_leaves > 0 ? 1 : 0;
+  if (P->leaf_plan) {   // leaf plans use the im2col filter gradient and the warp-tiled dy pack
+    P->allow_halo = 0;
+    P->pack_block = 0;
+  }
 #ifdef GLP_DIAG
   // diagnostic builds only (never the shipped library): GLP_DEBUG_CLK = device address of
   // >= 4 * grid uint64 counters (tools/clk_probe.py); GLP_DEBUG_SKIP = work-skipping bits
@@ -1825,7 +1956,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = (int)cdiv((long long)c.N * dy_hw, P->pack_block ? PACK_PT : PACKW_ROWS);
     if (P->halo_fdy) P->db_rows = P->hw.splits;   // one db partial per filter-gradient CTA
-    P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co);
+    P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co, P->leaves);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;
     P->off_dypk = P->sz_xpk;
@@ -1835,7 +1966,12 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
     P->off_dbpart = P->off_part + P->sz_part;
     P->ws_fwd = P->off_wpk + P->sz_wpk;
     P->ws_dgrad = P->off_wtpk + P->sz_wtpk;
-    P->ws_wgrad = P->off_dbpart + P->sz_dbpart;
+    if (P->leaves > 1) {   // leaf partials [dW | db] of the composed calls (summed by the tree)
+      P->leaf_stride = (size_t)rup((long long)c.Co * c.C * c.Kh * c.Kw + c.Co, 4);
+      P->sz_leaf = align1k((size_t)P->leaves * P->leaf_stride * 4);
+    }
+    P->off_leaf = P->off_dbpart + P->sz_dbpart;
+    P->ws_wgrad = P->off_leaf + P->sz_leaf;
     P->ws_bwd = P->ws_wgrad;
     // Samples in flight (the paper's C_out, Eq. 9 re-derived, R18) through the analyzer: the
     // forward kernel's resident rows (#SM x CTAs/SM x 128 GEMM rows) over the rows a sample
@@ -2322,6 +2458,48 @@ glp_status_t glp_sum2(const float *a, const float *b, float *out, size_t n, glp_
   sum2_kernel<<<ew_grid(n), 256, 0, st>>>(a, b, out, n);
   GLP_LAUNCH_CHECK("sum2_kernel");
   return GLP_OK;
+}
+
+glp_status_t glp_tree_sum(const float *const *parts, int n, float *out, size_t count,
+                          int accumulate, glp_stream_t stream) {
+  if (!parts || !out) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  for (int k = 0; k < n && k < 8; ++k)
+    if (!parts[k]) return fail(GLP_ERR_INVALID_VALUE, "NULL tree operand");
+  return run_tree(parts, n, out, count, accumulate ? 1 : 0, static_cast<cudaStream_t>(stream));
+}
+
+glp_status_t glp_tree_exchange(const float *const *subtrees, float *const *outs, int world, int rank,
+                               size_t count, glp_stream_t stream) {
+  if (!subtrees || !outs) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
+  if (world < 1 || world > 8 || (world & (world - 1)) || rank < 0 || rank >= world)
+    return fail(GLP_ERR_INVALID_VALUE, "world must be 1, 2, 4 or 8 and 0 <= rank < world");
+  Ptr8 a{};
+  MPtr8 b{};
+  for (int k = 0; k < world; ++k) {
+    if (!subtrees[k] || !outs[k]) return fail(GLP_ERR_INVALID_VALUE, "NULL peer pointer");
+    a.p[k] = subtrees[k];
+    b.p[k] = outs[k];
+  }
+  if (count == 0) return GLP_OK;
+  const size_t mine = count / world + 1;
+  tree_exchange_kernel<<<ew_grid(mine), 256, 0, static_cast<cudaStream_t>(stream)>>>(a, b, world, rank, count);
+  GLP_LAUNCH_CHECK("tree_exchange_kernel");
+  return GLP_OK;
+}
+
+glp_status_t glp_stage_reduce_leaves(glp_plan_t P, float *dw, float *db, size_t leaf_stride,
+                                     void *ws, size_t ws_bytes, glp_stream_t stream) {
+  glp_status_t s = stage_check(P, ws, ws_bytes);
+  if (s) return s;
+  if ((s = validate_ptrs({dw}))) return s;
+  if (P->leaves < 2 && leaf_stride == 0) leaf_stride = 1;   // one leaf: the stride is unused
+  if (leaf_stride == 0 || leaf_stride % 4)
+    return fail(GLP_ERR_INVALID_VALUE, "leaf_stride must be a positive multiple of 4 floats");
+  if (P->groups > 1) return fail(GLP_ERR_NOT_SUPPORTED, "leaf reduction of a grouped layer");
+  float *dwp = dw;
+  const BrOut dbt = br_out(*P, 1, &db);
+  return run_wgrad_reduce(*P, br_out(*P, 1, &dwp), db ? &dbt : nullptr, 0, static_cast<uint8_t *>(ws),
+                          static_cast<cudaStream_t>(stream), (long long)leaf_stride);
 }
 
 // ---- prior-art comparator: the paper's per-sample stream pool ----

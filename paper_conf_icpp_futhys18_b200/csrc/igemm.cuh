@@ -69,6 +69,21 @@ __device__ __forceinline__ void ring_next(int &s, uint32_t &ph, int S) {
   }
 }
 
+// k-block range [kb0, kb1) of filter-gradient split `split`.  Leaf plans (p.splits_per_leaf > 0,
+// the deterministic exchange): the pixel range is cut into leaves of p.kb_per_leaf k-blocks and
+// each leaf into p.splits_per_leaf splits that never cross a leaf boundary, so every leaf's split
+// partials are the same bits whichever rank (and local batch) computes the leaf.
+__device__ __forceinline__ void wgrad_kb_range(const IgemmParams &p, int split, int &kb0, int &kb1) {
+  if (p.splits_per_leaf > 0) {
+    const int leaf = split / p.splits_per_leaf, j = split - leaf * p.splits_per_leaf;
+    kb0 = leaf * p.kb_per_leaf + j * p.kb_per_split;
+    kb1 = min(kb0 + p.kb_per_split, (leaf + 1) * p.kb_per_leaf);
+  } else {
+    kb0 = split * p.kb_per_split;
+    kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+  }
+}
+
 __device__ __forceinline__ void decode_tile(int t, int n_tiles, int m_tiles, int &m_tile,
                                             int &n_tile, int &split) {
   n_tile = t % n_tiles;
@@ -218,8 +233,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
           const int nb0 = n0 + (int)rank * p.bn_smem;   // this CTA's part of the B tile
           int kb0 = 0, kb1 = p.kb_total;
           if (MODE == MODE_WGRAD) {
-            kb0 = split * p.kb_per_split;
-            kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+            wgrad_kb_range(p, split, kb0, kb1);
           }
           // per-tile geometry of the A gather
           uint32_t n_t = 0;
@@ -358,8 +372,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
         int kb0 = 0, kb1 = p.kb_total;
         if (MODE == MODE_WGRAD) {
-          kb0 = split * p.kb_per_split;
-          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+          wgrad_kb_range(p, split, kb0, kb1);
         }
         const int m0 = m_tile * C::BM, n0 = n_tile * p.bn;
         if (MODE != MODE_WGRAD) {
@@ -536,8 +549,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
           decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
           int kb0 = 0, kb1 = kb_total;
           if (MODE == MODE_WGRAD) {
-            kb0 = split * kb_per_split;
-            kb1 = min(kb0 + kb_per_split, kb_total);
+            wgrad_kb_range(p, split, kb0, kb1);
           }
           uint32_t acc = 0, d = tmem_base, cur = 0;
           int next_chunk = kb0;   // first k-block of the next chunk
@@ -581,8 +593,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
         int kb0 = 0, kb1 = kb_total;
         if (MODE == MODE_WGRAD) {
-          kb0 = split * kb_per_split;
-          kb1 = min(kb0 + kb_per_split, kb_total);
+          wgrad_kb_range(p, split, kb0, kb1);
         }
         const uint32_t a = it & 1u, aph = (it >> 1) & 1u;
         long long c0 = clk ? clock64() : 0;
@@ -666,8 +677,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
         decode_tile(tile, p.n_tiles, p.m_tiles, m_tile, n_tile, split);
         int kb0 = 0, kb1 = p.kb_total;
         if (MODE == MODE_WGRAD) {
-          kb0 = split * p.kb_per_split;
-          kb1 = min(kb0 + p.kb_per_split, p.kb_total);
+          wgrad_kb_range(p, split, kb0, kb1);
         }
         const int nch = (kb1 - kb0 + CK - 1) / CK;
         for (int ch = 0; ch < nch; ++ch, ++gch) {

@@ -164,14 +164,17 @@ __global__ void reduce_simt_dw(const float *__restrict__ part, float *__restrict
 // Block (32, 8) per tile of 32 output channels x 32 inner dW indices (i = ci*taps + t): warps read
 // 32 consecutive co of one partial row per split (coalesced), the tile is transposed through
 // shared memory, and dW[co][i] is written 32 consecutive i at a time.  grid (ceil(C*taps/32),
-// ceil(Co/32)).
+// ceil(Co/32), leaves).  Leaf plans (the deterministic exchange): blockIdx.z = leaf, `splits` are
+// that leaf's splits (partials leaf*splits ...), and its dW goes leaf_stride floats further.
 __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ part,
                                                     const BrOut dw, int Co, int C,
                                                     int taps, int Kw, int Cp, int ld, int mpad,
-                                                    int splits, int accumulate, int s2d, int Ks) {
+                                                    int splits, int accumulate, int s2d, int Ks,
+                                                    long long leaf_stride) {
   __shared__ float tile[32][33];
   pdl_launch_dependents();
   pdl_wait();
+  part += (size_t)blockIdx.z * splits * ((size_t)mpad * ld);
   const int inner = C * taps;
   const int i0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
   const int lane = threadIdx.x, ty = threadIdx.y;
@@ -220,7 +223,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
   for (int j = ty; j < 32; j += 8) {
     const int co = co0 + j, i = i0 + lane;
     if (co < Co && i < inner) {
-      float *d = dw.at(co, 0, (size_t)inner, (size_t)i);
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + blockIdx.z * leaf_stride;
       const float v = tile[lane][j];
       *d = accumulate ? *d + v : v;
     }
@@ -288,14 +291,20 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
 // the last block to finish for a channel group (atomic ticket) sums part2[0..G) in index order.
 // The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
 constexpr int DB_GROUPS = 128;   // multiple of 4
+// Leaf plans: blockIdx.z = leaf; its `rows` partial rows follow the previous leaves', its group sums
+// and tickets have their own slices, and its db goes leaf_stride floats further.
 __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
                                                  const BrOut db, int Co, int rows,
                                                  int accumulate, float *__restrict__ part2,
-                                                 unsigned int *__restrict__ tickets) {
+                                                 unsigned int *__restrict__ tickets,
+                                                 long long leaf_stride) {
   __shared__ float red[8][33];
   __shared__ bool last;
   pdl_launch_dependents();
   pdl_wait();
+  part += (size_t)blockIdx.z * rows * Co;
+  part2 += (size_t)blockIdx.z * DB_GROUPS * Co;
+  tickets += (size_t)blockIdx.z * gridDim.x;
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
   const int co = blockIdx.x * 32 + lane, g = blockIdx.y;
   // rows g + DB_GROUPS*(ty + 8*j), j = 0, 1, ...: four interleaved accumulators (j mod 4) keep
@@ -342,7 +351,7 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
         s3 += __ldcg(part2 + (size_t)(k + 3) * Co + co);
       }
       const float s = (s0 + s1) + (s2 + s3);
-      float *d = db.at(co, 0, 1, 0);
+      float *d = db.at(co, 0, 1, 0) + blockIdx.z * leaf_stride;
       *d = accumulate ? *d + s : s;
     }
     if (lane == 0) tickets[blockIdx.x] = 0;   // re-arm for the next call on this workspace

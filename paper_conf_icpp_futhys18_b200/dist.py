@@ -152,3 +152,60 @@ class TreeAllreduce:
                 self.add(recv, acc, acc)
             d <<= 1
         return acc
+
+
+class LeafTreeExchange:
+    """The deterministic gradient exchange as the library runs it (P264
+    convergence invariance extended across GPU counts):
+
+      1. the filter gradient of a leaf plan (glp_plan_options_t.wgrad_leaves = this rank's leaves)
+         reduces its split partials per leaf into `leaves` ([L, numel], one flat dW||db buffer per
+         leaf; glp_stage_reduce_leaves) -- the step packs x and dy once, only the reduction is split;
+      2. glp_tree_sum sums the rank's leaves with its subtree of the fixed 8-leaf binary tree;
+      3. world > 1: the top levels across ranks -- over torch symmetric memory, glp_tree_exchange
+         (each rank computes a slice of the top tree with NVLink peer loads and stores it into every
+         rank's buffer, between two symmetric-memory barriers), or, without symmetric memory,
+         recursive doubling over torch.distributed point-to-point (TreeAllreduce).
+    Every fp32 add is a node of the same tree, so the result is bitwise identical for 1, 2, 4 and
+    8 ranks."""
+
+    def __init__(self, numel, n_local_leaves, device, group=None, transport="auto"):
+        import torch
+        import torch.distributed as dist
+        self.numel, self.L, self.group = int(numel), int(n_local_leaves), group
+        self.leaves = torch.zeros(self.L, self.numel, device=device)
+        self.world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if self.world > 1 else 0
+        self.transport = "local"
+        if self.world > 1:
+            self.transport = "p2p"
+            if transport in ("auto", "symm") and torch.device(device).type == "cuda":
+                try:
+                    import torch.distributed._symmetric_memory as symm
+                    name = (group or dist.group.WORLD).group_name
+                    self.sub = symm.empty(self.numel, device=device)
+                    self.out = symm.empty(self.numel, device=device)
+                    self.hs = symm.rendezvous(self.sub, name)
+                    self.ho = symm.rendezvous(self.out, name)
+                    self.transport = "symm"
+                except Exception:
+                    if transport == "symm":
+                        raise
+        if self.transport != "symm":
+            self.sub = torch.empty(self.numel, device=device)
+
+    def __call__(self, flat):
+        """flat <- the tree over every rank's leaves (all ranks get the same bits)."""
+        from . import tree_sum
+        tree_sum([self.leaves[l] for l in range(self.L)], self.sub)
+        if self.transport == "local":
+            flat.copy_(self.sub)
+        elif self.transport == "symm":
+            from . import tree_exchange
+            self.hs.barrier(channel=0)
+            tree_exchange(self.hs.buffer_ptrs, self.ho.buffer_ptrs, self.rank, self.numel)
+            self.ho.barrier(channel=0)
+            flat.copy_(self.out)
+        else:
+            flat.copy_(TreeAllreduce(self.group)([self.sub]))
+        return flat

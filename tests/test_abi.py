@@ -129,7 +129,7 @@ def test_plan_options_abi():
     assert L.glp_conv_desc_create(ctypes.byref(d), 2, 3, 8, 8, 4, 3, 3, 1, 1, 1, 1) == 0
     p = ctypes.c_void_p()
     for bad in ({"halo_dgrad": 3}, {"max_kblocks_per_stage": 0}, {"wgrad_tile_n": 24},
-                {"smem_cap": 1000}):
+                {"smem_cap": 1000}, {"wgrad_leaves": 3}):
         ob = glp.plan_options(**bad)
         assert L.glp_plan_ex(ctypes.byref(p), d, 0, glp.GLP_MATH_BF16, 0, ctypes.byref(ob)) == 1
     with pytest.raises(ValueError):

@@ -585,40 +585,78 @@ def test_grouped_conv(shape, math):
             np.testing.assert_array_equal(v.cpu().numpy(), got[k], err_msg="staged " + k)
 
 
-def test_tree_exchange_bitwise_invariant_emulated_ranks():
-    """Deterministic gradient exchange (NEXT-2) on the device: leaf filter gradients from the same
-    leaf plan, the rank-local subtrees and the cross-rank levels all summed by glp_sum2, give
-    bitwise the same dW and db for 1, 2, 4 and 8 (emulated) ranks; exact on integer data."""
-    from paper_conf_icpp_futhys18_b200.dist import LEAVES, leaf_range, rank_leaves, tree_sum
-    N, C, H, W, Co, K, S, P = 16, 24, 13, 13, 40, 3, 1, 1
+@pytest.mark.parametrize("math", ["fp32", "tf32", "bf16"])
+def test_tree_exchange_bitwise_invariant_emulated_ranks(math):
+    """Deterministic gradient exchange (NEXT-2) as the library runs it, with 1, 2, 4 and 8 ranks
+    emulated on one device: each rank plans its local batch as 8/world leaves (wgrad_leaves),
+    packs x and dy ONCE, runs one filter-gradient GEMM whose splits never cross a leaf, reduces
+    per leaf (glp_stage_reduce_leaves), sums its leaves with glp_tree_sum (its subtree of the
+    8-leaf tree), and glp_tree_exchange -- called once per emulated rank with every rank's
+    buffers as the "peer" pointers -- completes the top of the tree into every rank's output.
+    dW||db is bitwise the same for every world size and every rank, equal to the composed
+    glp_conv_bwd_filter of the 8-leaf plan, within the bar of the oracle, exact on integers."""
+    from paper_conf_icpp_futhys18_b200.dist import LEAVES, rank_leaves
+    N, C, H, W, Co, K, S, P = 16, 24, 8, 8, 40, 3, 1, 1   # leaf = 2 images x 64 pixels
     Ho = oracle.out_dim(H, K, S, P)
-    add = lambda a, b, o: glp.sum2(a, b, o)
+    wsz = Co * C * K * K
+    numel = (wsz + Co + 3) // 4 * 4
     for exact, seed in ((False, 81), (True, 82)):
         d = gen_custom(N, C, H, W, Co, K, K, seed, exact=exact, Ho=Ho, Wo=Ho)
         t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
-        leaf = glp.ConvLayer(N // LEAVES, C, H, W, Co, K, S, P, math="bf16")
-        parts = []
-        for j in range(LEAVES):
-            a, b = leaf_range(N, j)
-            buf = torch.empty(Co * C * K * K + Co, device=DEV)
-            leaf.bwd_filter(t["x"][a:b].contiguous(), t["dy"][a:b].contiguous(),
-                            buf[:Co * C * K * K].view(Co, C, K, K), buf[Co * C * K * K:])
-            parts.append(buf)
         results = []
         for world in (1, 2, 4, 8):
-            subtrees = [tree_sum([parts[j] for j in rank_leaves(r, world)], add) for r in range(world)]
-            results.append(tree_sum(subtrees, add) if world > 1 else subtrees[0])
-        torch.cuda.synchronize()
-        ref = results[0].cpu().numpy()
+            nl = N // world
+            subs, outs = [], []
+            for r in range(world):
+                L = len(rank_leaves(r, world))
+                layer = glp.ConvLayer(nl, C, H, W, Co, K, S, P, math=math,
+                                      options={"wgrad_leaves": L})
+                leaves = torch.zeros(L, numel, device=DEV)
+                flat = leaves.view(-1)
+                layer.stage_pack(glp.GLP_PACK_X, t["x"][r * nl:(r + 1) * nl].contiguous())
+                layer.stage_pack(glp.GLP_PACK_DY_DB, t["dy"][r * nl:(r + 1) * nl].contiguous())
+                layer.stage_bwd_filter()
+                layer.stage_reduce_leaves(flat, flat[wsz:], numel)
+                sub = torch.empty(numel, device=DEV)
+                glp.tree_sum([leaves[l] for l in range(L)], sub)
+                subs.append(sub)
+                outs.append(torch.full((numel,), float("nan"), device=DEV))
+            for r in range(world):
+                glp.tree_exchange([x.data_ptr() for x in subs], [o.data_ptr() for o in outs], r, numel)
+            torch.cuda.synchronize()
+            for o in outs[1:]:
+                np.testing.assert_array_equal(o.cpu().numpy(), outs[0].cpu().numpy())
+            results.append(outs[0].cpu().numpy())
         for r in results[1:]:
-            np.testing.assert_array_equal(r.cpu().numpy(), ref)
-        dw, _ = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, S, P)
-        db = d["dy"].astype(np.float64).sum(axis=(0, 2, 3))
-        full = np.concatenate([dw.ravel(), db])
+            np.testing.assert_array_equal(r, results[0])
+        # the composed call of the 8-leaf plan (leaves reduced in the workspace, the same tree)
+        layer = glp.ConvLayer(N, C, H, W, Co, K, S, P, math=math, options={"wgrad_leaves": LEAVES})
+        dw = torch.empty(layer.w_shape, device=DEV)
+        db = torch.empty(Co, device=DEV)
+        layer.bwd_filter(t["x"], t["dy"], dw, db)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(dw.cpu().numpy().ravel(), results[0][:wsz])
+        np.testing.assert_array_equal(db.cpu().numpy(), results[0][wsz:wsz + Co])
+        rdw, rdb = oracle.conv_bwd_filter(d["x"], d["dy"], d["w"].shape, S, P)
+        full = np.concatenate([rdw.ravel(), rdb])
         if exact:
-            np.testing.assert_array_equal(ref, full.astype(np.float32))
+            np.testing.assert_array_equal(results[0][:wsz + Co], full.astype(np.float32))
         else:
-            assert np.abs(ref - full).max() / np.abs(full).max() <= TOL["bf16"]
+            assert oracle.normwise_err(results[0][:wsz + Co], full) <= TOL[math]
+
+
+def test_tree_sum_matches_sum2_tree():
+    """glp_tree_sum (one launch) is bitwise the dist.tree_sum of glp_sum2 adds, for 1-8 parts."""
+    from paper_conf_icpp_futhys18_b200.dist import tree_sum
+    g = torch.Generator(device="cpu").manual_seed(5)
+    for n in (1, 2, 4, 8):
+        parts = [(torch.randn(5003, generator=g) * 10.0 ** torch.empty(5003).uniform_(-6, 6,
+                  generator=g)).to(DEV) for _ in range(n)]
+        ref = tree_sum(parts, lambda a, b, o: glp.sum2(a, b, o))
+        out = torch.empty_like(parts[0])
+        glp.tree_sum(parts, out)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(out.cpu().numpy(), ref.cpu().numpy())
 
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])

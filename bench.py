@@ -69,6 +69,11 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-extra-modes", action="store_true",
                    help="skip the bf16 / tf32 lines measured beside the fp32 headline (1 GPU)")
+    p.add_argument("--dist-backend", choices=["nccl", "gloo"], default="nccl",
+                   help="(tests) process-group backend; gloo + --same-device runs the N-rank step "
+                        "on one GPU to exercise the multi-rank code path (timings meaningless)")
+    p.add_argument("--same-device", action="store_true",
+                   help="(tests) every rank on cuda:0 instead of cuda:LOCAL_RANK")
     p.add_argument("--dry-run", action="store_true",
                    help="(tests) launcher plumbing only: start the ranks, form a gloo process group "
                         "on CPU, all-reduce one tensor and print the line's n_gpus; no GPU work")
@@ -774,14 +779,17 @@ def run_glp(args, ws, rank, local):
     import torch
     import torch.distributed as dist
 
-    dev = torch.device("cuda", local)
+    dev = torch.device("cuda", 0 if args.same_device else local)
     torch.cuda.set_device(dev)
     G = ws
     if G > 1:
-        # the NCCL communicator lines (ring/tree/NVLS choice over NVLink) go to stderr
-        os.environ.setdefault("NCCL_DEBUG", "INFO")
-        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            # the NCCL communicator lines (ring/tree/NVLS choice over NVLink) go to stderr
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     from paper_conf_icpp_futhys18_b200.dist import FlatGrads
     layers = config(args.workload)
     grads = FlatGrads([l.w_shape for l in layers], device=dev)
@@ -833,7 +841,7 @@ def run_glp(args, ws, rank, local):
     else:
         def run_one():
             step(concurrent=not args.serial)
-    clocks = ClockSampler(local) if rank == 0 else None
+    clocks = ClockSampler(dev.index) if rank == 0 else None
     if clocks:
         clocks.start()
     if G > 1:
@@ -865,8 +873,13 @@ def run_glp(args, ws, rank, local):
             avg = sum(us) / len(us)
             kern.append({"layer": s.name, "pass": name, "avg_us": round(avg, 2),
                          "total_us": sum(us), "tflops": round(s.flops / (avg * 1e-6) / 1e12, 1)})
-    if args.dump and rank == 0:
-        dump_units(states, args.dump, args.workload, args.math)
+    if args.dump:
+        # one more full step (with the exchange): the attribution steps above skip it, so dW || db
+        # would hold this rank's unreduced gradients
+        step()
+        torch.cuda.synchronize()
+        if rank == 0:
+            dump_units(states, args.dump, args.workload, args.math)
     roofline = make_roofline(args, states, kern, ms_per_step)
     step_flops = sum(s.flops * (3 if s.dx is not None else 2) for s in states)
 
@@ -1146,7 +1159,7 @@ def main():
         dry_run(ws, rank)
         return
     import torch
-    if torch.cuda.device_count() < (local + 1):
+    if torch.cuda.device_count() < (1 if args.same_device else local + 1):
         sys.exit(f"bench.py: rank {rank} needs cuda:{local} but {torch.cuda.device_count()} "
                  "CUDA device(s) are visible (there is no CPU fallback)")
     if args.scheme == "pool":

@@ -289,7 +289,11 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
     const int real = (int)cdiv(kb_total, kbps);
     if (real != s) continue;
     const double waves = std::ceil(tiles_mn * (double)s * leaves / sm);
-    const double t = waves * (kbps * kb_s + 2e-6) + (double)s * leaves * mpad * npad * 8.0 / bw;
+    // + the fixed-order reduction: each output sums its s partials in dependent batches of 8
+    // loads (~1.2 us per batch when the reduction grid is too small to hide the latency: tiny
+    // layers with many splits spent 75 us in reduce_tc_dw at s = 512)
+    const double red = (double)mpad * npad < 148.0 * 1024 ? std::ceil(s / 8.0) * 1.2e-6 : 0.0;
+    const double t = waves * (kbps * kb_s + 2e-6) + (double)s * leaves * mpad * npad * 8.0 / bw + red;
     if (t < best_t * 0.999) {
       best_t = t;
       best = s;

@@ -134,6 +134,13 @@ class TreeAllreduce:
         acc = tree_sum(parts, self.add)
         if not (dist.is_available() and dist.is_initialized()):
             return acc
+        if acc.is_cuda and dist.get_backend(self.group) == "gloo":
+            # gloo moves host memory only: run the exchange on a host copy (IEEE fp32 adds are
+            # correctly rounded on both sides, so the bits are those of the device adds)
+            dev = acc.device
+            out = TreeAllreduce(self.group, add=lambda a, b, o: __import__("torch").add(a, b, out=o))(
+                [acc.cpu()])
+            return out.to(dev)
         world = dist.get_world_size(self.group)
         rank = dist.get_rank(self.group)   # rank within the group
         recv = acc.clone()

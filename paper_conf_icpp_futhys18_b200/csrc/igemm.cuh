@@ -527,7 +527,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
       }
       const uint64_t stage16 = stage_bytes >> 4, b16 = b_bytes >> 4;
       const uint64_t alo16 = A_BYTES1 >> 4, blo16 = b_bytes1 >> 4;   // lo planes (X3)
-      const int KS = p.ksub, kb_total = p.kb_total, kb_per_split = p.kb_per_split;
+      const int KS = p.ksub, kb_total = p.kb_total;
       const bool skip_mma = GLP_SKIP(p, 4);
       int rs = 0;
       uint32_t rph = 0, it = 0;

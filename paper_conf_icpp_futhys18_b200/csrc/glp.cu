@@ -1479,7 +1479,7 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw_in, const BrOut *db
   GLP_LAUNCH_CHECK("reduce_tc_dw");
   if (db) {
     DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
-    GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS, (unsigned)L),
+    GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), (unsigned)db_groups(P.db_rows / L), (unsigned)L),
                         dim3(256), 0, st, a.part, *db, d.Co, P.db_rows / L, acc_red, a.part2,
                         a.tickets, leaf_stride));
     GLP_LAUNCH_CHECK("reduce_db");
@@ -1630,7 +1630,7 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
     DbAux a = db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.simt_splits);
     GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
     float *dbs[1] = {db};
-    reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), DB_GROUPS), 256, 0, st>>>(
+    reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), (unsigned)db_groups(P.simt_splits)), 256, 0, st>>>(
         a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets, 0LL);
     GLP_LAUNCH_CHECK("reduce_db");
   }

@@ -290,7 +290,14 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
 // those, lanes = channels, coalesced), reduces its 8 warps in a fixed tree, and stores part2[g][co];
 // the last block to finish for a channel group (atomic ticket) sums part2[0..G) in index order.
 // The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
-constexpr int DB_GROUPS = 128;   // multiple of 4
+constexpr int DB_GROUPS = 128;   // the largest group count (multiple of 4)
+// Row groups of a db reduction over `rows` partial rows: ~32 rows per group, 4..DB_GROUPS, a
+// multiple of 4 -- a function of the row count only (small layers spent ~10 us in 128 nearly
+// empty groups plus the ticket pass).
+__host__ __device__ constexpr int db_groups(int rows) {
+  const int g = ((rows + 31) / 32 + 3) / 4 * 4;
+  return g < 4 ? 4 : (g > DB_GROUPS ? DB_GROUPS : g);
+}
 // Leaf plans: blockIdx.z = leaf; its `rows` partial rows follow the previous leaves', its group sums
 // and tickets have their own slices, and its db goes leaf_stride floats further.
 __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
@@ -303,6 +310,7 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
   pdl_launch_dependents();
   pdl_wait();
   part += (size_t)blockIdx.z * rows * Co;
+  const int G = gridDim.y;   // db_groups(rows), set by the launch
   part2 += (size_t)blockIdx.z * DB_GROUPS * Co;
   tickets += (size_t)blockIdx.z * gridDim.x;
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
@@ -312,9 +320,9 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
   // conv1), the tail goes to a0, then ((a0+a1)+(a2+a3)) — an order fixed by `rows` alone
   float a = 0.f;
   if (co < Co) {
-    constexpr int STEP = DB_GROUPS * 8;
+    const int STEP = G * 8;
     float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
-    int r = g + DB_GROUPS * ty;
+    int r = g + G * ty;
     const float *pc = part + co;
     for (; r + 3 * STEP < rows; r += 4 * STEP) {
       const float v0 = __ldg(pc + (size_t)r * Co), v1 = __ldg(pc + (size_t)(r + STEP) * Co);
@@ -336,7 +344,7 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
     __threadfence();
   }
   __syncthreads();
-  if (threadIdx.x == 0) last = (atomicAdd(tickets + blockIdx.x, 1u) == DB_GROUPS - 1);
+  if (threadIdx.x == 0) last = (atomicAdd(tickets + blockIdx.x, 1u) == (unsigned)G - 1);
   __syncthreads();
   if (last && ty == 0) {
     __threadfence();
@@ -344,7 +352,7 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
       // group sums in index order, four strided accumulators (k mod 4), then combined in order
       float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
 #pragma unroll 4
-      for (int k = 0; k < DB_GROUPS; k += 4) {
+      for (int k = 0; k < G; k += 4) {
         s0 += __ldcg(part2 + (size_t)k * Co + co);
         s1 += __ldcg(part2 + (size_t)(k + 1) * Co + co);
         s2 += __ldcg(part2 + (size_t)(k + 2) * Co + co);

@@ -719,13 +719,26 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
           const int lim = min(c_hi, p.N - n0) - c_lo;
           const uint32_t sb = sbias + 4u * (uint32_t)(n0 + c_lo);
           if (MODE == MODE_FWD && p.ybr.n > 1) {   // fused sibling group: per-branch tensors
+            // one branch lookup per 32-column chunk (a chunk straddling two branches, at most one
+            // per branch boundary, takes the per-element lookup)
 #pragma unroll
-            for (int j = 0; j < 4; ++j)
+            for (int j = 0; j < 4; ++j) {
+              if (32 * j >= lim) continue;
+              const int cf = n0 + c_lo + 32 * j, lj = min(32, lim - 32 * j);
+              if (p.ybr.branch(cf) == p.ybr.branch(cf + lj - 1)) {
+                float *o = p.ybr.at(cf, n, plane, pimg);
 #pragma unroll
-              for (int i = 0; i < 32; ++i)
-                if (32 * j + i < lim)
-                  *p.ybr.at(n0 + c_lo + 32 * j + i, n, plane, pimg) =
-                      S[32 * j + i] + lds_f32(sb + 4u * (uint32_t)(32 * j + i));
+                for (int i = 0; i < 32; ++i) {
+                  if (i < lj) o[0] = S[32 * j + i] + lds_f32(sb + 4u * (uint32_t)(32 * j + i));
+                  o += plane;
+                }
+              } else {
+#pragma unroll
+                for (int i = 0; i < 32; ++i)
+                  if (i < lj)
+                    *p.ybr.at(cf + i, n, plane, pimg) = S[32 * j + i] + lds_f32(sb + 4u * (uint32_t)(32 * j + i));
+              }
+            }
           } else {
             float *o = p.out + (size_t)n * p.out_c * plane + pimg + (size_t)(n0 + c_lo) * plane;
 #pragma unroll

@@ -8,7 +8,7 @@ namespace glp {
 struct FastDiv {
   uint32_t d, mul, shr;
   __host__ __device__ FastDiv() : d(1), mul(0), shr(0) {}
-  __host__ explicit FastDiv(uint32_t div) : d(div) {
+  __host__ __device__ explicit FastDiv(uint32_t div) : d(div) {
     uint32_t l = 0;
     while ((1ull << l) < div) ++l;
     shr = l;

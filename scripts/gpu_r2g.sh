@@ -1,0 +1,6 @@
+cd "$(dirname "$0")/.."
+WORKLOADS="1 2 3 5" STEPS=30 bash scripts/gpu_workloads.sh > /dev/null 2>&1
+timeout -s KILL 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file gpurun_out/launch_small_1.csv python bench.py --steps 1 --warmup 1 --workload 1 --math fp32 --no-cpu-baseline --no-e2e --no-graph --serial --no-extra-modes > /dev/null 2>&1
+timeout -s KILL 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file gpurun_out/launch_small_3.csv python bench.py --steps 1 --warmup 1 --workload 3 --math fp32 --no-cpu-baseline --no-e2e --no-graph --serial --no-extra-modes > /dev/null 2>&1

@@ -358,6 +358,7 @@ struct glp_plan_s {
   // halo forward (hfwd.cuh) for the same space-to-depth layers: x' staged once per tile for all
   // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
   int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
+  int red_wide = 0;     // dW reduction by reduce_tc_dw_wide (small filters, many splits)
   int hdg = 0;         // halo backward-data (hdgrad.cuh) for unit-stride layers where it pays
   HdgradParams hd{};
   int hd_grid = 0, hd_smem = 0;
@@ -1468,7 +1469,14 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw_in, const BrOut *db
     GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
                         dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32)),
                         dim3(256), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx, P.hw.ld,
-                        P.hw.mpad, P.hw.splits, accumulate, P.s2d, P.dxg.Kw));
+                        P.hw.mpad, P.hw.splits, accumulate, P.s2d, P.dxg.Kw, 0LL));
+    GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
+  } else if (P.red_wide) {   // small filter: 4 weight rows per block, splits over 8 phases
+    GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
+                        dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32), (unsigned)L),
+                        dim3(256), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
+                        P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128,
+                        P.wgrad.splits / L, acc_red, P.s2d, P.dxg.Kw, leaf_stride));
     GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
   } else
   GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw,
@@ -1960,6 +1968,12 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
                                    P->wgrad.n_tiles * P->wgrad.bn * 4);
     P->db_rows = (int)cdiv((long long)c.N * dy_hw, P->pack_block ? PACK_PT : PACKW_ROWS);
     if (P->halo_fdy) P->db_rows = P->hw.splits;   // one db partial per filter-gradient CTA
+    // dW reduction kernel (shape-only): filters whose 32 x 32 reduction tiles number < 64 take
+    // the 4-row x 8-phase variant (8x the blocks; LeNet conv1: 1 block -> 7)
+    if (!P->halo) {
+      const long long tiles32 = cdiv((long long)c.C * P->taps, 32) * cdiv(c.Co, 32);
+      P->red_wide = tiles32 < 64 && P->wgrad.splits / std::max(1, P->leaves) >= 16 ? 1 : 0;
+    }
     P->sz_dbpart = db_aux_bytes(P->db_rows, c.Co, P->leaves);
     // one layout serves every call: [xpk | dypk | wpk | wtpk | part | dbpart]
     P->off_xpk = 0;

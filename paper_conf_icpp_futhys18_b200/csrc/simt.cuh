@@ -240,16 +240,19 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
   }
 }
 
-// Many-split variant (the halo filter gradient's 148 one-per-CTA partials): block = 32 channels x
-// 8 split phases over 4 weight rows; thread (ty, lane) sums splits ty, ty+8, ... in ascending order,
-// then the 8 phase sums are added in phase order.  Fixed order, a function of `splits` only.
+// Many-split variant (the halo filter gradient's 148 one-per-CTA partials, and small filters whose
+// 32 x 32 tiles would leave most SMs idle): block = 32 channels x 8 split phases over 4 weight
+// rows; thread (ty, lane) sums splits ty, ty+8, ... in ascending order, then the 8 phase sums are
+// added in phase order.  Fixed order, a function of `splits` only.  Leaf plans: blockIdx.z = leaf.
 __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict__ part,
                                                          const BrOut dw, int Co, int C,
                                                          int taps, int Kw, int Cp, int ld, int mpad,
-                                                         int splits, int accumulate, int s2d, int Ks) {
+                                                         int splits, int accumulate, int s2d, int Ks,
+                                                         long long leaf_stride) {
   __shared__ float red[8][4][33];
   pdl_launch_dependents();
   pdl_wait();
+  part += (size_t)blockIdx.z * splits * ((size_t)mpad * ld);
   const int inner = C * taps;
   const int i0 = blockIdx.x * 4, co = blockIdx.y * 32 + (threadIdx.x & 31), ty = threadIdx.x >> 5;
   const size_t sstride = (size_t)mpad * ld;
@@ -270,13 +273,22 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
     }
     src[u] = part + (size_t)row * ld + (ok[u] ? co : 0);
   }
+  // splits ty, ty+8, ... added in ascending order; eight of them (32 loads) issued per batch,
+  // unconditionally (clamped split index), out-of-range values zeroed after the loads
   float a[4] = {0.f, 0.f, 0.f, 0.f};
-  for (int sp = ty; sp < splits; sp += 8) {
-    float v[4];
+  for (int sp0 = ty; sp0 < splits; sp0 += 64) {
+    float v[8][4];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) v[u] = ok[u] ? __ldg(src[u] + (size_t)sp * sstride) : 0.f;
+    for (int k = 0; k < 8; ++k) {
+      const size_t off = (size_t)min(sp0 + 8 * k, splits - 1) * sstride;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) a[u] += v[u];
+      for (int u = 0; u < 4; ++u) v[k][u] = __ldg(src[u] + off);
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (sp0 + 8 * k < splits && ok[u]) a[u] += v[k][u];
   }
 #pragma unroll
   for (int u = 0; u < 4; ++u) red[ty][u][threadIdx.x & 31] = a[u];
@@ -288,7 +300,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
     for (int k = 0; k < 8; ++k) t += red[k][u][lane];
     const int i = i0 + u;
     if (i < inner && co < Co) {
-      float *d = dw.at(co, 0, (size_t)inner, (size_t)i);
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + blockIdx.z * leaf_stride;
       *d = accumulate ? *d + t : t;
     }
   }

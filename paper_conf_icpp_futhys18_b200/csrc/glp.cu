@@ -1466,31 +1466,39 @@ glp_status_t run_wgrad_reduce(glp_plan_s &P, const BrOut &dw_in, const BrOut *db
   }
   const int acc_red = via_ws ? 0 : accumulate;
   if (P.halo) {
+    const DwRed r{part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx, P.hw.ld, P.hw.mpad, P.hw.splits,
+                  accumulate, P.s2d, P.dxg.Kw, 0LL};
     GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
                         dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32)),
-                        dim3(256), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx, P.hw.ld,
-                        P.hw.mpad, P.hw.splits, accumulate, P.s2d, P.dxg.Kw, 0LL));
+                        dim3(256), 0, st, r));
     GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
-  } else if (P.red_wide) {   // small filter: 4 weight rows per block, splits over 8 phases
-    GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide,
-                        dim3((unsigned)cdiv((long long)d.C * P.taps, 4), (unsigned)cdiv(d.Co, 32), (unsigned)L),
-                        dim3(256), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
-                        P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128,
-                        P.wgrad.splits / L, acc_red, P.s2d, P.dxg.Kw, leaf_stride));
-    GLP_LAUNCH_CHECK("reduce_tc_dw_wide");
-  } else
-  GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw,
-                      dim3((unsigned)cdiv((long long)d.C * P.taps, 32), (unsigned)cdiv(d.Co, 32), (unsigned)L),
-                      dim3(32, 8), 0, st, part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx,
-                      P.wgrad.n_tiles * P.wgrad.bn, P.wgrad.m_units * P.wgrad.cg * 128,
-                      P.wgrad.splits / L, acc_red, P.s2d, P.dxg.Kw, leaf_stride));
-  GLP_LAUNCH_CHECK("reduce_tc_dw");
-  if (db) {
-    DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
-    GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)cdiv(d.Co, 32), (unsigned)db_groups(P.db_rows / L), (unsigned)L),
-                        dim3(256), 0, st, a.part, *db, d.Co, P.db_rows / L, acc_red, a.part2,
-                        a.tickets, leaf_stride));
-    GLP_LAUNCH_CHECK("reduce_db");
+    if (db) {
+      DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
+      const DbRed q{a.part, *db, d.Co, P.db_rows, accumulate, a.part2, a.tickets, 0LL,
+                    db_groups(P.db_rows), (int)cdiv(d.Co, 32)};
+      GLP_CUDA(launch_pdl(P.pdl, reduce_db, dim3((unsigned)q.cx, (unsigned)q.G), dim3(256), 0, st, q));
+      GLP_LAUNCH_CHECK("reduce_db");
+    }
+  } else {
+    const DwRed r{part, dw, d.Co, d.C, P.taps, d.Kw, P.Cpx, P.wgrad.n_tiles * P.wgrad.bn,
+                  P.wgrad.m_units * P.wgrad.cg * 128, P.wgrad.splits / L, acc_red, P.s2d,
+                  P.dxg.Kw, leaf_stride};
+    // dW blocks: 32 x 32 tiles, or 4 weight rows x 32 channels for small filters (red_wide)
+    const int ax = (int)cdiv((long long)d.C * P.taps, P.red_wide ? 4 : 32), ay = (int)cdiv(d.Co, 32);
+    if (db) {   // dW and db reductions in one launch
+      DbAux a = db_aux(P, ws + P.off_dbpart, P.db_rows);
+      const DbRed q{a.part, *db, d.Co, P.db_rows / L, acc_red, a.part2, a.tickets, leaf_stride,
+                    db_groups(P.db_rows / L), (int)cdiv(d.Co, 32)};
+      const dim3 grid((unsigned)(ax * ay + q.cx * q.G), 1, (unsigned)L);
+      if (P.red_wide) GLP_CUDA(launch_pdl(P.pdl, reduce_wgrad<1>, grid, dim3(256), 0, st, r, q, ax, ay));
+      else GLP_CUDA(launch_pdl(P.pdl, reduce_wgrad<0>, grid, dim3(256), 0, st, r, q, ax, ay));
+      GLP_LAUNCH_CHECK("reduce_wgrad");
+    } else {
+      const dim3 grid((unsigned)ax, (unsigned)ay, (unsigned)L);
+      if (P.red_wide) GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw_wide, grid, dim3(256), 0, st, r));
+      else GLP_CUDA(launch_pdl(P.pdl, reduce_tc_dw, grid, dim3(256), 0, st, r));
+      GLP_LAUNCH_CHECK("reduce_tc_dw");
+    }
   }
   if (via_ws) {   // dW || db = the fixed tree over the leaves (glp_tree_sum order)
     const float *parts[8];
@@ -1638,8 +1646,9 @@ glp_status_t run_wgrad_simt(glp_plan_s &P, const float *x, const float *dy, floa
     DbAux a = db_aux(P, reinterpret_cast<uint8_t *>(dbp), P.simt_splits);
     GLP_CUDA(cudaMemsetAsync(a.tickets, 0, (size_t)cdiv(d.Co, 32) * 4, st));
     float *dbs[1] = {db};
-    reduce_db<<<dim3((unsigned)cdiv(d.Co, 32), (unsigned)db_groups(P.simt_splits)), 256, 0, st>>>(
-        a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets, 0LL);
+    const DbRed q{a.part, br_out(P, 1, dbs), d.Co, P.simt_splits, accumulate, a.part2, a.tickets,
+                  0LL, db_groups(P.simt_splits), (int)cdiv(d.Co, 32)};
+    reduce_db<<<dim3((unsigned)q.cx, (unsigned)q.G), 256, 0, st>>>(q);
     GLP_LAUNCH_CHECK("reduce_db");
   }
   return GLP_OK;

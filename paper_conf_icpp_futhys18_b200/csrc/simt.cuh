@@ -166,18 +166,22 @@ __global__ void reduce_simt_dw(const float *__restrict__ part, float *__restrict
 // shared memory, and dW[co][i] is written 32 consecutive i at a time.  grid (ceil(C*taps/32),
 // ceil(Co/32), leaves).  Leaf plans (the deterministic exchange): blockIdx.z = leaf, `splits` are
 // that leaf's splits (partials leaf*splits ...), and its dW goes leaf_stride floats further.
-__global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ part,
-                                                    const BrOut dw, int Co, int C,
-                                                    int taps, int Kw, int Cp, int ld, int mpad,
-                                                    int splits, int accumulate, int s2d, int Ks,
-                                                    long long leaf_stride) {
+struct DwRed {   // arguments of the dW reductions
+  const float *part;
+  BrOut dw;
+  int Co, C, taps, Kw, Cp, ld, mpad, splits, accumulate, s2d, Ks;
+  long long leaf_stride;
+};
+__device__ __forceinline__ void reduce_tc_dw_body(const DwRed &r, int bx, int by, int bz) {
   __shared__ float tile[32][33];
-  pdl_launch_dependents();
-  pdl_wait();
-  part += (size_t)blockIdx.z * splits * ((size_t)mpad * ld);
+  const float *part = r.part + (size_t)bz * r.splits * ((size_t)r.mpad * r.ld);
+  const BrOut &dw = r.dw;
+  const int Co = r.Co, C = r.C, taps = r.taps, Kw = r.Kw, Cp = r.Cp, ld = r.ld, mpad = r.mpad;
+  const int splits = r.splits, accumulate = r.accumulate, s2d = r.s2d, Ks = r.Ks;
+  const long long leaf_stride = r.leaf_stride;
   const int inner = C * taps;
-  const int i0 = blockIdx.x * 32, co0 = blockIdx.y * 32;
-  const int lane = threadIdx.x, ty = threadIdx.y;
+  const int i0 = bx * 32, co0 = by * 32;
+  const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
   const size_t sstride = (size_t)mpad * ld;
   const float *src[4];
   bool ok[4];
@@ -233,7 +237,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
   for (int j = ty; j < 32; j += 8) {
     const int co = co0 + j, i = i0 + lane;
     if (co < Co && i < inner) {
-      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + blockIdx.z * leaf_stride;
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + bz * leaf_stride;
       const float v = tile[lane][j];
       *d = accumulate ? *d + v : v;
     }
@@ -244,17 +248,15 @@ __global__ void __launch_bounds__(256) reduce_tc_dw(const float *__restrict__ pa
 // 32 x 32 tiles would leave most SMs idle): block = 32 channels x 8 split phases over 4 weight
 // rows; thread (ty, lane) sums splits ty, ty+8, ... in ascending order, then the 8 phase sums are
 // added in phase order.  Fixed order, a function of `splits` only.  Leaf plans: blockIdx.z = leaf.
-__global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict__ part,
-                                                         const BrOut dw, int Co, int C,
-                                                         int taps, int Kw, int Cp, int ld, int mpad,
-                                                         int splits, int accumulate, int s2d, int Ks,
-                                                         long long leaf_stride) {
+__device__ __forceinline__ void reduce_tc_dw_wide_body(const DwRed &rr, int bx, int by, int bz) {
   __shared__ float red[8][4][33];
-  pdl_launch_dependents();
-  pdl_wait();
-  part += (size_t)blockIdx.z * splits * ((size_t)mpad * ld);
+  const float *part = rr.part + (size_t)bz * rr.splits * ((size_t)rr.mpad * rr.ld);
+  const BrOut &dw = rr.dw;
+  const int Co = rr.Co, C = rr.C, taps = rr.taps, Kw = rr.Kw, Cp = rr.Cp, ld = rr.ld, mpad = rr.mpad;
+  const int splits = rr.splits, accumulate = rr.accumulate, s2d = rr.s2d, Ks = rr.Ks;
+  const long long leaf_stride = rr.leaf_stride;
   const int inner = C * taps;
-  const int i0 = blockIdx.x * 4, co = blockIdx.y * 32 + (threadIdx.x & 31), ty = threadIdx.x >> 5;
+  const int i0 = bx * 4, co = by * 32 + (threadIdx.x & 31), ty = threadIdx.x >> 5;
   const size_t sstride = (size_t)mpad * ld;
   const float *src[4];
   bool ok[4];
@@ -300,7 +302,7 @@ __global__ void __launch_bounds__(256) reduce_tc_dw_wide(const float *__restrict
     for (int k = 0; k < 8; ++k) t += red[k][u][lane];
     const int i = i0 + u;
     if (i < inner && co < Co) {
-      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + blockIdx.z * leaf_stride;
+      float *d = dw.at(co, 0, (size_t)inner, (size_t)i) + bz * leaf_stride;
       *d = accumulate ? *d + t : t;
     }
   }
@@ -322,21 +324,27 @@ __host__ __device__ constexpr int db_groups(int rows) {
 }
 // Leaf plans: blockIdx.z = leaf; its `rows` partial rows follow the previous leaves', its group sums
 // and tickets have their own slices, and its db goes leaf_stride floats further.
-__global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
-                                                 const BrOut db, int Co, int rows,
-                                                 int accumulate, float *__restrict__ part2,
-                                                 unsigned int *__restrict__ tickets,
-                                                 long long leaf_stride) {
+struct DbRed {   // arguments of the db reduction
+  const float *part;
+  BrOut db;
+  int Co, rows, accumulate;
+  float *part2;
+  unsigned int *tickets;
+  long long leaf_stride;
+  int G, cx;   // row groups (db_groups(rows)) and channel blocks (ceil(Co/32))
+};
+// block (bx = channel block, g = row group, bz = leaf)
+__device__ __forceinline__ void reduce_db_body(const DbRed &r, int bx, int g, int bz) {
   __shared__ float red[8][33];
   __shared__ bool last;
-  pdl_launch_dependents();
-  pdl_wait();
-  part += (size_t)blockIdx.z * rows * Co;
-  const int G = gridDim.y;   // db_groups(rows), set by the launch
-  part2 += (size_t)blockIdx.z * DB_GROUPS * Co;
-  tickets += (size_t)blockIdx.z * gridDim.x;
+  const int Co = r.Co, rows = r.rows, accumulate = r.accumulate, G = r.G;
+  const BrOut &db = r.db;
+  const long long leaf_stride = r.leaf_stride;
+  const float *part = r.part + (size_t)bz * rows * Co;
+  float *part2 = r.part2 + (size_t)bz * DB_GROUPS * Co;
+  unsigned int *tickets = r.tickets + (size_t)bz * r.cx;
   const int lane = threadIdx.x & 31, ty = threadIdx.x >> 5;
-  const int co = blockIdx.x * 32 + lane, g = blockIdx.y;
+  const int co = bx * 32 + lane;
   // rows g + DB_GROUPS*(ty + 8*j), j = 0, 1, ...: four interleaved accumulators (j mod 4) keep
   // four loads in flight (one dependent chain was latency-bound: ~47 L2 round trips for CaffeNet
   // conv1), the tail goes to a0, then ((a0+a1)+(a2+a3)) — an order fixed by `rows` alone
@@ -366,7 +374,7 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
     __threadfence();
   }
   __syncthreads();
-  if (threadIdx.x == 0) last = (atomicAdd(tickets + blockIdx.x, 1u) == (unsigned)G - 1);
+  if (threadIdx.x == 0) last = (atomicAdd(tickets + bx, 1u) == (unsigned)G - 1);
   __syncthreads();
   if (last && ty == 0) {
     __threadfence();
@@ -381,10 +389,44 @@ __global__ void __launch_bounds__(256) reduce_db(const float *__restrict__ part,
         s3 += __ldcg(part2 + (size_t)(k + 3) * Co + co);
       }
       const float s = (s0 + s1) + (s2 + s3);
-      float *d = db.at(co, 0, 1, 0) + blockIdx.z * leaf_stride;
+      float *d = db.at(co, 0, 1, 0) + bz * leaf_stride;
       *d = accumulate ? *d + s : s;
     }
-    if (lane == 0) tickets[blockIdx.x] = 0;   // re-arm for the next call on this workspace
+    if (lane == 0) tickets[bx] = 0;   // re-arm for the next call on this workspace
+  }
+}
+
+// Kernels.  reduce_tc_dw: grid (ceil(C*taps/32), ceil(Co/32), leaves); reduce_tc_dw_wide: grid
+// (ceil(C*taps/4), ceil(Co/32), leaves); reduce_db: grid (ceil(Co/32), G, leaves); block 256.
+// reduce_wgrad<WIDE>: the dW reduction and the db reduction in ONE launch (one node fewer on the
+// filter-gradient chain), grid (nA + cx * G, 1, leaves): blocks < nA = ax * ay are dW blocks
+// (bx = b % ax, by = b / ax), the rest db blocks -- the same bodies, the same per-element order.
+__global__ void __launch_bounds__(256) reduce_tc_dw(const DwRed r) {
+  pdl_launch_dependents();
+  pdl_wait();
+  reduce_tc_dw_body(r, blockIdx.x, blockIdx.y, blockIdx.z);
+}
+__global__ void __launch_bounds__(256) reduce_tc_dw_wide(const DwRed r) {
+  pdl_launch_dependents();
+  pdl_wait();
+  reduce_tc_dw_wide_body(r, blockIdx.x, blockIdx.y, blockIdx.z);
+}
+__global__ void __launch_bounds__(256) reduce_db(const DbRed r) {
+  pdl_launch_dependents();
+  pdl_wait();
+  reduce_db_body(r, blockIdx.x, blockIdx.y, blockIdx.z);
+}
+template <int WIDE>
+__global__ void __launch_bounds__(256) reduce_wgrad(const DwRed r, const DbRed q, int ax, int ay) {
+  pdl_launch_dependents();
+  pdl_wait();
+  const int b = blockIdx.x, nA = ax * ay;
+  if (b < nA) {
+    if (WIDE) reduce_tc_dw_wide_body(r, b % ax, b / ax, blockIdx.z);
+    else reduce_tc_dw_body(r, b % ax, b / ax, blockIdx.z);
+  } else {
+    const int bd = b - nA;
+    reduce_db_body(q, bd % q.cx, bd / q.cx, blockIdx.z);
   }
 }
 

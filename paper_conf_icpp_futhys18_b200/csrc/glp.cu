@@ -289,10 +289,14 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
     const int real = (int)cdiv(kb_total, kbps);
     if (real != s) continue;
     const double waves = std::ceil(tiles_mn * (double)s * leaves / sm);
-    // + the fixed-order reduction: each output sums its s partials in dependent batches of 8
-    // loads (~1.2 us per batch when the reduction grid is too small to hide the latency: tiny
-    // layers with many splits spent 75 us in reduce_tc_dw at s = 512)
-    const double red = (double)mpad * npad < 148.0 * 1024 ? std::ceil(s / 8.0) * 1.2e-6 : 0.0;
+    // + the fixed-order reduction: each output sums its s partials in dependent batches (~1.2 us
+    // per batch when the reduction grid is too small to hide the latency): batches of 8 splits
+    // in reduce_tc_dw, of 64 in the 8-phase reduce_tc_dw_wide that small filters (< 64 tiles of
+    // 32 x 32, ~mpad * npad < 64 Ki) use -- there the wider split grid pays (LeNet conv1: 144
+    // splits 18 us vs 72 splits 28 us, GEMM alone)
+    const double mn = (double)mpad * npad;
+    const double red = mn < 65536.0 ? std::ceil(s / 64.0) * 1.2e-6
+                       : mn < 148.0 * 1024 ? std::ceil(s / 8.0) * 1.2e-6 : 0.0;
     const double t = waves * (kbps * kb_s + 2e-6) + (double)s * leaves * mpad * npad * 8.0 / bw + red;
     if (t < best_t * 0.999) {
       best_t = t;
@@ -730,6 +734,10 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   } else if (mode == MODE_WGRAD) {
     pp.splits = choose_splits(pp.m_units * pp.n_tiles, pp.kb_total, pp.bn,
                               pp.m_units * pp.cg * 128, pp.n_tiles * pp.bn, elem, pp.cg, P.x3);
+#ifdef GLP_DIAG
+    if (const char *e = getenv("GLP_DEBUG_SPLITS"))   // diagnostics: forced split count
+      pp.splits = std::max(1, std::min((int)pp.kb_total, atoi(e)));
+#endif
     pp.kb_per_split = (int)cdiv(pp.kb_total, pp.splits);
     pp.splits = (int)cdiv(pp.kb_total, pp.kb_per_split);
   } else {

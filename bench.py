@@ -890,7 +890,7 @@ def run_glp(args, ws, rank, local):
         host_pinned = [{k: v.pin_memory() for k, v in s.host.items() if k not in s.shared_keys}
                        for s in states]
         out_host = torch.empty(nparams, pin_memory=True)
-        h2d = sum(v.numel() * 4 for hp in host_pinned for v in hp.values())
+        h2d_bytes = sum(v.numel() * 4 for hp in host_pinned for v in hp.values())
         d2h = nparams * 4
         ke = max(1, args.e2e_steps)
         step()
@@ -898,20 +898,49 @@ def run_glp(args, ws, rank, local):
         if G > 1:
             dist.barrier()
 
-        def e2e_step():
-            for s, hp in zip(states, host_pinned):
-                for k2, v in hp.items():
-                    s.t[k2].copy_(v, non_blocking=True)
-            step()
-            out_host.copy_(flat, non_blocking=True)
-        ems = time_steps(e2e_step, ke, stream)
+        # Pipelined like a training input loader: step k+1's inputs travel host -> device (a
+        # copy stream, into device staging buffers) while step k computes; each step starts with
+        # a device-to-device copy staging -> the step's own input tensors (the captured graph's
+        # addresses).  The timed region holds all K host -> device copies (the first one not
+        # overlapped), K steps and K device -> host reads of dW||db.
+        staging = [{k2: torch.empty_like(s.t[k2]) for k2 in hp} for s, hp in zip(states, host_pinned)]
+        cs = torch.cuda.Stream(device=dev)
+
+        def h2d():
+            with torch.cuda.stream(cs):
+                for st_, hp in zip(staging, host_pinned):
+                    for k2, v in hp.items():
+                        st_[k2].copy_(v, non_blocking=True)
+            ev = torch.cuda.Event()
+            ev.record(cs)
+            return ev
+
+        def e2e_run(k_steps):
+            ready = h2d()
+            for k in range(k_steps):
+                stream.wait_event(ready)
+                for s, st_ in zip(states, staging):
+                    for k2, v in st_.items():
+                        s.t[k2].copy_(v, non_blocking=True)
+                if k + 1 < k_steps:
+                    consumed = torch.cuda.Event()
+                    consumed.record(stream)
+                    cs.wait_event(consumed)
+                    ready = h2d()
+                step()
+                out_host.copy_(flat, non_blocking=True)
+
+        e2e_run(1)   # warm the copy path
+        torch.cuda.synchronize()
+        ems = time_steps(lambda: e2e_run(ke), 1, stream) / ke
         if G > 1:
             tt = torch.tensor([ems], device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ems = float(tt.item())
         e2e = {"value": round(images_per_step / (ems / 1e3), 1), "unit": UNIT,
-               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": round(ems, 3), "steps": ke}
+               "h2d_bytes_per_step": int(h2d_bytes), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": round(ems, 3), "steps": ke,
+               "pipelined": "step k+1's host->device copy overlaps step k (copy stream + device staging)"}
 
     weak = None
     if G > 1 and args.scaling == "strong" and not args.no_extra_modes:

@@ -157,7 +157,7 @@ typedef struct {
   int fused_dy_builders;  /* 0: model; 1: cp.async landing zone; 2 or 3: register builder groups   */
   int max_kblocks_per_stage; /* 1..4 (k-blocks per pipeline stage cap; 4 = default)                */
   int wgrad_tile_n;       /* 0: model; else the filter-gradient N tile (multiple of 16, <= 256)    */
-  int tile_units;         /* fwd/dgrad tile model applies below this many work units per slot (2)  */
+  int tile_units;         /* fwd/dgrad tile model applies below this many work units per slot (6)  */
   int bn_model;           /* 1: fwd/dgrad N-tile model for small grids; 0: always the default tile */
   int pack_block;         /* 0: warp-tiled activation pack; 1: block-tiled                         */
   int s2d_block;          /* 0: warp-per-32-pixel space-to-depth pack; 1: block-persistent          */

@@ -392,7 +392,7 @@ struct glp_plan_s {
   int fdy_ncg = 0;     // GLP_FDY_NCG=1|2|3: force the fused-dy builder variant (A/B runs)
   int allow_hdg = 1;   // GLP_HDGRAD=0: im2col backward-data everywhere (A/B runs); 2 = force where legal
   int wgrad_bn = 0;    // GLP_WGRAD_BN=n: filter-gradient N tile override (A/B runs; 0 = model)
-  int tile_units = 2;  // GLP_TILE_UNITS=u: fwd/dgrad tile model applies below u units per slot
+  int tile_units = 6;  // fwd/dgrad tile model applies below this many units per slot
   // Dynamic smem budget of the persistent GEMMs.  Below the 227 KB maximum it leaves room on
   // every SM for one block of the HBM-bound pack kernels (16.5 KB), so a pack issued on another
   // stream (e.g. the next layer's dy pack during a filter-gradient GEMM) runs beside the GEMM
@@ -1803,7 +1803,7 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
 
 glp_status_t glp_plan_options_default(glp_plan_options_t *o) {
   if (!o) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
-  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 2, 1, 0, 0, 232448, 0, 0};
+  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 6, 1, 0, 0, 232448, 0, 0};
   return GLP_OK;
 }
 

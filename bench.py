@@ -949,6 +949,26 @@ def run_glp(args, ws, rank, local):
     if G == 1 and not args.no_extra_modes:
         modes = {m: quick_mode(args, m, G, rank, dev) for m in ("bf16", "tf32") if m != args.math}
 
+    # kernels per timed step, counted (not modelled): the CUPTI tracker (libglp_tracker.so, the
+    # NEXT-4 resource tracker) records every kernel of one more step issued exactly as the timed
+    # ones; ours are the glp:: kernels.  Formula fallback where CUPTI is unavailable.
+    launches_src = "formula (packs, GEMMs, reductions per unit)"
+    per_step = sum(s.launches() for s in states)
+    if G == 1:   # (G > 1: the step holds collectives every rank must join)
+        try:
+            from paper_conf_icpp_futhys18_b200.tracker import Tracker
+            torch.cuda.synchronize()
+            with Tracker() as trk:
+                run_one()
+                torch.cuda.synchronize()
+            ours = [k for k in trk.kernels if "glp" in k.name]
+            if ours:
+                per_step = len(ours)
+                launches_src = (f"CUPTI kernel records of one extra step issued like the timed ones "
+                                f"({len(ours)} glp kernels, {len(trk.kernels) - len(ours)} other)")
+        except Exception as e:   # no CUPTI / tracker library: keep the formula
+            launches_src += f"; tracker unavailable: {type(e).__name__}"
+
     cpu = None
     if rank == 0 and G == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(layers, budget_s=12.0)
@@ -984,7 +1004,8 @@ def run_glp(args, ws, rank, local):
         "cpu_baseline": cpu,
         "clocks": clk,
         "e2e": e2e,
-        "gpu_launches": int(sum(s.launches() for s in states) * args.steps),
+        "gpu_launches": int(per_step * args.steps),
+        "gpu_launches_source": launches_src,
         "launch": ("cuda_graph" if use_graph else "eager") +
                   ("" if args.serial else
                    f" (step DAG: {len(step.levels)} levels, up to {step.width} concurrent units)"),

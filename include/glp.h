@@ -96,6 +96,8 @@ typedef struct {
    * glp_plan_kernel_attr(0) describes x 128) and the rows one sample occupies (H_o*W_o, or the
    * padded grid of the halo forward, x the N tiles). */
   long long s_slot_rows, s_rows_per_sample;
+  int wgrad_reduce_wide; /* 1: the dW split reduction runs 4 weight rows x 8 split phases per block
+                            (small filters: < 64 tiles of 32 x 32); 0: 32 x 32 tiles             */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

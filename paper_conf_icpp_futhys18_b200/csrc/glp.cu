@@ -2081,6 +2081,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->dgrad_halo = P->hdg;
   I->s_slot_rows = P->s_slot_rows;
   I->s_rows_per_sample = P->s_rows_per_sample;
+  I->wgrad_reduce_wide = P->red_wide;
   if (P->hdg) {
     I->grid_bwd_data = P->hd_grid;
     I->tile_n_bwd_data = P->hd.bn;

@@ -162,3 +162,29 @@ def test_tracker_exports_every_declared_symbol():
     fields = re.findall(r"\b(name|grid|block|cluster|regs|static_smem|dynamic_smem|queued_ns|"
                         r"submitted_ns|start_ns|end_ns|stream_id|correlation_id)\b", body)
     assert fields == [f for f, _ in tracker.KernelRecord._fields_]
+
+
+def _header_struct_fields(header, typedef_name):
+    """Field names of `typedef struct { ... } typedef_name;` in include/<header>, in order."""
+    src = open(os.path.join(ROOT, "include", header)).read()
+    end = src.index("} " + typedef_name + ";")
+    start = src.rindex("typedef struct {", 0, end)
+    body = re.sub(r"/\*.*?\*/", "", src[start + len("typedef struct {"):end], flags=re.S)
+    names = []
+    for decl in body.split(";"):
+        decl = " ".join(decl.split())
+        if not decl:
+            continue
+        decl = re.sub(r"^(unsigned |long long |long |const )*(int|size_t|double|float|long long|char)\b ?",
+                      "", decl)
+        names += [re.sub(r"\[.*\]", "", n).strip(" *") for n in decl.split(",")]
+    return names
+
+
+@pytest.mark.parametrize("typedef_name, cls", [
+    ("glp_plan_info_t", glp.PlanInfo), ("glp_plan_options_t", glp.PlanOptions),
+    ("glp_device_limits_t", glp.DeviceLimits), ("glp_kernel_attr_t", glp.KernelAttr)])
+def test_binding_structs_match_header(typedef_name, cls):
+    """The ctypes mirrors of the ABI structs list the header's fields in the header's order (a
+    field added on one side only would shift every later field)."""
+    assert _header_struct_fields("glp.h", typedef_name) == [f for f, _ in cls._fields_]

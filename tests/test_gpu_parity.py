@@ -585,8 +585,10 @@ def test_grouped_conv(shape, math):
             np.testing.assert_array_equal(v.cpu().numpy(), got[k], err_msg="staged " + k)
 
 
+@pytest.mark.parametrize("shape", [(16, 24, 8, 8, 40, 3, 1, 1), (16, 1, 36, 36, 20, 5, 1, 0)],
+                         ids=["c24k3", "small_filter"])
 @pytest.mark.parametrize("math", ["fp32", "tf32", "bf16"])
-def test_tree_exchange_bitwise_invariant_emulated_ranks(math):
+def test_tree_exchange_bitwise_invariant_emulated_ranks(math, shape):
     """Deterministic gradient exchange (NEXT-2) as the library runs it, with 1, 2, 4 and 8 ranks
     emulated on one device: each rank plans its local batch as 8/world leaves (wgrad_leaves),
     packs x and dy ONCE, runs one filter-gradient GEMM whose splits never cross a leaf, reduces
@@ -594,9 +596,11 @@ def test_tree_exchange_bitwise_invariant_emulated_ranks(math):
     8-leaf tree), and glp_tree_exchange -- called once per emulated rank with every rank's
     buffers as the "peer" pointers -- completes the top of the tree into every rank's output.
     dW||db is bitwise the same for every world size and every rank, equal to the composed
-    glp_conv_bwd_filter of the 8-leaf plan, within the bar of the oracle, exact on integers."""
+    glp_conv_bwd_filter of the 8-leaf plan, within the bar of the oracle, exact on integers.
+    small_filter (C*K*K = 25, leaf = 2 images x 1024 pixels): the per-leaf dW reductions run the
+    8-phase small-filter kernel (grid z = leaf)."""
     from paper_conf_icpp_futhys18_b200.dist import LEAVES, rank_leaves
-    N, C, H, W, Co, K, S, P = 16, 24, 8, 8, 40, 3, 1, 1   # leaf = 2 images x 64 pixels
+    N, C, H, W, Co, K, S, P = shape
     Ho = oracle.out_dim(H, K, S, P)
     wsz = Co * C * K * K
     numel = (wsz + Co + 3) // 4 * 4
@@ -631,6 +635,8 @@ def test_tree_exchange_bitwise_invariant_emulated_ranks(math):
             np.testing.assert_array_equal(r, results[0])
         # the composed call of the 8-leaf plan (leaves reduced in the workspace, the same tree)
         layer = glp.ConvLayer(N, C, H, W, Co, K, S, P, math=math, options={"wgrad_leaves": LEAVES})
+        if C == 1 and math != "bf16":
+            assert layer.info.wgrad_reduce_wide == 1
         dw = torch.empty(layer.w_shape, device=DEV)
         db = torch.empty(Co, device=DEV)
         layer.bwd_filter(t["x"], t["dy"], dw, db)

@@ -78,6 +78,9 @@ def parse_args():
                    help="(tests) launcher plumbing only: start the ranks, form a gloo process group "
                         "on CPU, all-reduce one tensor and print the line's n_gpus; no GPU work")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--plan-options", default="",
+                   help="JSON glp_plan_options_t fields for every plan (A/B runs of alternative "
+                        "kernels/tilings; recorded in config)")
     p.add_argument("--e2e-steps", type=int, default=5)
     p.add_argument("--serial", action="store_true",
                    help="issue the step on one stream (default: the real-network stream DAG)")
@@ -212,6 +215,9 @@ class ClockSampler:
 
 # ------------------------------------------------------------------------- GLP arm ------------
 
+PLAN_OPTIONS = {}   # --plan-options (A/B measurements of alternative plans; recorded in the line)
+
+
 class LayerState:
     def __init__(self, layer, n_local, n_global, shard, math, dev, grads, idx, leaves=0):
         import torch
@@ -223,7 +229,8 @@ class LayerState:
         # leaves > 1: a leaf plan (the deterministic exchange: splits never cross a batch leaf)
         self.conv = glp.ConvLayer(n_local, layer.C, layer.H, layer.W, layer.Co, layer.K, layer.S,
                                   layer.P, math=math, device=dev.index, groups=layer.groups,
-                                  options={"wgrad_leaves": leaves} if leaves > 0 else None)
+                                  options=dict(PLAN_OPTIONS, **({"wgrad_leaves": leaves} if leaves > 0 else {}))
+                                  or None)
         if shard is None:
             d = gen_layer(layer, n_global=n_global, batch=n_local)
         else:  # strong scaling: this rank's contiguous slice of the global batch
@@ -390,7 +397,8 @@ class GroupState:
         self.name = "+".join(m.name for m in members)
         self.n = n_local
         self.conv = glp.ConvLayer(n_local, l0.C, l0.H, l0.W, None, l0.K, l0.S, l0.P, math=math,
-                                  device=dev.index, branches=[m.Co for m in members])
+                                  device=dev.index, branches=[m.Co for m in members],
+                                  options=PLAN_OPTIONS or None)
         ds = [gen_layer(m, n_global=n_global, batch=n_local) for m in members]
         self.host = {"x": torch.from_numpy(ds[0]["x"])}   # the shared input
         for i, d in enumerate(ds):
@@ -995,7 +1003,8 @@ def run_glp(args, ws, rank, local):
                    f"{sum(v.numel() * 4 for s in states for v in s.t.values()) / 1e9:.2f} GB)",
                    "step_gflop": round(step_flops / 1e9, 1),
                    "samples_in_flight": [i.samples_in_flight for i in info0],
-                   "wgrad_splits": [i.splits_wgrad for i in info0]},
+                   "wgrad_splits": [i.splits_wgrad for i in info0],
+                   **({"plan_options": PLAN_OPTIONS} if PLAN_OPTIONS else {})},
         "tflops_step": round(step_flops / (ms_per_step * 1e-3) / 1e12, 1),
         "roofline": roofline,
         "kernels": [{k: r[k] for k in ("layer", "pass", "avg_us", "tflops")} for r in kern],
@@ -1212,6 +1221,8 @@ def main():
     if torch.cuda.device_count() < (1 if args.same_device else local + 1):
         sys.exit(f"bench.py: rank {rank} needs cuda:{local} but {torch.cuda.device_count()} "
                  "CUDA device(s) are visible (there is no CPU fallback)")
+    if args.plan_options:
+        PLAN_OPTIONS.update(json.loads(args.plan_options))
     if args.scheme == "pool":
         if rank == 0:
             run_pool(args)

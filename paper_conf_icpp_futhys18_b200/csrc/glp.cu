@@ -523,15 +523,21 @@ glp_status_t plan_halo(glp_plan_s &P) {
   return GLP_OK;
 }
 
-// Halo backward-data (hdgrad.cuh): unit stride, square kernel, bf16, the flipped-tap Wt of the
-// im2col-TMA dgrad, 64-channel blocks of C_o, and a tile geometry (R output rows padded to a pitch
-// of WQ >= W + K - 1 pixels, R*WQ = 128) that wastes at most 30 % of the rows.  Used when the
-// im2col A traffic dominates: >= 9 taps and C_i <= 128 (each A byte feeds few columns).
+// Halo backward-data (hdgrad.cuh): unit stride, square kernel, bf16 or tf32 (not 3xTF32), the
+// flipped-tap Wt of the im2col-TMA dgrad, 128-byte channel blocks of C_o (64 bf16 / 32 tf32), and a
+// tile geometry (R output rows padded to a pitch of WQ >= W + K - 1 pixels, R*WQ = 128) that
+// wastes at most 30 % of the rows.  Used when the im2col A traffic dominates: >= 9 taps and
+// C_i <= 128 (each A byte feeds few columns).
+const void *hdgrad_fn(int elem) {
+  return elem == 2 ? reinterpret_cast<const void *>(hdgrad_kernel<2>)
+                   : reinterpret_cast<const void *>(hdgrad_kernel<4>);
+}
 glp_status_t plan_hdgrad(glp_plan_s &P) {
   P.hdg = 0;
   const glp_conv_desc_s &d = P.d;
-  if (!P.allow_hdg || P.elem != 2 || d.nbr > 1 || d.Sh != 1 || d.Sw != 1 || d.Kh != d.Kw ||
-      d.Ph != d.Pw || d.Ph > d.Kh - 1 || !P.dgrad.a_tma || P.Cop % 64 != 0)
+  const int cb = 128 / P.elem;   // channels per 128-byte block
+  if (!P.allow_hdg || P.x3 || P.simt || d.nbr > 1 || d.Sh != 1 || d.Sw != 1 || d.Kh != d.Kw ||
+      d.Ph != d.Pw || d.Ph > d.Kh - 1 || !P.dgrad.a_tma || P.dgrad.krow != 128 || P.Cop % cb != 0)
     return GLP_OK;
   const int K = d.Kh, taps = K * K;
   int WQ = 8;
@@ -556,7 +562,7 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   h.N = d.N;
   h.tiles_img = tiles_img;
   h.units = (int)cdiv((long long)d.N * tiles_img, 2);
-  h.ncb = P.Cop / 64;
+  h.ncb = P.Cop / cb;
   h.cop = P.Cop;
   h.bn = bn;
   h.ci = d.C;
@@ -584,10 +590,10 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   if (h.b_stages < 3) return GLP_OK;
   P.hd_smem = 1024 + h.a_stages * h.a_bytes + h.b_stages * h.b_bytes +
               8 * (2 * h.a_stages + 2 * h.b_stages + 4) + 16;
-  GLP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void *>(hdgrad_kernel),
-                                cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
-  glp_status_t s = analyze_kernel(P, reinterpret_cast<const void *>(hdgrad_kernel), HD_THREADS,
-                                  P.hd_smem, h.tmem_cols, P.hd_attr);
+  GLP_CUDA(cudaFuncSetAttribute(hdgrad_fn(P.elem), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                232448));
+  glp_status_t s = analyze_kernel(P, hdgrad_fn(P.elem), HD_THREADS, P.hd_smem, h.tmem_cols,
+                                  P.hd_attr);
   if (s) return s;
   // persistent grid: the analyzer's resident CTA-pair slots (#SM x CTAs/SM / 2), at most the units
   long long pairs = std::min<long long>(h.units, (long long)P.sm_count * P.hd_attr.model / 2);
@@ -1284,14 +1290,15 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   return launch_igemm<MODE_FWD>(P, pp, p, m, st);
 }
 
-glp_status_t encode_4d_nhwc(CUtensorMap *map, const void *ptr, int cpitch, int W, int H, int N,
-                            uint32_t box_w, uint32_t box_h) {
+glp_status_t encode_4d_nhwc(CUtensorMap *map, int elem, const void *ptr, int cpitch, int W, int H,
+                            int N, uint32_t box_w, uint32_t box_h) {
   cuuint64_t dims[4] = {(cuuint64_t)cpitch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
-  cuuint64_t strides[3] = {(cuuint64_t)cpitch * 2, (cuuint64_t)W * cpitch * 2,
-                           (cuuint64_t)H * W * cpitch * 2};
-  cuuint32_t box[4] = {64u, box_w, box_h, 1u};
+  cuuint64_t strides[3] = {(cuuint64_t)cpitch * elem, (cuuint64_t)W * cpitch * elem,
+                           (cuuint64_t)H * W * cpitch * elem};
+  cuuint32_t box[4] = {(cuuint32_t)(128 / elem), box_w, box_h, 1u};   // one 128-byte channel block
   cuuint32_t es[4] = {1, 1, 1, 1};
-  CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void *>(ptr), dims,
+  CUresult r = g_encode(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                        4, const_cast<void *>(ptr), dims,
                         strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled (4d) failed (" + std::to_string((int)r) + ")");
@@ -1302,11 +1309,12 @@ glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   const glp_conv_desc_s &d = P.d;
   Maps m;
   glp_status_t s = cached_maps(P, 1, ws, m, [&](Maps &q) {
-    glp_status_t r = encode_4d_nhwc(&q.a, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
+    glp_status_t r = encode_4d_nhwc(&q.a, P.elem, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
                                     (uint32_t)P.hd.WQ, (uint32_t)(P.hd.R + P.hd.K - 1));
     if (r) return r;
-    return encode_2d(&q.b, 2, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
-                     (uint64_t)P.dgrad.Kpad * 2, 64u, (uint32_t)(P.hd.bn / 2), CU_TENSOR_MAP_SWIZZLE_128B);
+    return encode_2d(&q.b, P.elem, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
+                     (uint64_t)P.dgrad.Kpad * P.elem, (uint32_t)(128 / P.elem), (uint32_t)(P.hd.bn / 2),
+                     CU_TENSOR_MAP_SWIZZLE_128B);
   });
   if (s) return s;
   CUtensorMap &mapDy = m.a, &mapW = m.b;
@@ -1330,7 +1338,7 @@ glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   cfg.attrs = attr;
   cfg.numAttrs = P.pdl ? 2 : 1;
   void *args[] = {&p, &mapDy, &mapW};
-  GLP_CUDA(cudaLaunchKernelExC(&cfg, reinterpret_cast<void *>(hdgrad_kernel), args));
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, hdgrad_fn(P.elem), args));
   GLP_LAUNCH_CHECK("hdgrad_kernel");
   return GLP_OK;
 }

@@ -40,7 +40,7 @@ struct HdgradParams {
   int N;                   // images
   int tiles_img;           // ceil(H / R)
   int units;               // ceil(N * tiles_img / 2)
-  int ncb;                 // 64-channel blocks of C_o (the GEMM K per tap)
+  int ncb;                 // 128-byte channel blocks of C_o (64 bf16 / 32 tf32; the K per tap)
   int cop;                 // channel pitch of the packed dy / K pitch per tap of Wt
   int bn;                  // C_i rounded up to 16 (<= 256)
   int ci;                  // valid output channels
@@ -56,9 +56,17 @@ struct HdgradParams {
   int dbg_skip;            // diagnostics: bit0 skip A loads, bit1 skip B loads, bit2 MMAs, bit3 stores
 };
 
+// ELEM 2: bf16 operands, 64-channel blocks (kind::f16); ELEM 4: tf32 operands stored as fp32 bit
+// patterns, 32-channel blocks (kind::tf32).  Either way a channel block is one 128-byte K-major row
+// per pixel and four MMAs (K = 16 bf16 / 8 tf32) consume it, so the halo geometry, the rings and
+// the descriptors are the same bytes.
+template <int ELEM>
 __global__ void __launch_bounds__(HD_THREADS, 1)
     hdgrad_kernel(const __grid_constant__ HdgradParams p, const __grid_constant__ CUtensorMap tmapDy,
                   const __grid_constant__ CUtensorMap tmapW) {
+  constexpr int CB = 128 / ELEM;                   // channels per 128-byte block
+  constexpr uint32_t FMT = ELEM == 2 ? 1u : 2u;    // instruction-descriptor operand format
+  constexpr int KIND = ELEM == 2 ? 0 : 1;          // kind::f16 / kind::tf32
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   const uint32_t base = (raw + 1023u) & ~1023u;
@@ -130,7 +138,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
         mbar_wait(aempty(as), aph ^ 1u);
         const uint32_t sA = sA0 + (uint32_t)(as * p.a_bytes);
         if (leader) mbar_arrive_expect_tx_e(afull(as), la ? (uint32_t)(2 * halo_rows * 128) : 0u);
-        if (la) tma_load_4d_cg2_e(sA, &tmapDy, mapa_shared(afull(as), 0), cb * 64, -p.Q, r0 - p.Q, n);
+        if (la) tma_load_4d_cg2_e(sA, &tmapDy, mapa_shared(afull(as), 0), cb * CB, -p.Q, r0 - p.Q, n);
         if (++as == SA) {
           as = 0;
           aph ^= 1u;
@@ -144,7 +152,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
           if (lb)
             for (int j = 0; j < nsub; ++j)
               tma_load_2d_cg2_e(sB + (uint32_t)(j * p.b_tap_bytes), &tmapW, mapa_shared(bfull(bs), 0),
-                                (t0 + j) * p.cop + cb * 64, (int)rank * half);
+                                (t0 + j) * p.cop + cb * CB, (int)rank * half);
           if (++bs == SB) {
             bs = 0;
             bph ^= 1u;
@@ -154,7 +162,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
     }
   } else if (warp == 5 && leader) {
     // ===================================== MMA issuer ======================================
-    const uint32_t idesc = make_idesc(1u, 0u, 0u, 256u, (uint32_t)p.bn);
+    const uint32_t idesc = make_idesc(FMT, 0u, 0u, 256u, (uint32_t)p.bn);
     const bool skip_mma = GLP_SKIP(p, 4);
     int as = 0, bs = 0;
     uint32_t aph = 0, bph = 0, it = 0;
@@ -182,7 +190,7 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
             const uint64_t sh = (uint64_t)((kh * p.WQ + (GLP_SKIP(p, 32) ? 0 : kw)) * 8);
             const uint64_t db = db0 + (uint64_t)(j * (p.b_tap_bytes >> 4));
             const uint32_t acc = (cb | t0 | j) ? 1u : 0u;
-            if (!skip_mma || (cb | t0 | j) == 0) mma_kblock_e<0, 2, 4, 2>(d0, da0 + sh, db, idesc, acc);
+            if (!skip_mma || (cb | t0 | j) == 0) mma_kblock_e<KIND, 2, 4, 2>(d0, da0 + sh, db, idesc, acc);
             if (++kw == p.K) {
               kw = 0;
               ++kh;

@@ -704,35 +704,38 @@ HDG_SHAPES = [
 ]
 
 
+@pytest.mark.parametrize("math", ["bf16", "tf32"])
 @pytest.mark.parametrize("shape", HDG_SHAPES, ids=lambda s: s[0])
-def test_halo_dgrad(shape):
-    """Shared-halo backward-data (4-D TMA halo of the packed dy per 64-channel block, flipped taps by
-    row shift, CTA pairs with M = 256 MMAs): bit-exact on integer data, within 1e-4
-    of the rounding-emulated oracle and 2e-2 of the fp64 oracle on random data, bitwise invariant
-    across samples-in-flight overrides."""
-    layer = _layer(shape, "bf16", halo_dgrad=2)
+def test_halo_dgrad(shape, math):
+    """Shared-halo backward-data (4-D TMA halo of the packed dy per 128-byte channel block -- 64
+    bf16 / 32 tf32 channels -- flipped taps by row shift, CTA pairs with M = 256 MMAs): bit-exact
+    on integer data, within 1e-4 of the rounding-emulated oracle and the mode's bar of the fp64
+    oracle on random data, bitwise invariant across samples-in-flight overrides."""
+    layer = _layer(shape, math, halo_dgrad=2)
     assert layer.info.dgrad_halo == 1
     d = _data(shape, exact=True, seed=53)
     got = _run(layer, d)
     ref = _oracle(d, shape[7], shape[8])
     np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32))
     d = _data(shape, seed=54)
-    runs = [_run(_layer(shape, "bf16", S, halo_dgrad=2), d)["dx"] for S in (0, 1, 0)]
+    runs = [_run(_layer(shape, math, S, halo_dgrad=2), d)["dx"] for S in (0, 1, 0)]
     ref = _oracle(d, shape[7], shape[8])["dx"]
-    emu = _oracle(d, shape[7], shape[8], x=EMU["bf16"](d["x"]), w=EMU["bf16"](d["w"]),
-                  dy=EMU["bf16"](d["dy"]))["dx"]
-    assert np.abs(runs[0] - ref).max() / np.abs(ref).max() <= TOL["bf16"]
+    emu = _oracle(d, shape[7], shape[8], x=EMU[math](d["x"]), w=EMU[math](d["w"]),
+                  dy=EMU[math](d["dy"]))["dx"]
+    assert np.abs(runs[0] - ref).max() / np.abs(ref).max() <= TOL[math]
     assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= 1e-4
     for other in runs[1:]:
         np.testing.assert_array_equal(other, runs[0])
 
 
 def test_halo_dgrad_model_choice():
-    """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) and
-    keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would be junk)."""
-    assert _layer(HDG_SHAPES[0], "bf16").info.dgrad_halo == 1
-    assert _layer(SHAPES[6], "bf16").info.dgrad_halo == 0
-    assert _layer(HDG_SHAPES[0], "tf32").info.dgrad_halo == 0
+    """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) in bf16
+    and tf32, keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would
+    be junk), and for 3xTF32 (no two-plane halo kernel)."""
+    for math in ("bf16", "tf32"):
+        assert _layer(HDG_SHAPES[0], math).info.dgrad_halo == 1
+        assert _layer(SHAPES[6], math).info.dgrad_halo == 0
+    assert _layer(HDG_SHAPES[0], "fp32").info.dgrad_halo == 0
 
 
 @pytest.mark.parametrize("ncg", ["1", "2"])

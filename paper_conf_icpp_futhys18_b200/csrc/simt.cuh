@@ -308,12 +308,12 @@ __device__ __forceinline__ void reduce_tc_dw_wide_body(const DwRed &rr, int bx, 
   }
 }
 
-// db[co] = sum over rows of part[row][co] (rows = N * pixel tiles, or SIMT splits), fixed order.
-// db[co] = sum over `rows` partial rows, deterministic and parallel over row groups:
-// grid (ceil(Co/32), DB_GROUPS).  Block (x, g) sums rows g, g+G, ... (thread ty takes every 8th of
-// those, lanes = channels, coalesced), reduces its 8 warps in a fixed tree, and stores part2[g][co];
-// the last block to finish for a channel group (atomic ticket) sums part2[0..G) in index order.
-// The order depends only on `rows` (a shape quantity), never on the grid size, S or timing.
+// db[co] = sum over `rows` partial rows of part[row][co] (rows = N * pixel tiles, or SIMT splits),
+// deterministic and parallel over G = db_groups(rows) row groups: block (channel block x, group g)
+// sums rows g, g+G, ... (thread ty takes every 8th of those, lanes = channels, coalesced), reduces
+// its 8 warps in a fixed tree, and stores part2[g][co]; the last block to finish for a channel
+// block (atomic ticket) sums part2[0..G) in index order.  The order depends only on `rows` (a
+// shape quantity), never on the grid size, S or timing.
 constexpr int DB_GROUPS = 128;   // the largest group count (multiple of 4)
 // Row groups of a db reduction over `rows` partial rows: ~32 rows per group, 4..DB_GROUPS, a
 // multiple of 4 -- a function of the row count only (small layers spent ~10 us in 128 nearly

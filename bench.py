@@ -33,7 +33,8 @@ from glp_workloads import CONFIG_NAMES, LEVELS, SHARED, SIBLINGS, config, gen_la
 
 METRIC = "conv fwd+bwd images/sec"
 # the arithmetic each --math mode computes in (fp32 = 3xTF32 on tcgen05: fp32-accurate)
-DTYPE = {"fp32": "fp32 (3xtf32)", "tf32": "tf32", "bf16": "bf16"}
+DTYPE = {"fp32": "fp32 (split: tf32 hi*hi + 2 bf16 cross terms; 3xtf32 on non-TMA layers)",
+         "tf32": "tf32", "bf16": "bf16"}
 UNIT = "images/s"
 NOMINAL_TF32_OVER_BF16 = 1.1 / 2.25   # B200_PROFILING.md nominal dense ratio
 
@@ -1033,7 +1034,12 @@ def make_roofline(args, states, kern, ms_per_step):
     fp32-equivalent flop, /3).  The sustained figure is given as context."""
     peaks = load_peaks()
     dom = max(kern, key=lambda r: r["total_us"])
-    ratio = {"bf16": 1.0, "tf32": NOMINAL_TF32_OVER_BF16, "fp32": NOMINAL_TF32_OVER_BF16 / 3}[args.math]
+    # fp32: the dominant kernel's own split -- 3xTF32 (three tf32 MMAs per flop: tf32 peak / 3)
+    # or the mixed split (one tf32 + two bf16 MMAs, bf16 at twice the tf32 rate: tf32 peak / 2)
+    mixed = args.math == "fp32" and any(getattr(s.conv.info, "fp32_split", 0) for s in states
+                                        if dom["layer"] == s.name)
+    ratio = {"bf16": 1.0, "tf32": NOMINAL_TF32_OVER_BF16,
+             "fp32": NOMINAL_TF32_OVER_BF16 / (2 if mixed else 3)}[args.math]
     peak_tf = peaks["bf16_tflops"] * ratio
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
@@ -1043,7 +1049,8 @@ def make_roofline(args, states, kern, ms_per_step):
         except Exception:
             traffic = None
     src = {"bf16": " bf16 burst", "tf32": " bf16 burst x 1.1/2.25 (tf32)",
-           "fp32": " bf16 burst x 1.1/2.25 / 3 (3xTF32: three tf32 MMAs per flop)"}[args.math]
+           "fp32": (" bf16 burst x 1.1/2.25 / 2 (mixed split: one tf32 + two bf16 MMAs per flop)"
+                    if mixed else " bf16 burst x 1.1/2.25 / 3 (3xTF32: three tf32 MMAs per flop)")}[args.math]
     out = {"bound": "tensor", "achieved": dom["tflops"], "peak": round(peak_tf, 1),
            "unit": "TFLOP/s", "frac": round(dom["tflops"] / peak_tf, 4), "traffic": traffic,
            "kernel": f"{kernel_name(states, dom)} {dom['layer']} {dom['pass']}",
@@ -1051,8 +1058,9 @@ def make_roofline(args, states, kern, ms_per_step):
            "share_of_step": round(dom["total_us"] / 1e3 / (ms_per_step * args.steps), 4),
            "frac_of_sustained_peak": round(dom["tflops"] / (peaks["bf16_tflops_sustained"] * ratio), 4)}
     if args.math == "fp32":
-        # the same kernel against the tensor pipe's nominal tf32 rate (1.1 PF/s dense, /3)
-        out["frac_of_nominal_tf32"] = round(dom["tflops"] / (1100.0 / 3), 4)
+        # the same kernel against the tensor pipe's nominal tf32 rate (1.1 PF/s dense, /2 or /3)
+        out["frac_of_nominal_tf32"] = round(dom["tflops"] / (1100.0 / (2 if mixed else 3)), 4)
+        out["fp32_split"] = "tf32 hi*hi + 2 bf16 cross terms" if mixed else "3xTF32"
     return out
 
 

@@ -254,6 +254,15 @@ def split_3xtf32(a):
     return hi, lo
 
 
+def split_mixed(a):
+    """Mixed fp32 split (DESIGN.md §7 "1xTF32 + 2xBF16"): hi = rna_tf32(a), bhi = rne_bf16(hi),
+    blo = rne_bf16(a - hi) (fp32 subtraction, exact).  The products the MMAs form are hi*hi (tf32),
+    bhi*blo' and blo*bhi' (bf16); a product a*b' is then represented to ~2^-18 of |a b'|."""
+    a = _f32(a)
+    hi = round_tf32_rna(a)
+    return hi, round_bf16_rne(hi), round_bf16_rne((a - hi).astype(np.float32))
+
+
 def normwise_err(got, ref):
     """DESIGN.md R11: max_i |g_i - r_i| / max_i |r_i| (per tensor)."""
     ref = np.asarray(ref, np.float64)

@@ -39,7 +39,7 @@ class PlanInfo(ctypes.Structure):
                 ("wgrad_halo", _c_int), ("fwd_halo", _c_int),
                 ("wgrad_fused_dy", _c_int), ("dgrad_halo", _c_int),
                 ("s_slot_rows", ctypes.c_longlong), ("s_rows_per_sample", ctypes.c_longlong),
-                ("wgrad_reduce_wide", _c_int)]
+                ("wgrad_reduce_wide", _c_int), ("fp32_split", _c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -63,7 +63,7 @@ class PlanOptions(ctypes.Structure):
                 ("fused_dy_builders", _c_int), ("max_kblocks_per_stage", _c_int),
                 ("wgrad_tile_n", _c_int), ("tile_units", _c_int), ("bn_model", _c_int),
                 ("pack_block", _c_int), ("s2d_block", _c_int), ("smem_cap", _c_int), ("pdl", _c_int),
-                ("wgrad_leaves", _c_int)]
+                ("wgrad_leaves", _c_int), ("fp32_split", _c_int)]
 
 
 def plan_options(**kw) -> PlanOptions:

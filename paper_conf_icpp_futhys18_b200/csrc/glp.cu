@@ -208,9 +208,11 @@ void *kernel_ptr() {
 template <int MODE, int CG>
 void *igemm_ptr_m(int elem, int krow, int x3) {
   if (elem == 2) return krow == 128 ? kernel_ptr<MODE, 2, 128, CG, 0>() : kernel_ptr<MODE, 2, 64, CG, 0>();
+  if (x3 == 2) return kernel_ptr<MODE, 4, 128, CG, 2>();
   return x3 ? kernel_ptr<MODE, 4, 128, CG, 1>() : kernel_ptr<MODE, 4, 128, CG, 0>();
 }
-// x3: the 3xTF32 variant (GLP_MATH_FP32: hi/lo operand planes, three MMAs per k-step)
+// x3: 1 = the 3xTF32 variant (GLP_MATH_FP32: hi/lo operand planes, three MMAs per k-step);
+// 2 = the mixed split (tf32 hi*hi + two bf16 cross terms)
 void *igemm_ptr(int mode, int elem, int krow, int cg, int x3) {
   if (cg == 2) {
     if (mode == MODE_FWD) return igemm_ptr_m<MODE_FWD, 2>(elem, krow, x3);
@@ -314,7 +316,7 @@ int choose_splits(int tiles_mn, int kb_total, int bn, int mpad, int npad, int el
 struct MapCache {
   struct Entry {
     const void *ws = nullptr;
-    CUtensorMap a, b, a2, b2;   // a2, b2: the lo planes of a 3xTF32 plan
+    CUtensorMap a, b, a2, b2, a3, b3;   // a2, b2: lo planes (3xTF32) / bf16(hi) (mixed); a3, b3: bf16(v - hi)
   };
   Entry e[3][8];
   int next[3] = {0, 0, 0};
@@ -363,6 +365,7 @@ struct glp_plan_s {
   // taps, W' resident per CTA, outputs on the padded grid (invalid rows dropped)
   int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
   int red_wide = 0;     // dW reduction by reduce_tc_dw_wide (small filters, many splits)
+  int mix = 0;          // GLP_MATH_FP32 by the mixed split (tf32 hi*hi + bf16 cross terms)
   int hdg = 0;         // halo backward-data (hdgrad.cuh) for unit-stride layers where it pays
   HdgradParams hd{};
   int hd_grid = 0, hd_smem = 0;
@@ -754,6 +757,10 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   // 3xTF32 accumulation chunk (shape-only constant: 16 k-blocks = K 512): bounds the error of the
   // tensor core's round-toward-zero accumulation to ~1e-6 normwise
   pp.chunk_kb = P.x3 ? 16 : 0;
+#ifdef GLP_DIAG
+  if (const char *e = getenv("GLP_DEBUG_CHUNK"))   // diagnostics: chunk length A/B
+    if (P.x3) pp.chunk_kb = std::max(1, atoi(e));
+#endif
   const int a_bytes = planes * (mode == MODE_WGRAD ? 128 * BKP * elem : 128 * pp.krow);
   const int b_row = planes * (mode == MODE_WGRAD ? BKP * elem : pp.krow);
   // forward: the bias vector is staged once per CTA in smem (every column a tile can touch)
@@ -784,7 +791,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   pp.smem = 1024 + pp.stages * stage_bytes + 8 * (2 * pp.stages + 4) + 16 + 16 + 4 * pp.bias_floats;
   pp.tiles = pp.m_units * pp.n_tiles * pp.splits;   // work units (tile pairs for cg = 2)
 
-  void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg, P.x3);
+  void *fn = igemm_ptr(mode, elem, pp.krow, pp.cg, P.mix ? 2 : P.x3);
   // The attribute is per function (not per plan): always allow the largest tile of any plan.
   GLP_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
   cudaFuncAttributes fa;
@@ -819,7 +826,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
 // The tensor maps of one pass: A (activation gather), B (dense operand) and, for 3xTF32 plans,
 // the same two over the lo planes.
 struct Maps {
-  CUtensorMap a, b, a2, b2;
+  CUtensorMap a, b, a2, b2, a3, b3;
 };
 
 glp_status_t validate_ptrs(std::initializer_list<const void *> ps) {
@@ -905,7 +912,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
 template <int MODE>
 glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmParams &p,
                           const Maps &m, cudaStream_t st) {
-  void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg, P.x3);
+  void *fn = igemm_ptr(MODE, P.elem, pp.krow, pp.cg, P.mix ? 2 : P.x3);
   cudaLaunchConfig_t cfg;
   memset(&cfg, 0, sizeof(cfg));
   cfg.gridDim = dim3((unsigned)pp.grid);
@@ -921,11 +928,13 @@ glp_status_t launch_igemm(const glp_plan_s &P, const PassPlan &pp, const IgemmPa
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = P.pdl ? 2 : 1;
-  // single-plane plans pass their hi maps again in the lo slots (never read)
+  // plans with fewer planes pass their hi maps again in the unused slots (never read)
   const CUtensorMap &b2 = P.x3 ? m.b2 : m.b, &a2 = P.x3 ? m.a2 : m.a;
+  const CUtensorMap &b3 = P.mix ? m.b3 : m.b, &a3 = P.mix ? m.a3 : m.a;
   void *args[] = {const_cast<IgemmParams *>(&p), const_cast<CUtensorMap *>(&m.b),
                   const_cast<CUtensorMap *>(&m.a), const_cast<CUtensorMap *>(&b2),
-                  const_cast<CUtensorMap *>(&a2)};
+                  const_cast<CUtensorMap *>(&a2), const_cast<CUtensorMap *>(&b3),
+                  const_cast<CUtensorMap *>(&a3)};
   GLP_CUDA(cudaLaunchKernelExC(&cfg, fn, args));
   GLP_LAUNCH_CHECK("igemm_kernel");
   return GLP_OK;
@@ -970,6 +979,24 @@ DbAux db_aux(const glp_plan_s &P, uint8_t *base, int rows) {
 }
 
 // lo: byte offset of dst's lo plane (3xTF32 plans: the region's lo_* offset; 0 otherwise)
+// Operand planes of a plan (1; 3xTF32: hi, lo; mixed: hi, bf16(hi), bf16(v - hi)), the byte
+// offset of plane pl from the hi plane (L = the hi plane's bytes), its element size and the TMA
+// swizzle of its 128-row k-block tiles (the bf16 planes of the mixed split are 64-byte rows).
+int nplanes(const glp_plan_s &P) { return P.mix ? 3 : (P.x3 ? 2 : 1); }
+long long plane_offset(const glp_plan_s &P, int pl, long long L) {
+  return pl == 0 ? 0 : (P.mix && pl == 2 ? L + L / 2 : L);
+}
+int plane_elem(const glp_plan_s &P, int pl) { return (P.mix && pl) ? 2 : P.elem; }
+CUtensorMap *plane_map(CUtensorMap *m1, CUtensorMap *m2, CUtensorMap *m3, int pl) {
+  return pl == 0 ? m1 : pl == 1 ? m2 : m3;
+}
+// The packs' plane argument (pack.cuh plane_off): 3xTF32, the lo plane's byte offset L (the hi
+// plane's bytes); the mixed split, -((L/2) << 32 | (L - delta/2)) -- the bf16(hi) plane's byte
+// offset from a destination pointer `delta` bytes into the hi plane, and the bf16 plane size.
+long long plo(const glp_plan_s &P, long long L, long long delta = 0) {
+  if (!P.mix) return L;
+  return -(long long)(((unsigned long long)(L / 2) << 32) | (unsigned long long)(L - delta / 2));
+}
 glp_status_t launch_pack_act(const glp_plan_s &P, const float *src, void *dst, long long lo, int C,
                              int HW, int Cp, float *db_part, cudaStream_t st, int Ws = 1,
                              int Wd = 1, int HWd = -1, int co_off = 0, int Cw = -1, int db_ld = -1,
@@ -1014,12 +1041,12 @@ glp_status_t launch_pack_dy(const glp_plan_s &P, const BrIn &dy, uint8_t *ws, bo
   const int Ws = P.halo ? d.Wo : 1, Wd = P.halo ? P.dxg.W : 1;
   const int HWd = P.halo ? P.dxg.H * P.dxg.W : -1;
   if (dy.n <= 1)
-    return launch_pack_act(P, dy.p[0], ws + P.off_dypk, P.lo_dypk, d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
+    return launch_pack_act(P, dy.p[0], ws + P.off_dypk, plo(P, P.lo_dypk), d.Co, d.Ho * d.Wo, P.Cop, dbp, st, Ws, Wd,
                            HWd, 0, -1, -1, P.y_img_c);
   for (int b = 0; b < dy.n; ++b) {
     const int off = d.br_off[b], cb = d.br_off[b + 1] - off;
     const int cw = (b == dy.n - 1) ? P.Cop - off : cb;
-    glp_status_t s = launch_pack_act(P, dy.p[b], ws + P.off_dypk, P.lo_dypk, cb, d.Ho * d.Wo, P.Cop, dbp, st,
+    glp_status_t s = launch_pack_act(P, dy.p[b], ws + P.off_dypk, plo(P, P.lo_dypk), cb, d.Ho * d.Wo, P.Cop, dbp, st,
                                      Ws, Wd, HWd, off, cw, d.Co);
     if (s) return s;
   }
@@ -1035,7 +1062,7 @@ glp_status_t run_pack_w_fwd_one(glp_plan_s &P, const float *w, int co_off, int C
   d.Co = Co;   // rows [co_off, co_off + Co) of the forward B operand
   void *wpk = ws + P.off_wpk + (size_t)co_off * P.fwd.Kpad * P.elem;
   const size_t wn = (size_t)d.Co * P.fwd.Kpad;
-  const long long lo = P.lo_wpk;
+  const long long lo = plo(P, P.lo_wpk, (long long)co_off * P.fwd.Kpad * P.elem);
   if (P.s2d) {
     if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_w_fwd_s2d<2>, dim3(ew_grid(wn)), dim3(256), 0, st, w, wpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cpx, P.fwd.Kpad, 0LL));
@@ -1076,14 +1103,14 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
       if (P.elem == 2)
         GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<2, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
       else
-        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<4, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
+        GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp_t<4, 4, 3>, grid, dim3(128), 0, st, x, dst, d.N, d.H, d.W, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, plo(P, P.lo_xpk)));
       GLP_LAUNCH_CHECK("pack_s2d_warp_t");
       return GLP_OK;
     }
     if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<2>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<4>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d_warp<4>, grid, dim3(128), 0, st, x, dst, d.N, d.C, d.H, d.W, P.s2d, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, plo(P, P.lo_xpk)));
     GLP_LAUNCH_CHECK("pack_s2d_warp");
     return GLP_OK;
   }
@@ -1098,11 +1125,11 @@ glp_status_t launch_pack_x(const glp_plan_s &P, const float *x, void *dst, cudaS
     if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_s2d<2>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, P.lo_xpk));
+      GLP_CUDA(launch_pdl(P.pdl, pack_s2d<4>, dim3(grid), dim3(256), smem, st, x, dst, d.N, d.C, d.H, d.W, S, d.Ph, P.dxg.H, P.dxg.W, P.Cpx, P.x_img_c, plo(P, P.lo_xpk)));
     GLP_LAUNCH_CHECK("pack_s2d");
     return GLP_OK;
   }
-  return launch_pack_act(P, x, dst, P.lo_xpk, d.C, d.H * d.W, P.Cpx, nullptr, st, 1, 1, -1, 0, -1,
+  return launch_pack_act(P, x, dst, plo(P, P.lo_xpk), d.C, d.H * d.W, P.Cpx, nullptr, st, 1, 1, -1, 0, -1,
                          -1, P.x_img_c);
 }
 
@@ -1121,11 +1148,11 @@ glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStr
       if (P.elem == 2)
         GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<2>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, 0LL));
       else
-        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<4>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, P.lo_wtpk));
+        GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_rows<4>, dim3((unsigned)d.C), dim3(256), sm, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, plo(P, P.lo_wtpk)));
     } else if (P.elem == 2)
       GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<2>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, 0LL));
     else
-      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, P.lo_wtpk));
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad<4>, grid, dim3(256), 0, st, w.p[b], wtpk, co, d.C, P.taps, P.Cop, P.dgrad.Kpad, flip, off, off, hi, plo(P, P.lo_wtpk)));
     GLP_LAUNCH_CHECK("pack_w_dgrad");
   }
   return GLP_OK;
@@ -1149,7 +1176,7 @@ glp_status_t run_pack_w_both(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStre
   if (P.elem == 2)
     GLP_CUDA(launch_pdl(P.pdl, pack_w_both<2>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip, 0LL, 0LL));
   else
-    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<4>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip, P.lo_wpk, P.lo_wtpk));
+    GLP_CUDA(launch_pdl(P.pdl, pack_w_both<4>, grid, dim3(256), smem, st, w.p[0], wp, wt, d.Co, d.C, P.taps, P.Cpx, P.Cop, P.fwd.Kpad, P.dgrad.Kpad, flip, plo(P, P.lo_wpk), plo(P, P.lo_wtpk)));
   GLP_LAUNCH_CHECK("pack_w_both");
   return GLP_OK;
 }
@@ -1179,6 +1206,8 @@ glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, Maps &m, F enc
       m.b = e.b;
       m.a2 = e.a2;
       m.b2 = e.b2;
+      m.a3 = e.a3;
+      m.b3 = e.b3;
       return GLP_OK;
     }
   memset(&m, 0, sizeof(m));
@@ -1191,6 +1220,8 @@ glp_status_t cached_maps(glp_plan_s &P, int pass, const void *ws, Maps &m, F enc
   e.b = m.b;
   e.a2 = m.a2;
   e.b2 = m.b2;
+  e.a3 = m.a3;
+  e.b3 = m.b3;
   return GLP_OK;
 }
 
@@ -1263,17 +1294,19 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
   const int BK = pp.krow / P.elem;
   Maps m;
   glp_status_t s = cached_maps(P, 0, ws, m, [&](Maps &q) {
-    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
-      const long long lw = pl ? P.lo_wpk : 0, lx = pl ? P.lo_xpk : 0;
-      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<uint8_t *>(wpk) + lw,
-                                 (uint64_t)pp.Kpad, (uint64_t)d.Co, (uint64_t)pp.Kpad * P.elem,
-                                 (uint32_t)BK, (uint32_t)pp.bn_smem, swz_kmajor(pp.krow));
+    for (int pl = 0; pl < nplanes(P); ++pl) {   // hi plane, then the lo / bf16 planes
+      const long long lw = plane_offset(P, pl, P.lo_wpk), lx = plane_offset(P, pl, P.lo_xpk);
+      const int e = plane_elem(P, pl);
+      const CUtensorMapSwizzle sw = swz_kmajor(e * BK);   // 128- or 64-byte rows
+      glp_status_t r = encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<uint8_t *>(wpk) + lw,
+                                 (uint64_t)pp.Kpad, (uint64_t)d.Co, (uint64_t)pp.Kpad * e,
+                                 (uint32_t)BK, (uint32_t)pp.bn_smem, sw);
       if (r) return r;
       if (!pp.a_tma) continue;
       if ((r = get_encode_im2col())) return r;
-      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<uint8_t *>(xpk) + lx, P.Cpx, d.W,
+      r = encode_im2col(plane_map(&q.a, &q.a2, &q.a3, pl), e, static_cast<uint8_t *>(xpk) + lx, P.Cpx, d.W,
                         d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1), d.Ph - (d.Kh - 1), BK, 128,
-                        d.Sw, d.Sh, swz_kmajor(pp.krow));
+                        d.Sw, d.Sh, sw);
       if (r) return r;
     }
     return GLP_OK;
@@ -1352,18 +1385,20 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   const int BK = pp.krow / P.elem;
   Maps m;
   glp_status_t s = cached_maps(P, 1, ws, m, [&](Maps &q) {
-    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
-      const long long lw = pl ? P.lo_wtpk : 0, ld = pl ? P.lo_dypk : 0;
-      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<uint8_t *>(wtpk) + lw,
-                                 (uint64_t)pp.Kpad, (uint64_t)d.C, (uint64_t)pp.Kpad * P.elem,
-                                 (uint32_t)BK, (uint32_t)pp.bn_smem, swz_kmajor(pp.krow));
+    for (int pl = 0; pl < nplanes(P); ++pl) {   // hi plane, then the lo / bf16 planes
+      const long long lw = plane_offset(P, pl, P.lo_wtpk), ld = plane_offset(P, pl, P.lo_dypk);
+      const int e = plane_elem(P, pl);
+      const CUtensorMapSwizzle sw = swz_kmajor(e * BK);   // 128- or 64-byte rows
+      glp_status_t r = encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<uint8_t *>(wtpk) + lw,
+                                 (uint64_t)pp.Kpad, (uint64_t)d.C, (uint64_t)pp.Kpad * e,
+                                 (uint32_t)BK, (uint32_t)pp.bn_smem, sw);
       if (r) return r;
       if (!pp.a_tma) continue;
       // dx pixel (h, w) reads dy at (h - (Kh-1-Ph) + kh', w - (Kw-1-Pw) + kw') with kh' = Kh-1-kh
       if ((r = get_encode_im2col())) return r;
-      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<const uint8_t *>(dypk) + ld, P.Cop,
+      r = encode_im2col(plane_map(&q.a, &q.a2, &q.a3, pl), e, static_cast<const uint8_t *>(dypk) + ld, P.Cop,
                         d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw), -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK,
-                        128, 1, 1, swz_kmajor(pp.krow));
+                        128, 1, 1, sw);
       if (r) return r;
     }
     return GLP_OK;
@@ -1435,18 +1470,21 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
   const int BKP = 128 / P.elem, EPA = pp.krow / P.elem;
   Maps m;
   glp_status_t s = cached_maps(P, 2, ws, m, [&](Maps &q) {
-    for (int pl = 0; pl < (P.x3 ? 2 : 1); ++pl) {   // hi plane, then (3xTF32) the lo plane
-      const long long ld = pl ? P.lo_dypk : 0, lx = pl ? P.lo_xpk : 0;
-      glp_status_t r = encode_2d(pl ? &q.b2 : &q.b, P.elem, static_cast<const uint8_t *>(dypk) + ld,
+    for (int pl = 0; pl < nplanes(P); ++pl) {   // hi plane, then the lo / bf16 planes
+      const long long ld = plane_offset(P, pl, P.lo_dypk), lx = plane_offset(P, pl, P.lo_xpk);
+      const int e = plane_elem(P, pl);
+      // MN-major atoms of EPA elements: 32 tf32 (128-byte rows, 32-byte swizzle base) or, for the
+      // bf16 planes of the mixed split, 32 bf16 (64-byte rows, SWIZZLE_64B)
+      const CUtensorMapSwizzle sw = e == P.elem ? swz_mnmajor(P.elem, pp.krow) : CU_TENSOR_MAP_SWIZZLE_64B;
+      glp_status_t r = encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<const uint8_t *>(dypk) + ld,
                                  (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
-                                 (uint64_t)P.Cop * P.elem, (uint32_t)EPA, (uint32_t)BKP,
-                                 swz_mnmajor(P.elem, pp.krow));
+                                 (uint64_t)P.Cop * e, (uint32_t)EPA, (uint32_t)BKP, sw);
       if (r) return r;
       if (!pp.a_tma) continue;
       if ((r = get_encode_im2col())) return r;
-      r = encode_im2col(pl ? &q.a2 : &q.a, P.elem, static_cast<const uint8_t *>(xpk) + lx, P.Cpx,
+      r = encode_im2col(plane_map(&q.a, &q.a2, &q.a3, pl), e, static_cast<const uint8_t *>(xpk) + lx, P.Cpx,
                         d.W, d.H, d.N, -d.Pw, -d.Ph, d.Pw - (d.Kw - 1), d.Ph - (d.Kh - 1), EPA,
-                        BKP, d.Sw, d.Sh, swz_mnmajor(P.elem, pp.krow));
+                        BKP, d.Sw, d.Sh, sw);
       if (r) return r;
     }
     return GLP_OK;
@@ -1811,7 +1849,7 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
 
 glp_status_t glp_plan_options_default(glp_plan_options_t *o) {
   if (!o) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
-  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 6, 1, 0, 0, 232448, 0, 0};
+  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 6, 1, 0, 0, 232448, 0, 0, 1};
   return GLP_OK;
 }
 
@@ -1831,6 +1869,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
       o.smem_cap > 232448 || (o.wgrad_leaves != 0 && o.wgrad_leaves != 1 && o.wgrad_leaves != 2 &&
                               o.wgrad_leaves != 4 && o.wgrad_leaves != 8))
     return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
+  if (o.fp32_split < 0 || o.fp32_split > 1) return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
   if (o.wgrad_leaves > 0 && (math == GLP_MATH_FP32_SIMT || d->nbr > 1))
     return fail(GLP_ERR_NOT_SUPPORTED, "wgrad leaves: tensor-core single-layer plans only");
   *out = nullptr;
@@ -1956,12 +1995,23 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
                                                std::to_string(ch) + " == 0");
       }
   }
+  // the mixed fp32 split (option fp32_split): every pass must take its operands by TMA with
+  // 128-byte tf32 rows (the packs write one representation for all three passes): channel
+  // pitches multiples of 32 and unit stride (the backward-data TMA gather)
+  P->mix = (P->x3 && o.fp32_split && P->Cpx % 32 == 0 && P->Cop % 32 == 0 && P->d.Sh == 1 &&
+            P->d.Sw == 1) ? 1 : 0;
   if (!P->simt) {
     if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
         (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {
       delete P;
       if (cur != device) cudaSetDevice(cur);
       return s;
+    }
+    if (P->mix && !(P->fwd.a_tma && P->dgrad.a_tma && P->wgrad.a_tma && P->fwd.krow == 128 &&
+                    P->dgrad.krow == 128 && P->wgrad.krow == 128)) {
+      delete P;
+      if (cur != device) cudaSetDevice(cur);
+      return fail(GLP_ERR_INTERNAL, "mixed fp32 split planned for a non-TMA pass");
     }
     if ((s = plan_halo(*P)) || (s = plan_hfwd(*P)) || (s = plan_hdgrad(*P))) {
       delete P;
@@ -2090,6 +2140,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->s_slot_rows = P->s_slot_rows;
   I->s_rows_per_sample = P->s_rows_per_sample;
   I->wgrad_reduce_wide = P->red_wide;
+  I->fp32_split = P->mix;
   if (P->hdg) {
     I->grid_bwd_data = P->hd_grid;
     I->tile_n_bwd_data = P->hd.bn;
@@ -2476,7 +2527,7 @@ glp_status_t glp_debug_im2col(glp_plan_t P, const float *x, int n, float *col, v
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   uint8_t *wsb = static_cast<uint8_t *>(ws);
   void *xpk = wsb + P->off_xpk;
-  if ((s = launch_pack_act(*P, x, xpk, P->lo_xpk, P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st)))
+  if ((s = launch_pack_act(*P, x, xpk, plo(*P, P->lo_xpk), P->d.C, P->d.H * P->d.W, P->Cp, nullptr, st)))
     return s;
   // the direct (non space-to-depth) gather geometry of the layer
   glp_plan_s Q = *P;

@@ -126,17 +126,34 @@ __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS,
 // half of the tile's columns per warp (warp w: TMEM lanes 32*(w%4), columns half w/4) -- then
 // store the sum.  The buffers alternate chunk by chunk across tiles, so the MMA issuer never
 // waits for the final stores.
+//
+// X3 = 2 (GLP_MATH_FP32 with plan option fp32_split = 1): the mixed split.  The packs write a tf32
+// hi plane and two bf16 planes, bf16(hi) and bf16(v - hi) (pack.cuh); a k-block slot holds
+// [A_hi | A_bhi | A_blo] and [B_hi | B_bhi | B_blo] (the bf16 tiles are 64-byte rows: K-major
+// SWIZZLE_64B, or MN-major 32-element SWIZZLE_64B atoms), the same bytes as 3xTF32's two planes;
+// tmapA2 / tmapB2 are the bf16(hi) planes, tmapA3 / tmapB3 the bf16(v - hi) planes.  The MMA
+// issuer runs hi*hi in tf32 and the two cross terms in bf16 (mma_kblock_mix_e): 8 MMA issue slots
+// per k-block instead of 12.  TMA operands only (the plan refuses the split for cp.async layers);
+// the chunked accumulation and the epilogue are those of X3 = 1.
 template <int MODE, int ELEM, int KROW, int CG, int X3>
 __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
     igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB,
                  const __grid_constant__ CUtensorMap tmapA, const __grid_constant__ CUtensorMap tmapB2,
-                 const __grid_constant__ CUtensorMap tmapA2) {
+                 const __grid_constant__ CUtensorMap tmapA2, const __grid_constant__ CUtensorMap tmapB3,
+                 const __grid_constant__ CUtensorMap tmapA3) {
   using C = TileCfg<ELEM, KROW>;
   static_assert(!X3 || (ELEM == 4 && KROW == 128), "3xTF32 uses 128-byte tf32 rows");
+  constexpr bool MIX = X3 == 2;
   constexpr int EW = X3 ? 8 : 4;    // epilogue warps 0 .. EW-1
   constexpr int PW = EW;            // producer warps PW .. PW+3 (TMA: warp PW alone)
   constexpr int MW = EW + 4;        // TMEM allocator + MMA issuer
-  constexpr uint32_t PL = X3 ? 2u : 1u;                 // operand planes (hi, lo)
+  constexpr uint32_t PL = X3 ? 2u : 1u;                 // operand planes' bytes (hi, lo)
+  constexpr uint32_t NPL = MIX ? 3u : PL;               // loaded planes (mixed: hi, bhi, blo)
+  // byte offset of plane pl in a k-block's A or B slot of one-plane size `one`: 3xTF32 lo at
+  // +one; mixed bf16(hi) at +one, bf16(v - hi) at +1.5 one (2-byte elements)
+  auto plane_byte_off = [](uint32_t pl, uint32_t one) -> uint32_t {
+    return pl == 0 ? 0u : (MIX && pl == 2) ? one + one / 2 : one;
+  };
   constexpr uint32_t A_BYTES1 = C::a_bytes(MODE);       // one plane of one k-block's A
   constexpr uint32_t A_BYTES = PL * A_BYTES1;
   extern __shared__ uint8_t smem_raw[];
@@ -189,6 +206,10 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
     if (X3) {
       tma_prefetch(&tmapB2);
       if (a_tma) tma_prefetch(&tmapA2);
+    }
+    if (MIX) {
+      tma_prefetch(&tmapB3);
+      tma_prefetch(&tmapA3);
     }
   }
   tc_fence_before();
@@ -302,19 +323,21 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
               const uint32_t sB = stg + sB_off + (uint32_t)sub * b_bytes;
               if (MODE != MODE_WGRAD) {
 #pragma unroll
-                for (uint32_t pl = 0; pl < PL; ++pl) {
-                  const CUtensorMap *mA = pl ? &tmapA2 : &tmapA, *mB = pl ? &tmapB2 : &tmapB;
+                for (uint32_t pl = 0; pl < NPL; ++pl) {
+                  const CUtensorMap *mA = pl == 0 ? &tmapA : pl == 1 ? &tmapA2 : &tmapA3;
+                  const CUtensorMap *mB = pl == 0 ? &tmapB : pl == 1 ? &tmapB2 : &tmapB3;
+                  const uint32_t oA = plane_byte_off(pl, A_BYTES1), oB = plane_byte_off(pl, b_bytes1);
                   if (la) {
                     if (CG == 1)
-                      tma_load_im2col_4d_e(sA + pl * A_BYTES1, mA, bar, cb * C::BK, w_t, h_t,
+                      tma_load_im2col_4d_e(sA + oA, mA, bar, cb * C::BK, w_t, h_t,
                                            (int)n_t, (uint16_t)kw, (uint16_t)kh);
                     else
-                      tma_load_im2col_4d_cg2_e(sA + pl * A_BYTES1, mA, bar, cb * C::BK, w_t, h_t,
+                      tma_load_im2col_4d_cg2_e(sA + oA, mA, bar, cb * C::BK, w_t, h_t,
                                                (int)n_t, (uint16_t)kw, (uint16_t)kh);
                   }
                   if (lb) {
-                    if (CG == 1) tma_load_2d_e(sB + pl * b_bytes1, mB, bar, kb * C::BK, nb0);
-                    else tma_load_2d_cg2_e(sB + pl * b_bytes1, mB, bar, kb * C::BK, nb0);
+                    if (CG == 1) tma_load_2d_e(sB + oB, mB, bar, kb * C::BK, nb0);
+                    else tma_load_2d_cg2_e(sB + oB, mB, bar, kb * C::BK, nb0);
                   }
                 }
                 if (++cb == cbs) {
@@ -330,27 +353,30 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
                 g.div_w.divmod(rem, oh, ow);
                 const int h0 = (int)oh * g.im_sh - g.im_ph, w0 = (int)ow * g.im_sw - g.im_pw;
 #pragma unroll
-                for (uint32_t pl = 0; pl < PL; ++pl) {
-                  const CUtensorMap *mA = pl ? &tmapA2 : &tmapA, *mB = pl ? &tmapB2 : &tmapB;
-                  const uint32_t pA = sA + pl * A_BYTES1, pB = sB + pl * b_bytes1;
+                for (uint32_t pl = 0; pl < NPL; ++pl) {
+                  const CUtensorMap *mA = pl == 0 ? &tmapA : pl == 1 ? &tmapA2 : &tmapA3;
+                  const CUtensorMap *mB = pl == 0 ? &tmapB : pl == 1 ? &tmapB2 : &tmapB3;
+                  const uint32_t pA = sA + plane_byte_off(pl, A_BYTES1), pB = sB + plane_byte_off(pl, b_bytes1);
+                  // MN atom stride: the bf16 planes of the mixed split have 64-byte atom rows
+                  const uint32_t lbo = (MIX && pl) ? C::MN_LBO / 2 : C::MN_LBO;
                   if (la) {
 #pragma unroll
                     for (int a = 0; a < NA; ++a) {
                       if (CG == 1)
-                        tma_load_im2col_4d_e(pA + (uint32_t)a * C::MN_LBO, mA, bar, ac[a], w0,
+                        tma_load_im2col_4d_e(pA + (uint32_t)a * lbo, mA, bar, ac[a], w0,
                                              h0, (int)n, akw[a], akh[a]);
                       else
-                        tma_load_im2col_4d_cg2_e(pA + (uint32_t)a * C::MN_LBO, mA, bar, ac[a],
+                        tma_load_im2col_4d_cg2_e(pA + (uint32_t)a * lbo, mA, bar, ac[a],
                                                  w0, h0, (int)n, akw[a], akh[a]);
                     }
                   }
                   if (lb) {
                     for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
                       if (CG == 1)
-                        tma_load_2d_e(pB + (uint32_t)a * C::MN_LBO, mB, bar, nb0 + a * C::EPA,
+                        tma_load_2d_e(pB + (uint32_t)a * lbo, mB, bar, nb0 + a * C::EPA,
                                       kb * C::BKP);
                       else
-                        tma_load_2d_cg2_e(pB + (uint32_t)a * C::MN_LBO, mB, bar,
+                        tma_load_2d_cg2_e(pB + (uint32_t)a * lbo, mB, bar,
                                           nb0 + a * C::EPA, kb * C::BKP);
                     }
                   }
@@ -365,6 +391,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
       }
     } else if (KROW == 128 && CG == 1) {
       // -------- cp.async gather (SWIZZLE_128B layouts only) --------
+      if (MIX) __trap();   // the mixed split is planned for TMA operands only
       int rs = 0;          // ring slot and its phase, advanced incrementally
         uint32_t rph = 0;
       for (int tile = unit0; tile < total_tiles; tile += ustep) {
@@ -527,6 +554,23 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
       }
       const uint64_t stage16 = stage_bytes >> 4, b16 = b_bytes >> 4;
       const uint64_t alo16 = A_BYTES1 >> 4, blo16 = b_bytes1 >> 4;   // lo planes (X3)
+      // mixed split: descriptors of the bf16(hi) planes as a constant difference to the tf32 hi
+      // descriptor of the same slot (start address + plane offset, bf16 layout fields), and the
+      // bf16(v - hi) planes half a tf32 plane further; bf16 tiles are 64-byte rows (SWIZZLE_64B)
+      uint64_t dA1 = 0, dB1 = 0;
+      const uint64_t ablo16 = (A_BYTES1 / 2) >> 4, bblo16 = (b_bytes1 / 2) >> 4;
+      const uint32_t idesc_b = make_idesc(1u, mn, mn, 128u * CG, (uint32_t)p.bn);
+      constexpr int BSTEP = (MODE == MODE_WGRAD) ? (16 * 64) >> 4 : 32 >> 4;
+      if (MIX) {
+        const uint32_t aB = base + A_BYTES1, bB = base + (uint32_t)p.ksub * A_BYTES + b_bytes1;
+        const uint64_t a1 = (MODE == MODE_WGRAD) ? make_sdesc(aB, C::MN_LBO / 2, 512u, 4u)
+                                                 : make_sdesc(aB, 16u, 512u, 4u);
+        const uint64_t b1 = (MODE == MODE_WGRAD) ? make_sdesc(bB, C::MN_LBO / 2, 512u, 4u)
+                                                 : make_sdesc(bB, 16u, 512u, 4u);
+        dA1 = a1 - da0;
+        dB1 = b1 - db0;
+      }
+      (void)idesc_b;
       const int KS = p.ksub, kb_total = p.kb_total;
       const bool skip_mma = GLP_SKIP(p, 4);
       int rs = 0;
@@ -570,8 +614,12 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
                 acc = 0;
                 next_chunk += CK;
               }
-              mma_kblock_x3_e<CG, KSTEPS, DSTEP>(d, da + (uint64_t)(sub * (A_BYTES >> 4)),
-                                                db + (uint64_t)sub * b16, alo16, blo16, idesc, acc);
+              const uint64_t a_ = da + (uint64_t)(sub * (A_BYTES >> 4)), b_ = db + (uint64_t)sub * b16;
+              if constexpr (MIX)
+                mma_kblock_mix_e<CG, DSTEP, BSTEP>(d, a_, b_, a_ + dA1, b_ + dB1, a_ + dA1 + ablo16,
+                                                   b_ + dB1 + bblo16, idesc, idesc_b, acc);
+              else
+                mma_kblock_x3_e<CG, KSTEPS, DSTEP>(d, a_, b_, alo16, blo16, idesc, acc);
               acc = 1;
             }
             mma_commit_e<CG>(empty(rs));

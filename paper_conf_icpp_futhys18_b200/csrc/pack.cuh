@@ -21,6 +21,34 @@ __device__ __forceinline__ uint32_t tf32_plane(float v, int pl) {
   return pl ? f32_to_tf32_rna(v - __uint_as_float(hi)) : hi;
 }
 
+// The mixed fp32 split (plan option fp32_split = 1; DESIGN.md §7 "mixed split"): three planes,
+// plane 0 = hi = rna_tf32(v) (4-byte elements), plane 1 = rne_bf16(hi), plane 2 = rne_bf16(v - hi)
+// (2-byte elements; v - hi is exact in fp32).  The packs receive the planes in one argument:
+// lo > 0: 3xTF32 (plane 1 = tf32 lo at +lo bytes, same element size); lo < 0: mixed, M = -lo
+// holds two byte offsets from the destination pointer's element 0 -- plane 1 at M & 0xFFFFFFFF,
+// plane 2 a further M >> 32 (the bf16 plane size) -- so a destination pointer already advanced
+// into the hi plane (a fused-group branch's rows) still finds its bf16 elements; lo = 0: one
+// plane.
+__device__ __forceinline__ int plane_count(long long lo) { return lo == 0 ? 1 : (lo > 0 ? 2 : 3); }
+__device__ __forceinline__ int plane_esize(long long lo, int pl) { return (lo < 0 && pl) ? 2 : 4; }
+__device__ __forceinline__ long long plane_off(long long lo, int pl) {
+  if (pl == 0) return 0;
+  if (lo > 0) return lo;
+  const unsigned long long m = (unsigned long long)(-lo);
+  const long long p1 = (long long)(m & 0xFFFFFFFFull);
+  return pl == 1 ? p1 : p1 + (long long)(m >> 32);
+}
+// bf16 bits of plane pl (1 or 2) of the mixed split
+__device__ __forceinline__ uint32_t mix_bf16_bits(float v, int pl) {
+  const float hi = __uint_as_float(f32_to_tf32_rna(v));
+  const float t = pl == 1 ? hi : v - hi;
+  __nv_bfloat16 b = __float2bfloat16_rn(t);
+  return (uint32_t)*reinterpret_cast<uint16_t *>(&b);
+}
+__device__ __forceinline__ uint32_t mix_bf16x2(float a, float b, int pl) {
+  return mix_bf16_bits(a, pl) | (mix_bf16_bits(b, pl) << 16);
+}
+
 template <int ELEM>
 struct PackOut;
 template <>
@@ -44,7 +72,12 @@ struct PackOut<4> {
     uint4 u = make_uint4(f32_to_tf32_rna(a), f32_to_tf32_rna(b), f32_to_tf32_rna(c),
                          f32_to_tf32_rna(d));
     *reinterpret_cast<uint4 *>(static_cast<float *>(dst) + idx) = u;
-    if (lo) {
+    if (lo < 0) {   // mixed split: bf16(hi), bf16(v - hi)
+#pragma unroll
+      for (int pl = 1; pl <= 2; ++pl)
+        *reinterpret_cast<uint2 *>(static_cast<uint8_t *>(dst) + plane_off(lo, pl) + idx * 2) =
+            make_uint2(mix_bf16x2(a, b, pl), mix_bf16x2(c, d, pl));
+    } else if (lo) {
       uint4 l = make_uint4(f32_to_tf32_rna(a - __uint_as_float(u.x)),
                            f32_to_tf32_rna(b - __uint_as_float(u.y)),
                            f32_to_tf32_rna(c - __uint_as_float(u.z)),
@@ -55,9 +88,15 @@ struct PackOut<4> {
   __device__ __forceinline__ static void store1(void *dst, size_t idx, float a, long long lo = 0) {
     const uint32_t h = f32_to_tf32_rna(a);
     static_cast<uint32_t *>(dst)[idx] = h;
-    if (lo)
+    if (lo < 0) {
+#pragma unroll
+      for (int pl = 1; pl <= 2; ++pl)
+        *reinterpret_cast<uint16_t *>(static_cast<uint8_t *>(dst) + plane_off(lo, pl) + idx * 2) =
+            (uint16_t)mix_bf16_bits(a, pl);
+    } else if (lo) {
       *reinterpret_cast<uint32_t *>(static_cast<uint8_t *>(dst) + lo + idx * 4) =
           f32_to_tf32_rna(a - __uint_as_float(h));
+    }
   }
 };
 
@@ -236,12 +275,17 @@ __global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ s
   // round + pack this lane's row, stage it in the warp's slab; 3xTF32 (lo_off != 0) stages and
   // writes the hi plane, then the lo plane through the same slab
   uint8_t *row = slab[warp] + lane * RB;
-  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;
+  const int planes = ELEM == 4 ? plane_count(lo_off) : 1;
   for (int pl = 0; pl < planes; ++pl) {
+    const int es = ELEM == 4 ? plane_esize(lo_off, pl) : 2;   // element bytes of this plane
 #pragma unroll
     for (int j = 0; j < 32; j += 8) {
       uint4 u0, u1;
-      if (ELEM == 2) {
+      if (ELEM == 4 && es == 2) {   // mixed split: a bf16 plane
+        u0 = make_uint4(mix_bf16x2(v[j], v[j + 1], pl), mix_bf16x2(v[j + 2], v[j + 3], pl),
+                        mix_bf16x2(v[j + 4], v[j + 5], pl), mix_bf16x2(v[j + 6], v[j + 7], pl));
+        *reinterpret_cast<uint4 *>(row + j * 2) = u0;
+      } else if (ELEM == 2) {
         __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
         __nv_bfloat162 c = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
         u0 = make_uint4(*reinterpret_cast<uint32_t *>(&a), *reinterpret_cast<uint32_t *>(&b),
@@ -259,15 +303,28 @@ __global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ s
     __syncwarp();
     // write back: chunk k of the 32-row slab -> row k / CPR, 16-byte chunk k % CPR
     constexpr int CPR = 32 * ELEM / 16;                   // 16-byte chunks per row (4 bf16, 8 tf32)
-    uint8_t *dpl = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0);
+    uint8_t *dpl = static_cast<uint8_t *>(dst) + (ELEM == 4 ? plane_off(lo_off, pl) : 0);
+    if (ELEM == 4 && es == 2) {   // a bf16 plane of the mixed split: 4 chunks per row
 #pragma unroll
-    for (int i = 0; i < CPR; ++i) {
-      const int k = i * 32 + lane, r = k / CPR, ch = k % CPR;
-      const long long qr = q0 + r;
-      const int c = c0 + ch * (16 / ELEM);
-      if (qr < total && c < Cw) {
-        const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
-        *reinterpret_cast<uint4 *>(dpl + ((size_t)qr * Cp + co_off + c) * ELEM) = val;
+      for (int i = 0; i < 4; ++i) {
+        const int k = i * 32 + lane, r = k / 4, ch = k % 4;
+        const long long qr = q0 + r;
+        const int c = c0 + ch * 8;
+        if (qr < total && c < Cw) {
+          const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+          *reinterpret_cast<uint4 *>(dpl + ((size_t)qr * Cp + co_off + c) * 2) = val;
+        }
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < CPR; ++i) {
+        const int k = i * 32 + lane, r = k / CPR, ch = k % CPR;
+        const long long qr = q0 + r;
+        const int c = c0 + ch * (16 / ELEM);
+        if (qr < total && c < Cw) {
+          const uint4 val = *reinterpret_cast<const uint4 *>(slab[warp] + r * RB + ch * 16);
+          *reinterpret_cast<uint4 *>(dpl + ((size_t)qr * Cp + co_off + c) * ELEM) = val;
+        }
       }
     }
     __syncwarp();
@@ -429,12 +486,17 @@ __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x
     }
   }
   uint8_t *row = slab[warp] + lane * RB;
-  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;   // 3xTF32: hi plane, then lo plane
+  const int planes = ELEM == 4 ? plane_count(lo_off) : 1;   // 3xTF32: hi, lo; mixed: hi, bf16 x2
   for (int pl = 0; pl < planes; ++pl) {
+    const int es = ELEM == 4 ? plane_esize(lo_off, pl) : 2;
 #pragma unroll
     for (int j = 0; j < S2DW_MAXC; j += 8) {
       if (j >= Cps) break;
-      if (ELEM == 2) {
+      if (ELEM == 4 && es == 2) {
+        *reinterpret_cast<uint4 *>(row + j * 2) =
+            make_uint4(mix_bf16x2(v[j], v[j + 1], pl), mix_bf16x2(v[j + 2], v[j + 3], pl),
+                       mix_bf16x2(v[j + 4], v[j + 5], pl), mix_bf16x2(v[j + 6], v[j + 7], pl));
+      } else if (ELEM == 2) {
         __nv_bfloat162 a = __floats2bfloat162_rn(v[j], v[j + 1]), b = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
         __nv_bfloat162 cq = __floats2bfloat162_rn(v[j + 4], v[j + 5]), d = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
         *reinterpret_cast<uint4 *>(row + j * 2) =
@@ -451,8 +513,9 @@ __global__ void __launch_bounds__(128) pack_s2d_warp(const float *__restrict__ x
     }
     __syncwarp();
     // the warp's rows q0 .. q0+31 are contiguous in dst: chunk k -> row k / cpr, chunk k % cpr
-    const int cpr = Cps * ELEM / 16;
-    uint8_t *out = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0) + (size_t)q0 * Cps * ELEM;
+    const int cpr = Cps * es / 16;
+    uint8_t *out = static_cast<uint8_t *>(dst) + (ELEM == 4 ? plane_off(lo_off, pl) : 0) +
+                   (size_t)q0 * Cps * es;
     const int nrows = (int)min(32LL, total - q0);
     for (int k = lane; k < nrows * cpr; k += 32) {
       const int r = k / cpr, ch = k - r * cpr;
@@ -510,15 +573,20 @@ __global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__
     }
   }
   uint8_t *rowp = slab[warp] + lane * RB;
-  const int planes = (ELEM == 4 && lo_off) ? 2 : 1;   // 3xTF32: hi plane, then lo plane
+  const int planes = ELEM == 4 ? plane_count(lo_off) : 1;   // 3xTF32: hi, lo; mixed: hi, bf16 x2
   for (int pl = 0; pl < planes; ++pl) {
+    const int es = ELEM == 4 ? plane_esize(lo_off, pl) : 2;
 #pragma unroll
     for (int j = 0; j < S2DW_MAXC; j += 8) {
       if (j >= Cps) break;
       float u[8];
 #pragma unroll
       for (int k = 0; k < 8; ++k) u[k] = (j + k < NC) ? v[(j + k < NC) ? j + k : 0] : 0.f;
-      if (ELEM == 2) {
+      if (ELEM == 4 && es == 2) {
+        *reinterpret_cast<uint4 *>(rowp + j * 2) =
+            make_uint4(mix_bf16x2(u[0], u[1], pl), mix_bf16x2(u[2], u[3], pl),
+                       mix_bf16x2(u[4], u[5], pl), mix_bf16x2(u[6], u[7], pl));
+      } else if (ELEM == 2) {
         __nv_bfloat162 a = __floats2bfloat162_rn(u[0], u[1]), b = __floats2bfloat162_rn(u[2], u[3]);
         __nv_bfloat162 cq = __floats2bfloat162_rn(u[4], u[5]), d = __floats2bfloat162_rn(u[6], u[7]);
         *reinterpret_cast<uint4 *>(rowp + j * 2) =
@@ -534,8 +602,9 @@ __global__ void __launch_bounds__(128) pack_s2d_warp_t(const float *__restrict__
       }
     }
     __syncwarp();
-    const int cpr = Cps * ELEM / 16;
-    uint8_t *out = static_cast<uint8_t *>(dst) + (pl ? lo_off : 0) + (size_t)q0 * Cps * ELEM;
+    const int cpr = Cps * es / 16;
+    uint8_t *out = static_cast<uint8_t *>(dst) + (ELEM == 4 ? plane_off(lo_off, pl) : 0) +
+                   (size_t)q0 * Cps * es;
     const int nrows = (int)min(32LL, total - q0);
     for (int k = lane; k < nrows * cpr; k += 32) {
       const int r = k / cpr, ch = k - r * cpr;

@@ -255,6 +255,39 @@ __device__ __forceinline__ void mma_kblock_x3_e(uint32_t d_tmem, uint64_t adesc,
 #undef GLP_X3_HEAD
 }
 
+// Mixed fp32 split k-block (GLP_MATH_FP32 with plan option fp32_split = 1): A and B each have a
+// tf32 hi plane (descriptors a, b) and two bf16 planes, bf16(hi) (a1, b1) and bf16(v - hi)
+// (a2, b2).  In this fixed order: four kind::tf32 MMAs hi*hi (K = 8 each, descriptors advanced by
+// TSTEP 16-byte units), two kind::f16 MMAs bf16(hi_A)*bf16(lo_B) and two bf16(lo_A)*bf16(hi_B)
+// (K = 16 each, advanced by BSTEP), all into one TMEM accumulator; `accumulate` applies to the
+// first MMA only.  Eight MMA issue slots per 32-deep k-block instead of 3xTF32's twelve.
+template <int CG, int TSTEP, int BSTEP>
+__device__ __forceinline__ void mma_kblock_mix_e(uint32_t d_tmem, uint64_t a, uint64_t b,
+                                                 uint64_t a1, uint64_t b1, uint64_t a2, uint64_t b2,
+                                                 uint32_t idesc_t, uint32_t idesc_b,
+                                                 uint32_t accumulate) {
+#define GLP_MX_T(CGS, X, Y, P) "@P_e tcgen05.mma.cta_group::" CGS ".kind::tf32 [%0], " X ", " Y ", %7, " P ";\n\t"
+#define GLP_MX_B(CGS, X, Y) "@P_e tcgen05.mma.cta_group::" CGS ".kind::f16 [%0], " X ", " Y ", %8, q;\n\t"
+#define GLP_MX(CGS)                                                                          \
+  asm volatile("{\n\t.reg .pred P_e, p, q;\n\t.reg .b64 x, y;\n\t"                         \
+               "elect.sync _|P_e, 0xffffffff;\n\tsetp.ne.b32 p, %9, 0;\n\tsetp.eq.b32 q, %7, %7;\n\t" \
+               GLP_MX_T(CGS, "%1", "%2", "p")                                                \
+               "add.s64 x, %1, %10;\n\tadd.s64 y, %2, %10;\n\t" GLP_MX_T(CGS, "x", "y", "q")   \
+               "add.s64 x, x, %10;\n\tadd.s64 y, y, %10;\n\t" GLP_MX_T(CGS, "x", "y", "q")     \
+               "add.s64 x, x, %10;\n\tadd.s64 y, y, %10;\n\t" GLP_MX_T(CGS, "x", "y", "q")     \
+               GLP_MX_B(CGS, "%3", "%6")                                                      \
+               "add.s64 x, %3, %11;\n\tadd.s64 y, %6, %11;\n\t" GLP_MX_B(CGS, "x", "y")        \
+               GLP_MX_B(CGS, "%5", "%4")                                                      \
+               "add.s64 x, %5, %11;\n\tadd.s64 y, %4, %11;\n\t" GLP_MX_B(CGS, "x", "y") "}"    \
+               ::"r"(d_tmem), "l"(a), "l"(b), "l"(a1), "l"(b1), "l"(a2), "l"(b2), "r"(idesc_t),  \
+               "r"(idesc_b), "r"(accumulate), "n"(TSTEP), "n"(BSTEP) : "memory")
+  if (CG == 1) GLP_MX("1");
+  else GLP_MX("2");
+#undef GLP_MX
+#undef GLP_MX_B
+#undef GLP_MX_T
+}
+
 template <int CG>
 __device__ __forceinline__ void mma_commit_e(uint32_t bar) {
   if (CG == 1)

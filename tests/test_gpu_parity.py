@@ -86,13 +86,18 @@ def test_parity_random(shape, math):
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s[0])
 def test_parity_rounding_emulated(shape, math):
     """Oracle on the operands rounded exactly as the pack step defines (oracle.round_*):
-    catches indexing bugs that the 2e-2 tolerance would hide.  3xTF32: the oracle of the three
-    products the MMAs form, hi*hi + hi*lo + lo*hi with (hi, lo) = oracle.split_3xtf32 (each
-    pass is linear in each operand, so the sum of three oracle calls), at 1e-6."""
+    catches indexing bugs that the 2e-2 tolerance would hide.  fp32: the oracle of the products
+    the MMAs form (each pass is linear in each operand, so a sum of oracle calls) -- the mixed
+    split's hi*hi + bhi*blo + blo*bhi (oracle.split_mixed) where the plan takes it, else 3xTF32's
+    hi*hi + hi*lo + lo*hi (oracle.split_3xtf32) -- at 5e-6."""
     d = _data(shape, seed=5)
-    got = _run(_layer(shape, math), d)
+    layer = _layer(shape, math)
+    got = _run(layer, d)
     S, P = shape[7], shape[8]
-    if math == "fp32":
+    if math == "fp32" and layer.info.fp32_split:   # the mixed split's own products
+        ref = _mixed_emulated(d, S, P)
+        bar = 5e-6
+    elif math == "fp32":
         sp = {k: oracle.split_3xtf32(d[k]) for k in ("x", "w", "dy")}
         parts = [_oracle(d, S, P, x=sp["x"][i], w=sp["w"][j], dy=sp["dy"][i])
                  for i, j in ((0, 0), (0, 1), (1, 0))]
@@ -109,6 +114,94 @@ def test_parity_rounding_emulated(shape, math):
         bar = 1e-4
     errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
     assert all(e <= bar for e in errs.values()), errs
+
+
+# layers whose three passes all take TMA operands (channel pitches % 32, unit stride): the mixed
+# fp32 split applies (plan option fp32_split = 1)
+MIX_SHAPES = [
+    ("gnet_conv_1", 4, 160, 7, 7, 320, 3, 1, 1),            # CTA pairs, ragged M tile
+    ("caffenet_conv3", 2, 256, 13, 13, 384, 3, 1, 1),
+    ("c96_k5_conv2", 2, 96, 27, 27, 256, 5, 1, 2),          # CaffeNet conv2 geometry, K = 2400
+    ("c32_k3_ragged", 3, 32, 11, 13, 64, 3, 1, 1),
+    ("c64_1x1", 5, 64, 7, 7, 96, 1, 1, 0),
+    ("lenet_conv2", 4, 20, 12, 12, 50, 5, 1, 0),            # channel pitches padded to 32
+]
+
+
+def _mixed_emulated(d, S, P):
+    """Oracle of exactly the products the mixed split's MMAs form: hi*hi + bhi*blo' + blo*bhi'
+    with (hi, bhi, blo) = oracle.split_mixed (each pass linear in each operand)."""
+    sp = {k: oracle.split_mixed(d[k]) for k in ("x", "w", "dy")}
+    pairs = ((0, 0), (1, 2), (2, 1))
+    parts = [_oracle(d, S, P, x=sp["x"][i], w=sp["w"][j], dy=sp["dy"][i]) for i, j in pairs]
+    pw = [_oracle(d, S, P, x=sp["x"][i], dy=sp["dy"][j])["dw"] for i, j in pairs]
+    ref = {k: parts[0][k] + parts[1][k] + parts[2][k] for k in ("y", "dx")}
+    ref["y"] -= 2 * d["b"].astype(np.float64)[None, :, None, None]   # bias counted once
+    ref["dw"] = pw[0] + pw[1] + pw[2]
+    ref["db"] = parts[0]["db"]
+    return ref
+
+
+@pytest.mark.parametrize("shape", MIX_SHAPES, ids=lambda s: s[0])
+def test_fp32_mixed_split(shape):
+    """GLP_MATH_FP32 with fp32_split = 1 (tf32 hi*hi + two bf16 cross terms): the plan takes the
+    split; bit-exact on integer data; within 1e-5 of the fp64 oracle and 5e-6 of the oracle of
+    the split's own products on random data; bitwise invariant across samples in flight."""
+    layer = _layer(shape, "fp32", fp32_split=1)
+    assert layer.info.fp32_split == 1
+    S, P = shape[7], shape[8]
+    d = _data(shape, exact=True, seed=91)
+    got = _run(layer, d)
+    ref = _oracle(d, S, P)
+    for k in ref:
+        np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+    d = _data(shape, seed=92)
+    runs = [_run(_layer(shape, "fp32", s_, fp32_split=1), d) for s_ in (0, 1, 0)]
+    ref = _oracle(d, S, P)
+    emu = _mixed_emulated(d, S, P)
+    errs = {k: oracle.normwise_err(runs[0][k], ref[k]) for k in ref}
+    eerr = {k: oracle.normwise_err(runs[0][k], emu[k]) for k in emu}
+    assert all(e <= TOL["fp32"] for e in errs.values()), errs
+    assert all(e <= 5e-6 for e in eerr.values()), eerr
+    for r in runs[1:]:
+        for k in r:
+            np.testing.assert_array_equal(r[k], runs[0][k], err_msg=k)
+
+
+@pytest.mark.parametrize("shape", MIX_SHAPES[:4], ids=lambda s: s[0])
+def test_fp32_3xtf32_on_tma_layers(shape):
+    """fp32_split = 0 keeps 3xTF32 on layers the mixed split would take (CTA pairs, TMA operands):
+    bit-exact on integers and within 5e-6 of the oracle of its own three products."""
+    layer = _layer(shape, "fp32", fp32_split=0)
+    assert layer.info.fp32_split == 0
+    S, P = shape[7], shape[8]
+    d = _data(shape, exact=True, seed=93)
+    got = _run(layer, d)
+    ref = _oracle(d, S, P)
+    for k in ref:
+        np.testing.assert_array_equal(got[k], ref[k].astype(np.float32), err_msg=k)
+    d = _data(shape, seed=94)
+    got = _run(layer, d)
+    sp = {k: oracle.split_3xtf32(d[k]) for k in ("x", "w", "dy")}
+    parts = [_oracle(d, S, P, x=sp["x"][i], w=sp["w"][j], dy=sp["dy"][i])
+             for i, j in ((0, 0), (0, 1), (1, 0))]
+    pw = [_oracle(d, S, P, x=sp["x"][i], dy=sp["dy"][j])["dw"] for i, j in ((0, 0), (0, 1), (1, 0))]
+    ref = {k: parts[0][k] + parts[1][k] + parts[2][k] for k in ("y", "dx")}
+    ref["y"] -= 2 * d["b"].astype(np.float64)[None, :, None, None]
+    ref["dw"] = pw[0] + pw[1] + pw[2]
+    ref["db"] = parts[0]["db"]
+    errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
+    assert all(e <= 5e-6 for e in errs.values()), errs
+
+
+def test_fp32_mixed_split_falls_back():
+    """Layers with a pass that is not TMA-fed (channel pitch % 32 != 0, or stride > 1) keep 3xTF32
+    under fp32_split = 1; the default is the mixed split; fp32_split = 0 selects 3xTF32."""
+    assert _layer(SHAPES[7], "fp32", fp32_split=1).info.fp32_split == 0    # C = 1: cp.async gather
+    assert _layer(SHAPES[2], "fp32", fp32_split=1).info.fp32_split == 0    # stride 4
+    assert _layer(SHAPES[3], "fp32", fp32_split=1).info.fp32_split == 0    # stride 2
+    assert _layer(MIX_SHAPES[0], "fp32").info.fp32_split == 1
+    assert _layer(MIX_SHAPES[0], "fp32", fp32_split=0).info.fp32_split == 0
 
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])

@@ -274,6 +274,29 @@ def test_rounding_error_bounds():
     assert np.all(np.abs(x.astype(np.float64) - hi - lo) <= 2.0 ** -22 * np.abs(x))
 
 
+def test_split_mixed_bounds():
+    """Mixed split (oracle.split_mixed): hi = rna_tf32(x) and x - hi exact in fp32 (as 3xTF32);
+    blo = rne_bf16(x - hi) leaves |x - hi - blo| <= 2^-8 |x - hi| <= 2^-19 |x|; bhi = rne_bf16(hi)
+    is a bf16 value within 2^-8 of hi; and the three products the MMAs form represent x*y to
+    |x y - (hi_x hi_y + bhi_x blo_y + blo_x bhi_y)| <= 2^-17 |x y| (the two cross terms' bf16
+    rounding, 2^-8 of a term <= 2^-11 |x y|, plus the dropped lo*lo)."""
+    rng = np.random.default_rng(2)
+    x = (rng.standard_normal(200000) * np.exp(rng.uniform(-20, 20, 200000))).astype(np.float32)
+    y = (rng.standard_normal(200000) * np.exp(rng.uniform(-20, 20, 200000))).astype(np.float32)
+    hi, bhi, blo = oracle.split_mixed(x)
+    np.testing.assert_array_equal(hi, oracle.round_tf32_rna(x))
+    x64 = x.astype(np.float64)
+    assert np.all((x64 - hi) == (x - hi).astype(np.float64))
+    assert np.all(np.abs(x64 - hi - blo) <= 2.0 ** -8 * np.abs(x64 - hi))
+    assert np.all(np.abs(x64 - hi - blo) <= 2.0 ** -19 * np.abs(x64))
+    assert np.all((bhi.view(np.uint32) & 0xFFFF) == 0) and np.all((blo.view(np.uint32) & 0xFFFF) == 0)
+    assert np.all(np.abs(bhi.astype(np.float64) - hi) <= 2.0 ** -8 * np.abs(hi.astype(np.float64)))
+    hy, bhy, bly = oracle.split_mixed(y)
+    prod = (hi.astype(np.float64) * hy + bhi.astype(np.float64) * bly + blo.astype(np.float64) * bhy)
+    xy = x64 * y.astype(np.float64)
+    assert np.all(np.abs(xy - prod) <= 2.0 ** -17 * np.abs(xy))
+
+
 def test_sampled_wgrad_element_matches_full():
     N, C, H, W, Co, K, S, P = 3, 4, 9, 9, 5, 3, 2, 1
     Ho = oracle.out_dim(H, K, S, P)

@@ -98,6 +98,7 @@ struct IgemmParams {
   int part_mpad;         // wgrad partial rows per split (m_tiles * 128)
   int a_tma;             // 1: A operand by im2col TMA (one thread); 0: cp.async gather
   int ksub;              // k-blocks per pipeline stage (1 or 2; cp.async path: 1)
+  int b3d;               // wgrad: the MN-major B tile by one 3-D TMA load (all atoms) per plane
   long long lo_off_a;    // 3xTF32: byte offset from the packed A source's hi plane to its lo plane
   int chunk_kb;          // 3xTF32: k-blocks per TMEM accumulation chunk (summed in fp32 registers)
 #ifdef GLP_DIAG

@@ -152,6 +152,23 @@ glp_status_t encode_2d(CUtensorMap *map, int elem, const void *ptr, uint64_t inn
   return GLP_OK;
 }
 
+// The filter gradient's MN-major B operand (dy packed [pixels][C_o pitch]) as a 3-D tensor
+// {atom elements, pixels, atoms}: one box {EPA, BKP, atoms} lands atom-major -- the MN-major
+// layout with one atom column of BKP rows per atom -- in a single TMA.
+glp_status_t encode_mn3d(CUtensorMap *map, int elem, const void *ptr, uint64_t cpitch, uint64_t pixels,
+                         uint32_t epa, uint32_t bkp, uint32_t natoms, CUtensorMapSwizzle swz) {
+  cuuint64_t dims[3] = {(cuuint64_t)epa, (cuuint64_t)pixels, (cuuint64_t)(cpitch / epa)};
+  cuuint64_t strides[2] = {(cuuint64_t)(cpitch * elem), (cuuint64_t)(epa * elem)};
+  cuuint32_t box[3] = {epa, bkp, natoms};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = g_encode(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                        3, const_cast<void *>(ptr), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled (3d) failed (" + std::to_string((int)r) + ")");
+  return GLP_OK;
+}
+
 using TmapIm2colFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
                                   const cuuint64_t *, const cuuint64_t *, const int *, const int *,
                                   cuuint32_t, cuuint32_t, const cuuint32_t *, CUtensorMapInterleave,
@@ -366,6 +383,7 @@ struct glp_plan_s {
   int halo_fdy = 0;     // fused-dy halo filter gradient (hwgrad_kernel<NCG>): no dy pack for it
   int red_wide = 0;     // dW reduction by reduce_tc_dw_wide (small filters, many splits)
   int mix = 0;          // GLP_MATH_FP32 by the mixed split (tf32 hi*hi + bf16 cross terms)
+  int wgrad_b3d = 0;    // filter-gradient B tile by one 3-D TMA per plane (all atoms)
   int hdg = 0;         // halo backward-data (hdgrad.cuh) for unit-stride layers where it pays
   HdgradParams hd{};
   int hd_grid = 0, hd_smem = 0;
@@ -902,6 +920,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   p.bn_smem = pp.bn_smem;
   p.stages = pp.stages;
   p.ksub = pp.ksub;
+  p.b3d = (mode == MODE_WGRAD && P.wgrad_b3d) ? 1 : 0;
   p.tmem_cols = pp.tmem_cols;
   p.acc_cols = pp.acc_cols;
   p.part_ld = pp.n_tiles * pp.bn;
@@ -1476,9 +1495,13 @@ glp_status_t run_wgrad_gemm(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const f
       // MN-major atoms of EPA elements: 32 tf32 (128-byte rows, 32-byte swizzle base) or, for the
       // bf16 planes of the mixed split, 32 bf16 (64-byte rows, SWIZZLE_64B)
       const CUtensorMapSwizzle sw = e == P.elem ? swz_mnmajor(P.elem, pp.krow) : CU_TENSOR_MAP_SWIZZLE_64B;
-      glp_status_t r = encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<const uint8_t *>(dypk) + ld,
-                                 (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
-                                 (uint64_t)P.Cop * e, (uint32_t)EPA, (uint32_t)BKP, sw);
+      glp_status_t r = P.wgrad_b3d
+          ? encode_mn3d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<const uint8_t *>(dypk) + ld,
+                        (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo, (uint32_t)EPA, (uint32_t)BKP,
+                        (uint32_t)(pp.bn_smem / EPA), sw)
+          : encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, static_cast<const uint8_t *>(dypk) + ld,
+                      (uint64_t)P.Cop, (uint64_t)d.N * d.Ho * d.Wo,
+                      (uint64_t)P.Cop * e, (uint32_t)EPA, (uint32_t)BKP, sw);
       if (r) return r;
       if (!pp.a_tma) continue;
       if ((r = get_encode_im2col())) return r;
@@ -2007,6 +2030,16 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
       if (cur != device) cudaSetDevice(cur);
       return s;
     }
+    // filter-gradient B (dy) tile: one 3-D TMA per plane instead of one per atom (same smem bytes);
+    // the channel pitch must be whole atoms (the 3-D view's atom dimension; a partial last atom
+    // would read the next pixel's channels instead of the 2-D map's zero fill)
+    // and every tile must start on an atom (N tile and its per-CTA half multiples of the atom)
+    const int epa = P->wgrad.krow / P->elem;
+    P->wgrad_b3d = (P->wgrad.a_tma && P->wgrad.bn_smem / epa >= 2 && P->Cop % epa == 0 &&
+                    P->wgrad.bn % epa == 0 && P->wgrad.bn_smem % epa == 0) ? 1 : 0;
+#ifdef GLP_DIAG
+    if (const char *e = getenv("GLP_DEBUG_B3D")) P->wgrad_b3d = P->wgrad_b3d && atoi(e);
+#endif
     if (P->mix && !(P->fwd.a_tma && P->dgrad.a_tma && P->wgrad.a_tma && P->fwd.krow == 128 &&
                     P->dgrad.krow == 128 && P->wgrad.krow == 128)) {
       delete P;

@@ -371,13 +371,18 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
                     }
                   }
                   if (lb) {
-                    for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
-                      if (CG == 1)
-                        tma_load_2d_e(pB + (uint32_t)a * lbo, mB, bar, nb0 + a * C::EPA,
-                                      kb * C::BKP);
-                      else
-                        tma_load_2d_cg2_e(pB + (uint32_t)a * lbo, mB, bar,
-                                          nb0 + a * C::EPA, kb * C::BKP);
+                    if (p.b3d) {   // all of the tile's atoms in one 3-D load
+                      if (CG == 1) tma_load_3d_e(pB, mB, bar, 0, kb * C::BKP, nb0 / C::EPA);
+                      else tma_load_3d_cg2_e(pB, mB, bar, 0, kb * C::BKP, nb0 / C::EPA);
+                    } else {
+                      for (int a = 0; a < p.bn_smem / C::EPA; ++a) {
+                        if (CG == 1)
+                          tma_load_2d_e(pB + (uint32_t)a * lbo, mB, bar, nb0 + a * C::EPA,
+                                        kb * C::BKP);
+                        else
+                          tma_load_2d_cg2_e(pB + (uint32_t)a * lbo, mB, bar,
+                                            nb0 + a * C::EPA, kb * C::BKP);
+                      }
                     }
                   }
                 }

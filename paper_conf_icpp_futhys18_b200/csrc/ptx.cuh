@@ -161,6 +161,24 @@ __device__ __forceinline__ void tma_load_im2col_4d_e(uint32_t dst, const CUtenso
                "h"(off_w), "h"(off_h)
                : "memory");
 }
+// 3-D tiled loads: the filter gradient's MN-major B (dy) tile as ONE load of all its atoms
+// (tensor dims {atom elements, pixels, atoms}: the box lands atom-major, i.e. the MN-major layout)
+__device__ __forceinline__ void tma_load_3d_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                              int c0, int c1, int c2) {
+  asm volatile(GLP_ELECT
+               "@P_e cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+               " [%0], [%1, {%3, %4, %5}], [%2];\n\t}" ::"r"(dst),
+               "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_3d_cg2_e(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                                  int c0, int c1, int c2) {
+  asm volatile(GLP_ELECT
+               "@P_e cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+               " [%0], [%1, {%3, %4, %5}], [%2];\n\t}" ::"r"(dst),
+               "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+               : "memory");
+}
 __device__ __forceinline__ void tma_load_2d_cg2_e(uint32_t dst, const CUtensorMap *map,
                                                   uint32_t bar, int c0, int c1) {
   asm volatile(GLP_ELECT

@@ -177,12 +177,14 @@ typedef struct {
                              leaves and a leaf's N*H_o*W_o a multiple of the k-block (32 pixels
                              tf32 / fp32, 64 bf16); tensor-core single-layer plans (no fused
                              sibling groups).  Changes the split order, hence low bits, vs 1.      */
-  int fp32_split;         /* GLP_MATH_FP32 on tensor cores: 1 (default) the mixed split -- hi*hi in
-                             tf32 plus bf16(hi)*bf16(lo) and bf16(lo)*bf16(hi) in bf16 (8 instead
-                             of 12 MMA issue slots per k-block; representation error ~6e-7 normwise,
-                             that of an fp32 sgemm); 0 3xTF32 -- hi*hi + hi*lo + lo*hi, three
-                             kind::tf32 MMAs per k-step.  Layers whose passes do not all take TMA
-                             operands (channel pitch % 32, unit stride) keep 3xTF32.              */
+  int fp32_split;         /* GLP_MATH_FP32 on tensor cores: the mixed split -- hi*hi in tf32 plus
+                             bf16(hi)*bf16(lo) and bf16(lo)*bf16(hi) in bf16 (8 instead of 12 MMA
+                             issue slots per k-block; representation error ~6e-7 normwise, that of
+                             an fp32 sgemm) -- or 3xTF32 (hi*hi + hi*lo + lo*hi, three kind::tf32
+                             MMAs per k-step).  0: 3xTF32 everywhere; 1: the mixed split wherever
+                             every pass takes TMA operands (channel pitch % 32, unit stride);
+                             2 (default): as 1, for passes of >= 2 GFLOP (smaller layers measured
+                             faster in 3xTF32).  A shape-only choice: results stay deterministic. */
 } glp_plan_options_t;
 glp_status_t glp_plan_options_default(glp_plan_options_t *opts);
 /* opts may be NULL (defaults).  GLP_ERR_INVALID_VALUE for an out-of-range option. */

@@ -1872,7 +1872,7 @@ glp_status_t glp_analyze_eq7(const glp_device_limits_t *L, const glp_kernel_attr
 
 glp_status_t glp_plan_options_default(glp_plan_options_t *o) {
   if (!o) return fail(GLP_ERR_INVALID_VALUE, "NULL argument");
-  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 6, 1, 0, 0, 232448, 0, 0, 1};
+  *o = glp_plan_options_t{1, 1, 1, 1, 1, 1, 0, 4, 0, 6, 1, 0, 0, 232448, 0, 0, 2};
   return GLP_OK;
 }
 
@@ -1892,7 +1892,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
       o.smem_cap > 232448 || (o.wgrad_leaves != 0 && o.wgrad_leaves != 1 && o.wgrad_leaves != 2 &&
                               o.wgrad_leaves != 4 && o.wgrad_leaves != 8))
     return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
-  if (o.fp32_split < 0 || o.fp32_split > 1) return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
+  if (o.fp32_split < 0 || o.fp32_split > 2) return fail(GLP_ERR_INVALID_VALUE, "plan option out of range");
   if (o.wgrad_leaves > 0 && (math == GLP_MATH_FP32_SIMT || d->nbr > 1))
     return fail(GLP_ERR_NOT_SUPPORTED, "wgrad leaves: tensor-core single-layer plans only");
   *out = nullptr;
@@ -2021,8 +2021,11 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
   // the mixed fp32 split (option fp32_split): every pass must take its operands by TMA with
   // 128-byte tf32 rows (the packs write one representation for all three passes): channel
   // pitches multiples of 32 and unit stride (the backward-data TMA gather)
+  // and enough work per pass: below ~2 GFLOP (CIFAR-10 conv2/conv3) the third operand plane's TMA
+  // loads cost more than the MMA issue slots saved (measured: CIFAR-10 -2.3 %, GoogLeNet +3 %)
+  const double pass_flop = 2.0 * P->d.N * P->d.Ho * P->d.Wo * P->d.Co * P->d.C * P->d.Kh * P->d.Kw;
   P->mix = (P->x3 && o.fp32_split && P->Cpx % 32 == 0 && P->Cop % 32 == 0 && P->d.Sh == 1 &&
-            P->d.Sw == 1) ? 1 : 0;
+            P->d.Sw == 1 && (o.fp32_split == 1 || pass_flop >= 2e9)) ? 1 : 0;
   if (!P->simt) {
     if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
         (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {

@@ -196,12 +196,15 @@ def test_fp32_3xtf32_on_tma_layers(shape):
 
 def test_fp32_mixed_split_falls_back():
     """Layers with a pass that is not TMA-fed (channel pitch % 32 != 0, or stride > 1) keep 3xTF32
-    under fp32_split = 1; the default is the mixed split; fp32_split = 0 selects 3xTF32."""
+    under fp32_split = 1; the default (2) takes the mixed split for TMA-fed passes of >= 2 GFLOP
+    only; fp32_split = 0 selects 3xTF32."""
     assert _layer(SHAPES[7], "fp32", fp32_split=1).info.fp32_split == 0    # C = 1: cp.async gather
     assert _layer(SHAPES[2], "fp32", fp32_split=1).info.fp32_split == 0    # stride 4
     assert _layer(SHAPES[3], "fp32", fp32_split=1).info.fp32_split == 0    # stride 2
-    assert _layer(MIX_SHAPES[0], "fp32").info.fp32_split == 1
-    assert _layer(MIX_SHAPES[0], "fp32", fp32_split=0).info.fp32_split == 0
+    assert _layer(MIX_SHAPES[0], "fp32").info.fp32_split == 0                # 0.2 GFLOP per pass
+    big = ("caffenet_conv3_b8", 8, 256, 13, 13, 384, 3, 1, 1)                 # 2.4 GFLOP per pass
+    assert _layer(big, "fp32").info.fp32_split == 1
+    assert _layer(big, "fp32", fp32_split=0).info.fp32_split == 0
 
 
 @pytest.mark.parametrize("math", ["bf16", "tf32", "fp32", "fp32_simt"])

@@ -153,8 +153,9 @@ typedef struct {
   int wgrad_cta_pairs;    /* 1: CTA pairs for the filter gradient too; 0: not                      */
   int halo_wgrad;         /* 1: shared-halo filter gradient for space-to-depth layers; 0: im2col   */
   int halo_fwd;           /* 1: shared-halo forward for space-to-depth layers; 0: im2col           */
-  int halo_dgrad;         /* 1: shared-halo backward-data where the cost model picks it; 0: never;
-                             2: wherever legal                                                     */
+  int halo_dgrad;         /* 1: shared-halo backward-data where the cost model picks it (bf16,
+                             tf32); 0: never; 2: wherever legal (also the mixed fp32 split's
+                             three-plane halo kernel, measured slower than im2col: opt-in only)    */
   int fused_dy;           /* 1: the halo filter gradient builds its dy operand from fp32 dy; 0: it
                              reads the packed dy                                                   */
   int fused_dy_builders;  /* 0: model; 1: cp.async landing zone; 2 or 3: register builder groups   */
@@ -182,8 +183,10 @@ typedef struct {
                              issue slots per k-block; representation error ~6e-7 normwise, that of
                              an fp32 sgemm) -- or 3xTF32 (hi*hi + hi*lo + lo*hi, three kind::tf32
                              MMAs per k-step).  0: 3xTF32 everywhere; 1: the mixed split wherever
-                             every pass takes TMA operands (channel pitch % 32, unit stride);
-                             2 (default): as 1, for passes of >= 2 GFLOP (smaller layers measured
+                             the passes take 128-byte tf32 rows (channel pitches % 32; forward
+                             and filter gradient by TMA, backward-data by TMA or, strided, by the
+                             K-major cp.async gather); 2 (default): as 1 for unit-stride layers
+                             with passes of >= 2 GFLOP (smaller and strided layers measured
                              faster in 3xTF32).  A shape-only choice: results stay deterministic. */
 } glp_plan_options_t;
 glp_status_t glp_plan_options_default(glp_plan_options_t *opts);

@@ -544,20 +544,22 @@ glp_status_t plan_halo(glp_plan_s &P) {
   return GLP_OK;
 }
 
-// Halo backward-data (hdgrad.cuh): unit stride, square kernel, bf16 or tf32 (not 3xTF32), the
+// Halo backward-data (hdgrad.cuh): unit stride, square kernel, bf16, tf32 or the mixed fp32 split
+// (not 3xTF32; the mixed split with C_i <= 128: the epilogue's chunk sums in registers), the
 // flipped-tap Wt of the im2col-TMA dgrad, 128-byte channel blocks of C_o (64 bf16 / 32 tf32), and a
 // tile geometry (R output rows padded to a pitch of WQ >= W + K - 1 pixels, R*WQ = 128) that
 // wastes at most 30 % of the rows.  Used when the im2col A traffic dominates: >= 9 taps and
 // C_i <= 128 (each A byte feeds few columns).
-const void *hdgrad_fn(int elem) {
-  return elem == 2 ? reinterpret_cast<const void *>(hdgrad_kernel<2>)
-                   : reinterpret_cast<const void *>(hdgrad_kernel<4>);
+const void *hdgrad_fn(int elem, int mix) {
+  return elem == 2 ? reinterpret_cast<const void *>(hdgrad_kernel<2, 0>)
+         : mix     ? reinterpret_cast<const void *>(hdgrad_kernel<4, 1>)
+                   : reinterpret_cast<const void *>(hdgrad_kernel<4, 0>);
 }
 glp_status_t plan_hdgrad(glp_plan_s &P) {
   P.hdg = 0;
   const glp_conv_desc_s &d = P.d;
   const int cb = 128 / P.elem;   // channels per 128-byte block
-  if (!P.allow_hdg || P.x3 || P.simt || d.nbr > 1 || d.Sh != 1 || d.Sw != 1 || d.Kh != d.Kw ||
+  if (!P.allow_hdg || (P.x3 && !P.mix) || P.simt || d.nbr > 1 || d.Sh != 1 || d.Sw != 1 || d.Kh != d.Kw ||
       d.Ph != d.Pw || d.Ph > d.Kh - 1 || !P.dgrad.a_tma || P.dgrad.krow != 128 || P.Cop % cb != 0)
     return GLP_OK;
   const int K = d.Kh, taps = K * K;
@@ -570,6 +572,11 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   const int bn = (int)rup(d.C, 16);
   if (P.allow_hdg != 2 && (junk > 1.3 || taps < 9 || bn > 128)) return GLP_OK;
   if (bn > 256 || (bn / 2) % 16 != 0) return GLP_OK;   // CTA pairs: half of B per CTA, N % 32
+  if (P.mix && bn > 128) return GLP_OK;   // chunk sums: <= 128 fp32 registers per epilogue thread
+  // mixed split: opt-in only (halo_dgrad = 2).  Measured on CaffeNet conv2 (b256): 740 us against
+  // the im2col kernel's 723 us -- the 27-of-32 useful columns of a WQ = 32 row and the ragged last
+  // wave (13 rounds for 12.1 units per pair) cost more than the halo saves on the L2
+  if (P.mix && P.allow_hdg != 2) return GLP_OK;
   HdgradParams &h = P.hd;
   memset(&h, 0, sizeof(h));
   h.K = K;
@@ -591,9 +598,17 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   int tc = 32;
   while (tc < 2 * h.acc_cols) tc *= 2;
   h.tmem_cols = tc;
-  h.a_bytes = (int)rup((long long)(R + K - 1) * WQ * 128, 1024);
-  h.b_tap_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
-  h.a_stages = 3;
+  h.a_hi_bytes = (int)rup((long long)(R + K - 1) * WQ * 128, 1024);
+  h.b_hi_bytes = (int)rup((long long)(bn / 2) * 128, 1024);
+  if (P.mix) {   // + the two bf16 planes (64-byte rows)
+    h.a_bf_bytes = (int)rup((long long)(R + K - 1) * WQ * 64, 1024);
+    h.b_bf_bytes = (int)rup((long long)(bn / 2) * 64, 1024);
+    h.chunk_kb = P.dgrad.chunk_kb;   // the igemm passes' shape-only chunk (K = 32 per k-block)
+    if (h.chunk_kb <= 0) return GLP_OK;
+  }
+  h.a_bytes = h.a_hi_bytes + 2 * h.a_bf_bytes;
+  h.b_tap_bytes = h.b_hi_bytes + 2 * h.b_bf_bytes;
+  h.a_stages = P.mix ? 2 : 3;   // a mixed halo stage is twice the bytes (and 25 taps of MMAs)
 #ifdef GLP_DIAG
   if (const char *e = getenv("GLP_HD_ASTAGES")) h.a_stages = std::max(2, atoi(e));   // A/B runs
 #endif
@@ -611,9 +626,9 @@ glp_status_t plan_hdgrad(glp_plan_s &P) {
   if (h.b_stages < 3) return GLP_OK;
   P.hd_smem = 1024 + h.a_stages * h.a_bytes + h.b_stages * h.b_bytes +
               8 * (2 * h.a_stages + 2 * h.b_stages + 4) + 16;
-  GLP_CUDA(cudaFuncSetAttribute(hdgrad_fn(P.elem), cudaFuncAttributeMaxDynamicSharedMemorySize,
+  GLP_CUDA(cudaFuncSetAttribute(hdgrad_fn(P.elem, P.mix), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 232448));
-  glp_status_t s = analyze_kernel(P, hdgrad_fn(P.elem), HD_THREADS, P.hd_smem, h.tmem_cols,
+  glp_status_t s = analyze_kernel(P, hdgrad_fn(P.elem, P.mix), HD_THREADS, P.hd_smem, h.tmem_cols,
                                   P.hd_attr);
   if (s) return s;
   // persistent grid: the analyzer's resident CTA-pair slots (#SM x CTAs/SM / 2), at most the units
@@ -1343,15 +1358,17 @@ glp_status_t run_fwd_gemm(glp_plan_s &P, const BrIn &b, const BrOut &y, uint8_t 
 }
 
 glp_status_t encode_4d_nhwc(CUtensorMap *map, int elem, const void *ptr, int cpitch, int W, int H,
-                            int N, uint32_t box_w, uint32_t box_h) {
+                            int N, uint32_t box_w, uint32_t box_h, uint32_t box_c = 0,
+                            CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   cuuint64_t dims[4] = {(cuuint64_t)cpitch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
   cuuint64_t strides[3] = {(cuuint64_t)cpitch * elem, (cuuint64_t)W * cpitch * elem,
                            (cuuint64_t)H * W * cpitch * elem};
-  cuuint32_t box[4] = {(cuuint32_t)(128 / elem), box_w, box_h, 1u};   // one 128-byte channel block
+  // one 128-byte channel block (or box_c channels: the 64-byte bf16 rows of the mixed split)
+  cuuint32_t box[4] = {box_c ? box_c : (cuuint32_t)(128 / elem), box_w, box_h, 1u};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = g_encode(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
                         4, const_cast<void *>(ptr), dims,
-                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(GLP_ERR_CUDA, "cuTensorMapEncodeTiled (4d) failed (" + std::to_string((int)r) + ")");
   return GLP_OK;
@@ -1361,12 +1378,23 @@ glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   const glp_conv_desc_s &d = P.d;
   Maps m;
   glp_status_t s = cached_maps(P, 1, ws, m, [&](Maps &q) {
-    glp_status_t r = encode_4d_nhwc(&q.a, P.elem, ws + P.off_dypk, P.Cop, d.Wo, d.Ho, d.N,
-                                    (uint32_t)P.hd.WQ, (uint32_t)(P.hd.R + P.hd.K - 1));
-    if (r) return r;
-    return encode_2d(&q.b, P.elem, ws + P.off_wtpk, (uint64_t)P.dgrad.Kpad, (uint64_t)d.C,
-                     (uint64_t)P.dgrad.Kpad * P.elem, (uint32_t)(128 / P.elem), (uint32_t)(P.hd.bn / 2),
-                     CU_TENSOR_MAP_SWIZZLE_128B);
+    // one plane (bf16 / tf32), or the mixed split's tf32 hi plane and two bf16 planes (32
+    // channels per 64-byte row, SWIZZLE_64B)
+    const int CB = 128 / P.elem;
+    for (int pl = 0; pl < (P.mix ? 3 : 1); ++pl) {
+      const int e = plane_elem(P, pl);
+      const CUtensorMapSwizzle sw = e * CB == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
+      glp_status_t r = encode_4d_nhwc(plane_map(&q.a, &q.a2, &q.a3, pl), e,
+                                      ws + P.off_dypk + plane_offset(P, pl, P.lo_dypk), P.Cop, d.Wo,
+                                      d.Ho, d.N, (uint32_t)P.hd.WQ, (uint32_t)(P.hd.R + P.hd.K - 1),
+                                      (uint32_t)CB, sw);
+      if (r) return r;
+      r = encode_2d(plane_map(&q.b, &q.b2, &q.b3, pl), e, ws + P.off_wtpk + plane_offset(P, pl, P.lo_wtpk),
+                    (uint64_t)P.dgrad.Kpad, (uint64_t)d.C, (uint64_t)P.dgrad.Kpad * e, (uint32_t)CB,
+                    (uint32_t)(P.hd.bn / 2), sw);
+      if (r) return r;
+    }
+    return GLP_OK;
   });
   if (s) return s;
   CUtensorMap &mapDy = m.a, &mapW = m.b;
@@ -1389,8 +1417,8 @@ glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = P.pdl ? 2 : 1;
-  void *args[] = {&p, &mapDy, &mapW};
-  GLP_CUDA(cudaLaunchKernelExC(&cfg, hdgrad_fn(P.elem), args));
+  void *args[] = {&p, &mapDy, &mapW, &m.a2, &m.b2, &m.a3, &m.b3};
+  GLP_CUDA(cudaLaunchKernelExC(&cfg, hdgrad_fn(P.elem, P.mix), args));
   GLP_LAUNCH_CHECK("hdgrad_kernel");
   return GLP_OK;
 }
@@ -2018,14 +2046,19 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
                                                std::to_string(ch) + " == 0");
       }
   }
-  // the mixed fp32 split (option fp32_split): every pass must take its operands by TMA with
-  // 128-byte tf32 rows (the packs write one representation for all three passes): channel
-  // pitches multiples of 32 and unit stride (the backward-data TMA gather)
+  // the mixed fp32 split (option fp32_split): every pass must take its operands with 128-byte
+  // tf32 rows (the packs write one representation for all three passes): channel pitches
+  // (space-to-depth: of x') multiples of 32; forward and filter gradient by TMA, the backward-data
+  // by TMA or -- strided layers -- by the K-major cp.async gather;
   // and enough work per pass: below ~2 GFLOP (CIFAR-10 conv2/conv3) the third operand plane's TMA
-  // loads cost more than the MMA issue slots saved (measured: CIFAR-10 -2.3 %, GoogLeNet +3 %)
+  // loads cost more than the MMA issue slots saved (measured: CIFAR-10 -2.3 %, GoogLeNet +3 %).
+  // Strided layers only when forced (fp32_split = 1): CaffeNet conv1 measured forward 334 -> 316
+  // us but filter gradient 418 -> 442 us (its MN-major operands are shared-memory bound, and the
+  // 64-byte bf16 atoms read no cheaper), so the default keeps them on 3xTF32
   const double pass_flop = 2.0 * P->d.N * P->d.Ho * P->d.Wo * P->d.Co * P->d.C * P->d.Kh * P->d.Kw;
-  P->mix = (P->x3 && o.fp32_split && P->Cpx % 32 == 0 && P->Cop % 32 == 0 && P->d.Sh == 1 &&
-            P->d.Sw == 1 && (o.fp32_split == 1 || pass_flop >= 2e9)) ? 1 : 0;
+  P->mix = (P->x3 && o.fp32_split && P->Cpx % 32 == 0 && P->Cop % 32 == 0 &&
+            (P->d.Sh == P->d.Sw) && (P->d.Sh == 1 || o.fp32_split == 1) &&
+            (o.fp32_split == 1 || pass_flop >= 2e9)) ? 1 : 0;
   if (!P->simt) {
     if ((s = plan_pass(*P, P->fwd, MODE_FWD, L)) || (s = plan_pass(*P, P->dgrad, MODE_DGRAD, L)) ||
         (s = plan_pass(*P, P->wgrad, MODE_WGRAD, L))) {
@@ -2043,8 +2076,9 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
 #ifdef GLP_DIAG
     if (const char *e = getenv("GLP_DEBUG_B3D")) P->wgrad_b3d = P->wgrad_b3d && atoi(e);
 #endif
-    if (P->mix && !(P->fwd.a_tma && P->dgrad.a_tma && P->wgrad.a_tma && P->fwd.krow == 128 &&
-                    P->dgrad.krow == 128 && P->wgrad.krow == 128)) {
+    if (P->mix && !(P->fwd.a_tma && P->wgrad.a_tma && P->fwd.krow == 128 &&
+                    P->dgrad.krow == 128 && P->wgrad.krow == 128 &&
+                    (P->dgrad.a_tma || P->dgrad.cg == 1))) {
       delete P;
       if (cur != device) cudaSetDevice(cur);
       return fail(GLP_ERR_INTERNAL, "mixed fp32 split planned for a non-TMA pass");

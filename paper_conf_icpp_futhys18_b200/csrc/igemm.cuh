@@ -133,8 +133,9 @@ __device__ __forceinline__ bool fwd_gather(const Gather &g, uint32_t n, int ohS,
 // SWIZZLE_64B, or MN-major 32-element SWIZZLE_64B atoms), the same bytes as 3xTF32's two planes;
 // tmapA2 / tmapB2 are the bf16(hi) planes, tmapA3 / tmapB3 the bf16(v - hi) planes.  The MMA
 // issuer runs hi*hi in tf32 and the two cross terms in bf16 (mma_kblock_mix_e): 8 MMA issue slots
-// per k-block instead of 12.  TMA operands only (the plan refuses the split for cp.async layers);
-// the chunked accumulation and the epilogue are those of X3 = 1.
+// per k-block instead of 12.  TMA operands, except the K-major cp.async gather of a strided
+// backward-data (8-byte copies into the bf16 planes); the chunked accumulation and the epilogue
+// are those of X3 = 1.
 template <int MODE, int ELEM, int KROW, int CG, int X3>
 __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
     igemm_kernel(const __grid_constant__ IgemmParams p, const __grid_constant__ CUtensorMap tmapB,
@@ -396,7 +397,9 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
       }
     } else if (KROW == 128 && CG == 1) {
       // -------- cp.async gather (SWIZZLE_128B layouts only) --------
-      if (MIX) __trap();   // the mixed split is planned for TMA operands only
+      // (mixed split: the K-major gather only -- strided backward-data; the plan keeps the
+      // filter gradient of a mixed layer on TMA)
+      if (MIX && MODE == MODE_WGRAD) __trap();
       int rs = 0;          // ring slot and its phase, advanced incrementally
         uint32_t rph = 0;
       for (int tile = unit0; tile < total_tiles; tile += ustep) {
@@ -444,6 +447,7 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
               mbar_arrive_expect_tx(full(s), b_bytes);
               tma_load_2d(sB, &tmapB, full(s), kb * C::BK, n0);
               if (X3) tma_load_2d(sB + b_bytes1, &tmapB2, full(s), kb * C::BK, n0);
+              if (MIX) tma_load_2d(sB + b_bytes1 + b_bytes1 / 2, &tmapB3, full(s), kb * C::BK, n0);
             }
             const bool kv = (int)t < g.taps;
 #pragma unroll
@@ -473,7 +477,19 @@ __global__ void __launch_bounds__(X3 ? IGEMM_X3_THREADS : IGEMM_THREADS, 1)
                 src += ((size_t)(pbase[i] + (uint32_t)(ih * g.src_w + iw)) * (uint32_t)g.src_cp + c) *
                        ELEM;
               cp_async16(sA + dst0 + (uint32_t)i * 2048u, src, ok);
-              if (X3) cp_async16(sA + A_BYTES1 + dst0 + (uint32_t)i * 2048u, src + p.lo_off_a, ok);
+              if constexpr (MIX) {
+                // the chunk's 4 channels in the bf16(hi) and bf16(v - hi) planes: 8 bytes of a
+                // 64-byte SWIZZLE_64B row (16-byte chunk (j/2) ^ ((r/2) & 3), half j & 1); the
+                // bf16 planes start lo_off_a (the hi plane's bytes) and 1.5 x that past the hi one
+                const int r = rg + 16 * i;
+                const uint32_t dbf = (uint32_t)r * 64u +
+                                     ((uint32_t)(((j >> 1) ^ ((r >> 1) & 3)) << 4) | ((uint32_t)(j & 1) << 3));
+                const uint8_t *sb = srcb + p.lo_off_a + (src - srcb) / 2;
+                cp_async8(sA + A_BYTES1 + dbf, sb, ok);
+                cp_async8(sA + A_BYTES1 + A_BYTES1 / 2 + dbf, sb + p.lo_off_a / 2, ok);
+              } else if (X3) {
+                cp_async16(sA + A_BYTES1 + dst0 + (uint32_t)i * 2048u, src + p.lo_off_a, ok);
+              }
             }
             cp_async_mbar_arrive_noinc(full(s));
             c += C::BK;

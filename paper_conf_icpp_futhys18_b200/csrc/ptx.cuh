@@ -92,6 +92,12 @@ __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, bool v
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n)
                : "memory");
 }
+// 8-byte cp.async (.ca); zero-fills when !valid (the bf16 planes of the mixed split's gather)
+__device__ __forceinline__ void cp_async8(uint32_t dst, const void *src, bool valid) {
+  const uint32_t n = valid ? 8u : 0u;
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(dst), "l"(src), "r"(n)
+               : "memory");
+}
 // 4-byte cp.async (L1-allocating .ca: the only form for sizes < 16); zero-fills when !valid
 __device__ __forceinline__ void cp_async4(uint32_t dst, const void *src, bool valid) {
   const uint32_t n = valid ? 4u : 0u;

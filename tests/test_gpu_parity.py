@@ -125,6 +125,8 @@ MIX_SHAPES = [
     ("c32_k3_ragged", 3, 32, 11, 13, 64, 3, 1, 1),
     ("c64_1x1", 5, 64, 7, 7, 96, 1, 1, 0),
     ("lenet_conv2", 4, 20, 12, 12, 50, 5, 1, 0),            # channel pitches padded to 32
+    ("caffenet_conv1_s4", 2, 3, 67, 67, 96, 11, 4, 0),      # space-to-depth; strided dgrad gather
+    ("ragged_s2", 3, 13, 9, 11, 37, 3, 2, 1),               # s2d x' 52 -> 64 channels, ragged
 ]
 
 
@@ -195,12 +197,18 @@ def test_fp32_3xtf32_on_tma_layers(shape):
 
 
 def test_fp32_mixed_split_falls_back():
-    """Layers with a pass that is not TMA-fed (channel pitch % 32 != 0, or stride > 1) keep 3xTF32
-    under fp32_split = 1; the default (2) takes the mixed split for TMA-fed passes of >= 2 GFLOP
-    only; fp32_split = 0 selects 3xTF32."""
+    """Layers whose channel pitch is not a multiple of 32 (the forward / filter gradient would need
+    the cp.async gather) keep 3xTF32 under fp32_split = 1; strided layers take the mixed split
+    (forward and filter gradient by TMA on the space-to-depth x', the backward-data by the
+    K-major gather); the default (2) takes it for unit-stride layers with >= 2 GFLOP per pass
+    (CaffeNet conv1's filter gradient measured slower mixed); fp32_split = 0 selects 3xTF32."""
     assert _layer(SHAPES[7], "fp32", fp32_split=1).info.fp32_split == 0    # C = 1: cp.async gather
-    assert _layer(SHAPES[2], "fp32", fp32_split=1).info.fp32_split == 0    # stride 4
-    assert _layer(SHAPES[3], "fp32", fp32_split=1).info.fp32_split == 0    # stride 2
+    assert _layer(SHAPES[2], "fp32", fp32_split=1).info.fp32_split == 1    # stride 4, s2d
+    assert _layer(SHAPES[3], "fp32", fp32_split=1).info.fp32_split == 1    # stride 2, s2d
+    assert _layer(SHAPES[2], "fp32").info.fp32_split == 0                  # < 2 GFLOP per pass
+    conv1 = ("caffenet_conv1_b32", 32, 3, 227, 227, 96, 11, 4, 0)          # 6.7 GFLOP per pass
+    assert _layer(conv1, "fp32").info.fp32_split == 0
+    assert _layer(conv1, "fp32", fp32_split=1).info.fp32_split == 1
     assert _layer(MIX_SHAPES[0], "fp32").info.fp32_split == 0                # 0.2 GFLOP per pass
     big = ("caffenet_conv3_b8", 8, 256, 13, 13, 384, 3, 1, 1)                 # 2.4 GFLOP per pass
     assert _layer(big, "fp32").info.fp32_split == 1
@@ -800,26 +808,36 @@ HDG_SHAPES = [
 ]
 
 
-@pytest.mark.parametrize("math", ["bf16", "tf32"])
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
 @pytest.mark.parametrize("shape", HDG_SHAPES, ids=lambda s: s[0])
 def test_halo_dgrad(shape, math):
     """Shared-halo backward-data (4-D TMA halo of the packed dy per 128-byte channel block -- 64
     bf16 / 32 tf32 channels -- flipped taps by row shift, CTA pairs with M = 256 MMAs): bit-exact
     on integer data, within 1e-4 of the rounding-emulated oracle and the mode's bar of the fp64
-    oracle on random data, bitwise invariant across samples-in-flight overrides."""
-    layer = _layer(shape, math, halo_dgrad=2)
+    oracle on random data, bitwise invariant across samples-in-flight overrides.  fp32: the mixed
+    split (fp32_split = 1: tf32 hi and two bf16 halo tiles per channel block, the 64-byte bf16
+    rows shifted like the tf32 ones, chunked accumulation) against 1e-5 of the fp64 oracle and
+    5e-6 of the oracle of the split's own products."""
+    opts = dict(halo_dgrad=2, **({"fp32_split": 1} if math == "fp32" else {}))
+    layer = _layer(shape, math, **opts)
     assert layer.info.dgrad_halo == 1
+    if math == "fp32":
+        assert layer.info.fp32_split == 1
     d = _data(shape, exact=True, seed=53)
     got = _run(layer, d)
     ref = _oracle(d, shape[7], shape[8])
     np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32))
     d = _data(shape, seed=54)
-    runs = [_run(_layer(shape, math, S, halo_dgrad=2), d)["dx"] for S in (0, 1, 0)]
+    runs = [_run(_layer(shape, math, S, **opts), d)["dx"] for S in (0, 1, 0)]
     ref = _oracle(d, shape[7], shape[8])["dx"]
-    emu = _oracle(d, shape[7], shape[8], x=EMU[math](d["x"]), w=EMU[math](d["w"]),
-                  dy=EMU[math](d["dy"]))["dx"]
+    if math == "fp32":
+        emu, bar = _mixed_emulated(d, shape[7], shape[8])["dx"], 5e-6
+    else:
+        emu = _oracle(d, shape[7], shape[8], x=EMU[math](d["x"]), w=EMU[math](d["w"]),
+                      dy=EMU[math](d["dy"]))["dx"]
+        bar = 1e-4
     assert np.abs(runs[0] - ref).max() / np.abs(ref).max() <= TOL[math]
-    assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= 1e-4
+    assert np.abs(runs[0] - emu).max() / np.abs(emu).max() <= bar
     for other in runs[1:]:
         np.testing.assert_array_equal(other, runs[0])
 
@@ -827,11 +845,14 @@ def test_halo_dgrad(shape, math):
 def test_halo_dgrad_model_choice():
     """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) in bf16
     and tf32, keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would
-    be junk), and for 3xTF32 (no two-plane halo kernel)."""
+    be junk), for 3xTF32 (no two-plane halo kernel) and for the mixed fp32 split (its halo kernel
+    measured slower than the im2col one on conv2: opt-in with halo_dgrad = 2)."""
     for math in ("bf16", "tf32"):
         assert _layer(HDG_SHAPES[0], math).info.dgrad_halo == 1
         assert _layer(SHAPES[6], math).info.dgrad_halo == 0
-    assert _layer(HDG_SHAPES[0], "fp32").info.dgrad_halo == 0
+    assert _layer(HDG_SHAPES[0], "fp32", fp32_split=1).info.dgrad_halo == 0
+    assert _layer(HDG_SHAPES[0], "fp32", fp32_split=1, halo_dgrad=2).info.dgrad_halo == 1
+    assert _layer(HDG_SHAPES[0], "fp32", fp32_split=0).info.dgrad_halo == 0
 
 
 @pytest.mark.parametrize("ncg", ["1", "2"])

@@ -214,8 +214,12 @@ __global__ void __launch_bounds__(256) pack_nchw_to_nhwc(const float *__restrict
 // (32-row tile, channel), the 32 rows summed by a fixed transposing butterfly (lane c ends with
 // channel c's sum).  grid (ceil(Cw/32), ceil(N*HWd/256)), 256 threads.
 constexpr int PACKW_ROWS = 32;
+// __launch_bounds__(256, 2): two CTAs per SM (<= 128 registers).  The mixed split's third plane
+// raised the unbounded allocation to 142 registers, one CTA per SM, and the fp32 packs ran at
+// 2.7-3.0 TB/s (CaffeNet conv1 dy 282 us); bounded: 4.3-4.7 TB/s (180 us); 3 CTAs (80 registers,
+// 150 bytes of spills) measured slower.
 template <int ELEM>
-__global__ void __launch_bounds__(256) pack_act_warp(const float *__restrict__ src,
+__global__ void __launch_bounds__(256, 2) pack_act_warp(const float *__restrict__ src,
                                                      void *__restrict__ dst, int N, int C, int HW,
                                                      int Cp, float *__restrict__ db_part,
                                                      unsigned int *__restrict__ tickets,

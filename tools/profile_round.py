@@ -128,4 +128,5 @@ def main(rnd, rep, launches=None, workload=4, math="bf16"):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else None)
+    main(sys.argv[1], sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else None,
+         math=sys.argv[4] if len(sys.argv) > 4 else "bf16")

@@ -1991,7 +1991,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
   // diagnostic builds only (never the shipped library): GLP_DEBUG_CLK = device address of
   // >= 4 * grid uint64 counters (tools/clk_probe.py); GLP_DEBUG_SKIP = work-skipping bits
   if (const char *e = getenv("GLP_DEBUG_CLK")) P->dbg_clk = reinterpret_cast<unsigned long long *>(strtoull(e, nullptr, 10));
-  if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 31;
+  if (const char *e = getenv("GLP_DEBUG_SKIP")) P->dbg_skip = atoi(e) & 63;
 #endif
   // Channel pitch of the packed NHWC operands: a multiple of 32 channels (64-byte bf16 / 128-byte
   // tf32 rows, what the im2col TMA path needs) unless the channel count is tiny, where padding to

@@ -240,7 +240,9 @@ __global__ void __launch_bounds__(HD_THREADS, 1)
               d = tmem_base + cur * (uint32_t)p.acc_cols;
               acc = 0;
             }
-            const int rows = kh * p.WQ + kw;   // the tap's row shift in the halo tile
+            // the tap's row shift in the halo tile (diagnostics, GLP_DEBUG_SKIP bit 5: without
+            // the kw part -- 8-row-aligned operand starts only; results wrong)
+            const int rows = kh * p.WQ + (GLP_SKIP(p, 32) ? 0 : kw);
             const uint64_t a_ = da0 + (uint64_t)(rows * 8);
             const uint64_t ab = da0 + (uint64_t)(rows * 4);   // bf16 rows are 64 bytes
             const uint64_t b_ = db0 + (uint64_t)(j * (p.b_tap_bytes >> 4));

@@ -261,8 +261,14 @@ int choose_bn(int n) {
 // two work units per slot (measured: for the large CaffeNet layers smaller tiles cost more in
 // A re-reads and per-k-block overhead than the last-round quantisation they save).  Below that,
 // time ~ rounds * (k-block MMA cycles ~ 2*bn, floored by the issue loop) picks the tile.
+// kb_fixed: a per-k-block cost independent of the N tile, in the units of 2*bn (the MMA work).
+// The mixed fp32 split streams three operand planes per k-block against 8 cheap MMAs, so smaller
+// N tiles pay relatively more for operand delivery (4 pipeline stages of 48 KB cover fewer MMA
+// cycles): on CaffeNet's 13x13 layers N 192 x 5 rounds beats N 128 x 7 rounds (conv3 fwd 208 ->
+// 199 us, conv4 dgrad 315 -> 291 us, same box, repeated) while N 128 x 5 rounds still beats N 256
+// x 3 rounds for 256 channels (conv5 fwd 217 vs 227 us); kb_fixed = 80 reproduces both.
 void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, int &cg_out,
-                    int min_units = 2) {
+                    int min_units = 2, double kb_fixed = 0.0) {
   const int bn0 = choose_bn(n);
   const int cg0 = cg2_ok ? 2 : 1;
   bn_out = bn0;
@@ -277,7 +283,7 @@ void choose_tile_mn(int n, long long M, bool cg2_ok, int sm_count, int &bn_out, 
       const int bn = (int)rup(cdiv(n, nt), 16);
       if ((int)cdiv(n, bn) != nt || (cg == 2 && (bn / 2) % 8)) continue;
       const double rounds = std::ceil((double)m_units * nt / slots);
-      const double c = rounds * std::max(2.0 * bn, 224.0) * (1.0 + 0.03 * (nt - 1)) *
+      const double c = rounds * (std::max(2.0 * bn, 224.0) + kb_fixed) * (1.0 + 0.03 * (nt - 1)) *
                        (cg == 1 ? 1.02 : 1.0);
       if (c < best_c) {
         best_c = c;
@@ -754,7 +760,8 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const bool wg_cg2 = P.wgrad_cg2 && (pp.bn / 2) % EPA == 0;   // MN-major B halves: whole atoms
   if (pp.a_tma && pp.m_tiles >= 2 && P.allow_cg2 && (mode != MODE_WGRAD || wg_cg2)) pp.cg = 2;
   if (mode != MODE_WGRAD && P.bn_model) {
-    choose_tile_mn(pp.Ng, pp.M, pp.cg == 2, P.sm_count, pp.bn, pp.cg, P.tile_units);
+    choose_tile_mn(pp.Ng, pp.M, pp.cg == 2, P.sm_count, pp.bn, pp.cg, P.tile_units,
+                   P.mix ? 80.0 : 0.0);
     pp.bn_smem = pp.bn;
   }
   if (pp.cg == 2) pp.bn_smem = pp.bn / 2;

@@ -805,7 +805,11 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   const int b_row = planes * (mode == MODE_WGRAD ? BKP * elem : pp.krow);
   // forward: the bias vector is staged once per CTA in smem (every column a tile can touch)
   pp.bias_floats = (mode == MODE_FWD) ? (int)rup((long long)pp.n_tiles * pp.bn, 32) + 32 : 0;
-  const int budget = P.smem_cap - 1024 - 1024 - 4 * pp.bias_floats;   // alignment slack; barriers, TMEM slot
+  // ring budget: the cap minus the 1 KB alignment slack, the 4 extra barriers + TMEM slot + bias
+  // alignment (64 bytes) and the bias stage; each stage also takes its two 8-byte barriers (the
+  // exact layout of pp.smem below: a 1 KB reserve for the barriers cost the N = 192 mixed forward
+  // tiles their fourth stage by 512 bytes)
+  const int budget = P.smem_cap - 1024 - 64 - 4 * pp.bias_floats;
   // k-blocks per pipeline stage: as many (<= 4) as keep >= 3 stages in the ring.  One
   // full/empty round trip of the single MMA-issuing warp costs ~250-700 cycles whatever the stage
   // size (tools/sync_probe*.cu, GLP_DEBUG_SKIP=15 runs), more than the tensor work of one small-N
@@ -817,7 +821,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
            pp.kb_per_split >= 2 * (pp.ksub + 1))
       ++pp.ksub;
   const int stage_bytes = pp.ksub * kb_bytes;
-  pp.stages = std::min(8, budget / stage_bytes);
+  pp.stages = std::min(8, budget / (stage_bytes + 16));
 #ifdef GLP_DIAG
   if (const char *e = getenv("GLP_DEBUG_STAGES"))   // diagnostics: fewer ring stages
     pp.stages = std::max(2, std::min(pp.stages, atoi(e)));

@@ -99,6 +99,9 @@ typedef struct {
   int wgrad_reduce_wide; /* 1: the dW split reduction runs 4 weight rows x 8 split phases per block
                             (small filters: < 64 tiles of 32 x 32); 0: 32 x 32 tiles             */
   int fp32_split;        /* 1: this GLP_MATH_FP32 plan runs the mixed split (glp_plan_options_t)  */
+  int dgrad_s2d;         /* 1: strided layer whose backward-data runs as the stride-1 backward-data
+                            of its space-to-depth form (dx' over x', then scattered into dx);
+                            ws_bwd_data then includes the dx' buffer (N*S*S*C_in*H'*W' floats)    */
 } glp_plan_info_t;
 
 /* Per-SM limits (Table 2 "device property", P183-193) plus the sm_100a-only ones. */

@@ -39,7 +39,7 @@ class PlanInfo(ctypes.Structure):
                 ("wgrad_halo", _c_int), ("fwd_halo", _c_int),
                 ("wgrad_fused_dy", _c_int), ("dgrad_halo", _c_int),
                 ("s_slot_rows", ctypes.c_longlong), ("s_rows_per_sample", ctypes.c_longlong),
-                ("wgrad_reduce_wide", _c_int), ("fp32_split", _c_int)]
+                ("wgrad_reduce_wide", _c_int), ("fp32_split", _c_int), ("dgrad_s2d", _c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -193,15 +193,21 @@ glp_status_t get_encode_im2col() {
 // im2col tensor map over a packed NHWC activation [N][H][W][cpitch]: dims {cpitch, W, H, N};
 // bounding box of base pixels [lower, dim-1+upper] per spatial dim (W, H order), traversal
 // strides = conv strides; each load = `pixels` pixels x `chans` channels.
+// pitch_w / pitch_h: the allocated image width / height of the buffer when the tensor is the
+// top-left W x H region of a larger grid (the padded dy grid of halo plans); 0 = W / H.
 glp_status_t encode_im2col(CUtensorMap *map, int elem, const void *ptr, int cpitch, int W, int H,
                            int N, int lower_w, int lower_h, int upper_w, int upper_h, int chans,
-                           int pixels, int stride_w, int stride_h, CUtensorMapSwizzle swz) {
+                           int pixels, int stride_w, int stride_h, CUtensorMapSwizzle swz,
+                           int pitch_w = 0, int pitch_h = 0) {
+  if (pitch_w <= 0) pitch_w = W;
+  if (pitch_h <= 0) pitch_h = H;
   if (lower_w < -128 || lower_w > 127 || lower_h < -128 || lower_h > 127 || upper_w < -128 ||
       upper_w > 127 || upper_h < -128 || upper_h > 127)
     return fail(GLP_ERR_NOT_SUPPORTED, "im2col corner out of TMA range");
   const uint64_t e = (uint64_t)elem;
   cuuint64_t dims[4] = {(cuuint64_t)cpitch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
-  cuuint64_t strides[3] = {cpitch * e, (uint64_t)W * cpitch * e, (uint64_t)H * W * cpitch * e};
+  cuuint64_t strides[3] = {cpitch * e, (uint64_t)pitch_w * cpitch * e,
+                           (uint64_t)pitch_h * pitch_w * cpitch * e};
   int lower[2] = {lower_w, lower_h}, upper[2] = {upper_w, upper_h};
   cuuint32_t es[4] = {1, (cuuint32_t)stride_w, (cuuint32_t)stride_h, 1};
   CUresult r = g_encode_im2col(map, elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
@@ -213,7 +219,7 @@ glp_status_t encode_im2col(CUtensorMap *map, int elem, const void *ptr, int cpit
     return fail(GLP_ERR_CUDA, "cuTensorMapEncodeIm2col failed (" + std::to_string((int)r) + ")");
   // Same driver workaround CUTLASS applies to im2col descriptors of small tensors (< 128 KiB)
   // on drivers <= 13.1 (cute/atom/copy_traits_sm90_im2col.hpp).
-  if (g_driver_version <= 13010 && (uint64_t)N * H * W * cpitch * e < 131072)
+  if (g_driver_version <= 13010 && (uint64_t)N * pitch_h * pitch_w * cpitch * e < 131072)
     reinterpret_cast<uint64_t *>(map)[1] &= ~(1ull << 21);
   return GLP_OK;
 }
@@ -368,6 +374,11 @@ struct glp_plan_s {
   // or its space-to-depth form (s2d = stride S > 1: stride 1, ceil(K/S) taps, S*S*C channels).
   int s2d = 0;
   int s2d_blocks = 1;   // resident pack_s2d blocks per SM (occupancy API): its persistent grid
+  // backward-data of a space-to-depth layer as the stride-1 backward-data over x' (dx' in the
+  // workspace at off_dxs, then unpack_s2d_dx): 9 taps of unit stride instead of the 121-tap
+  // strided gather (CaffeNet conv1)
+  int s2d_dg = 0;
+  size_t off_dxs = 0, sz_dxs = 0;
   glp_conv_desc_s dxg;
   int Cpx = 0, tapsx = 0;
   PassPlan fwd, dgrad, wgrad;
@@ -704,8 +715,10 @@ glp_status_t plan_hfwd(glp_plan_s &P) {
 
 glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_limits_t &L) {
   const int elem = P.elem;
-  const glp_conv_desc_s &d = (mode == MODE_DGRAD) ? P.d : P.dxg;
+  // backward-data: the layer's own geometry, or (s2d_dg) the stride-1 space-to-depth one
+  const glp_conv_desc_s &d = (mode == MODE_DGRAD && !P.s2d_dg) ? P.d : P.dxg;
   const int Cpx = P.Cpx, tapsx = P.tapsx;
+  const int taps_dg = P.s2d_dg ? P.tapsx : P.taps;
   // A by im2col TMA when the channel pitch is a multiple of a 64-byte row; K-block rows of 128
   // bytes when the pitch allows, else 64 (bf16).  Otherwise the cp.async gather (128-byte rows).
   const int u64 = 64 / elem, u128 = 128 / elem;
@@ -740,7 +753,7 @@ glp_status_t plan_pass(glp_plan_s &P, PassPlan &pp, int mode, const glp_device_l
   } else if (mode == MODE_DGRAD) {
     pp.M = d.N * d.H * d.W;
     pp.Ng = d.C;
-    pp.Kpad = (int)rup((long long)P.taps * P.Cop, BK);
+    pp.Kpad = (int)rup((long long)taps_dg * P.Cop, BK);
     pp.kb_total = pp.Kpad / BK;
     pp.bn = choose_bn(d.C);
     pp.bn_smem = pp.bn;
@@ -882,7 +895,7 @@ glp_status_t validate_ptrs(std::initializer_list<const void *> ps) {
 }
 
 IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const void *src) {
-  const glp_conv_desc_s &d = (mode == MODE_DGRAD) ? P.d : P.dxg;
+  const glp_conv_desc_s &d = (mode == MODE_DGRAD && !P.s2d_dg) ? P.d : P.dxg;
   IgemmParams p;
   memset(&p, 0, sizeof(p));
   Gather &g = p.g;
@@ -892,7 +905,7 @@ IgemmParams make_params(const glp_plan_s &P, const PassPlan &pp, int mode, const
   g.pad = d.Ph;
   g.pad_w = d.Pw;
   g.kw = d.Kw;
-  g.taps = (mode == MODE_DGRAD) ? P.taps : P.tapsx;
+  g.taps = (mode == MODE_DGRAD && !P.s2d_dg) ? P.taps : P.tapsx;
   if (mode == MODE_DGRAD) {
     // halo plans pack dy on the padded dxg grid (zeros outside H_o x W_o): same values
     g.src_h = P.halo ? P.dxg.H : d.Ho;
@@ -1182,6 +1195,15 @@ glp_status_t run_pack_w_dgrad(glp_plan_s &P, const BrIn &w, uint8_t *ws, cudaStr
   const glp_conv_desc_s &d = P.d;
   void *wtpk = ws + P.off_wtpk;
   const int flip = P.dgrad.a_tma;  // the im2col-TMA dgrad walks taps flipped
+  if (P.s2d_dg) {   // Wt' of the space-to-depth weights, rows = the S*S*C x' channels
+    const dim3 g2((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)P.dxg.C);
+    if (P.elem == 2)
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_s2d<2>, g2, dim3(256), 0, st, w.p[0], wtpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cop, P.dgrad.Kpad, flip, 0LL));
+    else
+      GLP_CUDA(launch_pdl(P.pdl, pack_w_dgrad_s2d<4>, g2, dim3(256), 0, st, w.p[0], wtpk, d.Co, d.C, d.Kh, P.s2d, P.dxg.Kh, P.Cop, P.dgrad.Kpad, flip, plo(P, P.lo_wtpk)));
+    GLP_LAUNCH_CHECK("pack_w_dgrad_s2d");
+    return GLP_OK;
+  }
   const dim3 grid((unsigned)cdiv(P.dgrad.Kpad, 256), (unsigned)d.C);
   const int n = std::max(1, w.n);
   for (int b = 0; b < n; ++b) {
@@ -1436,7 +1458,11 @@ glp_status_t run_dgrad_halo(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
 
 glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t st) {
   if (P.hdg) return run_dgrad_halo(P, dx, ws, st);
-  const glp_conv_desc_s &d = P.d;
+  // space-to-depth layers: the stride-1 backward-data of the x' convolution into dx' (workspace),
+  // then dx' -> dx
+  const glp_conv_desc_s &d = P.s2d_dg ? P.dxg : P.d;
+  // halo plans pack dy on the padded x' grid: the dgrad's dy tensor is its top-left H_o x W_o
+  const int dy_pw = P.halo ? P.dxg.W : 0, dy_ph = P.halo ? P.dxg.H : 0;
   const PassPlan &pp = P.dgrad;
   void *wtpk = ws + P.off_wtpk;
   const void *dypk = ws + P.off_dypk;
@@ -1456,17 +1482,31 @@ glp_status_t run_dgrad_gemm(glp_plan_s &P, float *dx, uint8_t *ws, cudaStream_t 
       if ((r = get_encode_im2col())) return r;
       r = encode_im2col(plane_map(&q.a, &q.a2, &q.a3, pl), e, static_cast<const uint8_t *>(dypk) + ld, P.Cop,
                         d.Wo, d.Ho, d.N, -(d.Kw - 1 - d.Pw), -(d.Kh - 1 - d.Ph), -d.Pw, -d.Ph, BK,
-                        128, 1, 1, sw);
+                        128, 1, 1, sw, dy_pw, dy_ph);
       if (r) return r;
     }
     return GLP_OK;
   });
   if (s) return s;
   IgemmParams p = make_params(P, pp, MODE_DGRAD, dypk);
-  p.out = dx;
-  p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
+  if (!P.s2d_dg) {
+    p.out = dx;
+    p.out_c = P.x_img_c;   // channels per image of dx (the whole tensor for a conv group)
+    p.out_hw = d.H * d.W;
+    return launch_igemm<MODE_DGRAD>(P, pp, p, m, st);
+  }
+  float *dxs = reinterpret_cast<float *>(ws + P.off_dxs);
+  p.out = dxs;
+  p.out_c = d.C;
   p.out_hw = d.H * d.W;
-  return launch_igemm<MODE_DGRAD>(P, pp, p, m, st);
+  if ((s = launch_igemm<MODE_DGRAD>(P, pp, p, m, st))) return s;
+  const glp_conv_desc_s &o = P.d;
+  const long long total = (long long)o.N * o.C * o.H * o.W;
+  GLP_CUDA(launch_pdl(P.pdl, unpack_s2d_dx, dim3((unsigned)std::min<long long>(cdiv(total, 256), 148 * 16)),
+                      dim3(256), 0, st, (const float *)dxs, dx, o.N, o.C, o.H, o.W, P.s2d, o.Ph,
+                      P.dxg.H, P.dxg.W, P.x_img_c));
+  GLP_LAUNCH_CHECK("unpack_s2d_dx");
+  return GLP_OK;
 }
 
 glp_status_t run_wgrad_halo(glp_plan_s &P, uint8_t *ws, cudaStream_t st, const float *dy) {
@@ -2035,6 +2075,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
       }
     }
   }
+  P->s2d_dg = (P->s2d && d->nbr <= 1) ? 1 : 0;
   glp_device_limits_t L;
   glp_device_limits_b200(&L);
   L.sm_count = prop.multiProcessorCount;
@@ -2107,7 +2148,7 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
     const size_t dy_hw = P->halo ? (size_t)P->dxg.H * P->dxg.W : (size_t)c.Ho * c.Wo;
     const size_t pl_dy = align1k((size_t)c.N * dy_hw * P->Cop * P->elem);
     const size_t pl_w = align1k((size_t)c.Co * P->fwd.Kpad * P->elem);
-    const size_t pl_wt = align1k((size_t)c.C * P->dgrad.Kpad * P->elem);
+    const size_t pl_wt = align1k((size_t)(P->s2d_dg ? P->dxg.C : c.C) * P->dgrad.Kpad * P->elem);
     const size_t planes = P->x3 ? 2 : 1;
     P->sz_xpk = planes * pl_x;
     P->sz_dypk = planes * pl_dy;
@@ -2147,6 +2188,12 @@ glp_status_t glp_plan_ex(glp_plan_t *out, glp_conv_desc_t d, int device, glp_mat
     P->off_leaf = P->off_dbpart + P->sz_dbpart;
     P->ws_wgrad = P->off_leaf + P->sz_leaf;
     P->ws_bwd = P->ws_wgrad;
+    if (P->s2d_dg) {   // dx' of the space-to-depth backward-data, after every other region
+      P->off_dxs = P->ws_wgrad;
+      P->sz_dxs = align1k((size_t)c.N * P->dxg.C * P->dxg.H * P->dxg.W * 4);
+      P->ws_dgrad = P->off_dxs + P->sz_dxs;
+      P->ws_bwd = P->ws_dgrad;
+    }
     // Samples in flight (the paper's C_out, Eq. 9 re-derived, R18) through the analyzer: the
     // forward kernel's resident rows (#SM x CTAs/SM x 128 GEMM rows) over the rows a sample
     // occupies (H_o*W_o pixels -- the padded x' grid for the halo forward -- times the N tiles)
@@ -2222,6 +2269,7 @@ glp_status_t glp_plan_get_info(glp_plan_t P, glp_plan_info_t *I) {
   I->s_rows_per_sample = P->s_rows_per_sample;
   I->wgrad_reduce_wide = P->red_wide;
   I->fp32_split = P->mix;
+  I->dgrad_s2d = P->s2d_dg;
   if (P->hdg) {
     I->grid_bwd_data = P->hd_grid;
     I->tile_n_bwd_data = P->hd.bn;

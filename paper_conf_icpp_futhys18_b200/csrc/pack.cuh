@@ -681,6 +681,58 @@ __global__ void __launch_bounds__(256) pack_w_dgrad(const float *__restrict__ w,
   PackOut<ELEM>::store1(out, (size_t)ci * Kpad + k, v, lo_off);
 }
 
+// Space-to-depth backward-data (strided layers, DESIGN.md §7 "strided backward-data"): the
+// B operand of the stride-1 dgrad over x' -- Wt'[cs][t*Cop + co] = W'[co][tap(t)][cs] with the
+// space-to-depth weights W'[co][(kh', kw')][cs = (dh*S + dw)*C + c] = W[co][c][kh'*S + dh]
+// [kw'*S + dw] (zero past the K x K kernel), taps flipped when the dgrad walks them by TMA.
+// grid (ceil(Kpad / 256), Cs).
+template <int ELEM>
+__global__ void __launch_bounds__(256) pack_w_dgrad_s2d(const float *__restrict__ w, void *__restrict__ out,
+                                                        int Co, int C, int K, int S, int Ks, int Cop,
+                                                        int Kpad, int flip, long long lo_off) {
+  pdl_launch_dependents();
+  pdl_wait();
+  const int cs = blockIdx.y, k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= Kpad) return;
+  const int t = k / Cop, co = k - t * Cop, taps = Ks * Ks;
+  float v = 0.f;
+  if (t < taps && co < Co) {
+    const int tt = flip ? taps - 1 - t : t;
+    const int khs = tt / Ks, kws = tt - khs * Ks;
+    const int ph = cs / C, c = cs - ph * C, dh = ph / S, dw = ph - dh * S;
+    const int kh = khs * S + dh, kw = kws * S + dw;
+    if (kh < K && kw < K) v = __ldg(w + (((size_t)co * C + c) * K + kh) * K + kw);
+  }
+  PackOut<ELEM>::store1(out, (size_t)cs * Kpad + k, v, lo_off);
+}
+
+// dx from the space-to-depth gradient dx'[n][cs][h'][w'] (NCHW, Cs = S*S*C channels, H' x W'):
+// dx[n][c][h][w] = dx'[n][(dh*S + dw)*C + c][h'][w'] with h + P = S*h' + dh, w + P = S*w' + dw
+// (each x element sits once in x'); elements the x' grid does not reach get 0 (they reach no
+// output, Alg. 2 / DESIGN.md R2).  One thread per dx element, w fastest (coalesced
+// stores).  img_c: channels per image of the dx tensor (conv groups).
+__global__ void __launch_bounds__(256) unpack_s2d_dx(const float *__restrict__ dxs, float *__restrict__ dx,
+                                                     int N, int C, int H, int W, int S, int P,
+                                                     int Hs, int Ws, int img_c) {
+  pdl_launch_dependents();
+  pdl_wait();
+  const long long total = (long long)N * C * H * W;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int w = (int)(i % W);
+    long long r = i / W;
+    const int h = (int)(r % H);
+    r /= H;
+    const int c = (int)(r % C), n = (int)(r / C);
+    const int hp = h + P, wp = w + P;
+    const int h2 = hp / S, dh = hp - h2 * S, w2 = wp / S, dw = wp - w2 * S;
+    float v = 0.f;
+    if (h2 < Hs && w2 < Ws)
+      v = __ldg(dxs + (((size_t)n * S * S * C + (size_t)(dh * S + dw) * C + c) * Hs + h2) * Ws + w2);
+    dx[(((size_t)n * img_c + c) * H + h) * W + w] = v;
+  }
+}
+
 // Row-staged weight packs (default when a staged row fits 48 KB of shared memory).  The element-
 // per-thread kernels above read W with a stride of `taps` floats between neighbouring threads (one
 // 32-byte sector per 4-byte load); here one block owns one destination row, reads its source

@@ -842,6 +842,24 @@ def test_halo_dgrad(shape, math):
         np.testing.assert_array_equal(other, runs[0])
 
 
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+def test_strided_dgrad_space_to_depth(math):
+    """Strided layers whose forward runs on the space-to-depth x' (CaffeNet conv1, ragged_s2) take
+    the backward-data as the stride-1 backward-data of that form (dx' over x', then scattered into
+    dx; dgrad_s2d = 1): bit-exact on integer data against the oracle's col2im, which is written
+    for the strided layer itself (the exactness and emulated-rounding cases of SHAPES cover the
+    random data)."""
+    for shape in (SHAPES[2], SHAPES[3]):
+        layer = _layer(shape, math)
+        assert layer.info.dgrad_s2d == 1, shape[0]
+        d = _data(shape, exact=True, seed=57)
+        got = _run(layer, d)
+        ref = _oracle(d, shape[7], shape[8])
+        np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32), err_msg=shape[0])
+    # unit-stride layers keep their own backward-data
+    assert _layer(SHAPES[6], math).info.dgrad_s2d == 0
+
+
 def test_halo_dgrad_model_choice():
     """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) in bf16
     and tf32, keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would

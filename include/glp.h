@@ -166,7 +166,8 @@ typedef struct {
   int wgrad_tile_n;       /* 0: model; else the filter-gradient N tile (multiple of 16, <= 256)    */
   int tile_units;         /* fwd/dgrad tile model applies below this many work units per slot (6)  */
   int bn_model;           /* 1: fwd/dgrad N-tile model for small grids; 0: always the default tile */
-  int pack_block;         /* 0: warp-tiled activation pack; 1: block-tiled                         */
+  int pack_block;         /* 0: warp-tiled activation pack; 1: block-tiled; 2 (default): block-
+                             tiled for 4-byte operands (tf32, fp32 splits), warp-tiled for bf16  */
   int s2d_block;          /* 0: warp-per-32-pixel space-to-depth pack; 1: block-persistent          */
   int smem_cap;           /* dynamic shared memory budget of the persistent GEMMs, bytes (232448)  */
   int pdl;                /* 1: programmatic dependent launch between the plan's kernels; 0: not   */

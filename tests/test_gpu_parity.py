@@ -860,6 +860,22 @@ def test_strided_dgrad_space_to_depth(math):
     assert _layer(SHAPES[6], math).info.dgrad_s2d == 0
 
 
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+def test_pack_variants_same_operands(math):
+    """The warp-tiled and the block-tiled activation packs (plan option pack_block; the default
+    takes the block-tiled one for 4-byte operands) write the same operand bits: y, dx and dW are
+    bitwise equal; db (summed per row tile of the pack, 32 vs 128 rows) within summation-order
+    noise."""
+    for shape in (SHAPES[0], MIX_SHAPES[2], SHAPES[2]):
+        d = _data(shape, seed=58)
+        a = _run(_layer(shape, math, pack_block=0), d)
+        b = _run(_layer(shape, math, pack_block=1), d)
+        for k in ("y", "dx", "dw"):
+            np.testing.assert_array_equal(a[k], b[k], err_msg=f"{shape[0]} {k}")
+        scale = np.abs(d["dy"].astype(np.float64)).sum(axis=(0, 2, 3))
+        assert np.all(np.abs(a["db"].astype(np.float64) - b["db"]) <= 1e-6 * scale), shape[0]
+
+
 def test_halo_dgrad_model_choice():
     """The cost model picks the halo backward-data for CaffeNet conv2 (27x27, 5x5, C_i = 96) in bf16
     and tf32, keeps the im2col kernel for the 13x13 layers (conv3-5: half of the padded rows would

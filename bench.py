@@ -82,7 +82,7 @@ def parse_args():
     p.add_argument("--plan-options", default="",
                    help="JSON glp_plan_options_t fields for every plan (A/B runs of alternative "
                         "kernels/tilings; recorded in config)")
-    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--e2e-steps", type=int, default=20)
     p.add_argument("--serial", action="store_true",
                    help="issue the step on one stream (default: the real-network stream DAG)")
     p.add_argument("--no-graph", action="store_true",

@@ -1,6 +1,6 @@
 #!/bin/bash
 # every BASELINE.json workload (and the NEXT-3 variants) through bench.py: the fp32 (3xTF32)
-# headline line with the bf16 / tf32 lines beside it
+# headline line (mixed split / 3xTF32) with the bf16 / tf32 lines beside it
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out/workloads
 for w in ${WORKLOADS:-1 2 3 4 5 6 7 8 9}; do

@@ -856,6 +856,19 @@ def test_strided_dgrad_space_to_depth(math):
         got = _run(layer, d)
         ref = _oracle(d, shape[7], shape[8])
         np.testing.assert_array_equal(got["dx"], ref["dx"].astype(np.float32), err_msg=shape[0])
+    # the staged calls (the bench's path; bf16 conv1 packs dy lazily for its fused-dy filter
+    # gradient) give the same dx bits
+    shape = SHAPES[2]
+    layer = _layer(shape, math)
+    d = _data(shape, exact=True, seed=57)
+    t = {k: torch.from_numpy(v).to(DEV) for k, v in d.items()}
+    dx = torch.full(layer.x_shape, float("nan"), device=DEV)
+    layer.stage_pack(glp.GLP_PACK_W_BWD_DATA, t["w"])
+    layer.stage_pack(glp.GLP_PACK_DY, t["dy"])
+    layer.stage_bwd_data(dx)
+    torch.cuda.synchronize()
+    ref = _oracle(d, shape[7], shape[8])
+    np.testing.assert_array_equal(dx.cpu().numpy(), ref["dx"].astype(np.float32))
     # unit-stride layers keep their own backward-data
     assert _layer(SHAPES[6], math).info.dgrad_s2d == 0
 

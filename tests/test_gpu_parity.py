@@ -922,13 +922,17 @@ LONG_K = [("caffenet_conv2", 2, 96, 27, 27, 256, 5, 1, 2),    # dgrad K = 6400, 
           ("gnet_conv_4", 3, 192, 7, 7, 384, 3, 1, 1)]
 
 
+@pytest.mark.parametrize("split", [0, 1], ids=["3xtf32", "mixed"])
 @pytest.mark.parametrize("shape", LONG_K, ids=lambda s: s[0])
-def test_fp32_long_reductions(shape):
-    """GLP_MATH_FP32 (3xTF32) at the paper's longest reductions: the tensor core truncates each
-    MMA's fp32 result, so the error of one TMEM accumulator grows with K; the chunked fp32 register
-    accumulation keeps every output within the 1e-5 normwise bar (BASELINE.json north_star)."""
+def test_fp32_long_reductions(shape, split):
+    """GLP_MATH_FP32 (3xTF32, and the mixed split) at the paper's longest reductions: the tensor
+    core truncates each MMA's fp32 result, so the error of one TMEM accumulator grows with K; the
+    chunked fp32 register accumulation keeps every output within the 1e-5 normwise bar
+    (BASELINE.json north_star)."""
     d = _data(shape, seed=91)
-    got = _run(_layer(shape, "fp32"), d)
+    layer = _layer(shape, "fp32", fp32_split=split)
+    assert layer.info.fp32_split == split
+    got = _run(layer, d)
     ref = _oracle(d, shape[7], shape[8])
     errs = {k: oracle.normwise_err(got[k], ref[k]) for k in ref}
     assert all(e <= TOL["fp32"] for e in errs.values()), errs
